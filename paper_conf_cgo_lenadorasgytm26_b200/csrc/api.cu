@@ -1,0 +1,270 @@
+// api.cu -- the extern "C" entry points of include/granii.h: argument
+// validation, error reporting, dispatch to the kernels.  No compute here.
+#include <cstring>
+#include <string>
+
+#include "internal.h"
+
+namespace granii {
+static thread_local std::string g_last_error;
+void set_error(const std::string& m) { g_last_error = m; }
+granii_status fail(granii_status st, const std::string& m) {
+  g_last_error = m;
+  return st;
+}
+
+granii_status dev_info(DevInfo* out) {
+  int dev = -1;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return fail(GRANII_ERR_CUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
+  static thread_local DevInfo cache;
+  if (cache.device != dev) {
+    int sms = 0, l2 = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    cache.device = dev;
+    cache.sms = sms > 0 ? sms : 148;
+    cache.l2_bytes = l2 > 0 ? l2 : (126ll << 20);
+  }
+  *out = cache;
+  return GRANII_OK;
+}
+
+// defined in other translation units
+granii_status graph_create(int64_t, int64_t, const int32_t*, const int32_t*, uint32_t, int32_t, int32_t, cudaStream_t,
+                           granii_graph_s**);
+void graph_free(granii_graph_s*);
+void partition_bounds_host(int64_t N, const int64_t* rp, int G, int64_t* b);
+granii_status layer_workspace(const granii_graph_s*, granii_model, granii_composition, int64_t, int64_t, size_t*,
+                              size_t*);
+granii_status layer_forward(const granii_graph_s*, granii_model, granii_composition, const granii_layer_args*, float*,
+                            int64_t, float*, cudaStream_t);
+granii_status layer_backward(const granii_graph_s*, granii_composition, const granii_layer_args*, const float*, int64_t,
+                             const float*, int64_t, const float*, float*, int64_t, float*, cudaStream_t);
+granii_status select_impl(const granii_graph_s*, granii_model, int64_t, int64_t, const char*, uint32_t,
+                          granii_composition*, int32_t*, double*, int32_t*);
+granii_status comm_unique_id(void*);
+granii_status comm_create(const void*, int32_t, int32_t, granii_comm_s**);
+granii_status comm_destroy(granii_comm_s*);
+granii_status launch_softmax_xent(int64_t, int64_t, const float*, int64_t, const int32_t*, int64_t, float*, int64_t,
+                                  float*, cudaStream_t);
+granii_status launch_sgd(int64_t, float, const float*, float*, cudaStream_t);
+}  // namespace granii
+
+using namespace granii;
+
+static bool valid_comp(granii_model m, granii_composition c) {
+  if (m == GRANII_GCN) return c == GRANII_GCN_PRE_AGG || c == GRANII_GCN_PRE_UPD || c == GRANII_GCN_DYN_AGG || c == GRANII_GCN_DYN_UPD;
+  if (m == GRANII_GAT) return c == GRANII_GAT_REUSE || c == GRANII_GAT_RECOMP;
+  return false;
+}
+
+#define API_BEGIN try {
+#define API_END                                                          \
+  }                                                                      \
+  catch (const std::exception& ex) {                                     \
+    return fail(GRANII_ERR_CUDA, std::string("exception: ") + ex.what()); \
+  }                                                                      \
+  catch (...) {                                                          \
+    return fail(GRANII_ERR_CUDA, "unknown exception");                   \
+  }
+
+extern "C" {
+
+const char* granii_last_error(void) { return g_last_error.c_str(); }
+const char* granii_version(void) { return "granii-b200 0.1 sm_100a (tcgen05 3xTF32 GEMM, CSR SpMM/SDDMM)"; }
+
+granii_status granii_graph_csr_create(int64_t num_nodes, int64_t num_edges, const int32_t* d_src, const int32_t* d_dst,
+                                      uint32_t flags, int32_t part_rank, int32_t part_world, void* stream,
+                                      granii_graph* out) {
+  API_BEGIN
+  GR_ARG(out, "out is NULL");
+  GR_ARG(num_nodes >= 0 && num_edges >= 0, "negative size");
+  GR_ARG(num_nodes < (int64_t(1) << 31), "num_nodes must fit int32 column ids");
+  GR_ARG(num_edges == 0 || (d_src && d_dst), "NULL edge arrays");
+  GR_ARG((flags & ~(GRANII_ADD_SELF_LOOPS | GRANII_SYMMETRIZE)) == 0, "unknown flags");
+  GR_ARG(part_world >= 1 && part_rank >= 0 && part_rank < part_world, "bad partition rank/world");
+  GR_ARG(part_world <= 1 || num_nodes >= part_world, "fewer nodes than partitions");
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  granii_graph_s* g = nullptr;
+  GR_TRY(graph_create(num_nodes, num_edges, d_src, d_dst, flags, part_rank, part_world, (cudaStream_t)stream, &g));
+  *out = g;
+  return GRANII_OK;
+  API_END
+}
+
+granii_status granii_graph_destroy(granii_graph g) {
+  graph_free(g);
+  return GRANII_OK;
+}
+
+granii_status granii_graph_query(granii_graph g, granii_graph_info* o) {
+  GR_ARG(g && o, "NULL argument");
+  memset(o, 0, sizeof(*o));
+  o->num_nodes = g->N;
+  o->nnz = g->nnz;
+  o->row_begin = g->row_begin;
+  o->row_end = g->row_end;
+  o->local_nnz = g->local_nnz;
+  o->max_local_rows = g->max_rows;
+  o->part_rank = g->rank;
+  o->part_world = g->world;
+  o->symmetric = g->symmetric;
+  for (int i = 0; i < GRANII_NUM_FEATURES; ++i) o->features[i] = g->features[i];
+  return GRANII_OK;
+}
+
+granii_status granii_graph_export_csr(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx) {
+  API_BEGIN
+  GR_ARG(g && h_row_ptr && h_col_idx, "NULL argument");
+  GR_CUDA(cudaDeviceSynchronize());
+  GR_CUDA(cudaMemcpy(h_row_ptr, g->row_ptr, (g->n_rows + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+  if (g->local_nnz > 0)
+    GR_CUDA(cudaMemcpy(h_col_idx, g->col_idx, g->local_nnz * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  if (g->world > 1) {  // undo the gather-layout remap: report global column ids
+    for (int64_t i = 0; i < g->local_nnz; ++i) {
+      int64_t j = h_col_idx[i], owner = j / g->max_rows;
+      h_col_idx[i] = (int32_t)(g->bounds[owner] + (j - owner * g->max_rows));
+    }
+  }
+  return GRANII_OK;
+  API_END
+}
+
+granii_status granii_graph_dinv(granii_graph g, const float** d) {
+  GR_ARG(g && d, "NULL argument");
+  *d = g->dinv_rows;
+  return GRANII_OK;
+}
+
+granii_status granii_partition_bounds(int64_t num_nodes, const int64_t* h_row_ptr, int32_t world, int64_t* bounds) {
+  GR_ARG(h_row_ptr && bounds && world >= 1 && num_nodes >= 0, "bad argument");
+  partition_bounds_host(num_nodes, h_row_ptr, world, bounds);
+  return GRANII_OK;
+}
+
+granii_status granii_spmm(granii_graph g, const float* d_vals, const float* d_X, int64_t ldx, int64_t K, float* d_Y,
+                          int64_t ldy, const float* d_row_scale, const float* d_col_scale, uint32_t epilogue,
+                          void* stream) {
+  API_BEGIN
+  GR_ARG(g && d_X && d_Y, "NULL argument");
+  GR_ARG(K > 0 && ldx >= K && ldy >= K, "bad K / leading dimension");
+  GR_ARG((epilogue & ~GRANII_EPI_RELU) == 0, "unknown epilogue flags");
+  GR_ARG(d_X != d_Y, "X and Y must not alias");
+  return launch_spmm(g, d_vals, d_X, ldx, K, d_Y, ldy, d_row_scale, d_col_scale, epilogue & GRANII_EPI_RELU,
+                     (cudaStream_t)stream);
+  API_END
+}
+
+granii_status granii_sddmm(granii_graph g, uint32_t op, const float* d_U, int64_t ldu, const float* d_V, int64_t ldv,
+                           int64_t K, float scale, float* d_out, void* stream) {
+  API_BEGIN
+  GR_ARG(g && d_U && d_V && d_out, "NULL argument");
+  GR_ARG(K > 0 && ldu >= K && ldv >= K, "bad K / leading dimension");
+  GR_ARG((op & 0xF) <= GRANII_SDDMM_ADD && (op & ~0x3Fu) == 0, "unknown SDDMM op");
+  return launch_sddmm(g, op, d_U, ldu, d_V, ldv, K, scale, d_out, (cudaStream_t)stream);
+  API_END
+}
+
+granii_status granii_gemm_workspace_size(int64_t M, int64_t N, int64_t K, uint32_t flags, size_t* bytes) {
+  GR_ARG(bytes && M >= 0 && N >= 0 && K >= 0, "bad argument");
+  *bytes = gemm_workspace(M, N, K, flags);
+  return GRANII_OK;
+}
+
+granii_status granii_gemm(int64_t M, int64_t N, int64_t K, const float* d_A, int64_t lda, const float* d_B, int64_t ldb,
+                          float* d_C, int64_t ldc, const granii_gemm_epilogue* epi, uint32_t flags, void* d_ws,
+                          size_t ws_bytes, void* stream) {
+  API_BEGIN
+  GR_ARG(M >= 0 && N >= 0 && K > 0, "bad sizes");
+  GR_ARG(d_A && d_B, "NULL operand");
+  GR_ARG((flags & GRANII_GEMM_NO_STORE) || (d_C && ldc >= N), "bad C");
+  GR_ARG((flags & GRANII_GEMM_TRANS_A) ? lda >= M : lda >= K, "bad lda");
+  GR_ARG((flags & GRANII_GEMM_TRANS_B) ? ldb >= K : ldb >= N, "bad ldb");
+  GR_ARG((flags & ~0xFu) == 0, "unknown GEMM flags");
+  GR_ARG(d_ws || gemm_workspace(M, N, K, flags) == 0, "NULL workspace");
+  return launch_gemm(M, N, K, d_A, lda, d_B, ldb, d_C, ldc, epi, flags, d_ws, ws_bytes, (cudaStream_t)stream);
+  API_END
+}
+
+granii_status granii_layer_workspace_size(granii_graph g, granii_model m, granii_composition c, int64_t K1, int64_t K2,
+                                          size_t* ws, size_t* saved) {
+  API_BEGIN
+  GR_ARG(g && ws, "NULL argument");
+  GR_ARG(valid_comp(m, c), "composition does not belong to the model");
+  GR_ARG(K1 > 0 && K2 > 0, "bad embedding sizes");
+  return layer_workspace(g, m, c, K1, K2, ws, saved);
+  API_END
+}
+
+static granii_status check_args(granii_graph g, granii_model m, granii_composition c, const granii_layer_args* a) {
+  GR_ARG(g && a, "NULL argument");
+  GR_ARG(valid_comp(m, c), "composition does not belong to the model");
+  GR_ARG(a->K1 > 0 && a->K2 > 0 && a->ldh >= a->K1, "bad embedding sizes");
+  GR_ARG(a->H && a->W, "NULL H or W");
+  GR_ARG(a->act <= GRANII_ACT_RELU && a->attn <= GRANII_ATTN_DOT, "bad act/attn");
+  GR_ARG(m != GRANII_GAT || a->attn == GRANII_ATTN_DOT || (a->a_l && a->a_r), "GAT additive needs a_l, a_r");
+  GR_ARG(a->workspace, "NULL workspace");
+  if (g->world > 1) GR_ARG(a->comm && a->comm->world == g->world && a->comm->rank == g->rank,
+                           "partitioned graph needs the matching communicator");
+  else GR_ARG(!a->comm || a->comm->world == 1, "communicator given for an unpartitioned graph");
+  return GRANII_OK;
+}
+
+granii_status granii_layer_forward(granii_graph g, granii_model m, granii_composition c, const granii_layer_args* a,
+                                   float* d_out, int64_t ldo, float* d_saved, void* stream) {
+  API_BEGIN
+  GR_TRY(check_args(g, m, c, a));
+  GR_ARG(d_out && ldo >= a->K2, "bad output");
+  return layer_forward(g, m, c, a, d_out, ldo, d_saved, (cudaStream_t)stream);
+  API_END
+}
+
+granii_status granii_layer_backward(granii_graph g, granii_model m, granii_composition c, const granii_layer_args* a,
+                                    const float* d_out, int64_t ldo, const float* d_dout, int64_t lddo,
+                                    const float* d_saved, float* d_dH, int64_t lddh, float* d_dW, void* stream) {
+  API_BEGIN
+  GR_TRY(check_args(g, m, c, a));
+  if (m != GRANII_GCN) return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is not implemented (SURVEY N2)");
+  GR_ARG(g->symmetric, "backward needs a symmetric graph (created with GRANII_SYMMETRIZE): M^T = M");
+  GR_ARG(d_out && d_dout && d_dW && ldo >= a->K2 && lddo >= a->K2, "bad output / gradient");
+  GR_ARG(!d_dH || lddh >= a->K1, "bad lddh");
+  return layer_backward(g, c, a, d_out, ldo, d_dout, lddo, d_saved, d_dH, lddh, d_dW, (cudaStream_t)stream);
+  API_END
+}
+
+granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t K2, const char* calib_path,
+                            uint32_t flags, granii_composition* out, int32_t* candidates, double* predicted_ms,
+                            int32_t* n_candidates) {
+  API_BEGIN
+  GR_ARG(g && out, "NULL argument");
+  GR_ARG(m == GRANII_GCN || m == GRANII_GAT, "bad model");
+  GR_ARG(K1 > 0 && K2 > 0, "bad embedding sizes");
+  return select_impl(g, m, K1, K2, calib_path, flags, out, candidates, predicted_ms, n_candidates);
+  API_END
+}
+
+granii_status granii_comm_unique_id(void* id) {
+  GR_ARG(id, "NULL id");
+  return comm_unique_id(id);
+}
+granii_status granii_comm_create(const void* id, int32_t rank, int32_t world, granii_comm* out) {
+  GR_ARG(id && out && world >= 1 && rank >= 0 && rank < world, "bad argument");
+  return comm_create(id, rank, world, out);
+}
+granii_status granii_comm_destroy(granii_comm c) { return comm_destroy(c); }
+
+granii_status granii_softmax_xent(int64_t rows, int64_t C, const float* d_Z, int64_t ldz, const int32_t* d_y,
+                                  int64_t n_total, float* d_dZ, int64_t lddz, float* d_loss, void* stream) {
+  GR_ARG(rows >= 0 && C > 0 && ldz >= C && lddz >= C && n_total > 0, "bad sizes");
+  GR_ARG(rows == 0 || (d_Z && d_y && d_dZ), "NULL argument");
+  return launch_softmax_xent(rows, C, d_Z, ldz, d_y, n_total, d_dZ, lddz, d_loss, (cudaStream_t)stream);
+}
+
+granii_status granii_sgd(int64_t n, float lr, const float* d_grad, float* d_param, void* stream) {
+  GR_ARG(n >= 0 && (n == 0 || (d_grad && d_param)), "bad argument");
+  return launch_sgd(n, lr, d_grad, d_param, (cudaStream_t)stream);
+}
+
+}  // extern "C"

@@ -1,0 +1,93 @@
+// elementwise.cu -- small HBM-bound helpers around the layers: ReLU backward
+// mask, padded row copies, softmax cross-entropy (training loss) and SGD.
+#include <algorithm>
+#include <cmath>
+
+#include "internal.h"
+
+namespace granii {
+
+static unsigned blocks_for(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
+
+__global__ void k_relu_mask(int64_t rows, int64_t K, const float* __restrict__ out, int64_t ldo,
+                            const float* __restrict__ g, int64_t ldg, float* __restrict__ dst, int64_t ldd) {
+  const int64_t total = rows * K;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / K, k = i % K;
+    dst[r * ldd + k] = out[r * ldo + k] > 0.f ? g[r * ldg + k] : 0.f;   // ReLU'(0) = 0
+  }
+}
+
+__global__ void k_copy_rows(int64_t rows, int64_t K, const float* __restrict__ src, int64_t lds,
+                            float* __restrict__ dst, int64_t ldd) {
+  const int64_t total = rows * K;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / K, k = i % K;
+    dst[r * ldd + k] = src[r * lds + k];
+  }
+}
+
+// one warp per row
+__global__ void k_softmax_xent(int64_t rows, int64_t C, const float* __restrict__ Z, int64_t ldz,
+                               const int32_t* __restrict__ y, float inv_n, float* __restrict__ dZ, int64_t lddz,
+                               float* __restrict__ loss) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = warp; r < rows; r += nw) {
+    const float* z = Z + r * ldz;
+    float m = -INFINITY;
+    for (int64_t c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float s = 0.f;
+    for (int64_t c = lane; c < C; c += 32) s += expf(z[c] - m);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    const int32_t t = y[r];
+    for (int64_t c = lane; c < C; c += 32) {
+      const float p = expf(z[c] - m) / s;
+      dZ[r * lddz + c] = (p - (c == t ? 1.f : 0.f)) * inv_n;
+    }
+    if (loss && lane == 0) loss[r] = logf(s) + m - z[t];
+  }
+}
+
+__global__ void k_sgd(int64_t n, float lr, const float* __restrict__ g, float* __restrict__ p) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] -= lr * g[i];
+}
+
+granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
+                               float* dst, int64_t ldd, cudaStream_t st) {
+  if (rows * K == 0) return GRANII_OK;
+  k_relu_mask<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, out, ldo, g, ldg, dst, ldd);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,
+                               cudaStream_t st) {
+  if (rows * K == 0) return GRANII_OK;
+  k_copy_rows<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, src, lds, dst, ldd);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_softmax_xent(int64_t rows, int64_t C, const float* Z, int64_t ldz, const int32_t* y,
+                                  int64_t n_total, float* dZ, int64_t lddz, float* loss, cudaStream_t st) {
+  if (rows == 0) return GRANII_OK;
+  const unsigned b = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, 8), 148 * 16));
+  k_softmax_xent<<<b, 256, 0, st>>>(rows, C, Z, ldz, y, 1.f / (float)n_total, dZ, lddz, loss);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_sgd(int64_t n, float lr, const float* g, float* p, cudaStream_t st) {
+  if (n == 0) return GRANII_OK;
+  k_sgd<<<blocks_for(n), 256, 0, st>>>(n, lr, g, p);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+}  // namespace granii

@@ -1,0 +1,575 @@
+// gemm.cu -- the update GEMM (Θ = H W of Eq. 4)
+// on 5th-generation tensor cores, fp32-accurate.
+//
+// C[M x N] = A[M x K] · B[K x N] (+ fused epilogue: row scale = Eq. 1 row-
+// broadcast, GAT attention GEMVs el = C a_l / er = C a_r, ReLU).
+//
+// Tensor-core path, one CTA per 128 x BN output tile:
+//   warp 0      TMA producer: A tile (128 x 32 fp32, SWIZZLE_128B) and the
+//               pre-split B_hi / B_lo tiles (BN x 32, K-major) per stage
+//   warp 1      TMEM allocator + MMA issuer (one elected thread):
+//               3 x tcgen05.mma.kind::tf32 per 8-wide k step
+//               (A_hi B_hi + A_hi B_lo + A_lo B_hi -- the 3xTF32 split)
+//   warps 2..5  split A in shared memory (hi = rna(A), lo = rna(A - hi),
+//               in place + a second buffer; elementwise, so the swizzled layout
+//               is preserved), then the epilogue: tcgen05.ld 32x32b -> regs ->
+//               scale / GEMVs / ReLU -> global.
+// Pipelines: full[s] (TMA -> converters, tx bytes), conv[s] (converters ->
+// MMA), empty[s] (tcgen05.commit -> TMA), accum (last commit -> epilogue).
+// B (the weight, <= K1 x K2 floats) is split and transposed once per call
+// into the workspace by a tiny prep kernel.
+//
+// Fallback (lda % 4 != 0, transposed A, or no TMA alignment): fp32 SIMT tiles.
+// dW = Aᵀ B (reduction over the node dimension) uses a deterministic split-K
+// SIMT kernel + fixed-order reduction.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <mutex>
+
+#include "internal.h"
+
+namespace granii {
+
+// ======================================================================= PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::
+          "r"(smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void fence_barrier_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// UMMA shared-memory descriptor, K-major, SWIZZLE_128B (rows of 128 B, 8-row groups 1024 B apart).
+__device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);  // start address  [0,14)
+  d |= (uint64_t)1 << 16;                    // leading byte offset (unused for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;          // stride byte offset = 1024 B
+  d |= (uint64_t)1 << 46;                    // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;                    // SWIZZLE_128B
+  return d;
+}
+// instruction descriptor: D fp32, A/B tf32, both K-major, M = 128, N = BN
+__host__ __device__ constexpr uint32_t idesc_tf32(int M, int N) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+__device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ float tf32_rna(float x) {
+  uint32_t r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return __uint_as_float(r);
+}
+
+// ======================================================================= tcgen05 kernel
+constexpr int TC_BM = 128, TC_BK = 32;  // 32 fp32 = one 128-byte swizzle row
+
+template <int BN>
+struct TcCfg {
+  static constexpr int A_BYTES = TC_BM * TC_BK * 4;  // 16 KB
+  static constexpr int B_BYTES = BN * TC_BK * 4;
+  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int STAGES = (STAGE * 3 <= 200 * 1024) ? 3 : 2;
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int SMEM = STAGES * STAGE + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+struct TcEpi {
+  float* C;
+  int64_t ldc;
+  const float* row_scale;
+  const float* att_l;
+  const float* att_r;
+  float* out_l;  // [n_tiles_n][M] partials (or final when one N tile)
+  float* out_r;
+  int relu;
+  int store;
+};
+
+template <int BN>
+__global__ void __launch_bounds__(192, 1)
+    k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
+              const __grid_constant__ CUtensorMap tmBl, int M, int N, int K, TcEpi ep) {
+  using Cfg = TcCfg<BN>;
+  constexpr int S = Cfg::STAGES;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint64_t* bars = (uint64_t*)(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* accum = bars + 3 * S;
+  uint32_t* tmem_slot = (uint32_t*)(bars + 3 * S + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m0 = blockIdx.x * TC_BM, n0 = blockIdx.y * BN;
+  const int nk = (K + TC_BK - 1) / TC_BK;
+
+  auto a_hi = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto a_lo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto b_hi = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
+  auto b_lo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(accum, 1);
+    fence_barrier_init();
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmBh) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmBl) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(Cfg::TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A_BYTES + 2 * Cfg::B_BYTES);
+        tma_load_2d(&tmA, &full[s], a_hi(s), kb * TC_BK, m0);
+        tma_load_2d(&tmBh, &full[s], b_hi(s), kb * TC_BK, n0);
+        tma_load_2d(&tmBl, &full[s], b_lo(s), kb * TC_BK, n0);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      constexpr uint32_t idesc = idesc_tf32(TC_BM, BN);
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&conv[s], ph);
+        tc_fence_after();
+        const uint32_t ah = smem_u32(a_hi(s)), al = smem_u32(a_lo(s));
+        const uint32_t bh = smem_u32(b_hi(s)), bl = smem_u32(b_lo(s));
+#pragma unroll
+        for (int k = 0; k < TC_BK / 8; ++k) {  // tf32: K = 8 per MMA = 32 bytes
+          const uint32_t off = k * 32;
+          const uint64_t dah = desc_sw128(ah + off), dal = desc_sw128(al + off);
+          const uint64_t dbh = desc_sw128(bh + off), dbl = desc_sw128(bl + off);
+          mma_tf32(tmem, dah, dbh, idesc, (kb | k) ? 1u : 0u);
+          mma_tf32(tmem, dah, dbl, idesc, 1u);
+          mma_tf32(tmem, dal, dbh, idesc, 1u);
+        }
+        mma_commit(&empty[s]);
+      }
+      mma_commit(accum);
+    }
+  } else {
+    // ---------------- converters: split A into tf32 hi / lo in place
+    const int ct = threadIdx.x - 64;  // 0..127
+    for (int kb = 0; kb < nk; ++kb) {
+      const int s = kb % S;
+      const uint32_t ph = (kb / S) & 1;
+      mbar_wait(&full[s], ph);
+      float4* hi = reinterpret_cast<float4*>(a_hi(s));
+      float4* lo = reinterpret_cast<float4*>(a_lo(s));
+#pragma unroll
+      for (int i = 0; i < Cfg::A_BYTES / 16 / 128; ++i) {
+        const int idx = ct + i * 128;
+        float4 x = hi[idx];
+        float4 h, l;
+        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
+        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
+        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
+        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
+        hi[idx] = h;
+        lo[idx] = l;
+      }
+      fence_proxy_async();
+      mbar_arrive(&conv[s]);
+    }
+    // ---------------- epilogue: TMEM -> registers -> global
+    mbar_wait(accum, 0);
+    tc_fence_after();
+    const int quad = warp & 3;  // TMEM lanes [32*quad, 32*quad+32)
+    const int r = m0 + quad * 32 + lane;
+    const bool rok = r < M;
+    const float rsc = (ep.row_scale && rok) ? __ldg(ep.row_scale + r) : 1.f;
+    float el = 0.f, er = 0.f;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      float v[16];
+      tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + c0, v);
+      const int cb = n0 + c0;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        v[j] *= rsc;
+        if (cb + j < N) {
+          if (ep.att_l) el = fmaf(v[j], __ldg(ep.att_l + cb + j), el);
+          if (ep.att_r) er = fmaf(v[j], __ldg(ep.att_r + cb + j), er);
+        }
+        if (ep.relu) v[j] = fmaxf(v[j], 0.f);
+      }
+      if (ep.store && rok) {
+        float* crow = ep.C + (int64_t)r * ep.ldc + cb;
+        if (cb + 16 <= N && ((((uintptr_t)crow) & 15) == 0)) {
+#pragma unroll
+          for (int j = 0; j < 16; j += 4) *reinterpret_cast<float4*>(crow + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+        } else {
+#pragma unroll
+          for (int j = 0; j < 16; ++j)
+            if (cb + j < N) crow[j] = v[j];
+        }
+      }
+    }
+    if (rok) {
+      if (ep.out_l) ep.out_l[(int64_t)blockIdx.y * M + r] = el;
+      if (ep.out_r) ep.out_r[(int64_t)blockIdx.y * M + r] = er;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS));
+  }
+}
+
+// B (K x N, or N x K when transposed) -> Bt_hi / Bt_lo [Npad x Kpad], K-major, zero padded.
+__global__ void k_prep_b(int K, int N, const float* __restrict__ B, int64_t ldb, int transB, int Kpad, int Npad,
+                         float* __restrict__ hi, float* __restrict__ lo) {
+  const int64_t total = (int64_t)Npad * Kpad;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(i / Kpad), k = (int)(i % Kpad);
+    float x = 0.f;
+    if (n < N && k < K) x = transB ? B[(int64_t)n * ldb + k] : B[(int64_t)k * ldb + n];
+    const float h = tf32_rna(x);
+    hi[i] = h;
+    lo[i] = tf32_rna(x - h);
+  }
+}
+
+// sum the per-N-tile attention partials in fixed tile order
+__global__ void k_reduce_partials(int M, int tiles, const float* __restrict__ part, float* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
+    float s = 0.f;
+    for (int t = 0; t < tiles; ++t) s += part[(int64_t)t * M + i];
+    out[i] = s;
+  }
+}
+
+// ======================================================================= SIMT fallback
+// C = op(A) op(B), 64x64 tile / 256 threads, 4x4 per thread.  Deterministic.
+template <bool TA, bool TB>
+__global__ void __launch_bounds__(256) k_gemm_simt(int M, int N, int K, const float* __restrict__ A, int64_t lda,
+                                                   const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
+                                                   int64_t ldc, const float* __restrict__ rs, int relu) {
+  __shared__ float As[16][64 + 1];
+  __shared__ float Bs[16][64 + 1];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int m0 = blockIdx.x * 64, n0 = blockIdx.y * 64;
+  float acc[4][4] = {};
+  for (int k0 = 0; k0 < K; k0 += 16) {
+    for (int i = threadIdx.x; i < 16 * 64; i += 256) {
+      const int kk = i / 64, mm = i % 64;
+      const int gm = m0 + mm, gk = k0 + kk;
+      As[kk][mm] = (gm < M && gk < K) ? (TA ? A[(int64_t)gk * lda + gm] : A[(int64_t)gm * lda + gk]) : 0.f;
+      const int gn = n0 + mm;
+      Bs[kk][mm] = (gn < N && gk < K) ? (TB ? B[(int64_t)gn * ldb + gk] : B[(int64_t)gk * ldb + gn]) : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < 16; ++kk) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int gm = m0 + ty * 4 + i;
+    if (gm >= M) continue;
+    const float s = rs ? rs[gm] : 1.f;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int gn = n0 + tx * 4 + j;
+      if (gn < N) {
+        float v = acc[i][j] * s;
+        if (relu) v = fmaxf(v, 0.f);
+        C[(int64_t)gm * ldc + gn] = v;
+      }
+    }
+  }
+}
+
+// C[M x N] = Aᵀ B with A stored R x M, B stored R x N (R = reduction, e.g. nodes).
+// Split over R into `splits` chunks; partials [splits][M][N] then fixed-order sum.
+__global__ void __launch_bounds__(256) k_gemm_tn_part(int M, int N, int64_t R, int64_t chunk, const float* __restrict__ A,
+                                                      int64_t lda, const float* __restrict__ B, int64_t ldb,
+                                                      float* __restrict__ part) {
+  __shared__ float As[32][64 + 1];
+  __shared__ float Bs[32][64 + 1];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int m0 = blockIdx.x * 64, n0 = blockIdx.y * 64;
+  const int64_t r0 = blockIdx.z * chunk, r1 = min(R, r0 + chunk);
+  float acc[4][4] = {};
+  for (int64_t k0 = r0; k0 < r1; k0 += 32) {
+    for (int i = threadIdx.x; i < 32 * 64; i += 256) {
+      const int kk = i / 64, mm = i % 64;
+      const int64_t gk = k0 + kk;
+      As[kk][mm] = (m0 + mm < M && gk < r1) ? A[gk * lda + m0 + mm] : 0.f;
+      Bs[kk][mm] = (n0 + mm < N && gk < r1) ? B[gk * ldb + n0 + mm] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll 8
+    for (int kk = 0; kk < 32; ++kk) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+  float* P = part + (int64_t)blockIdx.z * M * N;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int gm = m0 + ty * 4 + i;
+    if (gm >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int gn = n0 + tx * 4 + j;
+      if (gn < N) P[(int64_t)gm * N + gn] = acc[i][j];
+    }
+  }
+}
+
+__global__ void k_sum_splits(int64_t MN, int splits, const float* __restrict__ part, float* __restrict__ C, int M, int N,
+                             int64_t ldc) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < MN; i += (int64_t)gridDim.x * blockDim.x) {
+    float s = 0.f;
+    for (int t = 0; t < splits; ++t) s += part[(int64_t)t * MN + i];
+    C[(i / N) * ldc + (i % N)] = s;
+  }
+}
+
+// ======================================================================= host side
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+  });
+  return fn;
+}
+
+static bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                     uint32_t box_inner, uint32_t box_outer) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld_elems * 4};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+static int pick_bn(int64_t N) {
+  if (N <= 16) return 16;
+  if (N <= 32) return 32;
+  if (N <= 48) return 48;
+  if (N <= 64) return 64;
+  if (N <= 96) return 96;
+  if (N <= 128) return 128;
+  if (N <= 192) return 192;
+  return 256;
+}
+
+static bool tc_eligible(int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, uint32_t flags) {
+  if (flags & GRANII_GEMM_TRANS_A) return false;
+  if (getenv("GRANII_GEMM_SIMT")) return false;
+  if (lda % 4 != 0 || ((uintptr_t)A & 15)) return false;
+  if (M <= 0 || N <= 0 || K <= 0) return false;
+  if (M > INT32_MAX || K > INT32_MAX) return false;
+  return true;
+}
+
+size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags) {
+  size_t ws = 0;
+  if (flags & GRANII_GEMM_TRANS_A) {
+    // split-K partials
+    const int64_t splits = std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(K, 4096)));
+    return (size_t)splits * M * N * 4 + 256;
+  }
+  const int bn = pick_bn(N);
+  const int64_t Npad = round_up(N, bn), Kpad = round_up(K, TC_BK);
+  ws += (size_t)2 * Npad * Kpad * 4 + 1024;
+  const int64_t tiles = ceil_div(N, bn);
+  ws += (size_t)2 * tiles * M * 4 + 256;  // attention partials
+  return ws;
+}
+
+template <int BN>
+static granii_status launch_tc_bn(int M, int N, int K, const CUtensorMap& ta, const CUtensorMap& tbh,
+                                  const CUtensorMap& tbl, const TcEpi& ep, cudaStream_t st) {
+  using Cfg = TcCfg<BN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    GR_CUDA(cudaFuncSetAttribute(k_gemm_tc<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+    attr_set = true;
+  }
+  dim3 grid((unsigned)ceil_div(M, TC_BM), (unsigned)ceil_div(N, BN));
+  k_gemm_tc<BN><<<grid, 192, Cfg::SMEM, st>>>(ta, tbh, tbl, M, N, K, ep);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+                          int64_t ldb, float* C, int64_t ldc, const granii_gemm_epilogue* epi, uint32_t flags,
+                          void* ws, size_t ws_bytes, cudaStream_t st) {
+  if (M == 0 || N == 0) return GRANII_OK;
+  const bool relu = flags & GRANII_GEMM_RELU;
+  const bool store = !(flags & GRANII_GEMM_NO_STORE);
+  const bool tb = flags & GRANII_GEMM_TRANS_B;
+  const float* rs = epi ? epi->row_scale : nullptr;
+  const bool att = epi && (epi->att_l || epi->att_r);
+  if (ws_bytes < gemm_workspace(M, N, K, flags)) return fail(GRANII_ERR_INVALID_ARG, "gemm workspace too small");
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+
+  if (flags & GRANII_GEMM_TRANS_A) {
+    if (att || rs || relu || tb) return fail(GRANII_ERR_UNSUPPORTED, "TRANS_A supports plain C = A^T B only");
+    // here K is the reduction (rows), A stored K x M, B stored K x N
+    const int64_t splits = std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(K, 4096)));
+    const int64_t chunk = round_up(ceil_div(K, splits), 32);
+    float* part = (float*)ws;
+    dim3 grid((unsigned)ceil_div(M, 64), (unsigned)ceil_div(N, 64), (unsigned)splits);
+    k_gemm_tn_part<<<grid, 256, 0, st>>>((int)M, (int)N, K, chunk, A, lda, B, ldb, part);
+    GR_CHECK_LAUNCH();
+    const int64_t MN = M * N;
+    k_sum_splits<<<(unsigned)std::min<int64_t>(ceil_div(MN, 256), 4096), 256, 0, st>>>(MN, (int)splits, part, C,
+                                                                                      (int)M, (int)N, ldc);
+    GR_CHECK_LAUNCH();
+    return GRANII_OK;
+  }
+
+  if (!tc_eligible(M, N, K, A, lda, flags)) {
+    if (att) return fail(GRANII_ERR_UNSUPPORTED, "attention epilogue needs the tensor-core path (lda % 4 == 0)");
+    dim3 grid((unsigned)ceil_div(M, 64), (unsigned)ceil_div(N, 64));
+    if (!store) return GRANII_OK;
+    if (tb) k_gemm_simt<false, true><<<grid, 256, 0, st>>>((int)M, (int)N, (int)K, A, lda, B, ldb, C, ldc, rs, relu);
+    else k_gemm_simt<false, false><<<grid, 256, 0, st>>>((int)M, (int)N, (int)K, A, lda, B, ldb, C, ldc, rs, relu);
+    GR_CHECK_LAUNCH();
+    return GRANII_OK;
+  }
+
+  const int bn = pick_bn(N);
+  const int64_t Npad = round_up(N, bn), Kpad = round_up(K, TC_BK);
+  uint8_t* w = (uint8_t*)(((uintptr_t)ws + 1023) & ~(uintptr_t)1023);
+  float* bhi = (float*)w;
+  float* blo = bhi + Npad * Kpad;
+  float* part_l = blo + Npad * Kpad;
+  const int64_t tiles = ceil_div(N, bn);
+  float* part_r = part_l + tiles * M;
+  k_prep_b<<<(unsigned)std::min<int64_t>(ceil_div(Npad * Kpad, 256), 4096), 256, 0, st>>>(
+      (int)K, (int)N, B, ldb, tb ? 1 : 0, (int)Kpad, (int)Npad, bhi, blo);
+  GR_CHECK_LAUNCH();
+
+  CUtensorMap ta, tbh, tbl;
+  if (!make_map(&ta, A, (uint64_t)K, (uint64_t)M, (uint64_t)lda, TC_BK, TC_BM) ||
+      !make_map(&tbh, bhi, (uint64_t)Kpad, (uint64_t)Npad, (uint64_t)Kpad, TC_BK, bn) ||
+      !make_map(&tbl, blo, (uint64_t)Kpad, (uint64_t)Npad, (uint64_t)Kpad, TC_BK, bn))
+    return fail(GRANII_ERR_CUDA, "cuTensorMapEncodeTiled failed");
+
+  TcEpi ep{C, ldc, rs, epi ? epi->att_l : nullptr, epi ? epi->att_r : nullptr, nullptr, nullptr, relu ? 1 : 0,
+           store ? 1 : 0};
+  if (epi && epi->att_l && epi->out_l) ep.out_l = tiles == 1 ? epi->out_l : part_l;
+  if (epi && epi->att_r && epi->out_r) ep.out_r = tiles == 1 ? epi->out_r : part_r;
+  switch (bn) {
+    case 16: GR_TRY(launch_tc_bn<16>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 32: GR_TRY(launch_tc_bn<32>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 48: GR_TRY(launch_tc_bn<48>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 64: GR_TRY(launch_tc_bn<64>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 96: GR_TRY(launch_tc_bn<96>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 128: GR_TRY(launch_tc_bn<128>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    case 192: GR_TRY(launch_tc_bn<192>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    default: GR_TRY(launch_tc_bn<256>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+  }
+  if (tiles > 1) {
+    const unsigned b = (unsigned)std::min<int64_t>(ceil_div(M, 256), 4096);
+    if (ep.out_l) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_l, epi->out_l);
+    if (ep.out_r) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_r, epi->out_r);
+    GR_CHECK_LAUNCH();
+  }
+  return GRANII_OK;
+}
+
+}  // namespace granii

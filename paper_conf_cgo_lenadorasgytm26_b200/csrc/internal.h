@@ -1,0 +1,98 @@
+// internal.h -- shared declarations of the B200 GRANII library (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/granii.h"
+
+namespace granii {
+
+// ----------------------------------------------------------------- errors
+struct Error {
+  granii_status st;
+  std::string msg;
+};
+void set_error(const std::string& m);
+granii_status fail(granii_status st, const std::string& m);
+#define GR_CUDA(call)                                                                      \
+  do {                                                                                     \
+    cudaError_t e_ = (call);                                                               \
+    if (e_ != cudaSuccess)                                                                 \
+      return ::granii::fail(GRANII_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+#define GR_CHECK_LAUNCH()                                                                  \
+  do {                                                                                     \
+    cudaError_t e_ = cudaGetLastError();                                                   \
+    if (e_ != cudaSuccess)                                                                 \
+      return ::granii::fail(GRANII_ERR_CUDA, std::string("launch: ") + cudaGetErrorString(e_)); \
+  } while (0)
+#define GR_TRY(x)                                \
+  do {                                           \
+    granii_status s_ = (x);                      \
+    if (s_ != GRANII_OK) return s_;              \
+  } while (0)
+#define GR_ARG(cond, msg)                                               \
+  do {                                                                  \
+    if (!(cond)) return ::granii::fail(GRANII_ERR_INVALID_ARG, msg);    \
+  } while (0)
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline int64_t round_up(int64_t a, int64_t b) { return ceil_div(a, b) * b; }
+
+// ----------------------------------------------------------------- device info
+struct DevInfo {
+  int device = -1;
+  int sms = 148;
+  int64_t l2_bytes = 126ll << 20;
+};
+granii_status dev_info(DevInfo* out);
+
+}  // namespace granii
+
+// ----------------------------------------------------------------- graph
+struct granii_graph_s {
+  int64_t N = 0;            // global nodes
+  int64_t nnz = 0;          // global stored entries
+  int64_t row_begin = 0, row_end = 0, n_rows = 0;
+  int64_t local_nnz = 0;
+  int32_t rank = 0, world = 1;
+  int64_t max_rows = 0;     // gather-layout block height
+  int64_t n_cols = 0;       // size of the column-id space (N, or world*max_rows)
+  int32_t symmetric = 0;
+  std::vector<int64_t> bounds;
+  int64_t* row_ptr = nullptr;     // device, n_rows+1, rebased
+  int32_t* col_idx = nullptr;     // device, local_nnz, column-id space
+  float* dinv_rows = nullptr;     // device, n_rows
+  float* dinv_cols = nullptr;     // device, n_cols (== dinv_rows when world == 1)
+  int32_t* order = nullptr;       // device, n_rows: owned rows by descending degree
+  int64_t features[GRANII_NUM_FEATURES] = {0};
+  int device = 0;
+  float avg_deg() const { return n_rows > 0 ? float(local_nnz) / float(n_rows) : 0.f; }
+};
+
+struct granii_comm_s {
+  void* nccl = nullptr;  // ncclComm_t
+  int32_t rank = 0, world = 1;
+};
+
+namespace granii {
+// kernels (launchers); all validate nothing -- callers in api.cu validate.
+granii_status launch_spmm(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                          float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, cudaStream_t st);
+granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U, int64_t ldu, const float* V,
+                           int64_t ldv, int64_t K, float scale, float* out, cudaStream_t st);
+size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags);
+granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+                          int64_t ldb, float* C, int64_t ldc, const granii_gemm_epilogue* epi, uint32_t flags,
+                          void* ws, size_t ws_bytes, cudaStream_t st);
+granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g,
+                               int64_t ldg, float* dst, int64_t ldd, cudaStream_t st);
+granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,
+                               cudaStream_t st);
+// comm
+granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
+granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);
+}  // namespace granii

@@ -1,0 +1,359 @@
+// layer.cu -- one GNN layer under an explicit composition (§III).
+//
+// GCN (Eq. 2 L115 / Eq. 3), GAT (Eq. 4-6).  Each composition
+// is the paper's primitive sequence with the element-wise work fused into the
+// primitive that produces or consumes it:
+//   PRE_AGG : SDDMM(dinv,dinv)->Ñ ; SpMM_w(Ñ, H)[K1] ; GEMM(·W)+σ
+//   PRE_UPD : SDDMM ; GEMM(H W) ; SpMM_w(Ñ, ·)[K2]+σ
+//   DYN_AGG : SpMM_u(Ã, H) with the pre-scale D̃^-½ in the gather and the
+//             post-scale in the epilogue [K1] ; GEMM(·W)+σ
+//   DYN_UPD : GEMM(H W) with the row-broadcast D̃^-½ in its epilogue ;
+//             SpMM_u(Ã, ·)[K2] with D̃^-½ in its epilogue +σ
+//   GAT_REUSE  : GEMM Θ = H W (+ el = Θ a_l, er = Θ a_r in the epilogue) ;
+//                SDDMM(el, er) + LeakyReLU + row softmax -> α ; SpMM_w(α, Θ)[K2]+σ
+//   GAT_RECOMP : GEMM (el, er only; Θ is never written) ; SDDMM -> α ;
+//                SpMM_w(α, H)[K1] ; GEMM(·W)+σ  (the extra GEMM of L135)
+// Multi-GPU (comm != NULL): rows are partitioned; the dense operand of every
+// SpMM / SDDMM is produced straight into this rank's slot of a padded gather
+// buffer and all-gathered in place with NCCL before the sparse step.
+#include <algorithm>
+#include <cmath>
+
+#include "internal.h"
+
+namespace granii {
+
+struct Bump {
+  uint8_t* base;
+  size_t off = 0;
+  explicit Bump(void* b) : base((uint8_t*)b) {}
+  float* take(size_t floats) {
+    off = (size_t)round_up((int64_t)off, 1024);
+    float* p = base ? (float*)(base + off) : nullptr;
+    off += floats * sizeof(float);
+    return p;
+  }
+  void* take_bytes(size_t bytes) {
+    off = (size_t)round_up((int64_t)off, 1024);
+    void* p = base ? base + off : nullptr;
+    off += bytes;
+    return p;
+  }
+};
+
+static inline int64_t ld4(int64_t k) { return round_up(k, 4); }
+
+struct Ctx {
+  const granii_graph_s* g;
+  granii_comm_s* comm;
+  cudaStream_t st;
+  bool dist() const { return comm && comm->world > 1; }
+};
+
+// dense operand of a sparse step: in the gather buffer (dist) or plain local rows.
+struct GatherBuf {
+  float* all = nullptr;  // n_cols x ld
+  float* mine = nullptr; // this rank's slot (n_rows x ld)
+  int64_t ld = 0;
+};
+
+static GatherBuf gather_buf(Bump& b, const Ctx& c, int64_t K) {
+  GatherBuf gb;
+  gb.ld = ld4(K);
+  if (c.dist()) {
+    gb.all = b.take((size_t)c.g->n_cols * gb.ld);
+    gb.mine = gb.all ? gb.all + (int64_t)c.g->rank * c.g->max_rows * gb.ld : nullptr;
+  } else {
+    gb.all = b.take((size_t)std::max<int64_t>(c.g->n_rows, 1) * gb.ld);
+    gb.mine = gb.all;
+  }
+  return gb;
+}
+
+static granii_status allgather(const Ctx& c, GatherBuf& gb) {
+  if (!c.dist()) return GRANII_OK;
+  const size_t count = (size_t)c.g->max_rows * gb.ld;
+  return comm_allgather(c.comm, gb.mine, gb.all, count, c.st);
+}
+
+// scalar per-row vector (er) gather: one float per row
+static float* vec_buf(Bump& b, const Ctx& c) {
+  return b.take((size_t)(c.dist() ? c.g->n_cols : std::max<int64_t>(c.g->n_rows, 1)));
+}
+
+static granii_status gemm_ws(Bump& b, int64_t M, int64_t N, int64_t K, uint32_t flags, void** p, size_t* n) {
+  *n = gemm_workspace(M, N, K, flags);
+  *p = b.take_bytes(*n);
+  return GRANII_OK;
+}
+
+// ---------------------------------------------------------------- forward (plan + run)
+// Running with base == nullptr only sizes the workspace (no launches).
+static granii_status forward_impl(const Ctx& c, granii_model m, granii_composition comp, const granii_layer_args* a,
+                                  float* out, int64_t ldo, float* saved, void* ws_base, size_t* ws_size,
+                                  size_t* saved_floats) {
+  const granii_graph_s* g = c.g;
+  const bool run = ws_base != nullptr;
+  Bump b(ws_base);
+  const int64_t R = g->n_rows, K1 = a->K1, K2 = a->K2;
+  const bool relu = a->act == GRANII_ACT_RELU;
+  const cudaStream_t st = c.st;
+  if (saved_floats) *saved_floats = 0;
+
+  // H with a 16-byte row stride for the TMA GEMM path / vector gathers
+  const float* H = a->H;
+  int64_t ldh = a->ldh;
+  const bool h_aligned = (ldh % 4 == 0) && (((uintptr_t)H & 15) == 0);
+  float* hpad = nullptr;
+  const bool agg_first_gather = c.dist() && (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_DYN_AGG ||
+                                             comp == GRANII_GAT_RECOMP);
+  GatherBuf hg;
+  if (agg_first_gather) {
+    hg = gather_buf(b, c, K1);  // H goes into the gather slot (aligned copy)
+    if (run) {
+      GR_TRY(launch_copy_rows(R, K1, H, ldh, hg.mine, hg.ld, st));
+      GR_TRY(allgather(c, hg));
+    }
+    H = hg.mine;
+    ldh = hg.ld;
+  } else if (!h_aligned) {
+    hpad = b.take((size_t)std::max<int64_t>(R, 1) * ld4(K1));
+    if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hpad, ld4(K1), st));
+    H = hpad;
+    ldh = ld4(K1);
+  }
+  const float* Xagg = agg_first_gather ? hg.all : H;  // aggregation source (column-id space)
+  const int64_t ldxagg = ldh;
+
+  if (m == GRANII_GCN) {
+    float* nval = nullptr;
+    if (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_PRE_UPD) {
+      nval = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
+      if (run) GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT, g->dinv_rows, 1, g->dinv_cols, 1, 1, 1.f, nval, st));
+    }
+    switch (comp) {
+      case GRANII_GCN_PRE_AGG:
+      case GRANII_GCN_DYN_AGG: {
+        // T = (Ñ H) or (D Ã D H), K1 wide; kept for the backward pass
+        const int64_t ldt = ld4(K1);
+        if (saved_floats) *saved_floats = (size_t)R * ldt;
+        float* T = saved ? saved : b.take((size_t)std::max<int64_t>(R, 1) * ldt);
+        void* gw;
+        size_t gn;
+        gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw, &gn);
+        if (run) {
+          if (comp == GRANII_GCN_PRE_AGG)
+            GR_TRY(launch_spmm(g, nval, Xagg, ldxagg, K1, T, ldt, nullptr, nullptr, false, st));
+          else
+            GR_TRY(launch_spmm(g, nullptr, Xagg, ldxagg, K1, T, ldt, g->dinv_rows, g->dinv_cols, false, st));
+          GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
+        }
+        break;
+      }
+      case GRANII_GCN_PRE_UPD:
+      case GRANII_GCN_DYN_UPD: {
+        GatherBuf tg = gather_buf(b, c, K2);
+        void* gw;
+        size_t gn;
+        gemm_ws(b, R, K2, K1, 0, &gw, &gn);
+        if (run) {
+          granii_gemm_epilogue ep{comp == GRANII_GCN_DYN_UPD ? g->dinv_rows : nullptr, nullptr, nullptr, nullptr,
+                                  nullptr};
+          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, tg.mine, tg.ld, &ep, 0, gw, gn, st));
+          GR_TRY(allgather(c, tg));
+          if (comp == GRANII_GCN_PRE_UPD)
+            GR_TRY(launch_spmm(g, nval, tg.all, tg.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+          else
+            GR_TRY(launch_spmm(g, nullptr, tg.all, tg.ld, K2, out, ldo, g->dinv_rows, nullptr, relu, st));
+        }
+        break;
+      }
+      default:
+        return fail(GRANII_ERR_INVALID_ARG, "composition does not belong to GCN");
+    }
+  } else {  // GAT
+    if (comp != GRANII_GAT_REUSE && comp != GRANII_GAT_RECOMP)
+      return fail(GRANII_ERR_INVALID_ARG, "composition does not belong to GAT");
+    const bool dot = a->attn == GRANII_ATTN_DOT;
+    float* alpha = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
+    const bool need_theta = comp == GRANII_GAT_REUSE || dot;
+    GatherBuf th;
+    if (need_theta) th = gather_buf(b, c, K2);
+    float* el = nullptr;
+    float* er_all = nullptr;
+    if (!dot) {
+      el = b.take((size_t)std::max<int64_t>(R, 1));
+      er_all = vec_buf(b, c);
+    }
+    void* gw;
+    size_t gn;
+    gemm_ws(b, R, K2, K1, 0, &gw, &gn);
+    if (run) {
+      float* er_mine = er_all ? (c.dist() ? er_all + (int64_t)g->rank * g->max_rows : er_all) : nullptr;
+      granii_gemm_epilogue ep{nullptr, dot ? nullptr : a->a_l, dot ? nullptr : a->a_r, el, er_mine};
+      uint32_t fl = need_theta ? 0u : GRANII_GEMM_NO_STORE;
+      GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, need_theta ? th.mine : nullptr, need_theta ? th.ld : K2,
+                         &ep, fl, gw, gn, st));
+      if (need_theta) GR_TRY(allgather(c, th));
+      if (!dot) {
+        if (c.dist()) {
+          GatherBuf eb{er_all, er_mine, 1};
+          GR_TRY(comm_allgather(c.comm, er_mine, er_all, (size_t)g->max_rows, st));
+          (void)eb;
+        }
+        GR_TRY(launch_sddmm(g, GRANII_SDDMM_ADD | GRANII_SDDMM_LEAKYRELU | GRANII_SDDMM_ROW_SOFTMAX, el, 1, er_all,
+                            1, 1, 1.f, alpha, st));
+      } else {
+        GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT | GRANII_SDDMM_ROW_SOFTMAX, th.mine, th.ld, th.all, th.ld, K2,
+                            1.f / std::sqrt((float)K2), alpha, st));
+      }
+    }
+    if (comp == GRANII_GAT_REUSE) {
+      if (run) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+    } else {
+      const int64_t ldt = ld4(K1);
+      float* T = b.take((size_t)std::max<int64_t>(R, 1) * ldt);
+      void* gw2;
+      size_t gn2;
+      gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
+      if (run) {
+        GR_TRY(launch_spmm(g, alpha, Xagg, ldxagg, K1, T, ldt, nullptr, nullptr, false, st));
+        GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
+                           st));
+      }
+    }
+  }
+  if (ws_size) *ws_size = b.off + 1024;
+  return GRANII_OK;
+}
+
+static granii_status backward_impl(const Ctx& c, granii_composition comp, const granii_layer_args* a,
+                                   const float* out, int64_t ldo, const float* dout, int64_t lddo,
+                                   const float* saved, float* dH, int64_t lddh, float* dW, void* ws_base,
+                                   size_t* ws_size) {
+  const granii_graph_s* g = c.g;
+  const bool run = ws_base != nullptr;
+  Bump b(ws_base);
+  const int64_t R = g->n_rows, K1 = a->K1, K2 = a->K2;
+  const cudaStream_t st = c.st;
+  const bool relu = a->act == GRANII_ACT_RELU;
+
+  // dY = dout ⊙ 1[out > 0]; written into a gather slot when the next sparse step needs it
+  const bool dy_gathered = comp == GRANII_GCN_PRE_UPD || comp == GRANII_GCN_DYN_UPD;
+  GatherBuf dyg = gather_buf(b, c, K2);
+  if (run) {
+    if (relu) GR_TRY(launch_relu_mask(R, K2, out, ldo, dout, lddo, dyg.mine, dyg.ld, st));
+    else GR_TRY(launch_copy_rows(R, K2, dout, lddo, dyg.mine, dyg.ld, st));
+  }
+  const float* dY = dyg.mine;
+  const int64_t lddy = dyg.ld;
+
+  // aligned H (needed by the dW GEMM of the *_UPD compositions)
+  const float* H = a->H;
+  int64_t ldh = a->ldh;
+  float* nval = nullptr;
+  if (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_PRE_UPD) {
+    nval = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
+    if (run) GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT, g->dinv_rows, 1, g->dinv_cols, 1, 1, 1.f, nval, st));
+  }
+  void* gwW;
+  size_t gnW;
+  gemm_ws(b, K1, K2, R, GRANII_GEMM_TRANS_A, &gwW, &gnW);
+  void* gwH;
+  size_t gnH;
+  gemm_ws(b, R, K1, K2, GRANII_GEMM_TRANS_B, &gwH, &gnH);
+  GatherBuf dtg;  // gathered operand for the dH SpMM (*_AGG)
+  float* dT = nullptr;
+  const int64_t ldt1 = ld4(K1), ldt2 = ld4(K2);
+  if (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_DYN_AGG) {
+    if (dH) dtg = gather_buf(b, c, K1);
+  } else {
+    dT = b.take((size_t)std::max<int64_t>(R, 1) * ldt2);
+  }
+
+  if (run) {
+    switch (comp) {
+      case GRANII_GCN_PRE_AGG:   // saved T = Ñ H
+      case GRANII_GCN_DYN_AGG: { // saved S' = D Ã D H
+        if (!saved) return fail(GRANII_ERR_INVALID_ARG, "this composition's backward needs d_saved");
+        GR_TRY(launch_gemm(K1, K2, R, saved, ldt1, dY, lddy, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
+        if (dH) {
+          granii_gemm_epilogue ep{comp == GRANII_GCN_DYN_AGG ? g->dinv_rows : nullptr, nullptr, nullptr, nullptr,
+                                  nullptr};
+          GR_TRY(launch_gemm(R, K1, K2, dY, lddy, a->W, K2, dtg.mine, dtg.ld, &ep, GRANII_GEMM_TRANS_B, gwH, gnH, st));
+          GR_TRY(allgather(c, dtg));
+          if (comp == GRANII_GCN_PRE_AGG)
+            GR_TRY(launch_spmm(g, nval, dtg.all, dtg.ld, K1, dH, lddh, nullptr, nullptr, false, st));
+          else
+            GR_TRY(launch_spmm(g, nullptr, dtg.all, dtg.ld, K1, dH, lddh, g->dinv_rows, nullptr, false, st));
+        }
+        break;
+      }
+      case GRANII_GCN_PRE_UPD:
+      case GRANII_GCN_DYN_UPD: {
+        GR_TRY(allgather(c, dyg));
+        if (comp == GRANII_GCN_PRE_UPD)
+          GR_TRY(launch_spmm(g, nval, dyg.all, dyg.ld, K2, dT, ldt2, nullptr, nullptr, false, st));
+        else
+          GR_TRY(launch_spmm(g, nullptr, dyg.all, dyg.ld, K2, dT, ldt2, g->dinv_rows, g->dinv_cols, false, st));
+        GR_TRY(launch_gemm(K1, K2, R, H, ldh, dT, ldt2, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
+        if (dH) GR_TRY(launch_gemm(R, K1, K2, dT, ldt2, a->W, K2, dH, lddh, nullptr, GRANII_GEMM_TRANS_B, gwH, gnH, st));
+        break;
+      }
+      default:
+        return fail(GRANII_ERR_INVALID_ARG, "composition does not belong to GCN");
+    }
+    if (c.dist()) GR_TRY(comm_allreduce_sum(c.comm, dW, (size_t)K1 * K2, st));
+  }
+  (void)dy_gathered;
+  if (ws_size) *ws_size = b.off + 1024;
+  return GRANII_OK;
+}
+
+granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_composition comp, int64_t K1,
+                              int64_t K2, size_t* ws, size_t* saved_floats) {
+  // size for the distributed layout whenever the graph is partitioned
+  granii_comm_s fake;
+  fake.world = g->world;
+  fake.rank = g->rank;
+  Ctx c{g, g->world > 1 ? &fake : nullptr, nullptr};
+  granii_layer_args a{};
+  a.K1 = K1;
+  a.K2 = K2;
+  a.ldh = K1;  // worst case: unaligned H needs a padded copy
+  a.act = GRANII_ACT_RELU;
+  size_t f = 0, f2 = 0, bwd = 0, sf = 0;
+  a.attn = GRANII_ATTN_ADDITIVE;
+  GR_TRY(forward_impl(c, m, comp, &a, nullptr, K2, nullptr, nullptr, &f, &sf));
+  if (m == GRANII_GAT) {
+    a.attn = GRANII_ATTN_DOT;
+    GR_TRY(forward_impl(c, m, comp, &a, nullptr, K2, nullptr, nullptr, &f2, &sf));
+    f = std::max(f, f2);
+  }
+  if (m == GRANII_GCN)
+    GR_TRY(backward_impl(c, comp, &a, nullptr, K2, nullptr, K2, nullptr, (float*)1, K1, nullptr, nullptr, &bwd));
+  *ws = std::max(f, bwd);
+  if (saved_floats) *saved_floats = sf;
+  return GRANII_OK;
+}
+
+granii_status layer_forward(const granii_graph_s* g, granii_model m, granii_composition comp,
+                            const granii_layer_args* a, float* out, int64_t ldo, float* saved, cudaStream_t st) {
+  Ctx c{g, a->comm, st};
+  size_t need = 0, sf = 0;
+  GR_TRY(forward_impl(c, m, comp, a, out, ldo, saved, nullptr, &need, &sf));
+  if (a->workspace_bytes < need) return fail(GRANII_ERR_INVALID_ARG, "layer workspace too small");
+  return forward_impl(c, m, comp, a, out, ldo, saved, a->workspace, &need, &sf);
+}
+
+granii_status layer_backward(const granii_graph_s* g, granii_composition comp, const granii_layer_args* a,
+                             const float* out, int64_t ldo, const float* dout, int64_t lddo, const float* saved,
+                             float* dH, int64_t lddh, float* dW, cudaStream_t st) {
+  Ctx c{g, a->comm, st};
+  size_t need = 0;
+  GR_TRY(backward_impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, nullptr, &need));
+  if (a->workspace_bytes < need) return fail(GRANII_ERR_INVALID_ARG, "layer workspace too small");
+  return backward_impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, a->workspace, &need);
+}
+
+}  // namespace granii

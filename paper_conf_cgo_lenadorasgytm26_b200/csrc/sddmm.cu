@@ -1,0 +1,255 @@
+// sddmm.cu -- g-SDDMM on Ã's pattern ("a standard matrix
+// multiplication guided by a sparse mask", L92 edge-based aggregation) and the
+// GAT attention of Eq. 4 (L127-L131; reading R8: single-head GAT [25]).
+//
+//   DOT : e = scale * <U_r, V_c>        K = 1 with U = V = dinv gives Ñ (Eq. 3)
+//   ADD : e = scale * (U_r + V_c)       K = 1 with U = el, V = er (additive attention)
+//   | LEAKYRELU : e = max(e, 0.2 e)
+//   | ROW_SOFTMAX : alpha_e = exp(e - m_r) / sum_r exp(e - m_r)
+//
+// B200 design: HBM-bound streaming over col_idx (4 B/entry)
+// plus an L2-resident gather of V (dinv/er: N floats) and a 4 B/entry write.
+// Group-per-row with LPG lanes striding the row keeps col_idx reads and e/alpha
+// writes coalesced; LPG follows the average degree.  For K > 1 a warp owns a
+// row: U_r lives in registers, LPG-lane groups each take an entry, gather V_c
+// with 16-byte loads and reduce with shuffles.  Softmax is fused: an online
+// (max, sum) pass over the row, a shuffle combine in fixed order, then a write
+// pass that recomputes e (V gathers hit L1/L2).  No atomics.
+#include <algorithm>
+#include <cmath>
+
+#include "internal.h"
+
+namespace granii {
+
+struct SddmmArgs {
+  int64_t n_rows;
+  const int64_t* __restrict__ row_ptr;
+  const int32_t* __restrict__ col_idx;
+  const float* __restrict__ U;
+  int64_t ldu;
+  const float* __restrict__ V;
+  int64_t ldv;
+  int64_t K;
+  float scale;
+  float* __restrict__ out;
+  const int32_t* __restrict__ order;
+};
+
+template <bool ADD, bool LRELU>
+__device__ __forceinline__ float score1(float u, float v, float scale) {
+  float e = ADD ? scale * (u + v) : scale * (u * v);
+  if (LRELU) e = e > 0.f ? e : 0.2f * e;
+  return e;
+}
+
+// K == 1: group of LPG lanes per row
+template <int LPG, bool ADD, bool LRELU, bool SOFTMAX>
+__global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
+    const int64_t t = t0 + grp;
+    const bool live = t < a.n_rows;
+    const int64_t row = live ? (a.order ? a.order[t] : t) : 0;
+    const int64_t rs = live ? a.row_ptr[row] : 0, re = live ? a.row_ptr[row + 1] : 0;
+    const float u = live ? __ldg(a.U + row * a.ldu) : 0.f;
+    if (!SOFTMAX) {
+      for (int64_t e = rs + lig; e < re; e += LPG)
+        a.out[e] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+      continue;
+    }
+    // online max / sum over this lane's entries
+    float m = -INFINITY, s = 0.f;
+    for (int64_t e = rs + lig; e < re; e += LPG) {
+      const float x = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+      if (x > m) {
+        s = s * expf(m - x) + 1.f;
+        m = x;
+      } else {
+        s += expf(x - m);
+      }
+    }
+    // combine within the group (xor butterfly, fixed order)
+#pragma unroll
+    for (int off = LPG / 2; off > 0; off >>= 1) {
+      const float m2 = __shfl_xor_sync(0xffffffffu, m, off), s2 = __shfl_xor_sync(0xffffffffu, s, off);
+      const float mn = fmaxf(m, m2);
+      const float a1 = (m == -INFINITY) ? 0.f : s * expf(m - mn);
+      const float a2 = (m2 == -INFINITY) ? 0.f : s2 * expf(m2 - mn);
+      m = mn;
+      s = a1 + a2;
+    }
+    const float inv = 1.f / s;
+    for (int64_t e = rs + lig; e < re; e += LPG) {
+      const float x = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+      a.out[e] = expf(x - m) * inv;
+    }
+  }
+}
+
+// K > 1 dot: warp per row, LPG lanes per entry, VEC-wide loads, NJ chunks per lane.
+template <int VEC, int LPG, int NJ>
+__global__ void __launch_bounds__(256) k_sddmm_dot(SddmmArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t < a.n_rows; t += nwarps) {
+    const int64_t row = a.order ? a.order[t] : t;
+    const int64_t rs = a.row_ptr[row], re = a.row_ptr[row + 1];
+    float u[NJ][VEC];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int v = 0; v < VEC; ++v) {
+        const int64_t k = (int64_t)(lig + j * LPG) * VEC + v;
+        u[j][v] = k < a.K ? __ldg(a.U + row * a.ldu + k) : 0.f;
+      }
+    for (int64_t e0 = rs; e0 < re; e0 += G) {
+      const int64_t e = e0 + grp;
+      const bool p = e < re;
+      const int32_t c = p ? __ldg(a.col_idx + e) : 0;
+      float acc = 0.f;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int64_t k = (int64_t)(lig + j * LPG) * VEC;
+        if (p && k < a.K) {
+          const float* vp = a.V + (int64_t)c * a.ldv + k;
+          if constexpr (VEC == 4) {
+            const float4 t4 = __ldg(reinterpret_cast<const float4*>(vp));
+            acc = fmaf(u[j][0], t4.x, acc);
+            acc = fmaf(u[j][1], t4.y, acc);
+            acc = fmaf(u[j][2], t4.z, acc);
+            acc = fmaf(u[j][3], t4.w, acc);
+          } else {
+            acc = fmaf(u[j][0], __ldg(vp), acc);
+          }
+        }
+      }
+#pragma unroll
+      for (int off = LPG / 2; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+      if (p && lig == 0) a.out[e] = a.scale * acc;
+    }
+  }
+}
+
+// row softmax in place over CSR values (used after the K > 1 dot SDDMM)
+template <int LPG>
+__global__ void __launch_bounds__(256) k_row_softmax(int64_t n_rows, const int64_t* __restrict__ row_ptr,
+                                                     float* __restrict__ x) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t0 = warp * G; t0 < n_rows; t0 += nwarps * G) {
+    const int64_t row = t0 + grp;
+    const bool live = row < n_rows;
+    const int64_t rs = live ? row_ptr[row] : 0, re = live ? row_ptr[row + 1] : 0;
+    float m = -INFINITY, s = 0.f;
+    for (int64_t e = rs + lig; e < re; e += LPG) {
+      const float v = x[e];
+      if (v > m) { s = s * expf(m - v) + 1.f; m = v; } else { s += expf(v - m); }
+    }
+#pragma unroll
+    for (int off = LPG / 2; off > 0; off >>= 1) {
+      const float m2 = __shfl_xor_sync(0xffffffffu, m, off), s2 = __shfl_xor_sync(0xffffffffu, s, off);
+      const float mn = fmaxf(m, m2);
+      const float a1 = (m == -INFINITY) ? 0.f : s * expf(m - mn);
+      const float a2 = (m2 == -INFINITY) ? 0.f : s2 * expf(m2 - mn);
+      m = mn;
+      s = a1 + a2;
+    }
+    const float inv = 1.f / s;
+    for (int64_t e = rs + lig; e < re; e += LPG) x[e] = expf(x[e] - m) * inv;
+  }
+}
+
+static int lpg_for_degree(float avg) {
+  if (avg >= 24.f) return 32;
+  if (avg >= 12.f) return 16;
+  if (avg >= 6.f) return 8;
+  return 4;
+}
+
+template <int LPG, bool ADD, bool LR, bool SM>
+static void go1(const SddmmArgs& a, int blocks, cudaStream_t st) {
+  k_sddmm1<LPG, ADD, LR, SM><<<blocks, 256, 0, st>>>(a);
+}
+
+template <bool ADD, bool LR, bool SM>
+static void go1_lpg(int lpg, const SddmmArgs& a, int blocks, cudaStream_t st) {
+  switch (lpg) {
+    case 32: go1<32, ADD, LR, SM>(a, blocks, st); break;
+    case 16: go1<16, ADD, LR, SM>(a, blocks, st); break;
+    case 8: go1<8, ADD, LR, SM>(a, blocks, st); break;
+    default: go1<4, ADD, LR, SM>(a, blocks, st); break;
+  }
+}
+
+granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U, int64_t ldu, const float* V,
+                           int64_t ldv, int64_t K, float scale, float* out, cudaStream_t st) {
+  if (g->n_rows == 0) return GRANII_OK;
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  const uint32_t base = op & 0xF;
+  const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
+  SddmmArgs a{g->n_rows, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order};
+  if (K == 1) {
+    const int lpg = lpg_for_degree(g->avg_deg());
+    const int64_t units = ceil_div(g->n_rows, 32 / lpg);
+    const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, 8), (int64_t)di.sms * 8));
+    const bool add = base == GRANII_SDDMM_ADD;
+    // dispatch the 8 (add, lrelu, softmax) variants
+    if (add) {
+      if (lr) { if (sm) go1_lpg<true, true, true>(lpg, a, blocks, st); else go1_lpg<true, true, false>(lpg, a, blocks, st); }
+      else { if (sm) go1_lpg<true, false, true>(lpg, a, blocks, st); else go1_lpg<true, false, false>(lpg, a, blocks, st); }
+    } else {
+      if (lr) { if (sm) go1_lpg<false, true, true>(lpg, a, blocks, st); else go1_lpg<false, true, false>(lpg, a, blocks, st); }
+      else { if (sm) go1_lpg<false, false, true>(lpg, a, blocks, st); else go1_lpg<false, false, false>(lpg, a, blocks, st); }
+    }
+    GR_CHECK_LAUNCH();
+    return GRANII_OK;
+  }
+  if (base != GRANII_SDDMM_DOT) return fail(GRANII_ERR_INVALID_ARG, "SDDMM ADD requires K == 1");
+  if (lr) return fail(GRANII_ERR_UNSUPPORTED, "LEAKYRELU with K > 1 is not supported");
+  const bool vec4 = (ldu % 4 == 0) && (ldv % 4 == 0) && ((uintptr_t)V % 16 == 0);
+  const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(g->n_rows, 8), (int64_t)di.sms * 8));
+#define GO(VEC, LPG, NJ) k_sddmm_dot<VEC, LPG, NJ><<<blocks, 256, 0, st>>>(a)
+  if (vec4) {
+    if (K <= 16) GO(4, 4, 1);
+    else if (K <= 32) GO(4, 8, 1);
+    else if (K <= 64) GO(4, 16, 1);
+    else if (K <= 128) GO(4, 32, 1);
+    else if (K <= 256) GO(4, 32, 2);
+    else if (K <= 512) GO(4, 32, 4);
+    else if (K <= 1024) GO(4, 32, 8);
+    else return fail(GRANII_ERR_UNSUPPORTED, "SDDMM DOT with K > 1024");
+  } else {
+    if (K <= 32) GO(1, 32, 1);
+    else if (K <= 64) GO(1, 32, 2);
+    else if (K <= 128) GO(1, 32, 4);
+    else if (K <= 256) GO(1, 32, 8);
+    else if (K <= 512) GO(1, 32, 16);
+    else return fail(GRANII_ERR_UNSUPPORTED, "unaligned SDDMM DOT with K > 512");
+  }
+#undef GO
+  GR_CHECK_LAUNCH();
+  if (sm) {
+    const int lpg = lpg_for_degree(g->avg_deg());
+    const int64_t units = ceil_div(g->n_rows, 32 / lpg);
+    const int b2 = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, 8), (int64_t)di.sms * 8));
+    switch (lpg) {
+      case 32: k_row_softmax<32><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
+      case 16: k_row_softmax<16><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
+      case 8: k_row_softmax<8><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
+      default: k_row_softmax<4><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
+    }
+    GR_CHECK_LAUNCH();
+  }
+  return GRANII_OK;
+}
+
+}  // namespace granii

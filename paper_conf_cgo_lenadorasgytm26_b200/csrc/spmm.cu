@@ -1,0 +1,296 @@
+// spmm.cu -- g-SpMM (+, x) on CSR (unweighted form L117):
+//   Y_i = rs_i * sum_{e in row i} w_e * cs_{c(e)} * X[c(e), k0:k0+kw]   (+ ReLU)
+//
+// B200 design: the op is a gather -- per stored entry it reads
+// one K-row of X (4K bytes) -- so it is bound by the L2->SM gather bandwidth
+// when X fits in L2 and by HBM when it does not.  Two schedules:
+//   * warp-per-row (dense-degree graphs): the warp loads 32 column ids (+w)
+//     coalesced, then G = 32/LPG lane groups each take one neighbour at a time
+//     and gather its row slice with 16-byte loads (VEC = 4), U neighbours per
+//     group in flight; groups are reduced with shuffles at the end.
+//   * group-per-row (sparse graphs, avg degree < 16): an LPG-lane group owns a
+//     row, 32/LPG rows per warp.
+// Rows are visited in the degree-descending schedule computed at graph
+// creation (round-robin over warps = LPT balance for power-law graphs).
+// Row/column scales fuse the two row-broadcasts of Eq. 2 (L115) into the
+// gather and the epilogue.  No atomics: each output row is written once by
+// one warp/group, reduction order fixed => bitwise reproducible.
+#include <algorithm>
+
+#include "internal.h"
+
+namespace granii {
+
+template <int VEC>
+struct VecT;
+template <>
+struct VecT<4> {
+  using T = float4;
+};
+template <>
+struct VecT<1> {
+  using T = float;
+};
+
+template <int VEC>
+__device__ __forceinline__ void ldv(const float* p, float (&v)[VEC]) {
+  if constexpr (VEC == 4) {
+    float4 t = __ldg(reinterpret_cast<const float4*>(p));
+    v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+  } else {
+    v[0] = __ldg(p);
+  }
+}
+template <int VEC>
+__device__ __forceinline__ void stv(float* p, const float (&v)[VEC]) {
+  if constexpr (VEC == 4) {
+    *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+  } else {
+    p[0] = v[0];
+  }
+}
+
+struct SpmmArgs {
+  int64_t n_rows;
+  const int64_t* __restrict__ row_ptr;
+  const int32_t* __restrict__ col_idx;
+  const float* __restrict__ vals;
+  const float* __restrict__ X;
+  int64_t ldx;
+  int64_t k0, kw;        // column slice [k0, k0+kw)
+  float* __restrict__ Y;
+  int64_t ldy;
+  const float* __restrict__ rs;
+  const float* __restrict__ cs;
+  int relu;
+  const int32_t* __restrict__ order;
+};
+
+// ------------------------------------------------------------------ warp-per-row
+template <int VEC, int LPG, int NJ, bool W, bool CS>
+__global__ void __launch_bounds__(256) k_spmm_warp(SpmmArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t < a.n_rows; t += nwarps) {
+    const int64_t row = a.order ? a.order[t] : t;
+    const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
+    float acc[NJ][VEC];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
+    bool colok[NJ];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) colok[j] = (int64_t)(lig + j * LPG) * VEC < a.kw;
+    const float* Xs = a.X + a.k0 + (int64_t)lig * VEC;
+    for (int64_t base = rs0; base < re; base += 32) {
+      const int64_t e = base + lane;
+      const bool valid = e < re;
+      int32_t c = valid ? __ldg(a.col_idx + e) : 0;
+      float w = valid ? (W ? __ldg(a.vals + e) : 1.f) : 0.f;
+      if (CS && valid) w *= __ldg(a.cs + c);
+      const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
+      // U = 2 neighbours per group per step (G*2 per warp) -> 2*NJ vector loads in flight
+      for (int i0 = 0; i0 < cnt; i0 += 2 * G) {
+        const int i1 = i0 + grp, i2 = i0 + G + grp;
+        const int32_t c1 = __shfl_sync(0xffffffffu, c, i1 & 31), c2 = __shfl_sync(0xffffffffu, c, i2 & 31);
+        const float w1 = __shfl_sync(0xffffffffu, w, i1 & 31), w2 = __shfl_sync(0xffffffffu, w, i2 & 31);
+        const bool p1 = i1 < cnt, p2 = i2 < cnt;
+        float x1[NJ][VEC], x2[NJ][VEC];
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          if (p1 && colok[j]) ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1[j]);
+          else
+#pragma unroll
+            for (int v = 0; v < VEC; ++v) x1[j][v] = 0.f;
+          if (p2 && colok[j]) ldv<VEC>(Xs + (int64_t)c2 * a.ldx + j * LPG * VEC, x2[j]);
+          else
+#pragma unroll
+            for (int v = 0; v < VEC; ++v) x2[j][v] = 0.f;
+        }
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w2, x2[j][v], fmaf(w1, x1[j][v], acc[j][v]));
+      }
+    }
+    // reduce the G groups (fixed butterfly order)
+#pragma unroll
+    for (int off = LPG; off < 32; off <<= 1)
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int v = 0; v < VEC; ++v) acc[j][v] += __shfl_xor_sync(0xffffffffu, acc[j][v], off);
+    if (grp == 0) {
+      const float s = a.rs ? __ldg(a.rs + row) : 1.f;
+      float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        if (!colok[j]) continue;
+        float o[VEC];
+#pragma unroll
+        for (int v = 0; v < VEC; ++v) {
+          o[v] = acc[j][v] * s;
+          if (a.relu) o[v] = fmaxf(o[v], 0.f);
+        }
+        stv<VEC>(y + j * LPG * VEC, o);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ group-per-row
+template <int VEC, int LPG, int NJ, bool W, bool CS>
+__global__ void __launch_bounds__(256) k_spmm_group(SpmmArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  bool colok[NJ];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) colok[j] = (int64_t)(lig + j * LPG) * VEC < a.kw;
+  const float* Xs = a.X + a.k0 + (int64_t)lig * VEC;
+  for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
+    const int64_t t = t0 + grp;
+    if (t >= a.n_rows) continue;
+    const int64_t row = a.order ? a.order[t] : t;
+    const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
+    float acc[NJ][VEC];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
+    int64_t e = rs0;
+    for (; e + 1 < re; e += 2) {
+      const int32_t c1 = __ldg(a.col_idx + e), c2 = __ldg(a.col_idx + e + 1);
+      float w1 = W ? __ldg(a.vals + e) : 1.f, w2 = W ? __ldg(a.vals + e + 1) : 1.f;
+      if (CS) { w1 *= __ldg(a.cs + c1); w2 *= __ldg(a.cs + c2); }
+      float x1[NJ][VEC], x2[NJ][VEC];
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        if (colok[j]) {
+          ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1[j]);
+          ldv<VEC>(Xs + (int64_t)c2 * a.ldx + j * LPG * VEC, x2[j]);
+        } else {
+#pragma unroll
+          for (int v = 0; v < VEC; ++v) x1[j][v] = x2[j][v] = 0.f;
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w2, x2[j][v], fmaf(w1, x1[j][v], acc[j][v]));
+    }
+    if (e < re) {
+      const int32_t c1 = __ldg(a.col_idx + e);
+      float w1 = W ? __ldg(a.vals + e) : 1.f;
+      if (CS) w1 *= __ldg(a.cs + c1);
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        if (!colok[j]) continue;
+        float x1[VEC];
+        ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1);
+#pragma unroll
+        for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w1, x1[v], acc[j][v]);
+      }
+    }
+    const float s = a.rs ? __ldg(a.rs + row) : 1.f;
+    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      if (!colok[j]) continue;
+      float o[VEC];
+#pragma unroll
+      for (int v = 0; v < VEC; ++v) {
+        o[v] = acc[j][v] * s;
+        if (a.relu) o[v] = fmaxf(o[v], 0.f);
+      }
+      stv<VEC>(y + j * LPG * VEC, o);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ dispatch
+template <int VEC, int LPG, int NJ>
+static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool cs, int sms, cudaStream_t st) {
+  const int threads = 256;
+  int64_t units = warp_mode ? a.n_rows : ceil_div(a.n_rows, 32 / LPG);
+  // enough warps for 8 resident blocks/SM, capped by the work available
+  int64_t blocks = std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 8);
+  blocks = std::max<int64_t>(blocks, 1);
+#define GR_L(K) K<<<(unsigned)blocks, threads, 0, st>>>(a)
+  if (warp_mode) {
+    if (w && cs) GR_L((k_spmm_warp<VEC, LPG, NJ, true, true>));
+    else if (w) GR_L((k_spmm_warp<VEC, LPG, NJ, true, false>));
+    else if (cs) GR_L((k_spmm_warp<VEC, LPG, NJ, false, true>));
+    else GR_L((k_spmm_warp<VEC, LPG, NJ, false, false>));
+  } else {
+    if (w && cs) GR_L((k_spmm_group<VEC, LPG, NJ, true, true>));
+    else if (w) GR_L((k_spmm_group<VEC, LPG, NJ, true, false>));
+    else if (cs) GR_L((k_spmm_group<VEC, LPG, NJ, false, true>));
+    else GR_L((k_spmm_group<VEC, LPG, NJ, false, false>));
+  }
+#undef GR_L
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+// Pick (VEC, LPG, NJ) for a slice of width kw.  VEC=4 needs 16-byte aligned rows.
+static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, bool w, bool cs, int sms,
+                                  cudaStream_t st) {
+  const int64_t kw = a.kw;
+  if (vec4) {
+    if (kw <= 16) return launch_cfg<4, 4, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 32) return launch_cfg<4, 8, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 64) return launch_cfg<4, 16, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 128) return launch_cfg<4, 32, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 256) return launch_cfg<4, 32, 2>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 512) return launch_cfg<4, 32, 4>(a, warp_mode, w, cs, sms, st);
+    return launch_cfg<4, 32, 8>(a, warp_mode, w, cs, sms, st);
+  }
+  if (kw <= 32) return launch_cfg<1, 32, 1>(a, warp_mode, w, cs, sms, st);
+  if (kw <= 64) return launch_cfg<1, 32, 2>(a, warp_mode, w, cs, sms, st);
+  if (kw <= 128) return launch_cfg<1, 32, 4>(a, warp_mode, w, cs, sms, st);
+  return launch_cfg<1, 32, 8>(a, warp_mode, w, cs, sms, st);
+}
+
+int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t l2_bytes) {
+  // Keep the gathered column slice of X resident in L2: split
+  // K into slices whose X footprint is <= ~45% of L2 when the graph is dense
+  // enough for re-use (avg degree >= 32) and X itself does not fit.
+  const int64_t maxw = vec4 ? 1024 : 256;
+  int64_t kw = std::min<int64_t>(K, maxw);
+  if (const char* env = getenv("GRANII_SPMM_SLICE")) {
+    int64_t v = atoll(env);
+    if (v > 0) return std::min<int64_t>(std::max<int64_t>(v, 1), maxw);
+  }
+  const double xbytes = (double)g->n_cols * (double)K * 4.0;
+  if (g->avg_deg() >= 32.f && xbytes > 0.45 * (double)l2_bytes) {
+    int64_t nsl = (int64_t)std::ceil(xbytes / (0.45 * (double)l2_bytes));
+    int64_t w = round_up(ceil_div(K, nsl), vec4 ? 64 : 32);
+    kw = std::min(kw, std::max<int64_t>(w, vec4 ? 64 : 32));
+  }
+  return kw;
+}
+
+granii_status launch_spmm(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                          float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, cudaStream_t st) {
+  if (g->n_rows == 0 || K == 0) return GRANII_OK;
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  const bool vec4 = (ldx % 4 == 0) && (ldy % 4 == 0) && ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0);
+  const bool warp_mode = g->avg_deg() >= 16.f;
+  SpmmArgs a{g->n_rows, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0, g->order};
+  const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
+  for (int64_t k0 = 0; k0 < K; k0 += kw) {
+    a.k0 = k0;
+    a.kw = std::min(kw, K - k0);
+    // slices of a vec4 launch must stay 16-byte aligned
+    GR_TRY(launch_slice(a, vec4 && (k0 % 4 == 0), warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
+  }
+  return GRANII_OK;
+}
+
+}  // namespace granii

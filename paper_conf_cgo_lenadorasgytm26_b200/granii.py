@@ -1,0 +1,295 @@
+"""Thin Python binding of include/granii.h (ctypes; argument marshalling only).
+
+Every function has the ABI's name and forwards torch tensors as raw device
+pointers plus the current CUDA stream.  All computation happens in
+libgranii.so; there is no CPU fallback: if the library is missing this module
+raises at import, and every compute call without a CUDA device returns
+GRANII_ERR_CUDA, raised here as GraniiError.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgranii.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: run `python -c 'import __graft_entry__ as g; g.build()'` "
+                      "(the CUDA library is required; there is no fallback)")
+_lib = ctypes.CDLL(LIB_PATH)
+
+# ---------------------------------------------------------------- constants (granii.h)
+OK, ERR_INVALID_ARG, ERR_OOM, ERR_CUDA, ERR_NCCL, ERR_UNSUPPORTED, ERR_NOT_CALIBRATED = range(7)
+ADD_SELF_LOOPS, SYMMETRIZE = 0x1, 0x2
+EPI_RELU = 0x1
+SDDMM_DOT, SDDMM_ADD, SDDMM_LEAKYRELU, SDDMM_ROW_SOFTMAX = 0x0, 0x1, 0x10, 0x20
+GEMM_TRANS_A, GEMM_TRANS_B, GEMM_RELU, GEMM_NO_STORE = 0x1, 0x2, 0x4, 0x8
+GCN, GAT = 0, 1
+GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD = 0, 1, 2, 3
+GAT_REUSE, GAT_RECOMP = 16, 17
+GCN_COMPS = (GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD)
+GAT_COMPS = (GAT_REUSE, GAT_RECOMP)
+COMP_NAMES = {0: "GCN_PRE_AGG", 1: "GCN_PRE_UPD", 2: "GCN_DYN_AGG", 3: "GCN_DYN_UPD", 16: "GAT_REUSE",
+              17: "GAT_RECOMP"}
+ACT_NONE, ACT_RELU = 0, 1
+ATTN_ADDITIVE, ATTN_DOT = 0, 1
+SELECT_NO_PREFILTER = 0x1
+MAX_CANDIDATES = 8
+NUM_FEATURES = 8
+
+_i64, _i32, _u32, _p, _f, _sz = (ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32, ctypes.c_void_p,
+                                 ctypes.c_float, ctypes.c_size_t)
+
+
+class graph_info(ctypes.Structure):
+    _fields_ = [("num_nodes", _i64), ("nnz", _i64), ("row_begin", _i64), ("row_end", _i64),
+                ("local_nnz", _i64), ("max_local_rows", _i64), ("part_rank", _i32), ("part_world", _i32),
+                ("symmetric", _i32), ("reserved", _i32), ("features", _i64 * NUM_FEATURES)]
+
+
+class gemm_epilogue(ctypes.Structure):
+    _fields_ = [("row_scale", _p), ("att_l", _p), ("att_r", _p), ("out_l", _p), ("out_r", _p)]
+
+
+class layer_args(ctypes.Structure):
+    _fields_ = [("K1", _i64), ("K2", _i64), ("H", _p), ("ldh", _i64), ("W", _p), ("a_l", _p), ("a_r", _p),
+                ("act", _u32), ("attn", _u32), ("workspace", _p), ("workspace_bytes", _sz), ("comm", _p)]
+
+
+_SIGS = {
+    "granii_last_error": ([], ctypes.c_char_p),
+    "granii_version": ([], ctypes.c_char_p),
+    "granii_graph_csr_create": ([_i64, _i64, _p, _p, _u32, _i32, _i32, _p, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_graph_destroy": ([_p], ctypes.c_int),
+    "granii_graph_query": ([_p, ctypes.POINTER(graph_info)], ctypes.c_int),
+    "granii_graph_export_csr": ([_p, _p, _p], ctypes.c_int),
+    "granii_graph_dinv": ([_p, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_partition_bounds": ([_i64, _p, _i32, _p], ctypes.c_int),
+    "granii_spmm": ([_p, _p, _p, _i64, _i64, _p, _i64, _p, _p, _u32, _p], ctypes.c_int),
+    "granii_sddmm": ([_p, _u32, _p, _i64, _p, _i64, _i64, _f, _p, _p], ctypes.c_int),
+    "granii_gemm_workspace_size": ([_i64, _i64, _i64, _u32, ctypes.POINTER(_sz)], ctypes.c_int),
+    "granii_gemm": ([_i64, _i64, _i64, _p, _i64, _p, _i64, _p, _i64, ctypes.POINTER(gemm_epilogue), _u32, _p, _sz,
+                     _p], ctypes.c_int),
+    "granii_layer_workspace_size": ([_p, ctypes.c_int, ctypes.c_int, _i64, _i64, ctypes.POINTER(_sz),
+                                     ctypes.POINTER(_sz)], ctypes.c_int),
+    "granii_layer_forward": ([_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(layer_args), _p, _i64, _p, _p],
+                             ctypes.c_int),
+    "granii_layer_backward": ([_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(layer_args), _p, _i64, _p, _i64, _p,
+                               _p, _i64, _p, _p], ctypes.c_int),
+    "granii_select": ([_p, ctypes.c_int, _i64, _i64, ctypes.c_char_p, _u32, ctypes.POINTER(ctypes.c_int),
+                       ctypes.POINTER(_i32), ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i32)], ctypes.c_int),
+    "granii_comm_unique_id": ([_p], ctypes.c_int),
+    "granii_comm_create": ([_p, _i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_comm_destroy": ([_p], ctypes.c_int),
+    "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
+    "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
+}
+for _name, (_args, _res) in _SIGS.items():
+    _fn = getattr(_lib, _name)
+    _fn.argtypes = _args
+    _fn.restype = _res
+
+EXPORTED = tuple(_SIGS)
+
+
+class GraniiError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: status {status}: {_lib.granii_last_error().decode()}")
+
+
+def _check(st: int, where: str):
+    if st != OK:
+        raise GraniiError(st, where)
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if isinstance(t, int):
+        return t
+    return t.data_ptr()
+
+
+def _stream(stream=None):
+    if stream is not None:
+        return stream.cuda_stream if hasattr(stream, "cuda_stream") else stream
+    return torch.cuda.current_stream().cuda_stream if torch.cuda.is_available() else None
+
+
+def _ld(t):
+    assert t.dim() == 2 and t.stride(1) == 1, "row-major 2-D tensor with unit column stride required"
+    return t.stride(0)
+
+
+def granii_version() -> str:
+    return _lib.granii_version().decode()
+
+
+def granii_last_error() -> str:
+    return _lib.granii_last_error().decode()
+
+
+# ---------------------------------------------------------------- graph
+class Graph:
+    """Owns a granii_graph handle (destroyed with the object)."""
+
+    def __init__(self, handle: int):
+        self.handle = handle
+        self.info = granii_graph_query(handle)
+
+    def __del__(self):
+        if getattr(self, "handle", None):
+            _lib.granii_graph_destroy(self.handle)
+            self.handle = None
+
+    @property
+    def n_rows(self):
+        return self.info.row_end - self.info.row_begin
+
+    @property
+    def nnz(self):
+        return self.info.local_nnz
+
+    def features(self):
+        return list(self.info.features)
+
+
+def granii_graph_csr_create(num_nodes: int, src: torch.Tensor, dst: torch.Tensor, flags: int = ADD_SELF_LOOPS,
+                            part_rank: int = 0, part_world: int = 1, stream=None) -> Graph:
+    assert src.dtype == torch.int32 and dst.dtype == torch.int32 and src.is_contiguous() and dst.is_contiguous()
+    h = _p()
+    _check(_lib.granii_graph_csr_create(num_nodes, src.numel(), _ptr(src), _ptr(dst), flags, part_rank, part_world,
+                                        _stream(stream), ctypes.byref(h)), "granii_graph_csr_create")
+    return Graph(h.value)
+
+
+def granii_graph_query(handle) -> graph_info:
+    info = graph_info()
+    _check(_lib.granii_graph_query(handle, ctypes.byref(info)), "granii_graph_query")
+    return info
+
+
+def granii_graph_export_csr(g: Graph):
+    import numpy as np
+    rp = np.zeros(g.n_rows + 1, np.int64)
+    ci = np.zeros(max(g.nnz, 1), np.int32)
+    _check(_lib.granii_graph_export_csr(g.handle, rp.ctypes.data, ci.ctypes.data), "granii_graph_export_csr")
+    return rp, ci[: g.nnz]
+
+
+def granii_graph_dinv(g: Graph) -> int:
+    p = _p()
+    _check(_lib.granii_graph_dinv(g.handle, ctypes.byref(p)), "granii_graph_dinv")
+    return p.value
+
+
+def granii_partition_bounds(row_ptr, world: int):
+    import numpy as np
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    b = np.zeros(world + 1, np.int64)
+    _check(_lib.granii_partition_bounds(rp.shape[0] - 1, rp.ctypes.data, world, b.ctypes.data),
+           "granii_partition_bounds")
+    return b
+
+
+# ---------------------------------------------------------------- primitives
+def granii_spmm(g: Graph, vals, X: torch.Tensor, K: int, Y: torch.Tensor, row_scale=None, col_scale=None,
+                epilogue: int = 0, stream=None):
+    _check(_lib.granii_spmm(g.handle, _ptr(vals), _ptr(X), _ld(X), K, _ptr(Y), _ld(Y), _ptr(row_scale),
+                            _ptr(col_scale), epilogue, _stream(stream)), "granii_spmm")
+
+
+def granii_sddmm(g: Graph, op: int, U, ldu: int, V, ldv: int, K: int, scale: float, out, stream=None):
+    _check(_lib.granii_sddmm(g.handle, op, _ptr(U), ldu, _ptr(V), ldv, K, scale, _ptr(out), _stream(stream)),
+           "granii_sddmm")
+
+
+def granii_gemm_workspace_size(M: int, N: int, K: int, flags: int = 0) -> int:
+    n = _sz()
+    _check(_lib.granii_gemm_workspace_size(M, N, K, flags, ctypes.byref(n)), "granii_gemm_workspace_size")
+    return n.value
+
+
+def granii_gemm(M: int, N: int, K: int, A, lda: int, B, ldb: int, C, ldc: int, flags: int = 0, row_scale=None,
+                att_l=None, att_r=None, out_l=None, out_r=None, workspace=None, stream=None):
+    need = granii_gemm_workspace_size(M, N, K, flags)
+    if workspace is None:
+        workspace = torch.empty(max(need, 1), dtype=torch.uint8, device=A.device)
+    ep = gemm_epilogue(_ptr(row_scale), _ptr(att_l), _ptr(att_r), _ptr(out_l), _ptr(out_r))
+    _check(_lib.granii_gemm(M, N, K, _ptr(A), lda, _ptr(B), ldb, _ptr(C), ldc, ctypes.byref(ep), flags,
+                            _ptr(workspace), workspace.numel(), _stream(stream)), "granii_gemm")
+
+
+# ---------------------------------------------------------------- layers
+def granii_layer_workspace_size(g: Graph, model: int, comp: int, K1: int, K2: int):
+    ws, sv = _sz(), _sz()
+    _check(_lib.granii_layer_workspace_size(g.handle, model, comp, K1, K2, ctypes.byref(ws), ctypes.byref(sv)),
+           "granii_layer_workspace_size")
+    return ws.value, sv.value
+
+
+def make_layer_args(K1, K2, H, W, a_l=None, a_r=None, act=ACT_RELU, attn=ATTN_ADDITIVE, workspace=None,
+                    comm=None) -> layer_args:
+    return layer_args(K1, K2, _ptr(H), _ld(H), _ptr(W), _ptr(a_l), _ptr(a_r), act, attn, _ptr(workspace),
+                      workspace.numel() if workspace is not None else 0, comm.handle if comm is not None else None)
+
+
+def granii_layer_forward(g: Graph, model: int, comp: int, args: layer_args, out: torch.Tensor, saved=None,
+                         stream=None):
+    _check(_lib.granii_layer_forward(g.handle, model, comp, ctypes.byref(args), _ptr(out), _ld(out), _ptr(saved),
+                                     _stream(stream)), "granii_layer_forward")
+
+
+def granii_layer_backward(g: Graph, model: int, comp: int, args: layer_args, out: torch.Tensor, dout: torch.Tensor,
+                          saved, dH, dW: torch.Tensor, stream=None):
+    _check(_lib.granii_layer_backward(g.handle, model, comp, ctypes.byref(args), _ptr(out), _ld(out), _ptr(dout),
+                                      _ld(dout), _ptr(saved), _ptr(dH), _ld(dH) if dH is not None else 0, _ptr(dW),
+                                      _stream(stream)), "granii_layer_backward")
+
+
+def granii_select(g: Graph, model: int, K1: int, K2: int, calib_path: str | None = None, flags: int = 0):
+    out = ctypes.c_int()
+    cands = (_i32 * MAX_CANDIDATES)()
+    pred = (ctypes.c_double * MAX_CANDIDATES)()
+    n = _i32()
+    _check(_lib.granii_select(g.handle, model, K1, K2, calib_path.encode() if calib_path else None, flags,
+                              ctypes.byref(out), cands, pred, ctypes.byref(n)), "granii_select")
+    return out.value, {cands[i]: pred[i] for i in range(n.value)}
+
+
+# ---------------------------------------------------------------- multi-GPU
+class Comm:
+    def __init__(self, handle: int, rank: int, world: int):
+        self.handle, self.rank, self.world = handle, rank, world
+
+    def __del__(self):
+        if getattr(self, "handle", None):
+            _lib.granii_comm_destroy(self.handle)
+            self.handle = None
+
+
+def granii_comm_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.granii_comm_unique_id(buf), "granii_comm_unique_id")
+    return buf.raw
+
+
+def granii_comm_create(uid: bytes, rank: int, world: int) -> Comm:
+    buf = ctypes.create_string_buffer(uid, 128)
+    h = _p()
+    _check(_lib.granii_comm_create(buf, rank, world, ctypes.byref(h)), "granii_comm_create")
+    return Comm(h.value, rank, world)
+
+
+# ---------------------------------------------------------------- training helpers
+def granii_softmax_xent(Z: torch.Tensor, y: torch.Tensor, n_total: int, dZ: torch.Tensor, loss=None, stream=None):
+    _check(_lib.granii_softmax_xent(Z.shape[0], Z.shape[1], _ptr(Z), _ld(Z), _ptr(y), n_total, _ptr(dZ), _ld(dZ),
+                                    _ptr(loss), _stream(stream)), "granii_softmax_xent")
+
+
+def granii_sgd(grad: torch.Tensor, param: torch.Tensor, lr: float, stream=None):
+    _check(_lib.granii_sgd(param.numel(), lr, _ptr(grad), _ptr(param), _stream(stream)), "granii_sgd")

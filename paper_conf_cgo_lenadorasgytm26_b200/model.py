@@ -1,0 +1,100 @@
+"""Multi-layer GNN driver over the C ABI (§VI-F, Fig. 4).
+
+GRANII selects one composition per layer from the input graph and the layer's
+embedding sizes, once per (graph, K1, K2), and reuses the decision across
+iterations (L409).  This module only sequences ABI calls and owns the device
+buffers (workspaces, activations, gradients) as torch tensors; every FLOP runs
+in libgranii.so.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import torch
+
+from . import granii as G
+
+
+def _pad4(k: int) -> int:
+    return (k + 3) // 4 * 4
+
+
+def alloc2d(rows: int, cols: int, device, fill=None) -> torch.Tensor:
+    """(rows, cols) fp32 view of a buffer whose row stride is padded to 16 bytes."""
+    buf = torch.empty((max(rows, 1), _pad4(cols)), dtype=torch.float32, device=device)
+    if fill is not None:
+        buf.fill_(fill)
+    return buf[:rows, :cols]
+
+
+@dataclass
+class LayerSpec:
+    model: int                  # G.GCN | G.GAT
+    K1: int
+    K2: int
+    act: int = G.ACT_RELU
+    attn: int = G.ATTN_ADDITIVE
+    comp: int | None = None     # None -> chosen by granii_select
+    W: torch.Tensor | None = None
+    a_l: torch.Tensor | None = None
+    a_r: torch.Tensor | None = None
+    predicted_ms: dict = field(default_factory=dict)
+
+
+class GNN:
+    """A stack of GCN/GAT layers on one (possibly row-partitioned) graph."""
+
+    def __init__(self, graph: G.Graph, layers: list[LayerSpec], device, comm: G.Comm | None = None,
+                 calib_path: str | None = None, select_flags: int = 0):
+        self.g, self.layers, self.device, self.comm = graph, layers, device, comm
+        for L in layers:
+            if L.comp is None:
+                L.comp, L.predicted_ms = G.granii_select(graph, L.model, L.K1, L.K2, calib_path, select_flags)
+        ws = 0
+        self.saved_floats = []
+        for L in layers:
+            w, s = G.granii_layer_workspace_size(graph, L.model, L.comp, L.K1, L.K2)
+            ws = max(ws, w)
+            self.saved_floats.append(s)
+        self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=device)
+        R = graph.n_rows
+        self.outs = [alloc2d(R, L.K2, device) for L in layers]
+        self.saved = [torch.empty(max(s, 1), dtype=torch.float32, device=device) if s else None
+                      for s in self.saved_floats]
+        self.grads_out = [alloc2d(R, L.K2, device) for L in layers]     # dL/d out_l
+        self.dW = [torch.empty((L.K1, L.K2), dtype=torch.float32, device=device) for L in layers]
+
+    def args(self, i: int, H: torch.Tensor) -> G.layer_args:
+        L = self.layers[i]
+        return G.make_layer_args(L.K1, L.K2, H, L.W, L.a_l, L.a_r, L.act, L.attn, self.workspace, self.comm)
+
+    def forward(self, H: torch.Tensor) -> torch.Tensor:
+        x = H
+        self._inputs = []
+        for i, L in enumerate(self.layers):
+            self._inputs.append(x)
+            G.granii_layer_forward(self.g, L.model, L.comp, self.args(i, x), self.outs[i], self.saved[i])
+            x = self.outs[i]
+        return x
+
+    def backward(self, dout_last: torch.Tensor, need_input_grad: bool = False):
+        """Backward through all layers (GCN only, L340); fills self.dW."""
+        dout = dout_last
+        for i in range(len(self.layers) - 1, -1, -1):
+            L = self.layers[i]
+            dH = self.grads_out[i - 1] if i > 0 else (alloc2d(self.g.n_rows, L.K1, self.device)
+                                                      if need_input_grad else None)
+            G.granii_layer_backward(self.g, L.model, L.comp, self.args(i, self._inputs[i]), self.outs[i], dout,
+                                    self.saved[i], dH, self.dW[i])
+            dout = dH
+        return dout
+
+    def train_step(self, H: torch.Tensor, labels: torch.Tensor, n_total: int, lr: float,
+                   dlogits: torch.Tensor, loss: torch.Tensor | None = None):
+        """forward -> softmax cross-entropy -> backward -> SGD update of every W."""
+        Z = self.forward(H)
+        G.granii_softmax_xent(Z, labels, n_total, dlogits, loss)
+        self.backward(dlogits)
+        for L, dW in zip(self.layers, self.dW):
+            G.granii_sgd(dW, L.W, lr)
+        return Z

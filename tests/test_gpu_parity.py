@@ -1,0 +1,356 @@
+"""Parity of the CUDA path (through the C ABI) with the fp64 oracle (-m gpu).
+
+Tolerance (BASELINE.json north_star): fp32 path
+    max_i |y_i - r_i| / max(|r_i|, 1e-3 * ||r||_inf) <= 1e-4
+CSR construction, partition and integer features: bit-exact.
+All inputs come from the seeded generators; expected values come only from oracle/.
+"""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_cgo_lenadorasgytm26_b200 import synth
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+DEV = torch.device("cuda:0") if torch.cuda.is_available() else None
+
+
+@pytest.fixture(scope="module")
+def G():
+    from paper_conf_cgo_lenadorasgytm26_b200 import granii
+    return granii
+
+
+def err(y, r):
+    y = np.asarray(y, np.float64)
+    r = np.asarray(r, np.float64)
+    if r.size == 0:
+        return 0.0
+    floor = 1e-3 * max(np.abs(r).max(), 1e-300)
+    return float(np.max(np.abs(y - r) / np.maximum(np.abs(r), floor)))
+
+
+def pad(t, k=None):
+    """copy a (rows, k) tensor to cuda with a 16-byte-aligned row stride"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import alloc2d
+    t = torch.as_tensor(t, dtype=torch.float32)
+    out = alloc2d(t.shape[0], t.shape[1], DEV)
+    out.copy_(t)
+    return out
+
+
+class Case:
+    def __init__(self, G, name, n, s, d, flags):
+        self.name, self.n, self.flags = name, n, flags
+        self.s, self.d = s, d
+        self.g = G.granii_graph_csr_create(n, s.to(DEV).contiguous(), d.to(DEV).contiguous(), flags)
+        self.rp, self.ci = O.csr_build(n, s, d, flags)
+
+
+_cache = {}
+
+
+def case(G, name):
+    if name in _cache:
+        return _cache[name]
+    F = O.ADD_SELF_LOOPS | O.SYMMETRIZE
+    if name == "tiny":
+        n = 37
+        s, d = synth.random_small(n, 100, 1)
+        c = Case(G, name, n, s, d, F)
+    elif name == "sparse":           # avg degree ~ 5 -> group-per-row schedules
+        n = 3000
+        s, d = synth.chung_lu(n, 6000, 2.5, seed=2)
+        c = Case(G, name, n, s, d, F)
+    elif name == "dense":            # avg degree ~ 80 with hubs -> warp-per-row schedules
+        n = 2500
+        s, d = synth.chung_lu(n, 100000, 2.1, seed=3, max_w_frac=0.05)
+        c = Case(G, name, n, s, d, F)
+    elif name == "directed":         # R-MAT, not symmetrised (GAT / arxiv-like)
+        n = 4000
+        s, d = synth.rmat(n, 30000, 0.57, 0.19, 0.19, seed=4)
+        c = Case(G, name, n, s, d, O.ADD_SELF_LOOPS)
+    elif name == "cora":
+        w = synth.WORKLOADS["cora"]
+        s, d = w.edges(0)
+        c = Case(G, name, w.n, s, d, F)
+    elif name == "pubmed":
+        w = synth.WORKLOADS["pubmed"]
+        s, d = w.edges(0)
+        c = Case(G, name, w.n, s, d, F)
+    else:
+        raise KeyError(name)
+    _cache[name] = c
+    return c
+
+
+# ------------------------------------------------------------------ a0 / a1 CSR + features
+@pytest.mark.parametrize("name", ["tiny", "sparse", "dense", "directed", "cora", "pubmed"])
+def test_csr_bit_exact(G, name):
+    c = case(G, name)
+    rp, ci = G.granii_graph_export_csr(c.g)
+    assert np.array_equal(rp, c.rp) and np.array_equal(ci, c.ci)
+    assert c.g.features() == [int(x) for x in O.features(c.rp)]
+
+
+@pytest.mark.parametrize("flags", [0, 1, 2, 3])
+def test_csr_flags_and_edge_cases(G, flags):
+    n = 50
+    s, d = synth.random_small(n, 200, 9)
+    g = G.granii_graph_csr_create(n, s.to(DEV), d.to(DEV), flags)
+    rp, ci = O.csr_build(n, s, d, flags)
+    grp, gci = G.granii_graph_export_csr(g)
+    assert np.array_equal(grp, rp) and np.array_equal(gci, ci)
+    e = torch.zeros(0, dtype=torch.int32, device=DEV)
+    g0 = G.granii_graph_csr_create(7, e, e, flags)
+    rp0, ci0 = O.csr_build(7, np.zeros(0, np.int32), np.zeros(0, np.int32), flags)
+    grp0, gci0 = G.granii_graph_export_csr(g0)
+    assert np.array_equal(grp0, rp0) and np.array_equal(gci0, ci0)
+    bad = torch.tensor([0, 50], dtype=torch.int32, device=DEV)
+    with pytest.raises(G.GraniiError) as ex:
+        G.granii_graph_csr_create(n, bad, bad, flags)
+    assert ex.value.status == G.ERR_INVALID_ARG
+
+
+# ------------------------------------------------------------------ SpMM
+KS = [1, 2, 3, 4, 16, 41, 47, 64, 100, 128, 129, 256, 602, 1024]
+
+
+@pytest.mark.parametrize("name", ["sparse", "dense"])
+@pytest.mark.parametrize("K", KS)
+def test_spmm_variants(G, name, K):
+    c = case(G, name)
+    n = c.n
+    X = synth.uniform_pm1(10, K, (n, K))
+    vals = synth.uniform_pm1(11, K, (c.ci.shape[0],))
+    rs = synth.uniform_pm1(12, 1, (n,))
+    cs = synth.uniform_pm1(12, 2, (n,))
+    Xd = pad(X)
+    Y = pad(torch.zeros(n, K))
+    # weighted + row/col scale + relu: Y_i = relu(rs_i sum_e w_e cs_c X_c)
+    G.granii_spmm(c.g, vals.to(DEV), Xd, K, Y, rs.to(DEV), cs.to(DEV), G.EPI_RELU)
+    rows = np.repeat(np.arange(n), np.diff(c.rp))
+    w = vals.numpy().astype(np.float64) * cs.numpy().astype(np.float64)[c.ci]
+    ref = np.maximum(rs.numpy()[:, None] * O.spmm(c.rp, c.ci, w, X), 0)
+    torch.cuda.synchronize()
+    assert err(Y.cpu(), ref) <= TOL
+    # unweighted, no scales, unaligned leading dimension (scalar path)
+    Xu = X.to(DEV).contiguous()
+    Yu = torch.zeros(n, K, device=DEV)
+    G.granii_spmm(c.g, None, Xu, K, Yu)
+    torch.cuda.synchronize()
+    assert err(Yu.cpu(), O.spmm(c.rp, c.ci, None, X)) <= TOL
+    del rows
+
+
+def test_spmm_forced_slices_match(G):
+    c = case(G, "dense")
+    K = 256
+    X = pad(synth.uniform_pm1(20, 1, (c.n, K)))
+    Y1, Y2 = pad(torch.zeros(c.n, K)), pad(torch.zeros(c.n, K))
+    G.granii_spmm(c.g, None, X, K, Y1)
+    os.environ["GRANII_SPMM_SLICE"] = "64"
+    try:
+        G.granii_spmm(c.g, None, X, K, Y2)
+    finally:
+        del os.environ["GRANII_SPMM_SLICE"]
+    torch.cuda.synchronize()
+    assert torch.equal(Y1, Y2), "column slicing must not change any bit"
+    assert err(Y1.cpu(), O.spmm(c.rp, c.ci, None, X.cpu())) <= TOL
+
+
+def test_spmm_deterministic(G):
+    c = case(G, "dense")
+    X = pad(synth.uniform_pm1(21, 1, (c.n, 64)))
+    Y1, Y2 = pad(torch.zeros(c.n, 64)), pad(torch.zeros(c.n, 64))
+    G.granii_spmm(c.g, None, X, 64, Y1)
+    G.granii_spmm(c.g, None, X, 64, Y2)
+    torch.cuda.synchronize()
+    assert torch.equal(Y1, Y2)
+
+
+# ------------------------------------------------------------------ SDDMM
+@pytest.mark.parametrize("name", ["sparse", "dense", "directed"])
+def test_sddmm_norm_and_attention(G, name):
+    c = case(G, name)
+    n, nnz = c.n, c.ci.shape[0]
+    dinv = O.dinv(c.rp)
+    dv = torch.tensor(dinv, dtype=torch.float32, device=DEV)
+    out = torch.zeros(nnz, device=DEV)
+    G.granii_sddmm(c.g, G.SDDMM_DOT, dv, 1, dv, 1, 1, 1.0, out)
+    torch.cuda.synchronize()
+    assert err(out.cpu(), O.sddmm(c.rp, c.ci, dinv, dinv)) <= TOL
+    el = synth.uniform_pm1(30, 1, (n,)) * 3
+    er = synth.uniform_pm1(30, 2, (n,)) * 3
+    G.granii_sddmm(c.g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el.to(DEV), 1, er.to(DEV), 1, 1, 1.0,
+                   out)
+    torch.cuda.synchronize()
+    rows = np.repeat(np.arange(n), np.diff(c.rp))
+    e = el.numpy().astype(np.float64)[rows] + er.numpy().astype(np.float64)[c.ci]
+    e = np.where(e > 0, e, 0.2 * e)
+    assert err(out.cpu(), O.edge_softmax(c.rp, e)) <= TOL
+
+
+@pytest.mark.parametrize("K", [2, 8, 41, 64, 128, 256, 512])
+def test_sddmm_dot_softmax(G, K):
+    c = case(G, "dense")
+    U = synth.uniform_pm1(31, K, (c.n, K))
+    V = synth.uniform_pm1(32, K, (c.n, K))
+    Ud, Vd = pad(U), pad(V)
+    out = torch.zeros(c.ci.shape[0], device=DEV)
+    G.granii_sddmm(c.g, G.SDDMM_DOT, Ud, Ud.stride(0), Vd, Vd.stride(0), K, 0.5, out)
+    torch.cuda.synchronize()
+    ref = 0.5 * O.sddmm(c.rp, c.ci, U, V)
+    assert err(out.cpu(), ref) <= TOL
+    G.granii_sddmm(c.g, G.SDDMM_DOT | G.SDDMM_ROW_SOFTMAX, Ud, Ud.stride(0), Vd, Vd.stride(0), K, 0.5, out)
+    torch.cuda.synchronize()
+    assert err(out.cpu(), O.edge_softmax(c.rp, ref)) <= TOL
+
+
+# ------------------------------------------------------------------ GEMM (tcgen05 3xTF32 + SIMT)
+GEMM_SHAPES = [(1, 16, 8), (129, 48, 37), (1000, 16, 1433), (2708, 16, 1433), (5000, 41, 602), (4096, 256, 602),
+               (3000, 1024, 100), (777, 200, 96), (1024, 512, 128), (300, 47, 256)]
+
+
+@pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
+def test_gemm_tc_fp32_accurate(G, M, N, K):
+    A = synth.uniform_pm1(40, M % 97, (M, K))
+    B = synth.glorot(41, N % 89, K, N, (K, N))
+    Ad, Bd = pad(A), B.to(DEV).contiguous()
+    C = pad(torch.zeros(M, N))
+    G.granii_gemm(M, N, K, Ad, Ad.stride(0), Bd, N, C, C.stride(0))
+    torch.cuda.synchronize()
+    ref = O.gemm(A, B)
+    assert err(C.cpu(), ref) <= TOL
+    # epilogue: row scale + attention GEMVs + ReLU, and transposed B
+    rs = synth.uniform_pm1(42, 1, (M,)).to(DEV)
+    al = synth.uniform_pm1(42, 2, (N,)).to(DEV)
+    ar = synth.uniform_pm1(42, 3, (N,)).to(DEV)
+    ol = torch.zeros(M, device=DEV)
+    orr = torch.zeros(M, device=DEV)
+    Bt = B.t().contiguous().to(DEV)
+    G.granii_gemm(M, N, K, Ad, Ad.stride(0), Bt, K, C, C.stride(0), G.GEMM_RELU | G.GEMM_TRANS_B, rs, al, ar, ol, orr)
+    torch.cuda.synchronize()
+    sref = rs.cpu().numpy().astype(np.float64)[:, None] * ref
+    assert err(C.cpu(), np.maximum(sref, 0)) <= TOL
+    assert err(ol.cpu(), sref @ al.cpu().numpy().astype(np.float64)) <= TOL
+    assert err(orr.cpu(), sref @ ar.cpu().numpy().astype(np.float64)) <= TOL
+
+
+def test_gemm_unaligned_and_transposed_a(G):
+    M, N, K = 2708, 16, 1433
+    A = synth.uniform_pm1(43, 1, (M, K))
+    B = synth.uniform_pm1(43, 2, (K, N))
+    C = torch.zeros(M, N, device=DEV)
+    G.granii_gemm(M, N, K, A.to(DEV).contiguous(), K, B.to(DEV).contiguous(), N, C, N)   # lda % 4 != 0 -> SIMT
+    torch.cuda.synchronize()
+    assert err(C.cpu(), O.gemm(A, B)) <= TOL
+    R = 20000
+    T = synth.uniform_pm1(44, 1, (R, 37))
+    D = synth.uniform_pm1(44, 2, (R, 19))
+    dW = torch.zeros(37, 19, device=DEV)
+    G.granii_gemm(37, 19, R, T.to(DEV).contiguous(), 37, D.to(DEV).contiguous(), 19, dW, 19, G.GEMM_TRANS_A)
+    torch.cuda.synchronize()
+    assert err(dW.cpu(), O.gemm(T, D, ta=True)) <= TOL
+
+
+# ------------------------------------------------------------------ layers
+def run_layer(G, c, model, comp, K1, K2, act, attn=0, seed=50, aligned=True):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    H = synth.features(seed, c.n, K1)
+    W = synth.glorot(seed, 2, K1, K2, (K1, K2))
+    al = synth.uniform_pm1(seed, 3, (K2,))
+    ar = synth.uniform_pm1(seed, 4, (K2,))
+    Hd = pad(H) if aligned else H.to(DEV).contiguous()
+    spec = LayerSpec(model, K1, K2, act, attn, comp=comp, W=W.to(DEV), a_l=al.to(DEV), a_r=ar.to(DEV))
+    net = GNN(c.g, [spec], DEV)
+    out = net.forward(Hd)
+    torch.cuda.synchronize()
+    return net, out, H, W, al, ar
+
+
+@pytest.mark.parametrize("comp", [0, 1, 2, 3])
+@pytest.mark.parametrize("name,K1,K2", [("cora", 1433, 16), ("pubmed", 32, 256), ("pubmed", 256, 32),
+                                         ("dense", 64, 64), ("tiny", 3, 5)])
+def test_gcn_forward_every_composition(G, comp, name, K1, K2):
+    c = case(G, name)
+    for aligned in (True, False):
+        _, out, H, W, _, _ = run_layer(G, c, G.GCN, comp, K1, K2, G.ACT_RELU, aligned=aligned)
+        ref, _ = O.gcn_forward(comp, c.rp, c.ci, H, W, 1)
+        assert err(out.cpu(), ref) <= TOL, (G.COMP_NAMES[comp], aligned)
+
+
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("attn", [0, 1])
+@pytest.mark.parametrize("name,K1,K2", [("directed", 64, 128), ("directed", 128, 512), ("cora", 1433, 16),
+                                         ("dense", 64, 256)])
+def test_gat_forward_both_compositions(G, comp, attn, name, K1, K2):
+    c = case(G, name)
+    _, out, H, W, al, ar = run_layer(G, c, G.GAT, comp, K1, K2, G.ACT_NONE, attn)
+    ref, _ = O.gat_forward(comp, c.rp, c.ci, H, W, al, ar, 0, dot=bool(attn))
+    assert err(out.cpu(), ref) <= TOL
+
+
+@pytest.mark.parametrize("comp", [0, 1, 2, 3])
+@pytest.mark.parametrize("name,K1,K2", [("pubmed", 32, 256), ("pubmed", 256, 32), ("dense", 48, 16)])
+def test_gcn_backward_every_composition(G, comp, name, K1, K2):
+    c = case(G, name)
+    net, out, H, W, _, _ = run_layer(G, c, G.GCN, comp, K1, K2, G.ACT_RELU)
+    Gup = synth.uniform_pm1(60, 1, (c.n, K2))
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    rdH, rdW = O.gcn_backward(comp, c.rp, c.ci, H, W, Gup, 1)
+    assert err(net.dW[0].cpu(), rdW) <= TOL
+    assert err(dH.cpu(), rdH) <= TOL
+
+
+def test_layer_determinism_and_comp_agreement(G):
+    c = case(G, "dense")
+    outs = []
+    for comp in (0, 1, 2, 3):
+        _, o, *_ = run_layer(G, c, G.GCN, comp, 64, 32, G.ACT_RELU)
+        _, o2, *_ = run_layer(G, c, G.GCN, comp, 64, 32, G.ACT_RELU)
+        assert torch.equal(o, o2)
+        outs.append(o.cpu().numpy())
+    for o in outs[1:]:
+        assert err(o, outs[0]) <= 2 * TOL
+
+
+# ------------------------------------------------------------------ selector + training helpers
+def test_select_prefilter_and_tiebreak(G):
+    c = case(G, "pubmed")
+    comp, pred = G.granii_select(c.g, G.GCN, 256, 32)
+    assert comp in (1, 3) and set(pred) == {1, 3}
+    comp, pred = G.granii_select(c.g, G.GCN, 32, 256)
+    assert comp in (0, 2) and set(pred) == {0, 2}
+    comp, pred = G.granii_select(c.g, G.GCN, 64, 64, flags=G.SELECT_NO_PREFILTER)
+    assert set(pred) == {0, 1, 2, 3} and pred[comp] == min(pred.values())
+    assert min(k for k, v in pred.items() if v == pred[comp]) == comp
+    comp, pred = G.granii_select(c.g, G.GAT, 64, 256)
+    assert comp in (16, 17) and set(pred) == {16, 17}
+
+
+def test_softmax_xent_and_sgd(G):
+    n, C = 1000, 41
+    Z = synth.uniform_pm1(70, 1, (n, C)) * 4
+    y = synth.labels(70, n, C)
+    dZ = torch.zeros(n, C, device=DEV)
+    loss = torch.zeros(n, device=DEV)
+    G.granii_softmax_xent(Z.to(DEV), y.to(DEV), n, dZ, loss)
+    torch.cuda.synchronize()
+    z = Z.numpy().astype(np.float64)
+    p = np.exp(z - z.max(1, keepdims=True))
+    p /= p.sum(1, keepdims=True)
+    onehot = np.zeros_like(p)
+    onehot[np.arange(n), y.numpy()] = 1
+    assert err(dZ.cpu(), (p - onehot) / n) <= TOL
+    assert err(loss.cpu(), -np.log(p[np.arange(n), y.numpy()])) <= TOL
+    w = torch.ones(100, device=DEV)
+    gr = torch.arange(100, dtype=torch.float32, device=DEV)
+    G.granii_sgd(gr, w, 0.5)
+    torch.cuda.synchronize()
+    assert torch.equal(w.cpu(), 1 - 0.5 * torch.arange(100, dtype=torch.float32))
