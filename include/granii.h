@@ -278,6 +278,25 @@ granii_status granii_softmax_xent(int64_t rows, int64_t C, const float* d_Z, int
 /* W -= lr * dW over n floats. */
 granii_status granii_sgd(int64_t n, float lr, const float* d_grad, float* d_param, void* stream);
 
+/* ------------------------------------------------------------------------ */
+/* Tracing (per-primitive CUDA-event timer; measurement support)             */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  char name[32];   /* primitive: spmm, sddmm, gemm_tc, gemm_simt, gemm_tn, csr, elementwise */
+  int64_t calls;   /* launcher calls recorded                                            */
+  int64_t launches;/* CUDA kernels launched by those calls                               */
+  double ms;       /* summed device time between events recorded on the launch stream    */
+  double bytes;    /* summed ALGORITHMIC bytes (DESIGN.md §6 per-unit figures)            */
+  double flops;    /* summed algorithmic flops                                           */
+} granii_prof_entry;
+
+/* Enable (1) / disable (0) event recording around every primitive; resets the table. */
+granii_status granii_profile_enable(int32_t on);
+/* Sync the device, aggregate the recorded events per primitive into out[0..*n). */
+granii_status granii_profile_read(granii_prof_entry* out, int32_t max_entries, int32_t* n);
+/* Total CUDA kernels this library has launched in this process (monotonic). */
+int64_t granii_launch_count(void);
+
 #if defined(__GNUC__)
 #pragma GCC visibility pop
 #endif

@@ -61,6 +61,7 @@ __global__ void k_sgd(int64_t n, float lr, const float* __restrict__ g, float* _
 granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
                                float* dst, int64_t ldd, cudaStream_t st) {
   if (rows * K == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, 12.0 * rows * K, 0.0, 1);
   k_relu_mask<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, out, ldo, g, ldg, dst, ldd);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
@@ -69,6 +70,7 @@ granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_
 granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,
                                cudaStream_t st) {
   if (rows * K == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, 8.0 * rows * K, 0.0, 1);
   k_copy_rows<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, src, lds, dst, ldd);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
@@ -77,6 +79,7 @@ granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_
 granii_status launch_softmax_xent(int64_t rows, int64_t C, const float* Z, int64_t ldz, const int32_t* y,
                                   int64_t n_total, float* dZ, int64_t lddz, float* loss, cudaStream_t st) {
   if (rows == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, 8.0 * rows * C + 8.0 * rows, 0.0, 1);
   const unsigned b = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, 8), 148 * 16));
   k_softmax_xent<<<b, 256, 0, st>>>(rows, C, Z, ldz, y, 1.f / (float)n_total, dZ, lddz, loss);
   GR_CHECK_LAUNCH();
@@ -85,6 +88,7 @@ granii_status launch_softmax_xent(int64_t rows, int64_t C, const float* Z, int64
 
 granii_status launch_sgd(int64_t n, float lr, const float* g, float* p, cudaStream_t st) {
   if (n == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, 12.0 * n, 2.0 * n, 1);
   k_sgd<<<blocks_for(n), 256, 0, st>>>(n, lr, g, p);
   GR_CHECK_LAUNCH();
   return GRANII_OK;

@@ -505,8 +505,12 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
   DevInfo di;
   GR_TRY(dev_info(&di));
 
+  // algorithmic bytes: A and B read once, C written once (fp32); flops 2MNK
+  const double gbytes = 4.0 * ((double)M * K + (double)K * N + (store ? (double)M * N : 0.0));
+  const double gflops = 2.0 * (double)M * N * K;
   if (flags & GRANII_GEMM_TRANS_A) {
     if (att || rs || relu || tb) return fail(GRANII_ERR_UNSUPPORTED, "TRANS_A supports plain C = A^T B only");
+    ProfScope ps("gemm_tn", st, gbytes, gflops, 2);
     // here K is the reduction (rows), A stored K x M, B stored K x N
     const int64_t splits = std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(K, 4096)));
     const int64_t chunk = round_up(ceil_div(K, splits), 32);
@@ -525,6 +529,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
     if (att) return fail(GRANII_ERR_UNSUPPORTED, "attention epilogue needs the tensor-core path (lda % 4 == 0)");
     dim3 grid((unsigned)ceil_div(M, 64), (unsigned)ceil_div(N, 64));
     if (!store) return GRANII_OK;
+    ProfScope ps("gemm_simt", st, gbytes, gflops, 1);
     if (tb) k_gemm_simt<false, true><<<grid, 256, 0, st>>>((int)M, (int)N, (int)K, A, lda, B, ldb, C, ldc, rs, relu);
     else k_gemm_simt<false, false><<<grid, 256, 0, st>>>((int)M, (int)N, (int)K, A, lda, B, ldb, C, ldc, rs, relu);
     GR_CHECK_LAUNCH();
@@ -533,6 +538,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
 
   const int bn = pick_bn(N);
   const int64_t Npad = round_up(N, bn), Kpad = round_up(K, TC_BK);
+  ProfScope ps("gemm_tc", st, gbytes, gflops, 2);
   uint8_t* w = (uint8_t*)(((uintptr_t)ws + 1023) & ~(uintptr_t)1023);
   float* bhi = (float*)w;
   float* blo = bhi + Npad * Kpad;
@@ -564,6 +570,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
     default: GR_TRY(launch_tc_bn<256>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
   }
   if (tiles > 1) {
+    ps.add_launches((ep.out_l ? 1 : 0) + (ep.out_r ? 1 : 0));
     const unsigned b = (unsigned)std::min<int64_t>(ceil_div(M, 256), 4096);
     if (ep.out_l) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_l, epi->out_l);
     if (ep.out_r) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_r, epi->out_r);

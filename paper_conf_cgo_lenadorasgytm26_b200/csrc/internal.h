@@ -50,6 +50,20 @@ struct DevInfo {
 };
 granii_status dev_info(DevInfo* out);
 
+// ----------------------------------------------------------------- tracing
+// RAII scope around one launcher call: counts kernel launches always; records
+// a pair of CUDA events on the launch stream when profiling is enabled.
+struct ProfScope {
+  ProfScope(const char* name, cudaStream_t st, double bytes, double flops, int launches);
+  ~ProfScope();
+  void add_launches(int n);
+  const char* name;
+  cudaStream_t st;
+  double bytes, flops;
+  int launches;
+  int slot;
+};
+
 }  // namespace granii
 
 // ----------------------------------------------------------------- graph

@@ -197,6 +197,10 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   const uint32_t base = op & 0xF;
   const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
   SddmmArgs a{g->n_rows, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order};
+  // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
+  const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
+  ProfScope ps("sddmm", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K,
+               (K > 1 && sm) ? 2 : 1);
   if (K == 1) {
     const int lpg = lpg_for_degree(g->avg_deg());
     const int64_t units = ceil_div(g->n_rows, 32 / lpg);

@@ -284,6 +284,11 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
   const bool warp_mode = g->avg_deg() >= 16.f;
   SpmmArgs a{g->n_rows, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0, g->order};
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
+  // algorithmic bytes: per entry col id (+w, +cs) + one K-row of X;
+  // per row row_ptr + the K-row of Y (+rs)
+  const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
+  const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) + R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0));
+  ProfScope ps("spmm", st, bytes, 2.0 * nnz * K, (int)ceil_div(K, kw));
   for (int64_t k0 = 0; k0 < K; k0 += kw) {
     a.k0 = k0;
     a.kw = std::min(kw, K - k0);

@@ -86,6 +86,9 @@ _SIGS = {
     "granii_comm_destroy": ([_p], ctypes.c_int),
     "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
     "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
+    "granii_profile_enable": ([_i32], ctypes.c_int),
+    "granii_profile_read": ([_p, _i32, ctypes.POINTER(_i32)], ctypes.c_int),
+    "granii_launch_count": ([], ctypes.c_int64),
 }
 for _name, (_args, _res) in _SIGS.items():
     _fn = getattr(_lib, _name)
@@ -293,3 +296,25 @@ def granii_softmax_xent(Z: torch.Tensor, y: torch.Tensor, n_total: int, dZ: torc
 
 def granii_sgd(grad: torch.Tensor, param: torch.Tensor, lr: float, stream=None):
     _check(_lib.granii_sgd(param.numel(), lr, _ptr(grad), _ptr(param), _stream(stream)), "granii_sgd")
+
+
+# ---------------------------------------------------------------- tracing
+class prof_entry(ctypes.Structure):
+    _fields_ = [("name", ctypes.c_char * 32), ("calls", _i64), ("launches", _i64), ("ms", ctypes.c_double),
+                ("bytes", ctypes.c_double), ("flops", ctypes.c_double)]
+
+
+def granii_profile_enable(on: bool = True):
+    _check(_lib.granii_profile_enable(1 if on else 0), "granii_profile_enable")
+
+
+def granii_profile_read() -> dict:
+    arr = (prof_entry * 32)()
+    n = _i32()
+    _check(_lib.granii_profile_read(arr, 32, ctypes.byref(n)), "granii_profile_read")
+    return {arr[i].name.decode(): {"calls": arr[i].calls, "launches": arr[i].launches, "ms": arr[i].ms,
+                                   "bytes": arr[i].bytes, "flops": arr[i].flops} for i in range(n.value)}
+
+
+def granii_launch_count() -> int:
+    return int(_lib.granii_launch_count())
