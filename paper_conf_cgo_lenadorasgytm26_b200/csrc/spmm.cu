@@ -67,12 +67,42 @@ struct SpmmArgs {
 };
 
 // ------------------------------------------------------------------ warp-per-row
+// One chunk of 32 entries of a row, one per lane: column id and weight.  Lanes
+// past the row's end reuse the row's last column with w = 0, so every later
+// step is branch-free (the padded gathers hit L1 and add exact zeros).
+template <bool W, bool CS>
+__device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t re, int lane, int32_t& c, float& w) {
+  const bool valid = e + lane < re;
+  const int64_t ee = valid ? e + lane : re - 1;
+  c = __ldg(a.col_idx + ee);
+  w = valid ? (W ? __ldg(a.vals + ee) : 1.f) : 0.f;
+  if (CS) w *= __ldg(a.cs + c);
+}
+
 template <int VEC, int LPG, int NJ, bool W, bool CS>
-__global__ void __launch_bounds__(256) k_spmm_warp(SpmmArgs a) {
+__global__ void __launch_bounds__(256, 3) k_spmm_warp(SpmmArgs a) {
   constexpr int G = 32 / LPG;
+  constexpr int U = 32 / G >= 4 ? 4 : 32 / G;  // neighbours per group per step; G*U divides 32
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  bool colok[NJ];
+  uint32_t coff[NJ];  // byte offset of this lane's j-th vector inside the slice
+  const int last = (int)((a.kw - 1) / VEC);  // last vector that holds a column of the slice
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    const int v = lig + j * LPG;
+    colok[j] = v <= last;
+    // lanes past the slice re-read its last vector (in bounds: ldx >= k0 + kw, rounded to VEC)
+    // so loads are unconditional; their sums are never stored
+    coff[j] = (uint32_t)((v <= last ? v : last) * VEC * 4);
+  }
+  // per-lane base of the column slice; row offset = c * row_bytes in one IMAD.WIDE.U32
+  const char* __restrict__ xb = reinterpret_cast<const char*>(a.X + a.k0);
+  const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
+  const char* xbj[NJ];  // one 64-bit base per vector: each gather address is a single IMAD.WIDE.U32
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) xbj[j] = xb + coff[j];
   for (int64_t t = warp; t < a.n_rows; t += nwarps) {
     const int64_t row = a.order ? a.order[t] : t;
     const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
@@ -81,39 +111,39 @@ __global__ void __launch_bounds__(256) k_spmm_warp(SpmmArgs a) {
     for (int j = 0; j < NJ; ++j)
 #pragma unroll
       for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
-    bool colok[NJ];
+    if (rs0 < re) {
+      int32_t cn;
+      float wn;
+      load_chunk<W, CS>(a, rs0, re, lane, cn, wn);
+      for (int64_t base = rs0; base < re; base += 32) {
+        const int32_t c = cn;
+        const float w = wn;
+        if (base + 32 < re) load_chunk<W, CS>(a, base + 32, re, lane, cn, wn);  // prefetch next chunk
+        const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
+        const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
+        for (int s = 0; s < steps; ++s) {
+          uint32_t cu[U];
+          float wu[U];
 #pragma unroll
-    for (int j = 0; j < NJ; ++j) colok[j] = (int64_t)(lig + j * LPG) * VEC < a.kw;
-    const float* Xs = a.X + a.k0 + (int64_t)lig * VEC;
-    for (int64_t base = rs0; base < re; base += 32) {
-      const int64_t e = base + lane;
-      const bool valid = e < re;
-      int32_t c = valid ? __ldg(a.col_idx + e) : 0;
-      float w = valid ? (W ? __ldg(a.vals + e) : 1.f) : 0.f;
-      if (CS && valid) w *= __ldg(a.cs + c);
-      const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
-      // U = 2 neighbours per group per step (G*2 per warp) -> 2*NJ vector loads in flight
-      for (int i0 = 0; i0 < cnt; i0 += 2 * G) {
-        const int i1 = i0 + grp, i2 = i0 + G + grp;
-        const int32_t c1 = __shfl_sync(0xffffffffu, c, i1 & 31), c2 = __shfl_sync(0xffffffffu, c, i2 & 31);
-        const float w1 = __shfl_sync(0xffffffffu, w, i1 & 31), w2 = __shfl_sync(0xffffffffu, w, i2 & 31);
-        const bool p1 = i1 < cnt, p2 = i2 < cnt;
-        float x1[NJ][VEC], x2[NJ][VEC];
+          for (int u = 0; u < U; ++u) {
+            const int i = s * G * U + u * G + grp;  // <= 31
+            cu[u] = (uint32_t)__shfl_sync(0xffffffffu, c, i);
+            wu[u] = __shfl_sync(0xffffffffu, w, i);
+          }
+          float x[U][NJ][VEC];
 #pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          if (p1 && colok[j]) ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1[j]);
-          else
+          for (int u = 0; u < U; ++u) {
 #pragma unroll
-            for (int v = 0; v < VEC; ++v) x1[j][v] = 0.f;
-          if (p2 && colok[j]) ldv<VEC>(Xs + (int64_t)c2 * a.ldx + j * LPG * VEC, x2[j]);
-          else
+            for (int j = 0; j < NJ; ++j)
+              ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
+          }
 #pragma unroll
-            for (int v = 0; v < VEC; ++v) x2[j][v] = 0.f;
+          for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int j = 0; j < NJ; ++j)
+#pragma unroll
+              for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
         }
-#pragma unroll
-        for (int j = 0; j < NJ; ++j)
-#pragma unroll
-          for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w2, x2[j][v], fmaf(w1, x1[j][v], acc[j][v]));
       }
     }
     // reduce the G groups (fixed butterfly order)
@@ -143,15 +173,26 @@ __global__ void __launch_bounds__(256) k_spmm_warp(SpmmArgs a) {
 
 // ------------------------------------------------------------------ group-per-row
 template <int VEC, int LPG, int NJ, bool W, bool CS>
-__global__ void __launch_bounds__(256) k_spmm_group(SpmmArgs a) {
+__global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   bool colok[NJ];
+  uint32_t coff[NJ];
+  const int last = (int)((a.kw - 1) / VEC);
 #pragma unroll
-  for (int j = 0; j < NJ; ++j) colok[j] = (int64_t)(lig + j * LPG) * VEC < a.kw;
-  const float* Xs = a.X + a.k0 + (int64_t)lig * VEC;
+  for (int j = 0; j < NJ; ++j) {
+    const int v = lig + j * LPG;
+    colok[j] = v <= last;
+    coff[j] = (uint32_t)((v <= last ? v : last) * VEC * 4);  // clamped: unconditional loads
+  }
+  const char* __restrict__ xb = reinterpret_cast<const char*>(a.X + a.k0);
+  const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
+  const char* xbj[NJ];  // one 64-bit base per vector: each gather address is a single IMAD.WIDE.U32
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) xbj[j] = xb + coff[j];
+  constexpr int U = 4;
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
@@ -162,39 +203,30 @@ __global__ void __launch_bounds__(256) k_spmm_group(SpmmArgs a) {
     for (int j = 0; j < NJ; ++j)
 #pragma unroll
       for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
-    int64_t e = rs0;
-    for (; e + 1 < re; e += 2) {
-      const int32_t c1 = __ldg(a.col_idx + e), c2 = __ldg(a.col_idx + e + 1);
-      float w1 = W ? __ldg(a.vals + e) : 1.f, w2 = W ? __ldg(a.vals + e + 1) : 1.f;
-      if (CS) { w1 *= __ldg(a.cs + c1); w2 *= __ldg(a.cs + c2); }
-      float x1[NJ][VEC], x2[NJ][VEC];
+    for (int64_t e = rs0; e < re; e += U) {
+      uint32_t cu[U];
+      float wu[U];
 #pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        if (colok[j]) {
-          ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1[j]);
-          ldv<VEC>(Xs + (int64_t)c2 * a.ldx + j * LPG * VEC, x2[j]);
-        } else {
+      for (int u = 0; u < U; ++u) {  // entries past the row end: last entry, weight 0
+        const bool ok = e + u < re;
+        const int64_t ee = ok ? e + u : re - 1;
+        cu[u] = (uint32_t)__ldg(a.col_idx + ee);
+        wu[u] = ok ? (W ? __ldg(a.vals + ee) : 1.f) : 0.f;
+        if (CS) wu[u] *= __ldg(a.cs + cu[u]);
+      }
+      float x[U][NJ][VEC];
 #pragma unroll
-          for (int v = 0; v < VEC; ++v) x1[j][v] = x2[j][v] = 0.f;
-        }
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
       }
 #pragma unroll
-      for (int j = 0; j < NJ; ++j)
+      for (int u = 0; u < U; ++u)
 #pragma unroll
-        for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w2, x2[j][v], fmaf(w1, x1[j][v], acc[j][v]));
-    }
-    if (e < re) {
-      const int32_t c1 = __ldg(a.col_idx + e);
-      float w1 = W ? __ldg(a.vals + e) : 1.f;
-      if (CS) w1 *= __ldg(a.cs + c1);
+        for (int j = 0; j < NJ; ++j)
 #pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        if (!colok[j]) continue;
-        float x1[VEC];
-        ldv<VEC>(Xs + (int64_t)c1 * a.ldx + j * LPG * VEC, x1);
-#pragma unroll
-        for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(w1, x1[v], acc[j][v]);
-      }
+          for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
     }
     const float s = a.rs ? __ldg(a.rs + row) : 1.f;
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
@@ -244,8 +276,14 @@ static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, 
   if (vec4) {
     if (kw <= 16) return launch_cfg<4, 4, 1>(a, warp_mode, w, cs, sms, st);
     if (kw <= 32) return launch_cfg<4, 8, 1>(a, warp_mode, w, cs, sms, st);
-    if (kw <= 64) return launch_cfg<4, 16, 1>(a, warp_mode, w, cs, sms, st);
-    if (kw <= 128) return launch_cfg<4, 32, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 64) {
+      if (warp_mode) return launch_cfg<4, 8, 2>(a, warp_mode, w, cs, sms, st);  // 4 groups x 2 float4
+      return launch_cfg<4, 16, 1>(a, warp_mode, w, cs, sms, st);
+    }
+    if (kw <= 128) {
+      if (warp_mode) return launch_cfg<4, 16, 2>(a, warp_mode, w, cs, sms, st);
+      return launch_cfg<4, 32, 1>(a, warp_mode, w, cs, sms, st);
+    }
     if (kw <= 256) return launch_cfg<4, 32, 2>(a, warp_mode, w, cs, sms, st);
     if (kw <= 512) return launch_cfg<4, 32, 4>(a, warp_mode, w, cs, sms, st);
     return launch_cfg<4, 32, 8>(a, warp_mode, w, cs, sms, st);
@@ -266,11 +304,14 @@ int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t 
     int64_t v = atoll(env);
     if (v > 0) return std::min<int64_t>(std::max<int64_t>(v, 1), maxw);
   }
-  const double xbytes = (double)g->n_cols * (double)K * 4.0;
-  if (g->avg_deg() >= 32.f && xbytes > 0.45 * (double)l2_bytes) {
-    int64_t nsl = (int64_t)std::ceil(xbytes / (0.45 * (double)l2_bytes));
-    int64_t w = round_up(ceil_div(K, nsl), vec4 ? 64 : 32);
-    kw = std::min(kw, std::max<int64_t>(w, vec4 ? 64 : 32));
+  const double per_col = (double)g->n_cols * 4.0;
+  if (g->avg_deg() >= 32.f && per_col * (double)K > 0.6 * (double)l2_bytes) {
+    const int64_t unit = vec4 ? 64 : 32;
+    const int64_t fit = (int64_t)(0.55 * (double)l2_bytes / per_col) / unit * unit;  // columns resident in L2
+    if (fit >= unit) {  // otherwise a slice cannot stay resident: do not re-read col_idx for nothing
+      const int64_t nsl = ceil_div(K, fit);
+      kw = std::min(kw, round_up(ceil_div(K, nsl), unit));
+    }
   }
   return kw;
 }
