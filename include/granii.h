@@ -111,6 +111,15 @@ granii_status granii_graph_dinv(granii_graph g, const float** d_dinv);
  * a host row_ptr; bounds is int64[world + 1].  Used by the distributed layer. */
 granii_status granii_partition_bounds(int64_t num_nodes, const int64_t* h_row_ptr, int32_t world,
                                       int64_t* bounds);
+/* Host helper (no device work): map global column ids to the padded gather
+ * layout, out[i] = owner(j)*max_rows + (j - bounds[owner(j)]) with
+ * bounds[owner] <= j < bounds[owner+1].  The device applies the same map at
+ * graph creation; tests compare the two. */
+granii_status granii_gather_layout_host(int64_t n, const int32_t* h_cols, const int64_t* bounds, int32_t world,
+                                        int64_t max_rows, int32_t* h_out);
+/* Like export_csr but col ids are returned exactly as stored on the device
+ * (gather-layout ids when partitioned). */
+granii_status granii_graph_export_local(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx);
 
 /* ------------------------------------------------------------------------ */
 /* Primitives (L80-L92).  All operate on this rank's rows of Ã.              */

@@ -132,6 +132,30 @@ granii_status granii_graph_export_csr(granii_graph g, int64_t* h_row_ptr, int32_
   API_END
 }
 
+granii_status granii_graph_export_local(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx) {
+  API_BEGIN
+  GR_ARG(g && h_row_ptr && h_col_idx, "NULL argument");
+  GR_CUDA(cudaDeviceSynchronize());
+  GR_CUDA(cudaMemcpy(h_row_ptr, g->row_ptr, (g->n_rows + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+  if (g->local_nnz > 0)
+    GR_CUDA(cudaMemcpy(h_col_idx, g->col_idx, g->local_nnz * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  return GRANII_OK;
+  API_END
+}
+
+granii_status granii_gather_layout_host(int64_t n, const int32_t* cols, const int64_t* bounds, int32_t world,
+                                        int64_t max_rows, int32_t* out) {
+  GR_ARG((n == 0 || (cols && out)) && bounds && world >= 1 && max_rows >= 1, "bad argument");
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t j = cols[i];
+    GR_ARG(j >= bounds[0] && j < bounds[world], "column outside the partitioned range");
+    int g = 0;
+    while (g + 1 < world && bounds[g + 1] <= j) ++g;
+    out[i] = (int32_t)(g * max_rows + (j - bounds[g]));
+  }
+  return GRANII_OK;
+}
+
 granii_status granii_graph_dinv(granii_graph g, const float** d) {
   GR_ARG(g && d, "NULL argument");
   *d = g->dinv_rows;

@@ -299,6 +299,179 @@ __global__ void k_prep_b(int K, int N, const float* __restrict__ B, int64_t ldb,
   }
 }
 
+// ======================================================================= Aᵀ·B on tensor cores
+// dW = Aᵀ B with A stored R x M, B stored R x N (R = nodes, the reduction).  Both
+// MMA operands are MN-major: TMA boxes of 32 elements (one 128-byte swizzle row)
+// x 32 reduction rows; an MN atom (32 wide) is 4 KB, atoms are LBO = 4 KB apart,
+// 8-row k groups SBO = 1 KB apart, one tf32 MMA (K = 8) consumes one k group.
+// Split-K over R (blockIdx.z) into a partial buffer [splits][M][N], summed later
+// in fixed order (deterministic).  Converters split A and B into hi / lo.
+__device__ __forceinline__ uint64_t desc_sw128_mn(uint32_t saddr, uint32_t lbo, uint32_t sbo = 1024) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);
+  d |= (uint64_t)(((lbo & 0x0FFFFFFFu) >> 4) & 0x3FFF) << 16;  // leading byte offset: stride between MN atoms
+  d |= (uint64_t)((sbo >> 4) & 0x3FFF) << 32;  // stride byte offset: between 8-row k groups
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)((lbo >> 28) & 7u) << 61;   // layout type (1 = SWIZZLE_128B_BASE32B for MN-major tf32)
+  return d;
+}
+__host__ __device__ constexpr uint32_t idesc_tf32_mn(int M, int N) {
+  return idesc_tf32(M, N) | (1u << 15) | (1u << 16);  // a_major = b_major = MN
+}
+
+template <int BN>
+struct TnCfg {
+  static constexpr int A_BYTES = TC_BM * TC_BK * 4;  // 128 (M) x 32 (k) fp32 = 4 MN atoms
+  static constexpr int B_BYTES = BN * TC_BK * 4;
+  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int STAGES = (STAGE * 3 <= 200 * 1024) ? 3 : 2;
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
+};
+
+template <int BN>
+__global__ void __launch_bounds__(192, 1)
+    k_gemm_tn_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, int M, int N,
+                 int kblocks_per_split, int total_kblocks, float* __restrict__ part, uint32_t dlbo, uint32_t dsbo,
+                 uint32_t dkstep) {
+  using Cfg = TnCfg<BN>;
+  constexpr int S = Cfg::STAGES;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint64_t* bars = (uint64_t*)(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* accum = bars + 3 * S;
+  uint32_t* tmem_slot = (uint32_t*)(bars + 3 * S + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int m0 = blockIdx.x * TC_BM, n0 = blockIdx.y * BN;
+  const int kb0 = blockIdx.z * kblocks_per_split;
+  const int nk = max(0, min(kblocks_per_split, total_kblocks - kb0));
+  auto a_hi = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto a_lo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto b_hi = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
+  auto b_lo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(accum, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(Cfg::TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  if (warp == 0) {
+    if (lane == 0) {
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
+        const int r = (kb0 + kb) * TC_BK;
+#pragma unroll
+        for (int t = 0; t < TC_BM / 32; ++t) tma_load_2d(&tmA, &full[s], a_hi(s) + t * 4096, m0 + 32 * t, r);
+#pragma unroll
+        for (int t = 0; t < BN / 32; ++t) tma_load_2d(&tmB, &full[s], b_hi(s) + t * 4096, n0 + 32 * t, r);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nk > 0) {
+      const uint32_t idesc = (idesc_tf32(TC_BM, BN) & ~(3u << 15)) | ((dkstep >> 16) << 15);
+      for (int kb = 0; kb < nk; ++kb) {
+        const int s = kb % S;
+        const uint32_t ph = (kb / S) & 1;
+        mbar_wait(&conv[s], ph);
+        tc_fence_after();
+        const uint32_t ah = smem_u32(a_hi(s)), al = smem_u32(a_lo(s));
+        const uint32_t bh = smem_u32(b_hi(s)), bl = smem_u32(b_lo(s));
+#pragma unroll
+        for (int k = 0; k < TC_BK / 8; ++k) {  // one 8-row k group (1 KB) per MMA
+          const uint32_t off = k * (dkstep & 0xFFFF);
+          const uint64_t dah = desc_sw128_mn(ah + off, dlbo, dsbo), dal = desc_sw128_mn(al + off, dlbo, dsbo);
+          const uint64_t dbh = desc_sw128_mn(bh + off, dlbo, dsbo), dbl = desc_sw128_mn(bl + off, dlbo, dsbo);
+          mma_tf32(tmem, dah, dbh, idesc, (kb | k) ? 1u : 0u);
+          mma_tf32(tmem, dah, dbl, idesc, 1u);
+          mma_tf32(tmem, dal, dbh, idesc, 1u);
+        }
+        mma_commit(&empty[s]);
+      }
+      mma_commit(accum);
+    }
+  } else {
+    const int ct = threadIdx.x - 64;
+    for (int kb = 0; kb < nk; ++kb) {
+      const int s = kb % S;
+      const uint32_t ph = (kb / S) & 1;
+      mbar_wait(&full[s], ph);
+      float4* ahp = reinterpret_cast<float4*>(a_hi(s));
+      float4* alp = reinterpret_cast<float4*>(a_lo(s));
+      float4* bhp = reinterpret_cast<float4*>(b_hi(s));
+      float4* blp = reinterpret_cast<float4*>(b_lo(s));
+#pragma unroll 4
+      for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) {
+        const float4 x = ahp[i];
+        float4 h, l;
+        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
+        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
+        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
+        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
+        ahp[i] = h;
+        alp[i] = l;
+      }
+#pragma unroll 4
+      for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) {
+        const float4 x = bhp[i];
+        float4 h, l;
+        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
+        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
+        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
+        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
+        bhp[i] = h;
+        blp[i] = l;
+      }
+      fence_proxy_async();
+      mbar_arrive(&conv[s]);
+    }
+    // epilogue: this split's partial tile (zeros if the split is empty)
+    const int quad = warp & 3;
+    const int r = m0 + quad * 32 + lane;
+    float* P = part + (int64_t)blockIdx.z * M * N;
+    if (nk > 0) {
+      mbar_wait(accum, 0);
+      tc_fence_after();
+    }
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      float v[16];
+      if (nk > 0) tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + c0, v);
+      else
+#pragma unroll
+        for (int j = 0; j < 16; ++j) v[j] = 0.f;
+      if (r < M) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j)
+          if (n0 + c0 + j < N) P[(int64_t)r * N + n0 + c0 + j] = v[j];
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS));
+  }
+}
+
 // sum the per-N-tile attention partials in fixed tile order
 __global__ void k_reduce_partials(int M, int tiles, const float* __restrict__ part, float* __restrict__ out) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
@@ -429,7 +602,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
 }
 
 static bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
-                     uint32_t box_inner, uint32_t box_outer) {
+                     uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
   auto enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {inner, outer};
@@ -437,7 +610,7 @@ static bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t 
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t es[2] = {1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
@@ -462,11 +635,31 @@ static bool tc_eligible(int64_t M, int64_t N, int64_t K, const float* A, int64_t
   return true;
 }
 
+// Aᵀ·B plan: BN multiple of 32 (TMA boxes of 32), split the reduction so the grid
+// fills the 148 SMs (one CTA per SM: ~190 KB smem), >= 8 k-blocks per split.
+struct TnPlan {
+  int bn;
+  int64_t mt, nt, total_kb, kb_per, splits;
+};
+static TnPlan tn_plan(int64_t M, int64_t N, int64_t R) {
+  TnPlan p;
+  p.bn = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
+  p.mt = ceil_div(M, TC_BM);
+  p.nt = ceil_div(N, p.bn);
+  p.total_kb = ceil_div(R, TC_BK);
+  int64_t splits = std::max<int64_t>(1, ceil_div(148, p.mt * p.nt));
+  splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.total_kb / 8));
+  p.kb_per = ceil_div(p.total_kb, splits);
+  p.splits = ceil_div(p.total_kb, p.kb_per);
+  return p;
+}
+static int64_t simt_tn_splits(int64_t R) { return std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(R, 4096))); }
+
 size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags) {
   size_t ws = 0;
   if (flags & GRANII_GEMM_TRANS_A) {
-    // split-K partials
-    const int64_t splits = std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(K, 4096)));
+    // split-K partials (tensor-core or SIMT plan, whichever is larger)
+    const int64_t splits = std::max(tn_plan(M, N, K).splits, simt_tn_splits(K));
     return (size_t)splits * M * N * 4 + 256;
   }
   const int bn = pick_bn(N);
@@ -510,9 +703,52 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
   const double gflops = 2.0 * (double)M * N * K;
   if (flags & GRANII_GEMM_TRANS_A) {
     if (att || rs || relu || tb) return fail(GRANII_ERR_UNSUPPORTED, "TRANS_A supports plain C = A^T B only");
-    ProfScope ps("gemm_tn", st, gbytes, gflops, 2);
     // here K is the reduction (rows), A stored K x M, B stored K x N
-    const int64_t splits = std::max<int64_t>(1, std::min<int64_t>(64, ceil_div(K, 4096)));
+    const bool tc = !getenv("GRANII_GEMM_SIMT") && lda % 4 == 0 && ldb % 4 == 0 && ((uintptr_t)A & 15) == 0 &&
+                    ((uintptr_t)B & 15) == 0 && M <= INT32_MAX && N <= INT32_MAX;
+    if (tc) {
+      const TnPlan p = tn_plan(M, N, K);
+      ProfScope ps("gemm_tn_tc", st, gbytes, gflops, 2);
+      float* part = (float*)ws;
+      // MN-major tf32 operands need the 128B swizzle with 32B atoms (descriptor layout type 1)
+      // debug override GRANII_TN_DESC=lbo,sbo,kstep,major,layout,tma_swizzle
+      uint32_t dlbo = 4096, dsbo = 512, dkstep = 1024, dmaj = 3, dlay = 1, dswz = 4;
+      if (const char* e = getenv("GRANII_TN_DESC"))
+        sscanf(e, "%u,%u,%u,%u,%u,%u", &dlbo, &dsbo, &dkstep, &dmaj, &dlay, &dswz);
+      dkstep = (dkstep & 0xFFFF) | (dmaj << 16);
+      dlbo = (dlbo & 0x0FFFFFFFu) | (dlay << 28);
+      CUtensorMap ta, tb;
+      if (!make_map(&ta, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, 32, TC_BK, (CUtensorMapSwizzle)dswz) ||
+          !make_map(&tb, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, 32, TC_BK, (CUtensorMapSwizzle)dswz))
+        return fail(GRANII_ERR_CUDA, "cuTensorMapEncodeTiled failed (TN)");
+      dim3 grid((unsigned)p.mt, (unsigned)p.nt, (unsigned)p.splits);
+#define GR_TN(BN)                                                                                       \
+  do {                                                                                                  \
+    static bool set_ = false;                                                                           \
+    if (!set_) {                                                                                        \
+      GR_CUDA(cudaFuncSetAttribute(k_gemm_tn_tc<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,       \
+                                   TnCfg<BN>::SMEM));                                                   \
+      set_ = true;                                                                                      \
+    }                                                                                                   \
+    k_gemm_tn_tc<BN><<<grid, 192, TnCfg<BN>::SMEM, st>>>(ta, tb, (int)M, (int)N, (int)p.kb_per,         \
+                                                         (int)p.total_kb, part, dlbo, dsbo, dkstep);    \
+  } while (0)
+      switch (p.bn) {
+        case 32: GR_TN(32); break;
+        case 64: GR_TN(64); break;
+        case 128: GR_TN(128); break;
+        default: GR_TN(256); break;
+      }
+#undef GR_TN
+      GR_CHECK_LAUNCH();
+      const int64_t MN = M * N;
+      k_sum_splits<<<(unsigned)std::min<int64_t>(ceil_div(MN, 256), 4096), 256, 0, st>>>(MN, (int)p.splits, part, C,
+                                                                                        (int)M, (int)N, ldc);
+      GR_CHECK_LAUNCH();
+      return GRANII_OK;
+    }
+    ProfScope ps("gemm_tn", st, gbytes, gflops, 2);
+    const int64_t splits = simt_tn_splits(K);
     const int64_t chunk = round_up(ceil_div(K, splits), 32);
     float* part = (float*)ws;
     dim3 grid((unsigned)ceil_div(M, 64), (unsigned)ceil_div(N, 64), (unsigned)splits);

@@ -68,6 +68,8 @@ _SIGS = {
     "granii_graph_export_csr": ([_p, _p, _p], ctypes.c_int),
     "granii_graph_dinv": ([_p, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_partition_bounds": ([_i64, _p, _i32, _p], ctypes.c_int),
+    "granii_gather_layout_host": ([_i64, _p, _p, _i32, _i64, _p], ctypes.c_int),
+    "granii_graph_export_local": ([_p, _p, _p], ctypes.c_int),
     "granii_spmm": ([_p, _p, _p, _i64, _i64, _p, _i64, _p, _p, _u32, _p], ctypes.c_int),
     "granii_sddmm": ([_p, _u32, _p, _i64, _p, _i64, _i64, _f, _p, _p], ctypes.c_int),
     "granii_gemm_workspace_size": ([_i64, _i64, _i64, _u32, ctypes.POINTER(_sz)], ctypes.c_int),
@@ -182,6 +184,24 @@ def granii_graph_export_csr(g: Graph):
     ci = np.zeros(max(g.nnz, 1), np.int32)
     _check(_lib.granii_graph_export_csr(g.handle, rp.ctypes.data, ci.ctypes.data), "granii_graph_export_csr")
     return rp, ci[: g.nnz]
+
+
+def granii_graph_export_local(g: Graph):
+    import numpy as np
+    rp = np.zeros(g.n_rows + 1, np.int64)
+    ci = np.zeros(max(g.nnz, 1), np.int32)
+    _check(_lib.granii_graph_export_local(g.handle, rp.ctypes.data, ci.ctypes.data), "granii_graph_export_local")
+    return rp, ci[: g.nnz]
+
+
+def granii_gather_layout_host(cols, bounds, world: int, max_rows: int):
+    import numpy as np
+    c = np.ascontiguousarray(cols, dtype=np.int32)
+    b = np.ascontiguousarray(bounds, dtype=np.int64)
+    out = np.zeros(max(c.shape[0], 1), np.int32)
+    _check(_lib.granii_gather_layout_host(c.shape[0], c.ctypes.data, b.ctypes.data, world, max_rows,
+                                          out.ctypes.data), "granii_gather_layout_host")
+    return out[: c.shape[0]]
 
 
 def granii_graph_dinv(g: Graph) -> int:

@@ -292,6 +292,25 @@ def test_gemm_unaligned_and_transposed_a(G):
     assert err(dW.cpu(), O.gemm(T, D, ta=True)) <= TOL
 
 
+@pytest.mark.parametrize("M,N,R", [(602, 256, 50000), (256, 41, 30000), (128, 32, 1000), (100, 47, 777),
+                                   (1024, 1024, 5000), (13, 7, 33)])
+def test_gemm_tn_tensor_core(G, M, N, R):
+    """dW = Aᵀ B over the node dimension: MN-major tcgen05 operands + split-K (aligned lds)."""
+    A = synth.uniform_pm1(45, M % 13, (R, M))
+    B = synth.uniform_pm1(46, N % 11, (R, N))
+    Ad, Bd = pad(A), pad(B)
+    C = torch.zeros(M, N, device=DEV)
+    G.granii_gemm(M, N, R, Ad, Ad.stride(0), Bd, Bd.stride(0), C, N, G.GEMM_TRANS_A)
+    torch.cuda.synchronize()
+    ref = O.gemm(A, B, ta=True)
+    assert err(C.cpu(), ref) <= TOL
+    assert normwise(C.cpu(), ref) <= 2e-5
+    C2 = torch.zeros(M, N, device=DEV)
+    G.granii_gemm(M, N, R, Ad, Ad.stride(0), Bd, Bd.stride(0), C2, N, G.GEMM_TRANS_A)
+    torch.cuda.synchronize()
+    assert torch.equal(C, C2), "split-K reduction must be deterministic"
+
+
 # ------------------------------------------------------------------ layers
 def run_layer(G, c, model, comp, K1, K2, act, attn=0, seed=50, aligned=True):
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
