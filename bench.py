@@ -115,7 +115,7 @@ def build_model(G, M, spec, g, dev, comm, gen_seed=0):
             ar = synth.glorot(gen_seed + 3, 2 * i + 1, 2 * k2, 1, (k2,), device=dev)
             layers.append(LayerSpec(G.GAT, k1, k2, G.ACT_NONE if last else G.ACT_RELU, G.ATTN_ADDITIVE, W=W,
                                     a_l=al, a_r=ar))
-    return GNN(g, layers, dev, comm)
+    return GNN(g, layers, dev, comm, training=spec["train"])
 
 
 def time_region(fn, steps, stream):
@@ -361,7 +361,7 @@ def main():
 def regret(G, spec, g, dev, comm, H, world, dist):
     """Time every candidate composition of every layer (forward; + backward when
     training) and compare with granii_select's pick (Table VI analog, L411-L427)."""
-    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec, alloc2d
+    from paper_conf_cgo_lenadorasgytm26_b200.model import DEFAULT_CALIB, GNN, LayerSpec, alloc2d
     dims = spec["dims"]
     out = {}
     stream = torch.cuda.current_stream()
@@ -375,8 +375,13 @@ def regret(G, spec, g, dev, comm, H, world, dist):
         ar = synth.uniform_pm1(9, 2 * i + 1, (k2,), device=dev)
         if x.shape[1] != k1:
             x = alloc2d(g.n_rows, k1, dev, fill=0.5)
-        sel, pred = G.granii_select(g, model, k1, k2)
-        sel_all, pred_all = G.granii_select(g, model, k1, k2, flags=G.SELECT_NO_PREFILTER)
+        train = spec["train"] and model == G.GCN
+        need_dH = i > 0                      # the input layer needs no dH (training)
+        fl = (G.SELECT_TRAINING | (0 if need_dH else G.SELECT_INPUT_LAYER)) if train else 0
+        calib = DEFAULT_CALIB if os.path.exists(DEFAULT_CALIB) else None
+        sel, pred = G.granii_select(g, model, k1, k2, calib, fl)
+        sel_all, pred_all = G.granii_select(g, model, k1, k2, calib, fl | G.SELECT_NO_PREFILTER)
+        sel_paper, _ = G.granii_select(g, model, k1, k2, calib, 0)   # forward-only selection, as the paper
         times = {}
         for c in comps:
             net = GNN(g, [LayerSpec(model, k1, k2, G.ACT_RELU, comp=c, W=W, a_l=al, a_r=ar)], dev, comm)
@@ -384,8 +389,8 @@ def regret(G, spec, g, dev, comm, H, world, dist):
 
             def fn():
                 net.forward(x)
-                if spec["train"] and model == G.GCN:
-                    net.backward(gup)
+                if train:
+                    net.backward(gup, need_input_grad=need_dH)
             for _ in range(2):
                 fn()
             t = time_region(fn, 5, stream)
@@ -409,10 +414,12 @@ def regret(G, spec, g, dev, comm, H, world, dist):
             "selected_no_prefilter": G.COMP_NAMES[sel_all],
             "regret": times[G.COMP_NAMES[sel]] / times[best] - 1.0,
             "regret_no_prefilter": times[G.COMP_NAMES[sel_all]] / times[best] - 1.0,
+            "selected_forward_only": G.COMP_NAMES[sel_paper],
+            "regret_forward_only": times[G.COMP_NAMES[sel_paper]] / times[best] - 1.0,
             "config_heuristic_regret": times[cfg] / times[best] - 1.0,
             "static_regret": times[static] / times[best] - 1.0,
             "predicted_ms": {G.COMP_NAMES[k]: v for k, v in pred_all.items()},
-            "mode": "fwd+bwd" if (spec["train"] and model == G.GCN) else "fwd"}
+            "mode": ("fwd+bwd" + ("" if need_dH else " (no dH: input layer)")) if train else "fwd"}
     return out
 
 

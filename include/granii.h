@@ -251,6 +251,10 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
 /* Selector (L237-L258)                                                      */
 /* ------------------------------------------------------------------------ */
 #define GRANII_SELECT_NO_PREFILTER 0x1u /* skip the embedding-size rule (L237-L239)   */
+/* Extension (the paper selects on the forward only, L340): add the backward
+ * primitives of each GCN composition to its cost; INPUT_LAYER drops dH. */
+#define GRANII_SELECT_TRAINING 0x2u
+#define GRANII_SELECT_INPUT_LAYER 0x4u
 #define GRANII_MAX_CANDIDATES 8
 
 /*
@@ -267,6 +271,14 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
 granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t K2, const char* calib_path,
                             uint32_t flags, granii_composition* out, int32_t* candidates,
                             double* predicted_ms, int32_t* n_candidates);
+/* Calibration support: the feature vector the cost model of primitive `prim`
+ * (0 spmm weighted, 1 spmm unweighted, 2 spmm unweighted + column scale,
+ * 3 sddmm K=1, 4 sddmm K=1 + softmax, 5 gemm, 6 gemm without store, 7 gemm Aᵀ·B,
+ * 8 elementwise, 9 all-gather) uses for this graph and widths (K1, K2);
+ * feats has room for 8 values; model_name (32 bytes) receives the model key
+ * the coefficients are stored under in the calibration file. */
+granii_status granii_cost_features(granii_graph g, int32_t prim, int64_t K1, int64_t K2, double* feats,
+                                   int32_t* n, char* model_name);
 
 /* ------------------------------------------------------------------------ */
 /* Multi-GPU (row partition, NCCL over NVLink)                                */

@@ -43,6 +43,7 @@ granii_status layer_backward(const granii_graph_s*, granii_composition, const gr
                              const float*, int64_t, const float*, float*, int64_t, float*, cudaStream_t);
 granii_status select_impl(const granii_graph_s*, granii_model, int64_t, int64_t, const char*, uint32_t,
                           granii_composition*, int32_t*, double*, int32_t*);
+granii_status cost_features_impl(const granii_graph_s*, int32_t, int64_t, int64_t, double*, int32_t*, char*);
 granii_status comm_unique_id(void*);
 granii_status comm_create(const void*, int32_t, int32_t, granii_comm_s**);
 granii_status comm_destroy(granii_comm_s*);
@@ -267,6 +268,12 @@ granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t 
   GR_ARG(K1 > 0 && K2 > 0, "bad embedding sizes");
   return select_impl(g, m, K1, K2, calib_path, flags, out, candidates, predicted_ms, n_candidates);
   API_END
+}
+
+granii_status granii_cost_features(granii_graph g, int32_t prim, int64_t K1, int64_t K2, double* feats, int32_t* n,
+                                   char* model_name) {
+  GR_ARG(g && feats && n, "NULL argument");
+  return cost_features_impl(g, prim, K1, K2, feats, n, model_name);
 }
 
 granii_status granii_comm_unique_id(void* id) {

@@ -315,6 +315,44 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   }
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(st));
+
+  // heavy-row segments (power-law hubs): rows with more than seg_len entries are cut
+  // into seg_len-entry warp-wide work items so a hub cannot set the kernel's tail
+  if (const char* e = getenv("GRANII_SEG")) g->seg_len = std::max<int64_t>(64, atoll(e));
+  if (g->n_rows > 0 && g->features[4] > g->seg_len) {
+    std::vector<int64_t> hrp(g->n_rows + 1);
+    CK(cudaMemcpy(hrp.data(), g->row_ptr, (g->n_rows + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+    int64_t nh = 0;
+    for (int64_t r = 0; r < g->n_rows; ++r) nh += (hrp[r + 1] - hrp[r]) > g->seg_len;
+    if (nh > 0) {
+      std::vector<int32_t> hrows(nh);
+      CK(cudaMemcpy(hrows.data(), g->order, nh * sizeof(int32_t), cudaMemcpyDeviceToHost));  // degree-descending
+      std::vector<int32_t> sptr(nh + 1, 0), sh, sr;
+      std::vector<int64_t> lo, hi;
+      for (int64_t h = 0; h < nh; ++h) {
+        const int64_t r = hrows[h];
+        for (int64_t b = hrp[r]; b < hrp[r + 1]; b += g->seg_len) {
+          lo.push_back(b);
+          hi.push_back(std::min(b + g->seg_len, hrp[r + 1]));
+          sh.push_back((int32_t)h);
+          sr.push_back((int32_t)r);
+        }
+        sptr[h + 1] = (int32_t)lo.size();
+      }
+      g->n_heavy = nh;
+      g->n_seg = (int64_t)lo.size();
+      CK(cudaMalloc(&g->seg_ptr, (nh + 1) * sizeof(int32_t)));
+      CK(cudaMalloc(&g->seg_lo, g->n_seg * sizeof(int64_t)));
+      CK(cudaMalloc(&g->seg_hi, g->n_seg * sizeof(int64_t)));
+      CK(cudaMemcpy(g->seg_ptr, sptr.data(), (nh + 1) * sizeof(int32_t), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(g->seg_lo, lo.data(), g->n_seg * sizeof(int64_t), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(g->seg_hi, hi.data(), g->n_seg * sizeof(int64_t), cudaMemcpyHostToDevice));
+      CK(cudaMalloc(&g->seg_heavy, g->n_seg * sizeof(int32_t)));
+      CK(cudaMalloc(&g->seg_row, g->n_seg * sizeof(int32_t)));
+      CK(cudaMemcpy(g->seg_heavy, sh.data(), g->n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(g->seg_row, sr.data(), g->n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
+    }
+  }
   cleanup();
   CK(cudaStreamSynchronize(st));
 #undef CK
@@ -329,6 +367,11 @@ void graph_free(granii_graph_s* g) {
   cudaFree(g->row_ptr);
   cudaFree(g->col_idx);
   cudaFree(g->order);
+  cudaFree(g->seg_ptr);
+  cudaFree(g->seg_lo);
+  cudaFree(g->seg_hi);
+  cudaFree(g->seg_heavy);
+  cudaFree(g->seg_row);
   delete g;
 }
 

@@ -82,6 +82,15 @@ struct granii_graph_s {
   float* dinv_rows = nullptr;     // device, n_rows
   float* dinv_cols = nullptr;     // device, n_cols (== dinv_rows when world == 1)
   int32_t* order = nullptr;       // device, n_rows: owned rows by descending degree
+  // heavy rows (degree > seg_len) = order[0 .. n_heavy); each is cut into segments of
+  // seg_len entries that are scheduled as independent warp-wide work items
+  int64_t seg_len = 2048;
+  int64_t n_heavy = 0, n_seg = 0;
+  int32_t* seg_ptr = nullptr;     // device, n_heavy+1: segments of heavy row h are [seg_ptr[h], seg_ptr[h+1])
+  int64_t* seg_lo = nullptr;      // device, n_seg: entry range of each segment
+  int64_t* seg_hi = nullptr;
+  int32_t* seg_heavy = nullptr;   // device, n_seg: heavy index h of each segment
+  int32_t* seg_row = nullptr;     // device, n_seg: row of each segment (= order[seg_heavy])
   int64_t features[GRANII_NUM_FEATURES] = {0};
   int device = 0;
   float avg_deg() const { return n_rows > 0 ? float(local_nnz) / float(n_rows) : 0.f; }

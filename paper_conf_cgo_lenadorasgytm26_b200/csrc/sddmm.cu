@@ -33,7 +33,11 @@ struct SddmmArgs {
   int64_t K;
   float scale;
   float* __restrict__ out;
-  const int32_t* __restrict__ order;
+  const int32_t* __restrict__ order;       // light rows (degree-descending), n_rows of them
+  int64_t n_seg;                           // heavy-row segments: warp-wide items
+  const int64_t* __restrict__ seg_lo;
+  const int64_t* __restrict__ seg_hi;
+  const int32_t* __restrict__ seg_row;
 };
 
 template <bool ADD, bool LRELU>
@@ -50,28 +54,58 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  // heavy-row segments: all 32 lanes stride the segment (scores only; the softmax of
+  // heavy rows is the segmented 3-phase pass launched afterwards)
+  for (int64_t t = warp; t < a.n_seg; t += nwarps) {
+    const int64_t row = a.seg_row[t], hi = a.seg_hi[t];
+    const float u = __ldg(a.U + row * a.ldu);
+    int64_t e = a.seg_lo[t] + lane;
+    for (; e + 96 < hi; e += 128) {
+      int32_t c[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) c[q] = __ldg(a.col_idx + e + 32 * q);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) a.out[e + 32 * q] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)c[q] * a.ldv), a.scale);
+    }
+    for (; e < hi; e += 32) a.out[e] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+  }
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     const bool live = t < a.n_rows;
-    const int64_t row = live ? (a.order ? a.order[t] : t) : 0;
+    const int64_t row = live ? a.order[t] : 0;
     const int64_t rs = live ? a.row_ptr[row] : 0, re = live ? a.row_ptr[row + 1] : 0;
     const float u = live ? __ldg(a.U + row * a.ldu) : 0.f;
-    if (!SOFTMAX) {
-      for (int64_t e = rs + lig; e < re; e += LPG)
-        a.out[e] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
-      continue;
-    }
-    // online max / sum over this lane's entries
+    // pass 1: scores (4 independent col -> V gathers in flight per lane), written to out;
+    // with SOFTMAX also the online (max, sum) of this lane's entries
+    constexpr int U4 = 4;
     float m = -INFINITY, s = 0.f;
-    for (int64_t e = rs + lig; e < re; e += LPG) {
-      const float x = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
-      if (x > m) {
-        s = s * expf(m - x) + 1.f;
-        m = x;
-      } else {
-        s += expf(x - m);
+    int64_t e = rs + lig;
+    for (; e + (U4 - 1) * LPG < re; e += U4 * LPG) {
+      int32_t c[U4];
+      float x[U4];
+#pragma unroll
+      for (int q = 0; q < U4; ++q) c[q] = __ldg(a.col_idx + e + q * LPG);
+#pragma unroll
+      for (int q = 0; q < U4; ++q) x[q] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)c[q] * a.ldv), a.scale);
+#pragma unroll
+      for (int q = 0; q < U4; ++q) a.out[e + q * LPG] = x[q];
+      if (SOFTMAX) {
+        const float mn = fmaxf(fmaxf(m, fmaxf(x[0], x[1])), fmaxf(x[2], x[3]));
+        s = (m == -INFINITY ? 0.f : s * expf(m - mn)) + expf(x[0] - mn) + expf(x[1] - mn) + expf(x[2] - mn) +
+            expf(x[3] - mn);
+        m = mn;
       }
     }
+    for (; e < re; e += LPG) {
+      const float x = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+      a.out[e] = x;
+      if (SOFTMAX) {
+        const float mn = fmaxf(m, x);
+        s = (m == -INFINITY ? 0.f : s * expf(m - mn)) + expf(x - mn);
+        m = mn;
+      }
+    }
+    if (!SOFTMAX) continue;
     // combine within the group (xor butterfly, fixed order)
 #pragma unroll
     for (int off = LPG / 2; off > 0; off >>= 1) {
@@ -83,10 +117,9 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
       s = a1 + a2;
     }
     const float inv = 1.f / s;
-    for (int64_t e = rs + lig; e < re; e += LPG) {
-      const float x = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
-      a.out[e] = expf(x - m) * inv;
-    }
+    // pass 2: normalise the stored scores in place (a coalesced 8 B/entry stream; each
+    // lane re-reads exactly the entries it wrote, so no synchronisation is needed)
+    for (int64_t e2 = rs + lig; e2 < re; e2 += LPG) a.out[e2] = expf(a.out[e2] - m) * inv;
   }
 }
 
@@ -97,9 +130,10 @@ __global__ void __launch_bounds__(256) k_sddmm_dot(SddmmArgs a) {
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t t = warp; t < a.n_rows; t += nwarps) {
-    const int64_t row = a.order ? a.order[t] : t;
-    const int64_t rs = a.row_ptr[row], re = a.row_ptr[row + 1];
+  for (int64_t t = warp; t < a.n_seg + a.n_rows; t += nwarps) {  // heavy segments first, then light rows
+    const bool seg = t < a.n_seg;
+    const int64_t row = seg ? a.seg_row[t] : a.order[t - a.n_seg];
+    const int64_t rs = seg ? a.seg_lo[t] : a.row_ptr[row], re = seg ? a.seg_hi[t] : a.row_ptr[row + 1];
     float u[NJ][VEC];
 #pragma unroll
     for (int j = 0; j < NJ; ++j)
@@ -138,15 +172,15 @@ __global__ void __launch_bounds__(256) k_sddmm_dot(SddmmArgs a) {
 
 // row softmax in place over CSR values (used after the K > 1 dot SDDMM)
 template <int LPG>
-__global__ void __launch_bounds__(256) k_row_softmax(int64_t n_rows, const int64_t* __restrict__ row_ptr,
-                                                     float* __restrict__ x) {
+__global__ void __launch_bounds__(256) k_row_softmax(int64_t n_rows, const int32_t* __restrict__ order,
+                                                     const int64_t* __restrict__ row_ptr, float* __restrict__ x) {
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t t0 = warp * G; t0 < n_rows; t0 += nwarps * G) {
-    const int64_t row = t0 + grp;
-    const bool live = row < n_rows;
+    const bool live = t0 + grp < n_rows;
+    const int64_t row = live ? order[t0 + grp] : 0;
     const int64_t rs = live ? row_ptr[row] : 0, re = live ? row_ptr[row + 1] : 0;
     float m = -INFINITY, s = 0.f;
     for (int64_t e = rs + lig; e < re; e += LPG) {
@@ -165,6 +199,68 @@ __global__ void __launch_bounds__(256) k_row_softmax(int64_t n_rows, const int64
     const float inv = 1.f / s;
     for (int64_t e = rs + lig; e < re; e += LPG) x[e] = expf(x[e] - m) * inv;
   }
+}
+
+// ---------------------------------------------------------------- segmented softmax of heavy rows
+__device__ __forceinline__ void ms_combine(float& m, float& s, float m2, float s2) {
+  const float mn = fmaxf(m, m2);
+  const float a1 = (m == -INFINITY) ? 0.f : s * expf(m - mn);
+  const float a2 = (m2 == -INFINITY) ? 0.f : s2 * expf(m2 - mn);
+  m = mn;
+  s = a1 + a2;
+}
+
+// phase 1: (max, sum exp) of each segment's scores (warp per segment, fixed lane order)
+__global__ void k_seg_stats(int64_t n_seg, const int64_t* __restrict__ lo, const int64_t* __restrict__ hi,
+                            const float* __restrict__ x, float2* __restrict__ ms) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t < n_seg; t += nwarps) {
+    float m = -INFINITY, s = 0.f;
+    for (int64_t e = lo[t] + lane; e < hi[t]; e += 32) ms_combine(m, s, x[e], 1.f);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1)
+      ms_combine(m, s, __shfl_xor_sync(0xffffffffu, m, off), __shfl_xor_sync(0xffffffffu, s, off));
+    if (lane == 0) ms[t] = make_float2(m, s);
+  }
+}
+
+// phase 2: combine the segments of each heavy row in order
+__global__ void k_heavy_stats(int64_t n_heavy, const int32_t* __restrict__ seg_ptr, const float2* __restrict__ ms,
+                              float2* __restrict__ hms) {
+  for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_heavy; h += (int64_t)gridDim.x * blockDim.x) {
+    float m = -INFINITY, s = 0.f;
+    for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) ms_combine(m, s, ms[q].x, ms[q].y);
+    hms[h] = make_float2(m, 1.f / s);
+  }
+}
+
+// phase 3: alpha = exp(e - m_row) / sum_row
+__global__ void k_seg_norm(int64_t n_seg, const int64_t* __restrict__ lo, const int64_t* __restrict__ hi,
+                           const int32_t* __restrict__ seg_heavy, const float2* __restrict__ hms, float* __restrict__ x) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t < n_seg; t += nwarps) {
+    const float2 r = hms[seg_heavy[t]];
+    for (int64_t e = lo[t] + lane; e < hi[t]; e += 32) x[e] = expf(x[e] - r.x) * r.y;
+  }
+}
+
+static granii_status heavy_softmax(const granii_graph_s* g, float* out, int sms, cudaStream_t st) {
+  if (g->n_seg == 0) return GRANII_OK;
+  float2 *ms = nullptr, *hms = nullptr;
+  GR_CUDA(cudaMallocAsync((void**)&ms, g->n_seg * sizeof(float2), st));
+  GR_CUDA(cudaMallocAsync((void**)&hms, g->n_heavy * sizeof(float2), st));
+  const unsigned bw = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(g->n_seg, 8), (int64_t)sms * 8));
+  k_seg_stats<<<bw, 256, 0, st>>>(g->n_seg, g->seg_lo, g->seg_hi, out, ms);
+  k_heavy_stats<<<(unsigned)ceil_div(g->n_heavy, 256), 256, 0, st>>>(g->n_heavy, g->seg_ptr, ms, hms);
+  k_seg_norm<<<bw, 256, 0, st>>>(g->n_seg, g->seg_lo, g->seg_hi, g->seg_heavy, hms, out);
+  GR_CHECK_LAUNCH();
+  GR_CUDA(cudaFreeAsync(ms, st));
+  GR_CUDA(cudaFreeAsync(hms, st));
+  return GRANII_OK;
 }
 
 static int lpg_for_degree(float avg) {
@@ -196,14 +292,16 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   GR_TRY(dev_info(&di));
   const uint32_t base = op & 0xF;
   const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
-  SddmmArgs a{g->n_rows, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order};
+  const int64_t n_light = g->n_rows - g->n_heavy;
+  SddmmArgs a{n_light, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order + g->n_heavy,
+              g->n_seg, g->seg_lo, g->seg_hi, g->seg_row};
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   ProfScope ps("sddmm", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K,
                (K > 1 && sm) ? 2 : 1);
   if (K == 1) {
     const int lpg = lpg_for_degree(g->avg_deg());
-    const int64_t units = ceil_div(g->n_rows, 32 / lpg);
+    const int64_t units = ceil_div(n_light, 32 / lpg) + g->n_seg;
     const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, 8), (int64_t)di.sms * 8));
     const bool add = base == GRANII_SDDMM_ADD;
     // dispatch the 8 (add, lrelu, softmax) variants
@@ -215,12 +313,13 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
       else { if (sm) go1_lpg<false, false, true>(lpg, a, blocks, st); else go1_lpg<false, false, false>(lpg, a, blocks, st); }
     }
     GR_CHECK_LAUNCH();
+    if (sm) GR_TRY(heavy_softmax(g, out, di.sms, st));
     return GRANII_OK;
   }
   if (base != GRANII_SDDMM_DOT) return fail(GRANII_ERR_INVALID_ARG, "SDDMM ADD requires K == 1");
   if (lr) return fail(GRANII_ERR_UNSUPPORTED, "LEAKYRELU with K > 1 is not supported");
   const bool vec4 = (ldu % 4 == 0) && (ldv % 4 == 0) && ((uintptr_t)V % 16 == 0);
-  const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(g->n_rows, 8), (int64_t)di.sms * 8));
+  const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n_light + g->n_seg, 8), (int64_t)di.sms * 8));
 #define GO(VEC, LPG, NJ) k_sddmm_dot<VEC, LPG, NJ><<<blocks, 256, 0, st>>>(a)
   if (vec4) {
     if (K <= 16) GO(4, 4, 1);
@@ -243,15 +342,16 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   GR_CHECK_LAUNCH();
   if (sm) {
     const int lpg = lpg_for_degree(g->avg_deg());
-    const int64_t units = ceil_div(g->n_rows, 32 / lpg);
+    const int64_t units = ceil_div(n_light, 32 / lpg);
     const int b2 = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, 8), (int64_t)di.sms * 8));
     switch (lpg) {
-      case 32: k_row_softmax<32><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
-      case 16: k_row_softmax<16><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
-      case 8: k_row_softmax<8><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
-      default: k_row_softmax<4><<<b2, 256, 0, st>>>(g->n_rows, g->row_ptr, out); break;
+      case 32: k_row_softmax<32><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      case 16: k_row_softmax<16><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      case 8: k_row_softmax<8><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      default: k_row_softmax<4><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
     }
     GR_CHECK_LAUNCH();
+    GR_TRY(heavy_softmax(g, out, di.sms, st));
   }
   return GRANII_OK;
 }

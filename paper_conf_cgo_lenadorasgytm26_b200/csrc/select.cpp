@@ -9,11 +9,14 @@
 // 3. Per-primitive cost models (L252-L258).  The paper trains XGBoost models
 //    on profiled SuiteSparse graphs; here each primitive has a small linear
 //    model over hardware-meaningful features of the featurized input (bytes
-//    streamed, bytes gathered from L2 vs HBM, flops, launches), with
+//    streamed, bytes gathered from L2 vs HBM, tensor flops, launches), with
 //    coefficients fitted by NNLS on a B200 calibration sweep
-//    (tools/calibrate.py) and built-in defaults derived from B200 peaks.
-//    Features come from the integer featurizer computed at graph creation,
-//    so selection is host-only and takes microseconds (paper: <= 7 ms, L365).
+//    (tools/calibrate.py -> calib/b200.txt) and built-in defaults.  Features
+//    come from the integer featurizer computed at graph creation, so selection
+//    is host-only and takes microseconds (paper: <= 7 ms, L365).
+// Extension (not in the paper, which selects on the forward only, L340):
+// GRANII_SELECT_TRAINING adds each composition's backward primitives, and
+// GRANII_SELECT_INPUT_LAYER drops the dH branch (not needed for layer 1).
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -26,21 +29,26 @@
 
 namespace granii {
 
-// coefficient vectors (ms per unit); feature order documented in features_*()
 struct CostModel {
   std::map<std::string, std::vector<double>> coef;
 };
 
+// feature vectors (all sizes in GB / TFLOP, time in ms)
+//   spmm            : [1, streamed GB (idx, weights, col-scale gather), out GB, gathered GB from L2, gathered GB from HBM]
+//   sddmm1          : [1, streamed GB]
+//   sddmm1_softmax  : [1, streamed GB]
+//   gemm            : [1, HBM GB, TFLOP]
+//   gemm_tn         : [1, HBM GB, TFLOP]
+//   elementwise     : [1, GB]
+//   allgather       : [1, GB received per GPU]
 static CostModel defaults() {
   CostModel m;
-  // spmm: [launch, idx GB, out GB, gathered GB served by L2, gathered GB served by HBM]
-  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 14.0, 1.0 / 4.5};
-  // sddmm1 (Ñ or GAT scores; K = 1): [launch, streamed GB]
+  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0};
   m.coef["sddmm1"] = {0.005, 1.0 / 5.5};
-  m.coef["sddmm1_softmax"] = {0.006, 1.0 / 5.0};
-  // gemm (3xTF32 tcgen05): [launch, HBM GB, TFLOP]
-  m.coef["gemm"] = {0.010, 1.0 / 6.0, 1.0 / 250.0};
-  // all-gather over NVLink: [launch, GB received per GPU]
+  m.coef["sddmm1_softmax"] = {0.006, 1.0 / 4.0};
+  m.coef["gemm"] = {0.010, 1.0 / 2.0, 1.0 / 250.0};
+  m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 250.0};
+  m.coef["elementwise"] = {0.004, 1.0 / 5.5};
   m.coef["allgather"] = {0.020, 1.0 / 700.0};
   return m;
 }
@@ -83,66 +91,117 @@ static granii_status load_model(const char* path, CostModel* out) {
   return GRANII_OK;
 }
 
-static double dot(const std::vector<double>& c, std::initializer_list<double> f) {
-  double s = 0;
-  size_t i = 0;
-  for (double x : f) s += c[i++] * x;
-  return s;
-}
-
 struct In {
   double R, nnz, ncols, avg, l2, world;
 };
 
-// fraction of gathered bytes served by L2: sliced SpMM keeps the
-// slice resident when the graph is dense; otherwise LRU-like hit ~ L2 / |X|.
+// fraction of gathered bytes served by L2: the sliced SpMM keeps
+// a slice resident when the graph is dense; otherwise LRU-like hit ~ L2 / |X|.
 static double l2_hit(const In& in, double K) {
   const double xbytes = in.ncols * K * 4.0;
   if (xbytes <= 0.8 * in.l2) return 1.0;
-  if (in.avg >= 32.0) return 1.0;  // K-sliced
+  if (in.avg >= 32.0 && in.ncols * 64.0 * 4.0 <= 0.55 * in.l2) return 1.0;  // K-sliced
   return std::max(0.0, std::min(1.0, 0.8 * in.l2 / xbytes));
 }
 
-double cost_spmm(const CostModel& m, const In& in, double K, bool weighted) {
-  const double gb = 1e-9;
-  const double gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
-  return dot(m.coef.at("spmm"), {1.0, in.nnz * (weighted ? 8.0 : 4.0) * gb, in.R * K * 4.0 * gb, gath * h,
-                                 gath * (1.0 - h)});
-}
-double cost_sddmm1(const CostModel& m, const In& in, bool softmax) {
-  const double gb = 1e-9;
-  if (softmax) return dot(m.coef.at("sddmm1_softmax"), {1.0, in.nnz * 12.0 * gb});
-  return dot(m.coef.at("sddmm1"), {1.0, in.nnz * 8.0 * gb});
-}
-double cost_gemm(const CostModel& m, const In& in, double K1, double K2, bool store) {
-  const double gb = 1e-9;
-  return dot(m.coef.at("gemm"), {1.0, in.R * (K1 + (store ? K2 : 0.0)) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12});
-}
-double cost_allgather(const CostModel& m, const In& in, double K) {
-  if (in.world <= 1) return 0.0;
-  return dot(m.coef.at("allgather"), {1.0, in.ncols * K * 4.0 * (in.world - 1) / in.world * 1e-9});
+// primitive ids of the feature API
+enum { P_SPMM_W = 0, P_SPMM_U = 1, P_SPMM_U_CS = 2, P_SDDMM1 = 3, P_SDDMM1_SM = 4, P_GEMM = 5, P_GEMM_NOSTORE = 6,
+       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9 };
+
+static const char* prim_model(int p) {
+  switch (p) {
+    case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: return "spmm";
+    case P_SDDMM1: return "sddmm1";
+    case P_SDDMM1_SM: return "sddmm1_softmax";
+    case P_GEMM: case P_GEMM_NOSTORE: return "gemm";
+    case P_GEMM_TN: return "gemm_tn";
+    case P_ELEMENTWISE: return "elementwise";
+    case P_ALLGATHER: return "allgather";
+  }
+  return "";
 }
 
-double composition_cost(const CostModel& m, const In& in, int comp, double K1, double K2) {
+// K = width of the primitive (SpMM/SDDMM) or (K1, K2) for the GEMMs
+static std::vector<double> features(const In& in, int p, double K1, double K2) {
+  const double gb = 1e-9;
+  switch (p) {
+    case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: {
+      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
+      const double idx = in.nnz * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 4.0 : 0.0)) * gb;
+      return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h)};
+    }
+    case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb};
+    case P_SDDMM1_SM: return {1.0, in.nnz * 16.0 * gb};
+    case P_GEMM: return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
+    case P_GEMM_NOSTORE: return {1.0, in.R * K1 * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
+    case P_GEMM_TN: return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
+    case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
+    case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};
+  }
+  return {};
+}
+
+static double cost(const CostModel& m, const In& in, int p, double K1, double K2 = 0) {
+  if (p == P_ALLGATHER && in.world <= 1) return 0.0;
+  const std::vector<double> f = features(in, p, K1, K2);
+  const std::vector<double>& c = m.coef.at(prim_model(p));
+  double s = 0;
+  for (size_t i = 0; i < f.size() && i < c.size(); ++i) s += c[i] * f[i];
+  return s;
+}
+
+double forward_cost(const CostModel& m, const In& in, int comp, double K1, double K2) {
   switch (comp) {
     case GRANII_GCN_PRE_AGG:
-      return cost_sddmm1(m, in, false) + cost_allgather(m, in, K1) + cost_spmm(m, in, K1, true) +
-             cost_gemm(m, in, K1, K2, true);
+      return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_W, K1) +
+             cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_PRE_UPD:
-      return cost_sddmm1(m, in, false) + cost_gemm(m, in, K1, K2, true) + cost_allgather(m, in, K2) +
-             cost_spmm(m, in, K2, true);
+      return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) +
+             cost(m, in, P_SPMM_W, K2);
     case GRANII_GCN_DYN_AGG:
-      return cost_allgather(m, in, K1) + cost_spmm(m, in, K1, false) + cost_gemm(m, in, K1, K2, true);
+      return cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_DYN_UPD:
-      return cost_gemm(m, in, K1, K2, true) + cost_allgather(m, in, K2) + cost_spmm(m, in, K2, false);
+      return cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);
     case GRANII_GAT_REUSE:
-      return cost_gemm(m, in, K1, K2, true) + cost_allgather(m, in, K2) + cost_sddmm1(m, in, true) +
-             cost_spmm(m, in, K2, true);
+      return cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SDDMM1_SM, 0) +
+             cost(m, in, P_SPMM_W, K2);
     case GRANII_GAT_RECOMP:
-      return cost_gemm(m, in, K1, K2, false) + cost_allgather(m, in, K1) + cost_sddmm1(m, in, true) +
-             cost_spmm(m, in, K1, true) + cost_gemm(m, in, K1, K2, true);
+      return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SDDMM1_SM, 0) +
+             cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
   }
   return 1e30;
+}
+
+// backward of the GCN compositions (layer.cu backward_impl), ReLU mask included
+double backward_cost(const CostModel& m, const In& in, int comp, double K1, double K2, bool need_dH) {
+  double t = cost(m, in, P_ELEMENTWISE, K2) + cost(m, in, P_GEMM_TN, K1, K2);
+  switch (comp) {
+    case GRANII_GCN_PRE_AGG:
+      t += cost(m, in, P_SDDMM1, 0);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_W, K1);
+      break;
+    case GRANII_GCN_PRE_UPD:
+      t += cost(m, in, P_SDDMM1, 0) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_W, K2);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
+      break;
+    case GRANII_GCN_DYN_AGG:
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U, K1);
+      break;
+    case GRANII_GCN_DYN_UPD:
+      t += cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U_CS, K2);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
+      break;
+    default:
+      return 0.0;
+  }
+  return t;
+}
+
+static In inputs_of(const granii_graph_s* g) {
+  DevInfo di;
+  if (dev_info(&di) != GRANII_OK) di = DevInfo();  // host-only selection still works
+  return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
+            (double)g->world};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K1, int64_t K2, const char* path,
@@ -150,10 +209,7 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
   if (!path || !*path) path = getenv("GRANII_CALIB");
   CostModel m;
   GR_TRY(load_model(path, &m));
-  DevInfo di;
-  if (dev_info(&di) != GRANII_OK) di = DevInfo();  // host-only selection still works
-  In in{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-        (double)g->world};
+  const In in = inputs_of(g);
   std::vector<int> c;
   if (model == GRANII_GCN) {
     if (flags & GRANII_SELECT_NO_PREFILTER) c = {GRANII_GCN_PRE_AGG, GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_AGG, GRANII_GCN_DYN_UPD};
@@ -162,10 +218,13 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
   } else {
     c = {GRANII_GAT_REUSE, GRANII_GAT_RECOMP};
   }
+  const bool train = (flags & GRANII_SELECT_TRAINING) && model == GRANII_GCN;
+  const bool need_dH = !(flags & GRANII_SELECT_INPUT_LAYER);
   int best = -1;
   double bc = 0;
   for (size_t i = 0; i < c.size(); ++i) {
-    const double t = composition_cost(m, in, c[i], (double)K1, (double)K2);
+    double t = forward_cost(m, in, c[i], (double)K1, (double)K2);
+    if (train) t += backward_cost(m, in, c[i], (double)K1, (double)K2, need_dH);
     if (cands) cands[i] = c[i];
     if (pred) pred[i] = t;
     if (best < 0 || t < bc) {  // strict: ties keep the lower id (candidates are in id order)
@@ -175,6 +234,19 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
   }
   if (ncand) *ncand = (int32_t)c.size();
   *out = (granii_composition)best;
+  return GRANII_OK;
+}
+
+granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t K1, int64_t K2, double* feats,
+                                 int32_t* n, char* model_name) {
+  if (prim < P_SPMM_W || prim > P_ALLGATHER) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
+  const std::vector<double> f = features(inputs_of(g), prim, (double)K1, (double)K2);
+  for (size_t i = 0; i < f.size(); ++i) feats[i] = f[i];
+  *n = (int32_t)f.size();
+  if (model_name) {
+    strncpy(model_name, prim_model(prim), 31);
+    model_name[31] = 0;
+  }
   return GRANII_OK;
 }
 

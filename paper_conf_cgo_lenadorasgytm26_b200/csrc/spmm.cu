@@ -51,7 +51,7 @@ __device__ __forceinline__ void stv(float* p, const float (&v)[VEC]) {
 }
 
 struct SpmmArgs {
-  int64_t n_rows;
+  int64_t n_rows;                          // light rows (scheduled through `order`)
   const int64_t* __restrict__ row_ptr;
   const int32_t* __restrict__ col_idx;
   const float* __restrict__ vals;
@@ -63,111 +63,165 @@ struct SpmmArgs {
   const float* __restrict__ rs;
   const float* __restrict__ cs;
   int relu;
-  const int32_t* __restrict__ order;
+  const int32_t* __restrict__ order;       // light rows, degree-descending
+  // heavy rows (degree > GRANII_SEG) are cut into segments: warp-wide work items whose
+  // unscaled partial sums go to `partial` [n_seg][ldp] and are combined in fixed order
+  int64_t n_seg;
+  const int64_t* __restrict__ seg_lo;
+  const int64_t* __restrict__ seg_hi;
+  float* __restrict__ partial;
+  int64_t ldp;
 };
 
-// ------------------------------------------------------------------ warp-per-row
 // One chunk of 32 entries of a row, one per lane: column id and weight.  Lanes
-// past the row's end reuse the row's last column with w = 0, so every later
-// step is branch-free (the padded gathers hit L1 and add exact zeros).
-template <bool W, bool CS>
+// past the range's end reuse its last column with w = 0, so every later step is
+// branch-free (the padded gathers hit L1 and add exact zeros).
+template <bool W>
 __device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t re, int lane, int32_t& c, float& w) {
   const bool valid = e + lane < re;
   const int64_t ee = valid ? e + lane : re - 1;
   c = __ldg(a.col_idx + ee);
   w = valid ? (W ? __ldg(a.vals + ee) : 1.f) : 0.f;
-  if (CS) w *= __ldg(a.cs + c);
 }
 
-template <int VEC, int LPG, int NJ, bool W, bool CS>
-__global__ void __launch_bounds__(256, 3) k_spmm_warp(SpmmArgs a) {
+// The whole warp accumulates entries [rs0, re): G = 32/LPG lane groups each take a
+// neighbour, U neighbours per group in flight; acc holds this lane's group partial.
+template <int VEC, int LPG, int NJ, bool W, bool CS, int U>
+__device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64_t re, int lane, int grp,
+                                           const char* const (&xbj)[NJ], uint32_t row_bytes, float (&acc)[NJ][VEC]) {
   constexpr int G = 32 / LPG;
-  constexpr int U = 32 / G >= 4 ? 4 : 32 / G;  // neighbours per group per step; G*U divides 32
-  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  bool colok[NJ];
-  uint32_t coff[NJ];  // byte offset of this lane's j-th vector inside the slice
-  const int last = (int)((a.kw - 1) / VEC);  // last vector that holds a column of the slice
+  if (rs0 >= re) return;
+  // distance-2 prefetch: (c0, w0, cs0) = next chunk, (c1, w1) = the chunk after; the
+  // dependent col-scale gather cs[c] of a chunk is issued one chunk before its use
+  int32_t c0, c1 = 0;
+  float w0, w1 = 0.f, cs0 = 1.f;
+  load_chunk<W>(a, rs0, re, lane, c0, w0);
+  if (CS) cs0 = __ldg(a.cs + c0);
+  if (rs0 + 32 < re) load_chunk<W>(a, rs0 + 32, re, lane, c1, w1);
+  for (int64_t base = rs0; base < re; base += 32) {
+    const int32_t c = c0;
+    const float w = CS ? w0 * cs0 : w0;
+    if (base + 32 < re) {
+      c0 = c1;
+      w0 = w1;
+      if (CS) cs0 = __ldg(a.cs + c0);                                      // c1 landed a chunk ago
+      if (base + 64 < re) load_chunk<W>(a, base + 64, re, lane, c1, w1);  // two chunks ahead
+    }
+    const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
+    const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
+    for (int s = 0; s < steps; ++s) {
+      uint32_t cu[U];
+      float wu[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int i = s * G * U + u * G + grp;  // <= 31
+        cu[u] = (uint32_t)__shfl_sync(0xffffffffu, c, i);
+        wu[u] = __shfl_sync(0xffffffffu, w, i);
+      }
+      float x[U][NJ][VEC];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
+    }
+  }
+}
+
+// per-lane column offsets of a slice: lanes past it re-read its last in-bounds
+// vector (ldx >= k0 + kw rounded to VEC), so gathers are unconditional; never stored
+template <int VEC, int LPG, int NJ>
+__device__ __forceinline__ void slice_setup(const SpmmArgs& a, int lig, bool (&colok)[NJ], const char* (&xbj)[NJ]) {
+  const int last = (int)((a.kw - 1) / VEC);
+  const char* __restrict__ xb = reinterpret_cast<const char*>(a.X + a.k0);
 #pragma unroll
   for (int j = 0; j < NJ; ++j) {
     const int v = lig + j * LPG;
     colok[j] = v <= last;
-    // lanes past the slice re-read its last vector (in bounds: ldx >= k0 + kw, rounded to VEC)
-    // so loads are unconditional; their sums are never stored
-    coff[j] = (uint32_t)((v <= last ? v : last) * VEC * 4);
+    xbj[j] = xb + (uint32_t)((v <= last ? v : last) * VEC * 4);  // one 64-bit base per vector
   }
-  // per-lane base of the column slice; row offset = c * row_bytes in one IMAD.WIDE.U32
-  const char* __restrict__ xb = reinterpret_cast<const char*>(a.X + a.k0);
-  const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
-  const char* xbj[NJ];  // one 64-bit base per vector: each gather address is a single IMAD.WIDE.U32
+}
+
+template <int NJ, int VEC>
+__device__ __forceinline__ void zero(float (&acc)[NJ][VEC]) {
 #pragma unroll
-  for (int j = 0; j < NJ; ++j) xbj[j] = xb + coff[j];
-  for (int64_t t = warp; t < a.n_rows; t += nwarps) {
-    const int64_t row = a.order ? a.order[t] : t;
-    const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
-    float acc[NJ][VEC];
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
+}
+
+// sum the G lane groups (fixed butterfly order)
+template <int LPG, int NJ, int VEC>
+__device__ __forceinline__ void reduce_groups(float (&acc)[NJ][VEC]) {
+#pragma unroll
+  for (int off = LPG; off < 32; off <<= 1)
 #pragma unroll
     for (int j = 0; j < NJ; ++j)
 #pragma unroll
-      for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
-    if (rs0 < re) {
-      int32_t cn;
-      float wn;
-      load_chunk<W, CS>(a, rs0, re, lane, cn, wn);
-      for (int64_t base = rs0; base < re; base += 32) {
-        const int32_t c = cn;
-        const float w = wn;
-        if (base + 32 < re) load_chunk<W, CS>(a, base + 32, re, lane, cn, wn);  // prefetch next chunk
-        const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
-        const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
-        for (int s = 0; s < steps; ++s) {
-          uint32_t cu[U];
-          float wu[U];
+      for (int v = 0; v < VEC; ++v) acc[j][v] += __shfl_xor_sync(0xffffffffu, acc[j][v], off);
+}
+
+template <int LPG, int NJ, int VEC>
+__device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], const float (&acc)[NJ][VEC], float s,
+                                          int relu) {
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const int i = s * G * U + u * G + grp;  // <= 31
-            cu[u] = (uint32_t)__shfl_sync(0xffffffffu, c, i);
-            wu[u] = __shfl_sync(0xffffffffu, w, i);
-          }
-          float x[U][NJ][VEC];
+  for (int j = 0; j < NJ; ++j) {
+    if (!colok[j]) continue;
+    float o[VEC];
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-#pragma unroll
-            for (int j = 0; j < NJ; ++j)
-              ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
-          }
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-#pragma unroll
-            for (int j = 0; j < NJ; ++j)
-#pragma unroll
-              for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
-        }
-      }
+    for (int v = 0; v < VEC; ++v) {
+      o[v] = acc[j][v] * s;
+      if (relu) o[v] = fmaxf(o[v], 0.f);
     }
-    // reduce the G groups (fixed butterfly order)
-#pragma unroll
-    for (int off = LPG; off < 32; off <<= 1)
-#pragma unroll
-      for (int j = 0; j < NJ; ++j)
-#pragma unroll
-        for (int v = 0; v < VEC; ++v) acc[j][v] += __shfl_xor_sync(0xffffffffu, acc[j][v], off);
-    if (grp == 0) {
-      const float s = a.rs ? __ldg(a.rs + row) : 1.f;
-      float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
-#pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        if (!colok[j]) continue;
-        float o[VEC];
-#pragma unroll
-        for (int v = 0; v < VEC; ++v) {
-          o[v] = acc[j][v] * s;
-          if (a.relu) o[v] = fmaxf(o[v], 0.f);
-        }
-        stv<VEC>(y + j * LPG * VEC, o);
-      }
+    stv<VEC>(y + j * LPG * VEC, o);
+  }
+}
+
+// heavy-row segments first (largest work first), as warp-wide items
+template <int VEC, int LPG, int NJ, bool W, bool CS, int U>
+__device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lane, int grp, int lig,
+                                           const bool (&colok)[NJ], const char* const (&xbj)[NJ],
+                                           uint32_t row_bytes) {
+  float acc[NJ][VEC];
+  zero(acc);
+  warp_range<VEC, LPG, NJ, W, CS, U>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc);
+  reduce_groups<LPG>(acc);
+  if (grp == 0) store_row<LPG>(a.partial + t * a.ldp + (int64_t)lig * VEC, colok, acc, 1.f, 0);
+}
+
+// ------------------------------------------------------------------ warp-per-row
+template <int VEC, int LPG, int NJ, bool W, bool CS, int UU = 0, int MINB = 3>
+__global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
+  constexpr int G = 32 / LPG;
+  constexpr int U = UU > 0 ? UU : (32 / G >= 4 ? 4 : 32 / G);  // neighbours per group per step; G*U divides 32
+  static_assert(32 % (G * U) == 0, "G*U must divide 32");
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  bool colok[NJ];
+  const char* xbj[NJ];
+  slice_setup<VEC, LPG>(a, lig, colok, xbj);
+  const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
+  for (int64_t t = warp; t < a.n_seg + a.n_rows; t += nwarps) {
+    if (t < a.n_seg) {
+      do_segment<VEC, LPG, NJ, W, CS, U>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+      continue;
     }
+    const int64_t row = a.order[t - a.n_seg];
+    float acc[NJ][VEC];
+    zero(acc);
+    warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
+    reduce_groups<LPG>(acc);
+    if (grp == 0)
+      store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
+                     a.relu);
   }
 }
 
@@ -175,34 +229,25 @@ __global__ void __launch_bounds__(256, 3) k_spmm_warp(SpmmArgs a) {
 template <int VEC, int LPG, int NJ, bool W, bool CS>
 __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   constexpr int G = 32 / LPG;
+  constexpr int U = 4;
+  constexpr int UW = 32 / G >= 4 ? 4 : 32 / G;
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   bool colok[NJ];
-  uint32_t coff[NJ];
-  const int last = (int)((a.kw - 1) / VEC);
-#pragma unroll
-  for (int j = 0; j < NJ; ++j) {
-    const int v = lig + j * LPG;
-    colok[j] = v <= last;
-    coff[j] = (uint32_t)((v <= last ? v : last) * VEC * 4);  // clamped: unconditional loads
-  }
-  const char* __restrict__ xb = reinterpret_cast<const char*>(a.X + a.k0);
+  const char* xbj[NJ];
+  slice_setup<VEC, LPG>(a, lig, colok, xbj);
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
-  const char* xbj[NJ];  // one 64-bit base per vector: each gather address is a single IMAD.WIDE.U32
-#pragma unroll
-  for (int j = 0; j < NJ; ++j) xbj[j] = xb + coff[j];
-  constexpr int U = 4;
+  for (int64_t t = warp; t < a.n_seg; t += nwarps)  // heavy segments: whole warps
+    do_segment<VEC, LPG, NJ, W, CS, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+  // light rows: one LPG-lane group per row
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
-    const int64_t row = a.order ? a.order[t] : t;
+    const int64_t row = a.order[t];
     const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
     float acc[NJ][VEC];
-#pragma unroll
-    for (int j = 0; j < NJ; ++j)
-#pragma unroll
-      for (int v = 0; v < VEC; ++v) acc[j][v] = 0.f;
+    zero(acc);
     for (int64_t e = rs0; e < re; e += U) {
       uint32_t cu[U];
       float wu[U];
@@ -228,19 +273,25 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
 #pragma unroll
           for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
     }
-    const float s = a.rs ? __ldg(a.rs + row) : 1.f;
-    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
-#pragma unroll
-    for (int j = 0; j < NJ; ++j) {
-      if (!colok[j]) continue;
-      float o[VEC];
-#pragma unroll
-      for (int v = 0; v < VEC; ++v) {
-        o[v] = acc[j][v] * s;
-        if (a.relu) o[v] = fmaxf(o[v], 0.f);
-      }
-      stv<VEC>(y + j * LPG * VEC, o);
-    }
+    store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
+                   a.relu);
+  }
+}
+
+// heavy rows: Y_r = rs_r * sum_{segments of r, in order} partial (+ ReLU)
+__global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heavy_rows,
+                               const int32_t* __restrict__ seg_ptr, const float* __restrict__ partial, int64_t ldp,
+                               int64_t k0, int64_t kw, float* __restrict__ Y, int64_t ldy,
+                               const float* __restrict__ rs, int relu) {
+  const int64_t total = n_heavy * kw;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t h = i / kw, k = i % kw;
+    float s = 0.f;
+    for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) s += partial[(int64_t)q * ldp + k];
+    const int64_t row = heavy_rows[h];
+    s *= rs ? rs[row] : 1.f;
+    if (relu) s = fmaxf(s, 0.f);
+    Y[row * ldy + k0 + k] = s;
   }
 }
 
@@ -248,11 +299,31 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
 template <int VEC, int LPG, int NJ>
 static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool cs, int sms, cudaStream_t st) {
   const int threads = 256;
-  int64_t units = warp_mode ? a.n_rows : ceil_div(a.n_rows, 32 / LPG);
+  int64_t units = (warp_mode ? a.n_rows : ceil_div(a.n_rows, 32 / LPG)) + a.n_seg;
   // enough warps for 8 resident blocks/SM, capped by the work available
   int64_t blocks = std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 8);
   blocks = std::max<int64_t>(blocks, 1);
 #define GR_L(K) K<<<(unsigned)blocks, threads, 0, st>>>(a)
+  // tuning hook (GRANII_SPMM_TUNE="U,MINB"): alternative unroll / occupancy for the
+  // unweighted warp-per-row kernels of the two dominant shapes
+  if constexpr (VEC == 4 && NJ == 2 && (LPG == 8 || LPG == 32)) {
+    const char* tune = getenv("GRANII_SPMM_TUNE");
+    if (warp_mode && !w && !cs && tune) {
+      int u = 0, mb = 0;
+      sscanf(tune, "%d,%d", &u, &mb);
+      const int64_t bl = std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 16));
+#define GR_T(U_, M_) k_spmm_warp<VEC, LPG, NJ, false, false, U_, M_><<<(unsigned)bl, threads, 0, st>>>(a)
+      if (u == 2 && mb == 4) GR_T(2, 4);
+      else if (u == 2 && mb == 3) GR_T(2, 3);
+      else if (u == 8 && mb == 2) GR_T(8, 2);
+      else if (u == 4 && mb == 4) GR_T(4, 4);
+      else if (u == 4 && mb == 2) GR_T(4, 2);
+      else GR_T(4, 3);
+#undef GR_T
+      GR_CHECK_LAUNCH();
+      return GRANII_OK;
+    }
+  }
   if (warp_mode) {
     if (w && cs) GR_L((k_spmm_warp<VEC, LPG, NJ, true, true>));
     else if (w) GR_L((k_spmm_warp<VEC, LPG, NJ, true, false>));
@@ -323,8 +394,13 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
   GR_TRY(dev_info(&di));
   const bool vec4 = (ldx % 4 == 0) && (ldy % 4 == 0) && ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0);
   const bool warp_mode = g->avg_deg() >= 16.f;
-  SpmmArgs a{g->n_rows, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0, g->order};
+  SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
+             g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0};
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
+  if (g->n_seg > 0) {  // stream-ordered scratch for the heavy-row partials (pool-backed, no sync)
+    a.ldp = round_up(kw, 4);
+    GR_CUDA(cudaMallocAsync((void**)&a.partial, (size_t)g->n_seg * a.ldp * sizeof(float), st));
+  }
   // algorithmic bytes: per entry col id (+w, +cs) + one K-row of X;
   // per row row_ptr + the K-row of Y (+rs)
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
@@ -335,7 +411,15 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
     a.kw = std::min(kw, K - k0);
     // slices of a vec4 launch must stay 16-byte aligned
     GR_TRY(launch_slice(a, vec4 && (k0 % 4 == 0), warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
+    if (g->n_seg > 0) {
+      const int64_t tot = g->n_heavy * a.kw;
+      k_spmm_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(
+          g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0);
+      GR_CHECK_LAUNCH();
+      ps.add_launches(1);
+    }
   }
+  if (a.partial) GR_CUDA(cudaFreeAsync(a.partial, st));
   return GRANII_OK;
 }
 

@@ -36,7 +36,7 @@ COMP_NAMES = {0: "GCN_PRE_AGG", 1: "GCN_PRE_UPD", 2: "GCN_DYN_AGG", 3: "GCN_DYN_
               17: "GAT_RECOMP"}
 ACT_NONE, ACT_RELU = 0, 1
 ATTN_ADDITIVE, ATTN_DOT = 0, 1
-SELECT_NO_PREFILTER = 0x1
+SELECT_NO_PREFILTER, SELECT_TRAINING, SELECT_INPUT_LAYER = 0x1, 0x2, 0x4
 MAX_CANDIDATES = 8
 NUM_FEATURES = 8
 
@@ -83,6 +83,8 @@ _SIGS = {
                                _p, _i64, _p, _p], ctypes.c_int),
     "granii_select": ([_p, ctypes.c_int, _i64, _i64, ctypes.c_char_p, _u32, ctypes.POINTER(ctypes.c_int),
                        ctypes.POINTER(_i32), ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i32)], ctypes.c_int),
+    "granii_cost_features": ([_p, _i32, _i64, _i64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i32),
+                              ctypes.c_char_p], ctypes.c_int),
     "granii_comm_unique_id": ([_p], ctypes.c_int),
     "granii_comm_create": ([_p, _i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_comm_destroy": ([_p], ctypes.c_int),
@@ -282,6 +284,18 @@ def granii_select(g: Graph, model: int, K1: int, K2: int, calib_path: str | None
     _check(_lib.granii_select(g.handle, model, K1, K2, calib_path.encode() if calib_path else None, flags,
                               ctypes.byref(out), cands, pred, ctypes.byref(n)), "granii_select")
     return out.value, {cands[i]: pred[i] for i in range(n.value)}
+
+
+P_SPMM_W, P_SPMM_U, P_SPMM_U_CS, P_SDDMM1, P_SDDMM1_SM, P_GEMM, P_GEMM_NOSTORE, P_GEMM_TN, P_ELEMENTWISE, \
+    P_ALLGATHER = range(10)
+
+
+def granii_cost_features(g: Graph, prim: int, K1: int, K2: int = 0):
+    f = (ctypes.c_double * 8)()
+    n = _i32()
+    name = ctypes.create_string_buffer(32)
+    _check(_lib.granii_cost_features(g.handle, prim, K1, K2, f, ctypes.byref(n), name), "granii_cost_features")
+    return name.value.decode(), [f[i] for i in range(n.value)]
 
 
 # ---------------------------------------------------------------- multi-GPU

@@ -8,11 +8,15 @@ in libgranii.so.
 """
 from __future__ import annotations
 
+import os
 from dataclasses import dataclass, field
 
 import torch
 
 from . import granii as G
+
+# B200 calibration of the per-primitive cost models (tools/calibrate.py)
+DEFAULT_CALIB = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "calib", "b200.txt")
 
 
 def _pad4(k: int) -> int:
@@ -45,11 +49,18 @@ class GNN:
     """A stack of GCN/GAT layers on one (possibly row-partitioned) graph."""
 
     def __init__(self, graph: G.Graph, layers: list[LayerSpec], device, comm: G.Comm | None = None,
-                 calib_path: str | None = None, select_flags: int = 0):
+                 calib_path: str | None = None, select_flags: int = 0, training: bool = False):
+        """training=True costs each candidate's backward too (extension; the paper selects on the
+        forward only, L340) and knows the input layer needs no dH."""
         self.g, self.layers, self.device, self.comm = graph, layers, device, comm
-        for L in layers:
+        if calib_path is None and os.path.exists(DEFAULT_CALIB):
+            calib_path = DEFAULT_CALIB
+        for i, L in enumerate(layers):
             if L.comp is None:
-                L.comp, L.predicted_ms = G.granii_select(graph, L.model, L.K1, L.K2, calib_path, select_flags)
+                fl = select_flags
+                if training:
+                    fl |= G.SELECT_TRAINING | (G.SELECT_INPUT_LAYER if i == 0 else 0)
+                L.comp, L.predicted_ms = G.granii_select(graph, L.model, L.K1, L.K2, calib_path, fl)
         ws = 0
         self.saved_floats = []
         for L in layers:

@@ -122,6 +122,26 @@ def _permutation(n: int, seed: int, stream: int, device) -> torch.Tensor:
     return torch.sort(keys, stable=True).indices
 
 
+def road(n: int, seed: int, device="cpu", p_extra: float = 0.05):
+    """Road-network-like graph (belgium_osm shape, Table II): a near-square
+    grid lattice (right / down neighbours, ids in grid order: spatial locality)
+    with a seeded fraction of lattice edges dropped and a few random shortcuts,
+    giving average degree ~3 and a near-uniform degree distribution."""
+    side = int(math.ceil(math.sqrt(n)))
+    i = torch.arange(n, dtype=torch.int64, device=device)
+    r, c = i // side, i % side
+    right = (c + 1 < side) & (i + 1 < n)
+    down = i + side < n
+    src = torch.cat([i[right], i[down]])
+    dst = torch.cat([i[right] + 1, i[down] + side])
+    keep = uniform_int(seed, 30, src.numel(), 1000, device) >= 300          # drop 30% of lattice edges
+    src, dst = src[keep], dst[keep]
+    k = int(p_extra * n)
+    es = uniform_int(seed, 31, k, n, device)
+    ed = torch.clamp(es + uniform_int(seed, 32, k, 64, device) - 32, 0, n - 1)  # short random links
+    return torch.cat([src, es]).to(torch.int32), torch.cat([dst, ed]).to(torch.int32)
+
+
 def ring(n: int, k: int):
     """k-regular ring lattice (k even): i -> i+1..i+k/2, undirected pairs."""
     src = torch.arange(n, dtype=torch.int64).repeat_interleave(k // 2)
@@ -159,6 +179,8 @@ class Workload:
     def edges(self, seed: int = 0, device="cpu"):
         if self.kind == "chung_lu":
             return chung_lu(self.n, self.m, self.gamma, seed, device, self.max_w_frac)
+        if self.kind == "road":
+            return road(self.n, seed, device)
         a, b, c = self.rmat_abc
         return rmat(self.n, self.m, a, b, c, seed, device)
 
@@ -183,6 +205,12 @@ WORKLOADS = {
     "products": Workload("products", 2449029, 64_000_000, "rmat", True, rmat_abc=(0.45, 0.22, 0.22),
                          dims={"K_in": 100, "K_hid": [32, 256, 1024], "K_out": 47},
                          cite="PAPER.md Table II L301, Table IV L381-L386"),
+    # selector-regret extremes of Table II: road-like and very dense
+    "belgium": Workload("belgium", 1441295, 0, "road", True, dims={"K": [32, 256, 1024]},
+                        cite="PAPER.md Table II L299 (belgium_osm: 1,441,295 nodes, 4,541,235 edges)"),
+    "mycielskian": Workload("mycielskian", 98303, 52_000_000, "chung_lu", True, gamma=4.0, max_w_frac=0.0005,
+                            dims={"K": [32, 256, 1024]},
+                            cite="PAPER.md Table II L298 (mycielskian17: 98,303 nodes, 100,245,742 edges)"),
 }
 
 

@@ -206,6 +206,49 @@ def test_spmm_deterministic(G):
     assert torch.equal(Y1, Y2)
 
 
+@pytest.mark.parametrize("name", ["sparse", "dense", "directed"])
+def test_heavy_row_segments(G, name, monkeypatch):
+    """Rows longer than GRANII_SEG entries are split into warp-wide segments whose
+    partials are combined in fixed order (SpMM) / by a 3-phase segmented softmax
+    (SDDMM).  Forcing a tiny segment length exercises that path on every hub."""
+    base = case(G, name)
+    monkeypatch.setenv("GRANII_SEG", "64")
+    g = G.granii_graph_csr_create(base.n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), base.flags)
+    monkeypatch.delenv("GRANII_SEG")
+    rp, ci, n = base.rp, base.ci, base.n
+    assert np.diff(rp).max() > 64
+    dv = torch.tensor(O.dinv(rp), dtype=torch.float32)
+    for K in (16, 41, 256):
+        X = synth.uniform_pm1(80, K, (n, K))
+        Y = pad(torch.zeros(n, K))
+        G.granii_spmm(g, None, pad(X), K, Y, dv.to(DEV), dv.to(DEV), G.EPI_RELU)
+        ref = np.maximum(dv.numpy()[:, None] * O.spmm(rp, ci, dv.numpy().astype(np.float64)[ci], X), 0)
+        torch.cuda.synchronize()
+        assert err(Y.cpu(), ref) <= TOL, K
+    out = torch.zeros(ci.shape[0], device=DEV)
+    el = synth.uniform_pm1(81, 1, (n,)) * 3
+    er = synth.uniform_pm1(81, 2, (n,)) * 3
+    G.granii_sddmm(g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el.to(DEV), 1, er.to(DEV), 1, 1, 1.0,
+                   out)
+    rows = np.repeat(np.arange(n), np.diff(rp))
+    e = el.numpy().astype(np.float64)[rows] + er.numpy().astype(np.float64)[ci]
+    torch.cuda.synchronize()
+    assert err(out.cpu(), O.edge_softmax(rp, np.where(e > 0, e, 0.2 * e)), rp) <= TOL
+    U = synth.uniform_pm1(82, 1, (n, 64))
+    Ud = pad(U)
+    G.granii_sddmm(g, G.SDDMM_DOT | G.SDDMM_ROW_SOFTMAX, Ud, Ud.stride(0), Ud, Ud.stride(0), 64, 0.125, out)
+    torch.cuda.synchronize()
+    assert err(out.cpu(), O.edge_softmax(rp, 0.125 * O.sddmm(rp, ci, U, U)), rp) <= TOL
+    c2 = Case.__new__(Case)
+    c2.n, c2.g, c2.rp, c2.ci = n, g, rp, ci
+    for comp in (0, 2, 3):
+        _, o, H, W, _, _ = run_layer(G, c2, G.GCN, comp, 48, 32, G.ACT_RELU)
+        assert err(o.cpu(), O.gcn_forward(comp, rp, ci, H, W, 1)[0]) <= TOL
+    for comp in (16, 17):
+        _, o, H, W, al, ar = run_layer(G, c2, G.GAT, comp, 32, 64, G.ACT_NONE)
+        assert err(o.cpu(), O.gat_forward(comp, rp, ci, H, W, al, ar, 0)[0]) <= TOL
+
+
 # ------------------------------------------------------------------ SDDMM
 @pytest.mark.parametrize("name", ["sparse", "dense", "directed"])
 def test_sddmm_norm_and_attention(G, name):
