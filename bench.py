@@ -170,6 +170,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-regret", action="store_true")
     ap.add_argument("--comp", default=None, help="force compositions, e.g. 1,3 (skips the selector)")
+    ap.add_argument("--cuda-graph", default="auto", choices=["auto", "on", "off"],
+                    help="capture the step in a CUDA graph (auto: when an eager step takes < 5 ms)")
     ap.add_argument("--out", default=None, help="also write the JSON line to this file")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -232,19 +234,49 @@ def main():
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
+    eager_ms = time_region(step, 2, stream)
     setup_s = time.perf_counter() - t_setup
+
+    # CUDA graph of the whole step (launch-bound small graphs): every call is stream-
+    # ordered with no host sync, scratch comes from the stream-ordered pool
+    use_graph = args.cuda_graph == "on" or (args.cuda_graph == "auto" and eager_ms < 5.0)
+    run = step
+    launches_per_step = None
+    if use_graph:
+        l0 = G.granii_launch_count()
+        step()
+        torch.cuda.synchronize()
+        launches_per_step = G.granii_launch_count() - l0
+        side = torch.cuda.Stream()
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            step()
+        stream.wait_stream(side)
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            step()
+        run = graph.replay
+        for _ in range(3):
+            run()
+        torch.cuda.synchronize()
 
     # ---------------------------------------------------------------- timed region
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     launches0 = G.granii_launch_count()
-    G.granii_profile_enable(True)
+    if not use_graph:
+        G.granii_profile_enable(True)     # per-primitive events on the launch stream, inside the region
     with Clocks(local) as clk:
-        ms = time_region(step, args.steps, stream)
+        ms = time_region(run, args.steps, stream)
+    if use_graph:
+        launches = launches_per_step * args.steps
+        G.granii_profile_enable(True)     # graph replays carry no host-side records: profile an eager pass
+        time_region(step, args.steps, stream)
+    else:
+        launches = G.granii_launch_count() - launches0
     prof = G.granii_profile_read()
     G.granii_profile_enable(False)
-    launches = G.granii_launch_count() - launches0
     if world > 1:
         dist.barrier()
         t = torch.tensor([ms], device=dev)
@@ -294,7 +326,9 @@ def main():
                    "gemm": "tcgen05 kind::tf32 3xTF32 (fp32-accurate)",
                    "l2": "no flush: per-step inputs exceed L2 (H %.0f MB, col_idx %.0f MB vs 126 MB L2)" % (
                        w.n * dims[0] * 4 / 1e6, info.nnz * 4 / 1e6),
-                   "parallelism": f"row-partition x{world}" + (" (NCCL all-gather)" if world > 1 else "")},
+                   "parallelism": f"row-partition x{world}" + (" (NCCL all-gather)" if world > 1 else ""),
+                   "cuda_graph": bool(use_graph),
+                   "profile_pass": "separate eager pass (graph replay)" if use_graph else "inside the timed region"},
         "clocks": clk.summary(),
         "gpu_launches": int(launches),
         "roofline": roof,

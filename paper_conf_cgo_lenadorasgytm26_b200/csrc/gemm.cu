@@ -4,24 +4,25 @@
 // C[M x N] = A[M x K] · B[K x N] (+ fused epilogue: row scale = Eq. 1 row-
 // broadcast, GAT attention GEMVs el = C a_l / er = C a_r, ReLU).
 //
-// Tensor-core path, one CTA per 128 x BN output tile:
-//   warp 0      TMA producer: A tile (128 x 32 fp32, SWIZZLE_128B) and the
-//               pre-split B_hi / B_lo tiles (BN x 32, K-major) per stage
-//   warp 1      TMEM allocator + MMA issuer (one elected thread):
-//               3 x tcgen05.mma.kind::tf32 per 8-wide k step
-//               (A_hi B_hi + A_hi B_lo + A_lo B_hi -- the 3xTF32 split)
-//   warps 2..5  split A in shared memory (hi = rna(A), lo = rna(A - hi),
-//               in place + a second buffer; elementwise, so the swizzled layout
-//               is preserved), then the epilogue: tcgen05.ld 32x32b -> regs ->
-//               scale / GEMVs / ReLU -> global.
-// Pipelines: full[s] (TMA -> converters, tx bytes), conv[s] (converters ->
-// MMA), empty[s] (tcgen05.commit -> TMA), accum (last commit -> epilogue).
-// B (the weight, <= K1 x K2 floats) is split and transposed once per call
-// into the workspace by a tiny prep kernel.
+// Tensor-core path: persistent (one CTA per SM over 128 x BN
+// tiles, BN <= 128; the N tiles of an M tile run back to back so A re-reads hit
+// L2), warp-specialised, 18 warps:
+//   warp 0       TMA producer: raw A stages (128 x 32 fp32, SWIZZLE_128B) and
+//                pre-split B_hi / B_lo stages (BN x 32, K-major)
+//   warp 1       TMEM allocator + single-thread MMA issuer: 3 x tcgen05.mma
+//                kind::tf32 per 8-wide k step with A read from TMEM
+//                (A_hi B_hi + A_hi B_lo + A_lo B_hi -- the 3xTF32 split), into
+//                one of two TMEM accumulators (epilogue overlap)
+//   warps 2..9   converters: split raw A rows into tf32 hi / lo and tcgen05.st
+//                them into TMEM; the raw smem stage is released immediately
+//   warps 10..17 epilogue: tcgen05.ld -> row scale / attention GEMVs / ReLU ->
+//                smem transpose -> full 128-byte line stores
+// B (the weight, <= K1 x K2 floats) is split and transposed once per call into
+// the workspace by a tiny prep kernel.
 //
-// Fallback (lda % 4 != 0, transposed A, or no TMA alignment): fp32 SIMT tiles.
-// dW = Aᵀ B (reduction over the node dimension) uses a deterministic split-K
-// SIMT kernel + fixed-order reduction.
+// dW = Aᵀ B (reduction over nodes): MN-major tf32 operands (SWIZZLE_128B_BASE32B)
+// with split-K and a fixed-order partial sum.  Fallbacks (unaligned lda / ldb):
+// fp32 SIMT tiles and a deterministic split-K SIMT kernel.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -113,12 +114,20 @@ constexpr int TC_BM = 128, TC_BK = 32;  // 32 fp32 = one 128-byte swizzle row
 
 template <int BN>
 struct TcCfg {
-  static constexpr int A_BYTES = TC_BM * TC_BK * 4;  // 16 KB
-  static constexpr int B_BYTES = BN * TC_BK * 4;
-  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int STAGES = (STAGE * 3 <= 200 * 1024) ? 3 : 2;
-  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
-  static constexpr int SMEM = STAGES * STAGE + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int A_BYTES = TC_BM * TC_BK * 4;                  // raw A stage: 128 x 32 fp32 = 16 KB
+  static constexpr int B_BYTES = BN * TC_BK * 4;                     // one of B_hi / B_lo
+  static constexpr int ACC_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : 128;  // one fp32 accumulator
+  static constexpr int TSTAGES = 4;                                  // split A (hi | lo) stages in TMEM
+  static constexpr int TMEM_COLS = 512;                              // 2 accumulators + TSTAGES x 64
+  static_assert(2 * ACC_COLS + TSTAGES * 64 <= TMEM_COLS, "TMEM budget");
+  static constexpr int EPI_BYTES = 8 * 32 * 33 * 4;                  // epilogue staging (8 warps x 32 x 33)
+  static constexpr int B_STAGE = 2 * B_BYTES;
+  // raw A stages (HBM stream), then B stages (L2, <= 4); 8 A stages measured no faster
+  static constexpr int RA = 4;
+  static constexpr int SB_FIT = (200 * 1024 - RA * A_BYTES - EPI_BYTES) / B_STAGE;
+  static constexpr int SB = SB_FIT > 4 ? 4 : SB_FIT;                 // B (hi, lo) stages in smem
+  static_assert(RA >= 2 && SB >= 2, "smem budget");
+  static constexpr int SMEM = RA * A_BYTES + SB * B_STAGE + EPI_BYTES + 1024 /*align*/ + 512 /*barriers*/;
 };
 
 struct TcEpi {
@@ -133,37 +142,69 @@ struct TcEpi {
   int store;
 };
 
+__device__ __forceinline__ void mma_tf32_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+      "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]), "r"(r[18]),
+      "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]),
+      "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+      : "memory");
+}
+
+// Persistent, warp-specialised, one CTA per SM looping over 128 x BN output tiles
+// (the N tiles of one M tile back to back so A's re-read hits L2).
+//   warp 0      TMA producer: raw A (128 x 32 fp32, SWIZZLE_128B) ring of RA stages and
+//               the pre-split B_hi / B_lo (BN x 32, K-major) ring of SB stages
+//   warps 2..9  converters (two groups alternating k-blocks): each thread takes one row of the raw A stage (conflict-free
+//               swizzled 16-byte reads), splits it into tf32 hi / lo and writes both into
+//               a TMEM A stage with tcgen05.st; the raw smem stage is released to the TMA
+//               right away (it no longer waits for the MMA)
+//   warp 1      TMEM allocator + single-thread MMA issuer: tcgen05.mma kind::tf32 with A
+//               read from TMEM, 3 per 8-wide k step (A_hi B_hi + A_hi B_lo + A_lo B_hi);
+//               tile i accumulates into TMEM buffer i & 1 while the epilogue drains the other
+//   warps 10..17 epilogue: tcgen05.ld -> scale / GEMVs / ReLU -> smem transpose -> 128 B stores;
+//               two warps per TMEM lane quadrant split the 32-column chunks (latency hiding)
+constexpr int TC_THREADS = 576;
+
 template <int BN>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(TC_THREADS, 1)
     k_gemm_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
               const __grid_constant__ CUtensorMap tmBl, int M, int N, int K, TcEpi ep) {
   using Cfg = TcCfg<BN>;
-  constexpr int S = Cfg::STAGES;
+  constexpr int RA = Cfg::RA, SB = Cfg::SB, TS = Cfg::TSTAGES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* bars = (uint64_t*)(smem + S * Cfg::STAGE);
-  uint64_t* full = bars;
-  uint64_t* conv = bars + S;
-  uint64_t* empty = bars + 2 * S;
-  uint64_t* accum = bars + 3 * S;
-  uint32_t* tmem_slot = (uint32_t*)(bars + 3 * S + 1);
+  uint8_t* sA = smem;                                   // RA x 16 KB
+  uint8_t* sB = smem + RA * Cfg::A_BYTES;               // SB x (B_hi | B_lo)
+  float* stage_out = (float*)(sB + SB * Cfg::B_STAGE);  // epilogue staging
+  uint64_t* bars = (uint64_t*)((uint8_t*)stage_out + Cfg::EPI_BYTES);
+  uint64_t* a_full = bars;                 // [RA] TMA -> converters
+  uint64_t* a_empty = a_full + RA;         // [RA] converters -> TMA
+  uint64_t* b_full = a_empty + RA;         // [SB] TMA -> MMA
+  uint64_t* b_empty = b_full + SB;         // [SB] MMA commit -> TMA
+  uint64_t* t_full = b_empty + SB;         // [TS] converters -> MMA (A in TMEM)
+  uint64_t* t_empty = t_full + TS;         // [TS] MMA commit -> converters
+  uint64_t* c_full = t_empty + TS;         // [2] MMA commit -> epilogue
+  uint64_t* c_empty = c_full + 2;          // [2] epilogue -> MMA
+  uint32_t* tmem_slot = (uint32_t*)(c_empty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int m0 = blockIdx.x * TC_BM, n0 = blockIdx.y * BN;
   const int nk = (K + TC_BK - 1) / TC_BK;
-
-  auto a_hi = [&](int s) { return smem + s * Cfg::STAGE; };
-  auto a_lo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
-  auto b_hi = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
-  auto b_lo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+  const int mt = (M + TC_BM - 1) / TC_BM, ntn = (N + BN - 1) / BN;
 
   if (warp == 0 && lane == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 128);
-      mbar_init(&empty[s], 1);
-    }
-    mbar_init(accum, 1);
+    for (int s = 0; s < RA; ++s) { mbar_init(&a_full[s], 1); mbar_init(&a_empty[s], 128); }
+    for (int s = 0; s < SB; ++s) { mbar_init(&b_full[s], 1); mbar_init(&b_empty[s], 1); }
+    for (int s = 0; s < TS; ++s) { mbar_init(&t_full[s], 128); mbar_init(&t_empty[s], 1); }
+    for (int b = 0; b < 2; ++b) { mbar_init(&c_full[b], 1); mbar_init(&c_empty[b], 256); }
     fence_barrier_init();
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmBh) : "memory");
@@ -178,105 +219,162 @@ __global__ void __launch_bounds__(192, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  const uint32_t tA0 = tmem + 2 * Cfg::ACC_COLS;  // first TMEM A stage (hi: +0..31, lo: +32..63)
 
+#define TC_TILE_LOOP for (int mi = blockIdx.x; mi < mt; mi += gridDim.x) for (int ni = 0; ni < ntn; ++ni
   if (warp == 0) {
     if (lane == 0) {
-      for (int kb = 0; kb < nk; ++kb) {
-        const int s = kb % S;
-        const uint32_t ph = (kb / S) & 1;
-        mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], Cfg::A_BYTES + 2 * Cfg::B_BYTES);
-        tma_load_2d(&tmA, &full[s], a_hi(s), kb * TC_BK, m0);
-        tma_load_2d(&tmBh, &full[s], b_hi(s), kb * TC_BK, n0);
-        tma_load_2d(&tmBl, &full[s], b_lo(s), kb * TC_BK, n0);
+      int it = 0;
+      TC_TILE_LOOP) {
+        const int m0 = mi * TC_BM, n0 = ni * BN;
+        for (int kb = 0; kb < nk; ++kb, ++it) {
+          const int ra = it % RA, sb = it % SB;
+          mbar_wait(&a_empty[ra], ((it / RA) & 1) ^ 1);
+          mbar_expect_tx(&a_full[ra], Cfg::A_BYTES);
+          tma_load_2d(&tmA, &a_full[ra], sA + ra * Cfg::A_BYTES, kb * TC_BK, m0);
+          mbar_wait(&b_empty[sb], ((it / SB) & 1) ^ 1);
+          mbar_expect_tx(&b_full[sb], Cfg::B_STAGE);
+          tma_load_2d(&tmBh, &b_full[sb], sB + sb * Cfg::B_STAGE, kb * TC_BK, n0);
+          tma_load_2d(&tmBl, &b_full[sb], sB + sb * Cfg::B_STAGE + Cfg::B_BYTES, kb * TC_BK, n0);
+        }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
       constexpr uint32_t idesc = idesc_tf32(TC_BM, BN);
-      for (int kb = 0; kb < nk; ++kb) {
-        const int s = kb % S;
-        const uint32_t ph = (kb / S) & 1;
-        mbar_wait(&conv[s], ph);
+      int it = 0, lt = 0;
+      TC_TILE_LOOP, ++lt) {
+        const int buf = lt & 1;
+        const uint32_t acc = tmem + (uint32_t)(buf * Cfg::ACC_COLS);
+        mbar_wait(&c_empty[buf], ((lt >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
         tc_fence_after();
-        const uint32_t ah = smem_u32(a_hi(s)), al = smem_u32(a_lo(s));
-        const uint32_t bh = smem_u32(b_hi(s)), bl = smem_u32(b_lo(s));
+        for (int kb = 0; kb < nk; ++kb, ++it) {
+          const int ts = it % TS, sb = it % SB;
+          mbar_wait(&t_full[ts], (it / TS) & 1);
+          mbar_wait(&b_full[sb], (it / SB) & 1);
+          tc_fence_after();
+          const uint32_t ahi = tA0 + ts * 64, alo = ahi + 32;
+          const uint32_t bh = smem_u32(sB + sb * Cfg::B_STAGE), bl = bh + Cfg::B_BYTES;
 #pragma unroll
-        for (int k = 0; k < TC_BK / 8; ++k) {  // tf32: K = 8 per MMA = 32 bytes
-          const uint32_t off = k * 32;
-          const uint64_t dah = desc_sw128(ah + off), dal = desc_sw128(al + off);
-          const uint64_t dbh = desc_sw128(bh + off), dbl = desc_sw128(bl + off);
-          mma_tf32(tmem, dah, dbh, idesc, (kb | k) ? 1u : 0u);
-          mma_tf32(tmem, dah, dbl, idesc, 1u);
-          mma_tf32(tmem, dal, dbh, idesc, 1u);
+          for (int k = 0; k < TC_BK / 8; ++k) {  // tf32: K = 8 per MMA (8 TMEM columns, 32 B of B rows)
+            const uint64_t dbh = desc_sw128(bh + k * 32), dbl = desc_sw128(bl + k * 32);
+            mma_tf32_ta(acc, ahi + k * 8, dbh, idesc, (kb | k) ? 1u : 0u);
+            mma_tf32_ta(acc, ahi + k * 8, dbl, idesc, 1u);
+            mma_tf32_ta(acc, alo + k * 8, dbh, idesc, 1u);
+          }
+          mma_commit(&b_empty[sb]);
+          mma_commit(&t_empty[ts]);
         }
-        mma_commit(&empty[s]);
+        mma_commit(&c_full[buf]);
       }
-      mma_commit(accum);
+    }
+  } else if (warp < 10) {
+    // ---------------- converters: raw A row -> tf32 hi / lo -> TMEM
+    const int quad = warp & 3;
+    const int cgroup = (warp - 2) >> 2;  // group g converts the k-blocks with it % 2 == g
+    const int row = quad * 32 + lane;    // TMEM lane == tile row
+    int it = 0;
+    TC_TILE_LOOP) {
+      for (int kb = 0; kb < nk; ++kb, ++it) {
+        if ((it & 1) != cgroup) continue;  // the other converter group takes this k-block
+        const int ra = it % RA, ts = it % TS;
+        mbar_wait(&a_full[ra], (it / RA) & 1);
+        const uint8_t* rowp = sA + ra * Cfg::A_BYTES + row * 128;
+        uint32_t hi[32], lo[32];
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {  // SWIZZLE_128B: 16-byte chunk c of row r sits at chunk c ^ (r & 7)
+          const float4 x = *reinterpret_cast<const float4*>(rowp + ((c ^ (row & 7)) << 4));
+          const float xs[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const float h = tf32_rna(xs[q]);
+            hi[c * 4 + q] = __float_as_uint(h);
+            lo[c * 4 + q] = __float_as_uint(tf32_rna(xs[q] - h));
+          }
+        }
+        fence_proxy_async();            // our generic reads before the TMA's next async write
+        mbar_arrive(&a_empty[ra]);      // raw stage free as soon as it is split
+        mbar_wait(&t_empty[ts], ((it / TS) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t tb = tA0 + ts * 64 + ((uint32_t)(quad * 32) << 16);
+        tmem_st32(tb, hi);
+        tmem_st32(tb + 32, lo);
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_fence_before();
+        mbar_arrive(&t_full[ts]);
+      }
     }
   } else {
-    // ---------------- converters: split A into tf32 hi / lo in place
-    const int ct = threadIdx.x - 64;  // 0..127
-    for (int kb = 0; kb < nk; ++kb) {
-      const int s = kb % S;
-      const uint32_t ph = (kb / S) & 1;
-      mbar_wait(&full[s], ph);
-      float4* hi = reinterpret_cast<float4*>(a_hi(s));
-      float4* lo = reinterpret_cast<float4*>(a_lo(s));
-#pragma unroll
-      for (int i = 0; i < Cfg::A_BYTES / 16 / 128; ++i) {
-        const int idx = ct + i * 128;
-        float4 x = hi[idx];
-        float4 h, l;
-        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
-        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
-        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
-        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
-        hi[idx] = h;
-        lo[idx] = l;
-      }
-      fence_proxy_async();
-      mbar_arrive(&conv[s]);
-    }
     // ---------------- epilogue: TMEM -> registers -> global
-    mbar_wait(accum, 0);
-    tc_fence_after();
-    const int quad = warp & 3;  // TMEM lanes [32*quad, 32*quad+32)
-    const int r = m0 + quad * 32 + lane;
-    const bool rok = r < M;
-    const float rsc = (ep.row_scale && rok) ? __ldg(ep.row_scale + r) : 1.f;
-    float el = 0.f, er = 0.f;
+    const int quad = warp & 3;          // TMEM lanes [32*quad, 32*quad+32)
+    const int half = (warp - 10) >> 2;  // which of the two warps of this quadrant
+    int lt = 0;
+    TC_TILE_LOOP, ++lt) {
+      const int buf = lt & 1;
+      const int m0 = mi * TC_BM, n0 = ni * BN, ntile = ni;
+      mbar_wait(&c_full[buf], (lt >> 1) & 1);
+      tc_fence_after();
+      const int rbase = m0 + quad * 32;  // this warp's 32 rows
+      const int r = rbase + lane;        // the row this thread holds in registers
+      const bool rok = r < M;
+      const float rsc = (ep.row_scale && rok) ? __ldg(ep.row_scale + r) : 1.f;
+      float el = 0.f, er = 0.f;
+      float* stg = stage_out + (warp - 10) * 32 * 33;
 #pragma unroll 1
-    for (int c0 = 0; c0 < BN; c0 += 16) {
-      float v[16];
-      tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + c0, v);
-      const int cb = n0 + c0;
+      for (int c0 = 32 * half; c0 < BN; c0 += 64) {  // this warp's 32-column chunks (BN % 16 == 0)
+        float v[32];
+        tmem_ld16(tmem + (uint32_t)(buf * Cfg::ACC_COLS) + ((uint32_t)(quad * 32) << 16) + c0, *(float(*)[16])v);
+        if (c0 + 16 < BN)
+          tmem_ld16(tmem + (uint32_t)(buf * Cfg::ACC_COLS) + ((uint32_t)(quad * 32) << 16) + c0 + 16,
+                    *(float(*)[16])(v + 16));
+        const int cb = n0 + c0;
 #pragma unroll
-      for (int j = 0; j < 16; ++j) {
-        v[j] *= rsc;
-        if (cb + j < N) {
-          if (ep.att_l) el = fmaf(v[j], __ldg(ep.att_l + cb + j), el);
-          if (ep.att_r) er = fmaf(v[j], __ldg(ep.att_r + cb + j), er);
+        for (int j = 0; j < 32; ++j) v[j] *= rsc;
+        if (ep.att_l || ep.att_r) {
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            if (cb + j < N && c0 + j < BN) {
+              if (ep.att_l) el = fmaf(v[j], __ldg(ep.att_l + cb + j), el);
+              if (ep.att_r) er = fmaf(v[j], __ldg(ep.att_r + cb + j), er);
+            }
         }
-        if (ep.relu) v[j] = fmaxf(v[j], 0.f);
-      }
-      if (ep.store && rok) {
-        float* crow = ep.C + (int64_t)r * ep.ldc + cb;
-        if (cb + 16 <= N && ((((uintptr_t)crow) & 15) == 0)) {
+        if (ep.relu)
 #pragma unroll
-          for (int j = 0; j < 16; j += 4) *reinterpret_cast<float4*>(crow + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-        } else {
+          for (int j = 0; j < 32; ++j) v[j] = fmaxf(v[j], 0.f);
+        if (ep.store) {
+          // transpose through shared memory so every store instruction writes whole
+          // 128-byte lines (8 lanes per row, 4 rows per instruction)
 #pragma unroll
-          for (int j = 0; j < 16; ++j)
-            if (cb + j < N) crow[j] = v[j];
+          for (int j = 0; j < 32; ++j) stg[lane * 33 + j] = v[j];
+          __syncwarp();
+          const int cc = (lane & 7) * 4;  // 4 consecutive columns
+          const bool cfull = (cb + cc + 4 <= N) && (c0 + cc + 4 <= BN) && ((ep.ldc & 3) == 0);
+#pragma unroll 4
+          for (int rr = lane >> 3; rr < 32; rr += 4) {
+            const int rowo = rbase + rr;
+            if (rowo >= M) break;
+            float* cp = ep.C + (int64_t)rowo * ep.ldc + cb + cc;
+            const float* sp = stg + rr * 33 + cc;
+            if (cfull && ((((uintptr_t)cp) & 15) == 0)) {
+              *reinterpret_cast<float4*>(cp) = make_float4(sp[0], sp[1], sp[2], sp[3]);
+            } else {
+#pragma unroll
+              for (int q = 0; q < 4; ++q)
+                if (cb + cc + q < N && c0 + cc + q < BN) cp[q] = sp[q];
+            }
+          }
+          __syncwarp();
         }
       }
-    }
-    if (rok) {
-      if (ep.out_l) ep.out_l[(int64_t)blockIdx.y * M + r] = el;
-      if (ep.out_r) ep.out_r[(int64_t)blockIdx.y * M + r] = er;
+      tc_fence_before();
+      mbar_arrive(&c_empty[buf]);  // accumulator drained: the MMA may overwrite it
+      if (rok) {
+        if (ep.out_l) ep.out_l[(int64_t)(2 * ntile + half) * M + r] = el;  // per-half partials
+        if (ep.out_r) ep.out_r[(int64_t)(2 * ntile + half) * M + r] = er;
+      }
     }
   }
+#undef TC_TILE_LOOP
   tc_fence_before();
   __syncthreads();
   if (warp == 1) {
@@ -284,6 +382,7 @@ __global__ void __launch_bounds__(192, 1)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS));
   }
 }
+
 
 // B (K x N, or N x K when transposed) -> Bt_hi / Bt_lo [Npad x Kpad], K-major, zero padded.
 __global__ void k_prep_b(int K, int N, const float* __restrict__ B, int64_t ldb, int transB, int Kpad, int Npad,
@@ -621,9 +720,7 @@ static int pick_bn(int64_t N) {
   if (N <= 48) return 48;
   if (N <= 64) return 64;
   if (N <= 96) return 96;
-  if (N <= 128) return 128;
-  if (N <= 192) return 192;
-  return 256;
+  return 128;  // wider N runs as consecutive 128-column tiles of the same M tile (A re-read hits L2)
 }
 
 static bool tc_eligible(int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, uint32_t flags) {
@@ -666,7 +763,7 @@ size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags) {
   const int64_t Npad = round_up(N, bn), Kpad = round_up(K, TC_BK);
   ws += (size_t)2 * Npad * Kpad * 4 + 1024;
   const int64_t tiles = ceil_div(N, bn);
-  ws += (size_t)2 * tiles * M * 4 + 256;  // attention partials
+  ws += (size_t)2 * 2 * tiles * M * 4 + 256;  // attention partials: 2 per N tile (epilogue halves)
   return ws;
 }
 
@@ -679,8 +776,11 @@ static granii_status launch_tc_bn(int M, int N, int K, const CUtensorMap& ta, co
     GR_CUDA(cudaFuncSetAttribute(k_gemm_tc<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
     attr_set = true;
   }
-  dim3 grid((unsigned)ceil_div(M, TC_BM), (unsigned)ceil_div(N, BN));
-  k_gemm_tc<BN><<<grid, 192, Cfg::SMEM, st>>>(ta, tbh, tbl, M, N, K, ep);
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  const int64_t tiles = ceil_div(M, TC_BM);  // persistent over M tiles; N tiles inside
+  const unsigned grid = (unsigned)std::min<int64_t>(tiles, di.sms);  // persistent: one CTA per SM
+  k_gemm_tc<BN><<<grid, TC_THREADS, Cfg::SMEM, st>>>(ta, tbh, tbl, M, N, K, ep);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
@@ -780,7 +880,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
   float* blo = bhi + Npad * Kpad;
   float* part_l = blo + Npad * Kpad;
   const int64_t tiles = ceil_div(N, bn);
-  float* part_r = part_l + tiles * M;
+  float* part_r = part_l + 2 * tiles * M;
   k_prep_b<<<(unsigned)std::min<int64_t>(ceil_div(Npad * Kpad, 256), 4096), 256, 0, st>>>(
       (int)K, (int)N, B, ldb, tb ? 1 : 0, (int)Kpad, (int)Npad, bhi, blo);
   GR_CHECK_LAUNCH();
@@ -793,23 +893,21 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
 
   TcEpi ep{C, ldc, rs, epi ? epi->att_l : nullptr, epi ? epi->att_r : nullptr, nullptr, nullptr, relu ? 1 : 0,
            store ? 1 : 0};
-  if (epi && epi->att_l && epi->out_l) ep.out_l = tiles == 1 ? epi->out_l : part_l;
-  if (epi && epi->att_r && epi->out_r) ep.out_r = tiles == 1 ? epi->out_r : part_r;
+  if (epi && epi->att_l && epi->out_l) ep.out_l = part_l;
+  if (epi && epi->att_r && epi->out_r) ep.out_r = part_r;
   switch (bn) {
     case 16: GR_TRY(launch_tc_bn<16>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
     case 32: GR_TRY(launch_tc_bn<32>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
     case 48: GR_TRY(launch_tc_bn<48>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
     case 64: GR_TRY(launch_tc_bn<64>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
     case 96: GR_TRY(launch_tc_bn<96>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
-    case 128: GR_TRY(launch_tc_bn<128>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
-    case 192: GR_TRY(launch_tc_bn<192>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
-    default: GR_TRY(launch_tc_bn<256>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
+    default: GR_TRY(launch_tc_bn<128>((int)M, (int)N, (int)K, ta, tbh, tbl, ep, st)); break;
   }
-  if (tiles > 1) {
+  if (ep.out_l || ep.out_r) {  // fixed-order sum of the per-(N tile, half) GEMV partials
     ps.add_launches((ep.out_l ? 1 : 0) + (ep.out_r ? 1 : 0));
     const unsigned b = (unsigned)std::min<int64_t>(ceil_div(M, 256), 4096);
-    if (ep.out_l) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_l, epi->out_l);
-    if (ep.out_r) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)tiles, part_r, epi->out_r);
+    if (ep.out_l) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)(2 * tiles), part_l, epi->out_l);
+    if (ep.out_r) k_reduce_partials<<<b, 256, 0, st>>>((int)M, (int)(2 * tiles), part_r, epi->out_r);
     GR_CHECK_LAUNCH();
   }
   return GRANII_OK;

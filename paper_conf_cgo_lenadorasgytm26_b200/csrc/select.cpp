@@ -211,8 +211,12 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
   GR_TRY(load_model(path, &m));
   const In in = inputs_of(g);
   std::vector<int> c;
+  // the embedding-size rule is a forward-only argument (narrower SpMM); with the
+  // backward in the cost (and no dH on the input layer) it no longer holds, so the
+  // training selection keeps all four GCN trees and lets the cost models decide
+  const bool prefilter = !(flags & (GRANII_SELECT_NO_PREFILTER | GRANII_SELECT_TRAINING));
   if (model == GRANII_GCN) {
-    if (flags & GRANII_SELECT_NO_PREFILTER) c = {GRANII_GCN_PRE_AGG, GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_AGG, GRANII_GCN_DYN_UPD};
+    if (!prefilter) c = {GRANII_GCN_PRE_AGG, GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_AGG, GRANII_GCN_DYN_UPD};
     else if (K1 >= K2) c = {GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_UPD};   // group ">=": update first
     else c = {GRANII_GCN_PRE_AGG, GRANII_GCN_DYN_AGG};                 // group "<": aggregate first
   } else {
