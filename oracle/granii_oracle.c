@@ -337,6 +337,47 @@ int oracle_gat_forward(int comp, int attn_dot, int64_t N, const int64_t* row_ptr
   return 0;
 }
 
+/* Per-row definition of the GAT layer (Eq. 4/5 read row by row) for sampled rows:
+ * Θ_j = H_j W for j in the row (and the row itself), e_ij = LeakyReLU(Θ_i a_l + Θ_j a_r),
+ * α = row softmax, Y_i = Σ_j α_ij Θ_j.  Rows are indices into (row_ptr, col_idx). */
+void oracle_gat_rows(int64_t n_sample, const int64_t* rows, const int64_t* row_ptr, const int32_t* col_idx,
+                     const double* H, int64_t K1, const double* W, int64_t K2, const double* a_l, const double* a_r,
+                     int act, double* out /* n_sample x K2 */) {
+#pragma omp parallel for schedule(dynamic, 4)
+  for (int64_t s = 0; s < n_sample; ++s) {
+    int64_t r = rows[s], b = row_ptr[r], t = row_ptr[r + 1], d = t - b;
+    double* th = (double*)malloc((size_t)(K2 * (d + 1)) * sizeof(double));  /* Θ of the neighbours, then Θ_r */
+    double* e = (double*)malloc((size_t)(d + 1) * sizeof(double));
+    for (int64_t q = 0; q <= d; ++q) {
+      int64_t j = q < d ? (int64_t)col_idx[b + q] : r;
+      for (int64_t c = 0; c < K2; ++c) {
+        double v = 0.0;
+        for (int64_t k = 0; k < K1; ++k) v += H[j * K1 + k] * W[k * K2 + c];
+        th[q * K2 + c] = v;
+      }
+    }
+    double el = 0.0;
+    for (int64_t c = 0; c < K2; ++c) el += th[d * K2 + c] * a_l[c];
+    double m = -INFINITY;
+    for (int64_t q = 0; q < d; ++q) {
+      double er = 0.0;
+      for (int64_t c = 0; c < K2; ++c) er += th[q * K2 + c] * a_r[c];
+      double x = el + er;
+      e[q] = x > 0.0 ? x : 0.2 * x;
+      if (e[q] > m) m = e[q];
+    }
+    double ssum = 0.0;
+    for (int64_t q = 0; q < d; ++q) ssum += exp(e[q] - m);
+    for (int64_t c = 0; c < K2; ++c) {
+      double v = 0.0;
+      for (int64_t q = 0; q < d; ++q) v += exp(e[q] - m) / ssum * th[q * K2 + c];
+      out[s * K2 + c] = (act == 1 && v < 0.0) ? 0.0 : v;
+    }
+    free(th);
+    free(e);
+  }
+}
+
 /* ------------------------------------------------------------------------ */
 /* O6: GCN backward (training, L340: the forward's composition is used;      */
 /* backward follows the forward's primitive order reversed [R14]).           */

@@ -53,6 +53,7 @@ def lib():
         _lib.oracle_gcn_forward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, p, p]
         _lib.oracle_gcn_rows.argtypes = [i64, p, p, p, p, p, i64, p, i64, ctypes.c_int, p]
         _lib.oracle_edge_softmax.argtypes = [i64, p, p, p]
+        _lib.oracle_gat_rows.argtypes = [i64, p, p, p, p, i64, p, i64, p, p, ctypes.c_int, p]
         _lib.oracle_gat_forward.argtypes = [ctypes.c_int, ctypes.c_int, i64, p, p, p, i64, p, i64, p, p,
                                             ctypes.c_int, p, p]
         _lib.oracle_gcn_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, p, p, p]
@@ -172,6 +173,18 @@ def gcn_rows(rows, row_ptr, col_idx, deg_of_col, H, W, act=1):
     out = np.zeros((rows.shape[0], W.shape[1]), np.float64)
     lib().oracle_gcn_rows(rows.shape[0], _p(rows), _p(rp), _p(ci), _p(dg), _p(H), H.shape[1], _p(W),
                           W.shape[1], act, _p(out))
+    return out
+
+
+def gat_rows(rows, row_ptr, col_idx, H, W, a_l, a_r, act=0):
+    """per-row definition of the (additive) GAT layer for sampled rows"""
+    rows = _np(rows, np.int64)
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, W = _np(H, np.float64), _np(W, np.float64)
+    al, ar = _np(a_l, np.float64), _np(a_r, np.float64)
+    out = np.zeros((rows.shape[0], W.shape[1]), np.float64)
+    lib().oracle_gat_rows(rows.shape[0], _p(rows), _p(rp), _p(ci), _p(H), H.shape[1], _p(W), W.shape[1], _p(al),
+                          _p(ar), act, _p(out))
     return out
 
 

@@ -292,6 +292,17 @@ def test_gat_matches_dense_masked_softmax(comp, dot):
     assert np.allclose(sums, 1.0, atol=1e-14)
 
 
+def test_gat_rows_matches_dense_definition():
+    rp, ci, A = csr_and_dense(54, n=40, m=200, flags=O.ADD_SELF_LOOPS)
+    rng = np.random.default_rng(16)
+    H, W = rng.uniform(-1, 1, (40, 5)), rng.uniform(-1, 1, (5, 9))
+    al, ar = rng.uniform(-1, 1, 9), rng.uniform(-1, 1, 9)
+    ref, _ = dense_gat(A, H, W, al, ar, False, O.GAT_REUSE)
+    rows = np.array([0, 3, 17, 39, 22])
+    assert rel(O.gat_rows(rows, rp, ci, H, W, al, ar), ref[rows]) < 1e-12
+    assert rel(O.gat_rows(rows, rp, ci, H, W, al, ar, act=1), np.maximum(ref[rows], 0)) < 1e-12
+
+
 def test_gat_closed_forms():
     rp, ci, A = csr_and_dense(52, n=25, m=100)
     rng = np.random.default_rng(12)
