@@ -18,6 +18,28 @@ __global__ void k_relu_mask(int64_t rows, int64_t K, const float* __restrict__ o
   }
 }
 
+// dst = (out == NULL || out > 0) ? g * rs[r] : 0  -- ReLU' mask (optional) fused with an
+// optional row scale (the inner D^-1/2 of the DYN_UPD backward, so its SpMM needs no column scale)
+__global__ void k_scale_mask(int64_t rows, int64_t K, const float* __restrict__ out, int64_t ldo,
+                             const float* __restrict__ g, int64_t ldg, const float* __restrict__ rs,
+                             float* __restrict__ dst, int64_t ldd) {
+  const int64_t total = rows * K;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / K, k = i % K;
+    const float v = g[r * ldg + k] * (rs ? rs[r] : 1.f);
+    dst[r * ldd + k] = (!out || out[r * ldo + k] > 0.f) ? v : 0.f;
+  }
+}
+
+granii_status launch_scale_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
+                                const float* rs, float* dst, int64_t ldd, cudaStream_t st) {
+  if (rows * K == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, (out ? 12.0 : 8.0) * rows * K, 0.0, 1);
+  k_scale_mask<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, out, ldo, g, ldg, rs, dst, ldd);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
 __global__ void k_copy_rows(int64_t rows, int64_t K, const float* __restrict__ src, int64_t lds,
                             float* __restrict__ dst, int64_t ldd) {
   const int64_t total = rows * K;

@@ -111,6 +111,8 @@ size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags);
 granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
                           int64_t ldb, float* C, int64_t ldc, const granii_gemm_epilogue* epi, uint32_t flags,
                           void* ws, size_t ws_bytes, cudaStream_t st);
+granii_status launch_scale_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
+                                const float* rs, float* dst, int64_t ldd, cudaStream_t st);
 granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g,
                                int64_t ldg, float* dst, int64_t ldd, cudaStream_t st);
 granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,

@@ -242,8 +242,9 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
   const bool dy_gathered = comp == GRANII_GCN_PRE_UPD || comp == GRANII_GCN_DYN_UPD;
   GatherBuf dyg = gather_buf(b, c, K2);
   if (run) {
-    if (relu) GR_TRY(launch_relu_mask(R, K2, out, ldo, dout, lddo, dyg.mine, dyg.ld, st));
-    else GR_TRY(launch_copy_rows(R, K2, dout, lddo, dyg.mine, dyg.ld, st));
+    // DYN_UPD: dT = D Ãᵀ (D dY) -- the inner D is applied here, so the SpMM has no column scale
+    const float* pre = comp == GRANII_GCN_DYN_UPD ? g->dinv_rows : nullptr;
+    GR_TRY(launch_scale_mask(R, K2, relu ? out : nullptr, ldo, dout, lddo, pre, dyg.mine, dyg.ld, st));
   }
   const float* dY = dyg.mine;
   const int64_t lddy = dyg.ld;
@@ -295,7 +296,7 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
         if (comp == GRANII_GCN_PRE_UPD)
           GR_TRY(launch_spmm(g, nval, dyg.all, dyg.ld, K2, dT, ldt2, nullptr, nullptr, false, st));
         else
-          GR_TRY(launch_spmm(g, nullptr, dyg.all, dyg.ld, K2, dT, ldt2, g->dinv_rows, g->dinv_cols, false, st));
+          GR_TRY(launch_spmm(g, nullptr, dyg.all, dyg.ld, K2, dT, ldt2, g->dinv_rows, nullptr, false, st));
         GR_TRY(launch_gemm(K1, K2, R, H, ldh, dT, ldt2, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
         if (dH) GR_TRY(launch_gemm(R, K1, K2, dT, ldt2, a->W, K2, dH, lddh, nullptr, GRANII_GEMM_TRANS_B, gwH, gnH, st));
         break;

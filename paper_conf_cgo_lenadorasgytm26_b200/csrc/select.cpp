@@ -188,7 +188,7 @@ double backward_cost(const CostModel& m, const In& in, int comp, double K1, doub
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U, K1);
       break;
     case GRANII_GCN_DYN_UPD:
-      t += cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U_CS, K2);
+      t += cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);  // inner D fused in the ReLU' pass
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
       break;
     default:
