@@ -41,7 +41,9 @@ struct Bump {
   }
 };
 
-static inline int64_t ld4(int64_t k) { return round_up(k, 4); }
+// leading dimension of internal dense buffers: 16-byte rows (TMA / float4), and whole
+// 32-byte L2 sectors once rows are >= 8 floats (each gathered row touches the fewest sectors)
+static inline int64_t ld4(int64_t k) { return k >= 8 ? round_up(k, 8) : round_up(k, 4); }
 
 struct Ctx {
   const granii_graph_s* g;

@@ -20,7 +20,8 @@ DEFAULT_CALIB = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__f
 
 
 def _pad4(k: int) -> int:
-    return (k + 3) // 4 * 4
+    """row stride: 16-byte rows, whole 32-byte sectors once a row has >= 8 floats"""
+    return (k + 7) // 8 * 8 if k >= 8 else (k + 3) // 4 * 4
 
 
 def alloc2d(rows: int, cols: int, device, fill=None) -> torch.Tensor:
