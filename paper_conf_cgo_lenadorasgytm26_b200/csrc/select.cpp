@@ -33,21 +33,24 @@ struct CostModel {
   std::map<std::string, std::vector<double>> coef;
 };
 
-// feature vectors (all sizes in GB / TFLOP, time in ms)
-//   spmm            : [1, streamed GB (idx, weights, col-scale gather), out GB, gathered GB from L2, gathered GB from HBM]
-//   sddmm1          : [1, streamed GB]
-//   sddmm1_softmax  : [1, streamed GB]
-//   gemm            : [1, HBM GB, TFLOP]
-//   gemm_tn         : [1, HBM GB, TFLOP]
+// feature vectors (all sizes in GB / TFLOP / millions, time in ms)
+//   spmm            : [1, streamed GB (idx, weights, col-scale gather), out GB, gathered GB from L2,
+//                      gathered GB from HBM, M rows, thousands of hub segments]
+//   sddmm1          : [1, streamed GB, M rows]
+//   sddmm1_softmax  : [1, streamed GB, M rows]
+//   gemm            : [1, HBM GB, TFLOP, thousands of 128x128 tiles]
+//   gemm_att        : [1, HBM GB, TFLOP, thousands of tiles, attention GEMV GB (M x K2 x 4)]
+//   gemm_tn         : [1, HBM GB, TFLOP, thousands of tiles]
 //   elementwise     : [1, GB]
 //   allgather       : [1, GB received per GPU]
 static CostModel defaults() {
   CostModel m;
-  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0};
-  m.coef["sddmm1"] = {0.005, 1.0 / 5.5};
-  m.coef["sddmm1_softmax"] = {0.006, 1.0 / 4.0};
-  m.coef["gemm"] = {0.010, 1.0 / 2.0, 1.0 / 250.0};
-  m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 250.0};
+  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0};
+  m.coef["sddmm1"] = {0.005, 1.0 / 5.5, 0.0};
+  m.coef["sddmm1_softmax"] = {0.006, 1.0 / 4.0, 0.0};
+  m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0};
+  m.coef["gemm_att"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 1.0 / 3.0};
+  m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
   m.coef["elementwise"] = {0.004, 1.0 / 5.5};
   m.coef["allgather"] = {0.020, 1.0 / 700.0};
   return m;
@@ -92,7 +95,7 @@ static granii_status load_model(const char* path, CostModel* out) {
 }
 
 struct In {
-  double R, nnz, ncols, avg, l2, world;
+  double R, nnz, ncols, avg, l2, world, nseg;
 };
 
 // fraction of gathered bytes served by L2: the sliced SpMM keeps
@@ -106,14 +109,15 @@ static double l2_hit(const In& in, double K) {
 
 // primitive ids of the feature API
 enum { P_SPMM_W = 0, P_SPMM_U = 1, P_SPMM_U_CS = 2, P_SDDMM1 = 3, P_SDDMM1_SM = 4, P_GEMM = 5, P_GEMM_NOSTORE = 6,
-       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9 };
+       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10 };
 
 static const char* prim_model(int p) {
   switch (p) {
     case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: return "spmm";
     case P_SDDMM1: return "sddmm1";
     case P_SDDMM1_SM: return "sddmm1_softmax";
-    case P_GEMM: case P_GEMM_NOSTORE: return "gemm";
+    case P_GEMM: return "gemm";
+    case P_GEMM_NOSTORE: case P_GEMM_ATT: return "gemm_att";
     case P_GEMM_TN: return "gemm_tn";
     case P_ELEMENTWISE: return "elementwise";
     case P_ALLGATHER: return "allgather";
@@ -128,13 +132,22 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
     case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: {
       const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
       const double idx = in.nnz * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 4.0 : 0.0)) * gb;
-      return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h)};
+      return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3};
     }
-    case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb};
-    case P_SDDMM1_SM: return {1.0, in.nnz * 16.0 * gb};
-    case P_GEMM: return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
-    case P_GEMM_NOSTORE: return {1.0, in.R * K1 * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
-    case P_GEMM_TN: return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12};
+    case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb, in.R * 1e-6};
+    case P_SDDMM1_SM: return {1.0, in.nnz * 16.0 * gb, in.R * 1e-6};
+    case P_GEMM:
+      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
+              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
+    case P_GEMM_ATT:  // GAT Θ = H W with the el / er GEMVs in the epilogue, Θ stored
+      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
+              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb};
+    case P_GEMM_NOSTORE:  // el / er only, Θ never written
+      return {1.0, in.R * K1 * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
+              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb};
+    case P_GEMM_TN:
+      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
+              std::ceil(K1 / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
     case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
     case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};
   }
@@ -163,7 +176,7 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
     case GRANII_GCN_DYN_UPD:
       return cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);
     case GRANII_GAT_REUSE:
-      return cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SDDMM1_SM, 0) +
+      return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SDDMM1_SM, 0) +
              cost(m, in, P_SPMM_W, K2);
     case GRANII_GAT_RECOMP:
       return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SDDMM1_SM, 0) +
@@ -201,7 +214,7 @@ static In inputs_of(const granii_graph_s* g) {
   DevInfo di;
   if (dev_info(&di) != GRANII_OK) di = DevInfo();  // host-only selection still works
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-            (double)g->world};
+            (double)g->world, (double)g->n_seg};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K1, int64_t K2, const char* path,
@@ -243,7 +256,7 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
 
 granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t K1, int64_t K2, double* feats,
                                  int32_t* n, char* model_name) {
-  if (prim < P_SPMM_W || prim > P_ALLGATHER) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
+  if (prim < P_SPMM_W || prim > P_GEMM_ATT) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
   const std::vector<double> f = features(inputs_of(g), prim, (double)K1, (double)K2);
   for (size_t i = 0; i < f.size(); ++i) feats[i] = f[i];
   *n = (int32_t)f.size();

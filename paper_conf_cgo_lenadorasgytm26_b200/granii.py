@@ -287,7 +287,7 @@ def granii_select(g: Graph, model: int, K1: int, K2: int, calib_path: str | None
 
 
 P_SPMM_W, P_SPMM_U, P_SPMM_U_CS, P_SDDMM1, P_SDDMM1_SM, P_GEMM, P_GEMM_NOSTORE, P_GEMM_TN, P_ELEMENTWISE, \
-    P_ALLGATHER = range(10)
+    P_ALLGATHER, P_GEMM_ATT = range(11)
 
 
 def granii_cost_features(g: Graph, prim: int, K1: int, K2: int = 0):

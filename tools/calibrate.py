@@ -39,6 +39,10 @@ GRAPHS = [
     ("rmat-400k", "rmat", 400_000, 4_000_000, None, 107, False),
     ("rmat-1.5m", "rmat", 1_500_000, 15_000_000, None, 108, True),
     ("road-800k", "road", 800_000, 0, None, 109, True),
+    ("rmat-200k-dir", "rmat", 200_000, 1_600_000, None, 110, False),
+    ("rmat-3m", "rmat", 3_000_000, 40_000_000, None, 111, True),
+    ("cl-250k-dense", "chung_lu", 250_000, 45_000_000, 2.8, 112, True),
+    ("cl-30k", "chung_lu", 30_000, 120_000, 2.4, 113, True),
 ]
 KS = [16, 32, 64, 128, 256, 512]
 GEMM_PAIRS = [(32, 32), (64, 256), (256, 64), (100, 256), (602, 256), (256, 41), (1024, 128), (128, 1024),
@@ -105,6 +109,8 @@ def sweep(quick=False):
             ws2 = torch.empty(G.granii_gemm_workspace_size(R, k2, k1, G.GEMM_NO_STORE), dtype=torch.uint8, device=DEV)
             rec(G.P_GEMM_NOSTORE, k1, k2, timed(lambda: G.granii_gemm(
                 R, k2, k1, A, A.stride(0), W, k2, None, k2, G.GEMM_NO_STORE, None, al, al, ol, ol, workspace=ws2)))
+            rec(G.P_GEMM_ATT, k1, k2, timed(lambda: G.granii_gemm(
+                R, k2, k1, A, A.stride(0), W, k2, C, C.stride(0), 0, None, al, al, ol, ol, workspace=ws2)))
             dW = torch.empty((k1, k2), device=DEV)
             ws3 = torch.empty(G.granii_gemm_workspace_size(k1, k2, R, G.GEMM_TRANS_A), dtype=torch.uint8, device=DEV)
             rec(G.P_GEMM_TN, k1, k2, timed(lambda: G.granii_gemm(k1, k2, R, A, A.stride(0), C, C.stride(0), dW, k2,
