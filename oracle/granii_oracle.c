@@ -444,3 +444,103 @@ int oracle_gcn_backward(int comp, int64_t N, const int64_t* row_ptr, const int32
   free(y); free(o); free(dY); free(dinv); free(a); free(b); free(c); free(nval);
   return 0;
 }
+
+/* ------------------------------------------------------------------------ */
+/* GAT backward (training; the paper trains GAT, L324/L340, */
+/* but gives no backward: this is the chain rule of the forward definition  */
+/* above, additive attention only [R22]).  Reverse of the forward's steps:  */
+/*   dY   = G ⊙ σ'(Y)                                                        */
+/*   REUSE  (Y = α Θ):     dα_ij = <dY_i, Θ_j>,  dΘ  = αᵀ dY                 */
+/*   RECOMP (Y = T W, T = α H): dW = Tᵀ dY, dT = dY Wᵀ,                      */
+/*                          dα_ij = <dT_i, H_j>,  dH  = αᵀ dT                */
+/*   softmax:   de_ij = α_ij (dα_ij - Σ_j' α_ij' dα_ij')                     */
+/*   LeakyReLU: dz_ij = de_ij · (z_ij > 0 ? 1 : 0.2),  z_ij = el_i + er_j    */
+/*   del_i = Σ_j dz_ij,  der_j = Σ_i dz_ij                                   */
+/*   el = Θ a_l, er = Θ a_r:  dΘ_att = del a_lᵀ + der a_rᵀ,                  */
+/*       da_l = Θᵀ del,  da_r = Θᵀ der                                       */
+/*   Θ = H W:  dW += Hᵀ dΘ_all,  dH += dΘ_all Wᵀ                             */
+/* (REUSE: dΘ_all = αᵀ dY + dΘ_att;  RECOMP: dΘ_all = dΘ_att.)               */
+/* αᵀ X is the literal transpose-scatter of the stored entries.             */
+/* ------------------------------------------------------------------------ */
+int oracle_gat_backward(int comp, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, const double* H,
+                        int64_t K1, const double* W, int64_t K2, const double* a_l, const double* a_r, int act,
+                        const double* G, double* dH /* nullable */, double* dW, double* da_l, double* da_r) {
+  int64_t nnz = row_ptr[N];
+  if (comp != OR_GAT_REUSE && comp != OR_GAT_RECOMP) return 1;
+  double* theta = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* el = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* er = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* z = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* e = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* alpha = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* y = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* dY = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* dal = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* dz = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* del = (double*)calloc((size_t)(N + 1), sizeof(double));
+  double* der = (double*)calloc((size_t)(N + 1), sizeof(double));
+  double* dth = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* t = (double*)malloc((size_t)(N * K1 + 1) * sizeof(double));
+  double* dT = (double*)malloc((size_t)(N * K1 + 1) * sizeof(double));
+  double* tmp = (double*)malloc((size_t)(K1 * K2 + N * K1 + 1) * sizeof(double));
+  /* forward (same steps as oracle_gat_forward) */
+  oracle_gemm(N, K2, K1, H, 0, W, 0, theta);
+  oracle_gemm(N, 1, K2, theta, 0, a_l, 0, el);
+  oracle_gemm(N, 1, K2, theta, 0, a_r, 0, er);
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) {
+      z[i] = el[r] + er[col_idx[i]];
+      e[i] = z[i] > 0.0 ? z[i] : 0.2 * z[i];
+    }
+  oracle_edge_softmax(N, row_ptr, e, alpha);
+  oracle_spmm(N, row_ptr, col_idx, alpha, H, K1, t);                          /* T = α H */
+  if (comp == OR_GAT_REUSE) oracle_spmm(N, row_ptr, col_idx, alpha, theta, K2, y);
+  else oracle_gemm(N, K2, K1, t, 0, W, 0, y);
+  /* dY = G ⊙ σ'(Y), ReLU'(0) = 0 */
+  for (int64_t i = 0; i < N * K2; ++i) dY[i] = (act == 1 && !(y[i] > 0.0)) ? 0.0 : G[i];
+  /* dα (SDDMM of the composition's operands) */
+  if (comp == OR_GAT_REUSE) {
+    oracle_sddmm(N, row_ptr, col_idx, dY, theta, K2, dal);                    /* <dY_i, Θ_j> */
+  } else {
+    oracle_gemm(K1, K2, N, t, 1, dY, 0, dW);                                  /* dW = Tᵀ dY */
+    oracle_gemm(N, K1, K2, dY, 0, W, 1, dT);                                  /* dT = dY Wᵀ */
+    oracle_sddmm(N, row_ptr, col_idx, dT, H, K1, dal);                        /* <dT_i, H_j> */
+  }
+  /* softmax and LeakyReLU backward, row by row */
+  for (int64_t r = 0; r < N; ++r) {
+    double s = 0.0;
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) s += alpha[i] * dal[i];
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i)
+      dz[i] = alpha[i] * (dal[i] - s) * (z[i] > 0.0 ? 1.0 : 0.2);
+  }
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) {
+      del[r] += dz[i];
+      der[col_idx[i]] += dz[i];
+    }
+  /* dΘ_att = del a_lᵀ + der a_rᵀ ; da = Θᵀ [del, der] */
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t c = 0; c < K2; ++c) dth[r * K2 + c] = del[r] * a_l[c] + der[r] * a_r[c];
+  oracle_gemm(K2, 1, N, theta, 1, del, 0, da_l);
+  oracle_gemm(K2, 1, N, theta, 1, der, 0, da_r);
+  if (comp == OR_GAT_REUSE) {
+    double* sc = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+    oracle_spmm_t(N, N, row_ptr, col_idx, alpha, dY, K2, sc);                 /* αᵀ dY */
+    for (int64_t i = 0; i < N * K2; ++i) dth[i] += sc[i];
+    free(sc);
+    oracle_gemm(K1, K2, N, H, 1, dth, 0, dW);                                 /* Hᵀ dΘ */
+    if (dH) oracle_gemm(N, K1, K2, dth, 0, W, 1, dH);                         /* dΘ Wᵀ */
+  } else {
+    oracle_gemm(K1, K2, N, H, 1, dth, 0, tmp);                                /* Hᵀ dΘ_att */
+    for (int64_t i = 0; i < K1 * K2; ++i) dW[i] += tmp[i];
+    if (dH) {
+      oracle_spmm_t(N, N, row_ptr, col_idx, alpha, dT, K1, dH);               /* αᵀ dT */
+      double* h2 = tmp + K1 * K2;
+      oracle_gemm(N, K1, K2, dth, 0, W, 1, h2);                               /* dΘ_att Wᵀ */
+      for (int64_t i = 0; i < N * K1; ++i) dH[i] += h2[i];
+    }
+  }
+  free(theta); free(el); free(er); free(z); free(e); free(alpha); free(y); free(dY); free(dal); free(dz);
+  free(del); free(der); free(dth); free(t); free(dT); free(tmp);
+  return 0;
+}

@@ -56,6 +56,8 @@ def lib():
         _lib.oracle_gat_rows.argtypes = [i64, p, p, p, p, i64, p, i64, p, p, ctypes.c_int, p]
         _lib.oracle_gat_forward.argtypes = [ctypes.c_int, ctypes.c_int, i64, p, p, p, i64, p, i64, p, p,
                                             ctypes.c_int, p, p]
+        _lib.oracle_gat_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, p, p, ctypes.c_int, p, p, p,
+                                             p, p]
         _lib.oracle_gcn_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, p, p, p]
     return _lib
 
@@ -223,3 +225,21 @@ def gcn_backward(comp, row_ptr, col_idx, H, W, G, act=1, need_dH=True):
     if rc:
         raise ValueError(f"bad composition {comp}")
     return dH, dW
+
+
+def gat_backward(comp, row_ptr, col_idx, H, W, a_l, a_r, G, act=0, need_dH=True):
+    """GAT backward (additive attention): returns (dH or None, dW, da_l, da_r)."""
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, W, G = _np(H, np.float64), _np(W, np.float64), _np(G, np.float64)
+    al, ar = _np(a_l, np.float64), _np(a_r, np.float64)
+    N, K1 = H.shape
+    K2 = W.shape[1]
+    dW = np.zeros((K1, K2), np.float64)
+    dH = np.zeros((N, K1), np.float64) if need_dH else None
+    dal = np.zeros(K2, np.float64)
+    dar = np.zeros(K2, np.float64)
+    rc = lib().oracle_gat_backward(comp, N, _p(rp), _p(ci), _p(H), K1, _p(W), K2, _p(al), _p(ar), act, _p(G),
+                                   _p(dH), _p(dW), _p(dal), _p(dar))
+    if rc:
+        raise ValueError(f"bad composition {comp}")
+    return dH, dW, dal, dar

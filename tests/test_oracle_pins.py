@@ -381,6 +381,69 @@ def test_gcn_backward_compositions_agree_and_identity_closed_form():
         assert rel(dW, H1.T @ G1) < 1e-14 and rel(dH, G1 @ W.T) < 1e-14
 
 
+# ------------------------------------------------------------------ GAT backward (N2, reading R22)
+def gat_loss(comp, rp, ci, H, W, al, ar, G, act):
+    return float((O.gat_forward(comp, rp, ci, H, W, al, ar, act)[0] * G).sum())
+
+
+@pytest.mark.parametrize("comp", O.GAT_COMPS)
+@pytest.mark.parametrize("flags", [O.SYMMETRIZE | O.ADD_SELF_LOOPS, O.ADD_SELF_LOOPS])
+def test_gat_backward_finite_differences(comp, flags):
+    """every gradient (W, H, a_l, a_r) against central differences of the pinned forward"""
+    rp, ci, _ = csr_and_dense(63, n=11, m=30, flags=flags)
+    rng = np.random.default_rng(16)
+    H, W = rng.uniform(-1, 1, (11, 4)), rng.uniform(-1, 1, (4, 3))
+    al, ar = rng.uniform(-1, 1, 3), rng.uniform(-1, 1, 3)
+    G = rng.standard_normal((11, 3))
+    h = 1e-6
+
+    def fd(X, f):
+        out = np.zeros_like(X)
+        for idx in np.ndindex(X.shape):
+            Xp, Xm = X.copy(), X.copy()
+            Xp[idx] += h
+            Xm[idx] -= h
+            out[idx] = (f(Xp) - f(Xm)) / (2 * h)
+        return out
+
+    for act in (0, 1):
+        dH, dW, dal, dar = O.gat_backward(comp, rp, ci, H, W, al, ar, G, act)
+        assert np.max(np.abs(dW - fd(W, lambda x: gat_loss(comp, rp, ci, H, x, al, ar, G, act)))) < 1e-7
+        assert np.max(np.abs(dH - fd(H, lambda x: gat_loss(comp, rp, ci, x, W, al, ar, G, act)))) < 1e-7
+        assert np.max(np.abs(dal - fd(al, lambda x: gat_loss(comp, rp, ci, H, W, x, ar, G, act)))) < 1e-7
+        assert np.max(np.abs(dar - fd(ar, lambda x: gat_loss(comp, rp, ci, H, W, al, x, G, act)))) < 1e-7
+
+
+def test_gat_backward_compositions_agree_and_closed_forms():
+    rp, ci, _ = csr_and_dense(64, n=80, m=500)
+    rng = np.random.default_rng(17)
+    H, W = rng.uniform(-1, 1, (80, 6)), rng.uniform(-1, 1, (6, 9))
+    al, ar = rng.uniform(-1, 1, 9), rng.uniform(-1, 1, 9)
+    G = rng.standard_normal((80, 9))
+    a = O.gat_backward(O.GAT_REUSE, rp, ci, H, W, al, ar, G, 1)
+    b = O.gat_backward(O.GAT_RECOMP, rp, ci, H, W, al, ar, G, 1)
+    for x, y in zip(a, b):
+        assert rel(x, y) < 1e-12
+    # need_dH=False leaves the parameter gradients unchanged
+    c = O.gat_backward(O.GAT_REUSE, rp, ci, H, W, al, ar, G, 1, need_dH=False)
+    assert c[0] is None and rel(c[1], a[1]) < 1e-15 and rel(c[2], a[2]) < 1e-15
+    # self-loop-only graph: α = I, so Y = Θ, dW = Hᵀ G, dH = G Wᵀ and the scores get no gradient
+    n = 10
+    rp1, ci1 = O.csr_build(n, np.zeros(0, np.int32), np.zeros(0, np.int32), O.ADD_SELF_LOOPS)
+    H1, G1 = rng.standard_normal((n, 6)), rng.standard_normal((n, 9))
+    for comp in O.GAT_COMPS:
+        dH, dW, dal, dar = O.gat_backward(comp, rp1, ci1, H1, W, al, ar, G1, 0)
+        assert rel(dW, H1.T @ G1) < 1e-14 and rel(dH, G1 @ W.T) < 1e-14
+        assert np.all(dal == 0) and np.all(dar == 0)
+    # a_l = a_r = 0: uniform attention α = D⁻¹Ã; dW and dH are the mean-aggregation GCN's
+    z = np.zeros(9)
+    dH, dW, dal, dar = O.gat_backward(O.GAT_REUSE, rp, ci, H, W, z, z, G, 0)
+    A = np.zeros((80, 80))
+    for r in range(80):
+        A[r, ci[rp[r]:rp[r + 1]]] = 1.0 / (rp[r + 1] - rp[r])
+    assert rel(dW, (A @ H).T @ G) < 1e-12 and rel(dH, A.T @ G @ W.T) < 1e-12
+
+
 # ------------------------------------------------------------------ generators
 def test_generator_is_device_independent_and_exact():
     a = synth.uniform_pm1(3, 4, (1000,))
