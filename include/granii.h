@@ -219,6 +219,8 @@ typedef struct {
   void* workspace;         /* device, >= granii_layer_workspace_size bytes               */
   size_t workspace_bytes;
   granii_comm comm;        /* NULL: whole graph on this GPU                              */
+  float* d_a_l;            /* GAT backward outputs dL/da_l, dL/da_r (K2 floats each,     */
+  float* d_a_r;            /*   all-reduced over comm); NULL: not computed               */
 } granii_layer_args;
 
 /* Workspace bytes and the number of floats of `saved` (state kept for backward). */
@@ -236,11 +238,16 @@ granii_status granii_layer_forward(granii_graph g, granii_model m, granii_compos
                                    const granii_layer_args* a, float* d_out, int64_t ldo, float* d_saved,
                                    void* stream);
 /*
- * GCN backward (training, L340: the forward's composition is kept).  For
- * out = sigma(M H W), M = D̃^{-1/2} Ã D̃^{-1/2}, upstream d_dout = dL/dout:
+ * Layer backward (training, L340: the forward's composition is kept).
+ * GCN: for out = sigma(M H W), M = D̃^{-1/2} Ã D̃^{-1/2}, upstream d_dout = dL/dout:
  *   dY = dout ⊙ 1[out > 0] (ReLU; identity otherwise), dW = (M H)ᵀ dY, dH = Mᵀ dY Wᵀ.
+ * GAT (additive attention; chain rule of Eq. 4-6, R22): dW, dH and,
+ *   through a->d_a_l / a->d_a_r, the attention-weight gradients; REUSE works at
+ *   K2, RECOMP at K1 (dT = dY Wᵀ first), as in their forwards.  d_saved is
+ *   required (Θ or T = α H, el, er written by the forward).  Dot attention ->
+ *   UNSUPPORTED.
  * d_dH may be NULL (input layer).  d_dW (K1 x K2) is all-reduced over comm.
- * Requires a symmetric graph (Mᵀ = M); GAT backward -> UNSUPPORTED.
+ * Requires a symmetric graph (Mᵀ = M; GAT: row j of Ã lists every i with j in N(i)).
  */
 granii_status granii_layer_backward(granii_graph g, granii_model m, granii_composition c,
                                     const granii_layer_args* a, const float* d_out, int64_t ldo,

@@ -544,3 +544,104 @@ int oracle_gat_backward(int comp, int64_t N, const int64_t* row_ptr, const int32
   free(del); free(der); free(dth); free(t); free(dT); free(tmp);
   return 0;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Magnitude of the GAT backward computation (tolerance scale, reading R19/ */
+/* R22): the same steps as oracle_gat_backward with every operand replaced  */
+/* by its absolute value and every difference by a sum, so each output is   */
+/* the sum of the absolute values of the terms that form it.  A fp32 path's */
+/* forward error is bounded by a small multiple of eps times this, so the   */
+/* parity tests measure error relative to max(|r|, magnitude) per row.      */
+/* (The softmax backward dα - c cancels by construction: near-one-hot rows  */
+/* have |dα - c| << |dα|.)                                                   */
+/* ------------------------------------------------------------------------ */
+int oracle_gat_backward_magnitude(int comp, int64_t N, const int64_t* row_ptr, const int32_t* col_idx,
+                                  const double* H, int64_t K1, const double* W, int64_t K2, const double* a_l,
+                                  const double* a_r, int act, const double* G, double* mdH, double* mdW,
+                                  double* mda_l, double* mda_r) {
+  int64_t nnz = row_ptr[N];
+  if (comp != OR_GAT_REUSE && comp != OR_GAT_RECOMP) return 1;
+  double* theta = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* el = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* er = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* z = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* e = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* alpha = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* y = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* t = (double*)malloc((size_t)(N * K1 + 1) * sizeof(double));
+  double* aH = (double*)malloc((size_t)(N * K1 + 1) * sizeof(double));
+  double* aW = (double*)malloc((size_t)(K1 * K2 + 1) * sizeof(double));
+  double* mth = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* mdY = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* mdT = (double*)malloc((size_t)(N * K1 + 1) * sizeof(double));
+  double* mda = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* mdz = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* mdel = (double*)calloc((size_t)(N + 1), sizeof(double));
+  double* mder = (double*)calloc((size_t)(N + 1), sizeof(double));
+  double* mdth = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* tmp = (double*)malloc((size_t)(K1 * K2 + 2 * N * (K1 > K2 ? K1 : K2) + 1) * sizeof(double));
+  double* aal = (double*)malloc((size_t)(K2 + 1) * sizeof(double));
+  double* aar = (double*)malloc((size_t)(K2 + 1) * sizeof(double));
+  /* forward values (α, Y) as in oracle_gat_forward */
+  oracle_gemm(N, K2, K1, H, 0, W, 0, theta);
+  oracle_gemm(N, 1, K2, theta, 0, a_l, 0, el);
+  oracle_gemm(N, 1, K2, theta, 0, a_r, 0, er);
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) {
+      z[i] = el[r] + er[col_idx[i]];
+      e[i] = z[i] > 0.0 ? z[i] : 0.2 * z[i];
+    }
+  oracle_edge_softmax(N, row_ptr, e, alpha);
+  oracle_spmm(N, row_ptr, col_idx, alpha, H, K1, t);
+  if (comp == OR_GAT_REUSE) oracle_spmm(N, row_ptr, col_idx, alpha, theta, K2, y);
+  else oracle_gemm(N, K2, K1, t, 0, W, 0, y);
+  /* magnitudes */
+  for (int64_t i = 0; i < N * K1; ++i) aH[i] = fabs(H[i]);
+  for (int64_t i = 0; i < K1 * K2; ++i) aW[i] = fabs(W[i]);
+  for (int64_t i = 0; i < K2; ++i) { aal[i] = fabs(a_l[i]); aar[i] = fabs(a_r[i]); }
+  oracle_gemm(N, K2, K1, aH, 0, aW, 0, mth);                                 /* |H||W| >= |Θ| */
+  for (int64_t i = 0; i < N * K2; ++i) mdY[i] = (act == 1 && !(y[i] > 0.0)) ? 0.0 : fabs(G[i]);
+  if (comp == OR_GAT_REUSE) {
+    oracle_sddmm(N, row_ptr, col_idx, mdY, mth, K2, mda);
+  } else {
+    oracle_gemm(N, K1, K2, mdY, 0, aW, 1, mdT);
+    oracle_sddmm(N, row_ptr, col_idx, mdT, aH, K1, mda);
+  }
+  for (int64_t r = 0; r < N; ++r) {
+    double s = 0.0;
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) s += alpha[i] * mda[i];
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i)
+      mdz[i] = alpha[i] * (mda[i] + s) * (z[i] > 0.0 ? 1.0 : 0.2);
+  }
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) {
+      mdel[r] += mdz[i];
+      mder[col_idx[i]] += mdz[i];
+    }
+  for (int64_t r = 0; r < N; ++r)
+    for (int64_t c = 0; c < K2; ++c) mdth[r * K2 + c] = mdel[r] * aal[c] + mder[r] * aar[c];
+  oracle_gemm(K2, 1, N, mth, 1, mdel, 0, mda_l);
+  oracle_gemm(K2, 1, N, mth, 1, mder, 0, mda_r);
+  if (comp == OR_GAT_REUSE) {
+    double* sc = tmp + K1 * K2 + N * K1;
+    oracle_spmm_t(N, N, row_ptr, col_idx, alpha, mdY, K2, sc);
+    for (int64_t i = 0; i < N * K2; ++i) mdth[i] += sc[i];
+    oracle_gemm(K1, K2, N, aH, 1, mdth, 0, mdW);
+    if (mdH) oracle_gemm(N, K1, K2, mdth, 0, aW, 1, mdH);
+  } else {
+    double* at = tmp + K1 * K2 + N * K1;
+    oracle_spmm(N, row_ptr, col_idx, alpha, aH, K1, at);                    /* α|H| >= |T| */
+    oracle_gemm(K1, K2, N, at, 1, mdY, 0, mdW);
+    oracle_gemm(K1, K2, N, aH, 1, mdth, 0, tmp);
+    for (int64_t i = 0; i < K1 * K2; ++i) mdW[i] += tmp[i];
+    if (mdH) {
+      oracle_spmm_t(N, N, row_ptr, col_idx, alpha, mdT, K1, mdH);
+      double* h2 = tmp + K1 * K2;
+      oracle_gemm(N, K1, K2, mdth, 0, aW, 1, h2);
+      for (int64_t i = 0; i < N * K1; ++i) mdH[i] += h2[i];
+    }
+  }
+  free(theta); free(el); free(er); free(z); free(e); free(alpha); free(y); free(t); free(aH); free(aW); free(mth);
+  free(mdY); free(mdT); free(mda); free(mdz); free(mdel); free(mder); free(mdth); free(tmp); free(aal); free(aar);
+  return 0;
+}

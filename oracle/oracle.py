@@ -58,6 +58,7 @@ def lib():
                                             ctypes.c_int, p, p]
         _lib.oracle_gat_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, p, p, ctypes.c_int, p, p, p,
                                              p, p]
+        _lib.oracle_gat_backward_magnitude.argtypes = _lib.oracle_gat_backward.argtypes
         _lib.oracle_gcn_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, p, p, p]
     return _lib
 
@@ -240,6 +241,24 @@ def gat_backward(comp, row_ptr, col_idx, H, W, a_l, a_r, G, act=0, need_dH=True)
     dar = np.zeros(K2, np.float64)
     rc = lib().oracle_gat_backward(comp, N, _p(rp), _p(ci), _p(H), K1, _p(W), K2, _p(al), _p(ar), act, _p(G),
                                    _p(dH), _p(dW), _p(dal), _p(dar))
+    if rc:
+        raise ValueError(f"bad composition {comp}")
+    return dH, dW, dal, dar
+
+
+def gat_backward_magnitude(comp, row_ptr, col_idx, H, W, a_l, a_r, G, act=0, need_dH=True):
+    """Tolerance scale of the GAT backward (R19/R22): each gradient entry's sum of |terms|."""
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, W, G = _np(H, np.float64), _np(W, np.float64), _np(G, np.float64)
+    al, ar = _np(a_l, np.float64), _np(a_r, np.float64)
+    N, K1 = H.shape
+    K2 = W.shape[1]
+    dW = np.zeros((K1, K2), np.float64)
+    dH = np.zeros((N, K1), np.float64) if need_dH else None
+    dal = np.zeros(K2, np.float64)
+    dar = np.zeros(K2, np.float64)
+    rc = lib().oracle_gat_backward_magnitude(comp, N, _p(rp), _p(ci), _p(H), K1, _p(W), K2, _p(al), _p(ar), act,
+                                             _p(G), _p(dH), _p(dW), _p(dal), _p(dar))
     if rc:
         raise ValueError(f"bad composition {comp}")
     return dH, dW, dal, dar

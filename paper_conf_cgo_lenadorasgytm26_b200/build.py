@@ -21,7 +21,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-fvisibility=hidden", "--expt-relaxed-constexpr",
          "-I" + os.path.join(ROOT, "include")]
-SOURCES = ["api.cu", "csr.cu", "spmm.cu", "sddmm.cu", "gemm.cu", "layer.cu", "elementwise.cu", "select.cpp", "profile.cpp",
+SOURCES = ["api.cu", "csr.cu", "spmm.cu", "sddmm.cu", "gemm.cu", "layer.cu", "gat_bwd.cu", "elementwise.cu", "select.cpp", "profile.cpp",
            "comm.cpp"]
 
 

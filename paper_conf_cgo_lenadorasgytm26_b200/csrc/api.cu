@@ -251,8 +251,10 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
                                     const float* d_saved, float* d_dH, int64_t lddh, float* d_dW, void* stream) {
   API_BEGIN
   GR_TRY(check_args(g, m, c, a));
-  if (m != GRANII_GCN) return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is not implemented (SURVEY N2)");
+  if (m == GRANII_GAT && a->attn != GRANII_ATTN_ADDITIVE)
+    return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is implemented for additive attention only (R22)");
   GR_ARG(g->symmetric, "backward needs a symmetric graph (created with GRANII_SYMMETRIZE): M^T = M");
+  GR_ARG(m == GRANII_GCN || d_saved, "GAT backward needs d_saved from the forward");
   GR_ARG(d_out && d_dout && d_dW && ldo >= a->K2 && lddo >= a->K2, "bad output / gradient");
   GR_ARG(!d_dH || lddh >= a->K1, "bad lddh");
   return layer_backward(g, c, a, d_out, ldo, d_dout, lddo, d_saved, d_dH, lddh, d_dW, (cudaStream_t)stream);

@@ -1,0 +1,393 @@
+// gat_bwd.cu -- GAT backward (training, reading R22).
+//
+// The paper trains GAT (Table III "T", L324) but gives no backward; this is the
+// chain rule of Eq. 4-6.  With z_ij = el_i + er_j, α = row softmax of
+// LeakyReLU(z), dY = dout ⊙ σ'(Y) and (dX, Z) = (dY, Θ) for REUSE or
+// (dT = dY Wᵀ, H) for RECOMP (each composition reverses its own forward):
+//   dα_ij = <dX_i, Z_j>                          (K-wide SDDMM)
+//   c_i   = Σ_j α_ij dα_ij = <dY_i, Y_i>         (row-local: Σ_j α_ij Z_j W.. = Y_i)
+//   dz_ij = α_ij (dα_ij - c_i) · (z_ij > 0 ? 1 : 0.2)
+//   del_i = Σ_j dz_ij        der_j = Σ_i dz_ij
+//   out_j = Σ_i α_ij dX_i + del_j u + der_j v    (REUSE: dΘ with u,v = a_l,a_r;
+//                                                 RECOMP: dH with u,v = W a_l, W a_r)
+// B200 design: two warp-per-row passes in the degree-descending schedule,
+// both gathers of K-wide rows (the SpMM's access pattern):
+//   pass A (rows i): online softmax statistics (m_i, s_i) from the er gathers,
+//     then dα by K-wide gathers of Z_j; writes del_i and the row record
+//     stat_i = {el_i, m_i, 1/s_i, c_i} (one 16-byte gather per edge in pass B).
+//   pass B (rows j, symmetric Ã: row j lists every i with j in N(i)): gathers
+//     stat_i and dX_i, recomputes α_ij from the record (α is never stored),
+//     dots dX_i with the register-resident Z_j, accumulates the transposed
+//     SpMM and der_j, and applies the rank-2 epilogue.
+// Lane groups of LPG lanes own one edge at a time (LPG = K/4 up to 32), NJ
+// float4 per lane cover K.  No atomics: every output is written once, in a
+// fixed reduction order (bitwise reproducible).
+#include <algorithm>
+#include <cmath>
+
+#include "internal.h"
+
+namespace granii {
+
+__device__ __forceinline__ float gb_warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// this lane's NJ float4 slices of a K-wide row; columns >= K read as 0
+// (p is 16-byte aligned with a row stride that is a multiple of 4 floats)
+template <int LPG, int NJ>
+__device__ __forceinline__ void gb_load_row(const float* __restrict__ p, int lg, int64_t K, float (&v)[NJ][4]) {
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    const int64_t col = 4 * (int64_t)(lg + j * LPG);
+    if (col < K) {
+      const float4 t = __ldg(reinterpret_cast<const float4*>(p + col));
+      v[j][0] = t.x;
+      v[j][1] = col + 1 < K ? t.y : 0.f;
+      v[j][2] = col + 2 < K ? t.z : 0.f;
+      v[j][3] = col + 3 < K ? t.w : 0.f;
+    } else {
+      v[j][0] = v[j][1] = v[j][2] = v[j][3] = 0.f;
+    }
+  }
+}
+
+template <int LPG, int NJ>
+__device__ __forceinline__ float gb_dot(const float (&x)[NJ][4], const float (&y)[NJ][4]) {
+  float d = 0.f;
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) d = fmaf(x[j][k], y[j][k], d);
+#pragma unroll
+  for (int o = LPG / 2; o; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);  // within the lane group
+  return d;
+}
+
+__device__ __forceinline__ float gb_lrelu(float z) { return z > 0.f ? z : 0.2f * z; }
+
+// dY = dout ⊙ σ'(out) and c_r = <dY_r, out_r> (= <dY_r, Y_r>: where ReLU clips, dY = 0); warp per row
+__global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, int64_t ldo,
+                           const float* __restrict__ g, int64_t ldg, int relu, float* __restrict__ dY, int64_t ldd,
+                           float* __restrict__ c) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < R; r += nw) {
+    float s = 0.f;
+    for (int64_t k = lane; k < K; k += 32) {
+      const float o = out[r * ldo + k];
+      const float d = (!relu || o > 0.f) ? g[r * ldg + k] : 0.f;  // ReLU'(0) = 0
+      dY[r * ldd + k] = d;
+      s = fmaf(d, o, s);
+    }
+    s = gb_warp_sum(s);
+    if (lane == 0) c[r] = s;
+  }
+}
+
+template <int LPG, int NJ, int U>
+__global__ void __launch_bounds__(256) k_gat_bwd_a(GatBwdArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w >= a.n_rows) return;
+  const int32_t r = a.order[w];
+  const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
+  const float eli = a.el[r];
+  // online softmax statistics of row r (each lane a strided subset, then merged)
+  float m = -INFINITY, s = 0.f;
+  for (int64_t e = b + lane; e < t; e += 32) {
+    const float ev = gb_lrelu(eli + __ldg(a.er + __ldg(a.col_idx + e)));
+    if (ev > m) {
+      s = s * expf(m - ev) + 1.f;
+      m = ev;
+    } else {
+      s += expf(ev - m);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, o), s2 = __shfl_xor_sync(0xffffffffu, s, o);
+    const float mn = fmaxf(m, m2);
+    s = (m == -INFINITY ? 0.f : s * expf(m - mn)) + (m2 == -INFINITY ? 0.f : s2 * expf(m2 - mn));
+    m = mn;
+  }
+  const float inv_s = s > 0.f ? 1.f / s : 0.f;
+  const float ci = a.c[r];
+  float xv[NJ][4];
+  gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, a.K, xv);
+  float dacc = 0.f;
+  for (int64_t e0 = b; e0 < t; e0 += G * U) {  // warp-uniform trip count
+    int32_t j[U];
+    bool valid[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t e = e0 + u * G + grp;
+      valid[u] = e < t;
+      j[u] = __ldg(a.col_idx + (valid[u] ? e : t - 1));
+    }
+    float zv[U][NJ][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const float d = gb_dot<LPG, NJ>(xv, zv[u]);
+      const float z = eli + __ldg(a.er + j[u]);
+      const float alpha = expf(gb_lrelu(z) - m) * inv_s;
+      const float dz = alpha * (d - ci) * (z > 0.f ? 1.f : 0.2f);
+      if (valid[u] && lg == 0) dacc += dz;
+    }
+  }
+  dacc = gb_warp_sum(dacc);
+  if (lane == 0) {
+    a.del[r] = dacc;
+    a.stat[r] = make_float4(eli, m, inv_s, ci);
+  }
+}
+
+template <int LPG, int NJ, int U>
+__global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w >= a.n_rows) return;
+  const int32_t r = a.order[w];
+  const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
+  const float erj = a.er[r];
+  float zr[NJ][4], acc[NJ][4];
+  gb_load_row<LPG, NJ>(a.Z + (int64_t)r * a.ldz, lg, a.K, zr);
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[j][k] = 0.f;
+  float dracc = 0.f;
+  for (int64_t e0 = b; e0 < t; e0 += G * U) {
+    int32_t i[U];
+    bool valid[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t e = e0 + u * G + grp;
+      valid[u] = e < t;
+      i[u] = __ldg(a.col_idx + (valid[u] ? e : t - 1));
+    }
+    float4 st[U];
+    float xv[U][NJ][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      st[u] = __ldg(a.stat_in + i[u]);
+      gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const float d = gb_dot<LPG, NJ>(xv[u], zr);
+      const float z = st[u].x + erj;
+      const float alpha = valid[u] ? expf(gb_lrelu(z) - st[u].y) * st[u].z : 0.f;
+      const float dz = alpha * (d - st[u].w) * (z > 0.f ? 1.f : 0.2f);
+      if (lg == 0) dracc += dz;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(alpha, xv[u][j][k], acc[j][k]);
+    }
+  }
+#pragma unroll
+  for (int o = LPG; o < 32; o <<= 1)
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) acc[j][k] += __shfl_xor_sync(0xffffffffu, acc[j][k], o);
+  const float der = gb_warp_sum(dracc);
+  const float delj = a.del_in[r];
+  if (grp == 0) {
+    float* o = a.out + (int64_t)r * a.ldo;
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      const int64_t col = 4 * (int64_t)(lg + j * LPG);
+      if (col >= a.K) continue;
+      float v[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int64_t cc = col + k < a.K ? col + k : col;  // clamped read; the value is not stored
+        v[k] = acc[j][k] + delj * __ldg(a.u + cc) + der * __ldg(a.v + cc);
+      }
+      if (a.vec_store && col + 3 < a.K) {
+        *reinterpret_cast<float4*>(o + col) = make_float4(v[0], v[1], v[2], v[3]);
+      } else {
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          if (col + k < a.K) o[col + k] = v[k];
+      }
+    }
+  }
+  if (lane == 0) a.der[r] = der;
+}
+
+template <int LPG, int NJ, int U>
+static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
+  const unsigned blocks = (unsigned)ceil_div(a.n_rows, 8);
+  if (pass == 0)
+    k_gat_bwd_a<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
+  else
+    k_gat_bwd_b<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
+}
+
+granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
+                              bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st) {
+  if (R == 0) return GRANII_OK;
+  ProfScope ps("elementwise", st, 12.0 * R * K + 4.0 * R, 2.0 * R * K, 1);
+  const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 8), 148 * 32));
+  k_gat_prep<<<blocks, 256, 0, st>>>(R, K, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBwdArgs& a, cudaStream_t st) {
+  if (a.n_rows == 0) return GRANII_OK;
+  const int64_t K = a.K;
+  if (K > 2048) return fail(GRANII_ERR_UNSUPPORTED, "GAT backward supports K <= 2048");
+  const double nnz = (double)g->local_nnz, R = (double)a.n_rows;
+  // algorithmic bytes (SURVEY §8(d) SpMM/SDDMM rows): A = col + er + Z row per entry, dX row + 8 B row_ptr
+  // + stat + del per row; B = col + stat + dX row per entry, Z row + out row + ... per row
+  const double bytes = pass == 0 ? nnz * (8.0 + 4.0 * K) + R * (4.0 * K + 8.0 + 28.0)
+                                 : nnz * (20.0 + 4.0 * K) + R * (8.0 * K + 8.0 + 16.0);
+  ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1);
+  if (K <= 16) gb_launch<4, 1, 2>(pass, a, st);
+  else if (K <= 32) gb_launch<8, 1, 2>(pass, a, st);
+  else if (K <= 64) gb_launch<16, 1, 2>(pass, a, st);
+  else if (K <= 128) gb_launch<32, 1, 4>(pass, a, st);
+  else if (K <= 256) gb_launch<32, 2, 2>(pass, a, st);
+  else if (K <= 512) gb_launch<32, 4, 2>(pass, a, st);
+  else if (K <= 1024) gb_launch<32, 8, 1>(pass, a, st);
+  else gb_launch<32, 16, 1>(pass, a, st);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+// ---------------------------------------------------------------- small dense helpers
+// partial[s][2][K] = Σ_{r in chunk s} H[r, :] * (d0[r], d1[r]); block (32, 8), fixed order
+__global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, int64_t ldh,
+                             const float* __restrict__ d0, const float* __restrict__ d1, int64_t chunk,
+                             float* __restrict__ partial) {
+  __shared__ float sp[8][33], sq[8][33];
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int64_t col = blockIdx.x * 32 + tx, s = blockIdx.y;
+  const int64_t r0 = s * chunk, r1 = (r0 + chunk < R) ? r0 + chunk : R;
+  float p = 0.f, q = 0.f;
+  if (col < K)
+    for (int64_t r = r0 + ty; r < r1; r += 8) {
+      const float h = H[r * ldh + col];
+      p = fmaf(h, __ldg(d0 + r), p);
+      q = fmaf(h, __ldg(d1 + r), q);
+    }
+  sp[ty][tx] = p;
+  sq[ty][tx] = q;
+  __syncthreads();
+  if (ty == 0 && col < K) {
+    float a = 0.f, c = 0.f;
+#pragma unroll
+    for (int y = 0; y < 8; ++y) {
+      a += sp[y][tx];
+      c += sq[y][tx];
+    }
+    partial[(s * 2 + 0) * K + col] = a;
+    partial[(s * 2 + 1) * K + col] = c;
+  }
+}
+
+__global__ void k_sum_chunks(int64_t n, int64_t S, const float* __restrict__ partial, float* __restrict__ out) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  float a = 0.f;
+  for (int64_t s = 0; s < S; ++s) a += partial[s * n + i];
+  out[i] = a;
+}
+
+static int64_t colreduce_chunks(int64_t R, int64_t K) {
+  const int64_t tiles = ceil_div(K, 32);
+  return std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 512), ceil_div(148 * 8, tiles)));
+}
+
+size_t colreduce2_workspace(int64_t R, int64_t K) { return (size_t)colreduce_chunks(R, K) * 2 * K * sizeof(float); }
+
+granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ldh, const float* d0, const float* d1,
+                                float* partial, float* out, cudaStream_t st) {
+  const int64_t S = colreduce_chunks(R, K), chunk = ceil_div(std::max<int64_t>(R, 1), S);
+  ProfScope ps("elementwise", st, 4.0 * R * K + 8.0 * R, 4.0 * R * K, 2);
+  k_colreduce2<<<dim3((unsigned)ceil_div(K, 32), (unsigned)S), dim3(32, 8), 0, st>>>(R, K, H, ldh, d0, d1, chunk,
+                                                                                   partial);
+  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, partial, out);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+// u = W a_l, v = W a_r (W: K1 x K2, ld K2); warp per row of W
+__global__ void k_matvec2(int64_t K1, int64_t K2, const float* __restrict__ W, const float* __restrict__ al,
+                          const float* __restrict__ ar, float* __restrict__ u, float* __restrict__ v) {
+  const int lane = threadIdx.x & 31;
+  const int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (r >= K1) return;
+  float a = 0.f, b = 0.f;
+  for (int64_t k = lane; k < K2; k += 32) {
+    const float x = W[r * K2 + k];
+    a = fmaf(x, al[k], a);
+    b = fmaf(x, ar[k], b);
+  }
+  a = gb_warp_sum(a);
+  b = gb_warp_sum(b);
+  if (lane == 0) {
+    u[r] = a;
+    v[r] = b;
+  }
+}
+
+// da_l = Wᵀ p, da_r = Wᵀ q (thread per column of W, fixed order over rows)
+__global__ void k_mattvec2(int64_t K1, int64_t K2, const float* __restrict__ W, const float* __restrict__ p,
+                           const float* __restrict__ q, float* __restrict__ dal, float* __restrict__ dar) {
+  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (k >= K2) return;
+  float a = 0.f, b = 0.f;
+  for (int64_t r = 0; r < K1; ++r) {
+    const float x = W[r * K2 + k];
+    a = fmaf(x, p[r], a);
+    b = fmaf(x, q[r], b);
+  }
+  if (dal) dal[k] = a;
+  if (dar) dar[k] = b;
+}
+
+// dW += p a_lᵀ + q a_rᵀ
+__global__ void k_rank2(int64_t K1, int64_t K2, float* __restrict__ dW, const float* __restrict__ p,
+                        const float* __restrict__ q, const float* __restrict__ al, const float* __restrict__ ar) {
+  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= K1 * K2) return;
+  const int64_t r = i / K2, k = i % K2;
+  dW[i] += p[r] * al[k] + q[r] * ar[k];
+}
+
+granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const float* a_l, const float* a_r,
+                                float* u, float* v, cudaStream_t st) {
+  ProfScope ps("elementwise", st, 4.0 * K1 * K2, 4.0 * K1 * K2, 1);
+  k_matvec2<<<(unsigned)ceil_div(K1, 8), 256, 0, st>>>(K1, K2, W, a_l, a_r, u, v);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* p, const float* q,
+                                  float* da_l, float* da_r, cudaStream_t st) {
+  ProfScope ps("elementwise", st, 4.0 * K1 * K2, 4.0 * K1 * K2, 1);
+  k_mattvec2<<<(unsigned)ceil_div(K2, 128), 128, 0, st>>>(K1, K2, W, p, q, da_l, da_r);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p, const float* q, const float* a_l,
+                               const float* a_r, cudaStream_t st) {
+  ProfScope ps("elementwise", st, 8.0 * K1 * K2, 4.0 * K1 * K2, 1);
+  k_rank2<<<(unsigned)ceil_div(K1 * K2, 256), 256, 0, st>>>(K1, K2, dW, p, q, a_l, a_r);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+}  // namespace granii

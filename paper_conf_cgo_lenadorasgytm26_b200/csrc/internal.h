@@ -117,6 +117,43 @@ granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_
                                int64_t ldg, float* dst, int64_t ldd, cudaStream_t st);
 granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,
                                cudaStream_t st);
+// GAT backward (gat_bwd.cu); pass 0 = rows i (del, stat), pass 1 = rows j (transposed SpMM, der)
+struct GatBwdArgs {
+  int64_t n_rows = 0;
+  const int64_t* row_ptr = nullptr;
+  const int32_t* col_idx = nullptr;
+  const int32_t* order = nullptr;
+  int64_t K = 0;
+  const float* dX = nullptr;  // pass 0: own rows; pass 1: column-id space
+  int64_t ldx = 0;
+  const float* Z = nullptr;   // pass 0: column-id space; pass 1: own rows
+  int64_t ldz = 0;
+  const float* el = nullptr;  // pass 0: own rows
+  const float* er = nullptr;  // pass 0: column-id space; pass 1: own rows
+  const float* c = nullptr;   // pass 0: own rows
+  float4* stat = nullptr;     // pass 0 out: {el, m, 1/s, c} per own row
+  const float4* stat_in = nullptr;  // pass 1: column-id space
+  float* del = nullptr;       // pass 0 out
+  const float* del_in = nullptr;    // pass 1: own rows
+  float* der = nullptr;       // pass 1 out
+  const float* u = nullptr;   // pass 1 epilogue vectors (K)
+  const float* v = nullptr;
+  float* out = nullptr;       // pass 1 out (own rows x K, ld ldo)
+  int64_t ldo = 0;
+  int vec_store = 0;
+};
+granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
+                              bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st);
+granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBwdArgs& a, cudaStream_t st);
+size_t colreduce2_workspace(int64_t R, int64_t K);
+granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ldh, const float* d0, const float* d1,
+                                float* partial, float* out, cudaStream_t st);
+granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const float* a_l, const float* a_r,
+                                float* u, float* v, cudaStream_t st);
+granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* p, const float* q,
+                                  float* da_l, float* da_r, cudaStream_t st);
+granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p, const float* q, const float* a_l,
+                               const float* a_r, cudaStream_t st);
 // comm
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);

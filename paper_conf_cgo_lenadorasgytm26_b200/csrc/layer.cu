@@ -89,6 +89,20 @@ static granii_status gemm_ws(Bump& b, int64_t M, int64_t N, int64_t K, uint32_t 
   return GRANII_OK;
 }
 
+// saved state of a GAT layer: [Θ (REUSE, R x ld4(K2)) | T = α H (RECOMP, R x ld4(K1))][el: R][er: R]
+struct GatSaved {
+  int64_t ldz, el, er;
+  size_t floats;
+};
+static GatSaved gat_saved_layout(int64_t R, granii_composition comp, int64_t K1, int64_t K2) {
+  GatSaved s;
+  s.ldz = ld4(comp == GRANII_GAT_REUSE ? K2 : K1);
+  s.el = R * s.ldz;
+  s.er = s.el + round_up(R, 4);
+  s.floats = (size_t)(s.er + round_up(R, 4));
+  return s;
+}
+
 // ---------------------------------------------------------------- forward (plan + run)
 // Running with base == nullptr only sizes the workspace (no launches).
 static granii_status forward_impl(const Ctx& c, granii_model m, granii_composition comp, const granii_layer_args* a,
@@ -179,13 +193,23 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     const bool dot = a->attn == GRANII_ATTN_DOT;
     float* alpha = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
     const bool need_theta = comp == GRANII_GAT_REUSE || dot;
+    // state kept for the backward (gat_saved_layout): Θ (REUSE) or T = α H (RECOMP), el, er
+    const GatSaved sv = gat_saved_layout(R, comp, K1, K2);
+    if (saved_floats) *saved_floats = sv.floats;
     GatherBuf th;
-    if (need_theta) th = gather_buf(b, c, K2);
+    if (need_theta) {
+      if (saved && comp == GRANII_GAT_REUSE && !c.dist()) {
+        th.ld = ld4(K2);
+        th.all = th.mine = saved;  // Θ goes straight into the saved state
+      } else {
+        th = gather_buf(b, c, K2);
+      }
+    }
     float* el = nullptr;
     float* er_all = nullptr;
     if (!dot) {
-      el = b.take((size_t)std::max<int64_t>(R, 1));
-      er_all = vec_buf(b, c);
+      el = saved ? saved + sv.el : b.take((size_t)std::max<int64_t>(R, 1));
+      er_all = (saved && !c.dist()) ? saved + sv.er : vec_buf(b, c);
     }
     void* gw;
     size_t gn;
@@ -196,6 +220,12 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       uint32_t fl = need_theta ? 0u : GRANII_GEMM_NO_STORE;
       GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, need_theta ? th.mine : nullptr, need_theta ? th.ld : K2,
                          &ep, fl, gw, gn, st));
+      if (saved && c.dist()) {  // keep this rank's Θ rows and er for the backward
+        if (comp == GRANII_GAT_REUSE)
+          GR_CUDA(cudaMemcpyAsync(saved, th.mine, sizeof(float) * (size_t)R * th.ld, cudaMemcpyDeviceToDevice, st));
+        if (!dot)
+          GR_CUDA(cudaMemcpyAsync(saved + sv.er, er_mine, sizeof(float) * (size_t)R, cudaMemcpyDeviceToDevice, st));
+      }
       if (need_theta) GR_TRY(allgather(c, th));
       if (!dot) {
         if (c.dist()) {
@@ -214,7 +244,7 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       if (run) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
     } else {
       const int64_t ldt = ld4(K1);
-      float* T = b.take((size_t)std::max<int64_t>(R, 1) * ldt);
+      float* T = saved ? saved : b.take((size_t)std::max<int64_t>(R, 1) * ldt);
       void* gw2;
       size_t gn2;
       gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
@@ -313,6 +343,174 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
   return GRANII_OK;
 }
 
+// ---------------------------------------------------------------- GAT backward (N2, reading R22; gat_bwd.cu)
+// REUSE  : dY ; pass A (dα = <dY_i, Θ_j>) ; pass B -> dΘ = αᵀ dY + del a_lᵀ + der a_rᵀ ;
+//          dW = Hᵀ dΘ ; dH = dΘ Wᵀ
+// RECOMP : dY ; dT = dY Wᵀ ; pass A (dα = <dT_i, H_j>) ; pass B -> dH = αᵀ dT + del (W a_l)ᵀ + der (W a_r)ᵀ ;
+//          dW = Tᵀ dY + (Hᵀ del) a_lᵀ + (Hᵀ der) a_rᵀ
+// both   : da_l = Wᵀ Hᵀ del, da_r = Wᵀ Hᵀ der
+// Multi-GPU: the gathered operands are er, Θ or H (pass A), dY or dT and the 16-byte row
+// records (pass B); dW and Hᵀ[del, der] are all-reduced.
+static GatherBuf local_buf(Bump& b, int64_t R, int64_t K) {
+  GatherBuf gb;
+  gb.ld = ld4(K);
+  gb.all = gb.mine = b.take((size_t)std::max<int64_t>(R, 1) * gb.ld);
+  return gb;
+}
+
+static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, const granii_layer_args* a,
+                                       const float* out, int64_t ldo, const float* dout, int64_t lddo,
+                                       const float* saved, float* dH, int64_t lddh, float* dW, void* ws_base,
+                                       size_t* ws_size) {
+  const granii_graph_s* g = c.g;
+  const bool run = ws_base != nullptr;
+  Bump b(ws_base);
+  const int64_t R = g->n_rows, K1 = a->K1, K2 = a->K2, Rr = std::max<int64_t>(R, 1);
+  const cudaStream_t st = c.st;
+  const bool relu = a->act == GRANII_ACT_RELU;
+  const bool reuse = comp == GRANII_GAT_REUSE;
+  const GatSaved sv = gat_saved_layout(R, comp, K1, K2);
+  if (run && !saved) return fail(GRANII_ERR_INVALID_ARG, "GAT backward needs d_saved from the forward");
+  const float* el = saved ? saved + sv.el : nullptr;
+  const float* er_own = saved ? saved + sv.er : nullptr;
+
+  // aligned H (own rows) and, for RECOMP on several GPUs, its gathered copy
+  const float* H = a->H;
+  int64_t ldh = a->ldh;
+  const bool h_aligned = (ldh % 4 == 0) && (((uintptr_t)H & 15) == 0);
+  GatherBuf hg;
+  const bool h_gather = !reuse && c.dist();
+  if (h_gather) {
+    hg = gather_buf(b, c, K1);
+    if (run) {
+      GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hg.mine, hg.ld, st));
+      GR_TRY(allgather(c, hg));
+    }
+    H = hg.mine;
+    ldh = hg.ld;
+  } else if (!h_aligned) {
+    float* hpad = b.take((size_t)Rr * ld4(K1));
+    if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hpad, ld4(K1), st));
+    H = hpad;
+    ldh = ld4(K1);
+  }
+  const float* H_all = h_gather ? hg.all : H;
+
+  GatherBuf dyg = reuse ? gather_buf(b, c, K2) : local_buf(b, R, K2);
+  GatherBuf dtg;
+  if (!reuse) dtg = gather_buf(b, c, K1);
+  float* cvec = b.take((size_t)Rr);
+  float* del = b.take((size_t)Rr);
+  float* der = b.take((size_t)Rr);
+  float* statb = b.take((size_t)4 * (c.dist() ? g->n_cols : Rr));
+  float* stat_mine = (c.dist() && statb) ? statb + (int64_t)4 * g->rank * g->max_rows : statb;
+  float* er_all = c.dist() ? vec_buf(b, c) : const_cast<float*>(er_own);
+  GatherBuf thg;  // REUSE: Θ in the column-id space
+  if (reuse) {
+    if (c.dist()) {
+      thg = gather_buf(b, c, K2);
+    } else {
+      thg.ld = sv.ldz;
+      thg.all = thg.mine = const_cast<float*>(saved);
+    }
+  }
+  float* bout = nullptr;  // pass B output
+  int64_t ldbo = 0;
+  if (reuse) {
+    bout = b.take((size_t)Rr * ld4(K2));
+    ldbo = ld4(K2);
+  } else if (dH) {
+    bout = dH;
+    ldbo = lddh;
+  } else {
+    bout = b.take((size_t)Rr * ld4(K1));
+    ldbo = ld4(K1);
+  }
+  float* uv = reuse ? nullptr : b.take((size_t)2 * K1);
+  float* pq = b.take((size_t)2 * K1);
+  float* partial = (float*)b.take_bytes(colreduce2_workspace(R, K1));
+  void* gwW;
+  size_t gnW;
+  gemm_ws(b, K1, K2, R, GRANII_GEMM_TRANS_A, &gwW, &gnW);
+  void* gwH;
+  size_t gnH;
+  gemm_ws(b, R, K1, K2, GRANII_GEMM_TRANS_B, &gwH, &gnH);
+
+  if (run) {
+    GR_TRY(launch_gat_prep(R, K2, out, ldo, dout, lddo, relu, dyg.mine, dyg.ld, cvec, st));
+    if (c.dist()) {
+      float* er_slot = er_all + (int64_t)g->rank * g->max_rows;
+      GR_CUDA(cudaMemcpyAsync(er_slot, er_own, sizeof(float) * (size_t)R, cudaMemcpyDeviceToDevice, st));
+      GR_TRY(comm_allgather(c.comm, er_slot, er_all, (size_t)g->max_rows, st));
+      if (reuse) {
+        GR_CUDA(cudaMemcpyAsync(thg.mine, saved, sizeof(float) * (size_t)R * sv.ldz, cudaMemcpyDeviceToDevice, st));
+        GR_TRY(allgather(c, thg));
+      }
+    }
+    if (!reuse)
+      GR_TRY(launch_gemm(R, K1, K2, dyg.mine, dyg.ld, a->W, K2, dtg.mine, dtg.ld, nullptr, GRANII_GEMM_TRANS_B, gwH,
+                         gnH, st));
+    GatBwdArgs pa;
+    pa.n_rows = R;
+    pa.row_ptr = g->row_ptr;
+    pa.col_idx = g->col_idx;
+    pa.order = g->order;
+    pa.K = reuse ? K2 : K1;
+    pa.dX = reuse ? dyg.mine : dtg.mine;
+    pa.ldx = reuse ? dyg.ld : dtg.ld;
+    pa.Z = reuse ? thg.all : H_all;
+    pa.ldz = reuse ? thg.ld : ldh;
+    pa.el = el;
+    pa.er = er_all;
+    pa.c = cvec;
+    pa.stat = reinterpret_cast<float4*>(stat_mine);
+    pa.del = del;
+    GR_TRY(launch_gat_bwd_pass(g, 0, pa, st));
+    if (c.dist()) {
+      GR_TRY(comm_allgather(c.comm, stat_mine, statb, (size_t)4 * g->max_rows, st));
+      GR_TRY(allgather(c, reuse ? dyg : dtg));
+    }
+    if (!reuse) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
+    GatBwdArgs pb;
+    pb.n_rows = R;
+    pb.row_ptr = g->row_ptr;
+    pb.col_idx = g->col_idx;
+    pb.order = g->order;
+    pb.K = pa.K;
+    pb.dX = reuse ? dyg.all : dtg.all;
+    pb.ldx = pa.ldx;
+    pb.Z = reuse ? saved : H;
+    pb.ldz = reuse ? sv.ldz : ldh;
+    pb.er = er_own;
+    pb.stat_in = reinterpret_cast<const float4*>(statb);
+    pb.del_in = del;
+    pb.der = der;
+    pb.u = reuse ? a->a_l : uv;
+    pb.v = reuse ? a->a_r : uv + K1;
+    pb.out = bout;
+    pb.ldo = ldbo;
+    pb.vec_store = (ldbo % 4 == 0) && (((uintptr_t)bout & 15) == 0);
+    GR_TRY(launch_gat_bwd_pass(g, 1, pb, st));
+    if (reuse) {
+      GR_TRY(launch_gemm(K1, K2, R, H, ldh, bout, ldbo, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
+      if (dH)
+        GR_TRY(launch_gemm(R, K1, K2, bout, ldbo, a->W, K2, dH, lddh, nullptr, GRANII_GEMM_TRANS_B, gwH, gnH, st));
+    } else {
+      GR_TRY(launch_gemm(K1, K2, R, saved, sv.ldz, dyg.mine, dyg.ld, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW,
+                         st));
+    }
+    GR_TRY(launch_colreduce2(R, K1, H, ldh, del, der, partial, pq, st));
+    if (c.dist()) {
+      GR_TRY(comm_allreduce_sum(c.comm, dW, (size_t)K1 * K2, st));
+      GR_TRY(comm_allreduce_sum(c.comm, pq, (size_t)2 * K1, st));
+    }
+    if (!reuse) GR_TRY(launch_gat_rank2(K1, K2, dW, pq, pq + K1, a->a_l, a->a_r, st));
+    if (a->d_a_l || a->d_a_r) GR_TRY(launch_gat_mattvec2(K1, K2, a->W, pq, pq + K1, a->d_a_l, a->d_a_r, st));
+  }
+  if (ws_size) *ws_size = b.off + 1024;
+  return GRANII_OK;
+}
+
 granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_composition comp, int64_t K1,
                               int64_t K2, size_t* ws, size_t* saved_floats) {
   // size for the distributed layout whenever the graph is partitioned
@@ -335,6 +533,8 @@ granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_co
   }
   if (m == GRANII_GCN)
     GR_TRY(backward_impl(c, comp, &a, nullptr, K2, nullptr, K2, nullptr, (float*)1, K1, nullptr, nullptr, &bwd));
+  else
+    GR_TRY(gat_backward_impl(c, comp, &a, nullptr, K2, nullptr, K2, nullptr, nullptr, K1, nullptr, nullptr, &bwd));
   *ws = std::max(f, bwd);
   if (saved_floats) *saved_floats = sf;
   return GRANII_OK;
@@ -354,9 +554,10 @@ granii_status layer_backward(const granii_graph_s* g, granii_composition comp, c
                              float* dH, int64_t lddh, float* dW, cudaStream_t st) {
   Ctx c{g, a->comm, st};
   size_t need = 0;
-  GR_TRY(backward_impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, nullptr, &need));
+  auto impl = (comp == GRANII_GAT_REUSE || comp == GRANII_GAT_RECOMP) ? gat_backward_impl : backward_impl;
+  GR_TRY(impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, nullptr, &need));
   if (a->workspace_bytes < need) return fail(GRANII_ERR_INVALID_ARG, "layer workspace too small");
-  return backward_impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, a->workspace, &need);
+  return impl(c, comp, a, out, ldo, dout, lddo, saved, dH, lddh, dW, a->workspace, &need);
 }
 
 }  // namespace granii

@@ -56,7 +56,8 @@ class gemm_epilogue(ctypes.Structure):
 
 class layer_args(ctypes.Structure):
     _fields_ = [("K1", _i64), ("K2", _i64), ("H", _p), ("ldh", _i64), ("W", _p), ("a_l", _p), ("a_r", _p),
-                ("act", _u32), ("attn", _u32), ("workspace", _p), ("workspace_bytes", _sz), ("comm", _p)]
+                ("act", _u32), ("attn", _u32), ("workspace", _p), ("workspace_bytes", _sz), ("comm", _p),
+                ("d_a_l", _p), ("d_a_r", _p)]
 
 
 _SIGS = {
@@ -149,7 +150,7 @@ class Graph:
         self.info = granii_graph_query(handle)
 
     def __del__(self):
-        if getattr(self, "handle", None):
+        if getattr(self, "handle", None) and _lib is not None:  # _lib is None at interpreter shutdown
             _lib.granii_graph_destroy(self.handle)
             self.handle = None
 
@@ -258,9 +259,11 @@ def granii_layer_workspace_size(g: Graph, model: int, comp: int, K1: int, K2: in
 
 
 def make_layer_args(K1, K2, H, W, a_l=None, a_r=None, act=ACT_RELU, attn=ATTN_ADDITIVE, workspace=None,
-                    comm=None) -> layer_args:
+                    comm=None, d_a_l=None, d_a_r=None) -> layer_args:
+    """d_a_l / d_a_r: GAT backward outputs (dL/da_l, dL/da_r), ignored by the forward."""
     return layer_args(K1, K2, _ptr(H), _ld(H), _ptr(W), _ptr(a_l), _ptr(a_r), act, attn, _ptr(workspace),
-                      workspace.numel() if workspace is not None else 0, comm.handle if comm is not None else None)
+                      workspace.numel() if workspace is not None else 0, comm.handle if comm is not None else None,
+                      _ptr(d_a_l), _ptr(d_a_r))
 
 
 def granii_layer_forward(g: Graph, model: int, comp: int, args: layer_args, out: torch.Tensor, saved=None,

@@ -75,10 +75,16 @@ class GNN:
                       for s in self.saved_floats]
         self.grads_out = [alloc2d(R, L.K2, device) for L in layers]     # dL/d out_l
         self.dW = [torch.empty((L.K1, L.K2), dtype=torch.float32, device=device) for L in layers]
+        # dL/da_l, dL/da_r of the GAT layers (None for GCN)
+        self.da = [(torch.empty(L.K2, dtype=torch.float32, device=device),
+                    torch.empty(L.K2, dtype=torch.float32, device=device)) if L.model == G.GAT else None
+                   for L in layers]
 
     def args(self, i: int, H: torch.Tensor) -> G.layer_args:
         L = self.layers[i]
-        return G.make_layer_args(L.K1, L.K2, H, L.W, L.a_l, L.a_r, L.act, L.attn, self.workspace, self.comm)
+        da = self.da[i] or (None, None)
+        return G.make_layer_args(L.K1, L.K2, H, L.W, L.a_l, L.a_r, L.act, L.attn, self.workspace, self.comm,
+                                 da[0], da[1])
 
     def forward(self, H: torch.Tensor) -> torch.Tensor:
         x = H
@@ -90,7 +96,7 @@ class GNN:
         return x
 
     def backward(self, dout_last: torch.Tensor, need_input_grad: bool = False):
-        """Backward through all layers (GCN only, L340); fills self.dW."""
+        """Backward through all layers (L340; GAT additive attention, R22); fills self.dW and self.da."""
         dout = dout_last
         for i in range(len(self.layers) - 1, -1, -1):
             L = self.layers[i]
@@ -107,6 +113,9 @@ class GNN:
         Z = self.forward(H)
         G.granii_softmax_xent(Z, labels, n_total, dlogits, loss)
         self.backward(dlogits)
-        for L, dW in zip(self.layers, self.dW):
+        for L, dW, da in zip(self.layers, self.dW, self.da):
             G.granii_sgd(dW, L.W, lr)
+            if da is not None:
+                G.granii_sgd(da[0], L.a_l, lr)
+                G.granii_sgd(da[1], L.a_r, lr)
         return Z

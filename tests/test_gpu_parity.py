@@ -408,6 +408,53 @@ def test_gcn_backward_every_composition(G, comp, name, K1, K2):
     assert err(dH.cpu(), rdH) <= TOL
 
 
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("name,K1,K2,act", [("pubmed", 32, 256, 1), ("pubmed", 64, 128, 0), ("dense", 48, 16, 1),
+                                             ("tiny", 3, 5, 0), ("sparse", 128, 47, 1), ("dense", 256, 1024, 0)])
+def test_gat_backward_both_compositions(G, comp, name, K1, K2, act):
+    """N2 (reading R22): dW, dH, da_l, da_r of both compositions against the oracle's chain rule"""
+    c = case(G, name)
+    net, out, H, W, al, ar = run_layer(G, c, G.GAT, comp, K1, K2, act, aligned=(K1 % 4 == 0))
+    Gup = synth.uniform_pm1(61, 1, (c.n, K2))
+    if act:
+        Y, _ = O.gat_forward(comp, c.rp, c.ci, H, W, al, ar, 0)
+        Gup[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0  # R20
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    ref = O.gat_backward(comp, c.rp, c.ci, H, W, al, ar, Gup, act)
+    mag = O.gat_backward_magnitude(comp, c.rp, c.ci, H, W, al, ar, Gup, act)
+    got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
+    for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, ref, mag):
+        assert gat_grad_ok(y.cpu(), r, m), nm
+
+
+def gat_grad_ok(y, r, m):
+    """R22: per row, |y - r|∞ <= 1e-4 |r|∞ + 4u |m|∞ (u = 2^-24, m = the computation's magnitude):
+    the softmax backward α(dα - Σα dα) cancels by construction on near-one-hot rows, and a fp32
+    path cannot resolve the difference below u·|dα|; elsewhere m ~ |r| and this is R19's 1e-4.
+    The worst-case bound grows linearly with the number of cancelling rows, so a 1e-3 normwise
+    guard is kept for the strongly cancelling aggregates (da = Θᵀ del over all rows)"""
+    y, r, m = (np.atleast_2d(np.asarray(x, np.float64)) for x in (y, r, m))
+    d = np.abs(y - r).max(1)
+    ok = d <= TOL * np.abs(r).max(1) + 4 * 2.0 ** -24 * m.max(1)
+    assert normwise(y, r) <= 10 * TOL
+    return bool(ok.all())
+
+
+def test_gat_backward_deterministic_and_input_layer(G):
+    c = case(G, "dense")
+    runs = []
+    for need in (True, True, False):
+        net, out, H, W, al, ar = run_layer(G, c, G.GAT, 16, 64, 128, G.ACT_RELU)
+        Gup = synth.uniform_pm1(62, 1, (c.n, 128))
+        dH = net.backward(pad(Gup), need_input_grad=need)
+        torch.cuda.synchronize()
+        runs.append((net.dW[0].clone(), net.da[0][0].clone(), None if dH is None else dH.clone()))
+    assert torch.equal(runs[0][0], runs[1][0]) and torch.equal(runs[0][1], runs[1][1])
+    assert torch.equal(runs[0][2], runs[1][2])
+    assert torch.equal(runs[0][0], runs[2][0]) and runs[2][2] is None   # no dH: same dW
+
+
 def test_layer_determinism_and_comp_agreement(G):
     c = case(G, "dense")
     outs = []

@@ -444,6 +444,28 @@ def test_gat_backward_compositions_agree_and_closed_forms():
     assert rel(dW, (A @ H).T @ G) < 1e-12 and rel(dH, A.T @ G @ W.T) < 1e-12
 
 
+@pytest.mark.parametrize("K1,K2", [(5, 7), (7, 5)])
+def test_gat_backward_magnitude_bounds_and_closed_form(K1, K2):
+    """the tolerance scale dominates every gradient entry (triangle inequality) and equals the
+    gradient when nothing can cancel (H, W, G >= 0, a_l = a_r = 0: dW = (αH)ᵀG, dH = αᵀ G Wᵀ)"""
+    rp, ci, _ = csr_and_dense(65, n=60, m=300)
+    rng = np.random.default_rng(18)
+    H, W = rng.uniform(-1, 1, (60, K1)), rng.uniform(-1, 1, (K1, K2))
+    al, ar = rng.uniform(-1, 1, K2), rng.uniform(-1, 1, K2)
+    G = rng.standard_normal((60, K2))
+    for comp in O.GAT_COMPS:
+        for act in (0, 1):
+            g = O.gat_backward(comp, rp, ci, H, W, al, ar, G, act)
+            m = O.gat_backward_magnitude(comp, rp, ci, H, W, al, ar, G, act)
+            for x, y in zip(g, m):
+                assert np.all(np.abs(x) <= y * (1 + 1e-12) + 1e-300)
+    Hp, Wp, Gp, z = np.abs(H), np.abs(W), np.abs(G), np.zeros(K2)
+    for comp in O.GAT_COMPS:
+        g = O.gat_backward(comp, rp, ci, Hp, Wp, z, z, Gp, 0)
+        m = O.gat_backward_magnitude(comp, rp, ci, Hp, Wp, z, z, Gp, 0)
+        assert rel(m[0], g[0]) < 1e-13 and rel(m[1], g[1]) < 1e-13
+
+
 # ------------------------------------------------------------------ generators
 def test_generator_is_device_independent_and_exact():
     a = synth.uniform_pm1(3, 4, (1000,))
