@@ -43,6 +43,8 @@ WORKLOADS = {
     "products-gat2-infer": dict(graph="products", model="gat", dims=[100, 256, 47], train=False),
     "arxiv-gat-infer": dict(graph="arxiv", model="gat", dims=[64, 256], train=False),
     "pubmed-gcn2-train": dict(graph="pubmed", model="gcn", dims=[256, 32, 32], train=True),
+    "products-gat2-train": dict(graph="products", model="gat", dims=[100, 256, 47], train=True),
+    "pubmed-gat2-train": dict(graph="pubmed", model="gat", dims=[64, 256, 32], train=True),
 }
 
 
@@ -129,32 +131,37 @@ def time_region(fn, steps, stream):
     return a.elapsed_time(b) / steps
 
 
-def host_csr(n, src, dst):
+def host_csr(n, src, dst, symmetrize=True):
     import oracle as O
-    return O.csr_build(n, src.cpu(), dst.cpu(), O.ADD_SELF_LOOPS | O.SYMMETRIZE)
+    return O.csr_build(n, src.cpu(), dst.cpu(), O.ADD_SELF_LOOPS | (O.SYMMETRIZE if symmetrize else 0))
 
 
-def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0):
-    """fp64 oracle (per-row definition of every layer, oracle_gcn_rows) on a row sample."""
+def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn"):
+    """fp64 oracle (per-row definition of every layer, oracle_gcn_rows / oracle_gat_rows) on a row sample."""
     import oracle as O
     n = rp.shape[0] - 1
     deg = np.diff(rp)
     rng = np.random.default_rng(seed)
     feats = [synth.features(seed + 7, n, k).numpy() for k in dims[:-1]]
     Ws = [synth.glorot(seed + 2, i, dims[i], dims[i + 1], (dims[i], dims[i + 1])).numpy() for i in range(len(dims) - 1)]
+    atts = [(synth.uniform_pm1(seed + 3, 2 * i, (dims[i + 1],)).numpy(),
+             synth.uniform_pm1(seed + 3, 2 * i + 1, (dims[i + 1],)).numpy()) for i in range(len(dims) - 1)]
     S = 256
     while True:
         rows = np.sort(rng.choice(n, size=min(S, n), replace=False))
         t0 = time.perf_counter()
         for i in range(len(dims) - 1):
-            O.gcn_rows(rows, rp, ci, deg, feats[i], Ws[i], 1)
+            if model == "gcn":
+                O.gcn_rows(rows, rp, ci, deg, feats[i], Ws[i], 1)
+            else:
+                O.gat_rows(rows, rp, ci, feats[i], Ws[i], atts[i][0], atts[i][1], 1)
         dt = time.perf_counter() - t0
         if dt >= target_s or S >= n:
             break
         S = int(min(n, S * max(2.0, min(16.0, 1.2 * target_s / max(dt, 1e-3)))))
     edges = float(deg[rows].sum()) * (len(dims) - 1)
     return {"value": edges / dt, "unit": "edges/s", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
-            "sample": f"fp64 oracle per-row forward (oracle_gcn_rows) of all {len(dims) - 1} layers on {rows.size} "
+            "sample": f"fp64 oracle per-row forward (oracle_{model}_rows) of all {len(dims) - 1} layers on {rows.size} "
                       f"random rows ({int(deg[rows].sum())} stored entries) of the same graph; backward not included",
             "seconds": dt}
 
@@ -377,8 +384,8 @@ def main():
     # ---------------------------------------------------------------- CPU oracle baseline
     if rank == 0 and world == 1 and not args.no_cpu:
         try:
-            rp, ci = host_csr(w.n, src, dst)
-            result["cpu_baseline"] = cpu_oracle_sample(rp, ci, dims)
+            rp, ci = host_csr(w.n, src, dst, w.symmetrize)
+            result["cpu_baseline"] = cpu_oracle_sample(rp, ci, dims, model=spec["model"])
         except Exception as e:  # never fail the bench on the baseline
             result["cpu_baseline"] = {"value": None, "error": str(e)[:200]}
 
@@ -409,7 +416,7 @@ def regret(G, spec, g, dev, comm, H, world, dist):
         ar = synth.uniform_pm1(9, 2 * i + 1, (k2,), device=dev)
         if x.shape[1] != k1:
             x = alloc2d(g.n_rows, k1, dev, fill=0.5)
-        train = spec["train"] and model == G.GCN
+        train = spec["train"]
         need_dH = i > 0                      # the input layer needs no dH (training)
         fl = (G.SELECT_TRAINING | (0 if need_dH else G.SELECT_INPUT_LAYER)) if train else 0
         calib = DEFAULT_CALIB if os.path.exists(DEFAULT_CALIB) else None
@@ -464,15 +471,15 @@ def run_reference(args, spec, w, world, rank):
     dims = spec["dims"]
     src, dst = w.edges(seed=0)
     t0 = time.perf_counter()
-    rp, ci = host_csr(w.n, src, dst)
+    rp, ci = host_csr(w.n, src, dst, w.symmetrize)
     t_csr = time.perf_counter() - t0
     budget = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
     res = None
     for _ in range(args.warmup):
-        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4)
+        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4, model=spec["model"])
     vals, secs = [], []
     for _ in range(args.steps):
-        res = cpu_oracle_sample(rp, ci, dims, target_s=budget)
+        res = cpu_oracle_sample(rp, ci, dims, target_s=budget, model=spec["model"])
         vals.append(res["value"])
         secs.append(res["seconds"])
     value = float(np.mean(vals))

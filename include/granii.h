@@ -281,7 +281,8 @@ granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t 
 /* Calibration support: the feature vector the cost model of primitive `prim`
  * (0 spmm weighted, 1 spmm unweighted, 2 spmm unweighted + column scale,
  * 3 sddmm K=1, 4 sddmm K=1 + softmax, 5 gemm, 6 gemm without store, 7 gemm Aᵀ·B,
- * 8 elementwise, 9 all-gather, 10 gemm with the GAT attention GEMVs) uses for this graph and widths (K1, K2);
+ * 8 elementwise, 9 all-gather, 10 gemm with the GAT attention GEMVs, 11 / 12 GAT backward passes A / B)
+ * uses for this graph and widths (K1, K2);
  * feats has room for 8 values; model_name (32 bytes) receives the model key
  * the coefficients are stored under in the calibration file. */
 granii_status granii_cost_features(granii_graph g, int32_t prim, int64_t K1, int64_t K2, double* feats,

@@ -12,9 +12,9 @@
 //                                                 RECOMP: dH with u,v = W a_l, W a_r)
 // B200 design: two warp-per-row passes in the degree-descending schedule,
 // both gathers of K-wide rows (the SpMM's access pattern):
-//   pass A (rows i): online softmax statistics (m_i, s_i) from the er gathers,
-//     then dα by K-wide gathers of Z_j; writes del_i and the row record
-//     stat_i = {el_i, m_i, 1/s_i, c_i} (one 16-byte gather per edge in pass B).
+//   pass A (rows i): one sweep of K-wide gathers of Z_j for dα with an online
+//     softmax (running max, Σ exp, Σ exp·(dα - c)·LeakyReLU'); writes del_i and the
+//     row record stat_i = {el_i, m_i, 1/s_i, c_i} (one 16-byte gather per edge in pass B).
 //   pass B (rows j, symmetric Ã: row j lists every i with j in N(i)): gathers
 //     stat_i and dX_i, recomputes α_ij from the record (α is never stored),
 //     dots dX_i with the register-resident Z_j, accumulates the transposed
@@ -54,15 +54,15 @@ __device__ __forceinline__ void gb_load_row(const float* __restrict__ p, int lg,
   }
 }
 
-template <int LPG, int NJ>
-__device__ __forceinline__ float gb_dot(const float (&x)[NJ][4], const float (&y)[NJ][4]) {
+// this lane's share of <x, y>; never reduced per entry: every use is linear in the dot, so
+// the lane shares are accumulated and reduced once per row
+template <int NJ>
+__device__ __forceinline__ float gb_pdot(const float (&x)[NJ][4], const float (&y)[NJ][4]) {
   float d = 0.f;
 #pragma unroll
   for (int j = 0; j < NJ; ++j)
 #pragma unroll
     for (int k = 0; k < 4; ++k) d = fmaf(x[j][k], y[j][k], d);
-#pragma unroll
-  for (int o = LPG / 2; o; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);  // within the lane group
   return d;
 }
 
@@ -87,62 +87,84 @@ __global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, 
   }
 }
 
+// Entries are consumed in chunks of 32: lane l loads the chunk's l-th column id and its
+// per-column scalars with one coalesced load (the next chunk is prefetched while this one is
+// processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
+// so only the K-wide row gathers sit on the critical path.
 template <int LPG, int NJ, int U>
 __global__ void __launch_bounds__(256) k_gat_bwd_a(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
+  static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (w >= a.n_rows) return;
   const int32_t r = a.order[w];
   const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
   const float eli = a.el[r];
-  // online softmax statistics of row r (each lane a strided subset, then merged)
-  float m = -INFINITY, s = 0.f;
-  for (int64_t e = b + lane; e < t; e += 32) {
-    const float ev = gb_lrelu(eli + __ldg(a.er + __ldg(a.col_idx + e)));
-    if (ev > m) {
-      s = s * expf(m - ev) + 1.f;
-      m = ev;
-    } else {
-      s += expf(ev - m);
-    }
-  }
-#pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    const float m2 = __shfl_xor_sync(0xffffffffu, m, o), s2 = __shfl_xor_sync(0xffffffffu, s, o);
-    const float mn = fmaxf(m, m2);
-    s = (m == -INFINITY ? 0.f : s * expf(m - mn)) + (m2 == -INFINITY ? 0.f : s2 * expf(m2 - mn));
-    m = mn;
-  }
-  const float inv_s = s > 0.f ? 1.f / s : 0.f;
   const float ci = a.c[r];
   float xv[NJ][4];
   gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, a.K, xv);
-  float dacc = 0.f;
-  for (int64_t e0 = b; e0 < t; e0 += G * U) {  // warp-uniform trip count
-    int32_t j[U];
-    bool valid[U];
+  // one sweep with an online softmax; per lane group: running max m, S = Σ w, Cw = Σ w·s',
+  // and per lane D = Σ w·s'·(this lane's share of dα), w = exp(e - m), s' = LeakyReLU'(z).
+  // del = (Σ_lanes D - c·Cw) / S: dα enters linearly, so it is never reduced per entry
+  float m = -INFINITY, S = 0.f, Cw = 0.f, D = 0.f;
+  int32_t cn = 0;
+  if (b < t) cn = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+  for (int64_t base = b; base < t; base += 32) {
+    const int32_t cc = cn;
+    if (base + 32 < t) cn = __ldg(a.col_idx + (base + 32 + lane < t ? base + 32 + lane : t - 1));  // prefetch
+    const int cnt = (int)(t - base < 32 ? t - base : 32);
+    const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
+    for (int q = 0; q < steps; ++q) {
+      int32_t j[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t e = e0 + u * G + grp;
-      valid[u] = e < t;
-      j[u] = __ldg(a.col_idx + (valid[u] ? e : t - 1));
-    }
-    float zv[U][NJ][4];
+      for (int u = 0; u < U; ++u) j[u] = __shfl_sync(0xffffffffu, cc, q * G * U + u * G + grp);
+      float zv[U][NJ][4], erj[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      for (int u = 0; u < U; ++u) {
+        erj[u] = __ldg(a.er + j[u]);
+        gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      }
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const float d = gb_dot<LPG, NJ>(xv, zv[u]);
-      const float z = eli + __ldg(a.er + j[u]);
-      const float alpha = expf(gb_lrelu(z) - m) * inv_s;
-      const float dz = alpha * (d - ci) * (z > 0.f ? 1.f : 0.2f);
-      if (valid[u] && lg == 0) dacc += dz;
+      for (int u = 0; u < U; ++u) {
+        if (q * G * U + u * G + grp < cnt) {
+          const float pd = gb_pdot<NJ>(xv, zv[u]);
+          const float z = eli + erj[u];
+          const float ev = gb_lrelu(z);
+          const float sl = z > 0.f ? 1.f : 0.2f;
+          if (ev > m) {
+            const float sc = __expf(m - ev);  // 0 on the first entry (m = -inf)
+            S = fmaf(S, sc, 1.f);
+            Cw = fmaf(Cw, sc, sl);
+            D = fmaf(D, sc, sl * pd);
+            m = ev;
+          } else {
+            const float w = __expf(ev - m);
+            S += w;
+            Cw = fmaf(w, sl, Cw);
+            D = fmaf(w * sl, pd, D);
+          }
+        }
+      }
     }
   }
-  dacc = gb_warp_sum(dacc);
+#pragma unroll
+  for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);  // lanes of a group share m
+#pragma unroll
+  for (int o = LPG; o < 32; o <<= 1) {  // merge the groups
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
+    const float S2 = __shfl_xor_sync(0xffffffffu, S, o), C2 = __shfl_xor_sync(0xffffffffu, Cw, o);
+    const float D2 = __shfl_xor_sync(0xffffffffu, D, o);
+    const float mn = fmaxf(m, m2);
+    const float f1 = m == -INFINITY ? 0.f : __expf(m - mn), f2 = m2 == -INFINITY ? 0.f : __expf(m2 - mn);
+    S = S * f1 + S2 * f2;
+    Cw = Cw * f1 + C2 * f2;
+    D = D * f1 + D2 * f2;
+    m = mn;
+  }
+  const float inv_s = S > 0.f ? 1.f / S : 0.f;
   if (lane == 0) {
-    a.del[r] = dacc;
+    a.del[r] = (D - ci * Cw) * inv_s;
     a.stat[r] = make_float4(eli, m, inv_s, ci);
   }
 }
@@ -150,6 +172,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_a(GatBwdArgs a) {
 template <int LPG, int NJ, int U>
 __global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
+  static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   if (w >= a.n_rows) return;
@@ -162,34 +185,38 @@ __global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
   for (int j = 0; j < NJ; ++j)
 #pragma unroll
     for (int k = 0; k < 4; ++k) acc[j][k] = 0.f;
-  float dracc = 0.f;
-  for (int64_t e0 = b; e0 < t; e0 += G * U) {
-    int32_t i[U];
-    bool valid[U];
+  // der = Σ_lanes Σ α s' (lane share of dα) - Σ α s' c_i, reduced once per row
+  float dpart = 0.f, dcorr = 0.f;
+  int32_t cn = 0;
+  if (b < t) cn = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+  for (int64_t base = b; base < t; base += 32) {
+    const int32_t cc = cn;
+    if (base + 32 < t) cn = __ldg(a.col_idx + (base + 32 + lane < t ? base + 32 + lane : t - 1));  // prefetch
+    const int cnt = (int)(t - base < 32 ? t - base : 32);
+    const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
+    for (int q = 0; q < steps; ++q) {
+      int32_t i[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t e = e0 + u * G + grp;
-      valid[u] = e < t;
-      i[u] = __ldg(a.col_idx + (valid[u] ? e : t - 1));
-    }
-    float4 st[U];
-    float xv[U][NJ][4];
+      for (int u = 0; u < U; ++u) i[u] = __shfl_sync(0xffffffffu, cc, q * G * U + u * G + grp);
+      float4 st[U];
+      float xv[U][NJ][4];
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      st[u] = __ldg(a.stat_in + i[u]);
-      gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
-    }
+      for (int u = 0; u < U; ++u) {
+        st[u] = __ldg(a.stat_in + i[u]);
+        gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+      }
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const float d = gb_dot<LPG, NJ>(xv[u], zr);
-      const float z = st[u].x + erj;
-      const float alpha = valid[u] ? expf(gb_lrelu(z) - st[u].y) * st[u].z : 0.f;
-      const float dz = alpha * (d - st[u].w) * (z > 0.f ? 1.f : 0.2f);
-      if (lg == 0) dracc += dz;
+      for (int u = 0; u < U; ++u) {
+        const float z = st[u].x + erj;
+        const float alpha = (q * G * U + u * G + grp < cnt) ? __expf(gb_lrelu(z) - st[u].y) * st[u].z : 0.f;
+        const float as = alpha * (z > 0.f ? 1.f : 0.2f);
+        dpart = fmaf(as, gb_pdot<NJ>(xv[u], zr), dpart);
+        if (lg == 0) dcorr = fmaf(as, st[u].w, dcorr);
 #pragma unroll
-      for (int j = 0; j < NJ; ++j)
+        for (int j = 0; j < NJ; ++j)
 #pragma unroll
-        for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(alpha, xv[u][j][k], acc[j][k]);
+          for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(alpha, xv[u][j][k], acc[j][k]);
+      }
     }
   }
 #pragma unroll
@@ -198,7 +225,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
     for (int j = 0; j < NJ; ++j)
 #pragma unroll
       for (int k = 0; k < 4; ++k) acc[j][k] += __shfl_xor_sync(0xffffffffu, acc[j][k], o);
-  const float der = gb_warp_sum(dracc);
+  const float der = gb_warp_sum(dpart) - gb_warp_sum(dcorr);
   const float delj = a.del_in[r];
   if (grp == 0) {
     float* o = a.out + (int64_t)r * a.ldo;
@@ -253,11 +280,13 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   const double bytes = pass == 0 ? nnz * (8.0 + 4.0 * K) + R * (4.0 * K + 8.0 + 28.0)
                                  : nnz * (20.0 + 4.0 * K) + R * (8.0 * K + 8.0 + 16.0);
   ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1);
-  if (K <= 16) gb_launch<4, 1, 2>(pass, a, st);
-  else if (K <= 32) gb_launch<8, 1, 2>(pass, a, st);
-  else if (K <= 64) gb_launch<16, 1, 2>(pass, a, st);
-  else if (K <= 128) gb_launch<32, 1, 4>(pass, a, st);
-  else if (K <= 256) gb_launch<32, 2, 2>(pass, a, st);
+  // lane-group width: 8 lanes x NJ float4 up to K = 128 (4 groups, more rows in flight),
+  // full-warp groups beyond
+  if (K <= 16) gb_launch<4, 1, 4>(pass, a, st);
+  else if (K <= 32) gb_launch<8, 1, 4>(pass, a, st);
+  else if (K <= 64) gb_launch<8, 2, 2>(pass, a, st);
+  else if (K <= 128) gb_launch<8, 4, 2>(pass, a, st);
+  else if (K <= 256) gb_launch<32, 2, 4>(pass, a, st);
   else if (K <= 512) gb_launch<32, 4, 2>(pass, a, st);
   else if (K <= 1024) gb_launch<32, 8, 1>(pass, a, st);
   else gb_launch<32, 16, 1>(pass, a, st);

@@ -41,6 +41,8 @@ struct CostModel {
 //   gemm            : [1, HBM GB, TFLOP, thousands of 128x128 tiles]
 //   gemm_att        : [1, HBM GB, TFLOP, thousands of tiles, attention GEMV GB (M x K2 x 4)]
 //   gemm_tn         : [1, HBM GB, TFLOP, thousands of tiles]
+//   gat_bwd_a/b     : [1, streamed GB (idx, er / row records), row GB, gathered GB from L2,
+//                      gathered GB from HBM, M rows]  (GAT backward passes, gat_bwd.cu)
 //   elementwise     : [1, GB]
 //   allgather       : [1, GB received per GPU]
 static CostModel defaults() {
@@ -51,6 +53,8 @@ static CostModel defaults() {
   m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0};
   m.coef["gemm_att"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 1.0 / 3.0};
   m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
+  m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0};
+  m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0};
   m.coef["elementwise"] = {0.004, 1.0 / 5.5};
   m.coef["allgather"] = {0.020, 1.0 / 700.0};
   return m;
@@ -109,7 +113,7 @@ static double l2_hit(const In& in, double K) {
 
 // primitive ids of the feature API
 enum { P_SPMM_W = 0, P_SPMM_U = 1, P_SPMM_U_CS = 2, P_SDDMM1 = 3, P_SDDMM1_SM = 4, P_GEMM = 5, P_GEMM_NOSTORE = 6,
-       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10 };
+       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10, P_GAT_BWD_A = 11, P_GAT_BWD_B = 12 };
 
 static const char* prim_model(int p) {
   switch (p) {
@@ -121,6 +125,8 @@ static const char* prim_model(int p) {
     case P_GEMM_TN: return "gemm_tn";
     case P_ELEMENTWISE: return "elementwise";
     case P_ALLGATHER: return "allgather";
+    case P_GAT_BWD_A: return "gat_bwd_a";
+    case P_GAT_BWD_B: return "gat_bwd_b";
   }
   return "";
 }
@@ -148,6 +154,11 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
     case P_GEMM_TN:
       return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
               std::ceil(K1 / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
+    case P_GAT_BWD_A: case P_GAT_BWD_B: {
+      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
+      const double idx = in.nnz * (p == P_GAT_BWD_A ? 8.0 : 20.0) * gb;
+      return {1.0, idx, in.R * K * (p == P_GAT_BWD_A ? 4.0 : 12.0) * gb, gath * h, gath * (1.0 - h), in.R * 1e-6};
+    }
     case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
     case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};
   }
@@ -185,7 +196,7 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
   return 1e30;
 }
 
-// backward of the GCN compositions (layer.cu backward_impl), ReLU mask included
+// backward of the compositions (layer.cu backward_impl / gat_backward_impl), ReLU mask included
 double backward_cost(const CostModel& m, const In& in, int comp, double K1, double K2, bool need_dH) {
   double t = cost(m, in, P_ELEMENTWISE, K2) + cost(m, in, P_GEMM_TN, K1, K2);
   switch (comp) {
@@ -203,6 +214,15 @@ double backward_cost(const CostModel& m, const In& in, int comp, double K1, doub
     case GRANII_GCN_DYN_UPD:
       t += cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);  // inner D fused in the ReLU' pass
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
+      break;
+    case GRANII_GAT_REUSE:  // gat_backward_impl: prep ; A, B at K2 ; dW = Hᵀ dΘ ; (dH = dΘ Wᵀ) ; Hᵀ[del, der]
+      t += cost(m, in, P_ALLGATHER, K2) * 2.0 + cost(m, in, P_GAT_BWD_A, K2) + cost(m, in, P_GAT_BWD_B, K2) +
+           cost(m, in, P_ELEMENTWISE, K1);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
+      break;
+    case GRANII_GAT_RECOMP:  // prep ; dT = dY Wᵀ ; A, B at K1 (B writes dH) ; dW = Tᵀ dY ; Hᵀ[del, der]
+      t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) * 2.0 + cost(m, in, P_GAT_BWD_A, K1) +
+           cost(m, in, P_GAT_BWD_B, K1) + cost(m, in, P_ELEMENTWISE, K1);
       break;
     default:
       return 0.0;
@@ -235,7 +255,7 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
   } else {
     c = {GRANII_GAT_REUSE, GRANII_GAT_RECOMP};
   }
-  const bool train = (flags & GRANII_SELECT_TRAINING) && model == GRANII_GCN;
+  const bool train = (flags & GRANII_SELECT_TRAINING) != 0;
   const bool need_dH = !(flags & GRANII_SELECT_INPUT_LAYER);
   int best = -1;
   double bc = 0;
@@ -256,7 +276,7 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
 
 granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t K1, int64_t K2, double* feats,
                                  int32_t* n, char* model_name) {
-  if (prim < P_SPMM_W || prim > P_GEMM_ATT) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
+  if (prim < P_SPMM_W || prim > P_GAT_BWD_B) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
   const std::vector<double> f = features(inputs_of(g), prim, (double)K1, (double)K2);
   for (size_t i = 0; i < f.size(); ++i) feats[i] = f[i];
   *n = (int32_t)f.size();

@@ -97,6 +97,27 @@ def sweep(quick=False):
         rec(G.P_SDDMM1, 0, 0, timed(lambda: G.granii_sddmm(g, G.SDDMM_DOT, dinv, 1, dinv, 1, 1, 1.0, out)))
         rec(G.P_SDDMM1_SM, 0, 0, timed(lambda: G.granii_sddmm(
             g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el, 1, el, 1, 1, 1.0, out)))
+        if sym:  # GAT backward passes (symmetric graphs; per-pass times from the library's tracer)
+            from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+            for K in KS:
+                k1 = 16
+                W = torch.full((k1, K), 0.01, device=DEV)
+                av = torch.full((K,), 0.05, device=DEV)
+                net = GNN(g, [LayerSpec(G.GAT, k1, K, G.ACT_RELU, comp=G.GAT_REUSE, W=W, a_l=av, a_r=av)], DEV)
+                X = alloc2d(R, k1, DEV, fill=0.5)
+                gup = alloc2d(R, K, DEV, fill=0.01)
+                net.forward(X)
+                net.backward(gup)
+                torch.cuda.synchronize()
+                G.granii_profile_enable(True)
+                for _ in range(3):
+                    net.backward(gup)
+                torch.cuda.synchronize()
+                prof = G.granii_profile_read()
+                G.granii_profile_enable(False)
+                rec(G.P_GAT_BWD_A, K, 0, prof["gat_bwd_a"]["ms"] / prof["gat_bwd_a"]["calls"])
+                rec(G.P_GAT_BWD_B, K, 0, prof["gat_bwd_b"]["ms"] / prof["gat_bwd_b"]["calls"])
+                del net, X, gup
         for (k1, k2) in GEMM_PAIRS:
             A = alloc2d(R, k1, DEV, fill=0.5)
             W = torch.full((k1, k2), 0.01, device=DEV)
