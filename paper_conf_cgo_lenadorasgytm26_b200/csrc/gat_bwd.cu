@@ -14,9 +14,11 @@
 // both gathers of K-wide rows (the SpMM's access pattern):
 //   pass A (rows i): one sweep of K-wide gathers of Z_j for dα with an online
 //     softmax (running max, Σ exp, Σ exp·(dα - c)·LeakyReLU'); writes del_i and the
-//     row record stat_i = {el_i, m_i, 1/s_i, c_i} (one 16-byte gather per edge in pass B).
+//     row record {el_i, m_i, 1/s_i, c_i} into the tail of dX's row i (columns
+//     [rec, rec+4), rec = K rounded to 4), so pass B's K-wide gather of dX_i
+//     brings the record along (and the all-gather of dX carries it to other GPUs).
 //   pass B (rows j, symmetric Ã: row j lists every i with j in N(i)): gathers
-//     stat_i and dX_i, recomputes α_ij from the record (α is never stored),
+//     dX_i with its record, recomputes α_ij from it (α is never stored),
 //     dots dX_i with the register-resident Z_j, accumulates the transposed
 //     SpMM and der_j, and applies the rank-2 epilogue.
 // Lane groups of LPG lanes own one edge at a time (LPG = K/4 up to 32), NJ
@@ -92,7 +94,7 @@ __global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, 
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
 template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256) k_gat_bwd_a(GatBwdArgs a) {
+__global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_a(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
@@ -165,12 +167,12 @@ __global__ void __launch_bounds__(256) k_gat_bwd_a(GatBwdArgs a) {
   const float inv_s = S > 0.f ? 1.f / S : 0.f;
   if (lane == 0) {
     a.del[r] = (D - ci * Cw) * inv_s;
-    a.stat[r] = make_float4(eli, m, inv_s, ci);
+    *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(eli, m, inv_s, ci);
   }
 }
 
 template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
+__global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bwd_b(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
@@ -202,7 +204,7 @@ __global__ void __launch_bounds__(256) k_gat_bwd_b(GatBwdArgs a) {
       float xv[U][NJ][4];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        st[u] = __ldg(a.stat_in + i[u]);
+        st[u] = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)i[u] * a.ldx + a.rec));
         gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
       }
 #pragma unroll

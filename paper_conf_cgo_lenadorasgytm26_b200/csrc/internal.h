@@ -131,8 +131,8 @@ struct GatBwdArgs {
   const float* el = nullptr;  // pass 0: own rows
   const float* er = nullptr;  // pass 0: column-id space; pass 1: own rows
   const float* c = nullptr;   // pass 0: own rows
-  float4* stat = nullptr;     // pass 0 out: {el, m, 1/s, c} per own row
-  const float4* stat_in = nullptr;  // pass 1: column-id space
+  float* dXw = nullptr;       // pass 0: dX's own rows, whose tail receives the row record
+  int64_t rec = 0;            // column of the 16-byte record {el, m, 1/s, c} in dX rows
   float* del = nullptr;       // pass 0 out
   const float* del_in = nullptr;    // pass 1: own rows
   float* der = nullptr;       // pass 1 out

@@ -349,8 +349,8 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
 // RECOMP : dY ; dT = dY Wᵀ ; pass A (dα = <dT_i, H_j>) ; pass B -> dH = αᵀ dT + del (W a_l)ᵀ + der (W a_r)ᵀ ;
 //          dW = Tᵀ dY + (Hᵀ del) a_lᵀ + (Hᵀ der) a_rᵀ
 // both   : da_l = Wᵀ Hᵀ del, da_r = Wᵀ Hᵀ der
-// Multi-GPU: the gathered operands are er, Θ or H (pass A), dY or dT and the 16-byte row
-// records (pass B); dW and Hᵀ[del, der] are all-reduced.
+// Multi-GPU: the gathered operands are er, Θ or H (pass A) and dY or dT with the 16-byte
+// row records in their row tails (pass B); dW and Hᵀ[del, der] are all-reduced.
 static GatherBuf local_buf(Bump& b, int64_t R, int64_t K) {
   GatherBuf gb;
   gb.ld = ld4(K);
@@ -396,14 +396,14 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   }
   const float* H_all = h_gather ? hg.all : H;
 
-  GatherBuf dyg = reuse ? gather_buf(b, c, K2) : local_buf(b, R, K2);
+  // dX (dY for REUSE, dT for RECOMP) rows carry pass A's 16-byte record after column rec
+  const int64_t rec = round_up(reuse ? K2 : K1, 4);
+  GatherBuf dyg = reuse ? gather_buf(b, c, rec + 4) : local_buf(b, R, K2);
   GatherBuf dtg;
-  if (!reuse) dtg = gather_buf(b, c, K1);
+  if (!reuse) dtg = gather_buf(b, c, rec + 4);
   float* cvec = b.take((size_t)Rr);
   float* del = b.take((size_t)Rr);
   float* der = b.take((size_t)Rr);
-  float* statb = b.take((size_t)4 * (c.dist() ? g->n_cols : Rr));
-  float* stat_mine = (c.dist() && statb) ? statb + (int64_t)4 * g->rank * g->max_rows : statb;
   float* er_all = c.dist() ? vec_buf(b, c) : const_cast<float*>(er_own);
   GatherBuf thg;  // REUSE: Θ in the column-id space
   if (reuse) {
@@ -463,13 +463,11 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pa.el = el;
     pa.er = er_all;
     pa.c = cvec;
-    pa.stat = reinterpret_cast<float4*>(stat_mine);
+    pa.dXw = reuse ? dyg.mine : dtg.mine;
+    pa.rec = rec;
     pa.del = del;
     GR_TRY(launch_gat_bwd_pass(g, 0, pa, st));
-    if (c.dist()) {
-      GR_TRY(comm_allgather(c.comm, stat_mine, statb, (size_t)4 * g->max_rows, st));
-      GR_TRY(allgather(c, reuse ? dyg : dtg));
-    }
+    if (c.dist()) GR_TRY(allgather(c, reuse ? dyg : dtg));  // rows + records
     if (!reuse) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
     GatBwdArgs pb;
     pb.n_rows = R;
@@ -482,7 +480,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pb.Z = reuse ? saved : H;
     pb.ldz = reuse ? sv.ldz : ldh;
     pb.er = er_own;
-    pb.stat_in = reinterpret_cast<const float4*>(statb);
+    pb.rec = rec;
     pb.del_in = del;
     pb.der = der;
     pb.u = reuse ? a->a_l : uv;
