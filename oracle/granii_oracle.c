@@ -645,3 +645,137 @@ int oracle_gat_backward_magnitude(int comp, int64_t N, const int64_t* row_ptr, c
   free(mdY); free(mdT); free(mda); free(mdz); free(mdel); free(mder); free(mdth); free(tmp); free(aal); free(aar);
   return 0;
 }
+
+/* ======================================================================== */
+/* N3: the other models of Table III (L67-L69, L307): SGC [27], TAGCN [28],  */
+/* GIN [24].  The paper names them and counts their compositions (L326) but  */
+/* gives no formulas; the definitions below are the cited models' [R23]:     */
+/*   S    = D̃^{-1/2} Ã D̃^{-1/2} (the GCN normalisation of Eq. 2/3)         */
+/*   SGC  : out = σ(S^k H W)                                                 */
+/*   TAGCN: out = σ(Σ_{j=0..k} S^j H W_j)   (W_j stacked: W + j*K1*K2)       */
+/*   GIN  : out = σ(ReLU(agg(H) W1) W2),  agg(X)_i = (1+ε) X_i + Σ_{j∈N(i)} X_j */
+/*          = Σ_{stored (i,j) of Ã} X_j + ε X_i  (Ã holds one self-loop/row) */
+/* Compositions (ids base + {0 PRE_AGG, 1 PRE_UPD, 2 DYN_AGG, 3 DYN_UPD}):   */
+/*   PRE: precomputed sparse values (Ñ by SDDMM; GIN: 1+ε on the diagonal),  */
+/*   DYN: unweighted SpMM with dense row-broadcasts (GIN: + ε X pass);       */
+/*   AGG: aggregate at the input width; UPD: GEMM first (TAGCN: Horner form  */
+/*   Z = H W_k; Z = S Z + H W_j for j = k-1..0).                             */
+/* ======================================================================== */
+enum { OR_SGC = 32, OR_TAGCN = 48, OR_GIN = 64 };
+
+/* one hop Y = S X under the composition's normalisation (tmp: N x K scratch) */
+static void or_hop(int dyn, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, const double* nval,
+                   const double* dinv, const double* X, int64_t K, double* Y, double* tmp) {
+  if (!dyn) {
+    oracle_spmm(N, row_ptr, col_idx, nval, X, K, Y);                  /* Ñ X */
+  } else {
+    oracle_rowbcast(N, K, dinv, X, tmp);                               /* D^-1/2 X */
+    oracle_spmm(N, row_ptr, col_idx, NULL, tmp, K, Y);                 /* Ã (.)    */
+    oracle_rowbcast(N, K, dinv, Y, tmp);                               /* D^-1/2 (.) */
+    memcpy(Y, tmp, (size_t)(N * K) * sizeof(double));
+  }
+}
+
+int oracle_sgc_forward(int comp, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, const double* H,
+                       int64_t K1, const double* W, int64_t K2, int hops, int act, double* out) {
+  int v = comp - OR_SGC;
+  if (v < 0 || v > 3 || hops < 0) return 1;
+  int dyn = v >= 2, upd = v & 1;
+  int64_t nnz = row_ptr[N], K = upd ? K2 : K1;
+  double* dinv = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* nval = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* x = (double*)malloc((size_t)(N * K + 1) * sizeof(double));
+  double* y = (double*)malloc((size_t)(N * K + 1) * sizeof(double));
+  double* tmp = (double*)malloc((size_t)(N * K + 1) * sizeof(double));
+  oracle_dinv(N, row_ptr, dinv);
+  if (!dyn) oracle_sddmm(N, row_ptr, col_idx, dinv, dinv, 1, nval);
+  if (upd) oracle_gemm(N, K2, K1, H, 0, W, 0, x);                      /* H W first */
+  else memcpy(x, H, (size_t)(N * K1) * sizeof(double));
+  for (int h = 0; h < hops; ++h) {
+    or_hop(dyn, N, row_ptr, col_idx, nval, dinv, x, K, y, tmp);
+    double* t = x; x = y; y = t;
+  }
+  if (upd) memcpy(out, x, (size_t)(N * K2) * sizeof(double));
+  else oracle_gemm(N, K2, K1, x, 0, W, 0, out);                        /* (S^k H) W */
+  act_inplace(N * K2, out, act);
+  free(dinv); free(nval); free(x); free(y); free(tmp);
+  return 0;
+}
+
+int oracle_tagcn_forward(int comp, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, const double* H,
+                         int64_t K1, const double* W, int64_t K2, int hops, int act, double* out) {
+  int v = comp - OR_TAGCN;
+  if (v < 0 || v > 3 || hops < 0) return 1;
+  int dyn = v >= 2, upd = v & 1;
+  int64_t nnz = row_ptr[N], Km = K1 > K2 ? K1 : K2;
+  double* dinv = (double*)malloc((size_t)(N + 1) * sizeof(double));
+  double* nval = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+  double* x = (double*)malloc((size_t)(N * Km + 1) * sizeof(double));
+  double* y = (double*)malloc((size_t)(N * Km + 1) * sizeof(double));
+  double* p = (double*)malloc((size_t)(N * K2 + 1) * sizeof(double));
+  double* tmp = (double*)malloc((size_t)(N * Km + 1) * sizeof(double));
+  oracle_dinv(N, row_ptr, dinv);
+  if (!dyn) oracle_sddmm(N, row_ptr, col_idx, dinv, dinv, 1, nval);
+  if (!upd) {                                      /* X_0 = H, X_{j+1} = S X_j ; out = Σ_j X_j W_j */
+    memcpy(x, H, (size_t)(N * K1) * sizeof(double));
+    for (int64_t i = 0; i < N * K2; ++i) out[i] = 0.0;
+    for (int j = 0; j <= hops; ++j) {
+      oracle_gemm(N, K2, K1, x, 0, W + (int64_t)j * K1 * K2, 0, p);
+      for (int64_t i = 0; i < N * K2; ++i) out[i] += p[i];
+      if (j < hops) {
+        or_hop(dyn, N, row_ptr, col_idx, nval, dinv, x, K1, y, tmp);
+        double* t = x; x = y; y = t;
+      }
+    }
+  } else {                                         /* Horner: Z = H W_k ; Z = S Z + H W_j, j = k-1..0 */
+    oracle_gemm(N, K2, K1, H, 0, W + (int64_t)hops * K1 * K2, 0, x);
+    for (int j = hops - 1; j >= 0; --j) {
+      or_hop(dyn, N, row_ptr, col_idx, nval, dinv, x, K2, y, tmp);
+      oracle_gemm(N, K2, K1, H, 0, W + (int64_t)j * K1 * K2, 0, p);
+      for (int64_t i = 0; i < N * K2; ++i) x[i] = y[i] + p[i];
+    }
+    memcpy(out, x, (size_t)(N * K2) * sizeof(double));
+  }
+  act_inplace(N * K2, out, act);
+  free(dinv); free(nval); free(x); free(y); free(p); free(tmp);
+  return 0;
+}
+
+/* GIN aggregation agg(X) = Σ_{stored (i,j)} X_j + ε X_i (every row of Ã holds its self-loop) */
+static void or_gin_agg(int dyn, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, double eps,
+                       const double* X, int64_t K, double* Y) {
+  if (!dyn) {                                      /* precomputed values: 1 + ε on the diagonal */
+    int64_t nnz = row_ptr[N];
+    double* vals = (double*)malloc((size_t)(nnz + 1) * sizeof(double));
+    for (int64_t r = 0; r < N; ++r)
+      for (int64_t e = row_ptr[r]; e < row_ptr[r + 1]; ++e) vals[e] = col_idx[e] == r ? 1.0 + eps : 1.0;
+    oracle_spmm(N, row_ptr, col_idx, vals, X, K, Y);
+    free(vals);
+  } else {                                         /* unweighted SpMM, then + ε X */
+    oracle_spmm(N, row_ptr, col_idx, NULL, X, K, Y);
+    for (int64_t i = 0; i < N * K; ++i) Y[i] += eps * X[i];
+  }
+}
+
+int oracle_gin_forward(int comp, int64_t N, const int64_t* row_ptr, const int32_t* col_idx, const double* H,
+                       int64_t K1, const double* W1, int64_t Kh, const double* W2, int64_t K2, double eps, int act,
+                       double* out) {
+  int v = comp - OR_GIN;
+  if (v < 0 || v > 3) return 1;
+  int dyn = v >= 2, upd = v & 1;
+  int64_t Km = K1 > Kh ? K1 : Kh;
+  double* a = (double*)malloc((size_t)(N * Km + 1) * sizeof(double));
+  double* b = (double*)malloc((size_t)(N * Km + 1) * sizeof(double));
+  if (!upd) {
+    or_gin_agg(dyn, N, row_ptr, col_idx, eps, H, K1, a);                 /* agg(H)      */
+    oracle_gemm(N, Kh, K1, a, 0, W1, 0, b);                              /* agg(H) W1   */
+  } else {
+    oracle_gemm(N, Kh, K1, H, 0, W1, 0, a);                              /* H W1        */
+    or_gin_agg(dyn, N, row_ptr, col_idx, eps, a, Kh, b);                 /* agg(H W1)   */
+  }
+  act_inplace(N * Kh, b, 1);                                             /* MLP ReLU    */
+  oracle_gemm(N, K2, Kh, b, 0, W2, 0, out);
+  act_inplace(N * K2, out, act);
+  free(a); free(b);
+  return 0;
+}

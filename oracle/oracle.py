@@ -21,6 +21,9 @@ GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD = 0, 1, 2, 3
 GAT_REUSE, GAT_RECOMP = 16, 17
 GCN_COMPS = (GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD)
 GAT_COMPS = (GAT_REUSE, GAT_RECOMP)
+SGC_COMPS = (32, 33, 34, 35)      # PRE_AGG, PRE_UPD, DYN_AGG, DYN_UPD
+TAGCN_COMPS = (48, 49, 50, 51)
+GIN_COMPS = (64, 65, 66, 67)
 
 
 def build(force: bool = False) -> str:
@@ -59,6 +62,10 @@ def lib():
         _lib.oracle_gat_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, p, p, ctypes.c_int, p, p, p,
                                              p, p]
         _lib.oracle_gat_backward_magnitude.argtypes = _lib.oracle_gat_backward.argtypes
+        _lib.oracle_sgc_forward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, ctypes.c_int, p]
+        _lib.oracle_tagcn_forward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, ctypes.c_int, p]
+        _lib.oracle_gin_forward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, p, i64, ctypes.c_double,
+                                            ctypes.c_int, p]
         _lib.oracle_gcn_backward.argtypes = [ctypes.c_int, i64, p, p, p, i64, p, i64, ctypes.c_int, p, p, p]
     return _lib
 
@@ -262,3 +269,39 @@ def gat_backward_magnitude(comp, row_ptr, col_idx, H, W, a_l, a_r, G, act=0, nee
     if rc:
         raise ValueError(f"bad composition {comp}")
     return dH, dW, dal, dar
+
+
+def sgc_forward(comp, row_ptr, col_idx, H, W, hops=2, act=0):
+    """SGC (R23): sigma(S^k H W)."""
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, W = _np(H, np.float64), _np(W, np.float64)
+    N, K1 = H.shape
+    out = np.zeros((N, W.shape[1]), np.float64)
+    if lib().oracle_sgc_forward(comp, N, _p(rp), _p(ci), _p(H), K1, _p(W), W.shape[1], hops, act, _p(out)):
+        raise ValueError(f"bad composition {comp}")
+    return out
+
+
+def tagcn_forward(comp, row_ptr, col_idx, H, Ws, act=0):
+    """TAGCN (R23): sigma(sum_j S^j H W_j); Ws has shape (hops+1, K1, K2)."""
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, Ws = _np(H, np.float64), _np(Ws, np.float64)
+    N, K1 = H.shape
+    hops, K2 = Ws.shape[0] - 1, Ws.shape[2]
+    out = np.zeros((N, K2), np.float64)
+    if lib().oracle_tagcn_forward(comp, N, _p(rp), _p(ci), _p(H), K1, _p(Ws), K2, hops, act, _p(out)):
+        raise ValueError(f"bad composition {comp}")
+    return out
+
+
+def gin_forward(comp, row_ptr, col_idx, H, W1, W2, eps=0.0, act=0):
+    """GIN (R23): sigma(ReLU(agg(H) W1) W2), agg = (1+eps) self + neighbour sum."""
+    rp, ci = _np(row_ptr, np.int64), _np(col_idx, np.int32)
+    H, W1, W2 = _np(H, np.float64), _np(W1, np.float64), _np(W2, np.float64)
+    N, K1 = H.shape
+    Kh, K2 = W1.shape[1], W2.shape[1]
+    out = np.zeros((N, K2), np.float64)
+    if lib().oracle_gin_forward(comp, N, _p(rp), _p(ci), _p(H), K1, _p(W1), Kh, _p(W2), K2, float(eps), act,
+                                _p(out)):
+        raise ValueError(f"bad composition {comp}")
+    return out

@@ -466,6 +466,70 @@ def test_gat_backward_magnitude_bounds_and_closed_form(K1, K2):
         assert rel(m[0], g[0]) < 1e-13 and rel(m[1], g[1]) < 1e-13
 
 
+# ------------------------------------------------------------------ N3: SGC / TAGCN / GIN (reading R23)
+def dense_S(A):
+    deg = A.sum(1)
+    dm = np.where(deg > 0, 1.0 / np.sqrt(np.where(deg > 0, deg, 1)), 0.0)
+    return np.diag(dm) @ A @ np.diag(dm)
+
+
+@pytest.mark.parametrize("comp", O.SGC_COMPS)
+@pytest.mark.parametrize("hops", [0, 1, 3])
+def test_sgc_equals_dense_power(comp, hops):
+    rp, ci, A = csr_and_dense(71)
+    rng = np.random.default_rng(21)
+    H, W = rng.uniform(-1, 1, (29, 6)), rng.uniform(-1, 1, (6, 4))
+    S = dense_S(A)
+    for act in (0, 1):
+        Y = np.linalg.matrix_power(S, hops) @ H @ W
+        assert rel(O.sgc_forward(comp, rp, ci, H, W, hops, act), np.maximum(Y, 0) if act else Y) < 1e-12
+
+
+def test_sgc_one_hop_is_gcn():
+    rp, ci, _ = csr_and_dense(72)
+    rng = np.random.default_rng(22)
+    H, W = rng.uniform(-1, 1, (29, 5)), rng.uniform(-1, 1, (5, 7))
+    for c_sgc, c_gcn in zip(O.SGC_COMPS, O.GCN_COMPS):
+        assert rel(O.sgc_forward(c_sgc, rp, ci, H, W, 1, 1), O.gcn_forward(c_gcn, rp, ci, H, W, 1)[0]) < 1e-12
+
+
+@pytest.mark.parametrize("comp", O.TAGCN_COMPS)
+@pytest.mark.parametrize("hops", [0, 1, 2, 3])
+def test_tagcn_equals_dense_polynomial(comp, hops):
+    rp, ci, A = csr_and_dense(73)
+    rng = np.random.default_rng(23)
+    H = rng.uniform(-1, 1, (29, 5))
+    Ws = rng.uniform(-1, 1, (hops + 1, 5, 3))
+    S = dense_S(A)
+    Y = sum(np.linalg.matrix_power(S, j) @ H @ Ws[j] for j in range(hops + 1))
+    for act in (0, 1):
+        assert rel(O.tagcn_forward(comp, rp, ci, H, Ws, act), np.maximum(Y, 0) if act else Y) < 1e-12
+    # only W_0 nonzero: a plain matmul, whatever the graph
+    W0 = np.zeros_like(Ws)
+    W0[0] = Ws[0]
+    assert rel(O.tagcn_forward(comp, rp, ci, H, W0, 0), H @ Ws[0]) < 1e-14
+
+
+@pytest.mark.parametrize("comp", O.GIN_COMPS)
+def test_gin_equals_dense_mlp(comp):
+    n = 31
+    s, d = synth.random_small(n, 120, 74)
+    rp, ci = O.csr_build(n, s, d, O.SYMMETRIZE | O.ADD_SELF_LOOPS)
+    A0 = dense_adj(n, s.numpy(), d.numpy(), True, False)
+    np.fill_diagonal(A0, 0.0)                  # neighbours j != i: GIN's own term is (1 + eps) H_i
+    rng = np.random.default_rng(24)
+    H, W1, W2 = rng.uniform(-1, 1, (n, 6)), rng.uniform(-1, 1, (6, 9)), rng.uniform(-1, 1, (9, 4))
+    for eps in (0.0, 0.37, -0.5):
+        agg = (1 + eps) * H + A0 @ H
+        Y = np.maximum(agg @ W1, 0) @ W2
+        for act in (0, 1):
+            got = O.gin_forward(comp, rp, ci, H, W1, W2, eps, act)
+            assert rel(got, np.maximum(Y, 0) if act else Y) < 1e-12
+    # self-loop-only graph: agg = (1 + eps) H
+    rp1, ci1 = O.csr_build(n, np.zeros(0, np.int32), np.zeros(0, np.int32), O.ADD_SELF_LOOPS)
+    assert rel(O.gin_forward(comp, rp1, ci1, H, W1, W2, 0.25, 0), np.maximum(1.25 * H @ W1, 0) @ W2) < 1e-14
+
+
 # ------------------------------------------------------------------ generators
 def test_generator_is_device_independent_and_exact():
     a = synth.uniform_pm1(3, 4, (1000,))
