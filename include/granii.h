@@ -189,7 +189,11 @@ granii_status granii_gemm(int64_t M, int64_t N, int64_t K, const float* d_A, int
 /* ------------------------------------------------------------------------ */
 /* Layers under an explicit composition (§III, Fig. 3 reading R10) */
 /* ------------------------------------------------------------------------ */
-typedef enum { GRANII_GCN = 0, GRANII_GAT = 1 } granii_model;
+/* SGC, TAGCN, GIN: the other models of Table III (L67-L69, L307), cited models' definitions
+ * (reading R23) with S = D̃^{-1/2} Ã D̃^{-1/2}:
+ *   SGC   out = σ(S^k H W)                 TAGCN out = σ(Σ_{j=0..k} S^j H W_j)
+ *   GIN   out = σ(ReLU(agg(H) W W2)),  agg(X)_i = (1+ε) X_i + Σ_{j∈N(i)} X_j  (needs self-loops in Ã) */
+typedef enum { GRANII_GCN = 0, GRANII_GAT = 1, GRANII_SGC = 2, GRANII_TAGCN = 3, GRANII_GIN = 4 } granii_model;
 
 typedef enum {
   GRANII_GCN_PRE_AGG = 0, /* Eq. 3, aggregate first: SDDMM Ñ ; SpMM_w(Ñ, H) ; GEMM (·W)       */
@@ -197,7 +201,17 @@ typedef enum {
   GRANII_GCN_DYN_AGG = 2, /* Eq. 2, aggregate first: SpMM_u(Ã, D̃^-½ H) ; D̃^-½ ; GEMM (·W)  */
   GRANII_GCN_DYN_UPD = 3, /* Eq. 2, update first:    GEMM (H W) ; D̃^-½ ; SpMM_u(Ã, ·) ; D̃^-½ */
   GRANII_GAT_REUSE = 16,  /* Eq. 5: Θ = H W ; α = Atten(Ã, Θ, W_A) ; SpMM_w(α, Θ)             */
-  GRANII_GAT_RECOMP = 17  /* Eq. 6: Θ-scores ; α ; SpMM_w(α, H) ; GEMM (·W)                    */
+  GRANII_GAT_RECOMP = 17, /* Eq. 6: Θ-scores ; α ; SpMM_w(α, H) ; GEMM (·W)                    */
+  /* SGC: k hops of S, PRE = Ñ by SDDMM + weighted SpMMs, DYN = unweighted SpMMs with the
+   * D̃^-½ scalings fused; AGG = hops at K1 then GEMM, UPD = GEMM then hops at K2 */
+  GRANII_SGC_PRE_AGG = 32, GRANII_SGC_PRE_UPD = 33, GRANII_SGC_DYN_AGG = 34, GRANII_SGC_DYN_UPD = 35,
+  /* TAGCN: AGG = X_0..X_k = S^j H at K1 side by side, one GEMM against the stacked W_j;
+   * UPD = Horner: Z = H W_k ; Z = S Z + H W_j (the addend fused in the SpMM epilogue) */
+  GRANII_TAGCN_PRE_AGG = 48, GRANII_TAGCN_PRE_UPD = 49, GRANII_TAGCN_DYN_AGG = 50, GRANII_TAGCN_DYN_UPD = 51,
+  /* GIN: PRE = weighted SpMM with 1+ε on the diagonal (values written per call), DYN =
+   * unweighted SpMM with + ε X_i fused in its epilogue; AGG = aggregate at K1 then W,
+   * UPD = H W then aggregate at Kh (ReLU fused); W2 last */
+  GRANII_GIN_PRE_AGG = 64, GRANII_GIN_PRE_UPD = 65, GRANII_GIN_DYN_AGG = 66, GRANII_GIN_DYN_UPD = 67
 } granii_composition;
 
 #define GRANII_ACT_NONE 0u
@@ -221,11 +235,20 @@ typedef struct {
   granii_comm comm;        /* NULL: whole graph on this GPU                              */
   float* d_a_l;            /* GAT backward outputs dL/da_l, dL/da_r (K2 floats each,     */
   float* d_a_r;            /*   all-reduced over comm); NULL: not computed               */
+  int32_t hops;            /* SGC / TAGCN: k >= 0 (TAGCN: W holds k+1 stacked K1 x K2)   */
+  float eps;               /* GIN: ε                                                     */
+  int64_t Kh;              /* GIN: MLP hidden width (W: K1 x Kh, W2: Kh x K2)            */
+  const float* W2;         /* GIN: second MLP weight                                     */
 } granii_layer_args;
 
-/* Workspace bytes and the number of floats of `saved` (state kept for backward). */
+/* Workspace bytes and the number of floats of `saved` (state kept for backward).
+ * GCN / GAT only; SGC / TAGCN / GIN need their shape parameters: use the _ex form. */
 granii_status granii_layer_workspace_size(granii_graph g, granii_model m, granii_composition c, int64_t K1,
                                           int64_t K2, size_t* workspace_bytes, size_t* saved_floats);
+/* Same for any model; reads the shape fields of *a (K1, K2, hops, Kh) only. */
+granii_status granii_layer_workspace_size_ex(granii_graph g, granii_model m, granii_composition c,
+                                             const granii_layer_args* a, size_t* workspace_bytes,
+                                             size_t* saved_floats);
 /*
  * out = sigma(layer(H)) for the owned rows (out: rows x K2, ld ldo).  Every
  * composition computes the same mathematical value (L192: only semantically
@@ -278,6 +301,12 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
 granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t K2, const char* calib_path,
                             uint32_t flags, granii_composition* out, int32_t* candidates,
                             double* predicted_ms, int32_t* n_candidates);
+/* Same for any model (GCN / GAT as above); reads the shape fields of *a (K1, K2, hops, Kh).
+ * SGC / TAGCN: the embedding-size rule picks AGG for K1 < K2 and UPD for K1 >= K2 (as GCN),
+ * GIN compares K1 with Kh; the cost models then choose PRE vs DYN.  Forward costs only. */
+granii_status granii_select_ex(granii_graph g, granii_model m, const granii_layer_args* a, const char* calib_path,
+                               uint32_t flags, granii_composition* out, int32_t* candidates,
+                               double* predicted_ms, int32_t* n_candidates);
 /* Calibration support: the feature vector the cost model of primitive `prim`
  * (0 spmm weighted, 1 spmm unweighted, 2 spmm unweighted + column scale,
  * 3 sddmm K=1, 4 sddmm K=1 + softmax, 5 gemm, 6 gemm without store, 7 gemm Aᵀ·B,

@@ -35,13 +35,13 @@ granii_status graph_create(int64_t, int64_t, const int32_t*, const int32_t*, uin
                            granii_graph_s**);
 void graph_free(granii_graph_s*);
 void partition_bounds_host(int64_t N, const int64_t* rp, int G, int64_t* b);
-granii_status layer_workspace(const granii_graph_s*, granii_model, granii_composition, int64_t, int64_t, size_t*,
-                              size_t*);
+granii_status layer_workspace(const granii_graph_s*, granii_model, granii_composition, const granii_layer_args*,
+                              size_t*, size_t*);
 granii_status layer_forward(const granii_graph_s*, granii_model, granii_composition, const granii_layer_args*, float*,
                             int64_t, float*, cudaStream_t);
 granii_status layer_backward(const granii_graph_s*, granii_composition, const granii_layer_args*, const float*, int64_t,
                              const float*, int64_t, const float*, float*, int64_t, float*, cudaStream_t);
-granii_status select_impl(const granii_graph_s*, granii_model, int64_t, int64_t, const char*, uint32_t,
+granii_status select_impl(const granii_graph_s*, granii_model, const granii_layer_args*, const char*, uint32_t,
                           granii_composition*, int32_t*, double*, int32_t*);
 granii_status cost_features_impl(const granii_graph_s*, int32_t, int64_t, int64_t, double*, int32_t*, char*);
 granii_status comm_unique_id(void*);
@@ -57,7 +57,19 @@ using namespace granii;
 static bool valid_comp(granii_model m, granii_composition c) {
   if (m == GRANII_GCN) return c == GRANII_GCN_PRE_AGG || c == GRANII_GCN_PRE_UPD || c == GRANII_GCN_DYN_AGG || c == GRANII_GCN_DYN_UPD;
   if (m == GRANII_GAT) return c == GRANII_GAT_REUSE || c == GRANII_GAT_RECOMP;
+  if (m == GRANII_SGC) return c >= GRANII_SGC_PRE_AGG && c <= GRANII_SGC_DYN_UPD;
+  if (m == GRANII_TAGCN) return c >= GRANII_TAGCN_PRE_AGG && c <= GRANII_TAGCN_DYN_UPD;
+  if (m == GRANII_GIN) return c >= GRANII_GIN_PRE_AGG && c <= GRANII_GIN_DYN_UPD;
   return false;
+}
+
+// shape fields of the layer arguments (K1, K2, hops, Kh), as used by sizing and selection
+static granii_status check_shape(granii_model m, const granii_layer_args* a) {
+  GR_ARG(a, "NULL argument");
+  GR_ARG(a->K1 > 0 && a->K2 > 0, "bad embedding sizes");
+  if (m == GRANII_SGC || m == GRANII_TAGCN) GR_ARG(a->hops >= 0 && a->hops <= 16, "hops must be in [0, 16]");
+  if (m == GRANII_GIN) GR_ARG(a->Kh > 0, "GIN needs the hidden width Kh > 0");
+  return GRANII_OK;
 }
 
 #define API_BEGIN try {
@@ -217,9 +229,23 @@ granii_status granii_layer_workspace_size(granii_graph g, granii_model m, granii
                                           size_t* ws, size_t* saved) {
   API_BEGIN
   GR_ARG(g && ws, "NULL argument");
+  GR_ARG(m == GRANII_GCN || m == GRANII_GAT, "SGC / TAGCN / GIN: use granii_layer_workspace_size_ex");
   GR_ARG(valid_comp(m, c), "composition does not belong to the model");
   GR_ARG(K1 > 0 && K2 > 0, "bad embedding sizes");
-  return layer_workspace(g, m, c, K1, K2, ws, saved);
+  granii_layer_args a{};
+  a.K1 = K1;
+  a.K2 = K2;
+  return layer_workspace(g, m, c, &a, ws, saved);
+  API_END
+}
+
+granii_status granii_layer_workspace_size_ex(granii_graph g, granii_model m, granii_composition c,
+                                             const granii_layer_args* a, size_t* ws, size_t* saved) {
+  API_BEGIN
+  GR_ARG(g && ws, "NULL argument");
+  GR_ARG(valid_comp(m, c), "composition does not belong to the model");
+  GR_TRY(check_shape(m, a));
+  return layer_workspace(g, m, c, a, ws, saved);
   API_END
 }
 
@@ -230,6 +256,9 @@ static granii_status check_args(granii_graph g, granii_model m, granii_compositi
   GR_ARG(a->H && a->W, "NULL H or W");
   GR_ARG(a->act <= GRANII_ACT_RELU && a->attn <= GRANII_ATTN_DOT, "bad act/attn");
   GR_ARG(m != GRANII_GAT || a->attn == GRANII_ATTN_DOT || (a->a_l && a->a_r), "GAT additive needs a_l, a_r");
+  GR_TRY(check_shape(m, a));
+  GR_ARG(m != GRANII_GIN || a->W2, "GIN needs W2");
+  GR_ARG(m != GRANII_GIN || g->self_loops, "GIN needs a graph created with GRANII_ADD_SELF_LOOPS (R23)");
   GR_ARG(a->workspace, "NULL workspace");
   if (g->world > 1) GR_ARG(a->comm && a->comm->world == g->world && a->comm->rank == g->rank,
                            "partitioned graph needs the matching communicator");
@@ -251,6 +280,8 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
                                     const float* d_saved, float* d_dH, int64_t lddh, float* d_dW, void* stream) {
   API_BEGIN
   GR_TRY(check_args(g, m, c, a));
+  if (m != GRANII_GCN && m != GRANII_GAT)
+    return fail(GRANII_ERR_UNSUPPORTED, "backward of SGC / TAGCN / GIN is not implemented (forward only, R23)");
   if (m == GRANII_GAT && a->attn != GRANII_ATTN_ADDITIVE)
     return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is implemented for additive attention only (R22)");
   GR_ARG(g->symmetric, "backward needs a symmetric graph (created with GRANII_SYMMETRIZE): M^T = M");
@@ -266,9 +297,23 @@ granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t 
                             int32_t* n_candidates) {
   API_BEGIN
   GR_ARG(g && out, "NULL argument");
-  GR_ARG(m == GRANII_GCN || m == GRANII_GAT, "bad model");
+  GR_ARG(m == GRANII_GCN || m == GRANII_GAT, "SGC / TAGCN / GIN: use granii_select_ex");
   GR_ARG(K1 > 0 && K2 > 0, "bad embedding sizes");
-  return select_impl(g, m, K1, K2, calib_path, flags, out, candidates, predicted_ms, n_candidates);
+  granii_layer_args a{};
+  a.K1 = K1;
+  a.K2 = K2;
+  return select_impl(g, m, &a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
+  API_END
+}
+
+granii_status granii_select_ex(granii_graph g, granii_model m, const granii_layer_args* a, const char* calib_path,
+                               uint32_t flags, granii_composition* out, int32_t* candidates, double* predicted_ms,
+                               int32_t* n_candidates) {
+  API_BEGIN
+  GR_ARG(g && out, "NULL argument");
+  GR_ARG(m >= GRANII_GCN && m <= GRANII_GIN, "bad model");
+  GR_TRY(check_shape(m, a));
+  return select_impl(g, m, a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
   API_END
 }
 

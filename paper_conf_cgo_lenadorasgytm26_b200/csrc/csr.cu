@@ -162,6 +162,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   g->rank = rank;
   g->world = world;
   g->symmetric = sym;
+  g->self_loops = loops;
   cudaGetDevice(&g->device);
 
   int* d_bad = nullptr;

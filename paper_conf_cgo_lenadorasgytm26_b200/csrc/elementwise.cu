@@ -117,3 +117,28 @@ granii_status launch_sgd(int64_t n, float lr, const float* g, float* p, cudaStre
 }
 
 }  // namespace granii
+
+namespace granii {
+
+// GIN PRE composition (R23): vals_e = 1 + eps where col(e) is the row's own diagonal, 1 elsewhere.
+// Column ids live in the gather layout when partitioned: the diagonal of local row r is diag0 + r.
+__global__ void k_gin_vals(int64_t R, const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+                           int64_t diag0, float one_eps, float* __restrict__ vals) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < R; r += nw)
+    for (int64_t e = row_ptr[r] + lane; e < row_ptr[r + 1]; e += 32)
+      vals[e] = (int64_t)col_idx[e] == diag0 + r ? one_eps : 1.f;
+}
+
+granii_status launch_gin_vals(const granii_graph_s* g, float eps, float* vals, cudaStream_t st) {
+  if (g->n_rows == 0) return GRANII_OK;
+  ProfScope ps("sddmm", st, 8.0 * (double)g->local_nnz + 8.0 * (double)g->n_rows, 0.0, 1);
+  const int64_t diag0 = g->world > 1 ? (int64_t)g->rank * g->max_rows : 0;
+  k_gin_vals<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(g->n_rows, 8), 148 * 32)), 256, 0, st>>>(
+      g->n_rows, g->row_ptr, g->col_idx, diag0, 1.f + eps, vals);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
+}  // namespace granii

@@ -76,6 +76,7 @@ struct granii_graph_s {
   int64_t max_rows = 0;     // gather-layout block height
   int64_t n_cols = 0;       // size of the column-id space (N, or world*max_rows)
   int32_t symmetric = 0;
+  int32_t self_loops = 0;   // every row of Ã holds its diagonal entry (GRANII_ADD_SELF_LOOPS)
   std::vector<int64_t> bounds;
   int64_t* row_ptr = nullptr;     // device, n_rows+1, rebased
   int32_t* col_idx = nullptr;     // device, local_nnz, column-id space
@@ -105,6 +106,12 @@ namespace granii {
 // kernels (launchers); all validate nothing -- callers in api.cu validate.
 granii_status launch_spmm(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                           float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, cudaStream_t st);
+// Y_i = act(rs_i * sum + beta * B_i): SpMM with a dense addend fused in the epilogue
+granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                             float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                             int64_t ldb, float beta, cudaStream_t st);
+// GIN's precomputed values: vals_e = 1 + eps on the diagonal entry of each row, 1 elsewhere
+granii_status launch_gin_vals(const granii_graph_s* g, float eps, float* vals, cudaStream_t st);
 granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U, int64_t ldu, const float* V,
                            int64_t ldv, int64_t K, float scale, float* out, cudaStream_t st);
 size_t gemm_workspace(int64_t M, int64_t N, int64_t K, uint32_t flags);

@@ -103,6 +103,228 @@ static GatSaved gat_saved_layout(int64_t R, granii_composition comp, int64_t K1,
   return s;
 }
 
+// ---------------------------------------------------------------- SGC / TAGCN / GIN (N3, reading R23)
+// Forward only.  Shared pieces: one hop of S = D̃^-½ Ã D̃^-½ is a weighted SpMM over Ñ (PRE)
+// or an unweighted SpMM with both scalings fused (DYN); multi-hop chains ping-pong between two
+// gather buffers (all-gathered between hops on several GPUs); the TAGCN Horner step and GIN's
+// ε self term are the SpMM's fused dense addend.
+static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_composition comp,
+                                      const granii_layer_args* a, float* out, int64_t ldo, void* ws_base,
+                                      size_t* ws_size) {
+  const granii_graph_s* g = c.g;
+  const bool run = ws_base != nullptr;
+  Bump b(ws_base);
+  const int64_t R = g->n_rows, Rr = std::max<int64_t>(R, 1), K1 = a->K1, K2 = a->K2;
+  const bool relu = a->act == GRANII_ACT_RELU;
+  const cudaStream_t st = c.st;
+  const int base = m == GRANII_SGC ? GRANII_SGC_PRE_AGG : m == GRANII_TAGCN ? GRANII_TAGCN_PRE_AGG : GRANII_GIN_PRE_AGG;
+  const int v = (int)comp - base;
+  const bool dyn = v >= 2, upd = (v & 1) != 0;
+  const int hops = a->hops;
+
+  // H: aligned own rows, and (aggregate-first) its gathered copy
+  const float* H = a->H;
+  int64_t ldh = a->ldh;
+  const bool h_aligned = (ldh % 4 == 0) && (((uintptr_t)H & 15) == 0);
+  GatherBuf hg;
+  const bool h_gather = c.dist() && !upd;
+  if (h_gather) {
+    hg = gather_buf(b, c, K1);
+    if (run) {
+      GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hg.mine, hg.ld, st));
+      GR_TRY(allgather(c, hg));
+    }
+    H = hg.mine;
+    ldh = hg.ld;
+  } else if (!h_aligned) {
+    float* hp = b.take((size_t)Rr * ld4(K1));
+    if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hp, ld4(K1), st));
+    H = hp;
+    ldh = ld4(K1);
+  }
+  const float* H_all = h_gather ? hg.all : H;
+
+  // sparse values of the PRE compositions (recomputed per call, stateless as GCN's Ñ, R13)
+  float* vals = nullptr;
+  if (!dyn) vals = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
+  if (run && !dyn) {
+    if (m == GRANII_GIN) GR_TRY(launch_gin_vals(g, a->eps, vals, st));
+    else GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT, g->dinv_rows, 1, g->dinv_cols, 1, 1, 1.f, vals, st));
+  }
+  // one hop Y = S X (+ beta B) (+ ReLU); X in the column-id space
+  auto hop = [&](const float* X, int64_t ldx, int64_t K, float* Y, int64_t ldy, bool rl, const float* B, int64_t ldb,
+                 float beta) -> granii_status {
+    if (!dyn) return launch_spmm_ex(g, vals, X, ldx, K, Y, ldy, nullptr, nullptr, rl, B, ldb, beta, st);
+    return launch_spmm_ex(g, nullptr, X, ldx, K, Y, ldy, g->dinv_rows, g->dinv_cols, rl, B, ldb, beta, st);
+  };
+
+  if (m == GRANII_SGC) {
+    const int64_t K = upd ? K2 : K1;
+    GatherBuf pb[2] = {gather_buf(b, c, K), gather_buf(b, c, K)};
+    float* T = upd ? nullptr : b.take((size_t)Rr * ld4(K1));  // S^k H (own rows) before the GEMM
+    void* gw;
+    size_t gn;
+    gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw, &gn);
+    if (run) {
+      const float* X = nullptr;
+      int64_t ldx = 0;
+      if (upd) {  // P = H W, then the hops at K2
+        if (hops == 0) {
+          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
+        } else {
+          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, pb[0].mine, pb[0].ld, nullptr, 0, gw, gn, st));
+          GR_TRY(allgather(c, pb[0]));
+          X = pb[0].all;
+          ldx = pb[0].ld;
+        }
+      } else {
+        X = H_all;
+        ldx = ldh;
+      }
+      for (int h = 0; h < hops; ++h) {
+        const bool last = h == hops - 1;
+        GatherBuf& nb = pb[(h + 1) & 1];
+        if (last && upd) {
+          GR_TRY(hop(X, ldx, K, out, ldo, relu, nullptr, 0, 0.f));
+        } else if (last) {
+          GR_TRY(hop(X, ldx, K, T, ld4(K1), false, nullptr, 0, 0.f));
+        } else {
+          GR_TRY(hop(X, ldx, K, nb.mine, nb.ld, false, nullptr, 0, 0.f));
+          GR_TRY(allgather(c, nb));
+          X = nb.all;
+          ldx = nb.ld;
+        }
+      }
+      if (!upd) {
+        const float* A = hops == 0 ? H : T;
+        const int64_t lda = hops == 0 ? ldh : ld4(K1);
+        GR_TRY(launch_gemm(R, K2, K1, A, lda, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
+      }
+    }
+  } else if (m == GRANII_TAGCN) {
+    if (!upd) {
+      // X_j = S^j H side by side (block stride Kb, 16-byte aligned), one GEMM with the stacked
+      // W_j (padded to Kb rows per block: Wc)
+      const int64_t Kb = round_up(K1, 4), ldc = ld4((hops + 1) * Kb);
+      float* Xc = b.take((size_t)Rr * ldc);
+      float* Wc = b.take((size_t)(hops + 1) * Kb * K2);
+      GatherBuf pb[2] = {gather_buf(b, c, K1), gather_buf(b, c, K1)};
+      void* gw;
+      size_t gn;
+      gemm_ws(b, R, K2, (hops + 1) * Kb, relu ? GRANII_GEMM_RELU : 0, &gw, &gn);
+      if (run) {
+        if (Kb != K1) {  // zero the padding columns / rows so the GEMM adds exact zeros
+          GR_CUDA(cudaMemset2DAsync(Xc + K1, ldc * sizeof(float), 0, (Kb - K1) * sizeof(float), (size_t)R, st));
+          for (int j = 1; j <= hops; ++j)
+            GR_CUDA(cudaMemset2DAsync(Xc + j * Kb + K1, ldc * sizeof(float), 0, (Kb - K1) * sizeof(float),
+                                      (size_t)R, st));
+          GR_CUDA(cudaMemsetAsync(Wc, 0, sizeof(float) * (size_t)(hops + 1) * Kb * K2, st));
+        }
+        for (int j = 0; j <= hops; ++j)
+          GR_CUDA(cudaMemcpyAsync(Wc + (int64_t)j * Kb * K2, a->W + (int64_t)j * K1 * K2,
+                                  sizeof(float) * (size_t)K1 * K2, cudaMemcpyDeviceToDevice, st));
+        GR_TRY(launch_copy_rows(R, K1, H, ldh, Xc, ldc, st));  // X_0 = H
+        const float* X = H_all;
+        int64_t ldx = ldh;
+        for (int j = 1; j <= hops; ++j) {
+          float* dst = Xc + (int64_t)(j)*Kb;
+          if (c.dist()) {
+            GatherBuf& nb = pb[j & 1];
+            GR_TRY(hop(X, ldx, K1, nb.mine, nb.ld, false, nullptr, 0, 0.f));
+            GR_TRY(launch_copy_rows(R, K1, nb.mine, nb.ld, dst, ldc, st));
+            if (j < hops) GR_TRY(allgather(c, nb));
+            X = nb.all;
+            ldx = nb.ld;
+          } else {
+            GR_TRY(hop(X, ldx, K1, dst, ldc, false, nullptr, 0, 0.f));
+            X = dst;
+            ldx = ldc;
+          }
+        }
+        GR_TRY(launch_gemm(R, K2, (hops + 1) * Kb, Xc, ldc, Wc, K2, out, ldo, nullptr,
+                           relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
+      }
+    } else {
+      // Horner: P = H [W_0 | ... | W_k] (one GEMM, blocks of stride Kb2), Z = P_k,
+      // Z = S Z + P_j for j = k-1..0 (the addend fused in the SpMM epilogue)
+      const int64_t Kb2 = round_up(K2, 4), NP = (hops + 1) * Kb2, ldp = ld4(NP);
+      float* P = b.take((size_t)Rr * ldp);
+      float* Wh = b.take((size_t)K1 * NP);
+      GatherBuf pb[2] = {gather_buf(b, c, K2), gather_buf(b, c, K2)};
+      void* gw;
+      size_t gn;
+      gemm_ws(b, R, NP, K1, 0, &gw, &gn);
+      void* gw0;
+      size_t gn0;
+      gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw0, &gn0);
+      if (run) {
+        if (hops == 0) {
+          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw0, gn0,
+                             st));
+        } else {
+          if (Kb2 != K2) GR_CUDA(cudaMemsetAsync(Wh, 0, sizeof(float) * (size_t)K1 * NP, st));
+          for (int j = 0; j <= hops; ++j)  // W_j (K1 x K2) into columns [j Kb2, j Kb2 + K2) of Wh
+            GR_CUDA(cudaMemcpy2DAsync(Wh + (int64_t)j * Kb2, NP * sizeof(float), a->W + (int64_t)j * K1 * K2,
+                                      K2 * sizeof(float), K2 * sizeof(float), (size_t)K1, cudaMemcpyDeviceToDevice,
+                                      st));
+          GR_TRY(launch_gemm(R, NP, K1, H, ldh, Wh, NP, P, ldp, nullptr, 0, gw, gn, st));
+          const float* X = P + (int64_t)hops * Kb2;
+          int64_t ldx = ldp;
+          if (c.dist()) {
+            GR_TRY(launch_copy_rows(R, K2, X, ldp, pb[0].mine, pb[0].ld, st));
+            GR_TRY(allgather(c, pb[0]));
+            X = pb[0].all;
+            ldx = pb[0].ld;
+          }
+          for (int j = hops - 1; j >= 0; --j) {
+            const float* Bj = P + (int64_t)j * Kb2;
+            if (j == 0) {
+              GR_TRY(hop(X, ldx, K2, out, ldo, relu, Bj, ldp, 1.f));
+            } else {
+              GatherBuf& nb = pb[(hops - j) & 1];
+              GR_TRY(hop(X, ldx, K2, nb.mine, nb.ld, false, Bj, ldp, 1.f));
+              GR_TRY(allgather(c, nb));
+              X = nb.all;
+              ldx = nb.ld;
+            }
+          }
+        }
+      }
+    }
+  } else {  // GIN
+    const int64_t Kh = a->Kh;
+    GatherBuf pg;
+    if (upd) pg = gather_buf(b, c, Kh);
+    float* U = b.take((size_t)Rr * ld4(upd ? Kh : K1));
+    float* V = upd ? nullptr : b.take((size_t)Rr * ld4(Kh));
+    void* gw1;
+    size_t gn1;
+    gemm_ws(b, R, Kh, K1, GRANII_GEMM_RELU, &gw1, &gn1);
+    void* gw2;
+    size_t gn2;
+    gemm_ws(b, R, K2, Kh, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
+    if (run) {
+      // agg(X) = Σ_{Ã} X_j + ε X_i: PRE folds ε into the diagonal values, DYN adds ε X_i in the epilogue
+      if (!upd) {
+        GR_TRY(launch_spmm_ex(g, vals, H_all, ldh, K1, U, ld4(K1), nullptr, nullptr, false, dyn ? H : nullptr, ldh,
+                              a->eps, st));
+        GR_TRY(launch_gemm(R, Kh, K1, U, ld4(K1), a->W, Kh, V, ld4(Kh), nullptr, GRANII_GEMM_RELU, gw1, gn1, st));
+        GR_TRY(launch_gemm(R, K2, Kh, V, ld4(Kh), a->W2, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
+                           st));
+      } else {
+        GR_TRY(launch_gemm(R, Kh, K1, H, ldh, a->W, Kh, pg.mine, pg.ld, nullptr, 0, gw1, gn1, st));
+        GR_TRY(allgather(c, pg));
+        GR_TRY(launch_spmm_ex(g, vals, pg.all, pg.ld, Kh, U, ld4(Kh), nullptr, nullptr, true, dyn ? pg.mine : nullptr,
+                              pg.ld, a->eps, st));
+        GR_TRY(launch_gemm(R, K2, Kh, U, ld4(Kh), a->W2, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
+                           st));
+      }
+    }
+  }
+  if (ws_size) *ws_size = b.off + 1024;
+  return GRANII_OK;
+}
+
 // ---------------------------------------------------------------- forward (plan + run)
 // Running with base == nullptr only sizes the workspace (no launches).
 static granii_status forward_impl(const Ctx& c, granii_model m, granii_composition comp, const granii_layer_args* a,
@@ -115,6 +337,8 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
   const bool relu = a->act == GRANII_ACT_RELU;
   const cudaStream_t st = c.st;
   if (saved_floats) *saved_floats = 0;
+  if (m == GRANII_SGC || m == GRANII_TAGCN || m == GRANII_GIN)
+    return ext_forward_impl(c, m, comp, a, out, ldo, ws_base, ws_size);
 
   // H with a 16-byte row stride for the TMA GEMM path / vector gathers
   const float* H = a->H;
@@ -509,16 +733,19 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   return GRANII_OK;
 }
 
-granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_composition comp, int64_t K1,
-                              int64_t K2, size_t* ws, size_t* saved_floats) {
+granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_composition comp,
+                              const granii_layer_args* shape, size_t* ws, size_t* saved_floats) {
   // size for the distributed layout whenever the graph is partitioned
   granii_comm_s fake;
   fake.world = g->world;
   fake.rank = g->rank;
   Ctx c{g, g->world > 1 ? &fake : nullptr, nullptr};
+  const int64_t K1 = shape->K1, K2 = shape->K2;
   granii_layer_args a{};
   a.K1 = K1;
   a.K2 = K2;
+  a.hops = shape->hops;
+  a.Kh = shape->Kh;
   a.ldh = K1;  // worst case: unaligned H needs a padded copy
   a.act = GRANII_ACT_RELU;
   size_t f = 0, f2 = 0, bwd = 0, sf = 0;
@@ -531,7 +758,7 @@ granii_status layer_workspace(const granii_graph_s* g, granii_model m, granii_co
   }
   if (m == GRANII_GCN)
     GR_TRY(backward_impl(c, comp, &a, nullptr, K2, nullptr, K2, nullptr, (float*)1, K1, nullptr, nullptr, &bwd));
-  else
+  else if (m == GRANII_GAT)
     GR_TRY(gat_backward_impl(c, comp, &a, nullptr, K2, nullptr, K2, nullptr, nullptr, K1, nullptr, nullptr, &bwd));
   *ws = std::max(f, bwd);
   if (saved_floats) *saved_floats = sf;

@@ -196,6 +196,30 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
   return 1e30;
 }
 
+// SGC / TAGCN / GIN (layer.cu ext_forward_impl; reading R23): k hops of the GCN SpMM (with an
+// all-gather before each on several GPUs), TAGCN's concatenated GEMM (AGG) or wide GEMM (UPD),
+// GIN's two MLP GEMMs around one aggregation at K1 (AGG) or Kh (UPD)
+double ext_forward_cost(const CostModel& m, const In& in, int comp, double K1, double K2, double k, double Kh) {
+  const bool dyn = (comp & 3) >= 2, upd = (comp & 1) != 0;
+  const int base = comp & ~3;
+  const int sp = base == GRANII_GIN_PRE_AGG ? (dyn ? P_SPMM_U : P_SPMM_W) : (dyn ? P_SPMM_U_CS : P_SPMM_W);
+  double t = dyn ? 0.0 : cost(m, in, P_SDDMM1, 0);
+  if (base == GRANII_SGC_PRE_AGG) {
+    const double K = upd ? K2 : K1;
+    t += cost(m, in, P_GEMM, K1, K2) + k * (cost(m, in, P_ALLGATHER, K) + cost(m, in, sp, K));
+  } else if (base == GRANII_TAGCN_PRE_AGG) {
+    if (upd)
+      t += cost(m, in, P_GEMM, K1, (k + 1) * K2) + k * (cost(m, in, P_ALLGATHER, K2) + cost(m, in, sp, K2));
+    else
+      t += cost(m, in, P_ELEMENTWISE, K1) + k * (cost(m, in, P_ALLGATHER, K1) + cost(m, in, sp, K1)) +
+           cost(m, in, P_GEMM, (k + 1) * K1, K2);
+  } else {
+    const double K = upd ? Kh : K1;
+    t += cost(m, in, P_GEMM, K1, Kh) + cost(m, in, P_GEMM, Kh, K2) + cost(m, in, P_ALLGATHER, K) + cost(m, in, sp, K);
+  }
+  return t;
+}
+
 // backward of the compositions (layer.cu backward_impl / gat_backward_impl), ReLU mask included
 double backward_cost(const CostModel& m, const In& in, int comp, double K1, double K2, bool need_dH) {
   double t = cost(m, in, P_ELEMENTWISE, K2) + cost(m, in, P_GEMM_TN, K1, K2);
@@ -237,8 +261,10 @@ static In inputs_of(const granii_graph_s* g) {
             (double)g->world, (double)g->n_seg};
 }
 
-granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K1, int64_t K2, const char* path,
-                          uint32_t flags, granii_composition* out, int32_t* cands, double* pred, int32_t* ncand) {
+granii_status select_impl(const granii_graph_s* g, granii_model model, const granii_layer_args* shape,
+                          const char* path, uint32_t flags, granii_composition* out, int32_t* cands, double* pred,
+                          int32_t* ncand) {
+  const int64_t K1 = shape->K1, K2 = shape->K2;
   if (!path || !*path) path = getenv("GRANII_CALIB");
   CostModel m;
   GR_TRY(load_model(path, &m));
@@ -252,15 +278,26 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, int64_t K
     if (!prefilter) c = {GRANII_GCN_PRE_AGG, GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_AGG, GRANII_GCN_DYN_UPD};
     else if (K1 >= K2) c = {GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_UPD};   // group ">=": update first
     else c = {GRANII_GCN_PRE_AGG, GRANII_GCN_DYN_AGG};                 // group "<": aggregate first
-  } else {
+  } else if (model == GRANII_GAT) {
     c = {GRANII_GAT_REUSE, GRANII_GAT_RECOMP};
+  } else {
+    // SGC / TAGCN: the GCN embedding-size rule on (K1, K2); GIN: on (K1, Kh), the width the
+    // aggregation runs at (R11 / R23)
+    const int base = model == GRANII_SGC ? GRANII_SGC_PRE_AGG : model == GRANII_TAGCN ? GRANII_TAGCN_PRE_AGG
+                                                                                         : GRANII_GIN_PRE_AGG;
+    const int64_t Kout = model == GRANII_GIN ? shape->Kh : K2;
+    if (!prefilter) c = {base, base + 1, base + 2, base + 3};
+    else if (K1 >= Kout) c = {base + 1, base + 3};
+    else c = {base, base + 2};
   }
-  const bool train = (flags & GRANII_SELECT_TRAINING) != 0;
+  const bool train = (flags & GRANII_SELECT_TRAINING) != 0 && model <= GRANII_GAT;
   const bool need_dH = !(flags & GRANII_SELECT_INPUT_LAYER);
   int best = -1;
   double bc = 0;
   for (size_t i = 0; i < c.size(); ++i) {
-    double t = forward_cost(m, in, c[i], (double)K1, (double)K2);
+    double t = model <= GRANII_GAT
+                   ? forward_cost(m, in, c[i], (double)K1, (double)K2)
+                   : ext_forward_cost(m, in, c[i], (double)K1, (double)K2, (double)shape->hops, (double)shape->Kh);
     if (train) t += backward_cost(m, in, c[i], (double)K1, (double)K2, need_dH);
     if (cands) cands[i] = c[i];
     if (pred) pred[i] = t;

@@ -71,6 +71,11 @@ struct SpmmArgs {
   const int64_t* __restrict__ seg_hi;
   float* __restrict__ partial;
   int64_t ldp;
+  // optional dense addend fused in the epilogue: Y_i = act(rs_i * sum + beta * B_i)
+  // (GIN's ε self term, TAGCN's Horner step); B holds the owned rows
+  const float* __restrict__ B;
+  int64_t ldb;
+  float beta;
 };
 
 // One chunk of 32 entries of a row, one per lane: column id and weight.  Lanes
@@ -170,14 +175,17 @@ __device__ __forceinline__ void reduce_groups(float (&acc)[NJ][VEC]) {
 
 template <int LPG, int NJ, int VEC>
 __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], const float (&acc)[NJ][VEC], float s,
-                                          int relu) {
+                                          int relu, const float* b = nullptr, float beta = 0.f) {
 #pragma unroll
   for (int j = 0; j < NJ; ++j) {
     if (!colok[j]) continue;
     float o[VEC];
+    float bv[VEC];
+    if (b) ldv<VEC>(b + j * LPG * VEC, bv);
 #pragma unroll
     for (int v = 0; v < VEC; ++v) {
       o[v] = acc[j][v] * s;
+      if (b) o[v] = fmaf(beta, bv[v], o[v]);
       if (relu) o[v] = fmaxf(o[v], 0.f);
     }
     stv<VEC>(y + j * LPG * VEC, o);
@@ -221,7 +229,7 @@ __global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
     reduce_groups<LPG>(acc);
     if (grp == 0)
       store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
-                     a.relu);
+                     a.relu, a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
   }
 }
 
@@ -274,7 +282,7 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
           for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
     }
     store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
-                   a.relu);
+                   a.relu, a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
   }
 }
 
@@ -282,7 +290,8 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
 __global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heavy_rows,
                                const int32_t* __restrict__ seg_ptr, const float* __restrict__ partial, int64_t ldp,
                                int64_t k0, int64_t kw, float* __restrict__ Y, int64_t ldy,
-                               const float* __restrict__ rs, int relu) {
+                               const float* __restrict__ rs, int relu, const float* __restrict__ B, int64_t ldb,
+                               float beta) {
   const int64_t total = n_heavy * kw;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t h = i / kw, k = i % kw;
@@ -290,6 +299,7 @@ __global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heav
     for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) s += partial[(int64_t)q * ldp + k];
     const int64_t row = heavy_rows[h];
     s *= rs ? rs[row] : 1.f;
+    if (B) s = fmaf(beta, B[row * ldb + k0 + k], s);
     if (relu) s = fmaxf(s, 0.f);
     Y[row * ldy + k0 + k] = s;
   }
@@ -389,13 +399,20 @@ int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t 
 
 granii_status launch_spmm(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                           float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, cudaStream_t st) {
+  return launch_spmm_ex(g, vals, X, ldx, K, Y, ldy, rs, cs, relu, nullptr, 0, 0.f, st);
+}
+
+granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                             float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                             int64_t ldb, float beta, cudaStream_t st) {
   if (g->n_rows == 0 || K == 0) return GRANII_OK;
   DevInfo di;
   GR_TRY(dev_info(&di));
-  const bool vec4 = (ldx % 4 == 0) && (ldy % 4 == 0) && ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0);
+  const bool vec4 = (ldx % 4 == 0) && (ldy % 4 == 0) && ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0) &&
+                    (!B || ((ldb % 4 == 0) && ((uintptr_t)B % 16 == 0)));
   const bool warp_mode = g->avg_deg() >= 16.f;
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
-             g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0};
+             g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0, B, ldb, beta};
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
   if (g->n_seg > 0) {  // stream-ordered scratch for the heavy-row partials (pool-backed, no sync)
     a.ldp = round_up(kw, 4);
@@ -404,7 +421,8 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
   // algorithmic bytes: per entry col id (+w, +cs) + one K-row of X;
   // per row row_ptr + the K-row of Y (+rs)
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
-  const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) + R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0));
+  const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) +
+                       R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0) + (B ? 4.0 * K : 0.0));
   ProfScope ps("spmm", st, bytes, 2.0 * nnz * K, (int)ceil_div(K, kw));
   for (int64_t k0 = 0; k0 < K; k0 += kw) {
     a.k0 = k0;
@@ -414,7 +432,7 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
     if (g->n_seg > 0) {
       const int64_t tot = g->n_heavy * a.kw;
       k_spmm_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(
-          g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0);
+          g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0, B, ldb, beta);
       GR_CHECK_LAUNCH();
       ps.add_launches(1);
     }

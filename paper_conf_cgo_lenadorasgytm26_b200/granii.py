@@ -27,13 +27,20 @@ ADD_SELF_LOOPS, SYMMETRIZE = 0x1, 0x2
 EPI_RELU = 0x1
 SDDMM_DOT, SDDMM_ADD, SDDMM_LEAKYRELU, SDDMM_ROW_SOFTMAX = 0x0, 0x1, 0x10, 0x20
 GEMM_TRANS_A, GEMM_TRANS_B, GEMM_RELU, GEMM_NO_STORE = 0x1, 0x2, 0x4, 0x8
-GCN, GAT = 0, 1
+GCN, GAT, SGC, TAGCN, GIN = 0, 1, 2, 3, 4
 GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD = 0, 1, 2, 3
 GAT_REUSE, GAT_RECOMP = 16, 17
 GCN_COMPS = (GCN_PRE_AGG, GCN_PRE_UPD, GCN_DYN_AGG, GCN_DYN_UPD)
 GAT_COMPS = (GAT_REUSE, GAT_RECOMP)
+SGC_COMPS = (32, 33, 34, 35)
+TAGCN_COMPS = (48, 49, 50, 51)
+GIN_COMPS = (64, 65, 66, 67)
+COMPS = {GCN: GCN_COMPS, GAT: GAT_COMPS, SGC: SGC_COMPS, TAGCN: TAGCN_COMPS, GIN: GIN_COMPS}
 COMP_NAMES = {0: "GCN_PRE_AGG", 1: "GCN_PRE_UPD", 2: "GCN_DYN_AGG", 3: "GCN_DYN_UPD", 16: "GAT_REUSE",
               17: "GAT_RECOMP"}
+for _m, _base in (("SGC", 32), ("TAGCN", 48), ("GIN", 64)):
+    for _i, _v in enumerate(("PRE_AGG", "PRE_UPD", "DYN_AGG", "DYN_UPD")):
+        COMP_NAMES[_base + _i] = f"{_m}_{_v}"
 ACT_NONE, ACT_RELU = 0, 1
 ATTN_ADDITIVE, ATTN_DOT = 0, 1
 SELECT_NO_PREFILTER, SELECT_TRAINING, SELECT_INPUT_LAYER = 0x1, 0x2, 0x4
@@ -57,7 +64,7 @@ class gemm_epilogue(ctypes.Structure):
 class layer_args(ctypes.Structure):
     _fields_ = [("K1", _i64), ("K2", _i64), ("H", _p), ("ldh", _i64), ("W", _p), ("a_l", _p), ("a_r", _p),
                 ("act", _u32), ("attn", _u32), ("workspace", _p), ("workspace_bytes", _sz), ("comm", _p),
-                ("d_a_l", _p), ("d_a_r", _p)]
+                ("d_a_l", _p), ("d_a_r", _p), ("hops", _i32), ("eps", _f), ("Kh", _i64), ("W2", _p)]
 
 
 _SIGS = {
@@ -82,6 +89,11 @@ _SIGS = {
                              ctypes.c_int),
     "granii_layer_backward": ([_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(layer_args), _p, _i64, _p, _i64, _p,
                                _p, _i64, _p, _p], ctypes.c_int),
+    "granii_layer_workspace_size_ex": ([_p, ctypes.c_int, ctypes.c_int, ctypes.POINTER(layer_args),
+                                        ctypes.POINTER(_sz), ctypes.POINTER(_sz)], ctypes.c_int),
+    "granii_select_ex": ([_p, ctypes.c_int, ctypes.POINTER(layer_args), ctypes.c_char_p, _u32,
+                          ctypes.POINTER(ctypes.c_int), ctypes.POINTER(_i32), ctypes.POINTER(ctypes.c_double),
+                          ctypes.POINTER(_i32)], ctypes.c_int),
     "granii_select": ([_p, ctypes.c_int, _i64, _i64, ctypes.c_char_p, _u32, ctypes.POINTER(ctypes.c_int),
                        ctypes.POINTER(_i32), ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i32)], ctypes.c_int),
     "granii_cost_features": ([_p, _i32, _i64, _i64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i32),
@@ -259,11 +271,34 @@ def granii_layer_workspace_size(g: Graph, model: int, comp: int, K1: int, K2: in
 
 
 def make_layer_args(K1, K2, H, W, a_l=None, a_r=None, act=ACT_RELU, attn=ATTN_ADDITIVE, workspace=None,
-                    comm=None, d_a_l=None, d_a_r=None) -> layer_args:
-    """d_a_l / d_a_r: GAT backward outputs (dL/da_l, dL/da_r), ignored by the forward."""
-    return layer_args(K1, K2, _ptr(H), _ld(H), _ptr(W), _ptr(a_l), _ptr(a_r), act, attn, _ptr(workspace),
-                      workspace.numel() if workspace is not None else 0, comm.handle if comm is not None else None,
-                      _ptr(d_a_l), _ptr(d_a_r))
+                    comm=None, d_a_l=None, d_a_r=None, hops=0, eps=0.0, Kh=0, W2=None) -> layer_args:
+    """d_a_l / d_a_r: GAT backward outputs (dL/da_l, dL/da_r), ignored by the forward.
+    hops (SGC / TAGCN), eps / Kh / W2 (GIN): the other models' shape and weights."""
+    return layer_args(K1, K2, _ptr(H), _ld(H) if H is not None else K1, _ptr(W), _ptr(a_l), _ptr(a_r), act, attn,
+                      _ptr(workspace), workspace.numel() if workspace is not None else 0,
+                      comm.handle if comm is not None else None, _ptr(d_a_l), _ptr(d_a_r), hops, eps, Kh, _ptr(W2))
+
+
+def shape_args(K1, K2, hops=0, Kh=0) -> layer_args:
+    """layer_args with only the shape fields set (sizing / selection)."""
+    return layer_args(K1=K1, K2=K2, ldh=K1, hops=hops, Kh=Kh)
+
+
+def granii_layer_workspace_size_ex(g: Graph, model: int, comp: int, args: layer_args):
+    ws, sv = _sz(), _sz()
+    _check(_lib.granii_layer_workspace_size_ex(g.handle, model, comp, ctypes.byref(args), ctypes.byref(ws),
+                                               ctypes.byref(sv)), "granii_layer_workspace_size_ex")
+    return ws.value, sv.value
+
+
+def granii_select_ex(g: Graph, model: int, args: layer_args, calib_path: str | None = None, flags: int = 0):
+    out = ctypes.c_int()
+    cands = (_i32 * MAX_CANDIDATES)()
+    pred = (ctypes.c_double * MAX_CANDIDATES)()
+    n = _i32()
+    _check(_lib.granii_select_ex(g.handle, model, ctypes.byref(args), calib_path.encode() if calib_path else None,
+                                 flags, ctypes.byref(out), cands, pred, ctypes.byref(n)), "granii_select_ex")
+    return out.value, {cands[i]: pred[i] for i in range(n.value)}
 
 
 def granii_layer_forward(g: Graph, model: int, comp: int, args: layer_args, out: torch.Tensor, saved=None,

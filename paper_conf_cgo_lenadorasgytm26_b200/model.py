@@ -40,9 +40,13 @@ class LayerSpec:
     act: int = G.ACT_RELU
     attn: int = G.ATTN_ADDITIVE
     comp: int | None = None     # None -> chosen by granii_select
-    W: torch.Tensor | None = None
+    W: torch.Tensor | None = None  # TAGCN: (hops+1, K1, K2) stacked; GIN: K1 x Kh
     a_l: torch.Tensor | None = None
     a_r: torch.Tensor | None = None
+    hops: int = 2               # SGC / TAGCN
+    eps: float = 0.0            # GIN
+    Kh: int = 0                 # GIN hidden width
+    W2: torch.Tensor | None = None  # GIN: Kh x K2
     predicted_ms: dict = field(default_factory=dict)
 
 
@@ -61,11 +65,12 @@ class GNN:
                 fl = select_flags
                 if training:
                     fl |= G.SELECT_TRAINING | (G.SELECT_INPUT_LAYER if i == 0 else 0)
-                L.comp, L.predicted_ms = G.granii_select(graph, L.model, L.K1, L.K2, calib_path, fl)
+                L.comp, L.predicted_ms = G.granii_select_ex(graph, L.model, G.shape_args(L.K1, L.K2, L.hops, L.Kh),
+                                                            calib_path, fl)
         ws = 0
         self.saved_floats = []
         for L in layers:
-            w, s = G.granii_layer_workspace_size(graph, L.model, L.comp, L.K1, L.K2)
+            w, s = G.granii_layer_workspace_size_ex(graph, L.model, L.comp, G.shape_args(L.K1, L.K2, L.hops, L.Kh))
             ws = max(ws, w)
             self.saved_floats.append(s)
         self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=device)
@@ -84,7 +89,7 @@ class GNN:
         L = self.layers[i]
         da = self.da[i] or (None, None)
         return G.make_layer_args(L.K1, L.K2, H, L.W, L.a_l, L.a_r, L.act, L.attn, self.workspace, self.comm,
-                                 da[0], da[1])
+                                 da[0], da[1], L.hops, L.eps, L.Kh, L.W2)
 
     def forward(self, H: torch.Tensor) -> torch.Tensor:
         x = H

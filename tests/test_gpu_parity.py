@@ -455,6 +455,90 @@ def test_gat_backward_deterministic_and_input_layer(G):
     assert torch.equal(runs[0][0], runs[2][0]) and runs[2][2] is None   # no dH: same dW
 
 
+# ------------------------------------------------------------------ N3: SGC / TAGCN / GIN (reading R23)
+def err_act(y, r, r_pre):
+    """row-normwise error of σ(y) against σ(r), normalised by the pre-activation row: ReLU is
+    1-Lipschitz, so the error is the pre-activation's (R19 on the value the kernels compute)"""
+    y, r, p = (np.asarray(x, np.float64) for x in (y, r, r_pre))
+    d = np.abs(y - r).max(1)
+    a = np.abs(p).max(1)
+    return float(np.max(d / np.maximum(a, 1e-6 * a.max())))
+
+
+def run_ext(G, c, spec, H, aligned=True):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN
+    Hd = pad(H) if aligned else H.to(DEV).contiguous()
+    net = GNN(c.g, [spec], DEV)
+    out = net.forward(Hd)
+    torch.cuda.synchronize()
+    return out.cpu()
+
+
+@pytest.mark.parametrize("comp", [32, 33, 34, 35])
+@pytest.mark.parametrize("name,K1,K2,hops", [("pubmed", 32, 16, 2), ("dense", 48, 64, 3), ("tiny", 3, 5, 1),
+                                              ("cora", 1433, 16, 2), ("sparse", 64, 64, 0)])
+def test_sgc_forward_every_composition(G, comp, name, K1, K2, hops):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import LayerSpec
+    c = case(G, name)
+    H = synth.features(80, c.n, K1)
+    W = synth.glorot(80, 2, K1, K2, (K1, K2))
+    for act in (0, 1):
+        out = run_ext(G, c, LayerSpec(G.SGC, K1, K2, act, comp=comp, W=W.to(DEV), hops=hops), H, aligned=K1 % 4 == 0)
+        ref = O.sgc_forward(comp, c.rp, c.ci, H, W, hops, act)
+        assert err_act(out, ref, O.sgc_forward(comp, c.rp, c.ci, H, W, hops, 0)) <= TOL, (G.COMP_NAMES[comp], act)
+
+
+@pytest.mark.parametrize("comp", [48, 49, 50, 51])
+@pytest.mark.parametrize("name,K1,K2,hops", [("pubmed", 32, 16, 2), ("dense", 30, 18, 3), ("tiny", 3, 5, 1),
+                                              ("cora", 1433, 16, 2), ("sparse", 64, 128, 0)])
+def test_tagcn_forward_every_composition(G, comp, name, K1, K2, hops):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import LayerSpec
+    c = case(G, name)
+    H = synth.features(81, c.n, K1)
+    Ws = synth.glorot(81, 2, K1, K2, (hops + 1, K1, K2))
+    for act in (0, 1):
+        spec = LayerSpec(G.TAGCN, K1, K2, act, comp=comp, W=Ws.to(DEV).contiguous(), hops=hops)
+        out = run_ext(G, c, spec, H, aligned=K1 % 4 == 0)
+        ref = O.tagcn_forward(comp, c.rp, c.ci, H, Ws, act)
+        assert err_act(out, ref, O.tagcn_forward(comp, c.rp, c.ci, H, Ws, 0)) <= TOL, (G.COMP_NAMES[comp], act)
+
+
+@pytest.mark.parametrize("comp", [64, 65, 66, 67])
+@pytest.mark.parametrize("name,K1,Kh,K2", [("pubmed", 32, 64, 16), ("dense", 48, 24, 40), ("tiny", 3, 7, 5),
+                                            ("cora", 1433, 64, 16), ("sparse", 128, 128, 47)])
+def test_gin_forward_every_composition(G, comp, name, K1, Kh, K2):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import LayerSpec
+    c = case(G, name)
+    H = synth.features(82, c.n, K1)
+    W1 = synth.glorot(82, 2, K1, Kh, (K1, Kh))
+    W2 = synth.glorot(82, 3, Kh, K2, (Kh, K2))
+    for eps, act in ((0.0, 0), (0.3, 1)):
+        spec = LayerSpec(G.GIN, K1, K2, act, comp=comp, W=W1.to(DEV), eps=eps, Kh=Kh, W2=W2.to(DEV))
+        out = run_ext(G, c, spec, H, aligned=K1 % 4 == 0)
+        ref = O.gin_forward(comp, c.rp, c.ci, H, W1, W2, eps, act)
+        pre = O.gin_forward(comp, c.rp, c.ci, H, W1, W2, eps, 0)
+        assert err_act(out, ref, pre) <= TOL, (G.COMP_NAMES[comp], eps, act)
+
+
+def test_ext_models_select_and_reject_backward(G):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    c = case(G, "pubmed")
+    comp, pred = G.granii_select_ex(c.g, G.SGC, G.shape_args(256, 32, hops=2))
+    assert comp in (33, 35) and set(pred) == {33, 35}                      # K1 >= K2: update first
+    comp, pred = G.granii_select_ex(c.g, G.TAGCN, G.shape_args(32, 256, hops=2))
+    assert comp in (48, 50) and set(pred) == {48, 50}
+    comp, pred = G.granii_select_ex(c.g, G.GIN, G.shape_args(32, 16, Kh=256))
+    assert comp in (64, 66)                                                 # K1 < Kh: aggregate first
+    comp, pred = G.granii_select_ex(c.g, G.GIN, G.shape_args(32, 16, Kh=256), flags=G.SELECT_NO_PREFILTER)
+    assert set(pred) == {64, 65, 66, 67} and comp == min(pred, key=lambda k: (pred[k], k))
+    W = synth.glorot(83, 2, 32, 16, (32, 16)).to(DEV)
+    net = GNN(c.g, [LayerSpec(G.SGC, 32, 16, 0, W=W, hops=2)], DEV)
+    H = pad(synth.features(83, c.n, 32))
+    net.forward(H)
+    with pytest.raises(G.GraniiError):
+        net.backward(pad(torch.zeros(c.n, 16)))
+
+
 def test_layer_determinism_and_comp_agreement(G):
     c = case(G, "dense")
     outs = []
