@@ -45,6 +45,11 @@ WORKLOADS = {
     "pubmed-gcn2-train": dict(graph="pubmed", model="gcn", dims=[256, 32, 32], train=True),
     "products-gat2-train": dict(graph="products", model="gat", dims=[100, 256, 47], train=True),
     "pubmed-gat2-train": dict(graph="pubmed", model="gat", dims=[64, 256, 32], train=True),
+    # N3 models (reading R23), inference: SGC / TAGCN with k = 2 hops, GIN with hidden width Kh
+    "reddit-sgc-infer": dict(graph="reddit", model="sgc", dims=[602, 41], hops=2, train=False),
+    "reddit-tagcn-infer": dict(graph="reddit", model="tagcn", dims=[602, 41], hops=2, train=False),
+    "reddit-gin-infer": dict(graph="reddit", model="gin", dims=[602, 41], kh=256, train=False),
+    "products-sgc-infer": dict(graph="products", model="sgc", dims=[100, 47], hops=2, train=False),
 }
 
 
@@ -102,21 +107,37 @@ class Clocks:
                 "reasons": reasons, "samples": len(self.rows)}
 
 
+MODEL_IDS = {"gcn": 0, "gat": 1, "sgc": 2, "tagcn": 3, "gin": 4}
+
+
+def layer_spec(G, spec, i, k1, k2, dev, seed, act, comp=None):
+    """layer i of the workload's model with seeded random-init weights"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import LayerSpec
+    model = MODEL_IDS[spec["model"]]
+    hops, kh = spec.get("hops", 2), spec.get("kh", 0)
+    if model == G.TAGCN:
+        W = synth.glorot(seed + 2, i, k1, k2, (hops + 1, k1, k2), device=dev).contiguous()
+    elif model == G.GIN:
+        W = synth.glorot(seed + 2, i, k1, kh, (k1, kh), device=dev).contiguous()
+    else:
+        W = synth.glorot(seed + 2, i, k1, k2, (k1, k2), device=dev).contiguous()
+    al = ar = W2 = None
+    if model == G.GAT:
+        al = synth.glorot(seed + 3, 2 * i, 2 * k2, 1, (k2,), device=dev)
+        ar = synth.glorot(seed + 3, 2 * i + 1, 2 * k2, 1, (k2,), device=dev)
+    if model == G.GIN:
+        W2 = synth.glorot(seed + 4, i, kh, k2, (kh, k2), device=dev).contiguous()
+    return LayerSpec(model, k1, k2, act, G.ATTN_ADDITIVE, comp=comp, W=W, a_l=al, a_r=ar, hops=hops, eps=0.1, Kh=kh,
+                     W2=W2)
+
+
 def build_model(G, M, spec, g, dev, comm, gen_seed=0):
-    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN
     dims = spec["dims"]
     layers = []
     for i in range(len(dims) - 1):
-        k1, k2 = dims[i], dims[i + 1]
         last = i == len(dims) - 2
-        W = synth.glorot(gen_seed + 2, i, k1, k2, (k1, k2), device=dev).contiguous()
-        if spec["model"] == "gcn":
-            layers.append(LayerSpec(G.GCN, k1, k2, G.ACT_NONE if last else G.ACT_RELU, W=W))
-        else:
-            al = synth.glorot(gen_seed + 3, 2 * i, 2 * k2, 1, (k2,), device=dev)
-            ar = synth.glorot(gen_seed + 3, 2 * i + 1, 2 * k2, 1, (k2,), device=dev)
-            layers.append(LayerSpec(G.GAT, k1, k2, G.ACT_NONE if last else G.ACT_RELU, G.ATTN_ADDITIVE, W=W,
-                                    a_l=al, a_r=ar))
+        layers.append(layer_spec(G, spec, i, dims[i], dims[i + 1], dev, gen_seed, G.ACT_NONE if last else G.ACT_RELU))
     return GNN(g, layers, dev, comm, training=spec["train"])
 
 
@@ -290,7 +311,9 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     n_layers = len(dims) - 1
-    edges_per_step = float(info.nnz) * n_layers
+    # stored entries processed per step: one aggregation pass per layer (k per SGC / TAGCN layer)
+    passes = spec.get("hops", 1) if spec["model"] in ("sgc", "tagcn") else 1
+    edges_per_step = float(info.nnz) * n_layers * passes
     value = edges_per_step / (ms / 1e3)
 
     # roofline of the dominant kernel (largest summed time in the timed region)
@@ -382,7 +405,10 @@ def main():
         result["selector"] = regret(G, spec, g, dev, comm, H, world, dist if world > 1 else None)
 
     # ---------------------------------------------------------------- CPU oracle baseline
-    if rank == 0 and world == 1 and not args.no_cpu:
+    if rank == 0 and world == 1 and not args.no_cpu and spec["model"] not in ("gcn", "gat"):
+        result["cpu_baseline"] = {"value": None, "reason": "no per-row oracle for the k-hop / MLP models (N3); "
+                                                            "the oracle is exercised by the parity tests"}
+    elif rank == 0 and world == 1 and not args.no_cpu:
         try:
             rp, ci = host_csr(w.n, src, dst, w.symmetrize)
             result["cpu_baseline"] = cpu_oracle_sample(rp, ci, dims, model=spec["model"])
@@ -409,23 +435,21 @@ def regret(G, spec, g, dev, comm, H, world, dist):
     x = H
     for i in range(len(dims) - 1):
         k1, k2 = dims[i], dims[i + 1]
-        model = G.GCN if spec["model"] == "gcn" else G.GAT
-        comps = G.GCN_COMPS if model == G.GCN else G.GAT_COMPS
-        W = synth.glorot(9, i, k1, k2, (k1, k2), device=dev).contiguous()
-        al = synth.uniform_pm1(9, 2 * i, (k2,), device=dev)
-        ar = synth.uniform_pm1(9, 2 * i + 1, (k2,), device=dev)
+        model = MODEL_IDS[spec["model"]]
+        comps = G.COMPS[model]
         if x.shape[1] != k1:
             x = alloc2d(g.n_rows, k1, dev, fill=0.5)
         train = spec["train"]
         need_dH = i > 0                      # the input layer needs no dH (training)
         fl = (G.SELECT_TRAINING | (0 if need_dH else G.SELECT_INPUT_LAYER)) if train else 0
         calib = DEFAULT_CALIB if os.path.exists(DEFAULT_CALIB) else None
-        sel, pred = G.granii_select(g, model, k1, k2, calib, fl)
-        sel_all, pred_all = G.granii_select(g, model, k1, k2, calib, fl | G.SELECT_NO_PREFILTER)
-        sel_paper, _ = G.granii_select(g, model, k1, k2, calib, 0)   # forward-only selection, as the paper
+        shape = G.shape_args(k1, k2, spec.get("hops", 2), spec.get("kh", 0))
+        sel, pred = G.granii_select_ex(g, model, shape, calib, fl)
+        sel_all, pred_all = G.granii_select_ex(g, model, shape, calib, fl | G.SELECT_NO_PREFILTER)
+        sel_paper, _ = G.granii_select_ex(g, model, shape, calib, 0)   # forward-only selection, as the paper
         times = {}
         for c in comps:
-            net = GNN(g, [LayerSpec(model, k1, k2, G.ACT_RELU, comp=c, W=W, a_l=al, a_r=ar)], dev, comm)
+            net = GNN(g, [layer_spec(G, spec, i, k1, k2, dev, 9, G.ACT_RELU, comp=c)], dev, comm)
             gup = alloc2d(g.n_rows, k2, dev, fill=0.01)
 
             def fn():
@@ -444,12 +468,13 @@ def regret(G, spec, g, dev, comm, H, world, dist):
         best = min(times, key=times.get)
         # Config heuristic (L305 / Table VI "Config."): update first iff K1 > K2, DGL-default
         # dynamic normalisation (L355); GAT: WiseGraph recomputes for increasing sizes (L357)
-        if model == G.GCN:
-            cfg = "GCN_DYN_UPD" if k1 > k2 else "GCN_DYN_AGG"
-            static = "GCN_DYN_AGG"
-        else:
+        if model == G.GAT:
             cfg = "GAT_RECOMP" if k1 < k2 else "GAT_REUSE"
             static = "GAT_REUSE"
+        else:
+            pre = spec["model"].upper()
+            cfg = f"{pre}_DYN_UPD" if k1 > k2 else f"{pre}_DYN_AGG"
+            static = f"{pre}_DYN_AGG"
         out[f"layer{i + 1}_{k1}x{k2}"] = {
             "ms": times, "best": best, "selected": G.COMP_NAMES[sel],
             "selected_no_prefilter": G.COMP_NAMES[sel_all],

@@ -164,6 +164,16 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   g->symmetric = sym;
   g->self_loops = loops;
   cudaGetDevice(&g->device);
+  {
+    // the per-call scratch of the hub-segment paths (SpMM partials, segmented softmax) comes
+    // from the stream-ordered pool: keep its memory instead of returning it to the driver at
+    // every synchronisation, so a steady-state step never maps memory on the host path
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, g->device) == cudaSuccess) {
+      uint64_t keep = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+  }
 
   int* d_bad = nullptr;
   unsigned long long* d_acc = nullptr;
@@ -353,6 +363,15 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
       CK(cudaMemcpy(g->seg_heavy, sh.data(), g->n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(g->seg_row, sr.data(), g->n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
     }
+  }
+  // sparse graphs are processed a lane group per row; rows with more than wide_deg entries
+  // (a prefix of the degree-descending order) get a whole warp so they cannot set the tail
+  if (g->n_rows > 0 && g->features[4] > g->wide_deg) {
+    std::vector<int64_t> hrp(g->n_rows + 1);
+    CK(cudaMemcpy(hrp.data(), g->row_ptr, (g->n_rows + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+    int64_t nw = 0;
+    for (int64_t r = 0; r < g->n_rows; ++r) nw += (hrp[r + 1] - hrp[r]) > g->wide_deg;
+    g->n_wide = nw;
   }
   cleanup();
   CK(cudaStreamSynchronize(st));

@@ -94,13 +94,10 @@ __global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, 
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
 template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_a(GatBwdArgs a) {
+__device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
-  const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
-  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (w >= a.n_rows) return;
-  const int32_t r = a.order[w];
+  const int lg = lane % LPG, grp = lane / LPG;
   const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
   const float eli = a.el[r];
   const float ci = a.c[r];
@@ -172,13 +169,10 @@ __global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2
 }
 
 template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bwd_b(GatBwdArgs a) {
+__device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, int lane) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
-  const int lane = threadIdx.x & 31, lg = lane % LPG, grp = lane / LPG;
-  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (w >= a.n_rows) return;
-  const int32_t r = a.order[w];
+  const int lg = lane % LPG, grp = lane / LPG;
   const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
   const float erj = a.er[r];
   float zr[NJ][4], acc[NJ][4];
@@ -253,9 +247,153 @@ __global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bw
   if (lane == 0) a.der[r] = der;
 }
 
+// ---------------------------------------------------------------- sparse graphs: group per row
+// avg degree < 16 (the SpMM's group-per-row regime): an LPG-lane group owns a row, 32/LPG rows
+// per warp, U entries per group in flight; no shuffles inside the (divergent) entry loops, the
+// lane shares are reduced within the group at the end.
+template <int LPG, int NJ, int U>
+__device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0, int lane) {
+  const int lg = lane % LPG;
+  const bool live = t0 < a.n_rows;
+  const int32_t r = live ? a.order[t0] : 0;
+  const int64_t b = live ? a.row_ptr[r] : 0, t = live ? a.row_ptr[r + 1] : 0;
+  const float eli = live ? a.el[r] : 0.f, ci = live ? a.c[r] : 0.f;
+  float xv[NJ][4];
+  gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, live ? a.K : 0, xv);
+  float m = -INFINITY, S = 0.f, Cw = 0.f, D = 0.f;
+  for (int64_t e = b; e < t; e += U) {
+    int32_t j[U];
+    float erj[U];
+    float zv[U][NJ][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      j[u] = __ldg(a.col_idx + (e + u < t ? e + u : t - 1));
+      erj[u] = __ldg(a.er + j[u]);
+      gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (e + u < t) {
+        const float pd = gb_pdot<NJ>(xv, zv[u]);
+        const float z = eli + erj[u];
+        const float ev = gb_lrelu(z);
+        const float sl = z > 0.f ? 1.f : 0.2f;
+        if (ev > m) {
+          const float sc = __expf(m - ev);
+          S = fmaf(S, sc, 1.f);
+          Cw = fmaf(Cw, sc, sl);
+          D = fmaf(D, sc, sl * pd);
+          m = ev;
+        } else {
+          const float w = __expf(ev - m);
+          S += w;
+          Cw = fmaf(w, sl, Cw);
+          D = fmaf(w * sl, pd, D);
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);
+  const float inv_s = S > 0.f ? 1.f / S : 0.f;
+  if (live && lg == 0) {
+    a.del[r] = (D - ci * Cw) * inv_s;
+    *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(eli, m, inv_s, ci);
+  }
+}
+
+template <int LPG, int NJ, int U>
+__device__ __forceinline__ void gat_b_group_row(const GatBwdArgs& a, int64_t t0, int lane) {
+  const int lg = lane % LPG;
+  const bool live = t0 < a.n_rows;
+  const int32_t r = live ? a.order[t0] : 0;
+  const int64_t b = live ? a.row_ptr[r] : 0, t = live ? a.row_ptr[r + 1] : 0;
+  const float erj = live ? a.er[r] : 0.f;
+  float zr[NJ][4], acc[NJ][4];
+  gb_load_row<LPG, NJ>(a.Z + (int64_t)r * a.ldz, lg, live ? a.K : 0, zr);
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc[j][k] = 0.f;
+  float dpart = 0.f, dcorr = 0.f;
+  for (int64_t e = b; e < t; e += U) {
+    int32_t i[U];
+    float4 st[U];
+    float xv[U][NJ][4];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      i[u] = __ldg(a.col_idx + (e + u < t ? e + u : t - 1));
+      st[u] = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)i[u] * a.ldx + a.rec));
+      gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const float z = st[u].x + erj;
+      const float alpha = (e + u < t) ? __expf(gb_lrelu(z) - st[u].y) * st[u].z : 0.f;
+      const float as = alpha * (z > 0.f ? 1.f : 0.2f);
+      dpart = fmaf(as, gb_pdot<NJ>(xv[u], zr), dpart);
+      if (lg == 0) dcorr = fmaf(as, st[u].w, dcorr);
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(alpha, xv[u][j][k], acc[j][k]);
+    }
+  }
+#pragma unroll
+  for (int o = LPG / 2; o; o >>= 1) {
+    dpart += __shfl_xor_sync(0xffffffffu, dpart, o);
+    dcorr += __shfl_xor_sync(0xffffffffu, dcorr, o);
+  }
+  if (!live) return;
+  const float der = dpart - dcorr;
+  const float delj = a.del_in[r];
+  float* o = a.out + (int64_t)r * a.ldo;
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    const int64_t col = 4 * (int64_t)(lg + j * LPG);
+    if (col >= a.K) continue;
+    float v[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int64_t cc = col + k < a.K ? col + k : col;
+      v[k] = acc[j][k] + delj * __ldg(a.u + cc) + der * __ldg(a.v + cc);
+    }
+    if (a.vec_store && col + 3 < a.K) {
+      *reinterpret_cast<float4*>(o + col) = make_float4(v[0], v[1], v[2], v[3]);
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (col + k < a.K) o[col + k] = v[k];
+    }
+  }
+  if (lg == 0) a.der[r] = der;
+}
+
+// One launch covers both schedules: warps [0, n_wide) take the wide rows order[0 .. n_wide)
+// (all rows of a dense graph), the remaining warps take G rows each, one per lane group.
+template <int LPG, int NJ, int U>
+__global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_a(GatBwdArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w < a.n_wide) gat_a_warp_row<LPG, NJ, U>(a, a.order[w], lane);
+  else gat_a_group_row<LPG, NJ, U>(a, a.n_wide + (w - a.n_wide) * G + lane / LPG, lane);
+}
+
+template <int LPG, int NJ, int U>
+__global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bwd_b(GatBwdArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (w < a.n_wide) gat_b_warp_row<LPG, NJ, U>(a, a.order[w], lane);
+  else gat_b_group_row<LPG, NJ, U>(a, a.n_wide + (w - a.n_wide) * G + lane / LPG, lane);
+}
+
 template <int LPG, int NJ, int U>
 static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
-  const unsigned blocks = (unsigned)ceil_div(a.n_rows, 8);
+  constexpr int G = 32 / LPG;
+  const int64_t warps = a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
+  const unsigned blocks = (unsigned)std::max<int64_t>(1, ceil_div(warps, 8));
   if (pass == 0)
     k_gat_bwd_a<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
   else
@@ -284,14 +422,18 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1);
   // lane-group width: 8 lanes x NJ float4 up to K = 128 (4 groups, more rows in flight),
   // full-warp groups beyond
-  if (K <= 16) gb_launch<4, 1, 4>(pass, a, st);
-  else if (K <= 32) gb_launch<8, 1, 4>(pass, a, st);
-  else if (K <= 64) gb_launch<8, 2, 2>(pass, a, st);
-  else if (K <= 128) gb_launch<8, 4, 2>(pass, a, st);
-  else if (K <= 256) gb_launch<32, 2, 4>(pass, a, st);
-  else if (K <= 512) gb_launch<32, 4, 2>(pass, a, st);
-  else if (K <= 1024) gb_launch<32, 8, 1>(pass, a, st);
-  else gb_launch<32, 16, 1>(pass, a, st);
+  // dense graphs (avg degree >= 16): a warp per row; sparse: a lane group per row, the wide
+  // rows (degree > g->wide_deg) a warp each
+  GatBwdArgs b = a;
+  b.n_wide = g->avg_deg() >= 16.f ? a.n_rows : std::min<int64_t>(g->n_wide, a.n_rows);
+  if (K <= 16) gb_launch<4, 1, 4>(pass, b, st);
+  else if (K <= 32) gb_launch<8, 1, 4>(pass, b, st);
+  else if (K <= 64) gb_launch<8, 2, 2>(pass, b, st);
+  else if (K <= 128) gb_launch<8, 4, 2>(pass, b, st);
+  else if (K <= 256) gb_launch<16, 4, 2>(pass, b, st);
+  else if (K <= 512) gb_launch<32, 4, 2>(pass, b, st);
+  else if (K <= 1024) gb_launch<32, 8, 1>(pass, b, st);
+  else gb_launch<32, 16, 1>(pass, b, st);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

@@ -92,6 +92,9 @@ struct granii_graph_s {
   int64_t* seg_hi = nullptr;
   int32_t* seg_heavy = nullptr;   // device, n_seg: heavy index h of each segment
   int32_t* seg_row = nullptr;     // device, n_seg: row of each segment (= order[seg_heavy])
+  // rows with more than wide_deg entries = order[0 .. n_wide): the sparse (group-per-row)
+  // schedules give them a whole warp
+  int64_t wide_deg = 32, n_wide = 0;
   int64_t features[GRANII_NUM_FEATURES] = {0};
   int device = 0;
   float avg_deg() const { return n_rows > 0 ? float(local_nnz) / float(n_rows) : 0.f; }
@@ -148,6 +151,7 @@ struct GatBwdArgs {
   float* out = nullptr;       // pass 1 out (own rows x K, ld ldo)
   int64_t ldo = 0;
   int vec_store = 0;
+  int64_t n_wide = 0;         // order[0 .. n_wide): a warp per row; the rest: a lane group per row
 };
 granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
                               bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st);

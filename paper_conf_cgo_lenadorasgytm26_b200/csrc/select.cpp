@@ -42,7 +42,7 @@ struct CostModel {
 //   gemm_att        : [1, HBM GB, TFLOP, thousands of tiles, attention GEMV GB (M x K2 x 4)]
 //   gemm_tn         : [1, HBM GB, TFLOP, thousands of tiles]
 //   gat_bwd_a/b     : [1, streamed GB (idx, er / row records), row GB, gathered GB from L2,
-//                      gathered GB from HBM, M rows]  (GAT backward passes, gat_bwd.cu)
+//                      gathered GB from HBM, M rows, M dependent gather steps]  (gat_bwd.cu)
 //   elementwise     : [1, GB]
 //   allgather       : [1, GB received per GPU]
 static CostModel defaults() {
@@ -53,8 +53,8 @@ static CostModel defaults() {
   m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0};
   m.coef["gemm_att"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 1.0 / 3.0};
   m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
-  m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0};
-  m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0};
+  m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
+  m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["elementwise"] = {0.004, 1.0 / 5.5};
   m.coef["allgather"] = {0.020, 1.0 / 700.0};
   return m;
@@ -157,7 +157,10 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
     case P_GAT_BWD_A: case P_GAT_BWD_B: {
       const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
       const double idx = in.nnz * (p == P_GAT_BWD_A ? 8.0 : 20.0) * gb;
-      return {1.0, idx, in.R * K * (p == P_GAT_BWD_A ? 4.0 : 12.0) * gb, gath * h, gath * (1.0 - h), in.R * 1e-6};
+      // dependent gather steps per warp (gat_bwd.cu: G lane groups x U entries per step)
+      const double gu = K <= 16 ? 32 : K <= 32 ? 16 : K <= 128 ? 8 : K <= 256 ? 4 : K <= 512 ? 2 : 1;
+      return {1.0, idx, in.R * K * (p == P_GAT_BWD_A ? 4.0 : 12.0) * gb, gath * h, gath * (1.0 - h), in.R * 1e-6,
+              (in.nnz / gu + 0.5 * in.R) * 1e-6};
     }
     case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
     case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};

@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """Selector regret over every BASELINE config graph plus the paper's Table II extremes
-(SURVEY §8(d) R1 belgium_osm-like road graph, R2 mycielskian17-like dense graph).
+(SURVEY §8(d) R1 belgium_osm-like road graph, R2 mycielskian17-like dense graph), for
+GCN and GAT and the N3 models (SGC, TAGCN with k = 2 hops, GIN with Kh = K2).
 
 For each (graph, K1, K2) every candidate composition of a single layer is timed
 (forward; CUDA events, best of 3 x 5 repetitions) and compared with granii_select's
@@ -23,13 +24,26 @@ from paper_conf_cgo_lenadorasgytm26_b200.model import DEFAULT_CALIB, GNN, LayerS
 DEV = torch.device("cuda:0")
 SWEEP = {
     "cora": ("gcn", [(1433, 16)]),
-    "pubmed": ("gcn", [(32, 32), (32, 256), (256, 32), (256, 256)]),
+    "pubmed": ("gcn+sgc+tagcn+gin", [(32, 32), (32, 256), (256, 32), (256, 256)]),
     "arxiv": ("gat", [(64, 128), (64, 256), (64, 512), (128, 256), (128, 512), (256, 512)]),
-    "reddit": ("gcn", [(602, 32), (602, 256), (602, 1024), (256, 41), (1024, 41), (32, 256)]),
+    "reddit": ("gcn+sgc+tagcn+gin", [(602, 32), (602, 256), (602, 1024), (256, 41), (1024, 41), (32, 256)]),
     "products": ("gcn+gat", [(100, 32), (100, 256), (100, 1024), (256, 47), (32, 256)]),
-    "belgium": ("gcn", [(32, 32), (32, 256), (256, 32), (256, 256), (1024, 32), (32, 1024)]),
+    "belgium": ("gcn+sgc+tagcn", [(32, 32), (32, 256), (256, 32), (256, 256), (1024, 32), (32, 1024)]),
     "mycielskian": ("gcn", [(32, 32), (32, 256), (256, 32), (256, 256), (1024, 32), (32, 1024)]),
 }
+MODELS = {"gcn": 0, "gat": 1, "sgc": 2, "tagcn": 3, "gin": 4}
+
+
+def spec_for(G, LayerSpec, model, k1, k2, comp=None):
+    """one layer of each model; SGC / TAGCN with k = 2 hops, GIN with hidden width Kh = k2 (K2 = k2)"""
+    W = synth.glorot(2, 0, k1, k2, (k1, k2), device=DEV).contiguous()
+    if model == G.TAGCN:
+        W = synth.glorot(2, 0, k1, k2, (3, k1, k2), device=DEV).contiguous()
+    al = synth.uniform_pm1(3, 0, (k2,), device=DEV)
+    ar = synth.uniform_pm1(3, 1, (k2,), device=DEV)
+    W2 = synth.glorot(2, 1, k2, k2, (k2, k2), device=DEV).contiguous() if model == G.GIN else None
+    return LayerSpec(model, k1, k2, G.ACT_RELU, comp=comp, W=W, a_l=al, a_r=ar, hops=2, eps=0.1,
+                     Kh=k2 if model == G.GIN else 0, W2=W2)
 
 
 def timeit(fn, reps=5, trials=3):
@@ -57,28 +71,30 @@ def main():
         g = G.granii_graph_csr_create(w.n, s, d, G.ADD_SELF_LOOPS | (G.SYMMETRIZE if w.symmetrize else 0))
         print(f"[{name}] n={w.n} nnz={g.nnz}", flush=True)
         for mname in models.split("+"):
-            model = G.GCN if mname == "gcn" else G.GAT
-            comps = G.GCN_COMPS if model == G.GCN else G.GAT_COMPS
+            model = MODELS[mname]
+            comps = G.COMPS[model]
             for (k1, k2) in pairs:
                 if model == G.GAT and k1 >= k2:
                     continue   # L330: GAT evaluated for increasing sizes only
                 H = alloc2d(w.n, k1, DEV)
                 H.copy_(synth.features(1, w.n, k1, device=DEV))
-                W = synth.glorot(2, 0, k1, k2, (k1, k2), device=DEV).contiguous()
-                al = synth.uniform_pm1(3, 0, (k2,), device=DEV)
-                ar = synth.uniform_pm1(3, 1, (k2,), device=DEV)
                 times = {}
                 for c in comps:
-                    net = GNN(g, [LayerSpec(model, k1, k2, G.ACT_RELU, comp=c, W=W, a_l=al, a_r=ar)], DEV)
+                    net = GNN(g, [spec_for(G, LayerSpec, model, k1, k2, c)], DEV)
                     times[G.COMP_NAMES[c]] = timeit(lambda: net.forward(H))
                     del net
-                sel, pred = G.granii_select(g, model, k1, k2, calib)
-                sel_np, _ = G.granii_select(g, model, k1, k2, calib, G.SELECT_NO_PREFILTER)
+                shape = G.shape_args(k1, k2, hops=2, Kh=k2 if model == G.GIN else 0)
+                sel, pred = G.granii_select_ex(g, model, shape, calib)
+                sel_np, _ = G.granii_select_ex(g, model, shape, calib, G.SELECT_NO_PREFILTER)
                 best = min(times, key=times.get)
-                if model == G.GCN:
-                    cfg, static = ("GCN_DYN_UPD" if k1 > k2 else "GCN_DYN_AGG"), "GCN_DYN_AGG"
-                else:
+                # Config heuristic (L305 / Table VI): update first iff K1 > K2 with DGL's dynamic
+                # normalisation (L355); static = the framework default: aggregate first, dynamic
+                # (DGL's GraphConv / SGConv / TAGConv / GINConv, L353), GAT reuse (L357)
+                pre = mname.upper()
+                if model == G.GAT:
                     cfg, static = ("GAT_RECOMP" if k1 < k2 else "GAT_REUSE"), "GAT_REUSE"
+                else:
+                    cfg, static = (f"{pre}_DYN_UPD" if k1 > k2 else f"{pre}_DYN_AGG"), f"{pre}_DYN_AGG"
                 row = {"graph": name, "model": mname, "K1": k1, "K2": k2, "ms": times, "best": best,
                        "selected": G.COMP_NAMES[sel], "regret": times[G.COMP_NAMES[sel]] / times[best] - 1,
                        "regret_no_prefilter": times[G.COMP_NAMES[sel_np]] / times[best] - 1,
@@ -95,7 +111,14 @@ def main():
                       "within_10pct": sum(x <= 0.10 for x in rg),
                       "max_config_regret": max(r["config_regret"] for r in out["rows"]),
                       "max_static_regret": max(r["static_regret"] for r in out["rows"])}
+    out["summary_by_model"] = {}
+    for mname in MODELS:
+        rr = [r["regret"] for r in out["rows"] if r["model"] == mname]
+        if rr:
+            out["summary_by_model"][mname] = {"n": len(rr), "max_regret": max(rr), "mean_regret": sum(rr) / len(rr),
+                                              "within_10pct": sum(x <= 0.10 for x in rr)}
     print(json.dumps(out["summary"]))
+    print(json.dumps(out["summary_by_model"]))
     path = sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/regret_sweep.json"
     json.dump(out, open(path, "w"), indent=1)
 
