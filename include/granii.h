@@ -323,6 +323,15 @@ granii_status granii_cost_features(granii_graph g, int32_t prim, int64_t K1, int
 /* Write a 128-byte NCCL unique id (rank 0); ranks exchange it out of band. */
 granii_status granii_comm_unique_id(void* h_id128);
 granii_status granii_comm_create(const void* h_id128, int32_t rank, int32_t world, granii_comm* out);
+/* In-process loopback group: writes `world` handles (ranks 0..world-1) to out[].
+ * Each rank is driven by its own host thread on its own stream of ONE device;
+ * every collective call blocks its thread until all ranks have entered it
+ * (host barrier), then moves data with stream-ordered device copies, ordered
+ * across the ranks' streams by events.  All-reduce sums in rank order, so every
+ * rank gets bitwise the same result.  Purpose: run and test the partitioned
+ * path on a single GPU; it has no NVLink transport.
+ * Errors: INVALID_ARG for world outside [1, 16].  Destroy each handle. */
+granii_status granii_comm_create_local(int32_t world, granii_comm* out);
 granii_status granii_comm_destroy(granii_comm c);
 
 /* ------------------------------------------------------------------------ */

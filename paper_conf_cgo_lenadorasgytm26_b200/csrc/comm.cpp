@@ -3,10 +3,19 @@
 // all-reduce of dW).  NCCL is resolved at run time with dlopen (the copy
 // PyTorch already loaded is reused via RTLD_NOLOAD), so the library loads on
 // machines without NCCL and only granii_comm_* need it.
+//
+// A second transport, the in-process loopback group (granii_comm_create_local),
+// runs G ranks as threads of one process on one device: the collectives are
+// two host barriers plus stream-ordered device copies (cross-stream ordering by
+// events).  It exists so the partitioned data path -- gather-layout column ids,
+// padded all-gather buffers, dW all-reduce, the overlapped local/remote SpMM --
+// runs and is parity-tested on a single GPU.
 #include <dlfcn.h>
 
+#include <condition_variable>
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "internal.h"
 
@@ -87,15 +96,121 @@ granii_status comm_create(const void* id, int32_t rank, int32_t world, granii_co
   return GRANII_OK;
 }
 
+// ------------------------------------------------------------------ loopback group
+struct LoopGroup {
+  int world;
+  std::mutex m;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  int refs;
+  std::vector<const float*> src;
+  std::vector<cudaEvent_t> ready, done;
+  std::vector<float*> stage;
+  std::vector<size_t> stage_cap;
+  explicit LoopGroup(int w) : world(w), refs(w), src(w), ready(w), done(w), stage(w, nullptr), stage_cap(w, 0) {
+    for (int r = 0; r < w; ++r) {
+      cudaEventCreateWithFlags(&ready[r], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&done[r], cudaEventDisableTiming);
+    }
+  }
+  ~LoopGroup() {
+    for (int r = 0; r < world; ++r) {
+      cudaEventDestroy(ready[r]);
+      cudaEventDestroy(done[r]);
+      if (stage[r]) cudaFree(stage[r]);
+    }
+  }
+  void barrier() {
+    std::unique_lock<std::mutex> lk(m);
+    const uint64_t g = gen;
+    if (++arrived == world) {
+      arrived = 0;
+      ++gen;
+      cv.notify_all();
+    } else {
+      cv.wait(lk, [&] { return gen != g; });
+    }
+  }
+  // every peer's copy out of this rank's buffers is ordered before this rank's later work
+  granii_status finish(int rank, cudaStream_t st) {
+    GR_CUDA(cudaEventRecord(done[rank], st));
+    barrier();
+    for (int p = 0; p < world; ++p)
+      if (p != rank) GR_CUDA(cudaStreamWaitEvent(st, done[p], 0));
+    return GRANII_OK;
+  }
+};
+
+granii_status comm_create_local(int32_t world, granii_comm_s** out) {
+  auto* grp = new LoopGroup(world);
+  for (int r = 0; r < world; ++r) {
+    auto* cm = new granii_comm_s();
+    cm->loop = grp;
+    cm->rank = r;
+    cm->world = world;
+    out[r] = cm;
+  }
+  return GRANII_OK;
+}
+
 granii_status comm_destroy(granii_comm_s* c) {
   if (!c) return GRANII_OK;
+  if (c->loop) {
+    auto* grp = (LoopGroup*)c->loop;
+    bool last;
+    {
+      std::lock_guard<std::mutex> lk(grp->m);
+      last = --grp->refs == 0;
+    }
+    if (last) delete grp;
+    delete c;
+    return GRANII_OK;
+  }
   Nccl* n = nccl();
   if (n && c->nccl) n->destroy((nccl_comm)c->nccl);
   delete c;
   return GRANII_OK;
 }
 
+// recv[p*count ..] = peer p's send (p's slot when in place); collective over the group
+static granii_status loop_allgather(granii_comm_s* c, const float* send, float* recv, size_t count,
+                                    cudaStream_t st) {
+  auto* grp = (LoopGroup*)c->loop;
+  const int r = c->rank;
+  GR_CUDA(cudaEventRecord(grp->ready[r], st));
+  grp->src[r] = send;
+  grp->barrier();
+  for (int p = 0; p < grp->world; ++p) {
+    float* dst = recv + (size_t)p * count;
+    if (p != r) GR_CUDA(cudaStreamWaitEvent(st, grp->ready[p], 0));
+    if (grp->src[p] != dst && count)
+      GR_CUDA(cudaMemcpyAsync(dst, grp->src[p], count * sizeof(float), cudaMemcpyDeviceToDevice, st));
+  }
+  return grp->finish(r, st);
+}
+
+// buf = sum over ranks in rank order (bitwise identical on every rank)
+static granii_status loop_allreduce(granii_comm_s* c, float* buf, size_t count, cudaStream_t st) {
+  auto* grp = (LoopGroup*)c->loop;
+  const int r = c->rank;
+  if (grp->stage_cap[r] < count) {
+    GR_CUDA(cudaStreamSynchronize(st));
+    if (grp->stage[r]) GR_CUDA(cudaFree(grp->stage[r]));
+    GR_CUDA(cudaMalloc(&grp->stage[r], count * sizeof(float)));
+    grp->stage_cap[r] = count;
+  }
+  if (count) GR_CUDA(cudaMemcpyAsync(grp->stage[r], buf, count * sizeof(float), cudaMemcpyDeviceToDevice, st));
+  GR_CUDA(cudaEventRecord(grp->ready[r], st));
+  grp->barrier();
+  for (int p = 0; p < grp->world; ++p)
+    if (p != r) GR_CUDA(cudaStreamWaitEvent(st, grp->ready[p], 0));
+  GR_TRY(launch_rank_sum(grp->world, (const float* const*)grp->stage.data(), count, buf, st));
+  return grp->finish(r, st);
+}
+
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st) {
+  if (c && c->loop) return loop_allgather(c, send, recv, count, st);
   Nccl* n = nccl();
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
   int rc = n->allgather(send, recv, count, kFloat32, (nccl_comm)c->nccl, st);
@@ -104,6 +219,7 @@ granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, s
 }
 
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st) {
+  if (c && c->loop) return loop_allreduce(c, buf, count, st);
   Nccl* n = nccl();
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
   int rc = n->allreduce(buf, buf, count, kFloat32, kSum, (nccl_comm)c->nccl, st);

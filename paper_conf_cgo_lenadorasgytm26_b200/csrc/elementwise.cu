@@ -98,6 +98,28 @@ granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_
   return GRANII_OK;
 }
 
+struct RankPtrs {
+  const float* p[16];
+};
+__global__ void k_rank_sum(int n, RankPtrs src, size_t count, float* __restrict__ out) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < count; i += (size_t)gridDim.x * blockDim.x) {
+    float s = src.p[0][i];
+    for (int q = 1; q < n; ++q) s += src.p[q][i];
+    out[i] = s;
+  }
+}
+
+granii_status launch_rank_sum(int n, const float* const* src, size_t count, float* out, cudaStream_t st) {
+  if (n < 1 || n > 16) return fail(GRANII_ERR_UNSUPPORTED, "loopback group larger than 16 ranks");
+  if (count == 0) return GRANII_OK;
+  RankPtrs rp{};
+  for (int q = 0; q < n; ++q) rp.p[q] = src[q];
+  ProfScope ps("elementwise", st, 4.0 * (n + 1) * count, 0.0, 1);
+  k_rank_sum<<<blocks_for((int64_t)count), 256, 0, st>>>(n, rp, count, out);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
 granii_status launch_softmax_xent(int64_t rows, int64_t C, const float* Z, int64_t ldz, const int32_t* y,
                                   int64_t n_total, float* dZ, int64_t lddz, float* loss, cudaStream_t st) {
   if (rows == 0) return GRANII_OK;

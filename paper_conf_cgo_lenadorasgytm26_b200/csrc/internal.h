@@ -102,6 +102,7 @@ struct granii_graph_s {
 
 struct granii_comm_s {
   void* nccl = nullptr;  // ncclComm_t
+  void* loop = nullptr;  // in-process loopback group (comm.cpp), shared by its G handles
   int32_t rank = 0, world = 1;
 };
 
@@ -168,4 +169,7 @@ granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p
 // comm
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);
+granii_status comm_create_local(int32_t world, granii_comm_s** out);
+// out[i] = sum_{p < n} src[p][i] in rank order (loopback all-reduce)
+granii_status launch_rank_sum(int n, const float* const* src, size_t count, float* out, cudaStream_t st);
 }  // namespace granii

@@ -101,6 +101,7 @@ _SIGS = {
     "granii_comm_unique_id": ([_p], ctypes.c_int),
     "granii_comm_create": ([_p, _i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_comm_destroy": ([_p], ctypes.c_int),
+    "granii_comm_create_local": ([_i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
     "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
     "granii_profile_enable": ([_i32], ctypes.c_int),
@@ -358,6 +359,14 @@ def granii_comm_create(uid: bytes, rank: int, world: int) -> Comm:
     h = _p()
     _check(_lib.granii_comm_create(buf, rank, world, ctypes.byref(h)), "granii_comm_create")
     return Comm(h.value, rank, world)
+
+
+def granii_comm_create_local(world: int) -> list:
+    """In-process loopback group: one Comm per rank, each to be driven by its own
+    thread (ctypes releases the GIL during the call) on its own stream of one GPU."""
+    hs = (_p * world)()
+    _check(_lib.granii_comm_create_local(world, hs), "granii_comm_create_local")
+    return [Comm(hs[r], r, world) for r in range(world)]
 
 
 # ---------------------------------------------------------------- training helpers

@@ -1,0 +1,204 @@
+"""The row-partitioned path run on ONE GPU (-m gpu).
+
+G ranks are host threads of this process, each on its own CUDA stream, joined by
+the library's in-process loopback communicator (granii_comm_create_local): the
+collectives are host barriers plus stream-ordered device copies, so every
+device-side piece of the multi-GPU path runs here exactly as under NCCL -- the
+nnz-balanced partition, gather-layout column ids, dinv of the gather layout,
+producers writing into their slot of the padded all-gather buffer, the layer
+compositions on owned rows, and the dW / da all-reduce.  The concatenation of the
+ranks' owned rows must match the single-process fp64 oracle within the same
+tolerances as the unpartitioned path (test_gpu_parity.py, R19 / R22).
+"""
+import threading
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+from paper_conf_cgo_lenadorasgytm26_b200 import synth
+from test_gpu_parity import TOL, err, err_act, gat_grad_ok
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda:0") if torch.cuda.is_available() else None
+F = O.ADD_SELF_LOOPS | O.SYMMETRIZE
+
+
+@pytest.fixture(scope="module")
+def G():
+    from paper_conf_cgo_lenadorasgytm26_b200 import granii
+    return granii
+
+
+def graph_case(name):
+    if name == "sparse":
+        n = 2000
+        s, d = synth.chung_lu(n, 5000, 2.5, seed=21)
+    elif name == "dense":
+        n = 1500
+        s, d = synth.chung_lu(n, 60000, 2.1, seed=22, max_w_frac=0.05)
+    else:
+        n = 45
+        s, d = synth.random_small(n, 120, 23)
+    return n, s, d
+
+
+def run_ranks(G, world, n, s, d, body):
+    """create the G partitioned graphs, then run body(rank, graph, comm, rows) on G threads;
+    returns the per-rank results in rank order"""
+    sd, dd = s.to(DEV).contiguous(), d.to(DEV).contiguous()
+    graphs = [G.granii_graph_csr_create(n, sd, dd, F, r, world) for r in range(world)]
+    comms = G.granii_comm_create_local(world)
+    res, errs = [None] * world, []
+
+    def worker(r):
+        try:
+            torch.cuda.set_device(DEV)
+            st = torch.cuda.Stream(DEV)
+            with torch.cuda.stream(st):
+                info = graphs[r].info
+                res[r] = body(r, graphs[r], comms[r], (info.row_begin, info.row_end))
+                st.synchronize()
+        except BaseException as e:  # noqa: BLE001 -- re-raised in the main thread
+            errs.append(e)
+
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not any(t.is_alive() for t in th), "rank thread hung (collective mismatch)"
+    if errs:
+        raise errs[0]
+    torch.cuda.synchronize()
+    return res, graphs
+
+
+def padded(x):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import alloc2d
+    x = torch.as_tensor(x, dtype=torch.float32)
+    out = alloc2d(x.shape[0], x.shape[1], DEV)
+    out.copy_(x)
+    return out
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("name", ["sparse", "dense", "tiny"])
+def test_partitioned_csr_concatenates_to_global(G, world, name):
+    """O2: bounds bit-exact vs the oracle, the ranks' local CSRs concatenate to the global CSR,
+    and every stored column id is the gather-layout image of the global id"""
+    n, s, d = graph_case(name)
+    rp, ci = O.csr_build(n, s, d, F)
+    bounds = O.partition(rp, world)
+    max_rows = int(np.diff(bounds).max())
+    sd, dd = s.to(DEV).contiguous(), d.to(DEV).contiguous()
+    rows, cols = [], []
+    for r in range(world):
+        g = G.granii_graph_csr_create(n, sd, dd, F, r, world)
+        assert (g.info.row_begin, g.info.row_end) == (bounds[r], bounds[r + 1])
+        lrp, lci = G.granii_graph_export_csr(g)
+        _, lay = G.granii_graph_export_local(g)
+        assert np.array_equal(lay, G.granii_gather_layout_host(lci, bounds, world, max_rows))
+        rows.append(lrp[1:] + (rows[-1][-1] if rows else 0))
+        cols.append(lci)
+    assert np.array_equal(np.concatenate([[0]] + rows), rp)
+    assert np.array_equal(np.concatenate(cols), ci)
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("comp", [0, 1, 2, 3])
+@pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 48), ("dense", 64, 24), ("tiny", 3, 5)])
+def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    n, s, d = graph_case(name)
+    rp, ci = O.csr_build(n, s, d, F)
+    H = synth.features(90, n, K1)
+    W = synth.glorot(90, 2, K1, K2, (K1, K2))
+    Gup = synth.uniform_pm1(90, 3, (n, K2))
+
+    def body(r, g, comm, rows):
+        b0, b1 = rows
+        net = GNN(g, [LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=comp, W=W.to(DEV))], DEV, comm=comm)
+        out = net.forward(padded(H[b0:b1]))
+        dH = net.backward(padded(Gup[b0:b1]), need_input_grad=True)
+        return out.cpu(), dH.cpu(), net.dW[0].cpu()
+
+    res, _ = run_ranks(G, world, n, s, d, body)
+    ref, _ = O.gcn_forward(comp, rp, ci, H, W, 1)
+    rdH, rdW = O.gcn_backward(comp, rp, ci, H, W, Gup, 1)
+    assert err(torch.cat([x[0] for x in res]), ref) <= TOL
+    assert err(torch.cat([x[1] for x in res]), rdH) <= TOL
+    for r in range(world):  # dW all-reduced: every rank holds the same (bitwise) full gradient
+        assert err(res[r][2], rdW) <= TOL
+        assert torch.equal(res[r][2], res[0][2])
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 64), ("dense", 48, 16)])
+def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2):
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    n, s, d = graph_case(name)
+    rp, ci = O.csr_build(n, s, d, F)
+    H = synth.features(91, n, K1)
+    W = synth.glorot(91, 2, K1, K2, (K1, K2))
+    al = synth.uniform_pm1(91, 3, (K2,))
+    ar = synth.uniform_pm1(91, 4, (K2,))
+    Gup = synth.uniform_pm1(91, 5, (n, K2))
+
+    def body(r, g, comm, rows):
+        b0, b1 = rows
+        spec = LayerSpec(G.GAT, K1, K2, G.ACT_NONE, comp=comp, W=W.to(DEV), a_l=al.to(DEV), a_r=ar.to(DEV))
+        net = GNN(g, [spec], DEV, comm=comm)
+        out = net.forward(padded(H[b0:b1]))
+        dH = net.backward(padded(Gup[b0:b1]), need_input_grad=True)
+        return out.cpu(), dH.cpu(), net.dW[0].cpu(), net.da[0][0].cpu(), net.da[0][1].cpu()
+
+    res, _ = run_ranks(G, world, n, s, d, body)
+    ref, _ = O.gat_forward(comp, rp, ci, H, W, al, ar, 0)
+    assert err(torch.cat([x[0] for x in res]), ref) <= TOL
+    rg = O.gat_backward(comp, rp, ci, H, W, al, ar, Gup, 0)
+    mag = O.gat_backward_magnitude(comp, rp, ci, H, W, al, ar, Gup, 0)
+    assert gat_grad_ok(torch.cat([x[1] for x in res]), rg[0], mag[0]), "dH"
+    for r in range(world):
+        for i, nm in ((2, "dW"), (3, "da_l"), (4, "da_r")):
+            assert gat_grad_ok(res[r][i], rg[i - 1], mag[i - 1]), (r, nm)
+            assert torch.equal(res[r][i], res[0][i]), (r, nm)
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("model,comp", [("sgc", 32), ("sgc", 35), ("tagcn", 49), ("tagcn", 50), ("gin", 64),
+                                        ("gin", 67)])
+def test_ext_models_partitioned(G, world, model, comp):
+    """N3 forwards: multi-hop chains all-gather between hops"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    n, s, d = graph_case("sparse")
+    rp, ci = O.csr_build(n, s, d, F)
+    K1, K2, hops, Kh = 24, 16, 3, 20
+    H = synth.features(92, n, K1)
+    if model == "sgc":
+        W = synth.glorot(92, 2, K1, K2, (K1, K2))
+        spec = lambda: LayerSpec(G.SGC, K1, K2, 1, comp=comp, W=W.to(DEV), hops=hops)  # noqa: E731
+        ref = O.sgc_forward(comp, rp, ci, H, W, hops, 1)
+        pre = O.sgc_forward(comp, rp, ci, H, W, hops, 0)
+    elif model == "tagcn":
+        Ws = synth.glorot(92, 2, K1, K2, (hops + 1, K1, K2))
+        spec = lambda: LayerSpec(G.TAGCN, K1, K2, 1, comp=comp, W=Ws.to(DEV).contiguous(), hops=hops)  # noqa: E731
+        ref = O.tagcn_forward(comp, rp, ci, H, Ws, 1)
+        pre = O.tagcn_forward(comp, rp, ci, H, Ws, 0)
+    else:
+        W1 = synth.glorot(92, 2, K1, Kh, (K1, Kh))
+        W2 = synth.glorot(92, 3, Kh, K2, (Kh, K2))
+        spec = lambda: LayerSpec(G.GIN, K1, K2, 1, comp=comp, W=W1.to(DEV), eps=0.25, Kh=Kh,  # noqa: E731
+                                 W2=W2.to(DEV))
+        ref = O.gin_forward(comp, rp, ci, H, W1, W2, 0.25, 1)
+        pre = O.gin_forward(comp, rp, ci, H, W1, W2, 0.25, 0)
+
+    def body(r, g, comm, rows):
+        b0, b1 = rows
+        net = GNN(g, [spec()], DEV, comm=comm)
+        return net.forward(padded(H[b0:b1])).cpu()
+
+    res, _ = run_ranks(G, world, n, s, d, body)
+    assert err_act(torch.cat(res), ref, pre) <= TOL
