@@ -28,6 +28,7 @@ typedef int (*fn_get_uid)(nccl_uid*);
 typedef int (*fn_init_rank)(nccl_comm*, int, nccl_uid, int);
 typedef int (*fn_allgather)(const void*, void*, size_t, int, nccl_comm, cudaStream_t);
 typedef int (*fn_allreduce)(const void*, void*, size_t, int, int, nccl_comm, cudaStream_t);
+typedef int (*fn_bcast)(const void*, void*, size_t, int, int, nccl_comm, cudaStream_t);
 typedef int (*fn_destroy)(nccl_comm);
 typedef const char* (*fn_errstr)(int);
 constexpr int kFloat32 = 7;  // ncclFloat32
@@ -39,6 +40,7 @@ struct Nccl {
   fn_init_rank init_rank = nullptr;
   fn_allgather allgather = nullptr;
   fn_allreduce allreduce = nullptr;
+  fn_bcast bcast = nullptr;
   fn_destroy destroy = nullptr;
   fn_errstr errstr = nullptr;
 };
@@ -56,10 +58,11 @@ Nccl* nccl() {
     n.init_rank = (fn_init_rank)dlsym(h, "ncclCommInitRank");
     n.allgather = (fn_allgather)dlsym(h, "ncclAllGather");
     n.allreduce = (fn_allreduce)dlsym(h, "ncclAllReduce");
+    n.bcast = (fn_bcast)dlsym(h, "ncclBroadcast");
     n.destroy = (fn_destroy)dlsym(h, "ncclCommDestroy");
     n.errstr = (fn_errstr)dlsym(h, "ncclGetErrorString");
   });
-  return (n.h && n.get_uid && n.init_rank && n.allgather && n.allreduce && n.destroy) ? &n : nullptr;
+  return (n.h && n.get_uid && n.init_rank && n.allgather && n.allreduce && n.bcast && n.destroy) ? &n : nullptr;
 }
 
 granii_status nccl_fail(Nccl* n, int rc, const char* what) {
@@ -154,8 +157,28 @@ granii_status comm_create_local(int32_t world, granii_comm_s** out) {
   return GRANII_OK;
 }
 
+static void free_side(granii_comm_s* c) {
+  if (c->ev) {
+    for (int i = 0; i <= c->world; ++i) cudaEventDestroy(c->ev[i]);
+    delete[] c->ev;
+  }
+  if (c->side) cudaStreamDestroy(c->side);
+}
+
+granii_status comm_side(granii_comm_s* c, cudaStream_t* side, cudaEvent_t** ev) {
+  if (!c->side) {
+    GR_CUDA(cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+    c->ev = new cudaEvent_t[c->world + 1];
+    for (int i = 0; i <= c->world; ++i) GR_CUDA(cudaEventCreateWithFlags(&c->ev[i], cudaEventDisableTiming));
+  }
+  *side = c->side;
+  *ev = c->ev;
+  return GRANII_OK;
+}
+
 granii_status comm_destroy(granii_comm_s* c) {
   if (!c) return GRANII_OK;
+  free_side(c);
   if (c->loop) {
     auto* grp = (LoopGroup*)c->loop;
     bool last;
@@ -190,6 +213,21 @@ static granii_status loop_allgather(granii_comm_s* c, const float* send, float* 
   return grp->finish(r, st);
 }
 
+// every rank copies block `root` from the root's buffer into its own (same layout)
+static granii_status loop_bcast(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st) {
+  auto* grp = (LoopGroup*)c->loop;
+  const int r = c->rank;
+  float* slot = buf_all + (size_t)root * count;
+  GR_CUDA(cudaEventRecord(grp->ready[r], st));
+  grp->src[r] = slot;
+  grp->barrier();
+  if (r != root && count) {
+    GR_CUDA(cudaStreamWaitEvent(st, grp->ready[root], 0));
+    GR_CUDA(cudaMemcpyAsync(slot, grp->src[root], count * sizeof(float), cudaMemcpyDeviceToDevice, st));
+  }
+  return grp->finish(r, st);
+}
+
 // buf = sum over ranks in rank order (bitwise identical on every rank)
 static granii_status loop_allreduce(granii_comm_s* c, float* buf, size_t count, cudaStream_t st) {
   auto* grp = (LoopGroup*)c->loop;
@@ -215,6 +253,16 @@ granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, s
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
   int rc = n->allgather(send, recv, count, kFloat32, (nccl_comm)c->nccl, st);
   if (rc) return nccl_fail(n, rc, "ncclAllGather");
+  return GRANII_OK;
+}
+
+granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st) {
+  if (c && c->loop) return loop_bcast(c, buf_all, count, root, st);
+  Nccl* n = nccl();
+  if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
+  float* slot = buf_all + (size_t)root * count;
+  int rc = n->bcast(slot, slot, count, kFloat32, root, (nccl_comm)c->nccl, st);
+  if (rc) return nccl_fail(n, rc, "ncclBroadcast");
   return GRANII_OK;
 }
 

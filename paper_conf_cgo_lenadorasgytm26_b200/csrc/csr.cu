@@ -122,6 +122,26 @@ __global__ void k_remap_cols(int64_t n, const int32_t* __restrict__ col, const i
   }
 }
 
+// owner_off[i][p] = offset in row i of its first entry whose gather-layout column lies in
+// block p (columns are sorted and the layout is monotone in the global id, so each owner's
+// entries are one contiguous run); owner_off[i][G] = deg_i
+__global__ void k_owner_offsets(int64_t R, const int64_t* __restrict__ rp, const int32_t* __restrict__ col, int G,
+                                int64_t max_rows, int32_t* __restrict__ off) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < R; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t lo = rp[i], hi = rp[i + 1];
+    for (int p = 0; p <= G; ++p) {
+      const int64_t key = (int64_t)p * max_rows;
+      int64_t a = lo, b = hi;  // lower_bound
+      while (a < b) {
+        const int64_t m = (a + b) >> 1;
+        if ((int64_t)col[m] < key) a = m + 1;
+        else b = m;
+      }
+      off[i * (G + 1) + p] = (int32_t)(a - lo);
+    }
+  }
+}
+
 __global__ void k_gather_layout_dinv(int64_t N, const float* __restrict__ dinv, const int64_t* __restrict__ bounds,
                                      int G, int64_t max_rows, float* __restrict__ out) {
   int64_t total = (int64_t)G * max_rows;
@@ -309,6 +329,11 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
                          cudaMemcpyDeviceToDevice, st));
     k_gather_layout_dinv<<<grid_for(g->n_cols), 256, 0, st>>>(N, dinv_full, d_bounds, world, g->max_rows,
                                                               g->dinv_cols);
+    // per-row owner ranges for the block-phased SpMM (layer.cu gathered_spmm, N1)
+    CK(cudaMalloc(&g->owner_off, std::max<int64_t>(g->n_rows, 1) * (world + 1) * sizeof(int32_t)));
+    if (g->n_rows > 0)
+      k_owner_offsets<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->row_ptr, g->col_idx, world, g->max_rows,
+                                                           g->owner_off);
     CK(cudaFreeAsync(d_bounds, st));
     CK(cudaStreamSynchronize(st));
     cudaFree(rp_full);
@@ -382,6 +407,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
 
 void graph_free(granii_graph_s* g) {
   if (!g) return;
+  cudaFree(g->owner_off);
   if (g->dinv_cols != g->dinv_rows) cudaFree(g->dinv_cols);
   cudaFree(g->dinv_rows);
   cudaFree(g->row_ptr);

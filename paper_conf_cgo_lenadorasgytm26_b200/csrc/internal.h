@@ -83,6 +83,8 @@ struct granii_graph_s {
   float* dinv_rows = nullptr;     // device, n_rows
   float* dinv_cols = nullptr;     // device, n_cols (== dinv_rows when world == 1)
   int32_t* order = nullptr;       // device, n_rows: owned rows by descending degree
+  int32_t* owner_off = nullptr;   // device, n_rows x (world+1) when world > 1: entries of row i whose
+                                  // column is owned by rank p are [rp_i + off[i][p], rp_i + off[i][p+1])
   // heavy rows (degree > seg_len) = order[0 .. n_heavy); each is cut into segments of
   // seg_len entries that are scheduled as independent warp-wide work items
   int64_t seg_len = 2048;
@@ -103,6 +105,8 @@ struct granii_graph_s {
 struct granii_comm_s {
   void* nccl = nullptr;  // ncclComm_t
   void* loop = nullptr;  // in-process loopback group (comm.cpp), shared by its G handles
+  cudaStream_t side = nullptr;             // collectives overlapped with compute (N1)
+  cudaEvent_t* ev = nullptr;               // world + 1 events on `side`
   int32_t rank = 0, world = 1;
 };
 
@@ -114,6 +118,17 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
 granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                              float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                              int64_t ldb, float beta, cudaStream_t st);
+// one phase of a block-phased aggregation over a partitioned graph (layer.cu gathered_spmm):
+// the entries whose column lies in rank `owner`'s gather block; partial = heavy-segment scratch
+// [n_seg][round_up(K,4)] kept across the phases (NULL if the graph has no segments)
+struct SpmmPhase {
+  int owner;
+  int first, last;
+  float* partial;
+};
+granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                                float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                                int64_t ldb, float beta, const SpmmPhase& ph, cudaStream_t st);
 // GIN's precomputed values: vals_e = 1 + eps on the diagonal entry of each row, 1 elsewhere
 granii_status launch_gin_vals(const granii_graph_s* g, float eps, float* vals, cudaStream_t st);
 granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U, int64_t ldu, const float* V,
@@ -170,6 +185,10 @@ granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);
 granii_status comm_create_local(int32_t world, granii_comm_s** out);
+// in-place broadcast of block `root` of a gather buffer (buf_all + root*count) to every rank
+granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st);
+// the communicator's side stream and per-block events (created on first use on the current device)
+granii_status comm_side(granii_comm_s* c, cudaStream_t* side, cudaEvent_t** ev);
 // out[i] = sum_{p < n} src[p][i] in rank order (loopback all-reduce)
 granii_status launch_rank_sum(int n, const float* const* src, size_t count, float* out, cudaStream_t st);
 }  // namespace granii

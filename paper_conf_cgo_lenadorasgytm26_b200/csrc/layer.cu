@@ -78,6 +78,55 @@ static granii_status allgather(const Ctx& c, GatherBuf& gb) {
   return comm_allgather(c.comm, gb.mine, gb.all, count, c.st);
 }
 
+// Aggregation Y = spmm(X) over a dense operand whose own rows are already in gb.mine.
+// One GPU: a plain SpMM.  Several GPUs (N1): instead of all-gather -> SpMM, the blocks are
+// broadcast one source rank at a time on the communicator's side stream, and the SpMM runs in
+// phases on the caller's stream -- this rank's block first (nothing to wait for), then every
+// other block as soon as its broadcast has landed -- so the transfer overlaps the aggregation.
+// Each row's entries owned by one rank are a contiguous run (sorted columns, monotone gather
+// layout: graph owner_off), so a phase is a plain SpMM over sub-ranges that continues from the
+// previous phase's raw partial; the epilogue runs in the last phase.  Phase order is fixed,
+// so results are run-to-run bitwise reproducible.  GRANII_COMM_OVERLAP=0: all-gather, then
+// one SpMM.
+static bool overlap_enabled() {
+  const char* e = getenv("GRANII_COMM_OVERLAP");
+  return !(e && e[0] == '0');
+}
+
+static granii_status gathered_spmm(const Ctx& c, GatherBuf& gb, const float* vals, int64_t K, float* Y, int64_t ldy,
+                                   const float* rs, const float* cs, bool relu, const float* B = nullptr,
+                                   int64_t ldb = 0, float beta = 0.f) {
+  const granii_graph_s* g = c.g;
+  if (!c.dist()) return launch_spmm_ex(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, c.st);
+  if (!overlap_enabled() || !g->owner_off) {
+    GR_TRY(allgather(c, gb));
+    return launch_spmm_ex(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, c.st);
+  }
+  cudaStream_t side;
+  cudaEvent_t* ev;
+  GR_TRY(comm_side(c.comm, &side, &ev));
+  const int G = g->world, me = g->rank;
+  const size_t count = (size_t)g->max_rows * gb.ld;
+  GR_CUDA(cudaEventRecord(ev[G], c.st));  // own block produced
+  GR_CUDA(cudaStreamWaitEvent(side, ev[G], 0));
+  for (int p = 0; p < G; ++p) {  // every rank issues the broadcasts in the same order
+    GR_TRY(comm_bcast_block(c.comm, gb.all, count, p, side));
+    GR_CUDA(cudaEventRecord(ev[p], side));
+  }
+  float* partial = nullptr;
+  if (g->n_seg > 0)
+    GR_CUDA(cudaMallocAsync((void**)&partial, (size_t)g->n_seg * round_up(K, 4) * sizeof(float), c.st));
+  for (int i = 0; i < G; ++i) {
+    const int p = i == 0 ? me : (i <= me ? i - 1 : i);  // own block, then the others ascending
+    if (p != me) GR_CUDA(cudaStreamWaitEvent(c.st, ev[p], 0));
+    SpmmPhase ph{p, i == 0, i == G - 1, partial};
+    GR_TRY(launch_spmm_phase(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, ph, c.st));
+  }
+  GR_CUDA(cudaStreamWaitEvent(c.st, ev[G - 1], 0));  // the side stream is idle (own send included)
+  if (partial) GR_CUDA(cudaFreeAsync(partial, c.st));
+  return GRANII_OK;
+}
+
 // scalar per-row vector (er) gather: one float per row
 static float* vec_buf(Bump& b, const Ctx& c) {
   return b.take((size_t)(c.dist() ? c.g->n_cols : std::max<int64_t>(c.g->n_rows, 1)));
@@ -349,11 +398,8 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
                                              comp == GRANII_GAT_RECOMP);
   GatherBuf hg;
   if (agg_first_gather) {
-    hg = gather_buf(b, c, K1);  // H goes into the gather slot (aligned copy)
-    if (run) {
-      GR_TRY(launch_copy_rows(R, K1, H, ldh, hg.mine, hg.ld, st));
-      GR_TRY(allgather(c, hg));
-    }
+    hg = gather_buf(b, c, K1);  // H goes into the gather slot (aligned copy); gathered by the SpMM
+    if (run) GR_TRY(launch_copy_rows(R, K1, H, ldh, hg.mine, hg.ld, st));
     H = hg.mine;
     ldh = hg.ld;
   } else if (!h_aligned) {
@@ -362,8 +408,8 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     H = hpad;
     ldh = ld4(K1);
   }
-  const float* Xagg = agg_first_gather ? hg.all : H;  // aggregation source (column-id space)
-  const int64_t ldxagg = ldh;
+  // aggregation source (column-id space): the gather buffer, or this GPU's rows
+  GatherBuf xg = agg_first_gather ? hg : GatherBuf{const_cast<float*>(H), const_cast<float*>(H), ldh};
 
   if (m == GRANII_GCN) {
     float* nval = nullptr;
@@ -383,9 +429,9 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
         gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw, &gn);
         if (run) {
           if (comp == GRANII_GCN_PRE_AGG)
-            GR_TRY(launch_spmm(g, nval, Xagg, ldxagg, K1, T, ldt, nullptr, nullptr, false, st));
+            GR_TRY(gathered_spmm(c, xg, nval, K1, T, ldt, nullptr, nullptr, false));
           else
-            GR_TRY(launch_spmm(g, nullptr, Xagg, ldxagg, K1, T, ldt, g->dinv_rows, g->dinv_cols, false, st));
+            GR_TRY(gathered_spmm(c, xg, nullptr, K1, T, ldt, g->dinv_rows, g->dinv_cols, false));
           GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
         }
         break;
@@ -400,11 +446,10 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
           granii_gemm_epilogue ep{comp == GRANII_GCN_DYN_UPD ? g->dinv_rows : nullptr, nullptr, nullptr, nullptr,
                                   nullptr};
           GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, tg.mine, tg.ld, &ep, 0, gw, gn, st));
-          GR_TRY(allgather(c, tg));
           if (comp == GRANII_GCN_PRE_UPD)
-            GR_TRY(launch_spmm(g, nval, tg.all, tg.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+            GR_TRY(gathered_spmm(c, tg, nval, K2, out, ldo, nullptr, nullptr, relu));
           else
-            GR_TRY(launch_spmm(g, nullptr, tg.all, tg.ld, K2, out, ldo, g->dinv_rows, nullptr, relu, st));
+            GR_TRY(gathered_spmm(c, tg, nullptr, K2, out, ldo, g->dinv_rows, nullptr, relu));
         }
         break;
       }
@@ -450,7 +495,7 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
         if (!dot)
           GR_CUDA(cudaMemcpyAsync(saved + sv.er, er_mine, sizeof(float) * (size_t)R, cudaMemcpyDeviceToDevice, st));
       }
-      if (need_theta) GR_TRY(allgather(c, th));
+      if (dot) GR_TRY(allgather(c, th));  // the dot scores gather Θ; the additive REUSE SpMM gathers it itself
       if (!dot) {
         if (c.dist()) {
           GatherBuf eb{er_all, er_mine, 1};
@@ -465,7 +510,10 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       }
     }
     if (comp == GRANII_GAT_REUSE) {
-      if (run) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+      if (run) {
+        if (dot) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+        else GR_TRY(gathered_spmm(c, th, alpha, K2, out, ldo, nullptr, nullptr, relu));
+      }
     } else {
       const int64_t ldt = ld4(K1);
       float* T = saved ? saved : b.take((size_t)std::max<int64_t>(R, 1) * ldt);
@@ -473,7 +521,7 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       size_t gn2;
       gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
       if (run) {
-        GR_TRY(launch_spmm(g, alpha, Xagg, ldxagg, K1, T, ldt, nullptr, nullptr, false, st));
+        GR_TRY(gathered_spmm(c, xg, alpha, K1, T, ldt, nullptr, nullptr, false));
         GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
                            st));
       }
@@ -538,21 +586,19 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
           granii_gemm_epilogue ep{comp == GRANII_GCN_DYN_AGG ? g->dinv_rows : nullptr, nullptr, nullptr, nullptr,
                                   nullptr};
           GR_TRY(launch_gemm(R, K1, K2, dY, lddy, a->W, K2, dtg.mine, dtg.ld, &ep, GRANII_GEMM_TRANS_B, gwH, gnH, st));
-          GR_TRY(allgather(c, dtg));
           if (comp == GRANII_GCN_PRE_AGG)
-            GR_TRY(launch_spmm(g, nval, dtg.all, dtg.ld, K1, dH, lddh, nullptr, nullptr, false, st));
+            GR_TRY(gathered_spmm(c, dtg, nval, K1, dH, lddh, nullptr, nullptr, false));
           else
-            GR_TRY(launch_spmm(g, nullptr, dtg.all, dtg.ld, K1, dH, lddh, g->dinv_rows, nullptr, false, st));
+            GR_TRY(gathered_spmm(c, dtg, nullptr, K1, dH, lddh, g->dinv_rows, nullptr, false));
         }
         break;
       }
       case GRANII_GCN_PRE_UPD:
       case GRANII_GCN_DYN_UPD: {
-        GR_TRY(allgather(c, dyg));
         if (comp == GRANII_GCN_PRE_UPD)
-          GR_TRY(launch_spmm(g, nval, dyg.all, dyg.ld, K2, dT, ldt2, nullptr, nullptr, false, st));
+          GR_TRY(gathered_spmm(c, dyg, nval, K2, dT, ldt2, nullptr, nullptr, false));
         else
-          GR_TRY(launch_spmm(g, nullptr, dyg.all, dyg.ld, K2, dT, ldt2, g->dinv_rows, nullptr, false, st));
+          GR_TRY(gathered_spmm(c, dyg, nullptr, K2, dT, ldt2, g->dinv_rows, nullptr, false));
         GR_TRY(launch_gemm(K1, K2, R, H, ldh, dT, ldt2, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
         if (dH) GR_TRY(launch_gemm(R, K1, K2, dT, ldt2, a->W, K2, dH, lddh, nullptr, GRANII_GEMM_TRANS_B, gwH, gnH, st));
         break;

@@ -76,7 +76,30 @@ struct SpmmArgs {
   const float* __restrict__ B;
   int64_t ldb;
   float beta;
+  // block-phased mode (owner_off != nullptr; layer.cu gathered_spmm, N1): only the entries whose
+  // column lies in rank `owner`'s block of the gather buffer.  `first`: start from zero, else from
+  // the raw partial already in Y (light rows) / partial (segments); `last`: apply the epilogue.
+  const int32_t* __restrict__ owner_off;   // [n_rows][G1]
+  const int32_t* __restrict__ seg_row;     // row of each heavy segment
+  int G1, owner, first, last;
 };
+
+// entry range of `row` restricted to the phase's owner block (whole row outside phased mode)
+__device__ __forceinline__ void phase_range(const SpmmArgs& a, int64_t row, int64_t& lo, int64_t& hi) {
+  if (!a.owner_off) return;
+  const int32_t* o = a.owner_off + row * a.G1 + a.owner;
+  const int64_t base = a.row_ptr[row];
+  lo = max(lo, base + (int64_t)o[0]);
+  hi = min(hi, base + (int64_t)o[1]);
+}
+
+// continue a phased accumulation from the raw partial stored by the previous phase
+template <int LPG, int NJ, int VEC>
+__device__ __forceinline__ void load_partial(const float* y, const bool (&colok)[NJ], float (&acc)[NJ][VEC]) {
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+    if (colok[j]) ldv<VEC>(y + j * LPG * VEC, acc[j]);
+}
 
 // One chunk of 32 entries of a row, one per lane: column id and weight.  Lanes
 // past the range's end reuse its last column with w = 0, so every later step is
@@ -199,9 +222,15 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
                                            uint32_t row_bytes) {
   float acc[NJ][VEC];
   zero(acc);
-  warp_range<VEC, LPG, NJ, W, CS, U>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc);
+  int64_t lo = a.seg_lo[t], hi = a.seg_hi[t];
+  float* part = a.partial + t * a.ldp + (int64_t)lig * VEC;
+  if (a.owner_off) {
+    phase_range(a, a.seg_row[t], lo, hi);
+    if (!a.first && grp == 0) load_partial<LPG>(part, colok, acc);
+  }
+  warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
   reduce_groups<LPG>(acc);
-  if (grp == 0) store_row<LPG>(a.partial + t * a.ldp + (int64_t)lig * VEC, colok, acc, 1.f, 0);
+  if (grp == 0) store_row<LPG>(part, colok, acc, 1.f, 0);
 }
 
 // ------------------------------------------------------------------ warp-per-row
@@ -225,11 +254,20 @@ __global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
     const int64_t row = a.order[t - a.n_seg];
     float acc[NJ][VEC];
     zero(acc);
-    warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
+    int64_t lo = a.row_ptr[row], hi = a.row_ptr[row + 1];
+    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+    if (a.owner_off) {
+      phase_range(a, row, lo, hi);
+      if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
+    }
+    warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
     reduce_groups<LPG>(acc);
-    if (grp == 0)
-      store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
-                     a.relu, a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+    if (grp == 0) {
+      if (a.owner_off && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
+      else
+        store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
+                       a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+    }
   }
 }
 
@@ -253,9 +291,14 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
     const int64_t row = a.order[t];
-    const int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
+    int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
     float acc[NJ][VEC];
     zero(acc);
+    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+    if (a.owner_off) {
+      phase_range(a, row, rs0, re);
+      if (!a.first) load_partial<LPG>(y, colok, acc);
+    }
     for (int64_t e = rs0; e < re; e += U) {
       uint32_t cu[U];
       float wu[U];
@@ -281,8 +324,10 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
 #pragma unroll
           for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
     }
-    store_row<LPG>(a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f,
-                   a.relu, a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+    if (a.owner_off && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
+    else
+      store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
+                     a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
   }
 }
 
@@ -402,9 +447,9 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
   return launch_spmm_ex(g, vals, X, ldx, K, Y, ldy, rs, cs, relu, nullptr, 0, 0.f, st);
 }
 
-granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
-                             float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
-                             int64_t ldb, float beta, cudaStream_t st) {
+static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                               float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                               int64_t ldb, float beta, const SpmmPhase* ph, cudaStream_t st) {
   if (g->n_rows == 0 || K == 0) return GRANII_OK;
   DevInfo di;
   GR_TRY(dev_info(&di));
@@ -414,22 +459,38 @@ granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const f
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
              g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0, B, ldb, beta};
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
-  if (g->n_seg > 0) {  // stream-ordered scratch for the heavy-row partials (pool-backed, no sync)
+  float* partial = nullptr;  // heavy-segment partials: this slice's columns start at partial + pk0
+  bool own_partial = false;
+  if (ph) {
+    a.owner_off = g->owner_off;
+    a.seg_row = g->seg_row;
+    a.G1 = g->world + 1;
+    a.owner = ph->owner;
+    a.first = ph->first;
+    a.last = ph->last;
+    a.ldp = round_up(K, 4);  // kept across the phases for every slice
+    partial = ph->partial;
+  } else if (g->n_seg > 0) {  // stream-ordered scratch for the heavy-row partials (pool-backed, no sync)
     a.ldp = round_up(kw, 4);
-    GR_CUDA(cudaMallocAsync((void**)&a.partial, (size_t)g->n_seg * a.ldp * sizeof(float), st));
+    GR_CUDA(cudaMallocAsync((void**)&partial, (size_t)g->n_seg * a.ldp * sizeof(float), st));
+    own_partial = true;
   }
+  const bool combine = g->n_seg > 0 && (!ph || ph->last);
   // algorithmic bytes: per entry col id (+w, +cs) + one K-row of X;
   // per row row_ptr + the K-row of Y (+rs)
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) +
                        R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0) + (B ? 4.0 * K : 0.0));
-  ProfScope ps("spmm", st, bytes, 2.0 * nnz * K, (int)ceil_div(K, kw));
+  // a phased aggregation books its algorithmic bytes once (in its last phase)
+  const bool book = !ph || ph->last;
+  ProfScope ps("spmm", st, book ? bytes : 0.0, book ? 2.0 * nnz * K : 0.0, (int)ceil_div(K, kw));
   for (int64_t k0 = 0; k0 < K; k0 += kw) {
     a.k0 = k0;
     a.kw = std::min(kw, K - k0);
+    a.partial = partial ? partial + (ph ? k0 : 0) : nullptr;
     // slices of a vec4 launch must stay 16-byte aligned
     GR_TRY(launch_slice(a, vec4 && (k0 % 4 == 0), warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
-    if (g->n_seg > 0) {
+    if (combine) {
       const int64_t tot = g->n_heavy * a.kw;
       k_spmm_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(
           g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0, B, ldb, beta);
@@ -437,8 +498,21 @@ granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const f
       ps.add_launches(1);
     }
   }
-  if (a.partial) GR_CUDA(cudaFreeAsync(a.partial, st));
+  if (own_partial) GR_CUDA(cudaFreeAsync(partial, st));
   return GRANII_OK;
+}
+
+granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                             float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                             int64_t ldb, float beta, cudaStream_t st) {
+  return spmm_impl(g, vals, X, ldx, K, Y, ldy, rs, cs, relu, B, ldb, beta, nullptr, st);
+}
+
+granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
+                                float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
+                                int64_t ldb, float beta, const SpmmPhase& ph, cudaStream_t st) {
+  if (!g->owner_off) return fail(GRANII_ERR_INVALID_ARG, "phased SpMM needs a partitioned graph");
+  return spmm_impl(g, vals, X, ldx, K, Y, ldy, rs, cs, relu, B, ldb, beta, &ph, st);
 }
 
 }  // namespace granii

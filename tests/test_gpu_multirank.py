@@ -6,7 +6,9 @@ collectives are host barriers plus stream-ordered device copies, so every
 device-side piece of the multi-GPU path runs here exactly as under NCCL -- the
 nnz-balanced partition, gather-layout column ids, dinv of the gather layout,
 producers writing into their slot of the padded all-gather buffer, the layer
-compositions on owned rows, and the dW / da all-reduce.  The concatenation of the
+compositions on owned rows, the block-phased SpMM that overlaps the per-block
+broadcasts (N1; GRANII_COMM_OVERLAP=0 falls back to all-gather -> SpMM), and the
+dW / da all-reduce.  The concatenation of the
 ranks' owned rows must match the single-process fp64 oracle within the same
 tolerances as the unpartitioned path (test_gpu_parity.py, R19 / R22).
 """
@@ -106,11 +108,13 @@ def test_partitioned_csr_concatenates_to_global(G, world, name):
     assert np.array_equal(np.concatenate(cols), ci)
 
 
+@pytest.mark.parametrize("overlap", ["1", "0"])
 @pytest.mark.parametrize("world", [2, 3, 4])
 @pytest.mark.parametrize("comp", [0, 1, 2, 3])
 @pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 48), ("dense", 64, 24), ("tiny", 3, 5)])
-def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2):
+def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2, overlap, monkeypatch):
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    monkeypatch.setenv("GRANII_COMM_OVERLAP", overlap)
     n, s, d = graph_case(name)
     rp, ci = O.csr_build(n, s, d, F)
     H = synth.features(90, n, K1)
@@ -165,6 +169,38 @@ def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2):
         for i, nm in ((2, "dW"), (3, "da_l"), (4, "da_r")):
             assert gat_grad_ok(res[r][i], rg[i - 1], mag[i - 1]), (r, nm)
             assert torch.equal(res[r][i], res[0][i]), (r, nm)
+
+
+@pytest.mark.parametrize("world", [3, 8])
+def test_phased_spmm_segments_slices_deterministic(G, world, monkeypatch):
+    """the block-phased aggregation with hub segments (GRANII_SEG=64: partials carried across
+    the phases, combined after the last) and forced K slices; bitwise reproducible"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    n, s, d = graph_case("dense")
+    rp, ci = O.csr_build(n, s, d, F)
+    K1, K2 = 72, 40
+    H = synth.features(94, n, K1)
+    W = synth.glorot(94, 2, K1, K2, (K1, K2))
+    Gup = synth.uniform_pm1(94, 3, (n, K2))
+    monkeypatch.setenv("GRANII_SEG", "64")
+    monkeypatch.setenv("GRANII_SPMM_SLICE", "16")
+    for comp in (0, 1, 2, 3):
+        def body(r, g, comm, rows):
+            b0, b1 = rows
+            outs = []
+            for _ in range(2):
+                net = GNN(g, [LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=comp, W=W.to(DEV))], DEV, comm=comm)
+                out = net.forward(padded(H[b0:b1]))
+                dH = net.backward(padded(Gup[b0:b1]), need_input_grad=True)
+                outs.append((out.cpu(), dH.cpu()))
+            return outs
+        res, _ = run_ranks(G, world, n, s, d, body)
+        ref, _ = O.gcn_forward(comp, rp, ci, H, W, 1)
+        rdH, _ = O.gcn_backward(comp, rp, ci, H, W, Gup, 1)
+        assert err(torch.cat([x[0][0] for x in res]), ref) <= TOL, comp
+        assert err(torch.cat([x[0][1] for x in res]), rdH) <= TOL, comp
+        for x in res:
+            assert torch.equal(x[0][0], x[1][0]) and torch.equal(x[0][1], x[1][1])
 
 
 @pytest.mark.parametrize("world", [2, 3])
