@@ -332,6 +332,15 @@ granii_status granii_comm_create(const void* h_id128, int32_t rank, int32_t worl
  * path on a single GPU; it has no NVLink transport.
  * Errors: INVALID_ARG for world outside [1, 16].  Destroy each handle. */
 granii_status granii_comm_create_local(int32_t world, granii_comm* out);
+/* TIMING STUB, not a transport: a rank-`rank` communicator whose collectives move no
+ * data (they only update the statistics below).  Layer outputs on a partitioned graph
+ * are WRONG with it.  It exists to time one rank's local work of a G-way partition on a
+ * single GPU (tools/scaling_projection.py).  Errors: INVALID_ARG. */
+granii_status granii_comm_create_stub(int32_t rank, int32_t world, granii_comm* out);
+/* Bytes this rank has received over the communicator's lifetime (all-gather: (G-1)
+ * blocks; block broadcast: one block unless root; all-reduce: the ring's 2(G-1)/G of the
+ * buffer) and the number of collective calls.  Host-side counters, any transport. */
+granii_status granii_comm_stats(granii_comm c, uint64_t* bytes_in, uint64_t* calls);
 granii_status granii_comm_destroy(granii_comm c);
 
 /* ------------------------------------------------------------------------ */

@@ -48,6 +48,7 @@ granii_status comm_unique_id(void*);
 granii_status comm_create(const void*, int32_t, int32_t, granii_comm_s**);
 granii_status comm_destroy(granii_comm_s*);
 granii_status comm_create_local(int32_t, granii_comm_s**);
+granii_status comm_create_stub(int32_t, int32_t, granii_comm_s**);
 granii_status launch_softmax_xent(int64_t, int64_t, const float*, int64_t, const int32_t*, int64_t, float*, int64_t,
                                   float*, cudaStream_t);
 granii_status launch_sgd(int64_t, float, const float*, float*, cudaStream_t);
@@ -335,6 +336,16 @@ granii_status granii_comm_create(const void* id, int32_t rank, int32_t world, gr
 granii_status granii_comm_create_local(int32_t world, granii_comm* out) {
   GR_ARG(out && world >= 1 && world <= 16, "bad argument");
   return comm_create_local(world, out);
+}
+granii_status granii_comm_create_stub(int32_t rank, int32_t world, granii_comm* out) {
+  GR_ARG(out && world >= 1 && rank >= 0 && rank < world, "bad argument");
+  return comm_create_stub(rank, world, out);
+}
+granii_status granii_comm_stats(granii_comm c, uint64_t* bytes_in, uint64_t* calls) {
+  GR_ARG(c && bytes_in && calls, "NULL argument");
+  *bytes_in = c->bytes_in;
+  *calls = c->calls;
+  return GRANII_OK;
 }
 granii_status granii_comm_destroy(granii_comm c) { return comm_destroy(c); }
 

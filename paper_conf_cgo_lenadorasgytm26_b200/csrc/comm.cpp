@@ -247,7 +247,21 @@ static granii_status loop_allreduce(granii_comm_s* c, float* buf, size_t count, 
   return grp->finish(r, st);
 }
 
+granii_status comm_create_stub(int32_t rank, int32_t world, granii_comm_s** out) {
+  auto* cm = new granii_comm_s();
+  cm->stub = 1;
+  cm->rank = rank;
+  cm->world = world;
+  *out = cm;
+  return GRANII_OK;
+}
+
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st) {
+  if (c) {
+    c->bytes_in += (uint64_t)count * sizeof(float) * (uint64_t)(c->world - 1);
+    ++c->calls;
+    if (c->stub) return GRANII_OK;
+  }
   if (c && c->loop) return loop_allgather(c, send, recv, count, st);
   Nccl* n = nccl();
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
@@ -257,6 +271,11 @@ granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, s
 }
 
 granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st) {
+  if (c) {
+    if (root != c->rank) c->bytes_in += (uint64_t)count * sizeof(float);
+    ++c->calls;
+    if (c->stub) return GRANII_OK;
+  }
   if (c && c->loop) return loop_bcast(c, buf_all, count, root, st);
   Nccl* n = nccl();
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");
@@ -267,6 +286,11 @@ granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, i
 }
 
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st) {
+  if (c) {  // ring all-reduce: 2 (G-1)/G of the buffer in, per rank
+    c->bytes_in += (uint64_t)(2.0 * count * sizeof(float) * (c->world - 1) / c->world);
+    ++c->calls;
+    if (c->stub) return GRANII_OK;
+  }
   if (c && c->loop) return loop_allreduce(c, buf, count, st);
   Nccl* n = nccl();
   if (!n || !c || !c->nccl) return fail(GRANII_ERR_NCCL, "communicator not initialised");

@@ -180,6 +180,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   auto g = new granii_graph_s();
   g->N = N;
   g->rank = rank;
+  if (const char* e = getenv("GRANII_SEG")) g->seg_len = std::max<int64_t>(64, atoll(e));
   g->world = world;
   g->symmetric = sym;
   g->self_loops = loops;
@@ -313,6 +314,10 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
     g->n_rows = g->row_end - g->row_begin;
     g->local_nnz = hrp[g->row_end] - hrp[g->row_begin];
     g->n_cols = (int64_t)world * g->max_rows;
+    for (int64_t i = 0; i < N; ++i) {  // hub segments of the whole graph (rank-independent selection)
+      const int64_t d = hrp[i + 1] - hrp[i];
+      if (d > g->seg_len) g->n_seg_global += ceil_div(d, g->seg_len);
+    }
     int64_t* d_bounds = nullptr;
     CK(cudaMallocAsync(&d_bounds, (world + 1) * sizeof(int64_t), st));
     CK(cudaMemcpyAsync(d_bounds, g->bounds.data(), (world + 1) * sizeof(int64_t), cudaMemcpyHostToDevice, st));
@@ -354,7 +359,6 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
 
   // heavy-row segments (power-law hubs): rows with more than seg_len entries are cut
   // into seg_len-entry warp-wide work items so a hub cannot set the kernel's tail
-  if (const char* e = getenv("GRANII_SEG")) g->seg_len = std::max<int64_t>(64, atoll(e));
   if (g->n_rows > 0 && g->features[4] > g->seg_len) {
     std::vector<int64_t> hrp(g->n_rows + 1);
     CK(cudaMemcpy(hrp.data(), g->row_ptr, (g->n_rows + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));

@@ -89,6 +89,7 @@ struct granii_graph_s {
   // seg_len entries that are scheduled as independent warp-wide work items
   int64_t seg_len = 2048;
   int64_t n_heavy = 0, n_seg = 0;
+  int64_t n_seg_global = -1;      // hub segments of the whole graph (partitioned graphs; -1: = n_seg)
   int32_t* seg_ptr = nullptr;     // device, n_heavy+1: segments of heavy row h are [seg_ptr[h], seg_ptr[h+1])
   int64_t* seg_lo = nullptr;      // device, n_seg: entry range of each segment
   int64_t* seg_hi = nullptr;
@@ -105,6 +106,8 @@ struct granii_graph_s {
 struct granii_comm_s {
   void* nccl = nullptr;  // ncclComm_t
   void* loop = nullptr;  // in-process loopback group (comm.cpp), shared by its G handles
+  int stub = 0;          // timing stub: collectives move no data (granii_comm_create_stub)
+  uint64_t bytes_in = 0, calls = 0;        // bytes this rank received / collective calls (stats)
   cudaStream_t side = nullptr;             // collectives overlapped with compute (N1)
   cudaEvent_t* ev = nullptr;               // world + 1 events on `side`
   int32_t rank = 0, world = 1;
@@ -185,6 +188,7 @@ granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);
 granii_status comm_create_local(int32_t world, granii_comm_s** out);
+granii_status comm_create_stub(int32_t rank, int32_t world, granii_comm_s** out);
 // in-place broadcast of block `root` of a gather buffer (buf_all + root*count) to every rank
 granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st);
 // the communicator's side stream and per-block events (created on first use on the current device)

@@ -17,7 +17,9 @@
 // Extension (not in the paper, which selects on the forward only, L340):
 // GRANII_SELECT_TRAINING adds each composition's backward primitives, and
 // GRANII_SELECT_INPUT_LAYER drops the dH branch (not needed for layer 1).
+#include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -44,7 +46,8 @@ struct CostModel {
 //   gat_bwd_a/b     : [1, streamed GB (idx, er / row records), row GB, gathered GB from L2,
 //                      gathered GB from HBM, M rows, M dependent gather steps]  (gat_bwd.cu)
 //   elementwise     : [1, GB]
-//   allgather       : [1, GB received per GPU]
+//   allgather       : [1, GB received per GPU]  (not calibrated: the pool has one GPU; the
+//                     slope is an assumed NCCL bus bandwidth of 0.65 TB/s on NVLink 5)
 static CostModel defaults() {
   CostModel m;
   m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0};
@@ -56,7 +59,7 @@ static CostModel defaults() {
   m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["elementwise"] = {0.004, 1.0 / 5.5};
-  m.coef["allgather"] = {0.020, 1.0 / 700.0};
+  m.coef["allgather"] = {0.020, 1.0 / 0.65};
   return m;
 }
 
@@ -177,24 +180,36 @@ static double cost(const CostModel& m, const In& in, int p, double K1, double K2
   return s;
 }
 
+// all-gather of a K-wide operand followed by its aggregation.  Several GPUs with the overlapped
+// block-phased SpMM (layer.cu gathered_spmm): the own block's phase runs under the transfer and
+// each later phase as its block lands, so the pair costs max(comm + one phase, all phases) plus
+// the (G-1) extra read+write passes over the partial output rows.
+static double agg_cost(const CostModel& m, const In& in, int p, double K) {
+  const double sp = cost(m, in, p, K);
+  if (in.world <= 1) return sp;
+  const double ag = cost(m, in, P_ALLGATHER, K);
+  const char* e = getenv("GRANII_COMM_OVERLAP");
+  if (e && e[0] == '0') return ag + sp;
+  const double rmw = (in.world - 1.0) * 2.0 * in.R * K * 4.0 * 1e-9 * m.coef.at("spmm")[2];
+  return std::max(ag + sp / in.world, sp) + rmw;
+}
+
 double forward_cost(const CostModel& m, const In& in, int comp, double K1, double K2) {
   switch (comp) {
     case GRANII_GCN_PRE_AGG:
-      return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_W, K1) +
-             cost(m, in, P_GEMM, K1, K2);
+      return cost(m, in, P_SDDMM1, 0) + agg_cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_PRE_UPD:
-      return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) +
-             cost(m, in, P_SPMM_W, K2);
+      return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_W, K2);
     case GRANII_GCN_DYN_AGG:
-      return cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
+      return agg_cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_DYN_UPD:
-      return cost(m, in, P_GEMM, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);
+      return cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_U, K2);
     case GRANII_GAT_REUSE:
-      return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SDDMM1_SM, 0) +
-             cost(m, in, P_SPMM_W, K2);
+      return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
+             agg_cost(m, in, P_SPMM_W, K2);
     case GRANII_GAT_RECOMP:
-      return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SDDMM1_SM, 0) +
-             cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
+      return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
+             agg_cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
   }
   return 1e30;
 }
@@ -229,17 +244,17 @@ double backward_cost(const CostModel& m, const In& in, int comp, double K1, doub
   switch (comp) {
     case GRANII_GCN_PRE_AGG:
       t += cost(m, in, P_SDDMM1, 0);
-      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_W, K1);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + agg_cost(m, in, P_SPMM_W, K1);
       break;
     case GRANII_GCN_PRE_UPD:
-      t += cost(m, in, P_SDDMM1, 0) + cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_W, K2);
+      t += cost(m, in, P_SDDMM1, 0) + agg_cost(m, in, P_SPMM_W, K2);
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
       break;
     case GRANII_GCN_DYN_AGG:
-      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U, K1);
+      if (need_dH) t += cost(m, in, P_GEMM, K2, K1) + agg_cost(m, in, P_SPMM_U, K1);
       break;
     case GRANII_GCN_DYN_UPD:
-      t += cost(m, in, P_ALLGATHER, K2) + cost(m, in, P_SPMM_U, K2);  // inner D fused in the ReLU' pass
+      t += agg_cost(m, in, P_SPMM_U, K2);  // inner D fused in the ReLU' pass
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
       break;
     case GRANII_GAT_REUSE:  // gat_backward_impl: prep ; A, B at K2 ; dW = Hᵀ dΘ ; (dH = dΘ Wᵀ) ; Hᵀ[del, der]
@@ -257,9 +272,17 @@ double backward_cost(const CostModel& m, const In& in, int comp, double K1, doub
   return t;
 }
 
+// On a partitioned graph every rank must choose the SAME composition (the compositions issue
+// different collectives), so the inputs are the whole graph's, averaged per rank -- never this
+// rank's own rows.
 static In inputs_of(const granii_graph_s* g) {
   DevInfo di;
   if (dev_info(&di) != GRANII_OK) di = DevInfo();  // host-only selection still works
+  if (g->world > 1) {
+    const double G = (double)g->world, N = (double)g->N, nnz = (double)g->nnz;
+    return In{N / G, nnz / G, (double)g->n_cols, N > 0 ? nnz / N : 0.0, (double)di.l2_bytes, G,
+              (double)std::max<int64_t>(g->n_seg_global, 0) / G};
+  }
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
             (double)g->world, (double)g->n_seg};
 }

@@ -102,6 +102,8 @@ _SIGS = {
     "granii_comm_create": ([_p, _i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_comm_destroy": ([_p], ctypes.c_int),
     "granii_comm_create_local": ([_i32, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_comm_create_stub": ([_i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_comm_stats": ([_p, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)], ctypes.c_int),
     "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
     "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
     "granii_profile_enable": ([_i32], ctypes.c_int),
@@ -367,6 +369,20 @@ def granii_comm_create_local(world: int) -> list:
     hs = (_p * world)()
     _check(_lib.granii_comm_create_local(world, hs), "granii_comm_create_local")
     return [Comm(hs[r], r, world) for r in range(world)]
+
+
+def granii_comm_create_stub(rank: int, world: int) -> Comm:
+    """TIMING STUB (collectives move no data): times one rank's local work on one GPU."""
+    h = _p()
+    _check(_lib.granii_comm_create_stub(rank, world, ctypes.byref(h)), "granii_comm_create_stub")
+    return Comm(h.value, rank, world)
+
+
+def granii_comm_stats(comm: Comm):
+    """(bytes received by this rank, collective calls) since the communicator was created"""
+    b, c = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_lib.granii_comm_stats(comm.handle, ctypes.byref(b), ctypes.byref(c)), "granii_comm_stats")
+    return b.value, c.value
 
 
 # ---------------------------------------------------------------- training helpers

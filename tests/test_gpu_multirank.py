@@ -238,3 +238,62 @@ def test_ext_models_partitioned(G, world, model, comp):
 
     res, _ = run_ranks(G, world, n, s, d, body)
     assert err_act(torch.cat(res), ref, pre) <= TOL
+
+
+def test_comm_aware_selection(G, monkeypatch):
+    """N1: on a partitioned graph the cost of every aggregation includes the all-gather of its
+    operand (N x K x 4 B x (G-1)/G received per GPU), overlapped with the block-phased SpMM"""
+    n, s, d = graph_case("sparse")
+    world = 8
+    g = G.granii_graph_csr_create(n, s.to(DEV).contiguous(), d.to(DEV).contiguous(), F, 3, world)
+    name, f = G.granii_cost_features(g, 9, 64)   # P_ALLGATHER at K = 64
+    assert name == "allgather"
+    ncols = world * g.info.max_local_rows
+    assert f[1] == pytest.approx(ncols * 64 * 4 * (world - 1) / world * 1e-9, rel=1e-12)
+    for model, K1, K2 in ((G.GAT, 32, 512), (G.GCN, 256, 64), (G.GCN, 64, 256)):
+        _, p_on = G.granii_select(g, model, K1, K2)
+        monkeypatch.setenv("GRANII_COMM_OVERLAP", "0")
+        _, p_off = G.granii_select(g, model, K1, K2)
+        monkeypatch.delenv("GRANII_COMM_OVERLAP")
+        assert set(p_on) == set(p_off)
+        for k in p_on:  # hiding the transfer can only lower the predicted time
+            assert p_off[k] >= p_on[k] - 1e-12, (model, k)
+
+
+@pytest.mark.parametrize("name", ["sparse", "dense"])
+def test_selection_identical_on_every_rank(G, name, monkeypatch):
+    """the compositions issue different collectives, so every rank of a partition must select the
+    same one: the selector's inputs on a partitioned graph are whole-graph quantities"""
+    n, s, d = graph_case(name)
+    monkeypatch.setenv("GRANII_SEG", "64")   # hub segments exist and are unevenly spread over ranks
+    sd, dd = s.to(DEV).contiguous(), d.to(DEV).contiguous()
+    for world in (2, 5, 8):
+        gs = [G.granii_graph_csr_create(n, sd, dd, F, r, world) for r in range(world)]
+        for model, K1, K2, fl in ((G.GCN, 64, 256, 0), (G.GCN, 256, 64, G.SELECT_TRAINING),
+                                  (G.GAT, 32, 128, G.SELECT_TRAINING | G.SELECT_INPUT_LAYER)):
+            picks = [G.granii_select(g, model, K1, K2, flags=fl) for g in gs]
+            assert all(p == picks[0] for p in picks), (world, model, picks)
+
+
+def test_comm_stats_count_the_exchanged_bytes(G):
+    """granii_comm_stats: a DYN_UPD forward on a G-way partition receives (G-1) blocks of the
+    K2-wide gather buffer per rank (block broadcasts), the backward the same again plus the
+    ring all-reduce of dW"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    n, s, d = graph_case("sparse")
+    world, K1, K2 = 4, 16, 24
+    W = synth.glorot(95, 2, K1, K2, (K1, K2))
+
+    def body(r, g, comm, rows):
+        b0, b1 = rows
+        net = GNN(g, [LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=3, W=W.to(DEV))], DEV, comm=comm)
+        net.forward(padded(synth.features(95, n, K1)[b0:b1]))
+        f = G.granii_comm_stats(comm)
+        net.backward(padded(synth.uniform_pm1(95, 3, (n, K2))[b0:b1]), need_input_grad=False)
+        return f, G.granii_comm_stats(comm), g.info.max_local_rows
+
+    res, _ = run_ranks(G, world, n, s, d, body)
+    for (fb, fc), (bb, bc), mr in res:
+        ld = (K2 + 7) // 8 * 8
+        assert fb == (world - 1) * mr * ld * 4 and fc == world
+        assert bb - fb == (world - 1) * mr * ld * 4 + int(2.0 * K1 * K2 * 4 * (world - 1) / world)
