@@ -26,6 +26,8 @@
 // fixed reduction order (bitwise reproducible).
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 
 #include "internal.h"
 
@@ -426,6 +428,25 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   // rows (degree > g->wide_deg) a warp each
   GatBwdArgs b = a;
   b.n_wide = g->avg_deg() >= 16.f ? a.n_rows : std::min<int64_t>(g->n_wide, a.n_rows);
+  // tuning hook GRANII_GATBWD="LPG,NJ,U" (tools: bench.py per_primitive_ms), if it covers K
+  if (const char* e = getenv("GRANII_GATBWD")) {
+    int l = 0, n = 0, u = 0;
+    sscanf(e, "%d,%d,%d", &l, &n, &u);
+    if ((int64_t)l * n * 4 >= K) {
+      bool ok = true;
+      if (l == 8 && n == 2 && u == 4) gb_launch<8, 2, 4>(pass, b, st);
+      else if (l == 16 && n == 1 && u == 4) gb_launch<16, 1, 4>(pass, b, st);
+      else if (l == 16 && n == 2 && u == 4) gb_launch<16, 2, 4>(pass, b, st);
+      else if (l == 16 && n == 2 && u == 2) gb_launch<16, 2, 2>(pass, b, st);
+      else if (l == 32 && n == 1 && u == 4) gb_launch<32, 1, 4>(pass, b, st);
+      else if (l == 32 && n == 1 && u == 2) gb_launch<32, 1, 2>(pass, b, st);
+      else ok = false;
+      if (ok) {
+        GR_CHECK_LAUNCH();
+        return GRANII_OK;
+      }
+    }
+  }
   if (K <= 16) gb_launch<4, 1, 4>(pass, b, st);
   else if (K <= 32) gb_launch<8, 1, 4>(pass, b, st);
   else if (K <= 64) gb_launch<8, 2, 2>(pass, b, st);

@@ -122,13 +122,16 @@ granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const f
                              float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                              int64_t ldb, float beta, cudaStream_t st);
 // one phase of a block-phased aggregation over a partitioned graph (layer.cu gathered_spmm):
-// the entries whose column lies in rank `owner`'s gather block; partial = heavy-segment scratch
-// [n_seg][round_up(K,4)] kept across the phases (NULL if the graph has no segments)
+// the entries whose column lies in the gather blocks [p0, p1), block `skip` excluded (-1: none);
+// partial = heavy-segment scratch [n_seg][round_up(K,4)] kept across the phases (NULL if the
+// graph has no segments)
 struct SpmmPhase {
-  int owner;
+  int p0, p1, skip;
   int first, last;
   float* partial;
 };
+// phases of an overlapped aggregation on a partitioned graph (select.cpp; 1 = all-gather first)
+int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale);
 granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                                 float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                                 int64_t ldb, float beta, const SpmmPhase& ph, cudaStream_t st);

@@ -80,14 +80,15 @@ static granii_status allgather(const Ctx& c, GatherBuf& gb) {
 
 // Aggregation Y = spmm(X) over a dense operand whose own rows are already in gb.mine.
 // One GPU: a plain SpMM.  Several GPUs (N1): instead of all-gather -> SpMM, the blocks are
-// broadcast one source rank at a time on the communicator's side stream, and the SpMM runs in
-// phases on the caller's stream -- this rank's block first (nothing to wait for), then every
-// other block as soon as its broadcast has landed -- so the transfer overlaps the aggregation.
-// Each row's entries owned by one rank are a contiguous run (sorted columns, monotone gather
-// layout: graph owner_off), so a phase is a plain SpMM over sub-ranges that continues from the
-// previous phase's raw partial; the epilogue runs in the last phase.  Phase order is fixed,
-// so results are run-to-run bitwise reproducible.  GRANII_COMM_OVERLAP=0: all-gather, then
-// one SpMM.
+// broadcast one source rank at a time (rank order) on the communicator's side stream while the
+// SpMM runs in P phases on the caller's stream: this rank's block first (nothing to wait for),
+// then the other G-1 blocks in P-1 chunks, each as soon as its last broadcast has landed -- the
+// transfer overlaps the aggregation.  Each row's entries owned by one rank are a contiguous run
+// (sorted columns, monotone gather layout: graph owner_off), so a phase is a plain SpMM over
+// sub-ranges that continues from the previous phase's raw partial; the epilogue runs in the last
+// phase.  P comes from the cost model (select.cpp agg_schedule; P = 1 = all-gather then one
+// SpMM); the phase order is fixed, so results are run-to-run bitwise reproducible.
+// GRANII_COMM_OVERLAP=0 forces P = 1, GRANII_COMM_PHASES=P forces P.
 static bool overlap_enabled() {
   const char* e = getenv("GRANII_COMM_OVERLAP");
   return !(e && e[0] == '0');
@@ -98,7 +99,8 @@ static granii_status gathered_spmm(const Ctx& c, GatherBuf& gb, const float* val
                                    int64_t ldb = 0, float beta = 0.f) {
   const granii_graph_s* g = c.g;
   if (!c.dist()) return launch_spmm_ex(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, c.st);
-  if (!overlap_enabled() || !g->owner_off) {
+  const int P = overlap_enabled() && g->owner_off ? comm_phases(g, K, vals != nullptr, cs != nullptr) : 1;
+  if (P <= 1) {
     GR_TRY(allgather(c, gb));
     return launch_spmm_ex(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, c.st);
   }
@@ -116,10 +118,14 @@ static granii_status gathered_spmm(const Ctx& c, GatherBuf& gb, const float* val
   float* partial = nullptr;
   if (g->n_seg > 0)
     GR_CUDA(cudaMallocAsync((void**)&partial, (size_t)g->n_seg * round_up(K, 4) * sizeof(float), c.st));
-  for (int i = 0; i < G; ++i) {
-    const int p = i == 0 ? me : (i <= me ? i - 1 : i);  // own block, then the others ascending
-    if (p != me) GR_CUDA(cudaStreamWaitEvent(c.st, ev[p], 0));
-    SpmmPhase ph{p, i == 0, i == G - 1, partial};
+  SpmmPhase own{me, me + 1, -1, 1, 0, partial};
+  GR_TRY(launch_spmm_phase(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, own, c.st));
+  // the other blocks in rank order ("other" index k -> rank k + (k >= me)), P-1 chunks
+  for (int q = 0; q < P - 1; ++q) {
+    const int k0 = (G - 1) * q / (P - 1), k1 = (G - 1) * (q + 1) / (P - 1);
+    const int r0 = k0 + (k0 >= me), rl = (k1 - 1) + (k1 - 1 >= me);  // first and last rank
+    GR_CUDA(cudaStreamWaitEvent(c.st, ev[rl], 0));
+    SpmmPhase ph{r0, rl + 1, (r0 < me && me < rl) ? me : -1, 0, q == P - 2, partial};
     GR_TRY(launch_spmm_phase(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, ph, c.st));
   }
   GR_CUDA(cudaStreamWaitEvent(c.st, ev[G - 1], 0));  // the side stream is idle (own send included)

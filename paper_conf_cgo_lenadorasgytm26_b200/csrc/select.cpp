@@ -65,6 +65,7 @@ static CostModel defaults() {
 
 static std::mutex g_mu;
 static std::map<std::string, CostModel> g_cache;
+static std::string g_last_path;  // calibration of the last selection (used by the phase planner)
 
 static granii_status load_model(const char* path, CostModel* out) {
   std::lock_guard<std::mutex> lk(g_mu);
@@ -72,6 +73,7 @@ static granii_status load_model(const char* path, CostModel* out) {
   auto it = g_cache.find(key);
   if (it != g_cache.end()) {
     *out = it->second;
+    if (!key.empty()) g_last_path = key;
     return GRANII_OK;
   }
   CostModel m = defaults();
@@ -97,20 +99,27 @@ static granii_status load_model(const char* path, CostModel* out) {
     fclose(f);
   }
   g_cache[key] = m;
+  g_last_path = key;
   *out = m;
   return GRANII_OK;
 }
 
 struct In {
   double R, nnz, ncols, avg, l2, world, nseg;
+  double xcols;  // rows of X an SpMM gathers from (a phased SpMM slices like the whole one: ncols)
 };
+
+static bool overlap_on() {
+  const char* e = getenv("GRANII_COMM_OVERLAP");
+  return !(e && e[0] == '0');
+}
 
 // fraction of gathered bytes served by L2: the sliced SpMM keeps
 // a slice resident when the graph is dense; otherwise LRU-like hit ~ L2 / |X|.
-static double l2_hit(const In& in, double K) {
-  const double xbytes = in.ncols * K * 4.0;
+static double l2_hit(const In& in, double K, double cols) {
+  const double xbytes = cols * K * 4.0;
   if (xbytes <= 0.8 * in.l2) return 1.0;
-  if (in.avg >= 32.0 && in.ncols * 64.0 * 4.0 <= 0.55 * in.l2) return 1.0;  // K-sliced
+  if (in.avg >= 32.0 && cols * 64.0 * 4.0 <= 0.55 * in.l2) return 1.0;  // K-sliced
   return std::max(0.0, std::min(1.0, 0.8 * in.l2 / xbytes));
 }
 
@@ -139,7 +148,7 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
   const double gb = 1e-9;
   switch (p) {
     case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: {
-      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
+      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K, in.xcols);
       const double idx = in.nnz * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 4.0 : 0.0)) * gb;
       return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3};
     }
@@ -158,7 +167,7 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
       return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
               std::ceil(K1 / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
     case P_GAT_BWD_A: case P_GAT_BWD_B: {
-      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K);
+      const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K, in.ncols);
       const double idx = in.nnz * (p == P_GAT_BWD_A ? 8.0 : 20.0) * gb;
       // dependent gather steps per warp (gat_bwd.cu: G lane groups x U entries per step)
       const double gu = K <= 16 ? 32 : K <= 32 ? 16 : K <= 128 ? 8 : K <= 256 ? 4 : K <= 512 ? 2 : 1;
@@ -180,19 +189,50 @@ static double cost(const CostModel& m, const In& in, int p, double K1, double K2
   return s;
 }
 
-// all-gather of a K-wide operand followed by its aggregation.  Several GPUs with the overlapped
-// block-phased SpMM (layer.cu gathered_spmm): the own block's phase runs under the transfer and
-// each later phase as its block lands, so the pair costs max(comm + one phase, all phases) plus
-// the (G-1) extra read+write passes over the partial output rows.
-static double agg_cost(const CostModel& m, const In& in, int p, double K) {
+// All-gather of a K-wide operand followed by its aggregation, on G > 1 GPUs (layer.cu
+// gathered_spmm).  P = 1: all-gather, then one SpMM.  P >= 2 (overlapped): the G blocks are
+// broadcast in rank order on a side stream (landing uniformly over the transfer time); the SpMM
+// runs the own block first, then the other G-1 blocks in P-1 chunks, each chunk once its last
+// block has landed.  Every phase after the first re-reads and re-writes the partial output rows
+// (plus a launch).  Returns the predicted time of the best P (rank-independent inputs, so every
+// rank plans the same schedule) and that P.
+static double agg_schedule(const CostModel& m, const In& in, int p, double K, int* best_P) {
   const double sp = cost(m, in, p, K);
+  if (best_P) *best_P = 1;
   if (in.world <= 1) return sp;
   const double ag = cost(m, in, P_ALLGATHER, K);
-  const char* e = getenv("GRANII_COMM_OVERLAP");
-  if (e && e[0] == '0') return ag + sp;
-  const double rmw = (in.world - 1.0) * 2.0 * in.R * K * 4.0 * 1e-9 * m.coef.at("spmm")[2];
-  return std::max(ag + sp / in.world, sp) + rmw;
+  double best = ag + sp;
+  if (!overlap_on()) return best;
+  const int G = (int)in.world;
+  const std::vector<double>& c = m.coef.at("spmm");
+  // per extra phase (measured on B200, products- and Reddit-shaped partitions at G = 8,
+  // profiles/r01/phase_overhead.json): ~40 us of launch + tail per K slice, ~0.45 ns per row
+  // (the dependent row-metadata chain, not hidden when a phase has few entries per row), and
+  // the read + write of the partial output rows
+  double slices = 1.0;
+  if (in.avg >= 32.0 && in.ncols * K * 4.0 > 0.6 * in.l2) {
+    const double fit = std::floor(0.55 * in.l2 / (in.ncols * 4.0) / 64.0) * 64.0;
+    if (fit >= 64.0) slices = std::ceil(K / fit);
+  }
+  const double h = 0.040 * slices + 0.45e-6 * in.R + 2.0 * in.R * K * 4.0 * 1e-9 * c[2];
+  for (int P = 2; P <= G; ++P) {
+    double t = sp / G;  // own block, under the transfer
+    int done = 0;
+    for (int q = 0; q < P - 1; ++q) {
+      const int n = (G - 1) * (q + 1) / (P - 1) - (G - 1) * q / (P - 1);  // blocks in this chunk
+      done += n;
+      const double landed = ag * (double)done / (G - 1);
+      t = std::max(t, landed) + sp * n / G + h;
+    }
+    if (t < best) {
+      best = t;
+      if (best_P) *best_P = P;
+    }
+  }
+  return best;
 }
+
+static double agg_cost(const CostModel& m, const In& in, int p, double K) { return agg_schedule(m, in, p, K, nullptr); }
 
 double forward_cost(const CostModel& m, const In& in, int comp, double K1, double K2) {
   switch (comp) {
@@ -281,10 +321,10 @@ static In inputs_of(const granii_graph_s* g) {
   if (g->world > 1) {
     const double G = (double)g->world, N = (double)g->N, nnz = (double)g->nnz;
     return In{N / G, nnz / G, (double)g->n_cols, N > 0 ? nnz / N : 0.0, (double)di.l2_bytes, G,
-              (double)std::max<int64_t>(g->n_seg_global, 0) / G};
+              (double)std::max<int64_t>(g->n_seg_global, 0) / G, (double)g->n_cols};
   }
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-            (double)g->world, (double)g->n_seg};
+            (double)g->world, (double)g->n_seg, (double)g->n_cols};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, const granii_layer_args* shape,
@@ -335,6 +375,27 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, const gra
   if (ncand) *ncand = (int32_t)c.size();
   *out = (granii_composition)best;
   return GRANII_OK;
+}
+
+// number of phases of an overlapped aggregation (1 = all-gather then SpMM); GRANII_COMM_PHASES
+// overrides.  weighted / col_scale pick the SpMM model (P_SPMM_W / P_SPMM_U_CS / P_SPMM_U).
+int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale) {
+  if (g->world <= 1) return 1;
+  if (const char* e = getenv("GRANII_COMM_PHASES")) {
+    const int P = atoi(e);
+    if (P >= 1) return std::min(P, (int)g->world);
+  }
+  std::string path;
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    path = g_last_path;
+  }
+  if (path.empty() && getenv("GRANII_CALIB")) path = getenv("GRANII_CALIB");
+  CostModel m;
+  if (load_model(path.empty() ? nullptr : path.c_str(), &m) != GRANII_OK) m = defaults();
+  int P = 1;
+  agg_schedule(m, inputs_of(g), weighted ? P_SPMM_W : col_scale ? P_SPMM_U_CS : P_SPMM_U, (double)K, &P);
+  return P;
 }
 
 granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t K1, int64_t K2, double* feats,

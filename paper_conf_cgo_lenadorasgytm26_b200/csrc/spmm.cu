@@ -77,20 +77,24 @@ struct SpmmArgs {
   int64_t ldb;
   float beta;
   // block-phased mode (owner_off != nullptr; layer.cu gathered_spmm, N1): only the entries whose
-  // column lies in rank `owner`'s block of the gather buffer.  `first`: start from zero, else from
-  // the raw partial already in Y (light rows) / partial (segments); `last`: apply the epilogue.
+  // column lies in the owner blocks [p0, p1) of the gather buffer, block `skip` excluded (-1: none).
+  // `first`: start from zero, else from the raw partial already in Y (light rows) / partial
+  // (segments); `last`: apply the epilogue.
   const int32_t* __restrict__ owner_off;   // [n_rows][G1]
   const int32_t* __restrict__ seg_row;     // row of each heavy segment
-  int G1, owner, first, last;
+  int G1, p0, p1, skip, first, last;
 };
 
-// entry range of `row` restricted to the phase's owner block (whole row outside phased mode)
-__device__ __forceinline__ void phase_range(const SpmmArgs& a, int64_t row, int64_t& lo, int64_t& hi) {
-  if (!a.owner_off) return;
-  const int32_t* o = a.owner_off + row * a.G1 + a.owner;
+// part r (0, or 1 after a skipped block) of the entries of `row` within [l0, h0) whose column lies
+// in the phase's owner blocks
+__device__ __forceinline__ void phase_part(const SpmmArgs& a, int64_t row, int r, int64_t l0, int64_t h0,
+                                           int64_t& lo, int64_t& hi) {
+  const int32_t* o = a.owner_off + row * a.G1;
   const int64_t base = a.row_ptr[row];
-  lo = max(lo, base + (int64_t)o[0]);
-  hi = min(hi, base + (int64_t)o[1]);
+  const int b0 = r == 0 ? a.p0 : a.skip + 1;
+  const int b1 = (r == 0 && a.skip >= 0) ? a.skip : a.p1;
+  lo = max(l0, base + (int64_t)o[b0]);
+  hi = min(h0, base + (int64_t)o[b1]);
 }
 
 // continue a phased accumulation from the raw partial stored by the previous phase
@@ -216,28 +220,40 @@ __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], con
 }
 
 // heavy-row segments first (largest work first), as warp-wide items
-template <int VEC, int LPG, int NJ, bool W, bool CS, int U>
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U>
 __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lane, int grp, int lig,
                                            const bool (&colok)[NJ], const char* const (&xbj)[NJ],
                                            uint32_t row_bytes) {
   float acc[NJ][VEC];
   zero(acc);
-  int64_t lo = a.seg_lo[t], hi = a.seg_hi[t];
   float* part = a.partial + t * a.ldp + (int64_t)lig * VEC;
-  if (a.owner_off) {
-    phase_range(a, a.seg_row[t], lo, hi);
+  if constexpr (PH) {
     if (!a.first && grp == 0) load_partial<LPG>(part, colok, acc);
+    for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {  // the range(s) are computed when needed
+      int64_t lo, hi;
+      phase_part(a, a.seg_row[t], r, a.seg_lo[t], a.seg_hi[t], lo, hi);
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
+    }
+  } else {
+    warp_range<VEC, LPG, NJ, W, CS, U>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc);
   }
-  warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
   reduce_groups<LPG>(acc);
   if (grp == 0) store_row<LPG>(part, colok, acc, 1.f, 0);
 }
 
 // ------------------------------------------------------------------ warp-per-row
-template <int VEC, int LPG, int NJ, bool W, bool CS, int UU = 0, int MINB = 3>
-__global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
+// defaults (tools/spmm_sweep.py on B200, Reddit- and products-shaped graphs): 16-byte gathers of
+// <= 2 vectors per lane keep 2 neighbours per group in flight at 4 blocks/SM (64 registers);
+// wider rows keep the register budget of 3 blocks/SM
+template <int VEC, int NJ>
+constexpr int spmm_minb() { return VEC == 4 && NJ <= 2 ? 4 : 3; }
+template <int VEC, int LPG, int NJ>
+constexpr int spmm_unroll() { return VEC == 4 && NJ <= 2 ? 2 : (LPG >= 8 ? 4 : 32 / (32 / LPG)); }
+
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int UU = 0, int MINB = 0>
+__global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k_spmm_warp(SpmmArgs a) {
   constexpr int G = 32 / LPG;
-  constexpr int U = UU > 0 ? UU : (32 / G >= 4 ? 4 : 32 / G);  // neighbours per group per step; G*U divides 32
+  constexpr int U = UU > 0 ? UU : spmm_unroll<VEC, LPG, NJ>();  // neighbours per group per step
   static_assert(32 % (G * U) == 0, "G*U must divide 32");
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -248,22 +264,26 @@ __global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
   for (int64_t t = warp; t < a.n_seg + a.n_rows; t += nwarps) {
     if (t < a.n_seg) {
-      do_segment<VEC, LPG, NJ, W, CS, U>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+      do_segment<VEC, LPG, NJ, W, CS, PH, U>(a, t, lane, grp, lig, colok, xbj, row_bytes);
       continue;
     }
     const int64_t row = a.order[t - a.n_seg];
     float acc[NJ][VEC];
     zero(acc);
-    int64_t lo = a.row_ptr[row], hi = a.row_ptr[row + 1];
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
-    if (a.owner_off) {
-      phase_range(a, row, lo, hi);
+    if constexpr (PH) {
       if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
+      for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
+        int64_t lo, hi;
+        phase_part(a, row, r, 0, INT64_MAX, lo, hi);
+        warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
+      }
+    } else {
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
     }
-    warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
     reduce_groups<LPG>(acc);
     if (grp == 0) {
-      if (a.owner_off && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
+      if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
       else
         store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
                        a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
@@ -272,7 +292,7 @@ __global__ void __launch_bounds__(256, MINB) k_spmm_warp(SpmmArgs a) {
 }
 
 // ------------------------------------------------------------------ group-per-row
-template <int VEC, int LPG, int NJ, bool W, bool CS>
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH>
 __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   constexpr int G = 32 / LPG;
   constexpr int U = 4;
@@ -285,20 +305,24 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   slice_setup<VEC, LPG>(a, lig, colok, xbj);
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
   for (int64_t t = warp; t < a.n_seg; t += nwarps)  // heavy segments: whole warps
-    do_segment<VEC, LPG, NJ, W, CS, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+    do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
   // light rows: one LPG-lane group per row
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
     const int64_t row = a.order[t];
-    int64_t rs0 = a.row_ptr[row], re = a.row_ptr[row + 1];
     float acc[NJ][VEC];
     zero(acc);
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
-    if (a.owner_off) {
-      phase_range(a, row, rs0, re);
-      if (!a.first) load_partial<LPG>(y, colok, acc);
-    }
+    if (PH && !a.first) load_partial<LPG>(y, colok, acc);
+    for (int part = 0; part < (PH && a.skip >= 0 ? 2 : 1); ++part) {
+      int64_t rs0, re;
+      if constexpr (PH) {
+        phase_part(a, row, part, 0, INT64_MAX, rs0, re);
+      } else {
+        rs0 = a.row_ptr[row];
+        re = a.row_ptr[row + 1];
+      }
     for (int64_t e = rs0; e < re; e += U) {
       uint32_t cu[U];
       float wu[U];
@@ -324,7 +348,8 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
 #pragma unroll
           for (int v = 0; v < VEC; ++v) acc[j][v] = fmaf(wu[u], x[u][j][v], acc[j][v]);
     }
-    if (a.owner_off && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
+    }
+    if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
     else
       store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
                      a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
@@ -351,7 +376,7 @@ __global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heav
 }
 
 // ------------------------------------------------------------------ dispatch
-template <int VEC, int LPG, int NJ>
+template <int VEC, int LPG, int NJ, bool PH>
 static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool cs, int sms, cudaStream_t st) {
   const int threads = 256;
   int64_t units = (warp_mode ? a.n_rows : ceil_div(a.n_rows, 32 / LPG)) + a.n_seg;
@@ -360,35 +385,40 @@ static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool 
   blocks = std::max<int64_t>(blocks, 1);
 #define GR_L(K) K<<<(unsigned)blocks, threads, 0, st>>>(a)
   // tuning hook (GRANII_SPMM_TUNE="U,MINB"): alternative unroll / occupancy for the
-  // unweighted warp-per-row kernels of the two dominant shapes
-  if constexpr (VEC == 4 && NJ == 2 && (LPG == 8 || LPG == 32)) {
+  // warp-per-row kernels of the dominant shapes (tools/spmm_sweep.py)
+  if constexpr (!PH && VEC == 4 && NJ == 2 && (LPG == 8 || LPG == 16 || LPG == 32)) {
     const char* tune = getenv("GRANII_SPMM_TUNE");
-    if (warp_mode && !w && !cs && tune) {
+    if (warp_mode && tune) {
       int u = 0, mb = 0;
       sscanf(tune, "%d,%d", &u, &mb);
       const int64_t bl = std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 16));
-#define GR_T(U_, M_) k_spmm_warp<VEC, LPG, NJ, false, false, U_, M_><<<(unsigned)bl, threads, 0, st>>>(a)
-      if (u == 2 && mb == 4) GR_T(2, 4);
-      else if (u == 2 && mb == 3) GR_T(2, 3);
-      else if (u == 8 && mb == 2) GR_T(8, 2);
-      else if (u == 4 && mb == 4) GR_T(4, 4);
-      else if (u == 4 && mb == 2) GR_T(4, 2);
-      else GR_T(4, 3);
+#define GR_T2(W_, C_, U_, M_) k_spmm_warp<VEC, LPG, NJ, W_, C_, false, U_, M_><<<(unsigned)bl, threads, 0, st>>>(a)
+#define GR_T(U_, M_)                  \
+  do {                                \
+    if (w && cs) GR_T2(true, true, U_, M_);   \
+    else if (w) GR_T2(true, false, U_, M_);   \
+    else if (cs) GR_T2(false, true, U_, M_);  \
+    else GR_T2(false, false, U_, M_);         \
+  } while (0)
+      if (u == 4 && mb == 4) GR_T(4, 4);
+      else if (u == 4 && mb == 3) GR_T(4, 3);
+      else GR_T(2, 3);
 #undef GR_T
+#undef GR_T2
       GR_CHECK_LAUNCH();
       return GRANII_OK;
     }
   }
   if (warp_mode) {
-    if (w && cs) GR_L((k_spmm_warp<VEC, LPG, NJ, true, true>));
-    else if (w) GR_L((k_spmm_warp<VEC, LPG, NJ, true, false>));
-    else if (cs) GR_L((k_spmm_warp<VEC, LPG, NJ, false, true>));
-    else GR_L((k_spmm_warp<VEC, LPG, NJ, false, false>));
+    if (w && cs) GR_L((k_spmm_warp<VEC, LPG, NJ, true, true, PH>));
+    else if (w) GR_L((k_spmm_warp<VEC, LPG, NJ, true, false, PH>));
+    else if (cs) GR_L((k_spmm_warp<VEC, LPG, NJ, false, true, PH>));
+    else GR_L((k_spmm_warp<VEC, LPG, NJ, false, false, PH>));
   } else {
-    if (w && cs) GR_L((k_spmm_group<VEC, LPG, NJ, true, true>));
-    else if (w) GR_L((k_spmm_group<VEC, LPG, NJ, true, false>));
-    else if (cs) GR_L((k_spmm_group<VEC, LPG, NJ, false, true>));
-    else GR_L((k_spmm_group<VEC, LPG, NJ, false, false>));
+    if (w && cs) GR_L((k_spmm_group<VEC, LPG, NJ, true, true, PH>));
+    else if (w) GR_L((k_spmm_group<VEC, LPG, NJ, true, false, PH>));
+    else if (cs) GR_L((k_spmm_group<VEC, LPG, NJ, false, true, PH>));
+    else GR_L((k_spmm_group<VEC, LPG, NJ, false, false, PH>));
   }
 #undef GR_L
   GR_CHECK_LAUNCH();
@@ -396,31 +426,34 @@ static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool 
 }
 
 // Pick (VEC, LPG, NJ) for a slice of width kw.  VEC=4 needs 16-byte aligned rows.
+template <bool PH>
 static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, bool w, bool cs, int sms,
                                   cudaStream_t st) {
   const int64_t kw = a.kw;
   if (vec4) {
-    if (kw <= 16) return launch_cfg<4, 4, 1>(a, warp_mode, w, cs, sms, st);
-    if (kw <= 32) return launch_cfg<4, 8, 1>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 16) return launch_cfg<4, 4, 1, PH>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 32) return launch_cfg<4, 8, 1, PH>(a, warp_mode, w, cs, sms, st);
     if (kw <= 64) {
-      if (warp_mode) return launch_cfg<4, 8, 2>(a, warp_mode, w, cs, sms, st);  // 4 groups x 2 float4
-      return launch_cfg<4, 16, 1>(a, warp_mode, w, cs, sms, st);
+      if (warp_mode) return launch_cfg<4, 8, 2, PH>(a, warp_mode, w, cs, sms, st);  // 4 groups x 2 float4
+      return launch_cfg<4, 16, 1, PH>(a, warp_mode, w, cs, sms, st);
     }
     if (kw <= 128) {
-      if (warp_mode) return launch_cfg<4, 16, 2>(a, warp_mode, w, cs, sms, st);
-      return launch_cfg<4, 32, 1>(a, warp_mode, w, cs, sms, st);
+      if (warp_mode) return launch_cfg<4, 16, 2, PH>(a, warp_mode, w, cs, sms, st);
+      return launch_cfg<4, 32, 1, PH>(a, warp_mode, w, cs, sms, st);
     }
-    if (kw <= 256) return launch_cfg<4, 32, 2>(a, warp_mode, w, cs, sms, st);
-    if (kw <= 512) return launch_cfg<4, 32, 4>(a, warp_mode, w, cs, sms, st);
-    return launch_cfg<4, 32, 8>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 256) return launch_cfg<4, 32, 2, PH>(a, warp_mode, w, cs, sms, st);
+    if (kw <= 512) return launch_cfg<4, 32, 4, PH>(a, warp_mode, w, cs, sms, st);
+    return launch_cfg<4, 32, 8, PH>(a, warp_mode, w, cs, sms, st);
   }
-  if (kw <= 32) return launch_cfg<1, 32, 1>(a, warp_mode, w, cs, sms, st);
-  if (kw <= 64) return launch_cfg<1, 32, 2>(a, warp_mode, w, cs, sms, st);
-  if (kw <= 128) return launch_cfg<1, 32, 4>(a, warp_mode, w, cs, sms, st);
-  return launch_cfg<1, 32, 8>(a, warp_mode, w, cs, sms, st);
+  if (kw <= 32) return launch_cfg<1, 32, 1, PH>(a, warp_mode, w, cs, sms, st);
+  if (kw <= 64) return launch_cfg<1, 32, 2, PH>(a, warp_mode, w, cs, sms, st);
+  if (kw <= 128) return launch_cfg<1, 32, 4, PH>(a, warp_mode, w, cs, sms, st);
+  return launch_cfg<1, 32, 8, PH>(a, warp_mode, w, cs, sms, st);
 }
 
-int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t l2_bytes) {
+// cols: rows of X the launch gathers from (the whole column space, or one owner block of a
+// phased aggregation, whose footprint is 1/G of it)
+int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t l2_bytes, int64_t cols) {
   // Keep the gathered column slice of X resident in L2: split
   // K into slices whose X footprint is <= ~45% of L2 when the graph is dense
   // enough for re-use (avg degree >= 32) and X itself does not fit.
@@ -430,7 +463,7 @@ int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t 
     int64_t v = atoll(env);
     if (v > 0) return std::min<int64_t>(std::max<int64_t>(v, 1), maxw);
   }
-  const double per_col = (double)g->n_cols * 4.0;
+  const double per_col = (double)cols * 4.0;
   if (g->avg_deg() >= 32.f && per_col * (double)K > 0.6 * (double)l2_bytes) {
     const int64_t unit = vec4 ? 64 : 32;
     const int64_t fit = (int64_t)(0.55 * (double)l2_bytes / per_col) / unit * unit;  // columns resident in L2
@@ -455,17 +488,22 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   GR_TRY(dev_info(&di));
   const bool vec4 = (ldx % 4 == 0) && (ldy % 4 == 0) && ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0) &&
                     (!B || ((ldb % 4 == 0) && ((uintptr_t)B % 16 == 0)));
-  const bool warp_mode = g->avg_deg() >= 16.f;
+  // a phase sees (p1 - p0 - [skip]) / G of every row on average
+  const float share = ph ? float(ph->p1 - ph->p0 - (ph->skip >= 0 ? 1 : 0)) / float(g->world) : 1.f;
+  const bool warp_mode = g->avg_deg() * share >= 16.f;
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
              g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0, B, ldb, beta};
-  const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes);
+  // phases slice like the whole aggregation: the 64-wide slices also keep the L1 hit rate
+  const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes, g->n_cols);
   float* partial = nullptr;  // heavy-segment partials: this slice's columns start at partial + pk0
   bool own_partial = false;
   if (ph) {
     a.owner_off = g->owner_off;
     a.seg_row = g->seg_row;
     a.G1 = g->world + 1;
-    a.owner = ph->owner;
+    a.p0 = ph->p0;
+    a.p1 = ph->p1;
+    a.skip = ph->skip;
     a.first = ph->first;
     a.last = ph->last;
     a.ldp = round_up(K, 4);  // kept across the phases for every slice
@@ -489,7 +527,9 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
     a.kw = std::min(kw, K - k0);
     a.partial = partial ? partial + (ph ? k0 : 0) : nullptr;
     // slices of a vec4 launch must stay 16-byte aligned
-    GR_TRY(launch_slice(a, vec4 && (k0 % 4 == 0), warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
+    const bool v4 = vec4 && (k0 % 4 == 0);
+    if (ph) GR_TRY(launch_slice<true>(a, v4, warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
+    else GR_TRY(launch_slice<false>(a, v4, warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
     if (combine) {
       const int64_t tot = g->n_heavy * a.kw;
       k_spmm_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(

@@ -12,6 +12,7 @@ dW / da all-reduce.  The concatenation of the
 ranks' owned rows must match the single-process fp64 oracle within the same
 tolerances as the unpartitioned path (test_gpu_parity.py, R19 / R22).
 """
+import os
 import threading
 
 import numpy as np
@@ -108,13 +109,25 @@ def test_partitioned_csr_concatenates_to_global(G, world, name):
     assert np.array_equal(np.concatenate(cols), ci)
 
 
-@pytest.mark.parametrize("overlap", ["1", "0"])
+# phases of the overlapped aggregation: "off" = all-gather then SpMM; "auto" = the cost model's P;
+# "2" = own block + one chunk; "16" = one phase per block (clamped to G)
+PHASES = ["off", "auto", "2", "16"]
+
+
+def set_phases(monkeypatch, phases):
+    monkeypatch.delenv("GRANII_COMM_PHASES", raising=False)
+    monkeypatch.setenv("GRANII_COMM_OVERLAP", "0" if phases == "off" else "1")
+    if phases not in ("off", "auto"):
+        monkeypatch.setenv("GRANII_COMM_PHASES", phases)
+
+
+@pytest.mark.parametrize("phases", PHASES)
 @pytest.mark.parametrize("world", [2, 3, 4])
 @pytest.mark.parametrize("comp", [0, 1, 2, 3])
 @pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 48), ("dense", 64, 24), ("tiny", 3, 5)])
-def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2, overlap, monkeypatch):
+def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2, phases, monkeypatch):
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
-    monkeypatch.setenv("GRANII_COMM_OVERLAP", overlap)
+    set_phases(monkeypatch, phases)
     n, s, d = graph_case(name)
     rp, ci = O.csr_build(n, s, d, F)
     H = synth.features(90, n, K1)
@@ -138,11 +151,13 @@ def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2, overlap,
         assert torch.equal(res[r][2], res[0][2])
 
 
+@pytest.mark.parametrize("phases", ["off", "16"])
 @pytest.mark.parametrize("world", [2, 4])
 @pytest.mark.parametrize("comp", [16, 17])
 @pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 64), ("dense", 48, 16)])
-def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2):
+def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2, phases, monkeypatch):
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    set_phases(monkeypatch, phases)
     n, s, d = graph_case(name)
     rp, ci = O.csr_build(n, s, d, F)
     H = synth.features(91, n, K1)
@@ -171,8 +186,9 @@ def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2):
             assert torch.equal(res[r][i], res[0][i]), (r, nm)
 
 
+@pytest.mark.parametrize("phases", ["2", "3", "16"])
 @pytest.mark.parametrize("world", [3, 8])
-def test_phased_spmm_segments_slices_deterministic(G, world, monkeypatch):
+def test_phased_spmm_segments_slices_deterministic(G, world, phases, monkeypatch):
     """the block-phased aggregation with hub segments (GRANII_SEG=64: partials carried across
     the phases, combined after the last) and forced K slices; bitwise reproducible"""
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
@@ -184,6 +200,7 @@ def test_phased_spmm_segments_slices_deterministic(G, world, monkeypatch):
     Gup = synth.uniform_pm1(94, 3, (n, K2))
     monkeypatch.setenv("GRANII_SEG", "64")
     monkeypatch.setenv("GRANII_SPMM_SLICE", "16")
+    set_phases(monkeypatch, phases)
     for comp in (0, 1, 2, 3):
         def body(r, g, comm, rows):
             b0, b1 = rows
@@ -284,6 +301,8 @@ def test_comm_stats_count_the_exchanged_bytes(G):
     world, K1, K2 = 4, 16, 24
     W = synth.glorot(95, 2, K1, K2, (K1, K2))
 
+    os.environ["GRANII_COMM_PHASES"] = "16"   # one broadcast per block in every regime
+
     def body(r, g, comm, rows):
         b0, b1 = rows
         net = GNN(g, [LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=3, W=W.to(DEV))], DEV, comm=comm)
@@ -292,7 +311,10 @@ def test_comm_stats_count_the_exchanged_bytes(G):
         net.backward(padded(synth.uniform_pm1(95, 3, (n, K2))[b0:b1]), need_input_grad=False)
         return f, G.granii_comm_stats(comm), g.info.max_local_rows
 
-    res, _ = run_ranks(G, world, n, s, d, body)
+    try:
+        res, _ = run_ranks(G, world, n, s, d, body)
+    finally:
+        os.environ.pop("GRANII_COMM_PHASES", None)
     for (fb, fc), (bb, bc), mr in res:
         ld = (K2 + 7) // 8 * 8
         assert fb == (world - 1) * mr * ld * 4 and fc == world

@@ -59,7 +59,12 @@ def rank_step_ms(G, spec, w, src, dst, flags, rank, world, dev, steps, warmup, c
     b0 = G.granii_comm_stats(comm)[0] if comm else 0
     ms = bench.time_region(step, steps, torch.cuda.current_stream())
     b1 = G.granii_comm_stats(comm)[0] if comm else 0
-    out = {"rank": rank, "rows": R, "local_nnz": info.local_nnz, "compute_ms": ms,
+    G.granii_profile_enable(True)   # per-primitive breakdown of one more step (not the timed ones)
+    step()
+    torch.cuda.synchronize()
+    prof = {k: round(v["ms"], 4) for k, v in G.granii_profile_read().items()}
+    G.granii_profile_enable(False)
+    out = {"rank": rank, "rows": R, "local_nnz": info.local_nnz, "compute_ms": ms, "per_primitive_ms": prof,
            "bytes_in_per_step": (b1 - b0) / steps, "compositions": [L.comp for L in net.layers]}
     del net, g, H
     torch.cuda.empty_cache()
@@ -74,8 +79,13 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--bw_gbs", type=float, default=650.0,
                     help="assumed NCCL bus bandwidth per GPU on NVLink 5 (not measurable on a 1-GPU pool)")
+    ap.add_argument("--overlap", default="1", choices=["0", "1"],
+                    help="GRANII_COMM_OVERLAP: 1 = block-phased SpMM (default), 0 = all-gather then SpMM")
+    ap.add_argument("--ranks", default=None, help="time only these ranks (e.g. 0,7)")
+    ap.add_argument("--comp", default=None, help="force the compositions, e.g. 3,3 (skips the selector)")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
+    os.environ["GRANII_COMM_OVERLAP"] = args.overlap
     from paper_conf_cgo_lenadorasgytm26_b200 import granii as G
     dev = torch.device("cuda", 0)
     torch.cuda.set_device(dev)
@@ -89,16 +99,19 @@ def main():
            "how": __doc__.split("\n\n")[1].replace("\n", " "), "per_G": {}}
     for world in [int(x) for x in args.gpus.split(",")]:
         ranks = []
-        for r in range(world):
-            o, nnz = rank_step_ms(G, spec, w, src, dst, flags, r, world, dev, args.steps, args.warmup)
+        sel = range(world) if not args.ranks else [int(x) for x in args.ranks.split(",") if int(x) < world]
+        for r in sel:
+            comps = [int(x) for x in args.comp.split(",")] if args.comp else None
+            o, nnz = rank_step_ms(G, spec, w, src, dst, flags, r, world, dev, args.steps, args.warmup, comps)
             ranks.append(o)
             print(json.dumps({"G": world, **o}), flush=True)
         tc = max(o["compute_ms"] for o in ranks)
+        world_n = len(ranks)
         bytes_in = max(o["bytes_in_per_step"] for o in ranks)
         tcomm = bytes_in / (args.bw_gbs * 1e9) * 1e3
         edges = float(nnz) * layers * passes
         res["per_G"][str(world)] = {
-            "max_rank_compute_ms": tc, "mean_rank_compute_ms": sum(o["compute_ms"] for o in ranks) / world,
+            "max_rank_compute_ms": tc, "mean_rank_compute_ms": sum(o["compute_ms"] for o in ranks) / world_n, "overlap": args.overlap,
             "bytes_in_per_rank_per_step": bytes_in, "modelled_comm_ms": tcomm,
             "no_overlap_ms": tc + tcomm, "overlap_bound_ms": max(tc, tcomm),
             "edges_per_s_no_overlap": edges / ((tc + tcomm) / 1e3),

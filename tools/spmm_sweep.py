@@ -23,8 +23,10 @@ def t(K, reps=5):
     return ms, g.nnz * K * 4 / ms / 1e9
 res = {}
 for K in [int(x) for x in os.environ.get("KS", "256,41,64,128,1024").split(",")]:
-    for tune in ["", "2,4", "2,3", "4,4", "4,2", "8,2"]:
-        for sl in ["", "64", "128", "256"]:
+    for tune in os.environ.get("TUNES", "def;2,4;4,4;4,2;8,2").split(";"):
+        tune = "" if tune == "def" else tune
+        for sl in os.environ.get("SLICES", "auto;64;128;256").split(";"):
+            sl = "" if sl == "auto" else sl
             if sl and int(sl) >= K: continue
             os.environ.pop("GRANII_SPMM_TUNE", None); os.environ.pop("GRANII_SPMM_SLICE", None)
             if tune: os.environ["GRANII_SPMM_TUNE"] = tune
