@@ -122,6 +122,11 @@ __global__ void k_remap_cols(int64_t n, const int32_t* __restrict__ col, const i
   }
 }
 
+__global__ void k_square(int64_t n, const float* __restrict__ x, float* __restrict__ y) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    y[i] = x[i] * x[i];
+}
+
 // owner_off[i][p] = offset in row i of its first entry whose gather-layout column lies in
 // block p (columns are sorted and the layout is monotone in the global id, so each owner's
 // entries are one contiguous run); owner_off[i][G] = deg_i
@@ -180,7 +185,6 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   auto g = new granii_graph_s();
   g->N = N;
   g->rank = rank;
-  if (const char* e = getenv("GRANII_SEG")) g->seg_len = std::max<int64_t>(64, atoll(e));
   g->world = world;
   g->symmetric = sym;
   g->self_loops = loops;
@@ -286,6 +290,16 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   g->features[5] = N > 0 ? (int64_t)hacc[2] : 0;
   g->features[6] = (int64_t)hacc[4];
   g->features[7] = (int64_t)hacc[3];
+  // hub segment length: a work item must stay short next to the average warp's share of the
+  // graph (a 2048-entry segment is ~250 dependent gather steps, a 300 us tail on a graph
+  // whose whole SpMM takes 50 us): nnz / (148 SMs x 64 warps), a power of two in [256, 2048],
+  // from the GLOBAL nnz so every rank of a partition cuts the same way
+  {
+    int64_t want = nnz / (148 * 64), sl = 256;
+    while (sl < 2048 && sl * 2 <= want) sl *= 2;
+    g->seg_len = sl;
+  }
+  if (const char* e = getenv("GRANII_SEG")) g->seg_len = std::max<int64_t>(64, atoll(e));
 
   // partition
   if (world <= 1) {
@@ -345,6 +359,10 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
     cudaFree(col_full);
     cudaFree(dinv_full);
   }
+
+  // dinv^2 of the owned rows: between two hops the post-scale and the next pre-scale are one
+  CK(cudaMalloc(&g->dinv2_rows, std::max<int64_t>(g->n_rows, 1) * sizeof(float)));
+  if (g->n_rows > 0) k_square<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->dinv_rows, g->dinv2_rows);
 
   // degree-descending schedule of the owned rows (stable radix sort: deterministic)
   CK(cudaMalloc(&g->order, std::max<int64_t>(g->n_rows, 1) * sizeof(int32_t)));
@@ -412,6 +430,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
 void graph_free(granii_graph_s* g) {
   if (!g) return;
   cudaFree(g->owner_off);
+  cudaFree(g->dinv2_rows);
   if (g->dinv_cols != g->dinv_rows) cudaFree(g->dinv_cols);
   cudaFree(g->dinv_rows);
   cudaFree(g->row_ptr);

@@ -82,6 +82,7 @@ struct granii_graph_s {
   int32_t* col_idx = nullptr;     // device, local_nnz, column-id space
   float* dinv_rows = nullptr;     // device, n_rows
   float* dinv_cols = nullptr;     // device, n_cols (== dinv_rows when world == 1)
+  float* dinv2_rows = nullptr;    // device, n_rows: 1 / deg (post-scale of one hop fused with the next pre-scale)
   int32_t* order = nullptr;       // device, n_rows: owned rows by descending degree
   int32_t* owner_off = nullptr;   // device, n_rows x (world+1) when world > 1: entries of row i whose
                                   // column is owned by rank p are [rp_i + off[i][p], rp_i + off[i][p+1])
@@ -130,6 +131,9 @@ struct SpmmPhase {
   int first, last;
   float* partial;
 };
+// K slices of a vec4 SpMM and the dynamic-normalisation pre-scale rule (spmm.cu)
+int64_t spmm_slices(double avg_deg, double cols, int64_t K, int64_t l2_bytes);
+bool dyn_prescale(double nnz, double rows, double avg_deg, double cols, int64_t K, int64_t l2_bytes);
 // phases of an overlapped aggregation on a partitioned graph (select.cpp; 1 = all-gather first)
 int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale);
 granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,

@@ -177,20 +177,36 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
   const bool dyn = v >= 2, upd = (v & 1) != 0;
   const int hops = a->hops;
 
+  // SGC DYN: hop inputs are kept pre-scaled by D̃^-½ (the first one by a row-broadcast pass or
+  // the GEMM epilogue, the next ones by fusing D̃^-1 = post-scale x next pre-scale into the hop's
+  // epilogue) instead of gathering dinv[c] in every hop and K slice -- when that moves fewer
+  // bytes (dyn_prescale)
+  DevInfo di;
+  if (dev_info(&di) != GRANII_OK) di = DevInfo();
+  const bool pre = m == GRANII_SGC && dyn && hops > 0 &&
+                   dyn_prescale((double)g->local_nnz, (double)R, g->avg_deg(), (double)g->n_cols, upd ? K2 : K1,
+                                di.l2_bytes);
   // H: aligned own rows, and (aggregate-first) its gathered copy
   const float* H = a->H;
   int64_t ldh = a->ldh;
   const bool h_aligned = (ldh % 4 == 0) && (((uintptr_t)H & 15) == 0);
   GatherBuf hg;
   const bool h_gather = c.dist() && !upd;
+  const bool h_scale = pre && !upd;
   if (h_gather) {
     hg = gather_buf(b, c, K1);
     if (run) {
-      GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hg.mine, hg.ld, st));
+      if (h_scale) GR_TRY(launch_scale_mask(R, K1, nullptr, 0, a->H, a->ldh, g->dinv_rows, hg.mine, hg.ld, st));
+      else GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hg.mine, hg.ld, st));
       GR_TRY(allgather(c, hg));
     }
     H = hg.mine;
     ldh = hg.ld;
+  } else if (h_scale) {
+    float* hp = b.take((size_t)Rr * ld4(K1));
+    if (run) GR_TRY(launch_scale_mask(R, K1, nullptr, 0, a->H, a->ldh, g->dinv_rows, hp, ld4(K1), st));
+    H = hp;
+    ldh = ld4(K1);
   } else if (!h_aligned) {
     float* hp = b.take((size_t)Rr * ld4(K1));
     if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hp, ld4(K1), st));
@@ -212,6 +228,13 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
     if (!dyn) return launch_spmm_ex(g, vals, X, ldx, K, Y, ldy, nullptr, nullptr, rl, B, ldb, beta, st);
     return launch_spmm_ex(g, nullptr, X, ldx, K, Y, ldy, g->dinv_rows, g->dinv_cols, rl, B, ldb, beta, st);
   };
+  // SGC hop: with pre-scaled inputs the row scale is D̃^-1 between hops, D̃^-½ after the last
+  auto sgc_hop = [&](const float* X, int64_t ldx, int64_t K, float* Y, int64_t ldy, bool rl,
+                     bool last) -> granii_status {
+    if (!pre) return hop(X, ldx, K, Y, ldy, rl, nullptr, 0, 0.f);
+    return launch_spmm_ex(g, nullptr, X, ldx, K, Y, ldy, last ? g->dinv_rows : g->dinv2_rows, nullptr, rl, nullptr,
+                          0, 0.f, st);
+  };
 
   if (m == GRANII_SGC) {
     const int64_t K = upd ? K2 : K1;
@@ -227,7 +250,8 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
         if (hops == 0) {
           GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
         } else {
-          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, pb[0].mine, pb[0].ld, nullptr, 0, gw, gn, st));
+          granii_gemm_epilogue ep{pre ? g->dinv_rows : nullptr, nullptr, nullptr, nullptr, nullptr};
+          GR_TRY(launch_gemm(R, K2, K1, H, ldh, a->W, K2, pb[0].mine, pb[0].ld, &ep, 0, gw, gn, st));
           GR_TRY(allgather(c, pb[0]));
           X = pb[0].all;
           ldx = pb[0].ld;
@@ -240,11 +264,11 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
         const bool last = h == hops - 1;
         GatherBuf& nb = pb[(h + 1) & 1];
         if (last && upd) {
-          GR_TRY(hop(X, ldx, K, out, ldo, relu, nullptr, 0, 0.f));
+          GR_TRY(sgc_hop(X, ldx, K, out, ldo, relu, true));
         } else if (last) {
-          GR_TRY(hop(X, ldx, K, T, ld4(K1), false, nullptr, 0, 0.f));
+          GR_TRY(sgc_hop(X, ldx, K, T, ld4(K1), false, true));
         } else {
-          GR_TRY(hop(X, ldx, K, nb.mine, nb.ld, false, nullptr, 0, 0.f));
+          GR_TRY(sgc_hop(X, ldx, K, nb.mine, nb.ld, false, false));
           GR_TRY(allgather(c, nb));
           X = nb.all;
           ldx = nb.ld;
@@ -402,12 +426,25 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
   float* hpad = nullptr;
   const bool agg_first_gather = c.dist() && (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_DYN_AGG ||
                                              comp == GRANII_GAT_RECOMP);
+  // GCN DYN_AGG: the pre-scale D̃^-½ H as its own row-broadcast pass when that moves fewer bytes
+  // than the gather-fused column scale (dyn_prescale; it rides on the gather-slot copy when
+  // partitioned)
+  DevInfo di;
+  if (dev_info(&di) != GRANII_OK) di = DevInfo();
+  const bool prescale = m == GRANII_GCN && comp == GRANII_GCN_DYN_AGG &&
+                        dyn_prescale((double)g->local_nnz, (double)R, g->avg_deg(), (double)g->n_cols, K1, di.l2_bytes);
   GatherBuf hg;
   if (agg_first_gather) {
     hg = gather_buf(b, c, K1);  // H goes into the gather slot (aligned copy); gathered by the SpMM
-    if (run) GR_TRY(launch_copy_rows(R, K1, H, ldh, hg.mine, hg.ld, st));
+    if (run && prescale) GR_TRY(launch_scale_mask(R, K1, nullptr, 0, H, ldh, g->dinv_rows, hg.mine, hg.ld, st));
+    else if (run) GR_TRY(launch_copy_rows(R, K1, H, ldh, hg.mine, hg.ld, st));
     H = hg.mine;
     ldh = hg.ld;
+  } else if (prescale) {
+    hpad = b.take((size_t)std::max<int64_t>(R, 1) * ld4(K1));
+    if (run) GR_TRY(launch_scale_mask(R, K1, nullptr, 0, a->H, a->ldh, g->dinv_rows, hpad, ld4(K1), st));
+    H = hpad;
+    ldh = ld4(K1);
   } else if (!h_aligned) {
     hpad = b.take((size_t)std::max<int64_t>(R, 1) * ld4(K1));
     if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hpad, ld4(K1), st));
@@ -436,8 +473,8 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
         if (run) {
           if (comp == GRANII_GCN_PRE_AGG)
             GR_TRY(gathered_spmm(c, xg, nval, K1, T, ldt, nullptr, nullptr, false));
-          else
-            GR_TRY(gathered_spmm(c, xg, nullptr, K1, T, ldt, g->dinv_rows, g->dinv_cols, false));
+          else  // the gathered operand is D̃^-½ H already when pre-scaled
+            GR_TRY(gathered_spmm(c, xg, nullptr, K1, T, ldt, g->dinv_rows, prescale ? nullptr : g->dinv_cols, false));
           GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw, gn, st));
         }
         break;

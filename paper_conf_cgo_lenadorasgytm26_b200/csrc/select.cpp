@@ -149,7 +149,10 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
   switch (p) {
     case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: {
       const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K, in.xcols);
-      const double idx = in.nnz * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 4.0 : 0.0)) * gb;
+      // every K slice re-streams the column ids (+ weights) and re-gathers the column scale
+      // (a dependent 4-byte gather costs a whole 32-byte L2 sector)
+      const double sl = (double)spmm_slices(in.avg, in.xcols, (int64_t)K, (int64_t)in.l2);
+      const double idx = in.nnz * sl * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 32.0 : 0.0)) * gb;
       return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3};
     }
     case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb, in.R * 1e-6};
@@ -240,7 +243,9 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
       return cost(m, in, P_SDDMM1, 0) + agg_cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_PRE_UPD:
       return cost(m, in, P_SDDMM1, 0) + cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_W, K2);
-    case GRANII_GCN_DYN_AGG:
+    case GRANII_GCN_DYN_AGG:  // pre-scale fused in the gather, or its own row-broadcast pass (layer.cu)
+      if (dyn_prescale(in.nnz, in.R, in.avg, in.xcols, (int64_t)K1, (int64_t)in.l2))
+        return cost(m, in, P_ELEMENTWISE, K1) + agg_cost(m, in, P_SPMM_U, K1) + cost(m, in, P_GEMM, K1, K2);
       return agg_cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
     case GRANII_GCN_DYN_UPD:
       return cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_U, K2);
@@ -260,10 +265,14 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
 double ext_forward_cost(const CostModel& m, const In& in, int comp, double K1, double K2, double k, double Kh) {
   const bool dyn = (comp & 3) >= 2, upd = (comp & 1) != 0;
   const int base = comp & ~3;
-  const int sp = base == GRANII_GIN_PRE_AGG ? (dyn ? P_SPMM_U : P_SPMM_W) : (dyn ? P_SPMM_U_CS : P_SPMM_W);
+  int sp = base == GRANII_GIN_PRE_AGG ? (dyn ? P_SPMM_U : P_SPMM_W) : (dyn ? P_SPMM_U_CS : P_SPMM_W);
   double t = dyn ? 0.0 : cost(m, in, P_SDDMM1, 0);
   if (base == GRANII_SGC_PRE_AGG) {
     const double K = upd ? K2 : K1;
+    if (dyn && k > 0 && dyn_prescale(in.nnz, in.R, in.avg, in.xcols, (int64_t)K, (int64_t)in.l2)) {
+      sp = P_SPMM_U;                               // pre-scaled hop inputs (layer.cu sgc_hop)
+      if (!upd) t += cost(m, in, P_ELEMENTWISE, K1);  // UPD: fused in the GEMM epilogue
+    }
     t += cost(m, in, P_GEMM, K1, K2) + k * (cost(m, in, P_ALLGATHER, K) + cost(m, in, sp, K));
   } else if (base == GRANII_TAGCN_PRE_AGG) {
     if (upd)

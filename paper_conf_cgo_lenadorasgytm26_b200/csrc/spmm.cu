@@ -64,6 +64,7 @@ struct SpmmArgs {
   const float* __restrict__ cs;
   int relu;
   const int32_t* __restrict__ order;       // light rows, degree-descending
+  int64_t n_lwide;                         // group-per-row kernel: order[0 .. n_lwide) get a warp each
   // heavy rows (degree > GRANII_SEG) are cut into segments: warp-wide work items whose
   // unscaled partial sums go to `partial` [n_seg][ldp] and are combined in fixed order
   int64_t n_seg;
@@ -241,6 +242,32 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
   if (grp == 0) store_row<LPG>(part, colok, acc, 1.f, 0);
 }
 
+// one row, the whole warp: G lane groups share its entries
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U>
+__device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lane, int grp, int lig,
+                                         const bool (&colok)[NJ], const char* const (&xbj)[NJ], uint32_t row_bytes) {
+    float acc[NJ][VEC];
+    zero(acc);
+    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+    if constexpr (PH) {
+      if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
+      for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
+        int64_t lo, hi;
+        phase_part(a, row, r, 0, INT64_MAX, lo, hi);
+        warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
+      }
+    } else {
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
+    }
+    reduce_groups<LPG>(acc);
+    if (grp == 0) {
+      if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
+      else
+        store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
+                       a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+    }
+}
+
 // ------------------------------------------------------------------ warp-per-row
 // defaults (tools/spmm_sweep.py on B200, Reddit- and products-shaped graphs): 16-byte gathers of
 // <= 2 vectors per lane keep 2 neighbours per group in flight at 4 blocks/SM (64 registers);
@@ -267,27 +294,7 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k
       do_segment<VEC, LPG, NJ, W, CS, PH, U>(a, t, lane, grp, lig, colok, xbj, row_bytes);
       continue;
     }
-    const int64_t row = a.order[t - a.n_seg];
-    float acc[NJ][VEC];
-    zero(acc);
-    float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
-    if constexpr (PH) {
-      if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
-      for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
-        int64_t lo, hi;
-        phase_part(a, row, r, 0, INT64_MAX, lo, hi);
-        warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
-      }
-    } else {
-      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
-    }
-    reduce_groups<LPG>(acc);
-    if (grp == 0) {
-      if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
-      else
-        store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
-                       a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
-    }
+    warp_row<VEC, LPG, NJ, W, CS, PH, U>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
   }
 }
 
@@ -304,10 +311,13 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   const char* xbj[NJ];
   slice_setup<VEC, LPG>(a, lig, colok, xbj);
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
-  for (int64_t t = warp; t < a.n_seg; t += nwarps)  // heavy segments: whole warps
-    do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
-  // light rows: one LPG-lane group per row
-  for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
+  // heavy segments, then the wide light rows (degree > wide_deg): whole warps, largest first
+  for (int64_t t = warp; t < a.n_seg + a.n_lwide; t += nwarps) {
+    if (t < a.n_seg) do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+    else warp_row<VEC, LPG, NJ, W, CS, PH, UW>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
+  }
+  // the other light rows: one LPG-lane group per row
+  for (int64_t t0 = a.n_lwide + warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
     const int64_t row = a.order[t];
@@ -379,7 +389,7 @@ __global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heav
 template <int VEC, int LPG, int NJ, bool PH>
 static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool cs, int sms, cudaStream_t st) {
   const int threads = 256;
-  int64_t units = (warp_mode ? a.n_rows : ceil_div(a.n_rows, 32 / LPG)) + a.n_seg;
+  int64_t units = (warp_mode ? a.n_rows : a.n_lwide + ceil_div(a.n_rows - a.n_lwide, 32 / LPG)) + a.n_seg;
   // enough warps for 8 resident blocks/SM, capped by the work available
   int64_t blocks = std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 8);
   blocks = std::max<int64_t>(blocks, 1);
@@ -453,6 +463,25 @@ static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, 
 
 // cols: rows of X the launch gathers from (the whole column space, or one owner block of a
 // phased aggregation, whose footprint is 1/G of it)
+// K slices of a vec4 SpMM over `cols` gathered rows (the automatic rule of spmm_slice_width)
+int64_t spmm_slices(double avg_deg, double cols, int64_t K, int64_t l2_bytes) {
+  int64_t kw = std::min<int64_t>(K, 1024);
+  const double per_col = cols * 4.0;
+  if (avg_deg >= 32.0 && per_col * (double)K > 0.6 * (double)l2_bytes) {
+    const int64_t fit = (int64_t)(0.55 * (double)l2_bytes / per_col) / 64 * 64;
+    if (fit >= 64) kw = std::min(kw, round_up(ceil_div(K, ceil_div(K, fit)), 64));
+  }
+  return ceil_div(K, std::max<int64_t>(kw, 1));
+}
+
+// Dynamic normalisation (Eq. 2): the pre-scale D̃^-½ of the aggregated operand is fused into the
+// SpMM gather (one dependent 4-byte gather -- a whole L2 sector -- per entry and K slice) unless
+// a separate row-broadcast pass (read + write N x K floats once) moves fewer bytes: dense graphs
+// whose SpMM is K-sliced (Reddit 602 -> 1024: 10 slices x 118 M entries x 32 B vs 1.1 GB)
+bool dyn_prescale(double nnz, double rows, double avg_deg, double cols, int64_t K, int64_t l2_bytes) {
+  return nnz * 32.0 * (double)spmm_slices(avg_deg, cols, K, l2_bytes) > rows * (double)K * 8.0;
+}
+
 int64_t spmm_slice_width(const granii_graph_s* g, int64_t K, bool vec4, int64_t l2_bytes, int64_t cols) {
   // Keep the gathered column slice of X resident in L2: split
   // K into slices whose X footprint is <= ~45% of L2 when the graph is dense
@@ -492,7 +521,8 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   const float share = ph ? float(ph->p1 - ph->p0 - (ph->skip >= 0 ? 1 : 0)) / float(g->world) : 1.f;
   const bool warp_mode = g->avg_deg() * share >= 16.f;
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
-             g->order + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, nullptr, 0, B, ldb, beta};
+             g->order + g->n_heavy, std::max<int64_t>(0, g->n_wide - g->n_heavy), g->n_seg, g->seg_lo, g->seg_hi,
+             nullptr, 0, B, ldb, beta};
   // phases slice like the whole aggregation: the 64-wide slices also keep the L1 hit rate
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes, g->n_cols);
   float* partial = nullptr;  // heavy-segment partials: this slice's columns start at partial + pk0

@@ -585,3 +585,15 @@ def test_softmax_xent_and_sgd(G):
     G.granii_sgd(gr, w, 0.5)
     torch.cuda.synchronize()
     assert torch.equal(w.cpu(), 1 - 0.5 * torch.arange(100, dtype=torch.float32))
+
+
+def test_select_candidates_are_the_offline_promoted_trees(G):
+    """N4: the online selector's candidate sets (prefilter on, L237-L239) are exactly the trees
+    the offline stage (offline.py, Algorithm 1 + pruning) promotes for each scenario"""
+    from paper_conf_cgo_lenadorasgytm26_b200 import offline as OF
+    c = case(G, "pubmed")
+    for model, name in ((G.GCN, "gcn"), (G.GAT, "gat")):
+        prom = OF.promoted_compositions(name)
+        for K1, K2, scen in ((256, 32, ">="), (64, 64, ">="), (32, 256, "<")):
+            _, pred = G.granii_select(c.g, model, K1, K2)
+            assert set(pred) == {cid for cid, sc in prom.items() if scen in sc}, (name, K1, K2)

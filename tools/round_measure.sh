@@ -1,14 +1,24 @@
 #!/bin/bash
-# one GPU session: calibration, every workload with regret, the default bench line, ncu evidence
+# one GPU session: calibration, every workload with regret, the regret sweep, the default bench line,
+# scaling projections, ncu evidence
 set -u
-mkdir -p gpurun_out/m
-timeout 900 python tools/calibrate.py --out calib/b200.txt > gpurun_out/m/calib.log 2>&1; cp calib/b200.txt calib/b200_samples.json gpurun_out/m/ 2>/dev/null
-for wl in reddit-gcn2-train reddit-gcn2-train-h32 reddit-gcn2-train-h1024 products-gcn2-infer products-gat2-infer arxiv-gat-infer pubmed-gcn2-train; do
-  timeout 600 python bench.py --workload $wl --steps 10 --warmup 3 --no-e2e --no-cpu --out gpurun_out/m/bench_$wl.json > gpurun_out/m/bench_$wl.log 2>&1
+M=gpurun_out/m
+mkdir -p $M
+timeout 1500 python -m pytest tests -m gpu -x -q > $M/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 $M/pytest_gpu.log
+timeout 1200 python tools/calibrate.py --out calib/b200.txt > $M/calib.log 2>&1; echo "calib rc=$?"
+cp calib/b200.txt calib/b200_samples.json $M/ 2>/dev/null
+for wl in reddit-gcn2-train reddit-gcn2-train-h32 reddit-gcn2-train-h1024 products-gcn2-infer products-gat2-infer products-gat2-train arxiv-gat-infer pubmed-gcn2-train pubmed-gat2-train reddit-sgc-infer reddit-tagcn-infer reddit-gin-infer products-sgc-infer; do
+  timeout 600 python bench.py --workload $wl --steps 10 --warmup 3 --no-e2e --no-cpu --out $M/bench_$wl.json > $M/bench_$wl.log 2>&1
   echo "$wl rc=$?"
 done
-timeout 900 python bench.py --steps 20 --warmup 5 --out gpurun_out/m/bench_default.json > gpurun_out/m/bench_default.log 2>&1; echo "default rc=$?"
+timeout 1500 python tools/regret_sweep.py $M/regret_sweep.json > $M/regret_sweep.log 2>&1; echo "regret sweep rc=$?"
+timeout 900 python bench.py --steps 20 --warmup 5 --out $M/bench_default.json > $M/bench_default.log 2>&1; echo "default rc=$?"
+for wl in reddit-gcn2-train products-gcn2-infer products-gat2-infer; do
+  timeout 600 python tools/scaling_projection.py --workload $wl --out $M/scaling_projection_$wl.json > $M/proj_$wl.log 2>&1; echo "proj $wl rc=$?"
+done
 B="python bench.py --steps 2 --warmup 3 --no-e2e --no-regret --no-cpu --cuda-graph off"
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/m/launches.csv $B > /dev/null 2>&1; echo "ncu launches rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm_warp -s 20 -c 5 -o gpurun_out/m/spmm_full $B > /dev/null 2>&1; echo "ncu spmm rc=$?"
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_gemm -s 4 -c 3 -o gpurun_out/m/gemm_full $B > /dev/null 2>&1; echo "ncu gemm rc=$?"
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $M/launches.csv $B > /dev/null 2>&1; echo "ncu launches rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm_warp -s 20 -c 5 -o $M/spmm_full $B > /dev/null 2>&1; echo "ncu spmm rc=$?"
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_gemm -s 4 -c 3 -o $M/gemm_full $B > /dev/null 2>&1; echo "ncu gemm rc=$?"
+for r in spmm_full gemm_full; do [ -f $M/$r.ncu-rep ] && python tools/ncu_summary.py $M/$r.ncu-rep > $M/${r}_summary.json; done
+ls $M
