@@ -339,6 +339,15 @@ def main():
                 "peak_note": f"hbm_gbs of {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}
     roof["frac"] = roof["achieved"] / roof["peak"]
     roof["traffic"] = traffic
+    if traffic and roof["bound"] == "hbm":  # what DRAM actually moved per launch (ncu) over the launch time
+        roof["dram_gbs_from_traffic"] = traffic / (kst["ms"] / max(kst["calls"], 1) / 1e3) / 1e9
+        roof["dram_frac"] = roof["dram_gbs_from_traffic"] / hbm
+    lp = os.path.join(ROOT, "profiles", "l2_peak.json")
+    if roof["bound"] == "hbm" and os.path.exists(lp):
+        # gathers served by L2: the algorithmic bytes against the measured L2 read peak
+        l2 = json.load(open(lp))["l2_read_gbs"]
+        roof["l2"] = {"peak": l2, "frac": achieved / l2, "note": "algorithmic bytes / measured L2 read bandwidth "
+                      "(profiles/l2_peak.json, tools/probe/l2_bw.cu); L1 hits can push it past 1"}
     roof["kernel"] = kname
     roof["share_of_step"] = share
     roof["algorithmic_bytes_per_launch"] = per_launch_bytes

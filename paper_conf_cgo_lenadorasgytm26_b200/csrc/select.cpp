@@ -36,8 +36,9 @@ struct CostModel {
 };
 
 // feature vectors (all sizes in GB / TFLOP / millions, time in ms)
-//   spmm            : [1, streamed GB (idx, weights, col-scale gather), out GB, gathered GB from L2,
-//                      gathered GB from HBM, M rows, thousands of hub segments]
+//   spmm            : [1, streamed GB (idx, weights; per K slice), out GB, gathered GB from L2,
+//                      gathered GB from HBM, M rows, thousands of hub segments,
+//                      G column-scale gathers (one dependent 4-byte gather per entry and K slice)]
 //   sddmm1          : [1, streamed GB, M rows]
 //   sddmm1_softmax  : [1, streamed GB, M rows]
 //   gemm            : [1, HBM GB, TFLOP, thousands of 128x128 tiles]
@@ -50,7 +51,7 @@ struct CostModel {
 //                     slope is an assumed NCCL bus bandwidth of 0.65 TB/s on NVLink 5)
 static CostModel defaults() {
   CostModel m;
-  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0};
+  m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0, 1.0};
   m.coef["sddmm1"] = {0.005, 1.0 / 5.5, 0.0};
   m.coef["sddmm1_softmax"] = {0.006, 1.0 / 4.0, 0.0};
   m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0};
@@ -152,8 +153,9 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
       // every K slice re-streams the column ids (+ weights) and re-gathers the column scale
       // (a dependent 4-byte gather costs a whole 32-byte L2 sector)
       const double sl = (double)spmm_slices(in.avg, in.xcols, (int64_t)K, (int64_t)in.l2);
-      const double idx = in.nnz * sl * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0) + (p == P_SPMM_U_CS ? 32.0 : 0.0)) * gb;
-      return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3};
+      const double idx = in.nnz * sl * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0)) * gb;
+      return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3,
+              p == P_SPMM_U_CS ? in.nnz * sl * 1e-9 : 0.0};
     }
     case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb, in.R * 1e-6};
     case P_SDDMM1_SM: return {1.0, in.nnz * 16.0 * gb, in.R * 1e-6};

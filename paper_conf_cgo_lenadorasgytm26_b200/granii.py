@@ -332,7 +332,7 @@ P_SPMM_W, P_SPMM_U, P_SPMM_U_CS, P_SDDMM1, P_SDDMM1_SM, P_GEMM, P_GEMM_NOSTORE, 
 
 
 def granii_cost_features(g: Graph, prim: int, K1: int, K2: int = 0):
-    f = (ctypes.c_double * 8)()
+    f = (ctypes.c_double * 16)()
     n = _i32()
     name = ctypes.create_string_buffer(32)
     _check(_lib.granii_cost_features(g.handle, prim, K1, K2, f, ctypes.byref(n), name), "granii_cost_features")
