@@ -422,8 +422,8 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   const double bytes = pass == 0 ? nnz * (8.0 + 4.0 * K) + R * (4.0 * K + 8.0 + 28.0)
                                  : nnz * (20.0 + 4.0 * K) + R * (8.0 * K + 8.0 + 16.0);
   ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1);
-  // lane-group width: 8 lanes x NJ float4 up to K = 128 (4 groups, more rows in flight),
-  // full-warp groups beyond
+  // lane-group width (tools/gatbwd_sweep.py on the products-shaped graph): 8 lanes x NJ float4
+  // up to K = 64 (4 groups per warp), 16 lanes up to 256, full-warp groups beyond
   // dense graphs (avg degree >= 16): a warp per row; sparse: a lane group per row, the wide
   // rows (degree > g->wide_deg) a warp each
   GatBwdArgs b = a;
@@ -440,6 +440,15 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
       else if (l == 16 && n == 2 && u == 2) gb_launch<16, 2, 2>(pass, b, st);
       else if (l == 32 && n == 1 && u == 4) gb_launch<32, 1, 4>(pass, b, st);
       else if (l == 32 && n == 1 && u == 2) gb_launch<32, 1, 2>(pass, b, st);
+      else if (l == 8 && n == 4 && u == 2) gb_launch<8, 4, 2>(pass, b, st);
+      else if (l == 16 && n == 4 && u == 2) gb_launch<16, 4, 2>(pass, b, st);
+      else if (l == 32 && n == 2 && u == 2) gb_launch<32, 2, 2>(pass, b, st);
+      else if (l == 32 && n == 2 && u == 1) gb_launch<32, 2, 1>(pass, b, st);
+      else if (l == 16 && n == 4 && u == 1) gb_launch<16, 4, 1>(pass, b, st);
+      else if (l == 32 && n == 4 && u == 2) gb_launch<32, 4, 2>(pass, b, st);
+      else if (l == 32 && n == 4 && u == 1) gb_launch<32, 4, 1>(pass, b, st);
+      else if (l == 16 && n == 8 && u == 1) gb_launch<16, 8, 1>(pass, b, st);
+      else if (l == 32 && n == 8 && u == 1) gb_launch<32, 8, 1>(pass, b, st);
       else ok = false;
       if (ok) {
         GR_CHECK_LAUNCH();
@@ -450,9 +459,16 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   if (K <= 16) gb_launch<4, 1, 4>(pass, b, st);
   else if (K <= 32) gb_launch<8, 1, 4>(pass, b, st);
   else if (K <= 64) gb_launch<8, 2, 2>(pass, b, st);
-  else if (K <= 128) gb_launch<8, 4, 2>(pass, b, st);
-  else if (K <= 256) gb_launch<16, 4, 2>(pass, b, st);
-  else if (K <= 512) gb_launch<32, 4, 2>(pass, b, st);
+  else if (K <= 128) gb_launch<16, 2, 2>(pass, b, st);  // products K=100: A 10.9 -> 9.8, B 13.0 -> 10.5 ms vs <8,4,2>
+  // pass A keeps one entry per group in flight beyond K = 128 (its online-softmax state is
+  // per entry): products K=256 18.8 -> 18.3 ms, K=512 39.1 -> 35.2 ms; pass B keeps two
+  else if (K <= 256) {
+    if (pass == 0) gb_launch<32, 2, 1>(pass, b, st);
+    else gb_launch<16, 4, 2>(pass, b, st);
+  } else if (K <= 512) {
+    if (pass == 0) gb_launch<32, 4, 1>(pass, b, st);
+    else gb_launch<32, 4, 2>(pass, b, st);
+  }
   else if (K <= 1024) gb_launch<32, 8, 1>(pass, b, st);
   else gb_launch<32, 16, 1>(pass, b, st);
   GR_CHECK_LAUNCH();
