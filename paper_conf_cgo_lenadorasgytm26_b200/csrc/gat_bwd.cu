@@ -96,11 +96,12 @@ __global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, 
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
 template <int LPG, int NJ, int U>
-__device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane) {
+__device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lg = lane % LPG, grp = lane / LPG;
-  const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
+  // a whole row, or (seg >= 0) one hub segment of it, whose online-softmax state goes to seg_a
+  const int64_t b = seg >= 0 ? a.seg_lo[seg] : a.row_ptr[r], t = seg >= 0 ? a.seg_hi[seg] : a.row_ptr[r + 1];
   const float eli = a.el[r];
   const float ci = a.c[r];
   float xv[NJ][4];
@@ -163,6 +164,10 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
     D = D * f1 + D2 * f2;
     m = mn;
   }
+  if (seg >= 0) {
+    if (lane == 0) a.seg_a[seg] = make_float4(m, S, Cw, D);
+    return;
+  }
   const float inv_s = S > 0.f ? 1.f / S : 0.f;
   if (lane == 0) {
     a.del[r] = (D - ci * Cw) * inv_s;
@@ -171,11 +176,12 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
 }
 
 template <int LPG, int NJ, int U>
-__device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, int lane) {
+__device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
   const int lg = lane % LPG, grp = lane / LPG;
-  const int64_t b = a.row_ptr[r], t = a.row_ptr[r + 1];
+  // a whole row, or (seg >= 0) one hub segment of it, whose partial sums go to seg_b / seg_der
+  const int64_t b = seg >= 0 ? a.seg_lo[seg] : a.row_ptr[r], t = seg >= 0 ? a.seg_hi[seg] : a.row_ptr[r + 1];
   const float erj = a.er[r];
   float zr[NJ][4], acc[NJ][4];
   gb_load_row<LPG, NJ>(a.Z + (int64_t)r * a.ldz, lg, a.K, zr);
@@ -224,6 +230,18 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
 #pragma unroll
       for (int k = 0; k < 4; ++k) acc[j][k] += __shfl_xor_sync(0xffffffffu, acc[j][k], o);
   const float der = gb_warp_sum(dpart) - gb_warp_sum(dcorr);
+  if (seg >= 0) {
+    if (grp == 0) {
+      float* o = a.seg_b + seg * a.ldp;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int64_t col = 4 * (int64_t)(lg + j * LPG);
+        if (col < a.K) *reinterpret_cast<float4*>(o + col) = make_float4(acc[j][0], acc[j][1], acc[j][2], acc[j][3]);
+      }
+    }
+    if (lane == 0) a.seg_der[seg] = der;
+    return;
+  }
   const float delj = a.del_in[r];
   if (grp == 0) {
     float* o = a.out + (int64_t)r * a.ldo;
@@ -378,8 +396,15 @@ __global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (w < a.n_wide) gat_a_warp_row<LPG, NJ, U>(a, a.order[w], lane);
-  else gat_a_group_row<LPG, NJ, U>(a, a.n_wide + (w - a.n_wide) * G + lane / LPG, lane);
+  // hub segments first (warp-wide items, largest rows first), then the wide rows (a warp each),
+  // then lane groups; one call site per schedule keeps the unrolled body inlined once
+  const int64_t wr = w - a.n_seg;
+  if (wr >= a.n_wide) {
+    gat_a_group_row<LPG, NJ, U>(a, a.n_wide + (wr - a.n_wide) * G + lane / LPG, lane);
+    return;
+  }
+  const bool sg = w < a.n_seg;
+  gat_a_warp_row<LPG, NJ, U>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
 }
 
 template <int LPG, int NJ, int U>
@@ -387,14 +412,57 @@ __global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bw
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  if (w < a.n_wide) gat_b_warp_row<LPG, NJ, U>(a, a.order[w], lane);
-  else gat_b_group_row<LPG, NJ, U>(a, a.n_wide + (w - a.n_wide) * G + lane / LPG, lane);
+  // hub segments first (warp-wide items, largest rows first), then the wide rows (a warp each),
+  // then lane groups; one call site per schedule keeps the unrolled body inlined once
+  const int64_t wr = w - a.n_seg;
+  if (wr >= a.n_wide) {
+    gat_b_group_row<LPG, NJ, U>(a, a.n_wide + (wr - a.n_wide) * G + lane / LPG, lane);
+    return;
+  }
+  const bool sg = w < a.n_seg;
+  gat_b_warp_row<LPG, NJ, U>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
+}
+
+// hub rows: merge the segments' online-softmax states in fixed order -> del and the row record
+__global__ void k_gat_a_combine(GatBwdArgs a) {
+  for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < a.n_heavy; h += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = a.heavy_rows[h];
+    float m = -INFINITY, S = 0.f, Cw = 0.f, D = 0.f;
+    for (int32_t q = a.seg_ptr[h]; q < a.seg_ptr[h + 1]; ++q) {
+      const float4 v = a.seg_a[q];
+      const float mn = fmaxf(m, v.x);
+      const float f1 = m == -INFINITY ? 0.f : __expf(m - mn), f2 = v.x == -INFINITY ? 0.f : __expf(v.x - mn);
+      S = S * f1 + v.y * f2;
+      Cw = Cw * f1 + v.z * f2;
+      D = D * f1 + v.w * f2;
+      m = mn;
+    }
+    const float ci = a.c[r], inv_s = S > 0.f ? 1.f / S : 0.f;
+    a.del[r] = (D - ci * Cw) * inv_s;
+    *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(a.el[r], m, inv_s, ci);
+  }
+}
+
+// hub rows: out_r = sum of the segments' partial rows (fixed order) + del_r u + der_r v
+__global__ void k_gat_b_combine(GatBwdArgs a) {
+  const int64_t total = a.n_heavy * a.K;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t h = i / a.K, k = i % a.K;
+    const int32_t r = a.heavy_rows[h];
+    float acc = 0.f, der = 0.f;
+    for (int32_t q = a.seg_ptr[h]; q < a.seg_ptr[h + 1]; ++q) {
+      acc += a.seg_b[(int64_t)q * a.ldp + k];
+      der += a.seg_der[q];
+    }
+    a.out[(int64_t)r * a.ldo + k] = acc + a.del_in[r] * a.u[k] + der * a.v[k];
+    if (k == 0) a.der[r] = der;
+  }
 }
 
 template <int LPG, int NJ, int U>
 static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
   constexpr int G = 32 / LPG;
-  const int64_t warps = a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
+  const int64_t warps = a.n_seg + a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
   const unsigned blocks = (unsigned)std::max<int64_t>(1, ceil_div(warps, 8));
   if (pass == 0)
     k_gat_bwd_a<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
@@ -412,6 +480,8 @@ granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ld
   return GRANII_OK;
 }
 
+static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cudaStream_t st);
+
 granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBwdArgs& a, cudaStream_t st) {
   if (a.n_rows == 0) return GRANII_OK;
   const int64_t K = a.K;
@@ -427,7 +497,51 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   // dense graphs (avg degree >= 16): a warp per row; sparse: a lane group per row, the wide
   // rows (degree > g->wide_deg) a warp each
   GatBwdArgs b = a;
-  b.n_wide = g->avg_deg() >= 16.f ? a.n_rows : std::min<int64_t>(g->n_wide, a.n_rows);
+  const bool dense = g->avg_deg() >= 16.f;
+  b.n_wide = dense ? a.n_rows : std::min<int64_t>(g->n_wide, a.n_rows);
+  // group-per-row graphs: hub rows (degree > seg_len, order[0 .. n_heavy)) are cut into the graph's
+  // warp-wide segments (a 655-entry pubmed hub was a 160-step serial tail at K=256: pass A 0.143 ->
+  // 0.073 ms, B 0.101 -> 0.054); on warp-per-row graphs the hubs start first and finish inside
+  // the pass (products: no gain), so they stay whole.  GRANII_GATBWD_SEG=0/1 forces either.
+  const char* se = getenv("GRANII_GATBWD_SEG");
+  const bool use_seg = se ? se[0] != '0' : !dense;
+  const int64_t nh = (a.n_rows == g->n_rows && use_seg) ? g->n_heavy : 0;
+  float* scratch = nullptr;
+  if (nh > 0) {
+    b.n_seg = g->n_seg;
+    b.seg_lo = g->seg_lo;
+    b.seg_hi = g->seg_hi;
+    b.seg_row = g->seg_row;
+    b.seg_ptr = g->seg_ptr;
+    b.heavy_rows = g->order;
+    b.n_heavy = nh;
+    b.order = a.order + nh;
+    b.n_rows = a.n_rows - nh;
+    b.n_wide = std::max<int64_t>(0, b.n_wide - nh);
+    b.ldp = round_up(K, 4);
+    const size_t fl = pass == 0 ? (size_t)g->n_seg * 4 : (size_t)g->n_seg * (b.ldp + 1);
+    GR_CUDA(cudaMallocAsync((void**)&scratch, fl * sizeof(float), st));
+    if (pass == 0) b.seg_a = reinterpret_cast<float4*>(scratch);
+    else {
+      b.seg_b = scratch;
+      b.seg_der = scratch + (size_t)g->n_seg * b.ldp;
+    }
+  }
+  granii_status rs = gb_dispatch(pass, b, dense, st);
+  if (rs == GRANII_OK && nh > 0) {
+    if (pass == 0)
+      k_gat_a_combine<<<(unsigned)ceil_div(nh, 128), 128, 0, st>>>(b);
+    else
+      k_gat_b_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(nh * K, 256), 4096)), 256, 0, st>>>(b);
+    GR_CHECK_LAUNCH();
+    ps.add_launches(1);
+  }
+  if (scratch) GR_CUDA(cudaFreeAsync(scratch, st));
+  return rs;
+}
+
+static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cudaStream_t st) {
+  const int64_t K = b.K;
   // tuning hook GRANII_GATBWD="LPG,NJ,U" (tools: bench.py per_primitive_ms), if it covers K
   if (const char* e = getenv("GRANII_GATBWD")) {
     int l = 0, n = 0, u = 0;
@@ -459,14 +573,18 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   if (K <= 16) gb_launch<4, 1, 4>(pass, b, st);
   else if (K <= 32) gb_launch<8, 1, 4>(pass, b, st);
   else if (K <= 64) gb_launch<8, 2, 2>(pass, b, st);
-  else if (K <= 128) gb_launch<16, 2, 2>(pass, b, st);  // products K=100: A 10.9 -> 9.8, B 13.0 -> 10.5 ms vs <8,4,2>
-  // pass A keeps one entry per group in flight beyond K = 128 (its online-softmax state is
-  // per entry): products K=256 18.8 -> 18.3 ms, K=512 39.1 -> 35.2 ms; pass B keeps two
-  else if (K <= 256) {
-    if (pass == 0) gb_launch<32, 2, 1>(pass, b, st);
+  // warp-per-row graphs (products-shaped sweep): 16-lane groups up to K = 128 (K=100: A 10.9 -> 9.8,
+  // B 13.0 -> 10.5 ms vs <8,4,2>); pass A keeps one entry per group in flight beyond K = 128 (K=256
+  // 18.8 -> 18.3 ms, K=512 39.1 -> 35.2 ms).  Group-per-row graphs keep more rows per warp (pubmed-
+  // shaped K=256: <32,2,1> for pass A cost 0.19 -> 0.25 ms)
+  else if (K <= 128) {
+    if (dense) gb_launch<16, 2, 2>(pass, b, st);
+    else gb_launch<8, 4, 2>(pass, b, st);
+  } else if (K <= 256) {
+    if (pass == 0 && dense) gb_launch<32, 2, 1>(pass, b, st);
     else gb_launch<16, 4, 2>(pass, b, st);
   } else if (K <= 512) {
-    if (pass == 0) gb_launch<32, 4, 1>(pass, b, st);
+    if (pass == 0 && dense) gb_launch<32, 4, 1>(pass, b, st);
     else gb_launch<32, 4, 2>(pass, b, st);
   }
   else if (K <= 1024) gb_launch<32, 8, 1>(pass, b, st);

@@ -122,6 +122,13 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
 granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                              float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                              int64_t ldb, float beta, cudaStream_t st);
+// GAT aggregation with the additive attention fused (Eq. 4-6): Y_i = act(rs_i * sum_e alpha_e X_c(e)),
+// alpha = row softmax of LeakyReLU(el_i + er_c) computed on the fly (online max / sum per row, no
+// SDDMM pass, no alpha array); warp-per-row graphs (spmm_att_supported), single GPU
+bool spmm_att_supported(const granii_graph_s* g);
+bool gat_fused_enabled();  // GRANII_GAT_FUSED != 0
+granii_status launch_spmm_att(const granii_graph_s* g, const float* el, const float* er, const float* X, int64_t ldx,
+                              int64_t K, float* Y, int64_t ldy, const float* rs, bool relu, cudaStream_t st);
 // one phase of a block-phased aggregation over a partitioned graph (layer.cu gathered_spmm):
 // the entries whose column lies in the gather blocks [p0, p1), block `skip` excluded (-1: none);
 // partial = heavy-segment scratch [n_seg][round_up(K,4)] kept across the phases (NULL if the
@@ -178,6 +185,17 @@ struct GatBwdArgs {
   int64_t ldo = 0;
   int vec_store = 0;
   int64_t n_wide = 0;         // order[0 .. n_wide): a warp per row; the rest: a lane group per row
+  // hub segments (set by launch_gat_bwd_pass from the graph): warp-wide items scheduled first,
+  // merged per heavy row (heavy_rows[0 .. n_heavy)) in fixed order by a combine kernel
+  int64_t n_seg = 0, n_heavy = 0, ldp = 0;
+  const int64_t* seg_lo = nullptr;
+  const int64_t* seg_hi = nullptr;
+  const int32_t* seg_row = nullptr;
+  const int32_t* seg_ptr = nullptr;
+  const int32_t* heavy_rows = nullptr;
+  float4* seg_a = nullptr;    // pass 0: online-softmax state {m, S, Cw, D} per segment
+  float* seg_b = nullptr;     // pass 1: partial output row per segment (ld ldp)
+  float* seg_der = nullptr;   // pass 1: partial der per segment
 };
 granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
                               bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st);

@@ -94,6 +94,11 @@ static bool overlap_enabled() {
   return !(e && e[0] == '0');
 }
 
+bool gat_fused_enabled() {
+  const char* e = getenv("GRANII_GAT_FUSED");
+  return !(e && e[0] == '0');
+}
+
 static granii_status gathered_spmm(const Ctx& c, GatherBuf& gb, const float* vals, int64_t K, float* Y, int64_t ldy,
                                    const float* rs, const float* cs, bool relu, const float* B = nullptr,
                                    int64_t ldb = 0, float beta = 0.f) {
@@ -503,7 +508,12 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     if (comp != GRANII_GAT_REUSE && comp != GRANII_GAT_RECOMP)
       return fail(GRANII_ERR_INVALID_ARG, "composition does not belong to GAT");
     const bool dot = a->attn == GRANII_ATTN_DOT;
-    float* alpha = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
+    // additive attention on one GPU over a warp-per-row graph: the scores, the row softmax and the
+    // aggregation are one fused SpMM (no SDDMM pass, no alpha array); GRANII_GAT_FUSED=0 disables
+    const bool out_aligned = (ldo % 4 == 0) && (((uintptr_t)out & 15) == 0);  // REUSE aggregates into out
+    const bool fused = !dot && !c.dist() && spmm_att_supported(g) && gat_fused_enabled() &&
+                       (comp == GRANII_GAT_RECOMP || out_aligned);
+    float* alpha = fused ? nullptr : b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
     const bool need_theta = comp == GRANII_GAT_REUSE || dot;
     // state kept for the backward (gat_saved_layout): Θ (REUSE) or T = α H (RECOMP), el, er
     const GatSaved sv = gat_saved_layout(R, comp, K1, K2);
@@ -545,8 +555,9 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
           GR_TRY(comm_allgather(c.comm, er_mine, er_all, (size_t)g->max_rows, st));
           (void)eb;
         }
-        GR_TRY(launch_sddmm(g, GRANII_SDDMM_ADD | GRANII_SDDMM_LEAKYRELU | GRANII_SDDMM_ROW_SOFTMAX, el, 1, er_all,
-                            1, 1, 1.f, alpha, st));
+        if (!fused)
+          GR_TRY(launch_sddmm(g, GRANII_SDDMM_ADD | GRANII_SDDMM_LEAKYRELU | GRANII_SDDMM_ROW_SOFTMAX, el, 1, er_all,
+                              1, 1, 1.f, alpha, st));
       } else {
         GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT | GRANII_SDDMM_ROW_SOFTMAX, th.mine, th.ld, th.all, th.ld, K2,
                             1.f / std::sqrt((float)K2), alpha, st));
@@ -555,6 +566,7 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     if (comp == GRANII_GAT_REUSE) {
       if (run) {
         if (dot) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
+        else if (fused) GR_TRY(launch_spmm_att(g, el, er_all, th.all, th.ld, K2, out, ldo, nullptr, relu, st));
         else GR_TRY(gathered_spmm(c, th, alpha, K2, out, ldo, nullptr, nullptr, relu));
       }
     } else {
@@ -564,7 +576,8 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       size_t gn2;
       gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
       if (run) {
-        GR_TRY(gathered_spmm(c, xg, alpha, K1, T, ldt, nullptr, nullptr, false));
+        if (fused) GR_TRY(launch_spmm_att(g, el, er_all, xg.all, xg.ld, K1, T, ldt, nullptr, false, st));
+        else GR_TRY(gathered_spmm(c, xg, alpha, K1, T, ldt, nullptr, nullptr, false));
         GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
                            st));
       }

@@ -252,9 +252,15 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
     case GRANII_GCN_DYN_UPD:
       return cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_U, K2);
     case GRANII_GAT_REUSE:
+      // one GPU, warp-per-row graph: scores + softmax fused into the aggregation (layer.cu), whose
+      // per-entry er gather is modelled like the column-scale gather of the unweighted SpMM
+      if (in.world <= 1 && in.avg >= 16.0 && gat_fused_enabled())
+        return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_SPMM_U_CS, K2);
       return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
              agg_cost(m, in, P_SPMM_W, K2);
     case GRANII_GAT_RECOMP:
+      if (in.world <= 1 && in.avg >= 16.0 && gat_fused_enabled())
+        return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
       return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
              agg_cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
   }

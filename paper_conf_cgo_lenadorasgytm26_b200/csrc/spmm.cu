@@ -84,6 +84,17 @@ struct SpmmArgs {
   const int32_t* __restrict__ owner_off;   // [n_rows][G1]
   const int32_t* __restrict__ seg_row;     // row of each heavy segment
   int G1, p0, p1, skip, first, last;
+  // fused additive attention (GAT, Eq. 4-6; ATT kernels): the weights are computed on the fly,
+  // w_e = exp(LeakyReLU(el_i + er_c) - m_i) / s_i with an online row max m_i and sum s_i; er
+  // travels in `cs` (prefetched a chunk ahead like a column scale), heavy segments leave their
+  // (m, s) in seg_ms for the softmax-aware combine
+  const float* __restrict__ el;
+  float2* __restrict__ seg_ms;
+};
+
+// online-softmax state of one row (or segment), warp-uniform m, per-lane partial s
+struct AttState {
+  float el, m, s;
 };
 
 // part r (0, or 1 after a skipped block) of the entries of `row` within [l0, h0) whose column lies
@@ -119,9 +130,10 @@ __device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t
 
 // The whole warp accumulates entries [rs0, re): G = 32/LPG lane groups each take a
 // neighbour, U neighbours per group in flight; acc holds this lane's group partial.
-template <int VEC, int LPG, int NJ, bool W, bool CS, int U>
+template <int VEC, int LPG, int NJ, bool W, bool CS, int U, bool ATT = false>
 __device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64_t re, int lane, int grp,
-                                           const char* const (&xbj)[NJ], uint32_t row_bytes, float (&acc)[NJ][VEC]) {
+                                           const char* const (&xbj)[NJ], uint32_t row_bytes, float (&acc)[NJ][VEC],
+                                           AttState* at = nullptr) {
   constexpr int G = 32 / LPG;
   if (rs0 >= re) return;
   // distance-2 prefetch: (c0, w0, cs0) = next chunk, (c1, w1) = the chunk after; the
@@ -133,7 +145,27 @@ __device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64
   if (rs0 + 32 < re) load_chunk<W>(a, rs0 + 32, re, lane, c1, w1);
   for (int64_t base = rs0; base < re; base += 32) {
     const int32_t c = c0;
-    const float w = CS ? w0 * cs0 : w0;
+    float w = CS ? w0 * cs0 : w0;
+    if constexpr (ATT) {
+      // scores of this chunk (cs0 = er of the lane's column; padding lanes have w0 = 0), chunk max
+      // over the warp, rescale of the running state when it grows, then the chunk's weights
+      const float z = at->el + cs0;
+      const float ev = w0 != 0.f ? (z > 0.f ? z : 0.2f * z) : -INFINITY;
+      float cm = ev;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) cm = fmaxf(cm, __shfl_xor_sync(0xffffffffu, cm, off));
+      if (cm > at->m) {  // warp-uniform
+        const float f = __expf(at->m - cm);  // 0 on the first chunk (m = -inf)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int v = 0; v < VEC; ++v) acc[j][v] *= f;
+        at->s *= f;
+        at->m = cm;
+      }
+      w = w0 != 0.f ? __expf(ev - at->m) : 0.f;
+      at->s += w;
+    }
     if (base + 32 < re) {
       c0 = c1;
       w0 = w1;
@@ -221,13 +253,24 @@ __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], con
 }
 
 // heavy-row segments first (largest work first), as warp-wide items
-template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U>
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U, bool ATT = false>
 __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lane, int grp, int lig,
                                            const bool (&colok)[NJ], const char* const (&xbj)[NJ],
                                            uint32_t row_bytes) {
   float acc[NJ][VEC];
   zero(acc);
   float* part = a.partial + t * a.ldp + (int64_t)lig * VEC;
+  if constexpr (ATT) {
+    AttState at{__ldg(a.el + a.seg_row[t]), -INFINITY, 0.f};
+    warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc, &at);
+    reduce_groups<LPG>(acc);
+    float st = at.s;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) st += __shfl_xor_sync(0xffffffffu, st, off);
+    if (grp == 0) store_row<LPG>(part, colok, acc, 1.f, 0);
+    if (lane == 0) a.seg_ms[t] = make_float2(at.m, st);
+    return;
+  }
   if constexpr (PH) {
     if (!a.first && grp == 0) load_partial<LPG>(part, colok, acc);
     for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {  // the range(s) are computed when needed
@@ -243,12 +286,24 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
 }
 
 // one row, the whole warp: G lane groups share its entries
-template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U>
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U, bool ATT = false>
 __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lane, int grp, int lig,
                                          const bool (&colok)[NJ], const char* const (&xbj)[NJ], uint32_t row_bytes) {
     float acc[NJ][VEC];
     zero(acc);
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
+    if constexpr (ATT) {
+      AttState at{__ldg(a.el + row), -INFINITY, 0.f};
+      warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj,
+                                                     row_bytes, acc, &at);
+      reduce_groups<LPG>(acc);
+      float st = at.s;
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) st += __shfl_xor_sync(0xffffffffu, st, off);
+      const float inv = st > 0.f ? 1.f / st : 0.f;
+      if (grp == 0) store_row<LPG>(y, colok, acc, (a.rs ? __ldg(a.rs + row) : 1.f) * inv, a.relu);
+      return;
+    }
     if constexpr (PH) {
       if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
       for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
@@ -277,7 +332,7 @@ constexpr int spmm_minb() { return VEC == 4 && NJ <= 2 ? 4 : 3; }
 template <int VEC, int LPG, int NJ>
 constexpr int spmm_unroll() { return VEC == 4 && NJ <= 2 ? 2 : (LPG >= 8 ? 4 : 32 / (32 / LPG)); }
 
-template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int UU = 0, int MINB = 0>
+template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int UU = 0, int MINB = 0, bool ATT = false>
 __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k_spmm_warp(SpmmArgs a) {
   constexpr int G = 32 / LPG;
   constexpr int U = UU > 0 ? UU : spmm_unroll<VEC, LPG, NJ>();  // neighbours per group per step
@@ -291,10 +346,10 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
   for (int64_t t = warp; t < a.n_seg + a.n_rows; t += nwarps) {
     if (t < a.n_seg) {
-      do_segment<VEC, LPG, NJ, W, CS, PH, U>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+      do_segment<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, t, lane, grp, lig, colok, xbj, row_bytes);
       continue;
     }
-    warp_row<VEC, LPG, NJ, W, CS, PH, U>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
+    warp_row<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
   }
 }
 
@@ -385,6 +440,30 @@ __global__ void k_spmm_combine(int64_t n_heavy, const int32_t* __restrict__ heav
   }
 }
 
+// heavy rows of the fused attention: Y_r = rs_r * sum_q partial_q exp(m_q - M) / sum_q s_q exp(m_q - M),
+// M = max_q m_q, segments in fixed order
+__global__ void k_spmm_combine_att(int64_t n_heavy, const int32_t* __restrict__ heavy_rows,
+                                   const int32_t* __restrict__ seg_ptr, const float* __restrict__ partial,
+                                   int64_t ldp, const float2* __restrict__ seg_ms, int64_t k0, int64_t kw,
+                                   float* __restrict__ Y, int64_t ldy, const float* __restrict__ rs, int relu) {
+  const int64_t total = n_heavy * kw;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t h = i / kw, k = i % kw;
+    float M = -INFINITY;
+    for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) M = fmaxf(M, seg_ms[q].x);
+    float v = 0.f, S = 0.f;
+    for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) {
+      const float f = seg_ms[q].x == -INFINITY ? 0.f : __expf(seg_ms[q].x - M);
+      v = fmaf(partial[(int64_t)q * ldp + k], f, v);
+      S = fmaf(seg_ms[q].y, f, S);
+    }
+    const int64_t row = heavy_rows[h];
+    float o = v * (S > 0.f ? 1.f / S : 0.f) * (rs ? rs[row] : 1.f);
+    if (relu) o = fmaxf(o, 0.f);
+    Y[row * ldy + k0 + k] = o;
+  }
+}
+
 // ------------------------------------------------------------------ dispatch
 template <int VEC, int LPG, int NJ, bool PH>
 static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool cs, int sms, cudaStream_t st) {
@@ -394,6 +473,13 @@ static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool 
   int64_t blocks = std::min<int64_t>(ceil_div(units, threads / 32), (int64_t)sms * 8);
   blocks = std::max<int64_t>(blocks, 1);
 #define GR_L(K) K<<<(unsigned)blocks, threads, 0, st>>>(a)
+  if constexpr (VEC == 4 && !PH) {
+    if (a.el) {  // fused attention: warp-per-row only (the caller checks spmm_att_supported)
+      GR_L((k_spmm_warp<VEC, LPG, NJ, false, true, false, 0, 0, true>));
+      GR_CHECK_LAUNCH();
+      return GRANII_OK;
+    }
+  }
   // tuning hook (GRANII_SPMM_TUNE="U,MINB"): alternative unroll / occupancy for the
   // warp-per-row kernels of the dominant shapes (tools/spmm_sweep.py)
   if constexpr (!PH && VEC == 4 && NJ == 2 && (LPG == 8 || LPG == 16 || LPG == 32)) {
@@ -511,7 +597,8 @@ granii_status launch_spmm(const granii_graph_s* g, const float* vals, const floa
 
 static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                                float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
-                               int64_t ldb, float beta, const SpmmPhase* ph, cudaStream_t st) {
+                               int64_t ldb, float beta, const SpmmPhase* ph, cudaStream_t st,
+                               const float* att_el = nullptr) {
   if (g->n_rows == 0 || K == 0) return GRANII_OK;
   DevInfo di;
   GR_TRY(dev_info(&di));
@@ -527,6 +614,15 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes, g->n_cols);
   float* partial = nullptr;  // heavy-segment partials: this slice's columns start at partial + pk0
   bool own_partial = false;
+  float2* seg_ms = nullptr;  // fused attention: (max, sum) of every heavy segment
+  if (att_el) {
+    if (ph || !warp_mode || !vec4 || vals || B)
+      return fail(GRANII_ERR_UNSUPPORTED, "fused attention SpMM: warp-per-row, aligned, unphased only");
+    a.el = att_el;
+    a.seg_row = g->seg_row;  // el of a heavy segment's row
+    if (g->n_seg > 0) GR_CUDA(cudaMallocAsync((void**)&seg_ms, (size_t)g->n_seg * sizeof(float2), st));
+    a.seg_ms = seg_ms;
+  }
   if (ph) {
     a.owner_off = g->owner_off;
     a.seg_row = g->seg_row;
@@ -548,7 +644,7 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   // per row row_ptr + the K-row of Y (+rs)
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) +
-                       R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0) + (B ? 4.0 * K : 0.0));
+                       R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0) + (B ? 4.0 * K : 0.0) + (att_el ? 4.0 : 0.0));
   // a phased aggregation books its algorithmic bytes once (in its last phase)
   const bool book = !ph || ph->last;
   ProfScope ps("spmm", st, book ? bytes : 0.0, book ? 2.0 * nnz * K : 0.0, (int)ceil_div(K, kw));
@@ -560,7 +656,13 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
     const bool v4 = vec4 && (k0 % 4 == 0);
     if (ph) GR_TRY(launch_slice<true>(a, v4, warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
     else GR_TRY(launch_slice<false>(a, v4, warp_mode, vals != nullptr, cs != nullptr, di.sms, st));
-    if (combine) {
+    if (combine && att_el) {
+      const int64_t tot = g->n_heavy * a.kw;
+      k_spmm_combine_att<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(
+          g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, seg_ms, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0);
+      GR_CHECK_LAUNCH();
+      ps.add_launches(1);
+    } else if (combine) {
       const int64_t tot = g->n_heavy * a.kw;
       k_spmm_combine<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(tot, 256), 4096)), 256, 0, st>>>(
           g->n_heavy, g->order, g->seg_ptr, a.partial, a.ldp, a.k0, a.kw, Y, ldy, rs, relu ? 1 : 0, B, ldb, beta);
@@ -569,6 +671,7 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
     }
   }
   if (own_partial) GR_CUDA(cudaFreeAsync(partial, st));
+  if (seg_ms) GR_CUDA(cudaFreeAsync(seg_ms, st));
   return GRANII_OK;
 }
 
@@ -576,6 +679,13 @@ granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const f
                              float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                              int64_t ldb, float beta, cudaStream_t st) {
   return spmm_impl(g, vals, X, ldx, K, Y, ldy, rs, cs, relu, B, ldb, beta, nullptr, st);
+}
+
+bool spmm_att_supported(const granii_graph_s* g) { return g->avg_deg() >= 16.f; }
+
+granii_status launch_spmm_att(const granii_graph_s* g, const float* el, const float* er, const float* X, int64_t ldx,
+                              int64_t K, float* Y, int64_t ldy, const float* rs, bool relu, cudaStream_t st) {
+  return spmm_impl(g, nullptr, X, ldx, K, Y, ldy, rs, er, relu, nullptr, 0, 0.f, nullptr, st, el);
 }
 
 granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,

@@ -391,6 +391,37 @@ def test_gat_forward_both_compositions(G, comp, attn, name, K1, K2):
     assert err(out.cpu(), ref) <= TOL
 
 
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("K1,K2,slice_", [(64, 256, None), (256, 40, None), (100, 256, "64"), (48, 1000, None)])
+def test_gat_fused_attention_spmm(G, comp, K1, K2, slice_, monkeypatch):
+    """Additive GAT on a warp-per-row graph runs scores + row softmax + aggregation as one SpMM
+    with an online (max, sum) per row.  Against the oracle and against the
+    unfused SDDMM -> SpMM path, with scores scaled up (a_l, a_r x 8) so the running max moves
+    inside rows, forced K slices, and hub segments (GRANII_SEG=64: softmax-aware combine)."""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    base = case(G, "dense")
+    monkeypatch.setenv("GRANII_SEG", "64")
+    g = G.granii_graph_csr_create(base.n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), base.flags)
+    monkeypatch.delenv("GRANII_SEG")
+    if slice_:
+        monkeypatch.setenv("GRANII_SPMM_SLICE", slice_)
+    rp, ci, n = base.rp, base.ci, base.n
+    H = synth.features(60, n, K1)
+    W = synth.glorot(60, 2, K1, K2, (K1, K2))
+    al = synth.uniform_pm1(60, 3, (K2,)) * 8
+    ar = synth.uniform_pm1(60, 4, (K2,)) * 8
+    outs = []
+    for fused in ("1", "0"):
+        monkeypatch.setenv("GRANII_GAT_FUSED", fused)
+        spec = LayerSpec(G.GAT, K1, K2, G.ACT_RELU, 0, comp=comp, W=W.to(DEV), a_l=al.to(DEV), a_r=ar.to(DEV))
+        net = GNN(g, [spec], DEV)
+        outs.append(net.forward(pad(H)).cpu().clone())
+        torch.cuda.synchronize()
+    ref, _ = O.gat_forward(comp, rp, ci, H, W, al, ar, 1)
+    assert err(outs[0], ref) <= TOL
+    assert err(outs[1], ref) <= TOL
+
+
 @pytest.mark.parametrize("comp", [0, 1, 2, 3])
 @pytest.mark.parametrize("name,K1,K2", [("pubmed", 32, 256), ("pubmed", 256, 32), ("dense", 48, 16)])
 def test_gcn_backward_every_composition(G, comp, name, K1, K2):
@@ -439,6 +470,32 @@ def gat_grad_ok(y, r, m):
     ok = d <= TOL * np.abs(r).max(1) + 4 * 2.0 ** -24 * m.max(1)
     assert normwise(y, r) <= 10 * TOL
     return bool(ok.all())
+
+
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("name,K1,K2", [("dense", 48, 100), ("pubmed", 64, 256), ("sparse", 40, 24)])
+def test_gat_backward_hub_segments(G, comp, name, K1, K2, monkeypatch):
+    """Hub rows cut into warp-wide segments in both backward passes (online-softmax states merged
+    per row in pass A, partial rows + der summed in pass B, fixed order): GRANII_SEG=64 makes
+    every row over 64 entries a hub, GRANII_GATBWD_SEG=1 forces the segmented schedule on the
+    warp-per-row graph too"""
+    base = case(G, name)
+    monkeypatch.setenv("GRANII_SEG", "64")
+    g = G.granii_graph_csr_create(base.n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), base.flags)
+    monkeypatch.delenv("GRANII_SEG")
+    monkeypatch.setenv("GRANII_GATBWD_SEG", "1")
+    assert np.diff(base.rp).max() > 64
+    c2 = Case.__new__(Case)
+    c2.n, c2.g, c2.rp, c2.ci = base.n, g, base.rp, base.ci
+    net, out, H, W, al, ar = run_layer(G, c2, G.GAT, comp, K1, K2, G.ACT_NONE)
+    Gup = synth.uniform_pm1(62, 1, (c2.n, K2))
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    ref = O.gat_backward(comp, c2.rp, c2.ci, H, W, al, ar, Gup, 0)
+    mag = O.gat_backward_magnitude(comp, c2.rp, c2.ci, H, W, al, ar, Gup, 0)
+    got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
+    for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, ref, mag):
+        assert gat_grad_ok(y.cpu(), r, m), nm
 
 
 def test_gat_backward_deterministic_and_input_layer(G):
