@@ -120,12 +120,63 @@ granii_status launch_rank_sum(int n, const float* const* src, size_t count, floa
   return GRANII_OK;
 }
 
+// C <= LPG * NV (the classifier widths: 41, 47): an LPG-lane group per row holds its logits in
+// registers -- one coalesced load, max and sum by fixed xor butterflies, one store -- so every load
+// of the 32 / LPG rows of a warp is in flight at once (the warp-per-row loop above re-reads the row
+// three times with a dependent round trip each)
+template <int LPG, int NV>
+__global__ void __launch_bounds__(256) k_softmax_xent_reg(int64_t rows, int64_t C, const float* __restrict__ Z,
+                                                          int64_t ldz, const int32_t* __restrict__ y, float inv_n,
+                                                          float* __restrict__ dZ, int64_t lddz,
+                                                          float* __restrict__ loss) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, lg = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r0 = warp * G; r0 < rows; r0 += nw * G) {
+    const int64_t r = r0 + lane / LPG;
+    const bool live = r < rows;
+    const float* z = Z + (live ? r : 0) * ldz;
+    float v[NV];
+    float m = -INFINITY;
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      const int64_t c = lg + q * LPG;
+      v[q] = (live && c < C) ? __ldg(z + c) : -INFINITY;
+      m = fmaxf(m, v[q]);
+    }
+#pragma unroll
+    for (int o = LPG / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    float s = 0.f;
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      v[q] = live ? expf(v[q] - m) : 0.f;
+      s += v[q];
+    }
+#pragma unroll
+    for (int o = LPG / 2; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (!live) continue;
+    const int32_t t = y[r];
+#pragma unroll
+    for (int q = 0; q < NV; ++q) {
+      const int64_t c = lg + q * LPG;
+      if (c < C) dZ[r * lddz + c] = (v[q] / s - (c == t ? 1.f : 0.f)) * inv_n;
+    }
+    if (loss && lg == 0) loss[r] = logf(s) + m - z[t];
+  }
+}
+
 granii_status launch_softmax_xent(int64_t rows, int64_t C, const float* Z, int64_t ldz, const int32_t* y,
                                   int64_t n_total, float* dZ, int64_t lddz, float* loss, cudaStream_t st) {
   if (rows == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, 8.0 * rows * C + 8.0 * rows, 0.0, 1);
   const unsigned b = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, 8), 148 * 16));
-  k_softmax_xent<<<b, 256, 0, st>>>(rows, C, Z, ldz, y, 1.f / (float)n_total, dZ, lddz, loss);
+  if (C <= 64) {
+    const unsigned b2 = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, 16), 148 * 16));
+    k_softmax_xent_reg<16, 4><<<b2, 256, 0, st>>>(rows, C, Z, ldz, y, 1.f / (float)n_total, dZ, lddz, loss);
+  } else {
+    k_softmax_xent<<<b, 256, 0, st>>>(rows, C, Z, ldz, y, 1.f / (float)n_total, dZ, lddz, loss);
+  }
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

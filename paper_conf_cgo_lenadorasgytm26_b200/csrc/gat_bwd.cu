@@ -603,12 +603,28 @@ __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, 
   const int64_t col = blockIdx.x * 32 + tx, s = blockIdx.y;
   const int64_t r0 = s * chunk, r1 = (r0 + chunk < R) ? r0 + chunk : R;
   float p = 0.f, q = 0.f;
-  if (col < K)
-    for (int64_t r = r0 + ty; r < r1; r += 8) {
+  if (col < K) {
+    int64_t r = r0 + ty;
+    for (; r + 24 < r1; r += 32) {  // four rows in flight per thread, summed in row order
+      float h[4], a0[4], a1[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        h[u] = H[(r + 8 * u) * ldh + col];
+        a0[u] = __ldg(d0 + r + 8 * u);
+        a1[u] = __ldg(d1 + r + 8 * u);
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        p = fmaf(h[u], a0[u], p);
+        q = fmaf(h[u], a1[u], q);
+      }
+    }
+    for (; r < r1; r += 8) {
       const float h = H[r * ldh + col];
       p = fmaf(h, __ldg(d0 + r), p);
       q = fmaf(h, __ldg(d1 + r), q);
     }
+  }
   sp[ty][tx] = p;
   sq[ty][tx] = q;
   __syncthreads();

@@ -510,8 +510,13 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     const bool dot = a->attn == GRANII_ATTN_DOT;
     // additive attention on one GPU over a warp-per-row graph: the scores, the row softmax and the
     // aggregation are one fused SpMM (no SDDMM pass, no alpha array); GRANII_GAT_FUSED=0 disables
+    // partitioned graphs: when the aggregation's schedule is a single all-gather (P = 1; the same
+    // on every rank) the gathered operand feeds the fused SpMM; an overlapped (phased) schedule
+    // keeps SDDMM -> phased SpMM
     const bool out_aligned = (ldo % 4 == 0) && (((uintptr_t)out & 15) == 0);  // REUSE aggregates into out
-    const bool fused = !dot && !c.dist() && spmm_att_supported(g) && gat_fused_enabled() &&
+    const int64_t agg_k = comp == GRANII_GAT_REUSE ? K2 : K1;
+    const int agg_p = c.dist() && overlap_enabled() && g->owner_off ? comm_phases(g, agg_k, true, false) : 1;
+    const bool fused = !dot && agg_p <= 1 && spmm_att_supported(g) && gat_fused_enabled() &&
                        (comp == GRANII_GAT_RECOMP || out_aligned);
     float* alpha = fused ? nullptr : b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
     const bool need_theta = comp == GRANII_GAT_REUSE || dot;
@@ -566,7 +571,10 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
     if (comp == GRANII_GAT_REUSE) {
       if (run) {
         if (dot) GR_TRY(launch_spmm(g, alpha, th.all, th.ld, K2, out, ldo, nullptr, nullptr, relu, st));
-        else if (fused) GR_TRY(launch_spmm_att(g, el, er_all, th.all, th.ld, K2, out, ldo, nullptr, relu, st));
+        else if (fused) {
+          GR_TRY(allgather(c, th));
+          GR_TRY(launch_spmm_att(g, el, er_all, th.all, th.ld, K2, out, ldo, nullptr, relu, st));
+        }
         else GR_TRY(gathered_spmm(c, th, alpha, K2, out, ldo, nullptr, nullptr, relu));
       }
     } else {
@@ -576,7 +584,10 @@ static granii_status forward_impl(const Ctx& c, granii_model m, granii_compositi
       size_t gn2;
       gemm_ws(b, R, K2, K1, relu ? GRANII_GEMM_RELU : 0, &gw2, &gn2);
       if (run) {
-        if (fused) GR_TRY(launch_spmm_att(g, el, er_all, xg.all, xg.ld, K1, T, ldt, nullptr, false, st));
+        if (fused) {
+          GR_TRY(allgather(c, xg));
+          GR_TRY(launch_spmm_att(g, el, er_all, xg.all, xg.ld, K1, T, ldt, nullptr, false, st));
+        }
         else GR_TRY(gathered_spmm(c, xg, alpha, K1, T, ldt, nullptr, nullptr, false));
         GR_TRY(launch_gemm(R, K2, K1, T, ldt, a->W, K2, out, ldo, nullptr, relu ? GRANII_GEMM_RELU : 0, gw2, gn2,
                            st));

@@ -252,17 +252,20 @@ double forward_cost(const CostModel& m, const In& in, int comp, double K1, doubl
     case GRANII_GCN_DYN_UPD:
       return cost(m, in, P_GEMM, K1, K2) + agg_cost(m, in, P_SPMM_U, K2);
     case GRANII_GAT_REUSE:
-      // one GPU, warp-per-row graph: scores + softmax fused into the aggregation (layer.cu), whose
-      // per-entry er gather is modelled like the column-scale gather of the unweighted SpMM
-      if (in.world <= 1 && in.avg >= 16.0 && gat_fused_enabled())
-        return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_SPMM_U_CS, K2);
-      return cost(m, in, P_GEMM_ATT, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
-             agg_cost(m, in, P_SPMM_W, K2);
-    case GRANII_GAT_RECOMP:
-      if (in.world <= 1 && in.avg >= 16.0 && gat_fused_enabled())
-        return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_SPMM_U_CS, K1) + cost(m, in, P_GEMM, K1, K2);
-      return cost(m, in, P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, 1) + cost(m, in, P_SDDMM1_SM, 0) +
-             agg_cost(m, in, P_SPMM_W, K1) + cost(m, in, P_GEMM, K1, K2);
+    case GRANII_GAT_RECOMP: {
+      // warp-per-row graph with a single-all-gather schedule: scores + softmax fused into the
+      // aggregation (layer.cu), whose per-entry er gather is modelled like the column-scale gather
+      // of the unweighted SpMM; otherwise SDDMM + row softmax, then the (possibly phased) SpMM
+      const bool reuse = comp == GRANII_GAT_REUSE;
+      const double K = reuse ? K2 : K1;
+      const double pre = cost(m, in, reuse ? P_GEMM_ATT : P_GEMM_NOSTORE, K1, K2) + cost(m, in, P_ALLGATHER, 1);
+      const double post = reuse ? 0.0 : cost(m, in, P_GEMM, K1, K2);
+      int P = 1;
+      const double agg = agg_schedule(m, in, P_SPMM_W, K, &P);
+      if (P <= 1 && in.avg >= 16.0 && gat_fused_enabled())
+        return pre + cost(m, in, P_ALLGATHER, K) + cost(m, in, P_SPMM_U_CS, K) + post;
+      return pre + cost(m, in, P_SDDMM1_SM, 0) + agg + post;
+    }
   }
   return 1e30;
 }

@@ -19,9 +19,12 @@ done
 B="python bench.py --steps 2 --warmup 3 --no-e2e --no-regret --no-cpu --cuda-graph off"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $M/launches.csv $B > /dev/null 2>&1; echo "ncu launches rc=$?"
 python tools/ncu_launches.py $M/launches.csv $M/ncu_launches_default_bench.txt $M/ncu_launches_share.json "$B" > /dev/null
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm_warp -s 20 -c 5 -o $M/spmm_full $B > /dev/null 2>&1; echo "ncu spmm rc=$?"
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_gemm -s 4 -c 3 -o $M/gemm_full $B > /dev/null 2>&1; echo "ncu gemm rc=$?"
+# full captures stay on the box (/tmp: gpurun copies back <= 64 MiB); summaries come back
+R=/tmp/ncu_reps; mkdir -p $R
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spmm_warp -s 20 -c 5 -o $R/spmm_full $B > /dev/null 2>&1; echo "ncu spmm rc=$?"
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_gemm -s 4 -c 3 -o $R/gemm_full $B > /dev/null 2>&1; echo "ncu gemm rc=$?"
 BG="python bench.py --workload products-gat2-train --steps 1 --warmup 3 --no-e2e --no-regret --no-cpu --cuda-graph off"
-timeout 900 ncu --set full --clock-control none -k regex:"k_gat_bwd|k_spmm_warp" -s 8 -c 6 -o $M/gat_train_full $BG > /dev/null 2>&1; echo "ncu gat rc=$?"
-for r in spmm_full gemm_full gat_train_full; do [ -f $M/$r.ncu-rep ] && python tools/ncu_summary.py $M/$r.ncu-rep > $M/${r}_summary.json; done
+timeout 900 ncu --set full --clock-control none -k regex:"k_gat_bwd|k_spmm_warp" -s 8 -c 6 -o $R/gat_train_full $BG > /dev/null 2>&1; echo "ncu gat rc=$?"
+for r in spmm_full gemm_full gat_train_full; do [ -f $R/$r.ncu-rep ] && python tools/ncu_summary.py $R/$r.ncu-rep > $M/${r}_summary.json; done
+[ -f $R/spmm_full.ncu-rep ] && ncu -i $R/spmm_full.ncu-rep --page raw --csv > $M/spmm_full_raw.csv 2>/dev/null
 ls $M
