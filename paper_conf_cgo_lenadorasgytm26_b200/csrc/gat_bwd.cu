@@ -391,8 +391,9 @@ __device__ __forceinline__ void gat_b_group_row(const GatBwdArgs& a, int64_t t0,
 
 // One launch covers both schedules: warps [0, n_wide) take the wide rows order[0 .. n_wide)
 // (all rows of a dense graph), the remaining warps take G rows each, one per lane group.
-template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_a(GatBwdArgs a) {
+template <int LPG, int NJ, int U, int MINB = 0>
+__global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))))
+    k_gat_bwd_a(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -407,8 +408,8 @@ __global__ void __launch_bounds__(256, NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2
   gat_a_warp_row<LPG, NJ, U>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
 }
 
-template <int LPG, int NJ, int U>
-__global__ void __launch_bounds__(256, NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1)) k_gat_bwd_b(GatBwdArgs a) {
+template <int LPG, int NJ, int U, int MINB = 0>
+__global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_b(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -459,15 +460,15 @@ __global__ void k_gat_b_combine(GatBwdArgs a) {
   }
 }
 
-template <int LPG, int NJ, int U>
+template <int LPG, int NJ, int U, int MINB = 0>
 static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
   constexpr int G = 32 / LPG;
   const int64_t warps = a.n_seg + a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
   const unsigned blocks = (unsigned)std::max<int64_t>(1, ceil_div(warps, 8));
   if (pass == 0)
-    k_gat_bwd_a<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
+    k_gat_bwd_a<LPG, NJ, U, MINB><<<blocks, 256, 0, st>>>(a);
   else
-    k_gat_bwd_b<LPG, NJ, U><<<blocks, 256, 0, st>>>(a);
+    k_gat_bwd_b<LPG, NJ, U, MINB><<<blocks, 256, 0, st>>>(a);
 }
 
 granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
@@ -544,11 +545,17 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
   const int64_t K = b.K;
   // tuning hook GRANII_GATBWD="LPG,NJ,U" (tools: bench.py per_primitive_ms), if it covers K
   if (const char* e = getenv("GRANII_GATBWD")) {
-    int l = 0, n = 0, u = 0;
-    sscanf(e, "%d,%d,%d", &l, &n, &u);
+    int l = 0, n = 0, u = 0, mb = 0;
+    sscanf(e, "%d,%d,%d,%d", &l, &n, &u, &mb);
     if ((int64_t)l * n * 4 >= K) {
       bool ok = true;
-      if (l == 8 && n == 2 && u == 4) gb_launch<8, 2, 4>(pass, b, st);
+      if (l == 16 && n == 2 && u == 2 && mb == 4) gb_launch<16, 2, 2, 4>(pass, b, st);
+      else if (l == 16 && n == 2 && u == 2 && mb == 5) gb_launch<16, 2, 2, 5>(pass, b, st);
+      else if (l == 8 && n == 2 && u == 2 && mb == 4) gb_launch<8, 2, 2, 4>(pass, b, st);
+      else if (l == 8 && n == 2 && u == 2 && mb == 5) gb_launch<8, 2, 2, 5>(pass, b, st);
+      else if (l == 16 && n == 2 && u == 4 && mb == 3) gb_launch<16, 2, 4, 3>(pass, b, st);
+      else if (l == 8 && n == 2 && u == 4 && mb == 3) gb_launch<8, 2, 4, 3>(pass, b, st);
+      else if (l == 8 && n == 2 && u == 4) gb_launch<8, 2, 4>(pass, b, st);
       else if (l == 16 && n == 1 && u == 4) gb_launch<16, 1, 4>(pass, b, st);
       else if (l == 16 && n == 2 && u == 4) gb_launch<16, 2, 4>(pass, b, st);
       else if (l == 16 && n == 2 && u == 2) gb_launch<16, 2, 2>(pass, b, st);
@@ -572,13 +579,19 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
   }
   if (K <= 16) gb_launch<4, 1, 4>(pass, b, st);
   else if (K <= 32) gb_launch<8, 1, 4>(pass, b, st);
-  else if (K <= 64) gb_launch<8, 2, 2>(pass, b, st);
+  // pass B on warp-per-row graphs at 4 blocks / SM (64 registers, a few spilled): products K=47
+  // 6.76 -> 6.22 ms, K=100 10.7 -> 10.3 ms (pass A is slower there)
+  else if (K <= 64) {
+    if (pass == 1 && dense) gb_launch<8, 2, 2, 4>(pass, b, st);
+    else gb_launch<8, 2, 2>(pass, b, st);
+  }
   // warp-per-row graphs (products-shaped sweep): 16-lane groups up to K = 128 (K=100: A 10.9 -> 9.8,
   // B 13.0 -> 10.5 ms vs <8,4,2>); pass A keeps one entry per group in flight beyond K = 128 (K=256
   // 18.8 -> 18.3 ms, K=512 39.1 -> 35.2 ms).  Group-per-row graphs keep more rows per warp (pubmed-
   // shaped K=256: <32,2,1> for pass A cost 0.19 -> 0.25 ms)
   else if (K <= 128) {
-    if (dense) gb_launch<16, 2, 2>(pass, b, st);
+    if (dense && pass == 1) gb_launch<16, 2, 2, 4>(pass, b, st);
+    else if (dense) gb_launch<16, 2, 2>(pass, b, st);
     else gb_launch<8, 4, 2>(pass, b, st);
   } else if (K <= 256) {
     if (pass == 0 && dense) gb_launch<32, 2, 1>(pass, b, st);

@@ -191,13 +191,18 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
   const bool pre = m == GRANII_SGC && dyn && hops > 0 &&
                    dyn_prescale((double)g->local_nnz, (double)R, g->avg_deg(), (double)g->n_cols, upd ? K2 : K1,
                                 di.l2_bytes);
+  // TAGCN DYN aggregate-first: the same trade -- every hop's input is D̃^-½ X_j from a row-broadcast
+  // pass (X_j itself is kept for the concatenated GEMM), the hop SpMM applies only D̃^-½ on rows
+  const bool pre_t = m == GRANII_TAGCN && dyn && !upd && hops > 0 &&
+                     dyn_prescale((double)g->local_nnz, (double)R, g->avg_deg(), (double)g->n_cols, K1, di.l2_bytes);
   // H: aligned own rows, and (aggregate-first) its gathered copy
   const float* H = a->H;
   int64_t ldh = a->ldh;
   const bool h_aligned = (ldh % 4 == 0) && (((uintptr_t)H & 15) == 0);
   GatherBuf hg;
   const bool h_gather = c.dist() && !upd;
-  const bool h_scale = pre && !upd;
+  const bool h_scale = (pre || pre_t) && !upd;
+  float* pscaled = nullptr;  // one GPU, TAGCN pre_t: the pre-scaled hop input, rewritten after every hop
   if (h_gather) {
     hg = gather_buf(b, c, K1);
     if (run) {
@@ -212,6 +217,7 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
     if (run) GR_TRY(launch_scale_mask(R, K1, nullptr, 0, a->H, a->ldh, g->dinv_rows, hp, ld4(K1), st));
     H = hp;
     ldh = ld4(K1);
+    pscaled = hp;
   } else if (!h_aligned) {
     float* hp = b.take((size_t)Rr * ld4(K1));
     if (run) GR_TRY(launch_copy_rows(R, K1, a->H, a->ldh, hp, ld4(K1), st));
@@ -307,11 +313,28 @@ static granii_status ext_forward_impl(const Ctx& c, granii_model m, granii_compo
         for (int j = 0; j <= hops; ++j)
           GR_CUDA(cudaMemcpyAsync(Wc + (int64_t)j * Kb * K2, a->W + (int64_t)j * K1 * K2,
                                   sizeof(float) * (size_t)K1 * K2, cudaMemcpyDeviceToDevice, st));
-        GR_TRY(launch_copy_rows(R, K1, H, ldh, Xc, ldc, st));  // X_0 = H
+        GR_TRY(launch_copy_rows(R, K1, pre_t ? a->H : H, pre_t ? a->ldh : ldh, Xc, ldc, st));  // X_0 = H
         const float* X = H_all;
         int64_t ldx = ldh;
         for (int j = 1; j <= hops; ++j) {
           float* dst = Xc + (int64_t)(j)*Kb;
+          if (pre_t) {  // X_j = D̃^-½ Ã (D̃^-½ X_{j-1}); then the next hop's pre-scaled input
+            GR_TRY(launch_spmm_ex(g, nullptr, X, ldx, K1, dst, ldc, g->dinv_rows, nullptr, false, nullptr, 0, 0.f,
+                                  st));
+            if (j == hops) break;
+            if (c.dist()) {
+              GatherBuf& nb = pb[j & 1];
+              GR_TRY(launch_scale_mask(R, K1, nullptr, 0, dst, ldc, g->dinv_rows, nb.mine, nb.ld, st));
+              GR_TRY(allgather(c, nb));
+              X = nb.all;
+              ldx = nb.ld;
+            } else {
+              GR_TRY(launch_scale_mask(R, K1, nullptr, 0, dst, ldc, g->dinv_rows, pscaled, ld4(K1), st));
+              X = pscaled;
+              ldx = ld4(K1);
+            }
+            continue;
+          }
           if (c.dist()) {
             GatherBuf& nb = pb[j & 1];
             GR_TRY(hop(X, ldx, K1, nb.mine, nb.ld, false, nullptr, 0, 0.f));

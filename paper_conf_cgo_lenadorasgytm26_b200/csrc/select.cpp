@@ -108,6 +108,7 @@ static granii_status load_model(const char* path, CostModel* out) {
 struct In {
   double R, nnz, ncols, avg, l2, world, nseg;
   double xcols;  // rows of X an SpMM gathers from (a phased SpMM slices like the whole one: ncols)
+  double maxd = 0, seg_len = 2048;  // longest row (featurizer feature 4) and the hub-segment length
 };
 
 static bool overlap_on() {
@@ -176,8 +177,11 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
       const double idx = in.nnz * (p == P_GAT_BWD_A ? 8.0 : 20.0) * gb;
       // dependent gather steps per warp (gat_bwd.cu: G lane groups x U entries per step)
       const double gu = K <= 16 ? 32 : K <= 32 ? 16 : K <= 128 ? 8 : K <= 256 ? 4 : K <= 512 ? 2 : 1;
+      // the longest dependent chain: a whole row on warp-per-row graphs, at most one hub segment
+      // on group-per-row graphs (gat_bwd.cu) -- the tail of small power-law graphs
+      const double chain = (in.avg >= 16.0 ? in.maxd : std::min(in.maxd, in.seg_len)) / gu;
       return {1.0, idx, in.R * K * (p == P_GAT_BWD_A ? 4.0 : 12.0) * gb, gath * h, gath * (1.0 - h), in.R * 1e-6,
-              (in.nnz / gu + 0.5 * in.R) * 1e-6};
+              (in.nnz / gu + 0.5 * in.R) * 1e-6, chain * 1e-3};
     }
     case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
     case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};
@@ -288,6 +292,10 @@ double ext_forward_cost(const CostModel& m, const In& in, int comp, double K1, d
   } else if (base == GRANII_TAGCN_PRE_AGG) {
     if (upd)
       t += cost(m, in, P_GEMM, K1, (k + 1) * K2) + k * (cost(m, in, P_ALLGATHER, K2) + cost(m, in, sp, K2));
+    else if (dyn && k > 0 && dyn_prescale(in.nnz, in.R, in.avg, in.xcols, (int64_t)K1, (int64_t)in.l2))
+      // pre-scaled hop inputs (layer.cu pre_t): a row-broadcast pass before every hop
+      t += cost(m, in, P_ELEMENTWISE, K1) * (k + 1) + k * (cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U, K1)) +
+           cost(m, in, P_GEMM, (k + 1) * K1, K2);
     else
       t += cost(m, in, P_ELEMENTWISE, K1) + k * (cost(m, in, P_ALLGATHER, K1) + cost(m, in, sp, K1)) +
            cost(m, in, P_GEMM, (k + 1) * K1, K2);
@@ -341,10 +349,11 @@ static In inputs_of(const granii_graph_s* g) {
   if (g->world > 1) {
     const double G = (double)g->world, N = (double)g->N, nnz = (double)g->nnz;
     return In{N / G, nnz / G, (double)g->n_cols, N > 0 ? nnz / N : 0.0, (double)di.l2_bytes, G,
-              (double)std::max<int64_t>(g->n_seg_global, 0) / G, (double)g->n_cols};
+              (double)std::max<int64_t>(g->n_seg_global, 0) / G, (double)g->n_cols, (double)g->features[4],
+              (double)g->seg_len};
   }
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-            (double)g->world, (double)g->n_seg, (double)g->n_cols};
+            (double)g->world, (double)g->n_seg, (double)g->n_cols, (double)g->features[4], (double)g->seg_len};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, const granii_layer_args* shape,
