@@ -109,6 +109,7 @@ struct In {
   double R, nnz, ncols, avg, l2, world, nseg;
   double xcols;  // rows of X an SpMM gathers from (a phased SpMM slices like the whole one: ncols)
   double maxd = 0, seg_len = 2048;  // longest row (featurizer feature 4) and the hub-segment length
+  double N = 0, top1 = 0;           // global nodes; share of entries in the top-1 % rows (feature 6)
 };
 
 static bool overlap_on() {
@@ -116,13 +117,21 @@ static bool overlap_on() {
   return !(e && e[0] == '0');
 }
 
-// fraction of gathered bytes served by L2: the sliced SpMM keeps
-// a slice resident when the graph is dense; otherwise LRU-like hit ~ L2 / |X|.
+// fraction of gathered bytes served by L2: the sliced SpMM keeps a slice resident
+// when the graph is dense; otherwise the L2 holds the C = 0.8 L2 / (4K) most-gathered rows of X.
+// Gathers follow column popularity (= degree on the symmetric graphs): the top 1 % of rows take a
+// share top1 of the entries (featurizer feature 6), the rest is taken as uniform -- so a skewed
+// (power-law) graph hits far more often than the capacity ratio C / N alone says.
 static double l2_hit(const In& in, double K, double cols) {
   const double xbytes = cols * K * 4.0;
   if (xbytes <= 0.8 * in.l2) return 1.0;
   if (in.avg >= 32.0 && cols * 64.0 * 4.0 <= 0.55 * in.l2) return 1.0;  // K-sliced
-  return std::max(0.0, std::min(1.0, 0.8 * in.l2 / xbytes));
+  const double cap = std::max(0.0, std::min(1.0, 0.8 * in.l2 / xbytes));
+  if (in.N <= 0 || in.top1 <= 0) return cap;
+  const double C = cap * cols, N1 = std::max(1.0, std::ceil(in.N / 100.0));
+  const double h = C <= N1 ? in.top1 * C / N1
+                           : in.top1 + (1.0 - in.top1) * std::min(1.0, (C - N1) / std::max(1.0, cols - N1));
+  return std::max(cap, std::min(1.0, h));
 }
 
 // primitive ids of the feature API
@@ -350,10 +359,11 @@ static In inputs_of(const granii_graph_s* g) {
     const double G = (double)g->world, N = (double)g->N, nnz = (double)g->nnz;
     return In{N / G, nnz / G, (double)g->n_cols, N > 0 ? nnz / N : 0.0, (double)di.l2_bytes, G,
               (double)std::max<int64_t>(g->n_seg_global, 0) / G, (double)g->n_cols, (double)g->features[4],
-              (double)g->seg_len};
+              (double)g->seg_len, N, nnz > 0 ? (double)g->features[6] / nnz : 0.0};
   }
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-            (double)g->world, (double)g->n_seg, (double)g->n_cols, (double)g->features[4], (double)g->seg_len};
+            (double)g->world, (double)g->n_seg, (double)g->n_cols, (double)g->features[4], (double)g->seg_len,
+            (double)g->N, g->nnz > 0 ? (double)g->features[6] / (double)g->nnz : 0.0};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, const granii_layer_args* shape,

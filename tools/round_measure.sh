@@ -13,6 +13,7 @@ for wl in reddit-gcn2-train reddit-gcn2-train-h32 reddit-gcn2-train-h1024 produc
 done
 timeout 1500 python tools/regret_sweep.py $M/regret_sweep.json > $M/regret_sweep.log 2>&1; echo "regret sweep rc=$?"
 timeout 900 python bench.py --steps 20 --warmup 5 --out $M/bench_default.json > $M/bench_default.log 2>&1; echo "default rc=$?"
+[ "${SKIP_NCU:-0}" = 1 ] && { ls $M; exit 0; }
 for wl in reddit-gcn2-train products-gcn2-infer products-gat2-infer; do
   timeout 600 python tools/scaling_projection.py --workload $wl --out $M/scaling_projection_$wl.json > $M/proj_$wl.log 2>&1; echo "proj $wl rc=$?"
 done
