@@ -106,64 +106,64 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
   const float ci = a.c[r];
   float xv[NJ][4];
   gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, a.K, xv);
-  // one sweep with an online softmax; per lane group: running max m, S = Σ w, Cw = Σ w·s',
-  // and per lane D = Σ w·s'·(this lane's share of dα), w = exp(e - m), s' = LeakyReLU'(z).
-  // del = (Σ_lanes D - c·Cw) / S: dα enters linearly, so it is never reduced per entry
+  // One sweep with an online softmax whose scalar work is done once per entry, by the lane that
+  // loaded the entry's column (chunk of 32): its er (gathered a chunk ahead), score, slope s'; the
+  // chunk's max over the warp (one rescale per chunk when it grows, warp-uniform m), then
+  // w = exp(e - m).  The owner lane keeps S = Σ w and Cw = Σ w·s'; the lane groups that gather the
+  // K-wide rows get w·s' by shuffle and keep D = Σ w·s'·(their share of dα).  Everything is
+  // reduced once per row: del = (Σ D - c·Σ Cw) / Σ S.
   float m = -INFINITY, S = 0.f, Cw = 0.f, D = 0.f;
-  int32_t cn = 0;
-  if (b < t) cn = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+  int32_t c0 = 0, c1 = 0;
+  float e0 = 0.f;
+  if (b < t) {
+    c0 = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+    e0 = __ldg(a.er + c0);
+    if (b + 32 < t) c1 = __ldg(a.col_idx + (b + 32 + lane < t ? b + 32 + lane : t - 1));
+  }
   for (int64_t base = b; base < t; base += 32) {
-    const int32_t cc = cn;
-    if (base + 32 < t) cn = __ldg(a.col_idx + (base + 32 + lane < t ? base + 32 + lane : t - 1));  // prefetch
+    const int32_t cc = c0;
+    const float erc = e0;
+    if (base + 32 < t) {  // distance-2 prefetch of the columns, distance 1 of their er
+      c0 = c1;
+      e0 = __ldg(a.er + c0);
+      if (base + 64 < t) c1 = __ldg(a.col_idx + (base + 64 + lane < t ? base + 64 + lane : t - 1));
+    }
     const int cnt = (int)(t - base < 32 ? t - base : 32);
+    const float z = eli + erc;
+    const float ev = lane < cnt ? gb_lrelu(z) : -INFINITY;
+    float cm = ev;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) cm = fmaxf(cm, __shfl_xor_sync(0xffffffffu, cm, o));
+    if (cm > m) {  // warp-uniform
+      const float f = __expf(m - cm);  // 0 on the first chunk (m = -inf)
+      S *= f;
+      Cw *= f;
+      D *= f;
+      m = cm;
+    }
+    const float w = lane < cnt ? __expf(ev - m) : 0.f;
+    const float ws = w * (z > 0.f ? 1.f : 0.2f);
+    S += w;
+    Cw += ws;
     const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
     for (int q = 0; q < steps; ++q) {
       int32_t j[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) j[u] = __shfl_sync(0xffffffffu, cc, q * G * U + u * G + grp);
-      float zv[U][NJ][4], erj[U];
+      float wu[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        erj[u] = __ldg(a.er + j[u]);
-        gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+        j[u] = __shfl_sync(0xffffffffu, cc, q * G * U + u * G + grp);
+        wu[u] = __shfl_sync(0xffffffffu, ws, q * G * U + u * G + grp);  // 0 past the chunk's end
       }
+      float zv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (q * G * U + u * G + grp < cnt) {
-          const float pd = gb_pdot<NJ>(xv, zv[u]);
-          const float z = eli + erj[u];
-          const float ev = gb_lrelu(z);
-          const float sl = z > 0.f ? 1.f : 0.2f;
-          if (ev > m) {
-            const float sc = __expf(m - ev);  // 0 on the first entry (m = -inf)
-            S = fmaf(S, sc, 1.f);
-            Cw = fmaf(Cw, sc, sl);
-            D = fmaf(D, sc, sl * pd);
-            m = ev;
-          } else {
-            const float w = __expf(ev - m);
-            S += w;
-            Cw = fmaf(w, sl, Cw);
-            D = fmaf(w * sl, pd, D);
-          }
-        }
-      }
+      for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+#pragma unroll
+      for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot<NJ>(xv, zv[u]), D);
     }
   }
-#pragma unroll
-  for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);  // lanes of a group share m
-#pragma unroll
-  for (int o = LPG; o < 32; o <<= 1) {  // merge the groups
-    const float m2 = __shfl_xor_sync(0xffffffffu, m, o);
-    const float S2 = __shfl_xor_sync(0xffffffffu, S, o), C2 = __shfl_xor_sync(0xffffffffu, Cw, o);
-    const float D2 = __shfl_xor_sync(0xffffffffu, D, o);
-    const float mn = fmaxf(m, m2);
-    const float f1 = m == -INFINITY ? 0.f : __expf(m - mn), f2 = m2 == -INFINITY ? 0.f : __expf(m2 - mn);
-    S = S * f1 + S2 * f2;
-    Cw = Cw * f1 + C2 * f2;
-    D = D * f1 + D2 * f2;
-    m = mn;
-  }
+  S = gb_warp_sum(S);
+  Cw = gb_warp_sum(Cw);
+  D = gb_warp_sum(D);
   if (seg >= 0) {
     if (lane == 0) a.seg_a[seg] = make_float4(m, S, Cw, D);
     return;
@@ -189,37 +189,52 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
   for (int j = 0; j < NJ; ++j)
 #pragma unroll
     for (int k = 0; k < 4; ++k) acc[j][k] = 0.f;
-  // der = Σ_lanes Σ α s' (lane share of dα) - Σ α s' c_i, reduced once per row
+  // der = Σ_lanes Σ α s' (lane share of dα) - Σ α s' c_i, reduced once per row.  The per-entry
+  // scalars are computed once, by the lane that loaded the entry's column: its record (gathered a
+  // chunk ahead), α and α·s'; the lane groups that gather the K-wide rows get them by shuffle, and
+  // the owner lane accumulates the α·s'·c_i correction itself.
   float dpart = 0.f, dcorr = 0.f;
-  int32_t cn = 0;
-  if (b < t) cn = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+  int32_t c0 = 0, c1 = 0;
+  float4 r0 = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (b < t) {
+    c0 = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
+    r0 = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)c0 * a.ldx + a.rec));
+    if (b + 32 < t) c1 = __ldg(a.col_idx + (b + 32 + lane < t ? b + 32 + lane : t - 1));
+  }
   for (int64_t base = b; base < t; base += 32) {
-    const int32_t cc = cn;
-    if (base + 32 < t) cn = __ldg(a.col_idx + (base + 32 + lane < t ? base + 32 + lane : t - 1));  // prefetch
+    const int32_t cc = c0;
+    const float4 rc = r0;
+    if (base + 32 < t) {  // distance-2 prefetch of the columns, distance 1 of their records
+      c0 = c1;
+      r0 = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)c0 * a.ldx + a.rec));
+      if (base + 64 < t) c1 = __ldg(a.col_idx + (base + 64 + lane < t ? base + 64 + lane : t - 1));
+    }
     const int cnt = (int)(t - base < 32 ? t - base : 32);
+    const float z = rc.x + erj;
+    const float al = lane < cnt ? __expf(gb_lrelu(z) - rc.y) * rc.z : 0.f;
+    const float as = al * (z > 0.f ? 1.f : 0.2f);
+    dcorr = fmaf(as, rc.w, dcorr);
     const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
     for (int q = 0; q < steps; ++q) {
       int32_t i[U];
+      float au[U], su[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) i[u] = __shfl_sync(0xffffffffu, cc, q * G * U + u * G + grp);
-      float4 st[U];
+      for (int u = 0; u < U; ++u) {
+        const int src = q * G * U + u * G + grp;
+        i[u] = __shfl_sync(0xffffffffu, cc, src);
+        au[u] = __shfl_sync(0xffffffffu, al, src);  // 0 past the chunk's end
+        su[u] = __shfl_sync(0xffffffffu, as, src);
+      }
       float xv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        st[u] = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)i[u] * a.ldx + a.rec));
-        gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
-      }
+      for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        const float z = st[u].x + erj;
-        const float alpha = (q * G * U + u * G + grp < cnt) ? __expf(gb_lrelu(z) - st[u].y) * st[u].z : 0.f;
-        const float as = alpha * (z > 0.f ? 1.f : 0.2f);
-        dpart = fmaf(as, gb_pdot<NJ>(xv[u], zr), dpart);
-        if (lg == 0) dcorr = fmaf(as, st[u].w, dcorr);
+        dpart = fmaf(su[u], gb_pdot<NJ>(xv[u], zr), dpart);
 #pragma unroll
         for (int j = 0; j < NJ; ++j)
 #pragma unroll
-          for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(alpha, xv[u][j][k], acc[j][k]);
+          for (int k = 0; k < 4; ++k) acc[j][k] = fmaf(au[u], xv[u][j][k], acc[j][k]);
       }
     }
   }
