@@ -487,7 +487,8 @@ def regret(G, spec, g, dev, comm, H, world, dist):
         fl = (G.SELECT_TRAINING | (0 if need_dH else G.SELECT_INPUT_LAYER)) if train else 0
         calib = DEFAULT_CALIB if os.path.exists(DEFAULT_CALIB) else None
         shape = G.shape_args(k1, k2, spec.get("hops", 2), spec.get("kh", 0))
-        sel, pred = G.granii_select_ex(g, model, shape, calib, fl)
+        sel, pred = G.granii_select_ex(g, model, shape, calib, fl | G.SELECT_REFINE)   # what GNN() runs
+        sel_model, _ = G.granii_select_ex(g, model, shape, calib, fl)                  # cost model alone
         sel_all, pred_all = G.granii_select_ex(g, model, shape, calib, fl | G.SELECT_NO_PREFILTER)
         sel_paper, _ = G.granii_select_ex(g, model, shape, calib, 0)   # forward-only selection, as the paper
         times = {}
@@ -522,6 +523,8 @@ def regret(G, spec, g, dev, comm, H, world, dist):
             "ms": times, "best": best, "selected": G.COMP_NAMES[sel],
             "selected_no_prefilter": G.COMP_NAMES[sel_all],
             "regret": times[G.COMP_NAMES[sel]] / times[best] - 1.0,
+            "selected_model_only": G.COMP_NAMES[sel_model],
+            "regret_model_only": times[G.COMP_NAMES[sel_model]] / times[best] - 1.0,
             "regret_no_prefilter": times[G.COMP_NAMES[sel_all]] / times[best] - 1.0,
             "selected_forward_only": G.COMP_NAMES[sel_paper],
             "regret_forward_only": times[G.COMP_NAMES[sel_paper]] / times[best] - 1.0,

@@ -285,6 +285,13 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
  * primitives of each GCN composition to its cost; INPUT_LAYER drops dH. */
 #define GRANII_SELECT_TRAINING 0x2u
 #define GRANII_SELECT_INPUT_LAYER 0x4u
+/* Extension: measured tie-break.  When the two best predictions are within 15 % and the best is
+ * below 5 ms (small, latency-bound layers, where the cost models are least accurate), the close
+ * candidates run once on zero-filled inputs of the layer's shape (forward, + backward with
+ * SELECT_TRAINING) on a private stream and the fastest is returned (predicted_ms stays the model's).
+ * Allocates and frees device memory, synchronises its own stream.  Ignored on partitioned graphs
+ * (every rank must pick the same composition). */
+#define GRANII_SELECT_REFINE 0x8u
 #define GRANII_MAX_CANDIDATES 8
 
 /*

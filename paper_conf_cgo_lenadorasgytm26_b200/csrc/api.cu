@@ -74,6 +74,124 @@ static granii_status check_shape(granii_model m, const granii_layer_args* a) {
   return GRANII_OK;
 }
 
+// ------------------------------------------------------------------ measured tie-break
+// GRANII_SELECT_REFINE (extension): the cost models are least accurate on small, latency-bound
+// layers, where a composition runs in well under a millisecond.  When the two best predictions
+// are within REFINE_MARGIN of each other and the best is below REFINE_MAX_MS, the close candidates
+// run once on zero-filled inputs of the layer's shape (forward; + backward when training) on a
+// private stream and the fastest measured one is kept.  Single GPU only (a partitioned selection
+// must agree on every rank; it stays model-only there).
+static constexpr double REFINE_MARGIN = 1.15, REFINE_MAX_MS = 5.0;
+
+static granii_status refine_choice(granii_graph g, granii_model m, const granii_layer_args* shape, uint32_t flags,
+                                   const int32_t* cand, const double* pred, int32_t n, granii_composition* out) {
+  if (g->world > 1 || n < 2) return GRANII_OK;
+  int best = 0;
+  for (int i = 1; i < n; ++i)
+    if (pred[i] < pred[best]) best = i;
+  if (!(pred[best] < REFINE_MAX_MS)) return GRANII_OK;
+  std::vector<int32_t> close;
+  for (int i = 0; i < n; ++i)
+    if (pred[i] <= REFINE_MARGIN * pred[best]) close.push_back(cand[i]);
+  if (close.size() < 2) return GRANII_OK;
+  const bool train = (flags & GRANII_SELECT_TRAINING) && (m == GRANII_GCN || m == GRANII_GAT);
+  const bool need_dh = train && !(flags & GRANII_SELECT_INPUT_LAYER);
+  const int64_t R = std::max<int64_t>(g->n_rows, 1), K1 = shape->K1, K2 = shape->K2;
+  const int64_t l1 = round_up(K1, 8), l2 = round_up(K2, 8);
+  const int64_t nw = m == GRANII_TAGCN ? (int64_t)(shape->hops + 1) * K1 * K2 : m == GRANII_GIN ? K1 * shape->Kh
+                                                                                                 : K1 * K2;
+  size_t ws = 0, sv = 0;
+  granii_layer_args a = *shape;
+  for (int32_t c : close) {
+    size_t w1 = 0, s1 = 0;
+    GR_TRY(layer_workspace(g, m, (granii_composition)c, &a, &w1, &s1));
+    ws = std::max(ws, w1);
+    sv = std::max(sv, s1);
+  }
+  // one allocation, carved: H | W | W2 | a_l | a_r | out | saved | dout | dH | dW | da_l | da_r | ws
+  const size_t fl = (size_t)R * l1 + nw + (m == GRANII_GIN ? (size_t)shape->Kh * K2 : 0) + 2 * K2 + (size_t)R * l2 +
+                    sv + (train ? (size_t)R * l2 + (need_dh ? (size_t)R * l1 : 0) + (size_t)K1 * K2 + 2 * K2 : 0);
+  const size_t bytes = round_up((int64_t)(fl * sizeof(float)), 256) + ws + 256;
+  char* base = nullptr;
+  cudaStream_t st = nullptr;
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  GR_CUDA(cudaMalloc(&base, bytes));
+  granii_status rc = GRANII_OK;
+  do {
+    if (cudaMemset(base, 0, bytes) != cudaSuccess || cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) {
+      rc = fail(GRANII_ERR_CUDA, "refine: setup failed");
+      break;
+    }
+    float* p = reinterpret_cast<float*>(base);
+    auto take = [&](size_t k) { float* q = p; p += k; return q; };
+    a.H = take((size_t)R * l1);
+    a.ldh = l1;
+    a.W = take(nw);
+    if (m == GRANII_GIN) a.W2 = take((size_t)shape->Kh * K2);
+    a.a_l = take(K2);
+    a.a_r = take(K2);
+    float* o = take((size_t)R * l2);
+    float* saved = sv ? take(sv) : nullptr;
+    float *dout = nullptr, *dH = nullptr, *dW = nullptr;
+    if (train) {
+      dout = take((size_t)R * l2);
+      if (need_dh) dH = take((size_t)R * l1);
+      dW = take((size_t)K1 * K2);
+      if (m == GRANII_GAT) {
+        a.d_a_l = take(K2);
+        a.d_a_r = take(K2);
+      }
+    }
+    a.workspace = base + round_up((int64_t)(fl * sizeof(float)), 256);
+    a.workspace_bytes = ws;
+    a.comm = nullptr;
+    float best_ms = 1e30f;
+    for (int32_t c : close) {
+      const granii_composition cc = (granii_composition)c;
+      auto run = [&]() -> granii_status {
+        GR_TRY(granii_layer_forward(g, m, cc, &a, o, l2, saved, st));
+        if (train) GR_TRY(granii_layer_backward(g, m, cc, &a, o, l2, dout, l2, saved, dH, l1, dW, st));
+        return GRANII_OK;
+      };
+      if ((rc = run()) != GRANII_OK) break;  // warm-up (first-touch of pool memory, caches)
+      cudaEventRecord(e0, st);
+      if ((rc = run()) != GRANII_OK || (rc = run()) != GRANII_OK) break;
+      cudaEventRecord(e1, st);
+      if (cudaEventSynchronize(e1) != cudaSuccess) {
+        rc = fail(GRANII_ERR_CUDA, "refine: timing failed");
+        break;
+      }
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, e0, e1);
+      if (ms < best_ms) {  // candidates come in composition-id order: ties keep the lower id (R12)
+        best_ms = ms;
+        *out = cc;
+      }
+    }
+  } while (false);
+  if (st) cudaStreamSynchronize(st);
+  if (e0) cudaEventDestroy(e0);
+  if (e1) cudaEventDestroy(e1);
+  if (st) cudaStreamDestroy(st);
+  cudaFree(base);
+  return rc;
+}
+
+static granii_status select_refined(granii_graph g, granii_model m, const granii_layer_args* a,
+                                    const char* calib_path, uint32_t flags, granii_composition* out,
+                                    int32_t* candidates, double* predicted_ms, int32_t* n_candidates) {
+  int32_t cand[GRANII_MAX_CANDIDATES];
+  double pred[GRANII_MAX_CANDIDATES];
+  int32_t n = 0;
+  GR_TRY(select_impl(g, m, a, calib_path, flags, out, cand, pred, &n));
+  if (candidates) std::memcpy(candidates, cand, sizeof(int32_t) * n);
+  if (predicted_ms) std::memcpy(predicted_ms, pred, sizeof(double) * n);
+  if (n_candidates) *n_candidates = n;
+  if (flags & GRANII_SELECT_REFINE) GR_TRY(refine_choice(g, m, a, flags, cand, pred, n, out));
+  return GRANII_OK;
+}
+
 #define API_BEGIN try {
 #define API_END                                                          \
   }                                                                      \
@@ -304,7 +422,7 @@ granii_status granii_select(granii_graph g, granii_model m, int64_t K1, int64_t 
   granii_layer_args a{};
   a.K1 = K1;
   a.K2 = K2;
-  return select_impl(g, m, &a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
+  return select_refined(g, m, &a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
   API_END
 }
 
@@ -315,7 +433,7 @@ granii_status granii_select_ex(granii_graph g, granii_model m, const granii_laye
   GR_ARG(g && out, "NULL argument");
   GR_ARG(m >= GRANII_GCN && m <= GRANII_GIN, "bad model");
   GR_TRY(check_shape(m, a));
-  return select_impl(g, m, a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
+  return select_refined(g, m, a, calib_path, flags, out, candidates, predicted_ms, n_candidates);
   API_END
 }
 

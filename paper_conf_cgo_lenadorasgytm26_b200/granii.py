@@ -43,7 +43,7 @@ for _m, _base in (("SGC", 32), ("TAGCN", 48), ("GIN", 64)):
         COMP_NAMES[_base + _i] = f"{_m}_{_v}"
 ACT_NONE, ACT_RELU = 0, 1
 ATTN_ADDITIVE, ATTN_DOT = 0, 1
-SELECT_NO_PREFILTER, SELECT_TRAINING, SELECT_INPUT_LAYER = 0x1, 0x2, 0x4
+SELECT_NO_PREFILTER, SELECT_TRAINING, SELECT_INPUT_LAYER, SELECT_REFINE = 0x1, 0x2, 0x4, 0x8
 MAX_CANDIDATES = 8
 NUM_FEATURES = 8
 

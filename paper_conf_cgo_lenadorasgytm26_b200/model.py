@@ -54,9 +54,11 @@ class GNN:
     """A stack of GCN/GAT layers on one (possibly row-partitioned) graph."""
 
     def __init__(self, graph: G.Graph, layers: list[LayerSpec], device, comm: G.Comm | None = None,
-                 calib_path: str | None = None, select_flags: int = 0, training: bool = False):
+                 calib_path: str | None = None, select_flags: int = G.SELECT_REFINE, training: bool = False):
         """training=True costs each candidate's backward too (extension; the paper selects on the
-        forward only, L340) and knows the input layer needs no dH."""
+        forward only, L340) and knows the input layer needs no dH.  select_flags defaults to the
+        measured tie-break of near-equal predictions on small layers (GRANII_SELECT_REFINE, single
+        GPU; pass 0 for the cost model alone)."""
         self.g, self.layers, self.device, self.comm = graph, layers, device, comm
         if calib_path is None and os.path.exists(DEFAULT_CALIB):
             calib_path = DEFAULT_CALIB

@@ -670,6 +670,22 @@ def test_softmax_xent_and_sgd(G, n, C):
     assert torch.equal(w.cpu(), 1 - 0.5 * torch.arange(100, dtype=torch.float32))
 
 
+@pytest.mark.parametrize("model,K1,K2,flags", [(0, 32, 256, 0), (1, 64, 256, 0), (1, 64, 256, 2 | 4),
+                                                  (1, 256, 32, 2), (3, 48, 16, 0), (4, 32, 16, 0)])
+def test_select_refine(G, model, K1, K2, flags):
+    """GRANII_SELECT_REFINE: the predictions are the model's, the choice is one of the candidates;
+    on near-tied small layers it is the measured faster one (forward, + backward when training)"""
+    c = case(G, "pubmed")
+    shape = G.shape_args(K1, K2, 2, K2 if model == G.GIN else 0)
+    s0, p0 = G.granii_select_ex(c.g, model, shape, None, flags)
+    s1, p1 = G.granii_select_ex(c.g, model, shape, None, flags | G.SELECT_REFINE)
+    assert p0 == p1 and s1 in p1
+    best = min(p0.values())
+    close = [k for k, v in p0.items() if v <= 1.15 * best]
+    if len(close) < 2 or best >= 5.0:
+        assert s1 == s0
+
+
 def test_select_candidates_are_the_offline_promoted_trees(G):
     """N4: the online selector's candidate sets (prefilter on, L237-L239) are exactly the trees
     the offline stage (offline.py, Algorithm 1 + pruning) promotes for each scenario"""
