@@ -197,6 +197,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-regret", action="store_true")
+    ap.add_argument("--no-cold", action="store_true", help="skip the warm / cold-L2 SpMM measurement")
     ap.add_argument("--comp", default=None, help="force compositions, e.g. 1,3 (skips the selector)")
     ap.add_argument("--cuda-graph", default="auto", choices=["auto", "on", "off"],
                     help="capture the step in a CUDA graph (auto: when an eager step takes < 5 ms)")
@@ -305,6 +306,13 @@ def main():
         launches = G.granii_launch_count() - launches0
     prof = G.granii_profile_read()
     G.granii_profile_enable(False)
+    # per-step spread: the same steps again, one event pair each (not the headline)
+    step_ms = []
+    for _ in range(args.steps):
+        step_ms.append(time_region(run, 1, stream))
+    step_ms.sort()
+    spread = {"p10": step_ms[len(step_ms) // 10], "p50": step_ms[len(step_ms) // 2],
+              "p90": step_ms[min(len(step_ms) - 1, (9 * len(step_ms)) // 10)]}
     if world > 1:
         dist.barrier()
         t = torch.tensor([ms], device=dev)
@@ -372,6 +380,7 @@ def main():
         "gpu_launches": int(launches),
         "roofline": roof,
         "per_primitive_ms": {k: v["ms"] / args.steps for k, v in prof.items()},
+        "step_ms_spread": spread,
         "overhead_ms": {"csr_create_incl_featurize": t_csr * 1e3, "select_all_layers": t_select * 1e3},
         "setup_s": setup_s,
     }
@@ -443,6 +452,10 @@ def main():
                                 "buffers; inputs double-buffered (step t+1's H2D on a copy stream under step t), "
                                 "serial_ms_per_step = copy then compute"}
 
+    # ---------------------------------------------------------------- SpMM warm vs cold L2
+    if world == 1 and not args.no_cold:
+        result["spmm_l2"] = spmm_cold_l2(G, g, dev, max(dims), stream)
+
     # ---------------------------------------------------------------- selector regret (rank 0 view)
     if not args.no_regret:
         result["selector"] = regret(G, spec, g, dev, comm, H, world, dist if world > 1 else None)
@@ -466,6 +479,29 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def spmm_cold_l2(G, g, dev, K, stream, reps=5):
+    """One unweighted SpMM with the D^-1/2 scalings at the step's widest K: warm (back to back) and
+    cold (a 2 x L2 = 252 MB buffer written between repetitions, outside the timed interval)."""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import alloc2d
+    X = alloc2d(g.n_rows, K, dev, fill=0.5)
+    Y = alloc2d(g.n_rows, K, dev)
+    dinv = G.granii_graph_dinv(g)
+    flush = torch.empty(63 * 1024 * 1024, dtype=torch.float32, device=dev)
+
+    def one():
+        G.granii_spmm(g, None, X, K, Y, dinv, dinv, 0)
+    one()
+    warm = time_region(one, reps, stream)
+    cold = []
+    for i in range(reps):
+        flush.fill_(float(i))
+        cold.append(time_region(one, 1, stream))
+    del X, Y, flush
+    return {"K": K, "warm_ms": warm, "cold_ms": sum(cold) / len(cold),
+            "how": "unweighted SpMM + row/col D^-1/2 at the widest layer width; cold = 252 MB (2 x L2) written "
+                   "before each repetition"}
 
 
 def regret(G, spec, g, dev, comm, H, world, dist):

@@ -109,7 +109,6 @@ struct In {
   double R, nnz, ncols, avg, l2, world, nseg;
   double xcols;  // rows of X an SpMM gathers from (a phased SpMM slices like the whole one: ncols)
   double maxd = 0, seg_len = 2048;  // longest row (featurizer feature 4) and the hub-segment length
-  double N = 0, top1 = 0;           // global nodes; share of entries in the top-1 % rows (feature 6)
 };
 
 static bool overlap_on() {
@@ -353,11 +352,10 @@ static In inputs_of(const granii_graph_s* g) {
     const double G = (double)g->world, N = (double)g->N, nnz = (double)g->nnz;
     return In{N / G, nnz / G, (double)g->n_cols, N > 0 ? nnz / N : 0.0, (double)di.l2_bytes, G,
               (double)std::max<int64_t>(g->n_seg_global, 0) / G, (double)g->n_cols, (double)g->features[4],
-              (double)g->seg_len, N, nnz > 0 ? (double)g->features[6] / nnz : 0.0};
+              (double)g->seg_len};
   }
   return In{(double)g->n_rows, (double)g->local_nnz, (double)g->n_cols, g->avg_deg(), (double)di.l2_bytes,
-            (double)g->world, (double)g->n_seg, (double)g->n_cols, (double)g->features[4], (double)g->seg_len,
-            (double)g->N, g->nnz > 0 ? (double)g->features[6] / (double)g->nnz : 0.0};
+            (double)g->world, (double)g->n_seg, (double)g->n_cols, (double)g->features[4], (double)g->seg_len};
 }
 
 granii_status select_impl(const granii_graph_s* g, granii_model model, const granii_layer_args* shape,
