@@ -454,7 +454,7 @@ def main():
 
     # ---------------------------------------------------------------- SpMM warm vs cold L2
     if world == 1 and not args.no_cold:
-        result["spmm_l2"] = spmm_cold_l2(G, g, dev, max(dims), stream)
+        result["spmm_l2"] = spmm_cold_l2(G, g, dev, dims[1], stream)
 
     # ---------------------------------------------------------------- selector regret (rank 0 view)
     if not args.no_regret:
@@ -482,7 +482,7 @@ def main():
 
 
 def spmm_cold_l2(G, g, dev, K, stream, reps=5):
-    """One unweighted SpMM with the D^-1/2 scalings at the step's widest K: warm (back to back) and
+    """One unweighted SpMM with the D^-1/2 scalings at the first layer's output width: warm (back to back) and
     cold (a 2 x L2 = 252 MB buffer written between repetitions, outside the timed interval)."""
     from paper_conf_cgo_lenadorasgytm26_b200.model import alloc2d
     X = alloc2d(g.n_rows, K, dev, fill=0.5)
@@ -500,7 +500,7 @@ def spmm_cold_l2(G, g, dev, K, stream, reps=5):
         cold.append(time_region(one, 1, stream))
     del X, Y, flush
     return {"K": K, "warm_ms": warm, "cold_ms": sum(cold) / len(cold),
-            "how": "unweighted SpMM + row/col D^-1/2 at the widest layer width; cold = 252 MB (2 x L2) written "
+            "how": "unweighted SpMM + row/col D^-1/2 at the first layer's output width; cold = 252 MB (2 x L2) written "
                    "before each repetition"}
 
 
