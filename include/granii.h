@@ -349,6 +349,15 @@ granii_status granii_comm_create_stub(int32_t rank, int32_t world, granii_comm* 
  * buffer) and the number of collective calls.  Host-side counters, any transport. */
 granii_status granii_comm_stats(granii_comm c, uint64_t* bytes_in, uint64_t* calls);
 granii_status granii_comm_destroy(granii_comm c);
+/* The communicator's two data collectives, as the layers use them (north_star (4)), for callers
+ * that exchange their own buffers (e.g. all-reducing a gradient they computed themselves):
+ *   all-gather: recv = [block of rank 0 | ... | block of rank G-1], `count` floats per block,
+ *               send may be recv + rank * count (in place);
+ *   all-reduce: buf = Σ_ranks buf (fp32 sum, in place).
+ * Device pointers, stream-ordered on `stream`; NCCL, loopback or stub transport (the stub moves
+ * no data).  Errors: INVALID_ARG (NULL), NCCL (transport failure). */
+granii_status granii_comm_allgather(granii_comm c, const float* d_send, float* d_recv, size_t count, void* stream);
+granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t count, void* stream);
 
 /* ------------------------------------------------------------------------ */
 /* Training-step helpers around the layers (not selected by GRANII)          */

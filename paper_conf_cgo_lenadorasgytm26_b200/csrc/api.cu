@@ -466,6 +466,14 @@ granii_status granii_comm_stats(granii_comm c, uint64_t* bytes_in, uint64_t* cal
   return GRANII_OK;
 }
 granii_status granii_comm_destroy(granii_comm c) { return comm_destroy(c); }
+granii_status granii_comm_allgather(granii_comm c, const float* d_send, float* d_recv, size_t count, void* stream) {
+  GR_ARG(c && d_send && d_recv, "NULL argument");
+  return comm_allgather(c, d_send, d_recv, count, (cudaStream_t)stream);
+}
+granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t count, void* stream) {
+  GR_ARG(c && d_buf, "NULL argument");
+  return comm_allreduce_sum(c, d_buf, count, (cudaStream_t)stream);
+}
 
 granii_status granii_softmax_xent(int64_t rows, int64_t C, const float* d_Z, int64_t ldz, const int32_t* d_y,
                                   int64_t n_total, float* d_dZ, int64_t lddz, float* d_loss, void* stream) {

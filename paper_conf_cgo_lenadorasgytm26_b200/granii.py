@@ -104,6 +104,8 @@ _SIGS = {
     "granii_comm_create_local": ([_i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_comm_create_stub": ([_i32, _i32, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_comm_stats": ([_p, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)], ctypes.c_int),
+    "granii_comm_allgather": ([_p, _p, _p, _sz, _p], ctypes.c_int),
+    "granii_comm_allreduce_sum": ([_p, _p, _sz, _p], ctypes.c_int),
     "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
     "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
     "granii_profile_enable": ([_i32], ctypes.c_int),
@@ -361,6 +363,16 @@ def granii_comm_create(uid: bytes, rank: int, world: int) -> Comm:
     h = _p()
     _check(_lib.granii_comm_create(buf, rank, world, ctypes.byref(h)), "granii_comm_create")
     return Comm(h.value, rank, world)
+
+
+def granii_comm_allgather(c: Comm, send: torch.Tensor, recv: torch.Tensor, count: int, stream=None):
+    _check(_lib.granii_comm_allgather(c.handle, _ptr(send), _ptr(recv), count, _stream(stream)),
+           "granii_comm_allgather")
+
+
+def granii_comm_allreduce_sum(c: Comm, buf: torch.Tensor, stream=None):
+    _check(_lib.granii_comm_allreduce_sum(c.handle, _ptr(buf), buf.numel(), _stream(stream)),
+           "granii_comm_allreduce_sum")
 
 
 def granii_comm_create_local(world: int) -> list:

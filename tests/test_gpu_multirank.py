@@ -319,3 +319,49 @@ def test_comm_stats_count_the_exchanged_bytes(G):
         ld = (K2 + 7) // 8 * 8
         assert fb == (world - 1) * mr * ld * 4 and fc == world
         assert bb - fb == (world - 1) * mr * ld * 4 + int(2.0 * K1 * K2 * 4 * (world - 1) / world)
+
+
+def test_comm_collectives_nccl_one_rank_and_loopback(G):
+    """The public collectives through both real transports: a 1-rank NCCL communicator (the library
+    dlopens the NCCL PyTorch loaded and calls ncclAllGather / ncclAllReduce on the caller's stream;
+    one rank is all a single-GPU box can form) and a 3-rank loopback group (one thread per rank)"""
+    n = 1000
+    x = torch.arange(n, dtype=torch.float32, device=DEV)
+    comm = G.granii_comm_create(G.granii_comm_unique_id(), 0, 1)
+    recv = torch.full((n,), -1.0, device=DEV)
+    G.granii_comm_allgather(comm, x, recv, n)
+    buf = x.clone()
+    G.granii_comm_allgather(comm, buf, buf, n)  # in place
+    red = x.clone()
+    G.granii_comm_allreduce_sum(comm, red)
+    torch.cuda.synchronize()
+    assert torch.equal(recv, x) and torch.equal(buf, x) and torch.equal(red, x)
+    del comm
+    world = 3
+    comms = G.granii_comm_create_local(world)
+    outs, sums, errs = [None] * world, [None] * world, []
+
+    def worker(r):
+        try:
+            torch.cuda.set_device(DEV)
+            st = torch.cuda.Stream(device=DEV)
+            with torch.cuda.stream(st):
+                all_ = torch.zeros(world * n, device=DEV)
+                all_[r * n:(r + 1) * n] = x + 1000.0 * r
+                G.granii_comm_allgather(comms[r], all_[r * n:(r + 1) * n], all_, n, st)
+                v = x * (r + 1)
+                G.granii_comm_allreduce_sum(comms[r], v, st)
+            st.synchronize()
+            outs[r], sums[r] = all_.cpu(), v.cpu()
+        except Exception as e:  # pragma: no cover - surfaced below
+            errs.append(e)
+    th = [threading.Thread(target=worker, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errs, errs
+    want = torch.cat([x.cpu() + 1000.0 * r for r in range(world)])
+    for r in range(world):
+        assert torch.equal(outs[r], want)
+        assert torch.equal(sums[r], x.cpu() * 6)
