@@ -255,8 +255,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           tc_fence_after();
           const uint32_t ahi = tA0 + ts * 64, alo = ahi + 32;
           const uint32_t bh = smem_u32(sB + sb * Cfg::B_STAGE), bl = bh + Cfg::B_BYTES;
+          // the last k-block of a K that is not a multiple of 32 (K1 = 100, 602) only issues the
+          // 8-wide steps that hold data: the rest would multiply TMA zero fill by zero B rows
+          const int ksteps = min(TC_BK / 8, (K - kb * TC_BK + 7) / 8);
 #pragma unroll
           for (int k = 0; k < TC_BK / 8; ++k) {  // tf32: K = 8 per MMA (8 TMEM columns, 32 B of B rows)
+            if (k >= ksteps) break;
             const uint64_t dbh = desc_sw128(bh + k * 32), dbl = desc_sw128(bl + k * 32);
             mma_tf32_ta(acc, ahi + k * 8, dbh, idesc, (kb | k) ? 1u : 0u);
             mma_tf32_ta(acc, ahi + k * 8, dbl, idesc, 1u);
