@@ -181,7 +181,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   using Cfg = TcCfg<BN>;
   constexpr int RA = Cfg::RA, SB = Cfg::SB, TS = Cfg::TSTAGES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  // 1 KB-aligned base by pointer arithmetic on the __shared__ array (an integer round trip would
+  // lose the address space and turn every staging access into a generic LD / ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sA = smem;                                   // RA x 16 KB
   uint8_t* sB = smem + RA * Cfg::A_BYTES;               // SB x (B_hi | B_lo)
   float* stage_out = (float*)(sB + SB * Cfg::B_STAGE);  // epilogue staging
@@ -335,12 +337,19 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 #pragma unroll
         for (int j = 0; j < 32; ++j) v[j] *= rsc;
         if (ep.att_l || ep.att_r) {
+          // lane j holds a_l / a_r of this chunk's column j (one coalesced load per chunk, 0 past N),
+          // broadcast by shuffle instead of a uniform global load per element
+          const bool cj = cb + lane < N && c0 + lane < BN;
+          const float alj = (ep.att_l && cj) ? __ldg(ep.att_l + cb + lane) : 0.f;
+          const float arj = (ep.att_r && cj) ? __ldg(ep.att_r + cb + lane) : 0.f;
 #pragma unroll
-          for (int j = 0; j < 32; ++j)
-            if (cb + j < N && c0 + j < BN) {
-              if (ep.att_l) el = fmaf(v[j], __ldg(ep.att_l + cb + j), el);
-              if (ep.att_r) er = fmaf(v[j], __ldg(ep.att_r + cb + j), er);
+          for (int j = 0; j < 32; ++j) {
+            const float a_l = __shfl_sync(0xffffffffu, alj, j), a_r = __shfl_sync(0xffffffffu, arj, j);
+            if (c0 + j < BN) {  // v[j] past the tile's columns was never loaded
+              el = fmaf(v[j], a_l, el);
+              er = fmaf(v[j], a_r, er);
             }
+          }
         }
         if (ep.relu)
 #pragma unroll
@@ -440,7 +449,9 @@ __global__ void __launch_bounds__(192, 1)
   using Cfg = TnCfg<BN>;
   constexpr int S = Cfg::STAGES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  // 1 KB-aligned base by pointer arithmetic on the __shared__ array (an integer round trip would
+  // lose the address space and turn every staging access into a generic LD / ST)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = (uint64_t*)(smem + S * Cfg::STAGE);
   uint64_t* full = bars;
   uint64_t* conv = bars + S;
