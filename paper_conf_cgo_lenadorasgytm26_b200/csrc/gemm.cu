@@ -109,6 +109,15 @@ __device__ __forceinline__ float tf32_rna(float x) {
   return __uint_as_float(r);
 }
 
+// The 3xTF32 split of the hot converters: hi = x rounded half-up (on the magnitude) to 10 mantissa
+// bits by integer add + mask, lo = x - hi (exact in fp32), passed with all its bits -- the tf32 MMA
+// reads the top 19 bits of every operand, so lo is truncated there.  3 instructions per element
+// (cvt.rna.tf32.f32 expands to ~5 on sm_100a, and the split needed two of them); finite inputs.
+__device__ __forceinline__ void tf32_split(float x, float& hi, float& lo) {
+  hi = __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+  lo = x - hi;
+}
+
 // ======================================================================= tcgen05 kernel
 constexpr int TC_BM = 128, TC_BK = 32;  // 32 fp32 = one 128-byte swizzle row
 
@@ -293,9 +302,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           const float xs[4] = {x.x, x.y, x.z, x.w};
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
-            const float h = tf32_rna(xs[q]);
+            float h, l;
+            tf32_split(xs[q], h, l);
             hi[c * 4 + q] = __float_as_uint(h);
-            lo[c * 4 + q] = __float_as_uint(tf32_rna(xs[q] - h));
+            lo[c * 4 + q] = __float_as_uint(l);
           }
         }
         fence_proxy_async();            // our generic reads before the TMA's next async write
@@ -535,10 +545,10 @@ __global__ void __launch_bounds__(192, 1)
       for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) {
         const float4 x = ahp[i];
         float4 h, l;
-        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
-        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
-        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
-        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
+        tf32_split(x.x, h.x, l.x);
+        tf32_split(x.y, h.y, l.y);
+        tf32_split(x.z, h.z, l.z);
+        tf32_split(x.w, h.w, l.w);
         ahp[i] = h;
         alp[i] = l;
       }
@@ -546,10 +556,10 @@ __global__ void __launch_bounds__(192, 1)
       for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) {
         const float4 x = bhp[i];
         float4 h, l;
-        h.x = tf32_rna(x.x); l.x = tf32_rna(x.x - h.x);
-        h.y = tf32_rna(x.y); l.y = tf32_rna(x.y - h.y);
-        h.z = tf32_rna(x.z); l.z = tf32_rna(x.z - h.z);
-        h.w = tf32_rna(x.w); l.w = tf32_rna(x.w - h.w);
+        tf32_split(x.x, h.x, l.x);
+        tf32_split(x.y, h.y, l.y);
+        tf32_split(x.z, h.z, l.z);
+        tf32_split(x.w, h.w, l.w);
         bhp[i] = h;
         blp[i] = l;
       }
