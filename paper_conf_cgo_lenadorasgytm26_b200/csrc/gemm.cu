@@ -344,8 +344,9 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           tmem_ld16(tmem + (uint32_t)(buf * Cfg::ACC_COLS) + ((uint32_t)(quad * 32) << 16) + c0 + 16,
                     *(float(*)[16])(v + 16));
         const int cb = n0 + c0;
+        if (ep.row_scale)
 #pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] *= rsc;
+          for (int j = 0; j < 32; ++j) v[j] *= rsc;
         if (ep.att_l || ep.att_r) {
           // lane j holds a_l / a_r of this chunk's column j (one coalesced load per chunk, 0 past N),
           // broadcast by shuffle instead of a uniform global load per element
