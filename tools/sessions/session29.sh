@@ -1,5 +1,5 @@
 set -u
-M=gpurun_out/s29; mkdir -p $M; R=/tmp/reps; mkdir -p $R
+M=gpurun_out/${SESS:-s29}; mkdir -p $M; R=/tmp/reps; mkdir -p $R
 B="python bench.py --workload products-gcn2-infer --steps 1 --warmup 2 --no-e2e --no-regret --no-cpu --no-cold --cuda-graph off"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_gemm_tc -s 2 -c 2 -o $R/pgemm $B > $M/ncu.log 2>&1; echo "ncu rc=$?"
 python tools/ncu_summary.py $R/pgemm.ncu-rep > $M/pgemm_summary.json
