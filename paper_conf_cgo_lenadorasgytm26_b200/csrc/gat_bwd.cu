@@ -58,6 +58,28 @@ __device__ __forceinline__ void gb_load_row(const float* __restrict__ p, int lg,
   }
 }
 
+// K % 4 == 0: the gathered K-wide row without per-element masks -- lanes past the row re-read
+// its last vector (finite data that only ever meets the zeros of the masked register-resident row,
+// or feeds columns that are never stored)
+template <int LPG, int NJ>
+__device__ __forceinline__ void gb_load_row_cl(const float* __restrict__ p, int lg, int64_t K, float (&v)[NJ][4]) {
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    const int64_t col = 4 * (int64_t)(lg + j * LPG);
+    const float4 t = __ldg(reinterpret_cast<const float4*>(p + (col < K ? col : K - 4)));
+    v[j][0] = t.x;
+    v[j][1] = t.y;
+    v[j][2] = t.z;
+    v[j][3] = t.w;
+  }
+}
+
+template <int LPG, int NJ, bool CL>
+__device__ __forceinline__ void gb_gather_row(const float* __restrict__ p, int lg, int64_t K, float (&v)[NJ][4]) {
+  if constexpr (CL) gb_load_row_cl<LPG, NJ>(p, lg, K, v);
+  else gb_load_row<LPG, NJ>(p, lg, K, v);
+}
+
 // this lane's share of <x, y>; never reduced per entry: every use is linear in the dot, so
 // the lane shares are accumulated and reduced once per row
 template <int NJ>
@@ -95,7 +117,7 @@ __global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, 
 // per-column scalars with one coalesced load (the next chunk is prefetched while this one is
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
-template <int LPG, int NJ, int U>
+template <int LPG, int NJ, int U, bool CL = false>
 __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
@@ -156,7 +178,7 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
       }
       float zv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
 #pragma unroll
       for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot<NJ>(xv, zv[u]), D);
     }
@@ -175,7 +197,7 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
   }
 }
 
-template <int LPG, int NJ, int U>
+template <int LPG, int NJ, int U, bool CL = false>
 __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
@@ -227,7 +249,7 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
       }
       float xv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         dpart = fmaf(su[u], gb_pdot<NJ>(xv[u], zr), dpart);
@@ -406,7 +428,7 @@ __device__ __forceinline__ void gat_b_group_row(const GatBwdArgs& a, int64_t t0,
 
 // One launch covers both schedules: warps [0, n_wide) take the wide rows order[0 .. n_wide)
 // (all rows of a dense graph), the remaining warps take G rows each, one per lane group.
-template <int LPG, int NJ, int U, int MINB = 0>
+template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
 __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))))
     k_gat_bwd_a(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
@@ -420,10 +442,10 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 4 : (NJ <= 4
     return;
   }
   const bool sg = w < a.n_seg;
-  gat_a_warp_row<LPG, NJ, U>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
+  gat_a_warp_row<LPG, NJ, U, CL>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
 }
 
-template <int LPG, int NJ, int U, int MINB = 0>
+template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
 __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 3 : (NJ <= 8 ? 2 : 1))) k_gat_bwd_b(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31;
@@ -436,7 +458,7 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 3 : (NJ <= 8
     return;
   }
   const bool sg = w < a.n_seg;
-  gat_b_warp_row<LPG, NJ, U>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
+  gat_b_warp_row<LPG, NJ, U, CL>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
 }
 
 // hub rows: merge the segments' online-softmax states in fixed order -> del and the row record
@@ -475,15 +497,15 @@ __global__ void k_gat_b_combine(GatBwdArgs a) {
   }
 }
 
-template <int LPG, int NJ, int U, int MINB = 0>
+template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
 static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
   constexpr int G = 32 / LPG;
   const int64_t warps = a.n_seg + a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
   const unsigned blocks = (unsigned)std::max<int64_t>(1, ceil_div(warps, 8));
   if (pass == 0)
-    k_gat_bwd_a<LPG, NJ, U, MINB><<<blocks, 256, 0, st>>>(a);
+    k_gat_bwd_a<LPG, NJ, U, MINB, CL><<<blocks, 256, 0, st>>>(a);
   else
-    k_gat_bwd_b<LPG, NJ, U, MINB><<<blocks, 256, 0, st>>>(a);
+    k_gat_bwd_b<LPG, NJ, U, MINB, CL><<<blocks, 256, 0, st>>>(a);
 }
 
 granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
@@ -558,6 +580,11 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
 
 static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cudaStream_t st) {
   const int64_t K = b.K;
+  // K % 4 == 0: pass A on warp-per-row graphs gathers the Z rows without per-element masks
+  // (products K=100: 9.4 -> 7.7 ms; GRANII_GATBWD_CL=0: masked).  Pass B keeps the masked loader:
+  // unmasked it needs 3 blocks / SM to avoid spills and loses (9.4 -> 9.9 ms).
+  const char* ce = getenv("GRANII_GATBWD_CL");
+  const bool cl = K % 4 == 0 && pass == 0 && !(ce && ce[0] == '0');
   // tuning hook GRANII_GATBWD="LPG,NJ,U" (tools: bench.py per_primitive_ms), if it covers K
   if (const char* e = getenv("GRANII_GATBWD")) {
     int l = 0, n = 0, u = 0, mb = 0;
@@ -597,17 +624,27 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
   // pass B on warp-per-row graphs at 4 blocks / SM (64 registers, a few spilled): products K=47
   // 6.76 -> 6.22 ms, K=100 10.7 -> 10.3 ms (pass A is slower there)
   else if (K <= 64) {
-    if (pass == 1 && dense) gb_launch<8, 2, 2, 4>(pass, b, st);
-    else gb_launch<8, 2, 2>(pass, b, st);
+    if (pass == 1 && dense) {
+      gb_launch<8, 2, 2, 4>(pass, b, st);
+    } else if (dense && cl) {
+      gb_launch<8, 2, 2, 0, true>(pass, b, st);
+    } else {
+      gb_launch<8, 2, 2>(pass, b, st);
+    }
   }
   // warp-per-row graphs (products-shaped sweep): 16-lane groups up to K = 128 (K=100: A 10.9 -> 9.8,
   // B 13.0 -> 10.5 ms vs <8,4,2>); pass A keeps one entry per group in flight beyond K = 128 (K=256
   // 18.8 -> 18.3 ms, K=512 39.1 -> 35.2 ms).  Group-per-row graphs keep more rows per warp (pubmed-
   // shaped K=256: <32,2,1> for pass A cost 0.19 -> 0.25 ms)
   else if (K <= 128) {
-    if (dense && pass == 1) gb_launch<16, 2, 2, 4>(pass, b, st);
-    else if (dense) gb_launch<16, 2, 2>(pass, b, st);
-    else gb_launch<8, 4, 2>(pass, b, st);
+    if (dense && pass == 1) {
+      gb_launch<16, 2, 2, 4>(pass, b, st);
+    } else if (dense) {
+      if (cl) gb_launch<16, 2, 2, 0, true>(pass, b, st);
+      else gb_launch<16, 2, 2>(pass, b, st);
+    } else {
+      gb_launch<8, 4, 2>(pass, b, st);
+    }
   } else if (K <= 256) {
     if (pass == 0 && dense) gb_launch<32, 2, 1>(pass, b, st);
     else gb_launch<16, 4, 2>(pass, b, st);
