@@ -646,10 +646,12 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
       gb_launch<8, 4, 2>(pass, b, st);
     }
   } else if (K <= 256) {
-    if (pass == 0 && dense) gb_launch<32, 2, 1>(pass, b, st);
+    if (pass == 0 && dense && cl) gb_launch<32, 2, 1, 0, true>(pass, b, st);
+    else if (pass == 0 && dense) gb_launch<32, 2, 1>(pass, b, st);
     else gb_launch<16, 4, 2>(pass, b, st);
   } else if (K <= 512) {
-    if (pass == 0 && dense) gb_launch<32, 4, 1>(pass, b, st);
+    if (pass == 0 && dense && cl) gb_launch<32, 4, 1, 0, true>(pass, b, st);
+    else if (pass == 0 && dense) gb_launch<32, 4, 1>(pass, b, st);
     else gb_launch<32, 4, 2>(pass, b, st);
   }
   else if (K <= 1024) gb_launch<32, 8, 1>(pass, b, st);
