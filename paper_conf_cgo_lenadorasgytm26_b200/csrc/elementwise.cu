@@ -9,44 +9,81 @@ namespace granii {
 
 static unsigned blocks_for(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, 256), 148 * 16)); }
 
-__global__ void k_relu_mask(int64_t rows, int64_t K, const float* __restrict__ out, int64_t ldo,
-                            const float* __restrict__ g, int64_t ldg, float* __restrict__ dst, int64_t ldd) {
-  const int64_t total = rows * K;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t r = i / K, k = i % K;
-    dst[r * ldd + k] = out[r * ldo + k] > 0.f ? g[r * ldg + k] : 0.f;   // ReLU'(0) = 0
+// Row-wise helpers: lane groups of L = 2^lg lanes own a row (L = the smallest power of two >= the
+// row's vector count, at most 32), so no per-element 64-bit division; 16-byte accesses when every
+// row start is 16-byte aligned (V = 4). Loads of one thread stay independent across the unrolled
+// column loop, which keeps enough bytes in flight per SM for HBM.
+template <int V> struct Vec;
+template <> struct Vec<4> {
+  using T = float4;
+  __device__ static T ld(const float* p) { return *reinterpret_cast<const float4*>(p); }
+  __device__ static void st(float* p, T v) { *reinterpret_cast<float4*>(p) = v; }
+  __device__ static float& at(T& v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
+};
+template <> struct Vec<1> {
+  using T = float;
+  __device__ static T ld(const float* p) { return *p; }
+  __device__ static void st(float* p, T v) { *p = v; }
+  __device__ static float& at(T& v, int) { return v; }
+};
+
+// dst = (out == NULL || out > 0) ? g * rs[r] : 0  -- ReLU' mask (optional, ReLU'(0) = 0) fused with an
+// optional row scale (the inner D^-1/2 of the DYN_UPD backward, so its SpMM needs no column scale);
+// out == rs == NULL is a padded row copy (g * 1.f is exact)
+template <int V>
+__global__ void __launch_bounds__(256) k_scale_mask(int64_t rows, int Kv, int lg, const float* __restrict__ out,
+                                                    int64_t ldo, const float* __restrict__ g, int64_t ldg,
+                                                    const float* __restrict__ rs, float* __restrict__ dst,
+                                                    int64_t ldd) {
+  using VT = Vec<V>;
+  const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int lig = threadIdx.x & ((1 << lg) - 1);
+  const int64_t ngrp = ((int64_t)gridDim.x * blockDim.x) >> lg;
+  for (int64_t r = tid >> lg; r < rows; r += ngrp) {
+    const float s = rs ? rs[r] : 1.f;
+#pragma unroll 2
+    for (int k = lig; k < Kv; k += 1 << lg) {
+      typename VT::T v = VT::ld(g + r * ldg + (int64_t)k * V);
+      typename VT::T o;
+      if (out) o = VT::ld(out + r * ldo + (int64_t)k * V);
+#pragma unroll
+      for (int i = 0; i < V; ++i) {
+        const float x = VT::at(v, i) * s;
+        VT::at(v, i) = (!out || VT::at(o, i) > 0.f) ? x : 0.f;
+      }
+      VT::st(dst + r * ldd + (int64_t)k * V, v);
+    }
   }
 }
 
-// dst = (out == NULL || out > 0) ? g * rs[r] : 0  -- ReLU' mask (optional) fused with an
-// optional row scale (the inner D^-1/2 of the DYN_UPD backward, so its SpMM needs no column scale)
-__global__ void k_scale_mask(int64_t rows, int64_t K, const float* __restrict__ out, int64_t ldo,
-                             const float* __restrict__ g, int64_t ldg, const float* __restrict__ rs,
-                             float* __restrict__ dst, int64_t ldd) {
-  const int64_t total = rows * K;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t r = i / K, k = i % K;
-    const float v = g[r * ldg + k] * (rs ? rs[r] : 1.f);
-    dst[r * ldd + k] = (!out || out[r * ldo + k] > 0.f) ? v : 0.f;
-  }
+static inline bool al16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+static void rowwise_shape(int64_t rows, int64_t K, bool v4, int* Kv, int* lg, unsigned* blocks) {
+  *Kv = (int)(v4 ? K / 4 : K);
+  int l = 0;
+  while (l < 5 && (1 << l) < *Kv) ++l;
+  *lg = l;
+  *blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows << l, 256), 148 * 16));
+}
+
+static granii_status scale_mask_impl(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g,
+                                     int64_t ldg, const float* rs, float* dst, int64_t ldd, cudaStream_t st) {
+  const bool v4 = K % 4 == 0 && ldg % 4 == 0 && ldd % 4 == 0 && al16(g) && al16(dst) &&
+                  (!out || (ldo % 4 == 0 && al16(out)));
+  int Kv, lg;
+  unsigned blocks;
+  rowwise_shape(rows, K, v4, &Kv, &lg, &blocks);
+  if (v4) k_scale_mask<4><<<blocks, 256, 0, st>>>(rows, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
+  else k_scale_mask<1><<<blocks, 256, 0, st>>>(rows, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
 }
 
 granii_status launch_scale_mask(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
                                 const float* rs, float* dst, int64_t ldd, cudaStream_t st) {
   if (rows * K == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, (out ? 12.0 : 8.0) * rows * K, 0.0, 1);
-  k_scale_mask<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, out, ldo, g, ldg, rs, dst, ldd);
-  GR_CHECK_LAUNCH();
-  return GRANII_OK;
-}
-
-__global__ void k_copy_rows(int64_t rows, int64_t K, const float* __restrict__ src, int64_t lds,
-                            float* __restrict__ dst, int64_t ldd) {
-  const int64_t total = rows * K;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t r = i / K, k = i % K;
-    dst[r * ldd + k] = src[r * lds + k];
-  }
+  return scale_mask_impl(rows, K, out, ldo, g, ldg, rs, dst, ldd, st);
 }
 
 // one warp per row
@@ -84,18 +121,14 @@ granii_status launch_relu_mask(int64_t rows, int64_t K, const float* out, int64_
                                float* dst, int64_t ldd, cudaStream_t st) {
   if (rows * K == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, 12.0 * rows * K, 0.0, 1);
-  k_relu_mask<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, out, ldo, g, ldg, dst, ldd);
-  GR_CHECK_LAUNCH();
-  return GRANII_OK;
+  return scale_mask_impl(rows, K, out, ldo, g, ldg, nullptr, dst, ldd, st);
 }
 
 granii_status launch_copy_rows(int64_t rows, int64_t K, const float* src, int64_t lds, float* dst, int64_t ldd,
                                cudaStream_t st) {
   if (rows * K == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, 8.0 * rows * K, 0.0, 1);
-  k_copy_rows<<<blocks_for(rows * K), 256, 0, st>>>(rows, K, src, lds, dst, ldd);
-  GR_CHECK_LAUNCH();
-  return GRANII_OK;
+  return scale_mask_impl(rows, K, nullptr, 0, src, lds, nullptr, dst, ldd, st);
 }
 
 struct RankPtrs {

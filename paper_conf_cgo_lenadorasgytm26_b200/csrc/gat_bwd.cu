@@ -94,22 +94,45 @@ __device__ __forceinline__ float gb_pdot(const float (&x)[NJ][4], const float (&
 
 __device__ __forceinline__ float gb_lrelu(float z) { return z > 0.f ? z : 0.2f * z; }
 
-// dY = dout ⊙ σ'(out) and c_r = <dY_r, out_r> (= <dY_r, Y_r>: where ReLU clips, dY = 0); warp per row
-__global__ void k_gat_prep(int64_t R, int64_t K, const float* __restrict__ out, int64_t ldo,
-                           const float* __restrict__ g, int64_t ldg, int relu, float* __restrict__ dY, int64_t ldd,
-                           float* __restrict__ c) {
-  const int lane = threadIdx.x & 31;
+// dY = dout ⊙ σ'(out) and c_r = <dY_r, out_r> (= <dY_r, Y_r>: where ReLU clips, dY = 0). Lane groups of
+// L = 2^lg lanes own a row (L = the smallest power of two >= the row's vector count, at most 32), with
+// 16-byte accesses when every row start is aligned (V = 4); the row loop is warp-uniform so the group's
+// shuffle reduction never diverges.
+template <int V>
+__global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int Kv, int lg, const float* __restrict__ out,
+                                                  int64_t ldo, const float* __restrict__ g, int64_t ldg, int relu,
+                                                  float* __restrict__ dY, int64_t ldd, float* __restrict__ c) {
+  const int L = 1 << lg, lane = threadIdx.x & 31, lig = lane & (L - 1);
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < R; r += nw) {
+  const int rpw = 32 >> lg;  // rows per warp
+  for (int64_t rb = warp * rpw; rb < R; rb += nw * rpw) {
+    const int64_t r = rb + (lane >> lg);
     float s = 0.f;
-    for (int64_t k = lane; k < K; k += 32) {
-      const float o = out[r * ldo + k];
-      const float d = (!relu || o > 0.f) ? g[r * ldg + k] : 0.f;  // ReLU'(0) = 0
-      dY[r * ldd + k] = d;
-      s = fmaf(d, o, s);
+    if (r < R) {
+#pragma unroll 2
+      for (int k = lig; k < Kv; k += L) {
+        float o[V], d[V];
+        if constexpr (V == 4) {
+          const float4 o4 = *reinterpret_cast<const float4*>(out + r * ldo + (int64_t)k * 4);
+          const float4 g4 = *reinterpret_cast<const float4*>(g + r * ldg + (int64_t)k * 4);
+          o[0] = o4.x, o[1] = o4.y, o[2] = o4.z, o[3] = o4.w;
+          d[0] = g4.x, d[1] = g4.y, d[2] = g4.z, d[3] = g4.w;
+        } else {
+          o[0] = out[r * ldo + k];
+          d[0] = g[r * ldg + k];
+        }
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+          if (relu && !(o[i] > 0.f)) d[i] = 0.f;  // ReLU'(0) = 0
+          s = fmaf(d[i], o[i], s);
+        }
+        if constexpr (V == 4) *reinterpret_cast<float4*>(dY + r * ldd + (int64_t)k * 4) = make_float4(d[0], d[1], d[2], d[3]);
+        else dY[r * ldd + k] = d[0];
+      }
     }
-    s = gb_warp_sum(s);
-    if (lane == 0) c[r] = s;
+    for (int off = L >> 1; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+    if (r < R && lig == 0) c[r] = s;
   }
 }
 
@@ -512,8 +535,14 @@ granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ld
                               bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st) {
   if (R == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, 12.0 * R * K + 4.0 * R, 2.0 * R * K, 1);
-  const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 8), 148 * 32));
-  k_gat_prep<<<blocks, 256, 0, st>>>(R, K, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
+  const bool v4 = K % 4 == 0 && ldo % 4 == 0 && ldg % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)out & 15u) == 0 &&
+                  ((uintptr_t)g & 15u) == 0 && ((uintptr_t)dY & 15u) == 0;
+  const int Kv = (int)(v4 ? K / 4 : K);
+  int lg = 0;
+  while (lg < 5 && (1 << lg) < Kv) ++lg;
+  const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(R << lg, 256), 148 * 16));
+  if (v4) k_gat_prep<4><<<blocks, 256, 0, st>>>(R, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
+  else k_gat_prep<1><<<blocks, 256, 0, st>>>(R, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

@@ -447,7 +447,8 @@ def test_gat_fused_empty_rows_no_self_loops(G, comp, monkeypatch):
 
 
 @pytest.mark.parametrize("comp", [0, 1, 2, 3])
-@pytest.mark.parametrize("name,K1,K2", [("pubmed", 32, 256), ("pubmed", 256, 32), ("dense", 48, 16)])
+@pytest.mark.parametrize("name,K1,K2", [("pubmed", 32, 256), ("pubmed", 256, 32), ("dense", 48, 16),
+                                        ("tiny", 5, 7), ("sparse", 47, 100)])
 def test_gcn_backward_every_composition(G, comp, name, K1, K2):
     c = case(G, name)
     net, out, H, W, _, _ = run_layer(G, c, G.GCN, comp, K1, K2, G.ACT_RELU)
