@@ -31,7 +31,7 @@ template <> struct Vec<1> {
 // optional row scale (the inner D^-1/2 of the DYN_UPD backward, so its SpMM needs no column scale);
 // out == rs == NULL is a padded row copy (g * 1.f is exact)
 template <int V>
-__global__ void __launch_bounds__(256) k_scale_mask(int64_t rows, int Kv, int lg, const float* __restrict__ out,
+__global__ void __launch_bounds__(256) k_scale_mask(int64_t rows, int K, int Kv, int lg, const float* __restrict__ out,
                                                     int64_t ldo, const float* __restrict__ g, int64_t ldg,
                                                     const float* __restrict__ rs, float* __restrict__ dst,
                                                     int64_t ldd) {
@@ -43,6 +43,13 @@ __global__ void __launch_bounds__(256) k_scale_mask(int64_t rows, int Kv, int lg
     const float s = rs ? rs[r] : 1.f;
 #pragma unroll 2
     for (int k = lig; k < Kv; k += 1 << lg) {
+      if (V > 1 && k * V + V > K) {  // ragged tail of a row whose start is aligned: element by element
+        for (int c = k * V; c < K; ++c) {
+          const float x = g[r * ldg + c] * s;
+          dst[r * ldd + c] = (!out || out[r * ldo + c] > 0.f) ? x : 0.f;
+        }
+        continue;
+      }
       typename VT::T v = VT::ld(g + r * ldg + (int64_t)k * V);
       typename VT::T o;
       if (out) o = VT::ld(out + r * ldo + (int64_t)k * V);
@@ -59,7 +66,7 @@ __global__ void __launch_bounds__(256) k_scale_mask(int64_t rows, int Kv, int lg
 static inline bool al16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
 static void rowwise_shape(int64_t rows, int64_t K, bool v4, int* Kv, int* lg, unsigned* blocks) {
-  *Kv = (int)(v4 ? K / 4 : K);
+  *Kv = (int)(v4 ? (K + 3) / 4 : K);
   int l = 0;
   while (l < 5 && (1 << l) < *Kv) ++l;
   *lg = l;
@@ -68,13 +75,13 @@ static void rowwise_shape(int64_t rows, int64_t K, bool v4, int* Kv, int* lg, un
 
 static granii_status scale_mask_impl(int64_t rows, int64_t K, const float* out, int64_t ldo, const float* g,
                                      int64_t ldg, const float* rs, float* dst, int64_t ldd, cudaStream_t st) {
-  const bool v4 = K % 4 == 0 && ldg % 4 == 0 && ldd % 4 == 0 && al16(g) && al16(dst) &&
+  const bool v4 = ldg % 4 == 0 && ldd % 4 == 0 && al16(g) && al16(dst) &&
                   (!out || (ldo % 4 == 0 && al16(out)));
   int Kv, lg;
   unsigned blocks;
   rowwise_shape(rows, K, v4, &Kv, &lg, &blocks);
-  if (v4) k_scale_mask<4><<<blocks, 256, 0, st>>>(rows, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
-  else k_scale_mask<1><<<blocks, 256, 0, st>>>(rows, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
+  if (v4) k_scale_mask<4><<<blocks, 256, 0, st>>>(rows, (int)K, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
+  else k_scale_mask<1><<<blocks, 256, 0, st>>>(rows, (int)K, Kv, lg, out, ldo, g, ldg, rs, dst, ldd);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

@@ -99,7 +99,7 @@ __device__ __forceinline__ float gb_lrelu(float z) { return z > 0.f ? z : 0.2f *
 // 16-byte accesses when every row start is aligned (V = 4); the row loop is warp-uniform so the group's
 // shuffle reduction never diverges.
 template <int V>
-__global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int Kv, int lg, const float* __restrict__ out,
+__global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int K, int Kv, int lg, const float* __restrict__ out,
                                                   int64_t ldo, const float* __restrict__ g, int64_t ldg, int relu,
                                                   float* __restrict__ dY, int64_t ldd, float* __restrict__ c) {
   const int L = 1 << lg, lane = threadIdx.x & 31, lig = lane & (L - 1);
@@ -113,6 +113,15 @@ __global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int Kv, int lg, con
 #pragma unroll 2
       for (int k = lig; k < Kv; k += L) {
         float o[V], d[V];
+        if (V > 1 && k * V + V > K) {  // ragged tail of a row whose start is aligned: element by element
+          for (int c = k * V; c < K; ++c) {
+            const float oc = out[r * ldo + c];
+            const float dc = (!relu || oc > 0.f) ? g[r * ldg + c] : 0.f;
+            dY[r * ldd + c] = dc;
+            s = fmaf(dc, oc, s);
+          }
+          continue;
+        }
         if constexpr (V == 4) {
           const float4 o4 = *reinterpret_cast<const float4*>(out + r * ldo + (int64_t)k * 4);
           const float4 g4 = *reinterpret_cast<const float4*>(g + r * ldg + (int64_t)k * 4);
@@ -535,14 +544,14 @@ granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ld
                               bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st) {
   if (R == 0) return GRANII_OK;
   ProfScope ps("elementwise", st, 12.0 * R * K + 4.0 * R, 2.0 * R * K, 1);
-  const bool v4 = K % 4 == 0 && ldo % 4 == 0 && ldg % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)out & 15u) == 0 &&
+  const bool v4 = ldo % 4 == 0 && ldg % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)out & 15u) == 0 &&
                   ((uintptr_t)g & 15u) == 0 && ((uintptr_t)dY & 15u) == 0;
-  const int Kv = (int)(v4 ? K / 4 : K);
+  const int Kv = (int)(v4 ? (K + 3) / 4 : K);
   int lg = 0;
   while (lg < 5 && (1 << lg) < Kv) ++lg;
   const unsigned blocks = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(R << lg, 256), 148 * 16));
-  if (v4) k_gat_prep<4><<<blocks, 256, 0, st>>>(R, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
-  else k_gat_prep<1><<<blocks, 256, 0, st>>>(R, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
+  if (v4) k_gat_prep<4><<<blocks, 256, 0, st>>>(R, (int)K, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
+  else k_gat_prep<1><<<blocks, 256, 0, st>>>(R, (int)K, Kv, lg, out, ldo, g, ldg, relu ? 1 : 0, dY, ldd, c);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
