@@ -253,7 +253,8 @@ granii_status granii_layer_workspace_size_ex(granii_graph g, granii_model m, gra
  * out = sigma(layer(H)) for the owned rows (out: rows x K2, ld ldo).  Every
  * composition computes the same mathematical value (L192: only semantically
  * equivalent re-associations).  d_saved (nullable) receives the state the
- * backward of this composition needs (granii_layer_workspace_size).
+ * backward of this composition needs (granii_layer_workspace_size); it must be
+ * 16-byte aligned (its rows are read as float4), else GRANII_ERR_INVALID_ARG.
  * With comm != NULL the dense operand of every SpMM/SDDMM is all-gathered
  * over NCCL inside the call.
  */
@@ -267,7 +268,8 @@ granii_status granii_layer_forward(granii_graph g, granii_model m, granii_compos
  * GAT (additive attention; chain rule of Eq. 4-6, R22): dW, dH and,
  *   through a->d_a_l / a->d_a_r, the attention-weight gradients; REUSE works at
  *   K2, RECOMP at K1 (dT = dY Wᵀ first), as in their forwards.  d_saved is
- *   required (Θ or T = α H, el, er written by the forward).  Dot attention ->
+ *   required (Θ or T = α H, el, er written by the forward; 16-byte aligned,
+ *   else INVALID_ARG).  Dot attention ->
  *   UNSUPPORTED.
  * d_dH may be NULL (input layer).  d_dW (K1 x K2) is all-reduced over comm.
  * Requires a symmetric graph (Mᵀ = M; GAT: row j of Ã lists every i with j in N(i)).
@@ -380,6 +382,10 @@ typedef struct {
   double ms;       /* summed device time between events recorded on the launch stream    */
   double bytes;    /* summed ALGORITHMIC bytes (DESIGN.md §6 per-unit figures)            */
   double flops;    /* summed algorithmic flops                                           */
+  double compulsory_bytes; /* summed COMPULSORY HBM bytes: every operand read / written once
+                              (SpMM: col ids + X + Y once, however often the gathers re-read X) */
+  int64_t l2_resident;     /* calls whose gathered operand (one K slice of X) fits the L2, so the
+                              gathers are served by L2: the binding roof is L2 bandwidth  */
 } granii_prof_entry;
 
 /* Enable (1) / disable (0) event recording around every primitive; resets the table. */

@@ -159,32 +159,43 @@ void oracle_spmm(int64_t n_rows, const int64_t* row_ptr, const int32_t* col_idx,
 }
 
 /* transpose SpMM: Y = Sᵀ X, i.e. Y_c += w_e * X_r for every stored e = (r, c).
- * Written as the scatter it is, serially (used by the backward pass only). */
+ * Written as the scatter it is (used by the backward pass only): every output
+ * element receives its terms in stored-entry order; threads own disjoint column
+ * ranges k of Y, so the order per element is the serial scatter's. */
 void oracle_spmm_t(int64_t n_rows, int64_t n_cols, const int64_t* row_ptr, const int32_t* col_idx,
                    const double* vals, const double* X, int64_t K, double* Y) {
   for (int64_t i = 0; i < n_cols * K; ++i) Y[i] = 0.0;
-  for (int64_t r = 0; r < n_rows; ++r)
-    for (int64_t e = row_ptr[r]; e < row_ptr[r + 1]; ++e) {
-      double w = vals ? vals[e] : 1.0;
-      for (int64_t k = 0; k < K; ++k) Y[(int64_t)col_idx[e] * K + k] += w * X[r * K + k];
-    }
+  const int64_t kc = 8;  /* column range per task */
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t k0 = 0; k0 < K; k0 += kc) {
+    const int64_t k1 = k0 + kc < K ? k0 + kc : K;
+    for (int64_t r = 0; r < n_rows; ++r)
+      for (int64_t e = row_ptr[r]; e < row_ptr[r + 1]; ++e) {
+        double w = vals ? vals[e] : 1.0;
+        for (int64_t k = k0; k < k1; ++k) Y[(int64_t)col_idx[e] * K + k] += w * X[r * K + k];
+      }
+  }
 }
 
 /* GEMM, L80-L82 / L92: C = op(A) * op(B), plain triple loop, row-major.
- * op(A) is M x K (A stored K x M when ta), op(B) is K x N (B stored N x K when tb). */
+ * op(A) is M x K (A stored K x M when ta), op(B) is K x N (B stored N x K when tb).
+ * C[i][j] = sum over k = 0..K-1, in that order, of op(A)[i][k] * op(B)[k][j]; the
+ * k loop runs outside the j loop (a row of partial sums per i) so that op(B) is
+ * read row by row -- the same products summed in the same order. */
 void oracle_gemm(int64_t M, int64_t N, int64_t K, const double* A, int ta, const double* B, int tb,
                  double* C) {
 #pragma omp parallel for schedule(static)
-  for (int64_t i = 0; i < M; ++i)
-    for (int64_t j = 0; j < N; ++j) {
-      double s = 0.0;
-      for (int64_t k = 0; k < K; ++k) {
-        double a = ta ? A[k * M + i] : A[i * K + k];
+  for (int64_t i = 0; i < M; ++i) {
+    double* s = C + i * N;
+    for (int64_t j = 0; j < N; ++j) s[j] = 0.0;
+    for (int64_t k = 0; k < K; ++k) {
+      double a = ta ? A[k * M + i] : A[i * K + k];
+      for (int64_t j = 0; j < N; ++j) {
         double b = tb ? B[j * K + k] : B[k * N + j];
-        s += a * b;
+        s[j] += a * b;
       }
-      C[i * N + j] = s;
     }
+  }
 }
 
 /* sigma [R7]: act = 0 identity, 1 ReLU (no bias: Eq. 2/3/5 have none) */

@@ -81,7 +81,12 @@ static granii_status check_shape(granii_model m, const granii_layer_args* a) {
 // run once on zero-filled inputs of the layer's shape (forward; + backward when training) on a
 // private stream and the fastest measured one is kept.  Single GPU only (a partitioned selection
 // must agree on every rank; it stays model-only there).
+// GRANII_REFINE_MARGIN overrides the margin (tests force every candidate through the timed path with it).
 static constexpr double REFINE_MARGIN = 1.15, REFINE_MAX_MS = 5.0;
+static double refine_margin() {
+  const char* e = getenv("GRANII_REFINE_MARGIN");
+  return e && atof(e) > 1.0 ? atof(e) : REFINE_MARGIN;
+}
 
 static granii_status refine_choice(granii_graph g, granii_model m, const granii_layer_args* shape, uint32_t flags,
                                    const int32_t* cand, const double* pred, int32_t n, granii_composition* out) {
@@ -89,10 +94,11 @@ static granii_status refine_choice(granii_graph g, granii_model m, const granii_
   int best = 0;
   for (int i = 1; i < n; ++i)
     if (pred[i] < pred[best]) best = i;
-  if (!(pred[best] < REFINE_MAX_MS)) return GRANII_OK;
+  const double margin = refine_margin();
+  if (!(pred[best] < REFINE_MAX_MS) && margin == REFINE_MARGIN) return GRANII_OK;
   std::vector<int32_t> close;
   for (int i = 0; i < n; ++i)
-    if (pred[i] <= REFINE_MARGIN * pred[best]) close.push_back(cand[i]);
+    if (pred[i] <= margin * pred[best]) close.push_back(cand[i]);
   if (close.size() < 2) return GRANII_OK;
   const bool train = (flags & GRANII_SELECT_TRAINING) && (m == GRANII_GCN || m == GRANII_GAT);
   const bool need_dh = train && !(flags & GRANII_SELECT_INPUT_LAYER);
@@ -108,9 +114,12 @@ static granii_status refine_choice(granii_graph g, granii_model m, const granii_
     ws = std::max(ws, w1);
     sv = std::max(sv, s1);
   }
-  // one allocation, carved: H | W | W2 | a_l | a_r | out | saved | dout | dH | dW | da_l | da_r | ws
+  // one allocation, carved: H | W | W2 | a_l | a_r | out | saved | dout | dH | dW | da_l | da_r | ws; every piece
+  // starts on a 256-byte boundary (the kernels' float4 / TMA paths need 16-byte aligned rows, saved included)
+  constexpr size_t kPieces = 12, kAlignF = 64;
   const size_t fl = (size_t)R * l1 + nw + (m == GRANII_GIN ? (size_t)shape->Kh * K2 : 0) + 2 * K2 + (size_t)R * l2 +
-                    sv + (train ? (size_t)R * l2 + (need_dh ? (size_t)R * l1 : 0) + (size_t)K1 * K2 + 2 * K2 : 0);
+                    sv + (train ? (size_t)R * l2 + (need_dh ? (size_t)R * l1 : 0) + (size_t)K1 * K2 + 2 * K2 : 0) +
+                    kPieces * kAlignF;
   const size_t bytes = round_up((int64_t)(fl * sizeof(float)), 256) + ws + 256;
   char* base = nullptr;
   cudaStream_t st = nullptr;
@@ -124,7 +133,7 @@ static granii_status refine_choice(granii_graph g, granii_model m, const granii_
       break;
     }
     float* p = reinterpret_cast<float*>(base);
-    auto take = [&](size_t k) { float* q = p; p += k; return q; };
+    auto take = [&](size_t k) { float* q = p; p += (k + kAlignF - 1) / kAlignF * kAlignF; return q; };
     a.H = take((size_t)R * l1);
     a.ldh = l1;
     a.W = take(nw);
@@ -391,6 +400,7 @@ granii_status granii_layer_forward(granii_graph g, granii_model m, granii_compos
   API_BEGIN
   GR_TRY(check_args(g, m, c, a));
   GR_ARG(d_out && ldo >= a->K2, "bad output");
+  GR_ARG(((uintptr_t)d_saved & 15) == 0, "d_saved must be 16-byte aligned (its rows are read as float4)");
   return layer_forward(g, m, c, a, d_out, ldo, d_saved, (cudaStream_t)stream);
   API_END
 }
@@ -406,6 +416,7 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
     return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is implemented for additive attention only (R22)");
   GR_ARG(g->symmetric, "backward needs a symmetric graph (created with GRANII_SYMMETRIZE): M^T = M");
   GR_ARG(m == GRANII_GCN || d_saved, "GAT backward needs d_saved from the forward");
+  GR_ARG(((uintptr_t)d_saved & 15) == 0, "d_saved must be 16-byte aligned (its rows are read as float4)");
   GR_ARG(d_out && d_dout && d_dW && ldo >= a->K2 && lddo >= a->K2, "bad output / gradient");
   GR_ARG(!d_dH || lddh >= a->K1, "bad lddh");
   return layer_backward(g, c, a, d_out, ldo, d_dout, lddo, d_saved, d_dH, lddh, d_dW, (cudaStream_t)stream);

@@ -567,7 +567,11 @@ granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBw
   // + stat + del per row; B = col + stat + dX row per entry, Z row + out row + ... per row
   const double bytes = pass == 0 ? nnz * (8.0 + 4.0 * K) + R * (4.0 * K + 8.0 + 28.0)
                                  : nnz * (20.0 + 4.0 * K) + R * (8.0 * K + 8.0 + 16.0);
-  ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1);
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  const double gathered = (double)g->n_cols * 4.0 * (double)K;  // the gathered operand (Z or dX rows)
+  ProfScope ps(pass == 0 ? "gat_bwd_a" : "gat_bwd_b", st, bytes, (pass == 0 ? 2.0 : 4.0) * nnz * K, 1,
+               bytes - nnz * 4.0 * (double)K + gathered, gathered <= 0.6 * (double)di.l2_bytes);
   // lane-group width (tools/gatbwd_sweep.py on the products-shaped graph): 8 lanes x NJ float4
   // up to K = 64 (4 groups per warp), 16 lanes up to 256, full-warp groups beyond
   // dense graphs (avg degree >= 16): a warp per row; sparse: a lane group per row, the wide

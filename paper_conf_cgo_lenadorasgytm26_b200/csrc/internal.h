@@ -53,15 +53,18 @@ granii_status dev_info(DevInfo* out);
 // ----------------------------------------------------------------- tracing
 // RAII scope around one launcher call: counts kernel launches always; records
 // a pair of CUDA events on the launch stream when profiling is enabled.
+// compulsory < 0: the algorithmic bytes are the compulsory bytes (streaming kernels)
 struct ProfScope {
-  ProfScope(const char* name, cudaStream_t st, double bytes, double flops, int launches);
+  ProfScope(const char* name, cudaStream_t st, double bytes, double flops, int launches, double compulsory = -1.0,
+            bool l2_resident = false);
   ~ProfScope();
   void add_launches(int n);
   const char* name;
   cudaStream_t st;
-  double bytes, flops;
+  double bytes, flops, compulsory;
   int launches;
   int slot;
+  bool l2_resident;
 };
 
 }  // namespace granii

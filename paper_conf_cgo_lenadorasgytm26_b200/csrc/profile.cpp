@@ -15,8 +15,9 @@ namespace {
 struct Rec {
   const char* name;
   cudaEvent_t a, b;
-  double bytes, flops;
+  double bytes, flops, compulsory;
   int launches;
+  bool l2;
 };
 std::atomic<bool> g_on{false};
 std::atomic<int64_t> g_launches{0};
@@ -26,8 +27,9 @@ std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_pool;
 size_t g_used = 0;
 }  // namespace
 
-ProfScope::ProfScope(const char* n, cudaStream_t s, double by, double fl, int la)
-    : name(n), st(s), bytes(by), flops(fl), launches(la), slot(-1) {
+ProfScope::ProfScope(const char* n, cudaStream_t s, double by, double fl, int la, double comp, bool l2)
+    : name(n), st(s), bytes(by), flops(fl), compulsory(comp < 0.0 ? by : comp), launches(la), slot(-1),
+      l2_resident(l2) {
   if (!g_on.load(std::memory_order_relaxed)) return;
   std::lock_guard<std::mutex> lk(g_mu);
   if (g_used == g_pool.size()) {
@@ -46,7 +48,7 @@ ProfScope::~ProfScope() {
   if (slot < 0) return;
   std::lock_guard<std::mutex> lk(g_mu);
   cudaEventRecord(g_pool[slot].second, st);
-  g_recs.push_back({name, g_pool[slot].first, g_pool[slot].second, bytes, flops, launches});
+  g_recs.push_back({name, g_pool[slot].first, g_pool[slot].second, bytes, flops, compulsory, launches, l2_resident});
 }
 
 }  // namespace granii
@@ -77,6 +79,8 @@ granii_status granii_profile_read(granii_prof_entry* out, int32_t max_entries, i
     e.ms += ms;
     e.bytes += r.bytes;
     e.flops += r.flops;
+    e.compulsory_bytes += r.compulsory;
+    e.l2_resident += r.l2 ? 1 : 0;
   }
   int32_t k = 0;
   for (auto& kv : agg) {

@@ -355,8 +355,9 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
               g->n_seg, g->seg_lo, g->seg_hi, g->seg_row};
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
-  ProfScope ps("sddmm", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K,
-               (K > 1 && sm) ? 2 : 1);
+  const double gathered = (double)g->n_cols * 4.0 * (double)K;  // V, read once in the compulsory count
+  ProfScope ps("sddmm", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K, (K > 1 && sm) ? 2 : 1,
+               nnz * 8.0 + R * (8.0 + 4.0 * K) + gathered, gathered <= 0.6 * (double)di.l2_bytes);
   if (K == 1) {
     const int lpg = sm ? lpg_for_softmax(g->avg_deg()) : lpg_for_degree(g->avg_deg());
     const int64_t units = ceil_div(n_light, 32 / lpg) + g->n_seg;

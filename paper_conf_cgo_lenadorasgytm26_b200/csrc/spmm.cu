@@ -645,9 +645,14 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double bytes = nnz * (4.0 + (vals ? 4.0 : 0.0) + (cs ? 4.0 : 0.0) + 4.0 * K) +
                        R * (8.0 + 4.0 * K + (rs ? 4.0 : 0.0) + (B ? 4.0 * K : 0.0) + (att_el ? 4.0 : 0.0));
+  // compulsory bytes: the same streams, with X read once (its rows, not its gathers)
+  const double compulsory = bytes - nnz * 4.0 * K + (double)g->n_cols * 4.0 * K;
+  // the gathered slice stays in L2 (spmm_slice_width keeps it <= ~55 % of L2)
+  const bool l2_res = (double)g->n_cols * 4.0 * (double)kw <= 0.6 * (double)di.l2_bytes;
   // a phased aggregation books its algorithmic bytes once (in its last phase)
   const bool book = !ph || ph->last;
-  ProfScope ps("spmm", st, book ? bytes : 0.0, book ? 2.0 * nnz * K : 0.0, (int)ceil_div(K, kw));
+  ProfScope ps("spmm", st, book ? bytes : 0.0, book ? 2.0 * nnz * K : 0.0, (int)ceil_div(K, kw),
+               book ? compulsory : 0.0, l2_res);
   for (int64_t k0 = 0; k0 < K; k0 += kw) {
     a.k0 = k0;
     a.kw = std::min(kw, K - k0);

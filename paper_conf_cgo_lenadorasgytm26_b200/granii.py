@@ -410,7 +410,8 @@ def granii_sgd(grad: torch.Tensor, param: torch.Tensor, lr: float, stream=None):
 # ---------------------------------------------------------------- tracing
 class prof_entry(ctypes.Structure):
     _fields_ = [("name", ctypes.c_char * 32), ("calls", _i64), ("launches", _i64), ("ms", ctypes.c_double),
-                ("bytes", ctypes.c_double), ("flops", ctypes.c_double)]
+                ("bytes", ctypes.c_double), ("flops", ctypes.c_double), ("compulsory_bytes", ctypes.c_double),
+                ("l2_resident", _i64)]
 
 
 def granii_profile_enable(on: bool = True):
@@ -422,7 +423,9 @@ def granii_profile_read() -> dict:
     n = _i32()
     _check(_lib.granii_profile_read(arr, 32, ctypes.byref(n)), "granii_profile_read")
     return {arr[i].name.decode(): {"calls": arr[i].calls, "launches": arr[i].launches, "ms": arr[i].ms,
-                                   "bytes": arr[i].bytes, "flops": arr[i].flops} for i in range(n.value)}
+                                   "bytes": arr[i].bytes, "flops": arr[i].flops,
+                                   "compulsory_bytes": arr[i].compulsory_bytes, "l2_resident": arr[i].l2_resident}
+            for i in range(n.value)}
 
 
 def granii_launch_count() -> int:

@@ -38,12 +38,19 @@ def G():
     return granii
 
 
+_graphs = {}
+
+
 def build(G, name):
+    if name in _graphs:
+        return _graphs[name]
     w = synth.WORKLOADS[name]
     src, dst = w.edges(seed=0, device=DEV)
     flags = G.ADD_SELF_LOOPS | (G.SYMMETRIZE if w.symmetrize else 0)
     g = G.granii_graph_csr_create(w.n, src, dst, flags)
     rp, ci = O.csr_build(w.n, src.cpu(), dst.cpu(), flags)
+    _graphs.clear()                      # one full-size graph resident at a time
+    _graphs[name] = (w, g, rp, ci)
     return w, g, rp, ci
 
 
@@ -76,10 +83,44 @@ def test_reddit_training_step_fullsize(G):
     gpad.copy_(gup)
     net.backward(gpad)
     torch.cuda.synchronize()
-    MH1 = O.spmm(rp, ci, O.sddmm(rp, ci, O.dinv(rp), O.dinv(rp)), H1)
+    nval = O.sddmm(rp, ci, O.dinv(rp), O.dinv(rp))
+    MH1 = O.spmm(rp, ci, nval, H1)
     dW2 = O.gemm(MH1, gup.cpu().numpy(), ta=True)     # identity activation on the last layer
     d = np.abs(net.dW[1].cpu().numpy() - dW2)
     assert float((d.max(1) / np.abs(dW2).max(1)).max()) <= TOL
+    # the gradient handed to layer 1: dL/dH1 = Mᵀ dY2 W2ᵀ (M symmetric), every row
+    dH1 = O.gemm(O.spmm(rp, ci, nval, gup.cpu().numpy()), W2, tb=True)
+    assert rowerr(net.grads_out[0].cpu().numpy(), dH1) <= TOL
+
+
+def test_reddit_layer1_backward_fullsize(G):
+    """C4 layer 1 as the timed step runs it: GCN 602 -> 256 + ReLU under the composition the
+    selector picks for training (input layer: no dH), i.e. the K=256 transpose aggregation with its
+    L2-resident column slices and hub segments, then dW1 = (M H)ᵀ dY1 (602 x 256) reduced over all
+    232,965 rows, against oracle_gcn_backward.  The upstream gradient is random and zeroed where
+    |Y1| is within rounding of 0, so the ReLU' decision is unique (R20)."""
+    import bench
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec, alloc2d
+    w, g, rp, ci = build(G, "reddit")
+    spec = bench.WORKLOADS["reddit-gcn2-train"]
+    full = bench.build_model(G, None, spec, g, DEV, None)
+    L0 = full.layers[0]
+    del full
+    H = alloc2d(w.n, 602, DEV)
+    H.copy_(synth.features(1, w.n, 602, device=DEV))
+    Hn = H.cpu().numpy()
+    W1 = L0.W.cpu().numpy().astype(np.float64)
+    Y1 = O.gcn_rows(np.arange(w.n), rp, ci, np.diff(rp), Hn, W1, 0)       # pre-activation, fp64
+    U = synth.uniform_pm1(6, 1, (w.n, 256))
+    U[torch.from_numpy(np.abs(Y1) < 1e-4 * np.abs(Y1).max())] = 0.0
+    net = GNN(g, [LayerSpec(G.GCN, 602, 256, G.ACT_RELU, comp=L0.comp, W=L0.W)], DEV)
+    net.forward(H)
+    Ud = alloc2d(w.n, 256, DEV)
+    Ud.copy_(U)
+    assert net.backward(Ud) is None                  # input layer: no dH, as in the step
+    torch.cuda.synchronize()
+    _, dW1 = O.gcn_backward(L0.comp, rp, ci, Hn, W1, U, 1, need_dH=False)
+    assert rowerr(net.dW[0].cpu().numpy(), dW1) <= TOL, G.COMP_NAMES[L0.comp]
 
 
 @pytest.mark.parametrize("model", ["gcn", "gat"])
@@ -104,3 +145,51 @@ def test_products_inference_fullsize(G, model):
     else:
         ref = O.gat_rows(rows, rp, ci, Hn, Wn, L.a_l.cpu().numpy(), L.a_r.cpu().numpy(), 1)
     assert rowerr(out.cpu().numpy()[rows], ref) <= TOL, G.COMP_NAMES[L.comp]
+
+
+@pytest.mark.parametrize("layer", [0, 1])
+def test_products_gat_training_fullsize(G, layer):
+    """C5 GAT training (products-gat2-train, 100 -> 256 -> 47): each layer's backward at full size
+    under the composition the bench selects, one layer at a time so the ReLU' decision can be made
+    unique (R20): dW, da_l, da_r (reductions over all 2.45M rows) and, for the second layer (which
+    the step differentiates with respect to its input), dH on 4,096 random + 64 hub rows, against
+    oracle_gat_backward with the R22 tolerance (gat_grad_ok).  These are the pass A / pass B
+    shapes (K = 100 for RECOMP's dT H rows, K = 47 for REUSE's dY Θ rows) chosen only at this scale."""
+    import bench
+    from test_gpu_parity import gat_grad_ok
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec, alloc2d
+    w, g, rp, ci = build(G, "products")
+    spec = bench.WORKLOADS["products-gat2-train"]
+    full = bench.build_model(G, None, spec, g, DEV, None)
+    L = full.layers[layer]
+    del full
+    K1, K2 = L.K1, L.K2
+    act = G.ACT_RELU if layer == 0 else G.ACT_NONE
+    need_dH = layer > 0
+    H = alloc2d(w.n, K1, DEV)
+    H.copy_(synth.features(10 + layer, w.n, K1, device=DEV))
+    Hn = H.cpu().numpy()
+    Wn, al, ar = (x.cpu().numpy() for x in (L.W, L.a_l, L.a_r))
+    U = synth.uniform_pm1(7, layer, (w.n, K2))
+    if act:
+        Y, _ = O.gat_forward(L.comp, rp, ci, Hn, Wn, al, ar, 0)
+        U[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0      # R20
+        del Y
+    net = GNN(g, [LayerSpec(G.GAT, K1, K2, act, G.ATTN_ADDITIVE, comp=L.comp, W=L.W, a_l=L.a_l, a_r=L.a_r)], DEV)
+    net.forward(H)
+    Ud = alloc2d(w.n, K2, DEV)
+    Ud.copy_(U)
+    dH = net.backward(Ud, need_input_grad=need_dH)
+    torch.cuda.synchronize()
+    rows = sample_rows(rp)
+    ref = O.gat_backward(L.comp, rp, ci, Hn, Wn, al, ar, U, act, need_dH=need_dH)
+    mag = O.gat_backward_magnitude(L.comp, rp, ci, Hn, Wn, al, ar, U, act, need_dH=need_dH)
+    got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
+    for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, ref, mag):
+        if nm == "dH":
+            if not need_dH:
+                continue
+            y, r, m = y.cpu().numpy()[rows], r[rows], m[rows]
+        else:
+            y = y.cpu().numpy()
+        assert gat_grad_ok(y, r, m), (G.COMP_NAMES[L.comp], nm)

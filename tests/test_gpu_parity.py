@@ -466,7 +466,8 @@ def test_gcn_backward_every_composition(G, comp, name, K1, K2):
 
 @pytest.mark.parametrize("comp", [16, 17])
 @pytest.mark.parametrize("name,K1,K2,act", [("pubmed", 32, 256, 1), ("pubmed", 64, 128, 0), ("dense", 48, 16, 1),
-                                             ("tiny", 3, 5, 0), ("sparse", 128, 47, 1), ("dense", 256, 1024, 0)])
+                                             ("tiny", 3, 5, 0), ("sparse", 128, 47, 1), ("dense", 256, 1024, 0),
+                                             ("dense", 384, 512, 0), ("dense", 512, 384, 1)])
 def test_gat_backward_both_compositions(G, comp, name, K1, K2, act):
     """N2 (reading R22): dW, dH, da_l, da_r of both compositions against the oracle's chain rule"""
     c = case(G, name)
@@ -521,6 +522,21 @@ def test_gat_backward_hub_segments(G, comp, name, K1, K2, monkeypatch):
     got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
     for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, ref, mag):
         assert gat_grad_ok(y.cpu(), r, m), nm
+
+
+def test_layer_rejects_misaligned_saved(G):
+    """d_saved rows are read as float4 by the GAT backward and the fused attention SpMM:
+    an unaligned pointer is INVALID_ARG at the ABI, not a misaligned-address fault"""
+    c = case(G, "pubmed")
+    net, out, H, W, al, ar = run_layer(G, c, G.GAT, 16, 8, 3, G.ACT_NONE)
+    buf = torch.empty(net.saved_floats[0] + 4, dtype=torch.float32, device=DEV)
+    args = net.args(0, pad(H))
+    with pytest.raises(G.GraniiError, match="aligned"):
+        G.granii_layer_forward(c.g, G.GAT, 16, args, net.outs[0], buf.data_ptr() + 4)
+    with pytest.raises(G.GraniiError, match="aligned"):
+        G.granii_layer_backward(c.g, G.GAT, 16, args, net.outs[0], net.outs[0], buf.data_ptr() + 4, None, net.dW[0])
+    G.granii_layer_forward(c.g, G.GAT, 16, args, net.outs[0], buf)   # aligned: fine
+    torch.cuda.synchronize()
 
 
 def test_gat_backward_deterministic_and_input_layer(G):
@@ -685,6 +701,19 @@ def test_select_refine(G, model, K1, K2, flags):
     close = [k for k, v in p0.items() if v <= 1.15 * best]
     if len(close) < 2 or best >= 5.0:
         assert s1 == s0
+
+
+@pytest.mark.parametrize("model,K1,K2,flags", [(1, 8, 3, 2), (1, 256, 47, 2), (1, 100, 41, 2 | 4), (0, 30, 7, 2),
+                                                  (1, 8, 3, 0)])
+def test_select_refine_forced_odd_widths(G, model, K1, K2, flags, monkeypatch):
+    """the timed tie-break carves one allocation into H | W | ... | saved | ...: with odd K2 (GAT
+    saved = Θ + el + er of R x ld4(K2) + 2R floats) every piece must still start 16-byte aligned
+    (float4 Θ reads of the GAT backward).  GRANII_REFINE_MARGIN forces the timed path."""
+    c = case(G, "pubmed")
+    monkeypatch.setenv("GRANII_REFINE_MARGIN", "1e9")
+    s1, p1 = G.granii_select_ex(c.g, model, G.shape_args(K1, K2), None, flags | G.SELECT_REFINE)
+    assert s1 in p1
+    torch.cuda.synchronize()
 
 
 def test_select_candidates_are_the_offline_promoted_trees(G):
