@@ -157,34 +157,191 @@ def host_csr(n, src, dst, symmetrize=True):
     return O.csr_build(n, src.cpu(), dst.cpu(), O.ADD_SELF_LOOPS | (O.SYMMETRIZE if symmetrize else 0))
 
 
-def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn"):
-    """fp64 oracle (per-row definition of every layer, oracle_gcn_rows / oracle_gat_rows) on a row sample."""
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+def _omp_threads(n):
+    """set the oracle's OpenMP thread count (libgomp is loaded with liboracle.so)"""
+    import ctypes
+    try:
+        ctypes.CDLL("libgomp.so.1").omp_set_num_threads(int(n))
+    except OSError:
+        pass
+
+
+def _sub_csr(rp, ci, rows):
+    """the CSR rows `rows` (global column ids kept): the oracle's primitives on sampled rows"""
+    deg = np.diff(rp)[rows]
+    srp = np.zeros(rows.size + 1, np.int64)
+    np.cumsum(deg, out=srp[1:])
+    idx = np.repeat(rp[rows] - srp[:-1], deg) + np.arange(srp[-1])
+    return srp, ci[idx]
+
+
+def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=False, threads=None):
+    """The fp64 oracle (oracle/) as it stands, timed on a random row sample S of the workload's own
+    graph -- every layer's forward rows, and for training the backward rows too:
+      GCN forward : oracle_gcn_rows(S)                        (Eq. 3 row by row)
+      GCN backward: Ñ_S = oracle_sddmm(dinv_S, dinv) on S's rows; dT_S = (Ñᵀ dY)_S and (Ñ X)_S by
+                    oracle_spmm over S's rows (Ñ symmetric); S's share of dW = (Ñ X)_Sᵀ dY_S by
+                    oracle_gemm; dH_S = dT_S Wᵀ by oracle_gemm below the input layer
+      GAT forward : oracle_gat_rows(S); GAT backward: not sampled (no per-row GAT backward in the
+                    oracle; the line says so)
+    Each layer gets its own seeded input of its width (the sample times the work, it does not chain
+    values).  edges/s = stored entries of S x layers / seconds, the GPU metric's unit."""
     import oracle as O
+    if threads is not None:
+        _omp_threads(threads)
     n = rp.shape[0] - 1
     deg = np.diff(rp)
+    dinv = O.dinv(rp)
     rng = np.random.default_rng(seed)
+    L = len(dims) - 1
     feats = [synth.features(seed + 7, n, k).numpy() for k in dims[:-1]]
-    Ws = [synth.glorot(seed + 2, i, dims[i], dims[i + 1], (dims[i], dims[i + 1])).numpy() for i in range(len(dims) - 1)]
+    Ws = [synth.glorot(seed + 2, i, dims[i], dims[i + 1], (dims[i], dims[i + 1])).numpy() for i in range(L)]
     atts = [(synth.uniform_pm1(seed + 3, 2 * i, (dims[i + 1],)).numpy(),
-             synth.uniform_pm1(seed + 3, 2 * i + 1, (dims[i + 1],)).numpy()) for i in range(len(dims) - 1)]
+             synth.uniform_pm1(seed + 3, 2 * i + 1, (dims[i + 1],)).numpy()) for i in range(L)]
+    ups = [synth.uniform_pm1(seed + 8, i, (n, dims[i + 1])).numpy() for i in range(L)] if train and model == "gcn" \
+        else None
     S = 256
     while True:
         rows = np.sort(rng.choice(n, size=min(S, n), replace=False))
+        srp, sci = _sub_csr(rp, ci, rows) if ups is not None else (None, None)
         t0 = time.perf_counter()
-        for i in range(len(dims) - 1):
+        for i in range(L):
             if model == "gcn":
                 O.gcn_rows(rows, rp, ci, deg, feats[i], Ws[i], 1)
             else:
                 O.gat_rows(rows, rp, ci, feats[i], Ws[i], atts[i][0], atts[i][1], 1)
+        if ups is not None:
+            nv = O.sddmm(srp, sci, dinv[rows], dinv)
+            for i in range(L - 1, -1, -1):
+                dT = O.spmm(srp, sci, nv, ups[i])                  # (Ñᵀ dY)_S
+                NX = O.spmm(srp, sci, nv, feats[i])                # (Ñ X)_S
+                O.gemm(NX, ups[i][rows], ta=True)                  # dW contribution of S
+                if i > 0:
+                    O.gemm(dT, Ws[i], tb=True)                     # dH_S
         dt = time.perf_counter() - t0
         if dt >= target_s or S >= n:
             break
         S = int(min(n, S * max(2.0, min(16.0, 1.2 * target_s / max(dt, 1e-3)))))
-    edges = float(deg[rows].sum()) * (len(dims) - 1)
-    return {"value": edges / dt, "unit": "edges/s", "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
-            "sample": f"fp64 oracle per-row forward (oracle_{model}_rows) of all {len(dims) - 1} layers on {rows.size} "
-                      f"random rows ({int(deg[rows].sum())} stored entries) of the same graph; backward not included",
-            "seconds": dt}
+    edges = float(deg[rows].sum()) * L
+    cores = threads if threads is not None else len(os.sched_getaffinity(0))
+    if threads is not None:
+        _omp_threads(len(os.sched_getaffinity(0)))
+    what = "forward" + (" + backward" if ups is not None else "")
+    note = "" if (not train or model == "gcn") else "; GAT backward not sampled (forward only)"
+    return {"value": edges / dt, "unit": "edges/s", "cores": cores, "kind": "oracle",
+            "sample": f"fp64 oracle {what} of all {L} layers on {rows.size} random rows "
+                      f"({int(deg[rows].sum())} stored entries) of the same graph{note}",
+            "mode": what, "seconds": dt}
+
+
+def l2_peak():
+    """L2 -> SM read bandwidth measured by tools/probe/l2_bw.cu on B200 (profiles/l2_peak.json);
+    not a driver measurement -- the line says so where it is used"""
+    lp = os.path.join(ROOT, "profiles", "l2_peak.json")
+    return json.load(open(lp))["l2_read_gbs"] if os.path.exists(lp) else None
+
+
+SPEC_HBM_GBS = 8000.0   # B200 HBM3e spec (DGX figure), the second denominator of SURVEY §8(d)
+
+
+def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
+    """Max-roof fraction of one primitive over the timed region:
+    GEMMs: t_roof = max(flops / tensor roof, bytes / HBM), the tensor roof for 3xTF32 being the
+      measured bf16 peak x 1/2 (tf32 nominal ratio) / 3 (passes);
+    gathers (spmm, sddmm, gat_bwd_*): every gathered byte crosses L2 -> SM and every compulsory
+      byte crosses DRAM at least once, t_roof = max(algorithmic / L2 read peak, compulsory / HBM);
+    streaming kernels: t_roof = bytes / HBM.
+    `bound` names the larger term, `achieved` is that term's bytes (flops) / measured time, so
+    frac = t_roof / t <= 1 up to L1 hits.  `traffic` = ncu dram bytes per call (or None) gives
+    what DRAM actually moved, against the measured and the 8 TB/s spec peak."""
+    calls = max(st["calls"], 1)
+    t = st["ms"] / 1e3
+    by, fl = st["bytes"], st["flops"]
+    comp = st.get("compulsory_bytes", by)
+    out = {"launch_ms": st["ms"] / calls, "calls_per_step_region": st["calls"]}
+    if name.startswith("gemm"):
+        tc = tc_peak / 2 / 3
+        t_tc, t_hbm = fl / (tc * 1e12), by / (hbm * 1e9)
+        if t_tc >= t_hbm:
+            out.update(bound="tensor", achieved=fl / t / 1e12, peak=tc, unit="TFLOP/s",
+                       peak_note=f"bf16 sustained {tc_peak} ({peak_src}) x 1/2 (tf32) / 3 (3xTF32 passes)")
+        else:
+            out.update(bound="hbm", achieved=by / t / 1e9, peak=hbm, unit="GB/s",
+                       peak_note=f"hbm_gbs of {peak_src} (tall-skinny GEMM below the ridge)")
+        out["tensor_frac"] = fl / t / 1e12 / tc
+    elif name in ("spmm", "sddmm", "gat_bwd_a", "gat_bwd_b") and l2:
+        t_l2, t_hbm = by / (l2 * 1e9), comp / (hbm * 1e9)
+        if t_l2 >= t_hbm:
+            out.update(bound="l2", achieved=by / t / 1e9, peak=l2, unit="GB/s",
+                       peak_note="L2 read peak measured by tools/probe/l2_bw.cu (profiles/l2_peak.json), "
+                                 "not a driver figure: algorithmic (gathered) bytes / t")
+        else:
+            out.update(bound="hbm", achieved=comp / t / 1e9, peak=hbm, unit="GB/s",
+                       peak_note=f"hbm_gbs of {peak_src}: compulsory bytes / t")
+        out["gathered"] = {"bytes_per_call": by / calls, "gbs": by / t / 1e9, "frac_l2": by / t / 1e9 / l2}
+        out["l2_resident_calls"] = st.get("l2_resident", 0)
+    else:
+        out.update(bound="hbm", achieved=by / t / 1e9, peak=hbm, unit="GB/s", peak_note=f"hbm_gbs of {peak_src}")
+    out["frac"] = out["achieved"] / out["peak"]
+    out["compulsory"] = {"bytes_per_call": comp / calls, "gbs": comp / t / 1e9, "frac_hbm": comp / t / 1e9 / hbm}
+    out["traffic"] = traffic
+    if traffic:
+        g = traffic / (st["ms"] / calls / 1e3) / 1e9
+        out["dram"] = {"bytes_per_call": traffic, "gbs": g, "frac_measured": g / hbm, "frac_spec_8tbs": g / SPEC_HBM_GBS,
+                       "source": "ncu dram__bytes_read+write per call (profiles/ncu_traffic.json)"}
+    return out
+
+
+class LaunchError(RuntimeError):
+    pass
+
+
+def launch_plan(gpus: int, env, device_count: int, impl: str = "granii"):
+    """How to honour `--gpus N` (one process per GPU, the driver's contract):
+    ("run", world) -- this process is one rank of a `world`-rank job (WORLD_SIZE set, or N = 1);
+    ("relaunch", N) -- no launcher around us: re-exec N ranks under torch.distributed.run.
+    LaunchError when the request cannot be honoured (WORLD_SIZE disagrees with --gpus, or the box
+    has fewer GPUs than asked): never silently measure fewer GPUs than the line claims."""
+    if gpus < 1:
+        raise LaunchError(f"--gpus must be >= 1 (got {gpus})")
+    ws = env.get("WORLD_SIZE")
+    if ws is not None:
+        world = int(ws)
+        if world != gpus:
+            raise LaunchError(f"--gpus {gpus} but the launcher started WORLD_SIZE={world} ranks")
+        return "run", world
+    if impl == "reference":           # rank 0 alone works; no GPU needed
+        return "run", gpus
+    if gpus == 1:
+        return "run", 1
+    if device_count < gpus:
+        raise LaunchError(f"--gpus {gpus} needs {gpus} visible GPUs, this box has {device_count}")
+    return "relaunch", gpus
+
+
+def relaunch_cmd(gpus: int, argv, port: int):
+    """the driver's own N > 1 launch line, for a bench started without torchrun"""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *argv]
+
+
+def _free_port():
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
 
 
 def main():
@@ -205,7 +362,13 @@ def main():
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    try:
+        plan, world = launch_plan(args.gpus, os.environ, torch.cuda.device_count(), args.impl)
+    except LaunchError as e:
+        print(f"bench.py: {e}", file=sys.stderr, flush=True)
+        sys.exit(2)
+    if plan == "relaunch":
+        sys.exit(subprocess.call(relaunch_cmd(world, sys.argv[1:], _free_port())))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     spec = WORKLOADS[args.workload]
@@ -219,11 +382,27 @@ def main():
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     comm = None
+    comm_info = None
     if world > 1:
+        if torch.cuda.device_count() <= local:
+            print(f"bench.py: rank {rank} has LOCAL_RANK {local} but only {torch.cuda.device_count()} GPUs",
+                  file=sys.stderr, flush=True)
+            sys.exit(2)
         dist.init_process_group("nccl", device_id=dev)
         uid = [G.granii_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         comm = G.granii_comm_create(uid[0], rank, world)
+        nranks, crank, ver = G.granii_comm_query(comm)
+        print(f"granii comm: rank {crank} nranks {nranks} (NCCL {ver}, WORLD_SIZE {world}, cuda:{local})",
+              file=sys.stderr, flush=True)
+        if nranks != world or crank != rank:
+            print(f"bench.py: NCCL communicator has {nranks} ranks (rank {crank}), expected {world} (rank {rank})",
+                  file=sys.stderr, flush=True)
+            sys.exit(3)
+        comm_info = {"nranks": nranks, "nccl_version": ver, "nranks_ok": True,
+                     "watchdog_ms": int(os.environ.get("GRANII_COMM_TIMEOUT_MS", "120000"))}
+        # failure detection: a collective stuck for longer than this aborts the communicator
+        G.granii_comm_watchdog(comm, comm_info["watchdog_ms"])
 
     # ---------------------------------------------------------------- setup (not timed)
     t_setup = time.perf_counter()
@@ -314,6 +493,7 @@ def main():
     spread = {"p10": step_ms[len(step_ms) // 10], "p50": step_ms[len(step_ms) // 2],
               "p90": step_ms[min(len(step_ms) - 1, (9 * len(step_ms)) // 10)]}
     if world > 1:
+        G.granii_comm_check(comm)          # raises with the watchdog's reason if a collective was aborted
         dist.barrier()
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -324,42 +504,23 @@ def main():
     edges_per_step = float(info.nnz) * n_layers * passes
     value = edges_per_step / (ms / 1e3)
 
-    # roofline of the dominant kernel (largest summed time in the timed region)
+    # roofline of the dominant kernel (largest summed time in the timed region) + every primitive
     hbm, tc_peak, peak_src = peaks()
-    top = max(prof.items(), key=lambda kv: kv[1]["ms"])
-    kname, kst = top
-    share = kst["ms"] / max(sum(v["ms"] for v in prof.values()), 1e-9)
-    traffic = None
+    traffic_tab = {}
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(args.workload, {}).get(kname)
+            traffic_tab = json.load(open(tp)).get(args.workload, {})
         except Exception:
-            traffic = None
-    per_launch_bytes = kst["bytes"] / max(kst["calls"], 1)
-    if kname.startswith("gemm"):
-        achieved = kst["flops"] / (kst["ms"] / 1e3) / 1e12
-        roof = {"bound": "tensor", "achieved": achieved, "peak": tc_peak / 2 / 3, "unit": "TFLOP/s",
-                "peak_note": f"bf16 sustained {tc_peak} ({peak_src}) x 1/2 (tf32 nominal ratio) / 3 (3xTF32 passes)"}
-    else:
-        achieved = kst["bytes"] / (kst["ms"] / 1e3) / 1e9
-        roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                "peak_note": f"hbm_gbs of {peak_src} (MEASURED_PEAKS.json copy bandwidth)"}
-    roof["frac"] = roof["achieved"] / roof["peak"]
-    roof["traffic"] = traffic
-    if traffic and roof["bound"] == "hbm":  # what DRAM actually moved per launch (ncu) over the launch time
-        roof["dram_gbs_from_traffic"] = traffic / (kst["ms"] / max(kst["calls"], 1) / 1e3) / 1e9
-        roof["dram_frac"] = roof["dram_gbs_from_traffic"] / hbm
-    lp = os.path.join(ROOT, "profiles", "l2_peak.json")
-    if roof["bound"] == "hbm" and os.path.exists(lp):
-        # gathers served by L2: the algorithmic bytes against the measured L2 read peak
-        l2 = json.load(open(lp))["l2_read_gbs"]
-        roof["l2"] = {"peak": l2, "frac": achieved / l2, "note": "algorithmic bytes / measured L2 read bandwidth "
-                      "(profiles/l2_peak.json, tools/probe/l2_bw.cu); L1 hits can push it past 1"}
+            traffic_tab = {}
+    per_prim = {k: primitive_roofline(k, v, hbm, tc_peak, peak_src, l2_peak(), traffic_tab.get(k))
+                for k, v in prof.items()}
+    kname = max(prof, key=lambda k: prof[k]["ms"])
+    roof = dict(per_prim[kname])
     roof["kernel"] = kname
-    roof["share_of_step"] = share
-    roof["algorithmic_bytes_per_launch"] = per_launch_bytes
-    roof["launch_ms"] = kst["ms"] / max(kst["calls"], 1)
+    roof["share_of_step"] = prof[kname]["ms"] / max(sum(v["ms"] for v in prof.values()), 1e-9)
+    roof["per_primitive"] = {k: {kk: v[kk] for kk in ("bound", "frac", "achieved", "peak", "unit", "launch_ms")}
+                             for k, v in per_prim.items()}
 
     result = {
         "metric": "GNN layer fwd/bwd ms & edges/s at 1/2/4/8 B200; % HBM roofline; selector regret",
@@ -374,6 +535,7 @@ def main():
                    "l2": "no flush: per-step inputs exceed L2 (H %.0f MB, col_idx %.0f MB vs 126 MB L2)" % (
                        w.n * dims[0] * 4 / 1e6, info.nnz * 4 / 1e6),
                    "parallelism": f"row-partition x{world}" + (" (NCCL all-gather)" if world > 1 else ""),
+                   "comm": comm_info,
                    "cuda_graph": bool(use_graph),
                    "profile_pass": "separate eager pass (graph replay)" if use_graph else "inside the timed region"},
         "clocks": clk.summary(),
@@ -467,7 +629,11 @@ def main():
     elif rank == 0 and world == 1 and not args.no_cpu:
         try:
             rp, ci = host_csr(w.n, src, dst, w.symmetrize)
-            result["cpu_baseline"] = cpu_oracle_sample(rp, ci, dims, model=spec["model"])
+            cb = cpu_oracle_sample(rp, ci, dims, model=spec["model"], train=spec["train"])
+            st = cpu_oracle_sample(rp, ci, dims, target_s=3.0, model=spec["model"], train=spec["train"], threads=1)
+            cb["single_thread"] = {"value": st["value"], "sample": st["sample"]}
+            cb["cpu_model"] = cpu_model()
+            result["cpu_baseline"] = cb
         except Exception as e:  # never fail the bench on the baseline
             result["cpu_baseline"] = {"value": None, "error": str(e)[:200]}
 
@@ -583,10 +749,10 @@ def run_reference(args, spec, w, world, rank):
     budget = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
     res = None
     for _ in range(args.warmup):
-        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4, model=spec["model"])
+        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4, model=spec["model"], train=spec["train"])
     vals, secs = [], []
     for _ in range(args.steps):
-        res = cpu_oracle_sample(rp, ci, dims, target_s=budget, model=spec["model"])
+        res = cpu_oracle_sample(rp, ci, dims, target_s=budget, model=spec["model"], train=spec["train"])
         vals.append(res["value"])
         secs.append(res["seconds"])
     value = float(np.mean(vals))

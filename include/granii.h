@@ -360,6 +360,30 @@ granii_status granii_comm_destroy(granii_comm c);
  * no data).  Errors: INVALID_ARG (NULL), NCCL (transport failure). */
 granii_status granii_comm_allgather(granii_comm c, const float* d_send, float* d_recv, size_t count, void* stream);
 granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t count, void* stream);
+/* What the transport reports: rank count and this rank (NCCL: ncclCommCount / ncclCommUserRank,
+ * so a launcher can check that N processes really formed one N-rank communicator) and the NCCL
+ * version (0 for loopback / stub).  Errors: NCCL if the communicator was aborted. */
+granii_status granii_comm_query(granii_comm c, int32_t* nranks, int32_t* rank, int32_t* nccl_version);
+/* Failure detection.  Starts (timeout_ms > 0) or stops (<= 0) a host watchdog
+ * thread for the communicator: every collective the library issues records an event on its
+ * stream (except under CUDA-graph capture); every ~20 ms the watchdog polls
+ * ncclCommGetAsyncError and the oldest incomplete collective.  An asynchronous error, a device
+ * error, or a collective pending longer than timeout_ms (a mismatched or missing collective on
+ * another rank hangs rather than fails) aborts the communicator (ncclCommAbort; loopback: marked
+ * failed) and every later collective or granii_comm_check on it returns GRANII_ERR_NCCL with the
+ * reason in granii_last_error().  The stub transport is never watched. */
+granii_status granii_comm_watchdog(granii_comm c, int64_t timeout_ms);
+/* GRANII_OK, or GRANII_ERR_NCCL with the watchdog's reason once the communicator was aborted. */
+granii_status granii_comm_check(granii_comm c);
+/* Register a device buffer that collectives will read / write (e.g. a layer workspace holding
+ * the gather buffers) with NCCL (ncclCommRegister), so NCCL can use it directly instead of
+ * staging through its own buffers where the algorithm supports it.  *handle is for
+ * granii_comm_deregister; NULL (and OK) on loopback / stub transports.  The buffer must stay
+ * allocated until deregistered.  Errors: UNSUPPORTED (NCCL without registration), NCCL. */
+granii_status granii_comm_register(granii_comm c, void* d_buf, size_t bytes, void** handle);
+granii_status granii_comm_deregister(granii_comm c, void* handle);
+/* Test support: one kernel that keeps `stream` busy for `us` microseconds (watchdog tests). */
+granii_status granii_debug_spin(int64_t us, void* stream);
 
 /* ------------------------------------------------------------------------ */
 /* Training-step helpers around the layers (not selected by GRANII)          */

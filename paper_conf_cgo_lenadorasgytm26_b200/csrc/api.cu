@@ -49,6 +49,11 @@ granii_status comm_create(const void*, int32_t, int32_t, granii_comm_s**);
 granii_status comm_destroy(granii_comm_s*);
 granii_status comm_create_local(int32_t, granii_comm_s**);
 granii_status comm_create_stub(int32_t, int32_t, granii_comm_s**);
+granii_status comm_watchdog(granii_comm_s*, int64_t);
+granii_status comm_check(granii_comm_s*);
+granii_status comm_query(granii_comm_s*, int32_t*, int32_t*, int32_t*);
+granii_status comm_register(granii_comm_s*, void*, size_t, void**);
+granii_status comm_deregister(granii_comm_s*, void*);
 granii_status launch_softmax_xent(int64_t, int64_t, const float*, int64_t, const int32_t*, int64_t, float*, int64_t,
                                   float*, cudaStream_t);
 granii_status launch_sgd(int64_t, float, const float*, float*, cudaStream_t);
@@ -484,6 +489,33 @@ granii_status granii_comm_allgather(granii_comm c, const float* d_send, float* d
 granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t count, void* stream) {
   GR_ARG(c && d_buf, "NULL argument");
   return comm_allreduce_sum(c, d_buf, count, (cudaStream_t)stream);
+}
+
+granii_status granii_comm_query(granii_comm c, int32_t* nranks, int32_t* rank, int32_t* nccl_version) {
+  GR_ARG(c && nranks && rank && nccl_version, "NULL argument");
+  return comm_query(c, nranks, rank, nccl_version);
+}
+granii_status granii_comm_watchdog(granii_comm c, int64_t timeout_ms) {
+  GR_ARG(c, "NULL communicator");
+  API_BEGIN
+  return comm_watchdog(c, timeout_ms);
+  API_END
+}
+granii_status granii_comm_check(granii_comm c) {
+  GR_ARG(c, "NULL communicator");
+  return comm_check(c);
+}
+granii_status granii_comm_register(granii_comm c, void* d_buf, size_t bytes, void** handle) {
+  GR_ARG(c && handle && (d_buf || bytes == 0), "NULL argument");
+  return comm_register(c, d_buf, bytes, handle);
+}
+granii_status granii_comm_deregister(granii_comm c, void* handle) {
+  GR_ARG(c, "NULL communicator");
+  return comm_deregister(c, handle);
+}
+granii_status granii_debug_spin(int64_t us, void* stream) {
+  GR_ARG(us >= 0 && us <= 60000000, "spin of 0..60 s");
+  return launch_spin(us, (cudaStream_t)stream);
 }
 
 granii_status granii_softmax_xent(int64_t rows, int64_t C, const float* d_Z, int64_t ldz, const int32_t* d_y,

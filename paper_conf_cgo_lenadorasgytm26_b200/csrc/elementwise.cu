@@ -160,6 +160,23 @@ granii_status launch_rank_sum(int n, const float* const* src, size_t count, floa
   return GRANII_OK;
 }
 
+// test support (granii_debug_spin): hold a stream busy for `us` microseconds of wall time
+__global__ void k_spin(int64_t ns) {
+  uint64_t t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  do {
+    __nanosleep(1000);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while ((int64_t)(t - t0) < ns);
+}
+
+granii_status launch_spin(int64_t us, cudaStream_t st) {
+  ProfScope ps("elementwise", st, 0.0, 0.0, 1);
+  k_spin<<<1, 1, 0, st>>>(us * 1000);
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
 // C <= LPG * NV (the classifier widths: 41, 47): an LPG-lane group per row holds its logits in
 // registers -- one coalesced load, max and sum by fixed xor butterflies, one store -- so every load
 // of the 32 / LPG rows of a warp is in flight at once (the warp-per-row loop above re-reads the row

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <string>
 #include <vector>
 
@@ -115,6 +116,8 @@ struct granii_comm_s {
   cudaStream_t side = nullptr;             // collectives overlapped with compute (N1)
   cudaEvent_t* ev = nullptr;               // world + 1 events on `side`
   int32_t rank = 0, world = 1;
+  void* wd = nullptr;                      // failure-detection watchdog (comm.cpp), NULL when off
+  std::atomic<int> failed{0};              // set once the communicator was aborted
 };
 
 namespace granii {
@@ -221,6 +224,12 @@ granii_status comm_create_stub(int32_t rank, int32_t world, granii_comm_s** out)
 granii_status comm_bcast_block(granii_comm_s* c, float* buf_all, size_t count, int root, cudaStream_t st);
 // the communicator's side stream and per-block events (created on first use on the current device)
 granii_status comm_side(granii_comm_s* c, cudaStream_t* side, cudaEvent_t** ev);
+granii_status comm_watchdog(granii_comm_s* c, int64_t timeout_ms);
+granii_status comm_check(granii_comm_s* c);
+granii_status comm_query(granii_comm_s* c, int32_t* nranks, int32_t* rank, int32_t* version);
+granii_status comm_register(granii_comm_s* c, void* buf, size_t bytes, void** handle);
+granii_status comm_deregister(granii_comm_s* c, void* handle);
 // out[i] = sum_{p < n} src[p][i] in rank order (loopback all-reduce)
 granii_status launch_rank_sum(int n, const float* const* src, size_t count, float* out, cudaStream_t st);
+granii_status launch_spin(int64_t us, cudaStream_t st);  // test support: one thread spins for `us` microseconds
 }  // namespace granii

@@ -106,6 +106,12 @@ _SIGS = {
     "granii_comm_stats": ([_p, ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)], ctypes.c_int),
     "granii_comm_allgather": ([_p, _p, _p, _sz, _p], ctypes.c_int),
     "granii_comm_allreduce_sum": ([_p, _p, _sz, _p], ctypes.c_int),
+    "granii_comm_query": ([_p, ctypes.POINTER(_i32), ctypes.POINTER(_i32), ctypes.POINTER(_i32)], ctypes.c_int),
+    "granii_comm_watchdog": ([_p, _i64], ctypes.c_int),
+    "granii_comm_check": ([_p], ctypes.c_int),
+    "granii_comm_register": ([_p, _p, _sz, ctypes.POINTER(_p)], ctypes.c_int),
+    "granii_comm_deregister": ([_p, _p], ctypes.c_int),
+    "granii_debug_spin": ([_i64, _p], ctypes.c_int),
     "granii_softmax_xent": ([_i64, _i64, _p, _i64, _p, _i64, _p, _i64, _p, _p], ctypes.c_int),
     "granii_sgd": ([_i64, _f, _p, _p, _p], ctypes.c_int),
     "granii_profile_enable": ([_i32], ctypes.c_int),
@@ -373,6 +379,36 @@ def granii_comm_allgather(c: Comm, send: torch.Tensor, recv: torch.Tensor, count
 def granii_comm_allreduce_sum(c: Comm, buf: torch.Tensor, stream=None):
     _check(_lib.granii_comm_allreduce_sum(c.handle, _ptr(buf), buf.numel(), _stream(stream)),
            "granii_comm_allreduce_sum")
+
+
+def granii_comm_query(c: Comm):
+    """(nranks, rank, nccl_version) as the transport reports them"""
+    n, r, v = _i32(), _i32(), _i32()
+    _check(_lib.granii_comm_query(c.handle, ctypes.byref(n), ctypes.byref(r), ctypes.byref(v)), "granii_comm_query")
+    return n.value, r.value, v.value
+
+
+def granii_comm_watchdog(c: Comm, timeout_ms: int):
+    _check(_lib.granii_comm_watchdog(c.handle, int(timeout_ms)), "granii_comm_watchdog")
+
+
+def granii_comm_check(c: Comm):
+    _check(_lib.granii_comm_check(c.handle), "granii_comm_check")
+
+
+def granii_comm_register(c: Comm, buf: torch.Tensor) -> int | None:
+    h = _p()
+    _check(_lib.granii_comm_register(c.handle, _ptr(buf), buf.numel() * buf.element_size(), ctypes.byref(h)),
+           "granii_comm_register")
+    return h.value
+
+
+def granii_comm_deregister(c: Comm, handle):
+    _check(_lib.granii_comm_deregister(c.handle, handle), "granii_comm_deregister")
+
+
+def granii_debug_spin(us: int, stream=None):
+    _check(_lib.granii_debug_spin(int(us), _stream(stream)), "granii_debug_spin")
 
 
 def granii_comm_create_local(world: int) -> list:

@@ -13,6 +13,7 @@ ranks' owned rows must match the single-process fp64 oracle within the same
 tolerances as the unpartitioned path (test_gpu_parity.py, R19 / R22).
 """
 import os
+import time
 import threading
 
 import numpy as np
@@ -365,3 +366,53 @@ def test_comm_collectives_nccl_one_rank_and_loopback(G):
     for r in range(world):
         assert torch.equal(outs[r], want)
         assert torch.equal(sums[r], x.cpu() * 6)
+
+
+def test_comm_query_register_and_watchdog_no_false_alarm(G):
+    """A 1-rank NCCL communicator reports nranks = 1 / rank 0 through ncclCommCount /
+    ncclCommUserRank; a registered buffer works as a collective operand; with the watchdog
+    running, collectives that complete never trip it"""
+    comm = G.granii_comm_create(G.granii_comm_unique_id(), 0, 1)
+    n, r, v = G.granii_comm_query(comm)
+    assert (n, r) == (1, 0) and v >= 21800          # NCCL 2.18+ encodes 2.18.0 as 21800
+    buf = torch.arange(4096, dtype=torch.float32, device=DEV)
+    try:
+        h = G.granii_comm_register(comm, buf)
+    except G.GraniiError as e:                      # NCCL without user-buffer registration
+        assert "ncclCommRegister" in str(e)
+        h = None
+    G.granii_comm_watchdog(comm, 2000)
+    want = buf.clone()
+    for _ in range(50):
+        G.granii_comm_allreduce_sum(comm, buf)
+    torch.cuda.synchronize()
+    time.sleep(0.1)
+    G.granii_comm_check(comm)
+    assert torch.equal(buf, want)
+    if h is not None:
+        G.granii_comm_deregister(comm, h)
+    G.granii_comm_watchdog(comm, 0)
+    del comm
+
+
+def test_comm_watchdog_aborts_a_stuck_collective(G):
+    """Failure detection: a collective held back on the device longer than the watchdog timeout
+    (here by a 1.5 s kernel queued before it on the same stream, standing in for a peer that
+    never arrives) aborts the communicator, and later calls fail with the reason instead of
+    hanging.  Loopback transport, so the abort is a flag and the GPU stays healthy."""
+    comm = G.granii_comm_create_local(1)[0]
+    G.granii_comm_watchdog(comm, 200)
+    x = torch.ones(1024, device=DEV)
+    G.granii_comm_allreduce_sum(comm, x)      # first call sizes the staging buffer (a host sync)
+    torch.cuda.synchronize()
+    time.sleep(0.3)
+    G.granii_comm_check(comm)                 # completed collectives never trip it
+    G.granii_debug_spin(1_500_000)
+    G.granii_comm_allreduce_sum(comm, x)
+    time.sleep(0.8)
+    with pytest.raises(G.GraniiError, match="pending"):
+        G.granii_comm_check(comm)
+    with pytest.raises(G.GraniiError, match="watchdog"):
+        G.granii_comm_allreduce_sum(comm, x)
+    torch.cuda.synchronize()
+    G.granii_comm_watchdog(comm, 0)
