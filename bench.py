@@ -42,6 +42,10 @@ WORKLOADS = {
     "products-gcn2-infer": dict(graph="products", model="gcn", dims=[100, 256, 47], train=False),
     "products-gat2-infer": dict(graph="products", model="gat", dims=[100, 256, 47], train=False),
     "arxiv-gat-infer": dict(graph="arxiv", model="gat", dims=[64, 256], train=False),
+    # C3 training on the directed R-MAT graph: the backward's transposed passes run over the CSR of
+    # Ãᵀ kept by GRANII_BUILD_TRANSPOSE (ogbn-arxiv: 128 features, 40 classes)
+    "arxiv-gat2-train": dict(graph="arxiv", model="gat", dims=[128, 256, 40], train=True),
+    "arxiv-gcn2-train": dict(graph="arxiv", model="gcn", dims=[128, 256, 40], train=True),
     "pubmed-gcn2-train": dict(graph="pubmed", model="gcn", dims=[256, 32, 32], train=True),
     "products-gat2-train": dict(graph="products", model="gat", dims=[100, 256, 47], train=True),
     "pubmed-gat2-train": dict(graph="pubmed", model="gat", dims=[64, 256, 32], train=True),
@@ -185,12 +189,13 @@ def _sub_csr(rp, ci, rows):
     return srp, ci[idx]
 
 
-def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=False, threads=None):
+def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=False, threads=None, rct=None):
     """The fp64 oracle (oracle/) as it stands, timed on a random row sample S of the workload's own
     graph -- every layer's forward rows, and for training the backward rows too:
       GCN forward : oracle_gcn_rows(S)                        (Eq. 3 row by row)
       GCN backward: Ñ_S = oracle_sddmm(dinv_S, dinv) on S's rows; dT_S = (Ñᵀ dY)_S and (Ñ X)_S by
-                    oracle_spmm over S's rows (Ñ symmetric); S's share of dW = (Ñ X)_Sᵀ dY_S by
+                    oracle_spmm over S's rows (of Ãᵀ = rct for a directed graph, else of Ã: Ñ
+                    symmetric); S's share of dW = (Ñ X)_Sᵀ dY_S by
                     oracle_gemm; dH_S = dT_S Wᵀ by oracle_gemm below the input layer
       GAT forward : oracle_gat_rows(S); GAT backward: not sampled (no per-row GAT backward in the
                     oracle; the line says so)
@@ -214,6 +219,7 @@ def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=Fa
     while True:
         rows = np.sort(rng.choice(n, size=min(S, n), replace=False))
         srp, sci = _sub_csr(rp, ci, rows) if ups is not None else (None, None)
+        trp, tci = _sub_csr(rct[0], rct[1], rows) if (ups is not None and rct is not None) else (srp, sci)
         t0 = time.perf_counter()
         for i in range(L):
             if model == "gcn":
@@ -222,8 +228,9 @@ def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=Fa
                 O.gat_rows(rows, rp, ci, feats[i], Ws[i], atts[i][0], atts[i][1], 1)
         if ups is not None:
             nv = O.sddmm(srp, sci, dinv[rows], dinv)
+            nvt = O.sddmm(trp, tci, dinv[rows], dinv) if rct is not None else nv
             for i in range(L - 1, -1, -1):
-                dT = O.spmm(srp, sci, nv, ups[i])                  # (Ñᵀ dY)_S
+                dT = O.spmm(trp, tci, nvt, ups[i])                 # (Ñᵀ dY)_S
                 NX = O.spmm(srp, sci, nv, feats[i])                # (Ñ X)_S
                 O.gemm(NX, ups[i][rows], ta=True)                  # dW contribution of S
                 if i > 0:
@@ -408,6 +415,8 @@ def main():
     t_setup = time.perf_counter()
     src, dst = w.edges(seed=0, device=dev)
     flags = G.ADD_SELF_LOOPS | (G.SYMMETRIZE if w.symmetrize else 0)
+    if spec["train"] and not w.symmetrize:
+        flags |= G.BUILD_TRANSPOSE        # directed graph: the backward needs Ãᵀ
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     g = G.granii_graph_csr_create(w.n, src, dst, flags, rank, world)
@@ -629,8 +638,10 @@ def main():
     elif rank == 0 and world == 1 and not args.no_cpu:
         try:
             rp, ci = host_csr(w.n, src, dst, w.symmetrize)
-            cb = cpu_oracle_sample(rp, ci, dims, model=spec["model"], train=spec["train"])
-            st = cpu_oracle_sample(rp, ci, dims, target_s=3.0, model=spec["model"], train=spec["train"], threads=1)
+            rct = host_csr(w.n, dst, src, False) if (spec["train"] and not w.symmetrize) else None
+            cb = cpu_oracle_sample(rp, ci, dims, model=spec["model"], train=spec["train"], rct=rct)
+            st = cpu_oracle_sample(rp, ci, dims, target_s=3.0, model=spec["model"], train=spec["train"], threads=1,
+                                   rct=rct)
             cb["single_thread"] = {"value": st["value"], "sample": st["sample"]}
             cb["cpu_model"] = cpu_model()
             result["cpu_baseline"] = cb
@@ -746,13 +757,14 @@ def run_reference(args, spec, w, world, rank):
     t0 = time.perf_counter()
     rp, ci = host_csr(w.n, src, dst, w.symmetrize)
     t_csr = time.perf_counter() - t0
+    rct = host_csr(w.n, dst, src, False) if (spec["train"] and not w.symmetrize) else None
     budget = max(2.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
     res = None
     for _ in range(args.warmup):
-        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4, model=spec["model"], train=spec["train"])
+        cpu_oracle_sample(rp, ci, dims, target_s=budget / 4, model=spec["model"], train=spec["train"], rct=rct)
     vals, secs = [], []
     for _ in range(args.steps):
-        res = cpu_oracle_sample(rp, ci, dims, target_s=budget, model=spec["model"], train=spec["train"])
+        res = cpu_oracle_sample(rp, ci, dims, target_s=budget, model=spec["model"], train=spec["train"], rct=rct)
         vals.append(res["value"])
         secs.append(res["seconds"])
     value = float(np.mean(vals))

@@ -62,6 +62,11 @@ typedef struct granii_graph_s* granii_graph;
 /* flags of granii_graph_csr_create */
 #define GRANII_ADD_SELF_LOOPS 0x1u /* Ã has self-edges (L113)                          */
 #define GRANII_SYMMETRIZE 0x2u     /* undirected input (L328): also insert (v,u)        */
+/* keep a second CSR, of Ãᵀ (rows = sources), for the backward on a directed graph:
+ * the transposed aggregations Mᵀ dY, αᵀ dY run over it.  Ignored
+ * (not needed) with SYMMETRIZE, where Ãᵀ = Ã.  Partitioned: this rank's rows of Ãᵀ
+ * over the SAME row block [b_r, b_{r+1}) as Ã, columns in the same gather layout. */
+#define GRANII_BUILD_TRANSPOSE 0x4u
 
 #define GRANII_NUM_FEATURES 8
 
@@ -75,7 +80,7 @@ typedef struct {
   int32_t part_rank;       /* this rank                                              */
   int32_t part_world;      /* number of row blocks                                   */
   int32_t symmetric;       /* 1 if Ã = Ãᵀ by construction (SYMMETRIZE)               */
-  int32_t reserved;
+  int32_t has_transpose;   /* 1 if a CSR of Ãᵀ is kept (BUILD_TRANSPOSE, not symmetric)  */
   /* input-featurizer features (L252-L256), integer and exact:
    * [0] N, [1] nnz, [2] sum deg, [3] sum deg^2, [4] max deg, [5] min deg,
    * [6] nnz held by the ceil(N/100) highest-degree rows, [7] rows with deg 0. */
@@ -94,8 +99,11 @@ typedef struct {
  *   block [b_r, b_{r+1}) with b_g = min{ r : row_ptr[r] >= ceil(g*nnz/G) };
  *   local column ids are remapped to the padded gather layout
  *   owner(j)*max_local_rows + (j - b_owner(j)) used by the layer's all-gather.
- * Syncs `stream` once (to learn nnz).  Errors: INVALID_ARG for ids outside
- * [0, num_nodes) or bad sizes; OOM; CUDA.
+ * BUILD_TRANSPOSE (directed graphs): the same build over the reversed edges,
+ *   with D̃ still Ã's row degrees (R4), kept beside Ã for the backward.
+ * Syncs `stream` (validation, nnz, the host-side schedule of hub rows: a few
+ * times, at creation only).  Errors: INVALID_ARG for ids outside
+ * [0, num_nodes) or bad sizes or unknown flags; OOM; CUDA.
  */
 granii_status granii_graph_csr_create(int64_t num_nodes, int64_t num_edges, const int32_t* d_src,
                                       const int32_t* d_dst, uint32_t flags, int32_t part_rank,
@@ -120,6 +128,11 @@ granii_status granii_gather_layout_host(int64_t n, const int32_t* h_cols, const 
 /* Like export_csr but col ids are returned exactly as stored on the device
  * (gather-layout ids when partitioned). */
 granii_status granii_graph_export_local(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx);
+/* This rank's rows of Ãᵀ (graph built with BUILD_TRANSPOSE, not symmetric), like export_csr:
+ * h_row_ptr int64[local rows + 1], h_col_idx int32[*nnz_t] global ids (size it with
+ * granii_graph_transpose_nnz).  INVALID_ARG when no transpose is kept. */
+granii_status granii_graph_transpose_nnz(granii_graph g, int64_t* nnz_t);
+granii_status granii_graph_export_transpose(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx);
 
 /* ------------------------------------------------------------------------ */
 /* Primitives (L80-L92).  All operate on this rank's rows of Ã.              */
@@ -272,7 +285,9 @@ granii_status granii_layer_forward(granii_graph g, granii_model m, granii_compos
  *   else INVALID_ARG).  Dot attention ->
  *   UNSUPPORTED.
  * d_dH may be NULL (input layer).  d_dW (K1 x K2) is all-reduced over comm.
- * Requires a symmetric graph (Mᵀ = M; GAT: row j of Ã lists every i with j in N(i)).
+ * The transposed aggregations (Mᵀ dY; GAT pass B: every i with j in N(i)) run over Ã
+ * itself when symmetric, else over the CSR of Ãᵀ kept by GRANII_BUILD_TRANSPOSE;
+ * a directed graph without it -> INVALID_ARG.
  */
 granii_status granii_layer_backward(granii_graph g, granii_model m, granii_composition c,
                                     const granii_layer_args* a, const float* d_out, int64_t ldo,

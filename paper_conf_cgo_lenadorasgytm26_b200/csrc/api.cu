@@ -32,7 +32,7 @@ granii_status dev_info(DevInfo* out) {
 
 // defined in other translation units
 granii_status graph_create(int64_t, int64_t, const int32_t*, const int32_t*, uint32_t, int32_t, int32_t, cudaStream_t,
-                           granii_graph_s**);
+                           granii_graph_s**, const int64_t* force_bounds = nullptr);
 void graph_free(granii_graph_s*);
 void partition_bounds_host(int64_t N, const int64_t* rp, int G, int64_t* b);
 granii_status layer_workspace(const granii_graph_s*, granii_model, granii_composition, const granii_layer_args*,
@@ -229,7 +229,7 @@ granii_status granii_graph_csr_create(int64_t num_nodes, int64_t num_edges, cons
   GR_ARG(num_nodes >= 0 && num_edges >= 0, "negative size");
   GR_ARG(num_nodes < (int64_t(1) << 31), "num_nodes must fit int32 column ids");
   GR_ARG(num_edges == 0 || (d_src && d_dst), "NULL edge arrays");
-  GR_ARG((flags & ~(GRANII_ADD_SELF_LOOPS | GRANII_SYMMETRIZE)) == 0, "unknown flags");
+  GR_ARG((flags & ~(GRANII_ADD_SELF_LOOPS | GRANII_SYMMETRIZE | GRANII_BUILD_TRANSPOSE)) == 0, "unknown flags");
   GR_ARG(part_world >= 1 && part_rank >= 0 && part_rank < part_world, "bad partition rank/world");
   GR_ARG(part_world <= 1 || num_nodes >= part_world, "fewer nodes than partitions");
   DevInfo di;
@@ -258,6 +258,7 @@ granii_status granii_graph_query(granii_graph g, granii_graph_info* o) {
   o->part_rank = g->rank;
   o->part_world = g->world;
   o->symmetric = g->symmetric;
+  o->has_transpose = g->T != nullptr;
   for (int i = 0; i < GRANII_NUM_FEATURES; ++i) o->features[i] = g->features[i];
   return GRANII_OK;
 }
@@ -277,6 +278,19 @@ granii_status granii_graph_export_csr(granii_graph g, int64_t* h_row_ptr, int32_
   }
   return GRANII_OK;
   API_END
+}
+
+granii_status granii_graph_transpose_nnz(granii_graph g, int64_t* nnz_t) {
+  GR_ARG(g && nnz_t, "NULL argument");
+  GR_ARG(g->T, "no transpose kept (create with GRANII_BUILD_TRANSPOSE on a directed graph)");
+  *nnz_t = g->T->local_nnz;
+  return GRANII_OK;
+}
+
+granii_status granii_graph_export_transpose(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx) {
+  GR_ARG(g, "NULL argument");
+  GR_ARG(g->T, "no transpose kept (create with GRANII_BUILD_TRANSPOSE on a directed graph)");
+  return granii_graph_export_csr(g->T, h_row_ptr, h_col_idx);
 }
 
 granii_status granii_graph_export_local(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx) {
@@ -419,7 +433,8 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
     return fail(GRANII_ERR_UNSUPPORTED, "backward of SGC / TAGCN / GIN is not implemented (forward only, R23)");
   if (m == GRANII_GAT && a->attn != GRANII_ATTN_ADDITIVE)
     return fail(GRANII_ERR_UNSUPPORTED, "GAT backward is implemented for additive attention only (R22)");
-  GR_ARG(g->symmetric, "backward needs a symmetric graph (created with GRANII_SYMMETRIZE): M^T = M");
+  GR_ARG(g->transposed(), "backward on a directed graph needs its transpose: create it with GRANII_BUILD_TRANSPOSE "
+                          "(or GRANII_SYMMETRIZE, where M^T = M)");
   GR_ARG(m == GRANII_GCN || d_saved, "GAT backward needs d_saved from the forward");
   GR_ARG(((uintptr_t)d_saved & 15) == 0, "d_saved must be 16-byte aligned (its rows are read as float4)");
   GR_ARG(d_out && d_dout && d_dW && ldo >= a->K2 && lddo >= a->K2, "bad output / gradient");

@@ -174,8 +174,11 @@ void partition_bounds_host(int64_t N, const int64_t* rp, int G, int64_t* b) {
   }
 }
 
+void graph_free(granii_graph_s* g);
+
 granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int32_t* d_dst, uint32_t flags,
-                           int32_t rank, int32_t world, cudaStream_t st, granii_graph_s** out) {
+                           int32_t rank, int32_t world, cudaStream_t st, granii_graph_s** out,
+                           const int64_t* force_bounds) {
   const int sym = (flags & GRANII_SYMMETRIZE) ? 1 : 0, loops = (flags & GRANII_ADD_SELF_LOOPS) ? 1 : 0;
   const int cb = key_bits(std::max<int64_t>(N, 2));
   GR_ARG(2 * cb <= 64, "num_nodes too large");
@@ -319,7 +322,8 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
     CK(cudaMemcpyAsync(hrp.data(), rp_full, (N + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     g->bounds.assign(world + 1, 0);
-    partition_bounds_host(N, hrp.data(), world, g->bounds.data());
+    if (force_bounds) g->bounds.assign(force_bounds, force_bounds + world + 1);  // Ãᵀ: Ã's row blocks
+    else partition_bounds_host(N, hrp.data(), world, g->bounds.data());
     int64_t mr = 0;
     for (int i = 0; i < world; ++i) mr = std::max(mr, g->bounds[i + 1] - g->bounds[i]);
     g->max_rows = std::max<int64_t>(mr, 1);
@@ -423,12 +427,38 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   cleanup();
   CK(cudaStreamSynchronize(st));
 #undef CK
+  if ((flags & GRANII_BUILD_TRANSPOSE) && !sym) {
+    // Ãᵀ = the same build over the reversed edges, over Ã's row blocks; D̃ stays Ã's row degrees
+    // (R4: Mᵀ = (D̃^-½ Ã D̃^-½)ᵀ = D̃^-½ Ãᵀ D̃^-½), so its dinv arrays are overwritten with Ã's
+    granii_graph_s* t = nullptr;
+    granii_status rt = graph_create(N, E, d_dst, d_src, flags & GRANII_ADD_SELF_LOOPS, rank, world, st, &t,
+                                    g->bounds.data());
+    if (rt != GRANII_OK) {
+      graph_free(g);
+      return rt;
+    }
+    cudaError_t e = cudaMemcpyAsync(t->dinv_rows, g->dinv_rows, std::max<int64_t>(g->n_rows, 1) * sizeof(float),
+                                    cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess && t->dinv_cols != t->dinv_rows)
+      e = cudaMemcpyAsync(t->dinv_cols, g->dinv_cols, g->n_cols * sizeof(float), cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(t->dinv2_rows, g->dinv2_rows, std::max<int64_t>(g->n_rows, 1) * sizeof(float),
+                          cudaMemcpyDeviceToDevice, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) {
+      graph_free(t);
+      graph_free(g);
+      return fail(GRANII_ERR_CUDA, std::string("transpose dinv: ") + cudaGetErrorString(e));
+    }
+    g->T = t;
+  }
   *out = g;
   return GRANII_OK;
 }
 
 void graph_free(granii_graph_s* g) {
   if (!g) return;
+  graph_free(g->T);
   cudaFree(g->owner_off);
   cudaFree(g->dinv2_rows);
   if (g->dinv_cols != g->dinv_rows) cudaFree(g->dinv_cols);

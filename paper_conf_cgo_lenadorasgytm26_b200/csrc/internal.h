@@ -105,6 +105,10 @@ struct granii_graph_s {
   int64_t wide_deg = 32, n_wide = 0;
   int64_t features[GRANII_NUM_FEATURES] = {0};
   int device = 0;
+  granii_graph_s* T = nullptr;    // Ãᵀ over the same owned rows (GRANII_BUILD_TRANSPOSE, directed graphs);
+                                  // its dinv arrays are Ã's (D̃ = Ã's row degrees, R4)
+  // the graph the transposed aggregations of the backward run over (Mᵀ = M when symmetric)
+  const granii_graph_s* transposed() const { return symmetric ? this : T; }
   float avg_deg() const { return n_rows > 0 ? float(local_nnz) / float(n_rows) : 0.f; }
 };
 

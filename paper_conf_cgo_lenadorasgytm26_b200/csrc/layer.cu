@@ -631,6 +631,10 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
   const int64_t R = g->n_rows, K1 = a->K1, K2 = a->K2;
   const cudaStream_t st = c.st;
   const bool relu = a->act == GRANII_ACT_RELU;
+  // the transposed aggregations (Mᵀ ·) run over Ãᵀ: Ã itself when symmetric, else the kept
+  // transpose (GRANII_BUILD_TRANSPOSE); same owned rows, same gather layout, Ã's D̃ (R4)
+  const granii_graph_s* gt = g->transposed() ? g->transposed() : g;  // (sizing of a graph without one)
+  const Ctx ct{gt, c.comm, c.st};
 
   // dY = dout ⊙ 1[out > 0]; written into a gather slot when the next sparse step needs it
   const bool dy_gathered = comp == GRANII_GCN_PRE_UPD || comp == GRANII_GCN_DYN_UPD;
@@ -648,8 +652,8 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
   int64_t ldh = a->ldh;
   float* nval = nullptr;
   if (comp == GRANII_GCN_PRE_AGG || comp == GRANII_GCN_PRE_UPD) {
-    nval = b.take((size_t)std::max<int64_t>(g->local_nnz, 1));
-    if (run) GR_TRY(launch_sddmm(g, GRANII_SDDMM_DOT, g->dinv_rows, 1, g->dinv_cols, 1, 1, 1.f, nval, st));
+    nval = b.take((size_t)std::max<int64_t>(gt->local_nnz, 1));  // Ñᵀ's values in Ãᵀ's pattern
+    if (run) GR_TRY(launch_sddmm(gt, GRANII_SDDMM_DOT, gt->dinv_rows, 1, gt->dinv_cols, 1, 1, 1.f, nval, st));
   }
   void* gwW;
   size_t gnW;
@@ -677,18 +681,18 @@ static granii_status backward_impl(const Ctx& c, granii_composition comp, const 
                                   nullptr};
           GR_TRY(launch_gemm(R, K1, K2, dY, lddy, a->W, K2, dtg.mine, dtg.ld, &ep, GRANII_GEMM_TRANS_B, gwH, gnH, st));
           if (comp == GRANII_GCN_PRE_AGG)
-            GR_TRY(gathered_spmm(c, dtg, nval, K1, dH, lddh, nullptr, nullptr, false));
+            GR_TRY(gathered_spmm(ct, dtg, nval, K1, dH, lddh, nullptr, nullptr, false));
           else
-            GR_TRY(gathered_spmm(c, dtg, nullptr, K1, dH, lddh, g->dinv_rows, nullptr, false));
+            GR_TRY(gathered_spmm(ct, dtg, nullptr, K1, dH, lddh, gt->dinv_rows, nullptr, false));
         }
         break;
       }
       case GRANII_GCN_PRE_UPD:
       case GRANII_GCN_DYN_UPD: {
         if (comp == GRANII_GCN_PRE_UPD)
-          GR_TRY(gathered_spmm(c, dyg, nval, K2, dT, ldt2, nullptr, nullptr, false));
+          GR_TRY(gathered_spmm(ct, dyg, nval, K2, dT, ldt2, nullptr, nullptr, false));
         else
-          GR_TRY(gathered_spmm(c, dyg, nullptr, K2, dT, ldt2, g->dinv_rows, nullptr, false));
+          GR_TRY(gathered_spmm(ct, dyg, nullptr, K2, dT, ldt2, gt->dinv_rows, nullptr, false));
         GR_TRY(launch_gemm(K1, K2, R, H, ldh, dT, ldt2, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
         if (dH) GR_TRY(launch_gemm(R, K1, K2, dT, ldt2, a->W, K2, dH, lddh, nullptr, GRANII_GEMM_TRANS_B, gwH, gnH, st));
         break;
@@ -731,6 +735,8 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   const bool reuse = comp == GRANII_GAT_REUSE;
   const GatSaved sv = gat_saved_layout(R, comp, K1, K2);
   if (run && !saved) return fail(GRANII_ERR_INVALID_ARG, "GAT backward needs d_saved from the forward");
+  // pass B walks Ãᵀ (row j lists every i with j in N(i)): Ã when symmetric, else the kept transpose
+  const granii_graph_s* gt = g->transposed() ? g->transposed() : g;
   const float* el = saved ? saved + sv.el : nullptr;
   const float* er_own = saved ? saved + sv.er : nullptr;
 
@@ -831,9 +837,9 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     if (!reuse) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
     GatBwdArgs pb;
     pb.n_rows = R;
-    pb.row_ptr = g->row_ptr;
-    pb.col_idx = g->col_idx;
-    pb.order = g->order;
+    pb.row_ptr = gt->row_ptr;
+    pb.col_idx = gt->col_idx;
+    pb.order = gt->order;
     pb.K = pa.K;
     pb.dX = reuse ? dyg.all : dtg.all;
     pb.ldx = pa.ldx;
@@ -848,7 +854,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pb.out = bout;
     pb.ldo = ldbo;
     pb.vec_store = (ldbo % 4 == 0) && (((uintptr_t)bout & 15) == 0);
-    GR_TRY(launch_gat_bwd_pass(g, 1, pb, st));
+    GR_TRY(launch_gat_bwd_pass(gt, 1, pb, st));
     if (reuse) {
       GR_TRY(launch_gemm(K1, K2, R, H, ldh, bout, ldbo, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
       if (dH)

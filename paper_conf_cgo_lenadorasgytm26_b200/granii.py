@@ -23,7 +23,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 # ---------------------------------------------------------------- constants (granii.h)
 OK, ERR_INVALID_ARG, ERR_OOM, ERR_CUDA, ERR_NCCL, ERR_UNSUPPORTED, ERR_NOT_CALIBRATED = range(7)
-ADD_SELF_LOOPS, SYMMETRIZE = 0x1, 0x2
+ADD_SELF_LOOPS, SYMMETRIZE, BUILD_TRANSPOSE = 0x1, 0x2, 0x4
 EPI_RELU = 0x1
 SDDMM_DOT, SDDMM_ADD, SDDMM_LEAKYRELU, SDDMM_ROW_SOFTMAX = 0x0, 0x1, 0x10, 0x20
 GEMM_TRANS_A, GEMM_TRANS_B, GEMM_RELU, GEMM_NO_STORE = 0x1, 0x2, 0x4, 0x8
@@ -54,7 +54,7 @@ _i64, _i32, _u32, _p, _f, _sz = (ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32
 class graph_info(ctypes.Structure):
     _fields_ = [("num_nodes", _i64), ("nnz", _i64), ("row_begin", _i64), ("row_end", _i64),
                 ("local_nnz", _i64), ("max_local_rows", _i64), ("part_rank", _i32), ("part_world", _i32),
-                ("symmetric", _i32), ("reserved", _i32), ("features", _i64 * NUM_FEATURES)]
+                ("symmetric", _i32), ("has_transpose", _i32), ("features", _i64 * NUM_FEATURES)]
 
 
 class gemm_epilogue(ctypes.Structure):
@@ -74,6 +74,8 @@ _SIGS = {
     "granii_graph_destroy": ([_p], ctypes.c_int),
     "granii_graph_query": ([_p, ctypes.POINTER(graph_info)], ctypes.c_int),
     "granii_graph_export_csr": ([_p, _p, _p], ctypes.c_int),
+    "granii_graph_transpose_nnz": ([_p, ctypes.POINTER(_i64)], ctypes.c_int),
+    "granii_graph_export_transpose": ([_p, _p, _p], ctypes.c_int),
     "granii_graph_dinv": ([_p, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_partition_bounds": ([_i64, _p, _i32, _p], ctypes.c_int),
     "granii_gather_layout_host": ([_i64, _p, _p, _i32, _i64, _p], ctypes.c_int),
@@ -210,6 +212,18 @@ def granii_graph_export_csr(g: Graph):
     ci = np.zeros(max(g.nnz, 1), np.int32)
     _check(_lib.granii_graph_export_csr(g.handle, rp.ctypes.data, ci.ctypes.data), "granii_graph_export_csr")
     return rp, ci[: g.nnz]
+
+
+def granii_graph_export_transpose(g: Graph):
+    """this rank's rows of Ãᵀ (BUILD_TRANSPOSE graphs): (row_ptr, global column ids)"""
+    import numpy as np
+    nt = _i64()
+    _check(_lib.granii_graph_transpose_nnz(g.handle, ctypes.byref(nt)), "granii_graph_transpose_nnz")
+    rp = np.zeros(g.n_rows + 1, np.int64)
+    ci = np.zeros(max(nt.value, 1), np.int32)
+    _check(_lib.granii_graph_export_transpose(g.handle, rp.ctypes.data, ci.ctypes.data),
+           "granii_graph_export_transpose")
+    return rp, ci[: nt.value]
 
 
 def granii_graph_export_local(g: Graph):

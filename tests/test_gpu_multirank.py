@@ -48,11 +48,11 @@ def graph_case(name):
     return n, s, d
 
 
-def run_ranks(G, world, n, s, d, body):
+def run_ranks(G, world, n, s, d, body, flags=F):
     """create the G partitioned graphs, then run body(rank, graph, comm, rows) on G threads;
     returns the per-rank results in rank order"""
     sd, dd = s.to(DEV).contiguous(), d.to(DEV).contiguous()
-    graphs = [G.granii_graph_csr_create(n, sd, dd, F, r, world) for r in range(world)]
+    graphs = [G.granii_graph_csr_create(n, sd, dd, flags, r, world) for r in range(world)]
     comms = G.granii_comm_create_local(world)
     res, errs = [None] * world, []
 
@@ -416,3 +416,61 @@ def test_comm_watchdog_aborts_a_stuck_collective(G):
         G.granii_comm_allreduce_sum(comm, x)
     torch.cuda.synchronize()
     G.granii_comm_watchdog(comm, 0)
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("comp", [0, 1, 2, 3, 16, 17])
+def test_directed_backward_partitioned(G, world, comp, monkeypatch):
+    """GRANII_BUILD_TRANSPOSE on a partitioned directed (R-MAT) graph: every rank keeps its rows of
+    Ãᵀ over Ã's row block, in the same gather layout; the transposed aggregations of the GCN and
+    GAT backward run over them (forced one-phase-per-block to exercise the phased Ãᵀ SpMM)"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    set_phases(monkeypatch, "16")
+    n = 1200
+    s, d = synth.rmat(n, 9000, 0.57, 0.19, 0.19, seed=26)
+    fl = G.ADD_SELF_LOOPS | G.BUILD_TRANSPOSE
+    rp, ci = O.csr_build(n, s, d, O.ADD_SELF_LOOPS)
+    rpt, cit = O.csr_build(n, d, s, O.ADD_SELF_LOOPS)       # Ãᵀ: the reversed edges
+    bounds = O.partition(rp, world)
+    K1, K2 = 24, 40
+    H = synth.features(97, n, K1)
+    W = synth.glorot(97, 2, K1, K2, (K1, K2))
+    al = synth.uniform_pm1(97, 3, (K2,))
+    ar = synth.uniform_pm1(97, 4, (K2,))
+    Gup = synth.uniform_pm1(97, 5, (n, K2))
+    gat = comp >= 16
+    if not gat:
+        _, Y = O.gcn_forward(comp, rp, ci, H, W, 1)
+        Gup[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0   # R20
+
+    def body(r, g, comm, rows):
+        b0, b1 = rows
+        trp, tci = G.granii_graph_export_transpose(g)
+        if gat:
+            spec = LayerSpec(G.GAT, K1, K2, G.ACT_NONE, comp=comp, W=W.to(DEV), a_l=al.to(DEV), a_r=ar.to(DEV))
+        else:
+            spec = LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=comp, W=W.to(DEV))
+        net = GNN(g, [spec], DEV, comm=comm)
+        net.forward(padded(H[b0:b1]))
+        dH = net.backward(padded(Gup[b0:b1]), need_input_grad=True)
+        da = (net.da[0][0].cpu(), net.da[0][1].cpu()) if gat else (None, None)
+        return (trp, tci), dH.cpu(), net.dW[0].cpu(), da[0], da[1]
+
+    res, _ = run_ranks(G, world, n, s, d, body, flags=fl)
+    for r in range(world):                                  # Ãᵀ rows of the block, bit-exact
+        b0, b1 = int(bounds[r]), int(bounds[r + 1])
+        trp, tci = res[r][0]
+        assert np.array_equal(trp, rpt[b0:b1 + 1] - rpt[b0]) and np.array_equal(tci, cit[rpt[b0]:rpt[b1]])
+    dH = torch.cat([x[1] for x in res])
+    if gat:
+        rg = O.gat_backward(comp, rp, ci, H, W, al, ar, Gup, 0)
+        mag = O.gat_backward_magnitude(comp, rp, ci, H, W, al, ar, Gup, 0)
+        assert gat_grad_ok(dH, rg[0], mag[0]), "dH"
+        for r in range(world):
+            for i, nm in ((2, "dW"), (3, "da_l"), (4, "da_r")):
+                assert gat_grad_ok(res[r][i], rg[i - 1], mag[i - 1]), (r, nm)
+    else:
+        rdH, rdW = O.gcn_backward(comp, rp, ci, H, W, Gup, 1)
+        assert err(dH, rdH) <= TOL
+        for r in range(world):
+            assert err(res[r][2], rdW) <= TOL

@@ -95,6 +95,16 @@ def case(G, name):
         n = 4000
         s, d = synth.rmat(n, 30000, 0.57, 0.19, 0.19, seed=4)
         c = Case(G, name, n, s, d, O.ADD_SELF_LOOPS)
+    elif name == "directed_t":       # the same, with Ãᵀ kept for the backward (BUILD_TRANSPOSE)
+        n = 4000
+        s, d = synth.rmat(n, 30000, 0.57, 0.19, 0.19, seed=4)
+        c = Case(G, name, n, s, d, O.ADD_SELF_LOOPS | 0x4)
+        c.rp, c.ci = O.csr_build(n, s, d, O.ADD_SELF_LOOPS)
+    elif name == "directed_dense_t":  # warp-per-row R-MAT (avg degree ~ 40) with Ãᵀ, hub rows
+        n = 3000
+        s, d = synth.rmat(n, 120000, 0.57, 0.19, 0.19, seed=5)
+        c = Case(G, name, n, s, d, O.ADD_SELF_LOOPS | 0x4)
+        c.rp, c.ci = O.csr_build(n, s, d, O.ADD_SELF_LOOPS)
     elif name == "cora":
         w = synth.WORKLOADS["cora"]
         s, d = w.edges(0)
@@ -537,6 +547,63 @@ def test_layer_rejects_misaligned_saved(G):
         G.granii_layer_backward(c.g, G.GAT, 16, args, net.outs[0], net.outs[0], buf.data_ptr() + 4, None, net.dW[0])
     G.granii_layer_forward(c.g, G.GAT, 16, args, net.outs[0], buf)   # aligned: fine
     torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("name", ["directed_t", "directed_dense_t"])
+def test_transpose_csr_bit_exact(G, name):
+    """BUILD_TRANSPOSE: the kept CSR of Ãᵀ equals the oracle's CSR of the reversed edge list,
+    bit for bit; a symmetrised graph keeps none (Ãᵀ = Ã); a directed graph without it refuses
+    the backward instead of computing Ã dY where Ãᵀ dY is meant"""
+    c = case(G, name)
+    rpt, cit = O.csr_build(c.n, c.d, c.s, O.ADD_SELF_LOOPS)
+    trp, tci = G.granii_graph_export_transpose(c.g)
+    assert c.g.info.has_transpose == 1
+    assert np.array_equal(trp, rpt) and np.array_equal(tci, cit)
+    assert case(G, "pubmed").g.info.has_transpose == 0
+    with pytest.raises(G.GraniiError):
+        G.granii_graph_export_transpose(case(G, "pubmed").g)
+    d = case(G, "directed")
+    net, out, H, W, _, _ = run_layer(G, d, G.GCN, 0, 8, 8, G.ACT_RELU)
+    with pytest.raises(G.GraniiError, match="BUILD_TRANSPOSE"):
+        net.backward(pad(torch.zeros(d.n, 8)))
+
+
+@pytest.mark.parametrize("comp", [0, 1, 2, 3])
+@pytest.mark.parametrize("name,K1,K2", [("directed_t", 32, 64), ("directed_t", 100, 47),
+                                        ("directed_dense_t", 64, 256), ("directed_dense_t", 256, 32)])
+def test_gcn_backward_directed(G, comp, name, K1, K2):
+    """O6 on a directed graph: dH = Mᵀ dY Wᵀ with Mᵀ = D̃^-½ Ãᵀ D̃^-½ over the kept transpose
+    (D̃ = Ã's row degrees, R4); against the oracle's literal transpose-scatter"""
+    c = case(G, name)
+    net, out, H, W, _, _ = run_layer(G, c, G.GCN, comp, K1, K2, G.ACT_RELU)
+    Gup = synth.uniform_pm1(64, 1, (c.n, K2))
+    _, Y = O.gcn_forward(comp, c.rp, c.ci, H, W, 1)
+    Gup[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0      # R20
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    rdH, rdW = O.gcn_backward(comp, c.rp, c.ci, H, W, Gup, 1)
+    assert err(net.dW[0].cpu(), rdW) <= TOL
+    assert err(dH.cpu(), rdH) <= TOL
+
+
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("name,K1,K2,act", [("directed_t", 64, 128, 0), ("directed_t", 128, 47, 1),
+                                             ("directed_dense_t", 48, 100, 0), ("directed_dense_t", 256, 64, 1)])
+def test_gat_backward_directed(G, comp, name, K1, K2, act):
+    """GAT backward (R22) on a directed graph: pass B walks Ãᵀ (row j lists every i with j in N(i))"""
+    c = case(G, name)
+    net, out, H, W, al, ar = run_layer(G, c, G.GAT, comp, K1, K2, act)
+    Gup = synth.uniform_pm1(65, 1, (c.n, K2))
+    if act:
+        Y, _ = O.gat_forward(comp, c.rp, c.ci, H, W, al, ar, 0)
+        Gup[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0  # R20
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    ref = O.gat_backward(comp, c.rp, c.ci, H, W, al, ar, Gup, act)
+    mag = O.gat_backward_magnitude(comp, c.rp, c.ci, H, W, al, ar, Gup, act)
+    got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
+    for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, ref, mag):
+        assert gat_grad_ok(y.cpu(), r, m), nm
 
 
 def test_gat_backward_deterministic_and_input_layer(G):
