@@ -28,7 +28,8 @@ SOURCES = ["api.cu", "csr.cu", "spmm.cu", "sddmm.cu", "gemm.cu", "layer.cu", "ga
 def _compile(src: str, verbose: bool) -> str:
     path = os.path.join(CSRC, src)
     obj = os.path.join(OBJ, src + ".o")
-    deps = [path, os.path.join(CSRC, "internal.h"), os.path.join(ROOT, "include", "granii.h")]
+    deps = [path, os.path.join(CSRC, "internal.h"), os.path.join(CSRC, "cache.cuh"),
+            os.path.join(ROOT, "include", "granii.h")]
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(d) for d in deps):
         return obj
     cmd = [NVCC, *ARCH, *FLAGS, "-c", path, "-o", obj]

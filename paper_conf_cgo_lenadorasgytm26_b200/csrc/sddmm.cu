@@ -21,6 +21,7 @@
 #include <algorithm>
 #include <cmath>
 
+#include "cache.cuh"
 #include "internal.h"
 
 namespace granii {
@@ -41,6 +42,7 @@ struct SddmmArgs {
   const int64_t* __restrict__ seg_lo;
   const int64_t* __restrict__ seg_hi;
   const int32_t* __restrict__ seg_row;
+  int l2hint;                              // cache.cuh: V kept in L2, col_idx / out streamed
 };
 
 template <bool ADD, bool LRELU>
@@ -57,6 +59,7 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const L2Pol pol = make_l2pol(a.l2hint);
   // heavy-row segments: all 32 lanes stride the segment (scores only; the softmax of
   // heavy rows is the segmented 3-phase pass launched afterwards)
   for (int64_t t = warp; t < a.n_seg; t += nwarps) {
@@ -66,11 +69,16 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
     for (; e + 96 < hi; e += 128) {
       int32_t c[4];
 #pragma unroll
-      for (int q = 0; q < 4; ++q) c[q] = __ldg(a.col_idx + e + 32 * q);
+      for (int q = 0; q < 4; ++q) c[q] = ldg_stream(a.col_idx + e + 32 * q, pol.stream);
 #pragma unroll
-      for (int q = 0; q < 4; ++q) a.out[e + 32 * q] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)c[q] * a.ldv), a.scale);
+      for (int q = 0; q < 4; ++q)
+        st_pol(a.out + e + 32 * q, score1<ADD, LRELU>(u, ldg_pol(a.V + (int64_t)c[q] * a.ldv, pol.keep), a.scale),
+               pol.stream);
     }
-    for (; e < hi; e += 32) a.out[e] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+    for (; e < hi; e += 32) {
+      const int32_t c = ldg_stream(a.col_idx + e, pol.stream);
+      st_pol(a.out + e, score1<ADD, LRELU>(u, ldg_pol(a.V + (int64_t)c * a.ldv, pol.keep), a.scale), pol.stream);
+    }
   }
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
@@ -85,11 +93,16 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
       for (; e + (U4 - 1) * LPG < re; e += U4 * LPG) {
         int32_t c[U4];
 #pragma unroll
-        for (int q = 0; q < U4; ++q) c[q] = __ldg(a.col_idx + e + q * LPG);
+        for (int q = 0; q < U4; ++q) c[q] = ldg_stream(a.col_idx + e + q * LPG, pol.stream);
 #pragma unroll
-        for (int q = 0; q < U4; ++q) a.out[e + q * LPG] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)c[q] * a.ldv), a.scale);
+        for (int q = 0; q < U4; ++q)
+          st_pol(a.out + e + q * LPG, score1<ADD, LRELU>(u, ldg_pol(a.V + (int64_t)c[q] * a.ldv, pol.keep), a.scale),
+                 pol.stream);
       }
-      for (; e < re; e += LPG) a.out[e] = score1<ADD, LRELU>(u, __ldg(a.V + (int64_t)__ldg(a.col_idx + e) * a.ldv), a.scale);
+      for (; e < re; e += LPG) {
+        const int32_t c = ldg_stream(a.col_idx + e, pol.stream);
+        st_pol(a.out + e, score1<ADD, LRELU>(u, ldg_pol(a.V + (int64_t)c * a.ldv, pol.keep), a.scale), pol.stream);
+      }
       continue;
     }
     // Fused row softmax.  Steps of U4 x LPG entries issue every load at once (lanes past the
@@ -105,10 +118,10 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
 #pragma unroll
       for (int q = 0; q < U4; ++q) {
         const int64_t e = rs + q * LPG + lig;
-        c[q] = __ldg(a.col_idx + (e < re ? e : re - 1));
+        c[q] = ldg_stream(a.col_idx + (e < re ? e : re - 1), pol.stream);
       }
 #pragma unroll
-      for (int q = 0; q < U4; ++q) x[q] = __ldg(a.V + (int64_t)c[q] * a.ldv);
+      for (int q = 0; q < U4; ++q) x[q] = ldg_pol(a.V + (int64_t)c[q] * a.ldv, pol.keep);
 #pragma unroll
       for (int q = 0; q < U4; ++q) {
         x[q] = rs + q * LPG + lig < re ? score1<ADD, LRELU>(u, x[q], a.scale) : -INFINITY;
@@ -121,17 +134,17 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
 #pragma unroll
         for (int q = 0; q < U4; ++q) {
           const int64_t e = e0 + q * LPG + lig;
-          c[q] = __ldg(a.col_idx + (e < re ? e : re - 1));
+          c[q] = ldg_stream(a.col_idx + (e < re ? e : re - 1), pol.stream);
         }
 #pragma unroll
-        for (int q = 0; q < U4; ++q) y[q] = __ldg(a.V + (int64_t)c[q] * a.ldv);
+        for (int q = 0; q < U4; ++q) y[q] = ldg_pol(a.V + (int64_t)c[q] * a.ldv, pol.keep);
         float mn = m;
 #pragma unroll
         for (int q = 0; q < U4; ++q) {
           const int64_t e = e0 + q * LPG + lig;
           y[q] = score1<ADD, LRELU>(u, y[q], a.scale);
           if (e < re) {
-            a.out[e] = y[q];
+            st_pol(a.out + (e), y[q], pol.stream);
             mn = fmaxf(mn, y[q]);
           } else {
             y[q] = -INFINITY;
@@ -165,10 +178,10 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
 #pragma unroll
       for (int q = 0; q < U4; ++q) {
         const int64_t e = rs + q * LPG + lig;
-        if (e < re) a.out[e] = x[q] * inv;
+        if (e < re) st_pol(a.out + (e), x[q] * inv, pol.stream);
       }
     } else {
-      for (int64_t e2 = rs + lig; e2 < re; e2 += LPG) a.out[e2] = __expf(a.out[e2] - mr) * inv;
+      for (int64_t e2 = rs + lig; e2 < re; e2 += LPG) st_pol(a.out + (e2), __expf(a.out[e2] - mr) * inv, pol.stream);
     }
   }
 }
@@ -352,7 +365,7 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
   const int64_t n_light = g->n_rows - g->n_heavy;
   SddmmArgs a{n_light, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order + g->n_heavy,
-              g->n_seg, g->seg_lo, g->seg_hi, g->seg_row};
+              g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, l2hint_enabled()};
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double gathered = (double)g->n_cols * 4.0 * (double)K;  // V, read once in the compulsory count

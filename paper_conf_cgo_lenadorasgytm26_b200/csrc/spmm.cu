@@ -17,6 +17,7 @@
 // one warp/group, reduction order fixed => bitwise reproducible.
 #include <algorithm>
 
+#include "cache.cuh"
 #include "internal.h"
 
 namespace granii {
@@ -39,6 +40,24 @@ __device__ __forceinline__ void ldv(const float* p, float (&v)[VEC]) {
     v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
   } else {
     v[0] = __ldg(p);
+  }
+}
+// the gathered operand: L2 policy `pol` (keep: evict_last)
+template <int VEC>
+__device__ __forceinline__ void ldv(const float* p, float (&v)[VEC], uint64_t pol) {
+  if constexpr (VEC == 4) {
+    float4 t = ldg_pol(reinterpret_cast<const float4*>(p), pol);
+    v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+  } else {
+    v[0] = ldg_pol(p, pol);
+  }
+}
+template <int VEC>
+__device__ __forceinline__ void stv(float* p, const float (&v)[VEC], uint64_t pol) {
+  if constexpr (VEC == 4) {
+    st_pol(reinterpret_cast<float4*>(p), make_float4(v[0], v[1], v[2], v[3]), pol);
+  } else {
+    st_pol(p, v[0], pol);
   }
 }
 template <int VEC>
@@ -90,6 +109,7 @@ struct SpmmArgs {
   // (m, s) in seg_ms for the softmax-aware combine
   const float* __restrict__ el;
   float2* __restrict__ seg_ms;
+  int l2hint;                              // L2 eviction priorities on (cache.cuh; GRANII_L2HINT)
 };
 
 // online-softmax state of one row (or segment), warp-uniform m, per-lane partial s
@@ -121,11 +141,12 @@ __device__ __forceinline__ void load_partial(const float* y, const bool (&colok)
 // past the range's end reuse its last column with w = 0, so every later step is
 // branch-free (the padded gathers hit L1 and add exact zeros).
 template <bool W>
-__device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t re, int lane, int32_t& c, float& w) {
+__device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t re, int lane, int32_t& c, float& w,
+                                           const L2Pol& pol) {
   const bool valid = e + lane < re;
   const int64_t ee = valid ? e + lane : re - 1;
-  c = __ldg(a.col_idx + ee);
-  w = valid ? (W ? __ldg(a.vals + ee) : 1.f) : 0.f;
+  c = ldg_stream(a.col_idx + ee, pol.stream);
+  w = valid ? (W ? ldg_stream(a.vals + ee, pol.stream) : 1.f) : 0.f;
 }
 
 // The whole warp accumulates entries [rs0, re): G = 32/LPG lane groups each take a
@@ -133,16 +154,16 @@ __device__ __forceinline__ void load_chunk(const SpmmArgs& a, int64_t e, int64_t
 template <int VEC, int LPG, int NJ, bool W, bool CS, int U, bool ATT = false>
 __device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64_t re, int lane, int grp,
                                            const char* const (&xbj)[NJ], uint32_t row_bytes, float (&acc)[NJ][VEC],
-                                           AttState* at = nullptr) {
+                                           const L2Pol& pol, AttState* at = nullptr) {
   constexpr int G = 32 / LPG;
   if (rs0 >= re) return;
   // distance-2 prefetch: (c0, w0, cs0) = next chunk, (c1, w1) = the chunk after; the
   // dependent col-scale gather cs[c] of a chunk is issued one chunk before its use
   int32_t c0, c1 = 0;
   float w0, w1 = 0.f, cs0 = 1.f;
-  load_chunk<W>(a, rs0, re, lane, c0, w0);
-  if (CS) cs0 = __ldg(a.cs + c0);
-  if (rs0 + 32 < re) load_chunk<W>(a, rs0 + 32, re, lane, c1, w1);
+  load_chunk<W>(a, rs0, re, lane, c0, w0, pol);
+  if (CS) cs0 = ldg_pol(a.cs + c0, pol.keep);
+  if (rs0 + 32 < re) load_chunk<W>(a, rs0 + 32, re, lane, c1, w1, pol);
   for (int64_t base = rs0; base < re; base += 32) {
     const int32_t c = c0;
     float w = CS ? w0 * cs0 : w0;
@@ -169,8 +190,8 @@ __device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64
     if (base + 32 < re) {
       c0 = c1;
       w0 = w1;
-      if (CS) cs0 = __ldg(a.cs + c0);                                      // c1 landed a chunk ago
-      if (base + 64 < re) load_chunk<W>(a, base + 64, re, lane, c1, w1);  // two chunks ahead
+      if (CS) cs0 = ldg_pol(a.cs + c0, pol.keep);                               // c1 landed a chunk ago
+      if (base + 64 < re) load_chunk<W>(a, base + 64, re, lane, c1, w1, pol);  // two chunks ahead
     }
     const int cnt = (int)((re - base) < 32 ? (re - base) : 32);
     const int steps = (cnt + G * U - 1) / (G * U);  // warp-uniform
@@ -188,7 +209,7 @@ __device__ __forceinline__ void warp_range(const SpmmArgs& a, int64_t rs0, int64
       for (int u = 0; u < U; ++u) {
 #pragma unroll
         for (int j = 0; j < NJ; ++j)
-          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
+          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j], pol.keep);
       }
 #pragma unroll
       for (int u = 0; u < U; ++u)
@@ -235,7 +256,8 @@ __device__ __forceinline__ void reduce_groups(float (&acc)[NJ][VEC]) {
 
 template <int LPG, int NJ, int VEC>
 __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], const float (&acc)[NJ][VEC], float s,
-                                          int relu, const float* b = nullptr, float beta = 0.f) {
+                                          int relu, const float* b = nullptr, float beta = 0.f,
+                                          const L2Pol* pol = nullptr) {
 #pragma unroll
   for (int j = 0; j < NJ; ++j) {
     if (!colok[j]) continue;
@@ -248,7 +270,8 @@ __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], con
       if (b) o[v] = fmaf(beta, bv[v], o[v]);
       if (relu) o[v] = fmaxf(o[v], 0.f);
     }
-    stv<VEC>(y + j * LPG * VEC, o);
+    if (pol) stv<VEC>(y + j * LPG * VEC, o, pol->stream);  // the output row: written once
+    else stv<VEC>(y + j * LPG * VEC, o);
   }
 }
 
@@ -256,13 +279,14 @@ __device__ __forceinline__ void store_row(float* y, const bool (&colok)[NJ], con
 template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U, bool ATT = false>
 __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lane, int grp, int lig,
                                            const bool (&colok)[NJ], const char* const (&xbj)[NJ],
-                                           uint32_t row_bytes) {
+                                           uint32_t row_bytes, const L2Pol& pol) {
   float acc[NJ][VEC];
   zero(acc);
   float* part = a.partial + t * a.ldp + (int64_t)lig * VEC;
   if constexpr (ATT) {
     AttState at{__ldg(a.el + a.seg_row[t]), -INFINITY, 0.f};
-    warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc, &at);
+    warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc, pol,
+                                                   &at);
     reduce_groups<LPG>(acc);
     float st = at.s;
 #pragma unroll
@@ -276,10 +300,10 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
     for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {  // the range(s) are computed when needed
       int64_t lo, hi;
       phase_part(a, a.seg_row[t], r, a.seg_lo[t], a.seg_hi[t], lo, hi);
-      warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc, pol);
     }
   } else {
-    warp_range<VEC, LPG, NJ, W, CS, U>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc);
+    warp_range<VEC, LPG, NJ, W, CS, U>(a, a.seg_lo[t], a.seg_hi[t], lane, grp, xbj, row_bytes, acc, pol);
   }
   reduce_groups<LPG>(acc);
   if (grp == 0) store_row<LPG>(part, colok, acc, 1.f, 0);
@@ -288,20 +312,21 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
 // one row, the whole warp: G lane groups share its entries
 template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U, bool ATT = false>
 __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lane, int grp, int lig,
-                                         const bool (&colok)[NJ], const char* const (&xbj)[NJ], uint32_t row_bytes) {
+                                         const bool (&colok)[NJ], const char* const (&xbj)[NJ], uint32_t row_bytes,
+                                         const L2Pol& pol) {
     float acc[NJ][VEC];
     zero(acc);
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
     if constexpr (ATT) {
       AttState at{__ldg(a.el + row), -INFINITY, 0.f};
       warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj,
-                                                     row_bytes, acc, &at);
+                                                     row_bytes, acc, pol, &at);
       reduce_groups<LPG>(acc);
       float st = at.s;
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) st += __shfl_xor_sync(0xffffffffu, st, off);
       const float inv = st > 0.f ? 1.f / st : 0.f;
-      if (grp == 0) store_row<LPG>(y, colok, acc, (a.rs ? __ldg(a.rs + row) : 1.f) * inv, a.relu);
+      if (grp == 0) store_row<LPG>(y, colok, acc, (a.rs ? __ldg(a.rs + row) : 1.f) * inv, a.relu, nullptr, 0.f, &pol);
       return;
     }
     if constexpr (PH) {
@@ -309,17 +334,18 @@ __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lan
       for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
         int64_t lo, hi;
         phase_part(a, row, r, 0, INT64_MAX, lo, hi);
-        warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc);
+        warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc, pol);
       }
     } else {
-      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc);
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc,
+                                         pol);
     }
     reduce_groups<LPG>(acc);
     if (grp == 0) {
       if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
       else
         store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
-                       a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+                       a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta, &pol);
     }
 }
 
@@ -344,12 +370,13 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k
   const char* xbj[NJ];
   slice_setup<VEC, LPG>(a, lig, colok, xbj);
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
+  const L2Pol pol = make_l2pol(a.l2hint);
   for (int64_t t = warp; t < a.n_seg + a.n_rows; t += nwarps) {
     if (t < a.n_seg) {
-      do_segment<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, t, lane, grp, lig, colok, xbj, row_bytes);
+      do_segment<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, t, lane, grp, lig, colok, xbj, row_bytes, pol);
       continue;
     }
-    warp_row<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
+    warp_row<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes, pol);
   }
 }
 
@@ -366,10 +393,11 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   const char* xbj[NJ];
   slice_setup<VEC, LPG>(a, lig, colok, xbj);
   const uint32_t row_bytes = (uint32_t)(a.ldx * 4);
+  const L2Pol pol = make_l2pol(a.l2hint);
   // heavy segments, then the wide light rows (degree > wide_deg): whole warps, largest first
   for (int64_t t = warp; t < a.n_seg + a.n_lwide; t += nwarps) {
-    if (t < a.n_seg) do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes);
-    else warp_row<VEC, LPG, NJ, W, CS, PH, UW>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes);
+    if (t < a.n_seg) do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes, pol);
+    else warp_row<VEC, LPG, NJ, W, CS, PH, UW>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes, pol);
   }
   // the other light rows: one LPG-lane group per row
   for (int64_t t0 = a.n_lwide + warp * G; t0 < a.n_rows; t0 += nwarps * G) {
@@ -395,16 +423,16 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
       for (int u = 0; u < U; ++u) {  // entries past the row end: last entry, weight 0
         const bool ok = e + u < re;
         const int64_t ee = ok ? e + u : re - 1;
-        cu[u] = (uint32_t)__ldg(a.col_idx + ee);
-        wu[u] = ok ? (W ? __ldg(a.vals + ee) : 1.f) : 0.f;
-        if (CS) wu[u] *= __ldg(a.cs + cu[u]);
+        cu[u] = (uint32_t)ldg_stream(a.col_idx + ee, pol.stream);
+        wu[u] = ok ? (W ? ldg_stream(a.vals + ee, pol.stream) : 1.f) : 0.f;
+        if (CS) wu[u] *= ldg_pol(a.cs + cu[u], pol.keep);
       }
       float x[U][NJ][VEC];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
 #pragma unroll
         for (int j = 0; j < NJ; ++j)
-          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j]);
+          ldv<VEC>(reinterpret_cast<const float*>(xbj[j] + (uint64_t)cu[u] * row_bytes), x[u][j], pol.keep);
       }
 #pragma unroll
       for (int u = 0; u < U; ++u)
@@ -417,7 +445,7 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
     if (PH && !a.last) store_row<LPG>(y, colok, acc, 1.f, 0);
     else
       store_row<LPG>(y, colok, acc, a.rs ? __ldg(a.rs + row) : 1.f, a.relu,
-                     a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta);
+                     a.B ? a.B + row * a.ldb + a.k0 + (int64_t)lig * VEC : nullptr, a.beta, &pol);
   }
 }
 
@@ -610,6 +638,7 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
              g->order + g->n_heavy, std::max<int64_t>(0, g->n_wide - g->n_heavy), g->n_seg, g->seg_lo, g->seg_hi,
              nullptr, 0, B, ldb, beta};
+  a.l2hint = l2hint_enabled();
   // phases slice like the whole aggregation: the 64-wide slices also keep the L1 hit rate
   const int64_t kw = spmm_slice_width(g, K, vec4, di.l2_bytes, g->n_cols);
   float* partial = nullptr;  // heavy-segment partials: this slice's columns start at partial + pk0
@@ -687,6 +716,11 @@ granii_status launch_spmm_ex(const granii_graph_s* g, const float* vals, const f
 }
 
 bool spmm_att_supported(const granii_graph_s* g) { return g->avg_deg() >= 16.f; }
+
+int l2hint_enabled() {
+  const char* e = getenv("GRANII_L2HINT");
+  return e && e[0] == '0' ? 0 : 1;
+}
 
 granii_status launch_spmm_att(const granii_graph_s* g, const float* el, const float* er, const float* X, int64_t ldx,
                               int64_t K, float* Y, int64_t ldy, const float* rs, bool relu, cudaStream_t st) {
