@@ -1,6 +1,8 @@
 // api.cu -- the extern "C" entry points of include/granii.h: argument
 // validation, error reporting, dispatch to the kernels.  No compute here.
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <string>
 
 #include "internal.h"
@@ -11,6 +13,22 @@ void set_error(const std::string& m) { g_last_error = m; }
 granii_status fail(granii_status st, const std::string& m) {
   g_last_error = m;
   return st;
+}
+
+int resident_ctas(const void* fn, int threads, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> cache;
+  std::lock_guard<std::mutex> lk(mu);
+  const auto key = std::make_pair(fn, threads);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem) != cudaSuccess || n < 1) {
+    cudaGetLastError();
+    n = 1;
+  }
+  cache[key] = n;
+  return n;
 }
 
 granii_status dev_info(DevInfo* out) {

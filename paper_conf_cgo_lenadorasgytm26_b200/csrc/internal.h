@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <atomic>
 #include <string>
 #include <vector>
@@ -50,6 +51,15 @@ struct DevInfo {
   int64_t l2_bytes = 126ll << 20;
 };
 granii_status dev_info(DevInfo* out);
+// CTAs of `fn` resident per SM at `threads` threads (cudaOccupancyMaxActiveBlocksPerMultiprocessor,
+// cached per kernel).  Grid-stride (persistent) kernels launch sms x this many CTAs: a grid of
+// 8 CTAs / SM where 6 fit runs in 1.33 waves, the last third on a quarter of the machine.
+int resident_ctas(const void* fn, int threads, size_t smem = 0);
+template <typename F>
+inline int64_t persistent_grid(F* fn, int threads, int sms, int64_t want) {
+  const int64_t cap = (int64_t)sms * resident_ctas((const void*)fn, threads);
+  return std::max<int64_t>(1, std::min<int64_t>(want, cap));
+}
 
 // ----------------------------------------------------------------- tracing
 // RAII scope around one launcher call: counts kernel launches always; records

@@ -342,17 +342,22 @@ static int lpg_for_degree(float avg) {
 }
 
 template <int LPG, bool ADD, bool LR, bool SM>
-static void go1(const SddmmArgs& a, int blocks, cudaStream_t st) {
-  k_sddmm1<LPG, ADD, LR, SM><<<blocks, 256, 0, st>>>(a);
+static void go1(const SddmmArgs& a, int blocks, int sms, cudaStream_t st) {
+  // three full waves of resident CTAs: the degree-ordered rows are irregular, and CTAs that start
+  // as others finish balance the tail (B200 products-shaped, scores + softmax per layer: 8 CTAs / SM
+  // where 6 fit 1.21 ms, persistent 1.07, 2 waves 1.01, 3 waves 0.99; GRANII_SDDMM_WAVES overrides)
+  const int wv = getenv("GRANII_SDDMM_WAVES") ? atoi(getenv("GRANII_SDDMM_WAVES")) : 3;
+  const int64_t b = persistent_grid(k_sddmm1<LPG, ADD, LR, SM>, 256, sms * std::max(wv, 1), blocks * std::max(wv, 1));
+  k_sddmm1<LPG, ADD, LR, SM><<<(unsigned)b, 256, 0, st>>>(a);
 }
 
 template <bool ADD, bool LR, bool SM>
-static void go1_lpg(int lpg, const SddmmArgs& a, int blocks, cudaStream_t st) {
+static void go1_lpg(int lpg, const SddmmArgs& a, int blocks, int sms, cudaStream_t st) {
   switch (lpg) {
-    case 32: go1<32, ADD, LR, SM>(a, blocks, st); break;
-    case 16: go1<16, ADD, LR, SM>(a, blocks, st); break;
-    case 8: go1<8, ADD, LR, SM>(a, blocks, st); break;
-    default: go1<4, ADD, LR, SM>(a, blocks, st); break;
+    case 32: go1<32, ADD, LR, SM>(a, blocks, sms, st); break;
+    case 16: go1<16, ADD, LR, SM>(a, blocks, sms, st); break;
+    case 8: go1<8, ADD, LR, SM>(a, blocks, sms, st); break;
+    default: go1<4, ADD, LR, SM>(a, blocks, sms, st); break;
   }
 }
 
@@ -378,11 +383,11 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
     const bool add = base == GRANII_SDDMM_ADD;
     // dispatch the 8 (add, lrelu, softmax) variants
     if (add) {
-      if (lr) { if (sm) go1_lpg<true, true, true>(lpg, a, blocks, st); else go1_lpg<true, true, false>(lpg, a, blocks, st); }
-      else { if (sm) go1_lpg<true, false, true>(lpg, a, blocks, st); else go1_lpg<true, false, false>(lpg, a, blocks, st); }
+      if (lr) { if (sm) go1_lpg<true, true, true>(lpg, a, blocks, di.sms, st); else go1_lpg<true, true, false>(lpg, a, blocks, di.sms, st); }
+      else { if (sm) go1_lpg<true, false, true>(lpg, a, blocks, di.sms, st); else go1_lpg<true, false, false>(lpg, a, blocks, di.sms, st); }
     } else {
-      if (lr) { if (sm) go1_lpg<false, true, true>(lpg, a, blocks, st); else go1_lpg<false, true, false>(lpg, a, blocks, st); }
-      else { if (sm) go1_lpg<false, false, true>(lpg, a, blocks, st); else go1_lpg<false, false, false>(lpg, a, blocks, st); }
+      if (lr) { if (sm) go1_lpg<false, true, true>(lpg, a, blocks, di.sms, st); else go1_lpg<false, true, false>(lpg, a, blocks, di.sms, st); }
+      else { if (sm) go1_lpg<false, false, true>(lpg, a, blocks, di.sms, st); else go1_lpg<false, false, false>(lpg, a, blocks, di.sms, st); }
     }
     GR_CHECK_LAUNCH();
     if (sm) GR_TRY(heavy_softmax(g, out, di.sms, st));
@@ -392,7 +397,8 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   if (lr) return fail(GRANII_ERR_UNSUPPORTED, "LEAKYRELU with K > 1 is not supported");
   const bool vec4 = (ldu % 4 == 0) && (ldv % 4 == 0) && ((uintptr_t)V % 16 == 0);
   const int blocks = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n_light + g->n_seg, 8), (int64_t)di.sms * 8));
-#define GO(VEC, LPG, NJ) k_sddmm_dot<VEC, LPG, NJ><<<blocks, 256, 0, st>>>(a)
+#define GO(VEC, LPG, NJ) \
+  k_sddmm_dot<VEC, LPG, NJ><<<(unsigned)persistent_grid(k_sddmm_dot<VEC, LPG, NJ>, 256, di.sms, blocks), 256, 0, st>>>(a)
   if (vec4) {
     if (K <= 16) GO(4, 4, 1);
     else if (K <= 32) GO(4, 8, 1);
@@ -417,10 +423,10 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
     const int64_t units = ceil_div(n_light, 32 / lpg);
     const int b2 = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(units, 8), (int64_t)di.sms * 8));
     switch (lpg) {
-      case 32: k_row_softmax<32><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
-      case 16: k_row_softmax<16><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
-      case 8: k_row_softmax<8><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
-      default: k_row_softmax<4><<<b2, 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      case 32: k_row_softmax<32><<<(unsigned)persistent_grid(k_row_softmax<32>, 256, di.sms, b2), 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      case 16: k_row_softmax<16><<<(unsigned)persistent_grid(k_row_softmax<16>, 256, di.sms, b2), 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      case 8: k_row_softmax<8><<<(unsigned)persistent_grid(k_row_softmax<8>, 256, di.sms, b2), 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
+      default: k_row_softmax<4><<<(unsigned)persistent_grid(k_row_softmax<4>, 256, di.sms, b2), 256, 0, st>>>(n_light, a.order, g->row_ptr, out); break;
     }
     GR_CHECK_LAUNCH();
     GR_TRY(heavy_softmax(g, out, di.sms, st));
