@@ -101,6 +101,14 @@ __global__ void k_deg_only(int64_t n, const int64_t* __restrict__ rp, int32_t* _
     deg[i] = (int32_t)(rp[i + 1] - rp[i]);
 }
 
+__global__ void k_ord_rp(int64_t n, const int32_t* __restrict__ order, const int64_t* __restrict__ rp,
+                         longlong2* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = order[i];
+    out[i] = make_longlong2(rp[r], rp[r + 1]);
+  }
+}
+
 __global__ void k_iota(int64_t n, int32_t* v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     v[i] = (int32_t)i;
@@ -376,6 +384,8 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
     CK(cub::DeviceRadixSort::SortPairsDescending(tmp, b4, deg, deg_sorted, iota, g->order, (int)g->n_rows, 0, 32,
                                                  st));
   }
+  CK(cudaMalloc(&g->ord_rp, std::max<int64_t>(g->n_rows, 1) * sizeof(longlong2)));
+  if (g->n_rows > 0) k_ord_rp<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->order, g->row_ptr, g->ord_rp);
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(st));
 
@@ -466,6 +476,7 @@ void graph_free(granii_graph_s* g) {
   cudaFree(g->row_ptr);
   cudaFree(g->col_idx);
   cudaFree(g->order);
+  cudaFree(g->ord_rp);
   cudaFree(g->seg_ptr);
   cudaFree(g->seg_lo);
   cudaFree(g->seg_hi);

@@ -98,6 +98,9 @@ struct granii_graph_s {
   float* dinv_cols = nullptr;     // device, n_cols (== dinv_rows when world == 1)
   float* dinv2_rows = nullptr;    // device, n_rows: 1 / deg (post-scale of one hop fused with the next pre-scale)
   int32_t* order = nullptr;       // device, n_rows: owned rows by descending degree
+  longlong2* ord_rp = nullptr;    // device, n_rows: {row_ptr[order[t]], row_ptr[order[t] + 1]} -- a row's
+                                  // entry range in schedule order, one coalesced load (no dependent
+                                  // random row_ptr access after order[t])
   int32_t* owner_off = nullptr;   // device, n_rows x (world+1) when world > 1: entries of row i whose
                                   // column is owned by rank p are [rp_i + off[i][p], rp_i + off[i][p+1])
   // heavy rows (degree > seg_len) = order[0 .. n_heavy); each is cut into segments of

@@ -38,6 +38,7 @@ struct SddmmArgs {
   float scale;
   float* __restrict__ out;
   const int32_t* __restrict__ order;       // light rows (degree-descending), n_rows of them
+  const longlong2* __restrict__ ord_rp;    // their entry ranges, same order
   int64_t n_seg;                           // heavy-row segments: warp-wide items
   const int64_t* __restrict__ seg_lo;
   const int64_t* __restrict__ seg_hi;
@@ -84,7 +85,8 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
     const int64_t t = t0 + grp;
     const bool live = t < a.n_rows;
     const int64_t row = live ? a.order[t] : 0;
-    const int64_t rs = live ? a.row_ptr[row] : 0, re = live ? a.row_ptr[row + 1] : 0;
+    const longlong2 rr = live ? a.ord_rp[t] : make_longlong2(0, 0);  // independent of order[t]
+    const int64_t rs = rr.x, re = rr.y;
     const float u = live ? __ldg(a.U + row * a.ldu) : 0.f;
     constexpr int U4 = 4;
     if constexpr (!SOFTMAX) {
@@ -370,7 +372,7 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
   const int64_t n_light = g->n_rows - g->n_heavy;
   SddmmArgs a{n_light, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order + g->n_heavy,
-              g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, l2hint_enabled()};
+              g->ord_rp + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, l2hint_enabled()};
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double gathered = (double)g->n_cols * 4.0 * (double)K;  // V, read once in the compulsory count

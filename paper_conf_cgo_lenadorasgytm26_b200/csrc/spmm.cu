@@ -83,6 +83,7 @@ struct SpmmArgs {
   const float* __restrict__ cs;
   int relu;
   const int32_t* __restrict__ order;       // light rows, degree-descending
+  const longlong2* __restrict__ ord_rp;    // their entry ranges, same order
   int64_t n_lwide;                         // group-per-row kernel: order[0 .. n_lwide) get a warp each
   // heavy rows (degree > GRANII_SEG) are cut into segments: warp-wide work items whose
   // unscaled partial sums go to `partial` [n_seg][ldp] and are combined in fixed order
@@ -311,16 +312,18 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
 
 // one row, the whole warp: G lane groups share its entries
 template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int U, bool ATT = false>
-__device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lane, int grp, int lig,
+__device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t t, int lane, int grp, int lig,
                                          const bool (&colok)[NJ], const char* const (&xbj)[NJ], uint32_t row_bytes,
                                          const L2Pol& pol) {
+    // t: position in the light-row schedule; the row and its entry range are independent loads
+    const int64_t row = a.order[t];
+    const longlong2 rr = a.ord_rp[t];
     float acc[NJ][VEC];
     zero(acc);
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
     if constexpr (ATT) {
       AttState at{__ldg(a.el + row), -INFINITY, 0.f};
-      warp_range<VEC, LPG, NJ, false, true, U, true>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj,
-                                                     row_bytes, acc, pol, &at);
+      warp_range<VEC, LPG, NJ, false, true, U, true>(a, rr.x, rr.y, lane, grp, xbj, row_bytes, acc, pol, &at);
       reduce_groups<LPG>(acc);
       float st = at.s;
 #pragma unroll
@@ -337,8 +340,7 @@ __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t row, int lan
         warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc, pol);
       }
     } else {
-      warp_range<VEC, LPG, NJ, W, CS, U>(a, a.row_ptr[row], a.row_ptr[row + 1], lane, grp, xbj, row_bytes, acc,
-                                         pol);
+      warp_range<VEC, LPG, NJ, W, CS, U>(a, rr.x, rr.y, lane, grp, xbj, row_bytes, acc, pol);
     }
     reduce_groups<LPG>(acc);
     if (grp == 0) {
@@ -376,7 +378,7 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k
       do_segment<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, t, lane, grp, lig, colok, xbj, row_bytes, pol);
       continue;
     }
-    warp_row<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes, pol);
+    warp_row<VEC, LPG, NJ, W, CS, PH, U, ATT>(a, t - a.n_seg, lane, grp, lig, colok, xbj, row_bytes, pol);
   }
 }
 
@@ -397,13 +399,14 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
   // heavy segments, then the wide light rows (degree > wide_deg): whole warps, largest first
   for (int64_t t = warp; t < a.n_seg + a.n_lwide; t += nwarps) {
     if (t < a.n_seg) do_segment<VEC, LPG, NJ, W, CS, PH, UW>(a, t, lane, grp, lig, colok, xbj, row_bytes, pol);
-    else warp_row<VEC, LPG, NJ, W, CS, PH, UW>(a, a.order[t - a.n_seg], lane, grp, lig, colok, xbj, row_bytes, pol);
+    else warp_row<VEC, LPG, NJ, W, CS, PH, UW>(a, t - a.n_seg, lane, grp, lig, colok, xbj, row_bytes, pol);
   }
   // the other light rows: one LPG-lane group per row
   for (int64_t t0 = a.n_lwide + warp * G; t0 < a.n_rows; t0 += nwarps * G) {
     const int64_t t = t0 + grp;
     if (t >= a.n_rows) continue;
     const int64_t row = a.order[t];
+    const longlong2 rr = a.ord_rp[t];
     float acc[NJ][VEC];
     zero(acc);
     float* y = a.Y + row * a.ldy + a.k0 + (int64_t)lig * VEC;
@@ -413,8 +416,8 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
       if constexpr (PH) {
         phase_part(a, row, part, 0, INT64_MAX, rs0, re);
       } else {
-        rs0 = a.row_ptr[row];
-        re = a.row_ptr[row + 1];
+        rs0 = rr.x;
+        re = rr.y;
       }
     for (int64_t e = rs0; e < re; e += U) {
       uint32_t cu[U];
@@ -636,7 +639,8 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   const float share = ph ? float(ph->p1 - ph->p0 - (ph->skip >= 0 ? 1 : 0)) / float(g->world) : 1.f;
   const bool warp_mode = g->avg_deg() * share >= 16.f;
   SpmmArgs a{g->n_rows - g->n_heavy, g->row_ptr, g->col_idx, vals, X, ldx, 0, 0, Y, ldy, rs, cs, relu ? 1 : 0,
-             g->order + g->n_heavy, std::max<int64_t>(0, g->n_wide - g->n_heavy), g->n_seg, g->seg_lo, g->seg_hi,
+             g->order + g->n_heavy, g->ord_rp + g->n_heavy, std::max<int64_t>(0, g->n_wide - g->n_heavy), g->n_seg,
+             g->seg_lo, g->seg_hi,
              nullptr, 0, B, ldb, beta};
   a.l2hint = l2hint_enabled();
   // phases slice like the whole aggregation: the 64-wide slices also keep the L1 hit rate
