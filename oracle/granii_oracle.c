@@ -104,7 +104,7 @@ void oracle_features(int64_t N, const int64_t* row_ptr, int64_t* out) {
     if (d < mn) mn = d;
     if (d == 0) z++;
   }
-  /* top-1% share: selection by repeated max (slow, obviously correct for test sizes) */
+  /* top-1% share: sort the degrees ascending, sum the last ceil(N/100) */
   qsort(deg, (size_t)N, sizeof(int64_t), cmp_u64);   /* degrees are >= 0: unsigned order == signed */
   int64_t k = (N + 99) / 100, top = 0;
   for (int64_t t = 0; t < k && t < N; ++t) top += deg[N - 1 - t];
