@@ -132,6 +132,11 @@ granii_status granii_graph_export_local(granii_graph g, int64_t* h_row_ptr, int3
  * h_row_ptr int64[local rows + 1], h_col_idx int32[*nnz_t] global ids (size it with
  * granii_graph_transpose_nnz).  INVALID_ARG when no transpose is kept. */
 granii_status granii_graph_transpose_nnz(granii_graph g, int64_t* nnz_t);
+/* Host wall time of graph creation by phase, ms4[0..3] = CSR build (validate, sort, dedupe,
+ * row_ptr / col_idx), featurize (degrees, dinv, the integer features: the input inspection
+ * whose overhead PAPER L365 quotes), partition + schedule (row blocks, degree order, hub
+ * segments), transpose (BUILD_TRANSPOSE).  Each phase ends at a stream sync. */
+granii_status granii_graph_timings(granii_graph g, double* ms4);
 granii_status granii_graph_export_transpose(granii_graph g, int64_t* h_row_ptr, int32_t* h_col_idx);
 
 /* ------------------------------------------------------------------------ */

@@ -298,6 +298,12 @@ granii_status granii_graph_export_csr(granii_graph g, int64_t* h_row_ptr, int32_
   API_END
 }
 
+granii_status granii_graph_timings(granii_graph g, double* ms4) {
+  GR_ARG(g && ms4, "NULL argument");
+  for (int i = 0; i < 4; ++i) ms4[i] = g->create_ms[i];
+  return GRANII_OK;
+}
+
 granii_status granii_graph_transpose_nnz(granii_graph g, int64_t* nnz_t) {
   GR_ARG(g && nnz_t, "NULL argument");
   GR_ARG(g->T, "no transpose kept (create with GRANII_BUILD_TRANSPOSE on a directed graph)");

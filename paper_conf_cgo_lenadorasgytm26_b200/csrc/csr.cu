@@ -12,6 +12,8 @@
 #include <algorithm>
 #include <cmath>
 
+#include <chrono>
+
 #include "internal.h"
 
 namespace granii {
@@ -211,6 +213,13 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
     }
   }
 
+  using clk = std::chrono::steady_clock;
+  auto t_mark = clk::now();
+  auto lap = [&](int phase) {  // called right after a stream sync: host time = device time of the phase
+    const auto now = clk::now();
+    g->create_ms[phase] += std::chrono::duration<double, std::milli>(now - t_mark).count();
+    t_mark = now;
+  };
   int* d_bad = nullptr;
   unsigned long long* d_acc = nullptr;
   uint64_t *k0 = nullptr, *k1 = nullptr;
@@ -275,6 +284,8 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   CK(cudaMalloc(&dinv_full, std::max<int64_t>(N, 1) * sizeof(float)));
   k_row_ptr<<<grid_for(N + 1), 256, 0, st>>>(N, k0, nnz, cb, rp_full);
   if (nnz > 0) k_cols<<<grid_for(nnz), 256, 0, st>>>(nnz, k0, (uint64_t(1) << cb) - 1, col_full);
+  CK(cudaStreamSynchronize(st));
+  lap(0);
 
   // degrees, dinv, features
   CK(cudaMallocAsync(&deg, std::max<int64_t>(N, 1) * sizeof(int32_t), st));
@@ -293,6 +304,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   unsigned long long hacc[8];
   CK(cudaMemcpyAsync(hacc, d_acc, sizeof(hacc), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
+  lap(1);
   g->features[0] = N;
   g->features[1] = nnz;
   g->features[2] = nnz;
@@ -436,6 +448,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   }
   cleanup();
   CK(cudaStreamSynchronize(st));
+  lap(2);
 #undef CK
   if ((flags & GRANII_BUILD_TRANSPOSE) && !sym) {
     // Ãᵀ = the same build over the reversed edges, over Ã's row blocks; D̃ stays Ã's row degrees
@@ -461,6 +474,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
       return fail(GRANII_ERR_CUDA, std::string("transpose dinv: ") + cudaGetErrorString(e));
     }
     g->T = t;
+    g->create_ms[3] = std::chrono::duration<double, std::milli>(clk::now() - t_mark).count();
   }
   *out = g;
   return GRANII_OK;

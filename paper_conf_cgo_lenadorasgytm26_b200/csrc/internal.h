@@ -118,6 +118,10 @@ struct granii_graph_s {
   int64_t wide_deg = 32, n_wide = 0;
   int64_t features[GRANII_NUM_FEATURES] = {0};
   int device = 0;
+  // host wall time of the creation phases (ms): CSR build (validate, sort, dedupe, row_ptr / col_idx),
+  // featurize (degrees, dinv, integer features), partition + schedule (order, ord_rp, hub segments),
+  // transpose (BUILD_TRANSPOSE) -- PAPER L365 quotes the featurizer's overhead on its own
+  double create_ms[4] = {0, 0, 0, 0};
   granii_graph_s* T = nullptr;    // Ãᵀ over the same owned rows (GRANII_BUILD_TRANSPOSE, directed graphs);
                                   // its dinv arrays are Ã's (D̃ = Ã's row degrees, R4)
   // the graph the transposed aggregations of the backward run over (Mᵀ = M when symmetric)

@@ -103,6 +103,11 @@ static granii_status gathered_spmm(const Ctx& c, GatherBuf& gb, const float* val
                                    const float* rs, const float* cs, bool relu, const float* B = nullptr,
                                    int64_t ldb = 0, float beta = 0.f) {
   const granii_graph_s* g = c.g;
+  // K % 4 != 0: the float4 gathers read the row's last vector whole, padding columns [K, K4) included
+  // (they only ever reach Y's padding); nothing writes them, so zero this rank's before anyone reads
+  if (K % 4 != 0 && g->n_rows > 0)
+    GR_CUDA(cudaMemset2DAsync(gb.mine + K, (size_t)gb.ld * sizeof(float), 0, (size_t)(round_up(K, 4) - K) * sizeof(float),
+                              (size_t)g->n_rows, c.st));
   if (!c.dist()) return launch_spmm_ex(g, vals, gb.all, gb.ld, K, Y, ldy, rs, cs, relu, B, ldb, beta, c.st);
   const int P = overlap_enabled() && g->owner_off ? comm_phases(g, K, vals != nullptr, cs != nullptr) : 1;
   if (P <= 1) {

@@ -75,6 +75,7 @@ _SIGS = {
     "granii_graph_query": ([_p, ctypes.POINTER(graph_info)], ctypes.c_int),
     "granii_graph_export_csr": ([_p, _p, _p], ctypes.c_int),
     "granii_graph_transpose_nnz": ([_p, ctypes.POINTER(_i64)], ctypes.c_int),
+    "granii_graph_timings": ([_p, _p], ctypes.c_int),
     "granii_graph_export_transpose": ([_p, _p, _p], ctypes.c_int),
     "granii_graph_dinv": ([_p, ctypes.POINTER(_p)], ctypes.c_int),
     "granii_partition_bounds": ([_i64, _p, _i32, _p], ctypes.c_int),
@@ -212,6 +213,13 @@ def granii_graph_export_csr(g: Graph):
     ci = np.zeros(max(g.nnz, 1), np.int32)
     _check(_lib.granii_graph_export_csr(g.handle, rp.ctypes.data, ci.ctypes.data), "granii_graph_export_csr")
     return rp, ci[: g.nnz]
+
+
+def granii_graph_timings(g: Graph) -> dict:
+    """host ms of the creation phases"""
+    ms = (ctypes.c_double * 4)()
+    _check(_lib.granii_graph_timings(g.handle, ms), "granii_graph_timings")
+    return {"csr_build": ms[0], "featurize": ms[1], "partition_schedule": ms[2], "transpose": ms[3]}
 
 
 def granii_graph_export_transpose(g: Graph):

@@ -27,6 +27,7 @@ def _pad4(k: int) -> int:
 def alloc2d(rows: int, cols: int, device, fill=None) -> torch.Tensor:
     """(rows, cols) fp32 view of a buffer whose row stride is padded to 16 bytes."""
     buf = torch.empty((max(rows, 1), _pad4(cols)), dtype=torch.float32, device=device)
+    buf[:, cols:].zero_()        # padding columns: read (never used) by the float4 gathers of a ragged last vector
     if fill is not None:
         buf.fill_(fill)
     return buf[:rows, :cols]
