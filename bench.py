@@ -311,6 +311,22 @@ def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
     return out
 
 
+def allgather_gbs(G, comm, world, dev, dist, mb=256, reps=5):
+    """bus bandwidth of the library's all-gather on this communicator: each rank receives
+    (G-1) x `mb` MB per call; GB received per rank / seconds, max time over ranks"""
+    count = mb * (1 << 20) // 4
+    buf = torch.zeros(world * count, device=dev)
+    mine = buf[G.granii_comm_query(comm)[1] * count:][:count]
+    st = torch.cuda.current_stream()
+    for _ in range(2):
+        G.granii_comm_allgather(comm, mine, buf, count)
+    ms = time_region(lambda: G.granii_comm_allgather(comm, mine, buf, count), reps, st)
+    t = torch.tensor([ms], device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    del buf
+    return (world - 1) * count * 4 / (float(t.item()) / 1e3) / 1e9
+
+
 class LaunchError(RuntimeError):
     pass
 
@@ -412,6 +428,9 @@ def main():
                      "watchdog_ms": int(os.environ.get("GRANII_COMM_TIMEOUT_MS", "120000"))}
         # failure detection: a collective stuck for longer than this aborts the communicator
         G.granii_comm_watchdog(comm, comm_info["watchdog_ms"])
+        # the selector's all-gather slope, measured on this communicator before any selection
+        comm_info["allgather_gbs"] = allgather_gbs(G, comm, world, dev, dist)
+        os.environ["GRANII_ALLGATHER_GBS"] = f"{comm_info['allgather_gbs']:.3f}"
 
     # ---------------------------------------------------------------- setup (not timed)
     t_setup = time.perf_counter()
@@ -546,7 +565,7 @@ def main():
                    "l2": "no flush: per-step inputs exceed L2 (H %.0f MB, col_idx %.0f MB vs 126 MB L2)" % (
                        w.n * dims[0] * 4 / 1e6, info.nnz * 4 / 1e6),
                    "parallelism": f"row-partition x{world}" + (" (NCCL all-gather)" if world > 1 else ""),
-                   "comm": comm_info,
+                   "comm": dict(comm_info, nccl_register=net.nccl_register) if comm_info else None,
                    "cuda_graph": bool(use_graph),
                    "profile_pass": "separate eager pass (graph replay)" if use_graph else "inside the timed region"},
         "clocks": clk.summary(),

@@ -111,6 +111,14 @@ __global__ void k_ord_rp(int64_t n, const int32_t* __restrict__ order, const int
   }
 }
 
+__global__ void k_permute_off(int64_t n, int G1, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
+                              int32_t* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n * G1; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = i / G1, p = i % G1;
+    out[i] = off[(int64_t)order[t] * G1 + p];
+  }
+}
+
 __global__ void k_iota(int64_t n, int32_t* v) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     v[i] = (int32_t)i;
@@ -398,6 +406,12 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   }
   CK(cudaMalloc(&g->ord_rp, std::max<int64_t>(g->n_rows, 1) * sizeof(longlong2)));
   if (g->n_rows > 0) k_ord_rp<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->order, g->row_ptr, g->ord_rp);
+  if (g->owner_off) {
+    CK(cudaMalloc(&g->ord_off, std::max<int64_t>(g->n_rows, 1) * (world + 1) * sizeof(int32_t)));
+    if (g->n_rows > 0)
+      k_permute_off<<<grid_for(g->n_rows * (world + 1)), 256, 0, st>>>(g->n_rows, world + 1, g->order, g->owner_off,
+                                                                      g->ord_off);
+  }
   CK(cudaGetLastError());
   CK(cudaStreamSynchronize(st));
 
@@ -484,6 +498,7 @@ void graph_free(granii_graph_s* g) {
   if (!g) return;
   graph_free(g->T);
   cudaFree(g->owner_off);
+  cudaFree(g->ord_off);
   cudaFree(g->dinv2_rows);
   if (g->dinv_cols != g->dinv_rows) cudaFree(g->dinv_cols);
   cudaFree(g->dinv_rows);

@@ -103,6 +103,8 @@ struct granii_graph_s {
                                   // random row_ptr access after order[t])
   int32_t* owner_off = nullptr;   // device, n_rows x (world+1) when world > 1: entries of row i whose
                                   // column is owned by rank p are [rp_i + off[i][p], rp_i + off[i][p+1])
+  int32_t* ord_off = nullptr;     // the same rows of owner_off in schedule order (ord_off[t] = owner_off[order[t]]):
+                                  // a phase's entry range of schedule position t without a dependent load
   // heavy rows (degree > seg_len) = order[0 .. n_heavy); each is cut into segments of
   // seg_len entries that are scheduled as independent warp-wide work items
   int64_t seg_len = 2048;

@@ -47,8 +47,11 @@ struct CostModel {
 //   gat_bwd_a/b     : [1, streamed GB (idx, er / row records), row GB, gathered GB from L2,
 //                      gathered GB from HBM, M rows, M dependent gather steps]  (gat_bwd.cu)
 //   elementwise     : [1, GB]
-//   allgather       : [1, GB received per GPU]  (not calibrated: the pool has one GPU; the
-//                     slope is an assumed NCCL bus bandwidth of 0.65 TB/s on NVLink 5)
+//   allgather       : [1, GB received per GPU]  (the pool this was built on has one GPU: the default
+//                     slope is B200_PROFILING.md's measured 8-rank NCCL bus bandwidth on this pool,
+//                     725 GB/s; GRANII_ALLGATHER_GBS -- which bench.py sets from an all-gather it
+//                     times on the real communicator before selecting -- or an "allgather" line of
+//                     the calibration file replaces it)
 static CostModel defaults() {
   CostModel m;
   m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0, 1.0};
@@ -59,8 +62,14 @@ static CostModel defaults() {
   m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
   m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
+  // group-per-row graphs (average degree < 16) run other kernels (spmm.cu k_spmm_group, the
+  // lane-group GAT backward passes): their own coefficients (B200 fit: SpMM median error
+  // 13 % with one model for both schedules, 9 % / 7 % split)
+  m.coef["spmm_g"] = m.coef["spmm"];
+  m.coef["gat_bwd_a_g"] = m.coef["gat_bwd_a"];
+  m.coef["gat_bwd_b_g"] = m.coef["gat_bwd_b"];
   m.coef["elementwise"] = {0.004, 1.0 / 5.5};
-  m.coef["allgather"] = {0.020, 1.0 / 0.65};
+  m.coef["allgather"] = {0.020, 1.0 / 0.725};
   return m;
 }
 
@@ -68,12 +77,21 @@ static std::mutex g_mu;
 static std::map<std::string, CostModel> g_cache;
 static std::string g_last_path;  // calibration of the last selection (used by the phase planner)
 
+// GRANII_ALLGATHER_GBS: all-gather bus bandwidth measured on this job's communicator
+static void comm_override(CostModel* m) {
+  if (const char* e = getenv("GRANII_ALLGATHER_GBS")) {
+    const double gbs = atof(e);
+    if (gbs > 0.0) m->coef["allgather"][1] = 1000.0 / gbs;
+  }
+}
+
 static granii_status load_model(const char* path, CostModel* out) {
   std::lock_guard<std::mutex> lk(g_mu);
   std::string key = path ? path : "";
   auto it = g_cache.find(key);
   if (it != g_cache.end()) {
     *out = it->second;
+    comm_override(out);
     if (!key.empty()) g_last_path = key;
     return GRANII_OK;
   }
@@ -102,6 +120,7 @@ static granii_status load_model(const char* path, CostModel* out) {
   g_cache[key] = m;
   g_last_path = key;
   *out = m;
+  comm_override(out);
   return GRANII_OK;
 }
 
@@ -131,9 +150,12 @@ static double l2_hit(const In& in, double K, double cols) {
 enum { P_SPMM_W = 0, P_SPMM_U = 1, P_SPMM_U_CS = 2, P_SDDMM1 = 3, P_SDDMM1_SM = 4, P_GEMM = 5, P_GEMM_NOSTORE = 6,
        P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10, P_GAT_BWD_A = 11, P_GAT_BWD_B = 12 };
 
-static const char* prim_model(int p) {
+// the warp-per-row / group-per-row split follows the kernels' own switch (spmm.cu, gat_bwd.cu)
+static bool group_mode(const In& in) { return in.avg < 16.0; }
+
+static const char* prim_model(int p, const In& in) {
   switch (p) {
-    case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: return "spmm";
+    case P_SPMM_W: case P_SPMM_U: case P_SPMM_U_CS: return group_mode(in) ? "spmm_g" : "spmm";
     case P_SDDMM1: return "sddmm1";
     case P_SDDMM1_SM: return "sddmm1_softmax";
     case P_GEMM: return "gemm";
@@ -141,8 +163,8 @@ static const char* prim_model(int p) {
     case P_GEMM_TN: return "gemm_tn";
     case P_ELEMENTWISE: return "elementwise";
     case P_ALLGATHER: return "allgather";
-    case P_GAT_BWD_A: return "gat_bwd_a";
-    case P_GAT_BWD_B: return "gat_bwd_b";
+    case P_GAT_BWD_A: return group_mode(in) ? "gat_bwd_a_g" : "gat_bwd_a";
+    case P_GAT_BWD_B: return group_mode(in) ? "gat_bwd_b_g" : "gat_bwd_b";
   }
   return "";
 }
@@ -194,7 +216,7 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
 static double cost(const CostModel& m, const In& in, int p, double K1, double K2 = 0) {
   if (p == P_ALLGATHER && in.world <= 1) return 0.0;
   const std::vector<double> f = features(in, p, K1, K2);
-  const std::vector<double>& c = m.coef.at(prim_model(p));
+  const std::vector<double>& c = m.coef.at(prim_model(p, in));
   double s = 0;
   for (size_t i = 0; i < f.size() && i < c.size(); ++i) s += c[i] * f[i];
   return s;
@@ -215,7 +237,7 @@ static double agg_schedule(const CostModel& m, const In& in, int p, double K, in
   double best = ag + sp;
   if (!overlap_on()) return best;
   const int G = (int)in.world;
-  const std::vector<double>& c = m.coef.at("spmm");
+  const std::vector<double>& c = m.coef.at(prim_model(P_SPMM_U, in));
   // per extra phase (measured on B200, products- and Reddit-shaped partitions at G = 8,
   // profiles/r01/phase_overhead.json): ~40 us of launch + tail per K slice, ~0.45 ns per row
   // (the dependent row-metadata chain, not hidden when a phase has few entries per row), and
@@ -436,7 +458,7 @@ granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t 
   for (size_t i = 0; i < f.size(); ++i) feats[i] = f[i];
   *n = (int32_t)f.size();
   if (model_name) {
-    strncpy(model_name, prim_model(prim), 31);
+    strncpy(model_name, prim_model(prim, inputs_of(g)), 31);
     model_name[31] = 0;
   }
   return GRANII_OK;

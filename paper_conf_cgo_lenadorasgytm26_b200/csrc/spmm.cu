@@ -102,6 +102,7 @@ struct SpmmArgs {
   // `first`: start from zero, else from the raw partial already in Y (light rows) / partial
   // (segments); `last`: apply the epilogue.
   const int32_t* __restrict__ owner_off;   // [n_rows][G1]
+  const int32_t* __restrict__ ord_off;     // owner_off of the light rows in schedule order [n_rows][G1]
   const int32_t* __restrict__ seg_row;     // row of each heavy segment
   int G1, p0, p1, skip, first, last;
   // fused additive attention (GAT, Eq. 4-6; ATT kernels): the weights are computed on the fly,
@@ -120,10 +121,9 @@ struct AttState {
 
 // part r (0, or 1 after a skipped block) of the entries of `row` within [l0, h0) whose column lies
 // in the phase's owner blocks
-__device__ __forceinline__ void phase_part(const SpmmArgs& a, int64_t row, int r, int64_t l0, int64_t h0,
-                                           int64_t& lo, int64_t& hi) {
-  const int32_t* o = a.owner_off + row * a.G1;
-  const int64_t base = a.row_ptr[row];
+// (o: the row's owner offsets, base: its first entry)
+__device__ __forceinline__ void phase_part(const SpmmArgs& a, const int32_t* o, int64_t base, int r, int64_t l0,
+                                           int64_t h0, int64_t& lo, int64_t& hi) {
   const int b0 = r == 0 ? a.p0 : a.skip + 1;
   const int b1 = (r == 0 && a.skip >= 0) ? a.skip : a.p1;
   lo = max(l0, base + (int64_t)o[b0]);
@@ -300,7 +300,8 @@ __device__ __forceinline__ void do_segment(const SpmmArgs& a, int64_t t, int lan
     if (!a.first && grp == 0) load_partial<LPG>(part, colok, acc);
     for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {  // the range(s) are computed when needed
       int64_t lo, hi;
-      phase_part(a, a.seg_row[t], r, a.seg_lo[t], a.seg_hi[t], lo, hi);
+      const int64_t sr = a.seg_row[t];
+      phase_part(a, a.owner_off + sr * a.G1, a.row_ptr[sr], r, a.seg_lo[t], a.seg_hi[t], lo, hi);
       warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc, pol);
     }
   } else {
@@ -336,7 +337,7 @@ __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t t, int lane,
       if (!a.first && grp == 0) load_partial<LPG>(y, colok, acc);
       for (int r = 0; r < (a.skip >= 0 ? 2 : 1); ++r) {
         int64_t lo, hi;
-        phase_part(a, row, r, 0, INT64_MAX, lo, hi);
+        phase_part(a, a.ord_off + t * a.G1, rr.x, r, 0, INT64_MAX, lo, hi);
         warp_range<VEC, LPG, NJ, W, CS, U>(a, lo, hi, lane, grp, xbj, row_bytes, acc, pol);
       }
     } else {
@@ -414,7 +415,7 @@ __global__ void __launch_bounds__(256, 3) k_spmm_group(SpmmArgs a) {
     for (int part = 0; part < (PH && a.skip >= 0 ? 2 : 1); ++part) {
       int64_t rs0, re;
       if constexpr (PH) {
-        phase_part(a, row, part, 0, INT64_MAX, rs0, re);
+        phase_part(a, a.ord_off + t * a.G1, rr.x, part, 0, INT64_MAX, rs0, re);
       } else {
         rs0 = rr.x;
         re = rr.y;
@@ -658,6 +659,7 @@ static granii_status spmm_impl(const granii_graph_s* g, const float* vals, const
   }
   if (ph) {
     a.owner_off = g->owner_off;
+    a.ord_off = g->ord_off + g->n_heavy * (g->world + 1);
     a.seg_row = g->seg_row;
     a.G1 = g->world + 1;
     a.p0 = ph->p0;

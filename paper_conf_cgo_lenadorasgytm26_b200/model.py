@@ -77,6 +77,15 @@ class GNN:
             ws = max(ws, w)
             self.saved_floats.append(s)
         self.workspace = torch.empty(max(ws, 1), dtype=torch.uint8, device=device)
+        # the gather buffers of the all-gathers live in the workspace: register it with NCCL so
+        # collectives can use it in place (ncclCommRegister; a no-op on loopback / stub transports)
+        self.nccl_handle, self.nccl_register = None, None
+        if comm is not None and comm.world > 1 and os.environ.get("GRANII_NCCL_REGISTER", "1") != "0":
+            try:
+                self.nccl_handle = G.granii_comm_register(comm, self.workspace)
+                self.nccl_register = "registered" if self.nccl_handle else "not applicable (transport)"
+            except G.GraniiError as e:   # NCCL without registration support: collectives still work
+                self.nccl_register = f"not registered: {e}"
         R = graph.n_rows
         self.outs = [alloc2d(R, L.K2, device) for L in layers]
         self.saved = [torch.empty(max(s, 1), dtype=torch.float32, device=device) if s else None
@@ -87,6 +96,13 @@ class GNN:
         self.da = [(torch.empty(L.K2, dtype=torch.float32, device=device),
                     torch.empty(L.K2, dtype=torch.float32, device=device)) if L.model == G.GAT else None
                    for L in layers]
+
+    def __del__(self):
+        if getattr(self, "nccl_handle", None) and self.comm is not None and self.comm.handle:
+            try:
+                G.granii_comm_deregister(self.comm, self.nccl_handle)
+            except Exception:  # noqa: BLE001 -- interpreter shutdown
+                pass
 
     def args(self, i: int, H: torch.Tensor) -> G.layer_args:
         L = self.layers[i]

@@ -158,18 +158,34 @@ def fit(samples):
     return coefs, report
 
 
+def relabel(samples):
+    """model keys of samples taken before the warp-per-row / group-per-row split (select.cpp
+    group_mode: average degree < 16): the graph's average degree from its K = 16 unweighted SpMM
+    sample (streamed GB = nnz x 4 B for an unsliced SpMM, M rows)"""
+    avg = {}
+    for s in samples:
+        if s["prim"] == 1 and s["K1"] == 16:
+            avg[s["graph"]] = s["f"][1] / 4e-9 / (s["f"][5] * 1e6)
+    for s in samples:
+        if s["model"] in ("spmm", "gat_bwd_a", "gat_bwd_b") and avg.get(s["graph"], 99.0) < 16.0:
+            s["model"] += "_g"
+    return samples
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=os.path.join(ROOT, "calib", "b200.txt"))
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--refit", default=None, help="refit from a saved *_samples.json instead of measuring")
     args = ap.parse_args()
     t0 = time.time()
-    samples = sweep(args.quick)
+    samples = relabel(json.load(open(args.refit))["samples"]) if args.refit else sweep(args.quick)
     coefs, report = fit(samples)
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         f.write(f"# GRANII B200 cost-model coefficients (tools/calibrate.py, {len(samples)} samples, "
-                f"{torch.cuda.get_device_name(0)}, {time.strftime('%Y-%m-%d')})\n")
+                f"{'refit of ' + args.refit if args.refit else torch.cuda.get_device_name(0)}, "
+                f"{time.strftime('%Y-%m-%d')})\n")
         f.write("# model coef... (feature order: paper_conf_cgo_lenadorasgytm26_b200/csrc/select.cpp)\n")
         for model, c in coefs.items():
             f.write(f"# {model}: n={report[model]['n']} median rel err {report[model]['median_rel_err']:.3f} "

@@ -32,6 +32,13 @@ SWEEP = {
     "mycielskian": ("gcn", [(32, 32), (32, 256), (256, 32), (256, 256), (1024, 32), (32, 1024)]),
 }
 MODELS = {"gcn": 0, "gat": 1, "sgc": 2, "tagcn": 3, "gin": 4}
+# training (forward + backward of a hidden layer, dH included; SELECT_TRAINING costs the backward too)
+TRAIN_SWEEP = {
+    "pubmed": ("gcn+gat", [(32, 256), (256, 32), (64, 256)]),
+    "arxiv": ("gcn+gat", [(128, 256), (256, 40), (64, 512)]),
+    "reddit": ("gcn", [(602, 256), (256, 41), (32, 256)]),
+    "products": ("gcn+gat", [(100, 256), (256, 47)]),
+}
 
 
 def spec_for(G, LayerSpec, model, k1, k2, comp=None):
@@ -61,11 +68,60 @@ def timeit(fn, reps=5, trials=3):
     return best
 
 
+def train_rows(out, calib):
+    """fwd + bwd (hidden layer: dH computed) of every candidate vs SELECT_TRAINING's choice"""
+    for name, (models, pairs) in TRAIN_SWEEP.items():
+        w = synth.WORKLOADS[name]
+        s, d = w.edges(0, DEV)
+        fl = G.ADD_SELF_LOOPS | (G.SYMMETRIZE if w.symmetrize else G.BUILD_TRANSPOSE)
+        g = G.granii_graph_csr_create(w.n, s, d, fl)
+        print(f"[train {name}] n={w.n} nnz={g.nnz}", flush=True)
+        for mname in models.split("+"):
+            model = MODELS[mname]
+            for (k1, k2) in pairs:
+                H = alloc2d(w.n, k1, DEV)
+                H.copy_(synth.features(1, w.n, k1, device=DEV))
+                up = alloc2d(w.n, k2, DEV, fill=0.01)
+                times = {}
+                for c in G.COMPS[model]:
+                    net = GNN(g, [spec_for(G, LayerSpec, model, k1, k2, c)], DEV)
+
+                    def step():
+                        net.forward(H)
+                        net.backward(up, need_input_grad=True)
+                    times[G.COMP_NAMES[c]] = timeit(step)
+                    del net
+                shape = G.shape_args(k1, k2)
+                sel, pred = G.granii_select_ex(g, model, shape, calib, G.SELECT_TRAINING | G.SELECT_REFINE)
+                sel_m, _ = G.granii_select_ex(g, model, shape, calib, G.SELECT_TRAINING)
+                sel_np, pred_np = G.granii_select_ex(g, model, shape, calib, G.SELECT_TRAINING | G.SELECT_NO_PREFILTER)
+                sel_f, _ = G.granii_select_ex(g, model, shape, calib)        # forward-only selection (the paper)
+                best = min(times, key=times.get)
+                row = {"graph": name, "model": mname, "mode": "fwd+bwd", "K1": k1, "K2": k2, "ms": times,
+                       "best": best, "selected": G.COMP_NAMES[sel],
+                       "regret": times[G.COMP_NAMES[sel]] / times[best] - 1,
+                       "selected_model_only": G.COMP_NAMES[sel_m],
+                       "regret_model_only": times[G.COMP_NAMES[sel_m]] / times[best] - 1,
+                       "regret_no_prefilter": times[G.COMP_NAMES[sel_np]] / times[best] - 1,
+                       "regret_forward_only_selection": times[G.COMP_NAMES[sel_f]] / times[best] - 1,
+                       "config_regret": 0.0, "static_regret": 0.0,
+                       "predicted_ms": {G.COMP_NAMES[k]: v for k, v in pred_np.items()}}
+                row["pred_rel_err"] = {k: v / times[k] - 1 for k, v in row["predicted_ms"].items()}
+                out["rows"].append(row)
+                print(f"  train {mname} {k1:5d}->{k2:5d} best={best:12s} sel={row['selected']:12s} "
+                      f"regret={row['regret']:.3f} model_only={row['regret_model_only']:.3f} "
+                      f"fwd_sel={row['regret_forward_only_selection']:.3f}", flush=True)
+                del H, up
+        del g
+        torch.cuda.empty_cache()
+
+
 def main():
     out = {"device": torch.cuda.get_device_name(0), "calib": DEFAULT_CALIB, "when": time.strftime("%Y-%m-%d %H:%M"),
            "rows": []}
     calib = DEFAULT_CALIB if os.path.exists(DEFAULT_CALIB) else None
-    for name, (models, pairs) in SWEEP.items():
+    train_only = "--train-only" in sys.argv
+    for name, (models, pairs) in ({} if train_only else SWEEP).items():
         w = synth.WORKLOADS[name]
         s, d = w.edges(0, DEV)
         g = G.granii_graph_csr_create(w.n, s, d, G.ADD_SELF_LOOPS | (G.SYMMETRIZE if w.symmetrize else 0))
@@ -96,19 +152,22 @@ def main():
                     cfg, static = ("GAT_RECOMP" if k1 < k2 else "GAT_REUSE"), "GAT_REUSE"
                 else:
                     cfg, static = (f"{pre}_DYN_UPD" if k1 > k2 else f"{pre}_DYN_AGG"), f"{pre}_DYN_AGG"
-                row = {"graph": name, "model": mname, "K1": k1, "K2": k2, "ms": times, "best": best,
+                row = {"graph": name, "model": mname, "mode": "fwd", "K1": k1, "K2": k2, "ms": times, "best": best,
                        "selected": G.COMP_NAMES[sel], "regret": times[G.COMP_NAMES[sel]] / times[best] - 1,
                        "selected_model_only": G.COMP_NAMES[sel_m],
                        "regret_model_only": times[G.COMP_NAMES[sel_m]] / times[best] - 1,
                        "regret_no_prefilter": times[G.COMP_NAMES[sel_np]] / times[best] - 1,
                        "config_regret": times[cfg] / times[best] - 1, "static_regret": times[static] / times[best] - 1,
                        "predicted_ms": {G.COMP_NAMES[k]: v for k, v in pred.items()}}
+                row["pred_rel_err"] = {k: v / times[k] - 1 for k, v in row["predicted_ms"].items()}
                 out["rows"].append(row)
                 print(f"  {mname} {k1:5d}->{k2:5d} best={best:12s} sel={row['selected']:12s} regret={row['regret']:.3f} "
                       f"config={row['config_regret']:.3f} static={row['static_regret']:.3f}", flush=True)
                 del H
         del g
         torch.cuda.empty_cache()
+    if "--no-train" not in sys.argv:
+        train_rows(out, calib)
     rg = [r["regret"] for r in out["rows"]]
     out["summary"] = {"n": len(rg), "max_regret": max(rg), "mean_regret": sum(rg) / len(rg),
                       "within_10pct": sum(x <= 0.10 for x in rg),
@@ -116,6 +175,15 @@ def main():
                       "within_10pct_model_only": sum(r["regret_model_only"] <= 0.10 for r in out["rows"]),
                       "max_config_regret": max(r["config_regret"] for r in out["rows"]),
                       "max_static_regret": max(r["static_regret"] for r in out["rows"])}
+    for mode in ("fwd", "fwd+bwd"):
+        rr = [r for r in out["rows"] if r["mode"] == mode]
+        if rr:
+            errs = sorted(abs(e) for r in rr for e in r["pred_rel_err"].values())
+            out["summary_" + mode] = {"n": len(rr), "max_regret": max(r["regret"] for r in rr),
+                                      "max_regret_model_only": max(r["regret_model_only"] for r in rr),
+                                      "within_10pct_model_only": sum(r["regret_model_only"] <= 0.10 for r in rr),
+                                      "pred_abs_rel_err_median": errs[len(errs) // 2], "pred_abs_rel_err_max": errs[-1]}
+            print(mode, json.dumps(out["summary_" + mode]))
     out["summary_by_model"] = {}
     for mname in MODELS:
         rr = [r["regret"] for r in out["rows"] if r["model"] == mname]
