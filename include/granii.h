@@ -384,6 +384,11 @@ granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t coun
  * so a launcher can check that N processes really formed one N-rank communicator) and the NCCL
  * version (0 for loopback / stub).  Errors: NCCL if the communicator was aborted. */
 granii_status granii_comm_query(granii_comm c, int32_t* nranks, int32_t* rank, int32_t* nccl_version);
+/* The aggregation schedule the planner picks for a K-wide SpMM on this partitioned graph (N1,
+ * DESIGN.md §7): phases (1 = all-gather then SpMM; P >= 2 = own block under the transfer, then the
+ * other blocks in P-1 chunks as they land) and the modelled times of both (ms).  Host only. */
+granii_status granii_comm_plan(granii_graph g, int64_t K, int32_t weighted, int32_t col_scale, int32_t* phases,
+                               double* ms_allgather_then_spmm, double* ms_planned);
 /* Failure detection.  Starts (timeout_ms > 0) or stops (<= 0) a host watchdog
  * thread for the communicator: every collective the library issues records an event on its
  * stream (except under CUDA-graph capture); every ~20 ms the watchdog polls

@@ -530,6 +530,16 @@ granii_status granii_comm_allreduce_sum(granii_comm c, float* d_buf, size_t coun
   return comm_allreduce_sum(c, d_buf, count, (cudaStream_t)stream);
 }
 
+granii_status granii_comm_plan(granii_graph g, int64_t K, int32_t weighted, int32_t col_scale, int32_t* phases,
+                               double* ms_allgather_then_spmm, double* ms_planned) {
+  GR_ARG(g && phases && K > 0, "bad argument");
+  double a = 0, b = 0;
+  *phases = comm_plan(g, K, weighted != 0, col_scale != 0, &a, &b);
+  if (ms_allgather_then_spmm) *ms_allgather_then_spmm = a;
+  if (ms_planned) *ms_planned = b;
+  return GRANII_OK;
+}
+
 granii_status granii_comm_query(granii_comm c, int32_t* nranks, int32_t* rank, int32_t* nccl_version) {
   GR_ARG(c && nranks && rank && nccl_version, "NULL argument");
   return comm_query(c, nranks, rank, nccl_version);

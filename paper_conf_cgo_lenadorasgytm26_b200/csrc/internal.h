@@ -172,6 +172,7 @@ int64_t spmm_slices(double avg_deg, double cols, int64_t K, int64_t l2_bytes);
 bool dyn_prescale(double nnz, double rows, double avg_deg, double cols, int64_t K, int64_t l2_bytes);
 // phases of an overlapped aggregation on a partitioned graph (select.cpp; 1 = all-gather first)
 int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale);
+int comm_plan(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale, double* t1, double* tp);
 granii_status launch_spmm_phase(const granii_graph_s* g, const float* vals, const float* X, int64_t ldx, int64_t K,
                                 float* Y, int64_t ldy, const float* rs, const float* cs, bool relu, const float* B,
                                 int64_t ldb, float beta, const SpmmPhase& ph, cudaStream_t st);

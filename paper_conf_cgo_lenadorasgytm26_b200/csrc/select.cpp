@@ -238,24 +238,33 @@ static double agg_schedule(const CostModel& m, const In& in, int p, double K, in
   if (!overlap_on()) return best;
   const int G = (int)in.world;
   const std::vector<double>& c = m.coef.at(prim_model(P_SPMM_U, in));
-  // per extra phase (measured on B200, products- and Reddit-shaped partitions at G = 8,
-  // profiles/r01/phase_overhead.json): ~40 us of launch + tail per K slice, ~0.45 ns per row
-  // (the dependent row-metadata chain, not hidden when a phase has few entries per row), and
-  // the read + write of the partial output rows
+  // a phase over n of the G owner blocks: the entries whose columns lie in them (n / G of them,
+  // every row visited: the model's per-row term stays whole) gathering from an n / G slice of the
+  // operand -- the own block alone (1 / G of X) often fits L2 where the whole X does not (G = 8
+  // products-shaped projection: 2 phases 2.66 ms of per-rank compute vs 3.07 ms unphased,
+  // profiles/r02/scaling_projection_products-gcn2-infer_P*.json); every phase after the first
+  // adds ~40 us of launch + tail per K slice and re-reads + re-writes the partial output rows
+  auto phase = [&](double n) {
+    In b = in;
+    b.nnz = in.nnz * n / G;
+    b.xcols = in.xcols * n / G;
+    b.nseg = in.nseg * n / G;
+    return cost(m, b, p, K);
+  };
   double slices = 1.0;
   if (in.avg >= 32.0 && in.ncols * K * 4.0 > 0.6 * in.l2) {
     const double fit = std::floor(0.55 * in.l2 / (in.ncols * 4.0) / 64.0) * 64.0;
     if (fit >= 64.0) slices = std::ceil(K / fit);
   }
-  const double h = 0.040 * slices + 0.45e-6 * in.R + 2.0 * in.R * K * 4.0 * 1e-9 * c[2];
+  const double h = 0.040 * slices + 2.0 * in.R * K * 4.0 * 1e-9 * c[2];
   for (int P = 2; P <= G; ++P) {
-    double t = sp / G;  // own block, under the transfer
+    double t = phase(1.0);  // own block, under the transfer
     int done = 0;
     for (int q = 0; q < P - 1; ++q) {
       const int n = (G - 1) * (q + 1) / (P - 1) - (G - 1) * q / (P - 1);  // blocks in this chunk
       done += n;
       const double landed = ag * (double)done / (G - 1);
-      t = std::max(t, landed) + sp * n / G + h;
+      t = std::max(t, landed) + phase((double)n) + h;
     }
     if (t < best) {
       best = t;
@@ -433,6 +442,13 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, const gra
 // number of phases of an overlapped aggregation (1 = all-gather then SpMM); GRANII_COMM_PHASES
 // overrides.  weighted / col_scale pick the SpMM model (P_SPMM_W / P_SPMM_U_CS / P_SPMM_U).
 int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale) {
+  return comm_plan(g, K, weighted, col_scale, nullptr, nullptr);
+}
+
+// the planner's choice and its predicted times (P = 1 and the chosen P), for diagnostics
+int comm_plan(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale, double* t1, double* tp) {
+  if (t1) *t1 = 0.0;
+  if (tp) *tp = 0.0;
   if (g->world <= 1) return 1;
   if (const char* e = getenv("GRANII_COMM_PHASES")) {
     const int P = atoi(e);
@@ -447,7 +463,11 @@ int comm_phases(const granii_graph_s* g, int64_t K, bool weighted, bool col_scal
   CostModel m;
   if (load_model(path.empty() ? nullptr : path.c_str(), &m) != GRANII_OK) m = defaults();
   int P = 1;
-  agg_schedule(m, inputs_of(g), weighted ? P_SPMM_W : col_scale ? P_SPMM_U_CS : P_SPMM_U, (double)K, &P);
+  const In in = inputs_of(g);
+  const int prim = weighted ? P_SPMM_W : col_scale ? P_SPMM_U_CS : P_SPMM_U;
+  const double best = agg_schedule(m, in, prim, (double)K, &P);
+  if (t1) *t1 = cost(m, in, P_ALLGATHER, (double)K) + cost(m, in, prim, (double)K);
+  if (tp) *tp = best;
   return P;
 }
 

@@ -110,6 +110,8 @@ _SIGS = {
     "granii_comm_allgather": ([_p, _p, _p, _sz, _p], ctypes.c_int),
     "granii_comm_allreduce_sum": ([_p, _p, _sz, _p], ctypes.c_int),
     "granii_comm_query": ([_p, ctypes.POINTER(_i32), ctypes.POINTER(_i32), ctypes.POINTER(_i32)], ctypes.c_int),
+    "granii_comm_plan": ([_p, _i64, _i32, _i32, ctypes.POINTER(_i32), ctypes.POINTER(ctypes.c_double),
+                          ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
     "granii_comm_watchdog": ([_p, _i64], ctypes.c_int),
     "granii_comm_check": ([_p], ctypes.c_int),
     "granii_comm_register": ([_p, _p, _sz, ctypes.POINTER(_p)], ctypes.c_int),
@@ -408,6 +410,14 @@ def granii_comm_query(c: Comm):
     n, r, v = _i32(), _i32(), _i32()
     _check(_lib.granii_comm_query(c.handle, ctypes.byref(n), ctypes.byref(r), ctypes.byref(v)), "granii_comm_query")
     return n.value, r.value, v.value
+
+
+def granii_comm_plan(g: Graph, K: int, weighted: bool = False, col_scale: bool = False):
+    """(phases, modelled ms of all-gather-then-SpMM, modelled ms of the planned schedule)"""
+    P, a, b = _i32(), ctypes.c_double(), ctypes.c_double()
+    _check(_lib.granii_comm_plan(g.handle, K, int(weighted), int(col_scale), ctypes.byref(P), ctypes.byref(a),
+                                 ctypes.byref(b)), "granii_comm_plan")
+    return P.value, a.value, b.value
 
 
 def granii_comm_watchdog(c: Comm, timeout_ms: int):

@@ -66,6 +66,12 @@ def rank_step_ms(G, spec, w, src, dst, flags, rank, world, dev, steps, warmup, c
     G.granii_profile_enable(False)
     out = {"rank": rank, "rows": R, "local_nnz": info.local_nnz, "compute_ms": ms, "per_primitive_ms": prof,
            "bytes_in_per_step": (b1 - b0) / steps, "compositions": [L.comp for L in net.layers]}
+    if world > 1:   # the planner's schedule for every aggregation width of the model (N1)
+        out["plan"] = {}
+        for K in sorted(set(dims)):
+            for kind, wgt, cs in (("weighted", True, False), ("unweighted", False, False), ("col_scale", False, True)):
+                P, t1, tp = G.granii_comm_plan(g, K, wgt, cs)
+                out["plan"][f"K{K}_{kind}"] = {"phases": P, "model_ms_allgather_then_spmm": t1, "model_ms_planned": tp}
     del net, g, H
     torch.cuda.empty_cache()
     return out, info.nnz
