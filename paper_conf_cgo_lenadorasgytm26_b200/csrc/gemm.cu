@@ -118,6 +118,16 @@ __device__ __forceinline__ void tf32_split(float x, float& hi, float& lo) {
   lo = x - hi;
 }
 
+// lo = x - trunc_tf32(x) (exact in fp32), for an MMA that reads x itself as the truncated hi
+__device__ __forceinline__ float4 tf32_lo_trunc(float4 x) {
+  float4 l;
+  l.x = x.x - __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
+  l.y = x.y - __uint_as_float(__float_as_uint(x.y) & 0xFFFFE000u);
+  l.z = x.z - __uint_as_float(__float_as_uint(x.z) & 0xFFFFE000u);
+  l.w = x.w - __uint_as_float(__float_as_uint(x.w) & 0xFFFFE000u);
+  return l;
+}
+
 // ======================================================================= tcgen05 kernel
 constexpr int TC_BM = 128, TC_BK = 32;  // 32 fp32 = one 128-byte swizzle row
 
@@ -442,22 +452,26 @@ __host__ __device__ constexpr uint32_t idesc_tf32_mn(int M, int N) {
   return idesc_tf32(M, N) | (1u << 15) | (1u << 16);  // a_major = b_major = MN
 }
 
-template <int BN>
+// BK: node rows per k-block.  16 halves a stage (raw A + A_lo + raw B + B_lo: 48 KB at BN = 256)
+// so 4 stages fit instead of 2 -- the 2-stage ring left the converters waiting on the TMA (ncu:
+// a third of their samples on the full barrier, tensor pipe 61 % active)
+template <int BN, int BK = TC_BK>
 struct TnCfg {
-  static constexpr int A_BYTES = TC_BM * TC_BK * 4;  // 128 (M) x 32 (k) fp32 = 4 MN atoms
-  static constexpr int B_BYTES = BN * TC_BK * 4;
+  static constexpr int A_BYTES = TC_BM * BK * 4;  // 128 (M) x BK (k) fp32 = 4 MN atoms
+  static constexpr int B_BYTES = BN * BK * 4;
   static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int STAGES = (STAGE * 3 <= 200 * 1024) ? 3 : 2;
+  static constexpr int STAGES_FIT = 200 * 1024 / STAGE;
+  static constexpr int STAGES = STAGES_FIT > 6 ? 6 : STAGES_FIT;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
 };
 
-template <int BN>
+template <int BN, int BK = TC_BK>
 __global__ void __launch_bounds__(192, 1)
     k_gemm_tn_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, int M, int N,
                  int kblocks_per_split, int total_kblocks, float* __restrict__ part, uint32_t dlbo, uint32_t dsbo,
-                 uint32_t dkstep) {
-  using Cfg = TnCfg<BN>;
+                 uint32_t dkstep, int raw_hi) {
+  using Cfg = TnCfg<BN, BK>;
   constexpr int S = Cfg::STAGES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1 KB-aligned base by pointer arithmetic on the __shared__ array (an integer round trip would
@@ -502,11 +516,11 @@ __global__ void __launch_bounds__(192, 1)
         const uint32_t ph = (kb / S) & 1;
         mbar_wait(&empty[s], ph ^ 1);
         mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
-        const int r = (kb0 + kb) * TC_BK;
+        const int r = (kb0 + kb) * BK;
 #pragma unroll
-        for (int t = 0; t < TC_BM / 32; ++t) tma_load_2d(&tmA, &full[s], a_hi(s) + t * 4096, m0 + 32 * t, r);
+        for (int t = 0; t < TC_BM / 32; ++t) tma_load_2d(&tmA, &full[s], a_hi(s) + t * 32 * BK * 4, m0 + 32 * t, r);
 #pragma unroll
-        for (int t = 0; t < BN / 32; ++t) tma_load_2d(&tmB, &full[s], b_hi(s) + t * 4096, n0 + 32 * t, r);
+        for (int t = 0; t < BN / 32; ++t) tma_load_2d(&tmB, &full[s], b_hi(s) + t * 32 * BK * 4, n0 + 32 * t, r);
       }
     }
   } else if (warp == 1) {
@@ -520,7 +534,7 @@ __global__ void __launch_bounds__(192, 1)
         const uint32_t ah = smem_u32(a_hi(s)), al = smem_u32(a_lo(s));
         const uint32_t bh = smem_u32(b_hi(s)), bl = smem_u32(b_lo(s));
 #pragma unroll
-        for (int k = 0; k < TC_BK / 8; ++k) {  // one 8-row k group (1 KB) per MMA
+        for (int k = 0; k < BK / 8; ++k) {  // one 8-row k group (1 KB) per MMA
           const uint32_t off = k * (dkstep & 0xFFFF);
           const uint64_t dah = desc_sw128_mn(ah + off, dlbo, dsbo), dal = desc_sw128_mn(al + off, dlbo, dsbo);
           const uint64_t dbh = desc_sw128_mn(bh + off, dlbo, dsbo), dbl = desc_sw128_mn(bl + off, dlbo, dsbo);
@@ -542,27 +556,37 @@ __global__ void __launch_bounds__(192, 1)
       float4* alp = reinterpret_cast<float4*>(a_lo(s));
       float4* bhp = reinterpret_cast<float4*>(b_hi(s));
       float4* blp = reinterpret_cast<float4*>(b_lo(s));
+      if (raw_hi) {
+        // the raw stage IS the hi operand: the tf32 MMA reads the top 19 bits of each fp32 (truncation),
+        // so hi = trunc(x) needs no store and only lo = x - trunc(x) (exact) is written -- half the
+        // converters' shared-memory stores (the kernel is shared-memory-bandwidth bound)
 #pragma unroll 4
-      for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) {
-        const float4 x = ahp[i];
-        float4 h, l;
-        tf32_split(x.x, h.x, l.x);
-        tf32_split(x.y, h.y, l.y);
-        tf32_split(x.z, h.z, l.z);
-        tf32_split(x.w, h.w, l.w);
-        ahp[i] = h;
-        alp[i] = l;
-      }
+        for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) alp[i] = tf32_lo_trunc(ahp[i]);
 #pragma unroll 4
-      for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) {
-        const float4 x = bhp[i];
-        float4 h, l;
-        tf32_split(x.x, h.x, l.x);
-        tf32_split(x.y, h.y, l.y);
-        tf32_split(x.z, h.z, l.z);
-        tf32_split(x.w, h.w, l.w);
-        bhp[i] = h;
-        blp[i] = l;
+        for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) blp[i] = tf32_lo_trunc(bhp[i]);
+      } else {
+#pragma unroll 4
+        for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) {
+          const float4 x = ahp[i];
+          float4 h, l;
+          tf32_split(x.x, h.x, l.x);
+          tf32_split(x.y, h.y, l.y);
+          tf32_split(x.z, h.z, l.z);
+          tf32_split(x.w, h.w, l.w);
+          ahp[i] = h;
+          alp[i] = l;
+        }
+#pragma unroll 4
+        for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) {
+          const float4 x = bhp[i];
+          float4 h, l;
+          tf32_split(x.x, h.x, l.x);
+          tf32_split(x.y, h.y, l.y);
+          tf32_split(x.z, h.z, l.z);
+          tf32_split(x.w, h.w, l.w);
+          bhp[i] = h;
+          blp[i] = l;
+        }
       }
       fence_proxy_async();
       mbar_arrive(&conv[s]);
@@ -761,18 +785,26 @@ static bool tc_eligible(int64_t M, int64_t N, int64_t K, const float* A, int64_t
 // Aᵀ·B plan: BN multiple of 32 (TMA boxes of 32), split the reduction so the grid
 // fills the 148 SMs (one CTA per SM: ~190 KB smem), >= 8 k-blocks per split.
 struct TnPlan {
-  int bn;
+  int bn, bk;
   int64_t mt, nt, total_kb, kb_per, splits;
 };
+// 16-row k-blocks (4 stages) when several output tiles share the grid (Reddit dW 602 x 256: 5 tiles,
+// 0.765 -> 0.695 ms per step; 602 x 1024: 2.83 -> 2.67); 32-row blocks for one or two tiles over many
+// splits (products GAT dW 100 x 256 and 256 x 47: 1.53 -> 1.68 ms with 16).  GRANII_TN_BK overrides.
+static int tn_bk(int64_t tiles) {
+  if (const char* e = getenv("GRANII_TN_BK")) return atoi(e) == 32 ? 32 : 16;
+  return tiles >= 4 ? 16 : 32;
+}
 static TnPlan tn_plan(int64_t M, int64_t N, int64_t R) {
   TnPlan p;
   p.bn = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
   // (a 128-wide N tile for N = 256 -- three pipeline stages instead of two -- measured 0.78 -> 0.95 ms on 602x256)
   p.mt = ceil_div(M, TC_BM);
   p.nt = ceil_div(N, p.bn);
-  p.total_kb = ceil_div(R, TC_BK);
+  p.bk = tn_bk(p.mt * p.nt);
+  p.total_kb = ceil_div(R, p.bk);
   int64_t splits = std::max<int64_t>(1, ceil_div(148, p.mt * p.nt));
-  splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.total_kb / 8));
+  splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.total_kb / (8 * TC_BK / p.bk)));
   p.kb_per = ceil_div(p.total_kb, splits);
   p.splits = ceil_div(p.total_kb, p.kb_per);
   return p;
@@ -839,26 +871,34 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
       float* part = (float*)ws;
       // MN-major tf32 operands need the 128B swizzle with 32B atoms (descriptor layout type 1)
       // debug override GRANII_TN_DESC=lbo,sbo,kstep,major,layout,tma_swizzle
-      uint32_t dlbo = 4096, dsbo = 512, dkstep = 1024, dmaj = 3, dlay = 1, dswz = 4;
+      // LBO = the byte stride between 32-wide MN atoms = one TMA box of 32 x bk fp32
+      uint32_t dlbo = 32 * p.bk * 4, dsbo = 512, dkstep = 1024, dmaj = 3, dlay = 1, dswz = 4;
       if (const char* e = getenv("GRANII_TN_DESC"))
         sscanf(e, "%u,%u,%u,%u,%u,%u", &dlbo, &dsbo, &dkstep, &dmaj, &dlay, &dswz);
       dkstep = (dkstep & 0xFFFF) | (dmaj << 16);
       dlbo = (dlbo & 0x0FFFFFFFu) | (dlay << 28);
       CUtensorMap ta, tb;
-      if (!make_map(&ta, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, 32, TC_BK, (CUtensorMapSwizzle)dswz) ||
-          !make_map(&tb, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, 32, TC_BK, (CUtensorMapSwizzle)dswz))
+      if (!make_map(&ta, A, (uint64_t)M, (uint64_t)K, (uint64_t)lda, 32, p.bk, (CUtensorMapSwizzle)dswz) ||
+          !make_map(&tb, B, (uint64_t)N, (uint64_t)K, (uint64_t)ldb, 32, p.bk, (CUtensorMapSwizzle)dswz))
         return fail(GRANII_ERR_CUDA, "cuTensorMapEncodeTiled failed (TN)");
       dim3 grid((unsigned)p.mt, (unsigned)p.nt, (unsigned)p.splits);
-#define GR_TN(BN)                                                                                       \
+      const char* rh = getenv("GRANII_TN_RAWHI");
+      const int raw_hi = rh ? (rh[0] != '0') : 1;
+#define GR_TN2(BN, BK)                                                                                  \
   do {                                                                                                  \
     static bool set_ = false;                                                                           \
     if (!set_) {                                                                                        \
-      GR_CUDA(cudaFuncSetAttribute(k_gemm_tn_tc<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize,       \
-                                   TnCfg<BN>::SMEM));                                                   \
+      GR_CUDA(cudaFuncSetAttribute(k_gemm_tn_tc<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,   \
+                                   TnCfg<BN, BK>::SMEM));                                               \
       set_ = true;                                                                                      \
     }                                                                                                   \
-    k_gemm_tn_tc<BN><<<grid, 192, TnCfg<BN>::SMEM, st>>>(ta, tb, (int)M, (int)N, (int)p.kb_per,         \
-                                                         (int)p.total_kb, part, dlbo, dsbo, dkstep);    \
+    k_gemm_tn_tc<BN, BK><<<grid, 192, TnCfg<BN, BK>::SMEM, st>>>(ta, tb, (int)M, (int)N, (int)p.kb_per, \
+                                                                 (int)p.total_kb, part, dlbo, dsbo, dkstep, raw_hi); \
+  } while (0)
+#define GR_TN(BN)                   \
+  do {                              \
+    if (p.bk == 16) GR_TN2(BN, 16); \
+    else GR_TN2(BN, 32);            \
   } while (0)
       switch (p.bn) {
         case 32: GR_TN(32); break;
@@ -867,6 +907,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
         default: GR_TN(256); break;
       }
 #undef GR_TN
+#undef GR_TN2
       GR_CHECK_LAUNCH();
       const int64_t MN = M * N;
       k_sum_splits<<<(unsigned)std::min<int64_t>(ceil_div(MN, 256), 4096), 256, 0, st>>>(MN, (int)p.splits, part, C,
