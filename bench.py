@@ -290,7 +290,12 @@ def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
         out["tensor_frac"] = fl / t / 1e12 / tc
     elif name in ("spmm", "sddmm", "gat_bwd_a", "gat_bwd_b") and l2:
         t_l2, t_hbm = by / (l2 * 1e9), comp / (hbm * 1e9)
-        if t_l2 >= t_hbm:
+        if traffic and st.get("l2_resident", 0) < calls:
+            # the gathered operand does not fit L2: its gathers are DRAM reads at a hit rate the
+            # algorithmic bytes cannot tell -- the binding roof is the DRAM traffic ncu measured
+            out.update(bound="hbm", achieved=traffic / (st["ms"] / calls / 1e3) / 1e9, peak=hbm, unit="GB/s",
+                       peak_note=f"hbm_gbs of {peak_src}: ncu DRAM bytes per call / t (operand exceeds L2)")
+        elif t_l2 >= t_hbm:
             out.update(bound="l2", achieved=by / t / 1e9, peak=l2, unit="GB/s",
                        peak_note="L2 read peak measured by tools/probe/l2_bw.cu (profiles/l2_peak.json), "
                                  "not a driver figure: algorithmic (gathered) bytes / t")
@@ -543,7 +548,12 @@ def main():
             traffic_tab = json.load(open(tp)).get(args.workload, {})
         except Exception:
             traffic_tab = {}
-    per_prim = {k: primitive_roofline(k, v, hbm, tc_peak, peak_src, l2_peak(), traffic_tab.get(k))
+    def traffic_of(k, v):   # DRAM bytes per call: the ncu rate of this primitive x its measured time per call
+        t = traffic_tab.get(k)
+        if isinstance(t, dict) and "dram_bytes_per_ms" in t:
+            return t["dram_bytes_per_ms"] * v["ms"] / max(v["calls"], 1)
+        return t if isinstance(t, (int, float)) else None
+    per_prim = {k: primitive_roofline(k, v, hbm, tc_peak, peak_src, l2_peak(), traffic_of(k, v))
                 for k, v in prof.items()}
     kname = max(prof, key=lambda k: prof[k]["ms"])
     roof = dict(per_prim[kname])

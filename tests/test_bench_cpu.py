@@ -62,3 +62,11 @@ def test_primitive_roofline_bounds():
     st = {"calls": 1, "ms": 1.0, "bytes": 3.25e9, "flops": 1e9}
     r = bench.primitive_roofline("gemm_tc", st, hbm, tc, "measured", l2)
     assert r["bound"] == "hbm" and abs(r["frac"] - 0.5) < 1e-9
+
+
+def test_roofline_gather_beyond_l2_uses_the_dram_counter():
+    """a gather whose operand exceeds L2 is bound by the DRAM traffic ncu measured, not by the
+    algorithmic bytes (whose L2 hit rate is unknown)"""
+    st = {"calls": 2, "ms": 10.0, "bytes": 100e9, "flops": 0.0, "compulsory_bytes": 5e9, "l2_resident": 0}
+    r = bench.primitive_roofline("spmm", st, 6500.0, 1386.0, "measured", 18000.0, traffic=26e9)
+    assert r["bound"] == "hbm" and abs(r["achieved"] - 5200.0) < 1e-6 and abs(r["frac"] - 0.8) < 1e-9
