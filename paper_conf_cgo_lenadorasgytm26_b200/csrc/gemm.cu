@@ -466,12 +466,15 @@ struct TnCfg {
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
 };
 
-template <int BN, int BK = TC_BK>
-__global__ void __launch_bounds__(192, 1)
+// NCW converter warps (warps 2 .. NCW+1); they are also the epilogue, NCW / 4 warps per TMEM lane
+// quadrant splitting the columns
+template <int BN, int BK = TC_BK, int NCW = 4>
+__global__ void __launch_bounds__(64 + 32 * NCW, 1)
     k_gemm_tn_tc(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, int M, int N,
                  int kblocks_per_split, int total_kblocks, float* __restrict__ part, uint32_t dlbo, uint32_t dsbo,
                  uint32_t dkstep, int raw_hi) {
   using Cfg = TnCfg<BN, BK>;
+  constexpr int NCT = 32 * NCW;  // converter threads
   constexpr int S = Cfg::STAGES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1 KB-aligned base by pointer arithmetic on the __shared__ array (an integer round trip would
@@ -494,7 +497,7 @@ __global__ void __launch_bounds__(192, 1)
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 128);
+      mbar_init(&conv[s], NCT);
       mbar_init(&empty[s], 1);
     }
     mbar_init(accum, 1);
@@ -561,12 +564,12 @@ __global__ void __launch_bounds__(192, 1)
         // so hi = trunc(x) needs no store and only lo = x - trunc(x) (exact) is written -- half the
         // converters' shared-memory stores (the kernel is shared-memory-bandwidth bound)
 #pragma unroll 4
-        for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) alp[i] = tf32_lo_trunc(ahp[i]);
+        for (int i = ct; i < Cfg::A_BYTES / 16; i += NCT) alp[i] = tf32_lo_trunc(ahp[i]);
 #pragma unroll 4
-        for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) blp[i] = tf32_lo_trunc(bhp[i]);
+        for (int i = ct; i < Cfg::B_BYTES / 16; i += NCT) blp[i] = tf32_lo_trunc(bhp[i]);
       } else {
 #pragma unroll 4
-        for (int i = ct; i < Cfg::A_BYTES / 16; i += 128) {
+        for (int i = ct; i < Cfg::A_BYTES / 16; i += NCT) {
           const float4 x = ahp[i];
           float4 h, l;
           tf32_split(x.x, h.x, l.x);
@@ -577,7 +580,7 @@ __global__ void __launch_bounds__(192, 1)
           alp[i] = l;
         }
 #pragma unroll 4
-        for (int i = ct; i < Cfg::B_BYTES / 16; i += 128) {
+        for (int i = ct; i < Cfg::B_BYTES / 16; i += NCT) {
           const float4 x = bhp[i];
           float4 h, l;
           tf32_split(x.x, h.x, l.x);
@@ -592,7 +595,8 @@ __global__ void __launch_bounds__(192, 1)
       mbar_arrive(&conv[s]);
     }
     // epilogue: this split's partial tile (zeros if the split is empty)
-    const int quad = warp & 3;
+    const int quad = warp & 3, half = (warp - 2) / 4;  // NCW / 4 warps share a quadrant's columns
+    constexpr int CPW = BN / (NCW / 4);
     const int r = m0 + quad * 32 + lane;
     float* P = part + (int64_t)blockIdx.z * M * N;
     if (nk > 0) {
@@ -600,7 +604,7 @@ __global__ void __launch_bounds__(192, 1)
       tc_fence_after();
     }
 #pragma unroll 1
-    for (int c0 = 0; c0 < BN; c0 += 16) {
+    for (int c0 = half * CPW; c0 < (half + 1) * CPW; c0 += 16) {
       float v[16];
       if (nk > 0) tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + c0, v);
       else
@@ -795,6 +799,12 @@ static int tn_bk(int64_t tiles) {
   if (const char* e = getenv("GRANII_TN_BK")) return atoi(e) == 32 ? 32 : 16;
   return tiles >= 4 ? 16 : 32;
 }
+// 8 converter / epilogue warps (B200: Reddit dW 0.677 -> 0.662 ms per step, products GAT 1.54 -> 1.52;
+// GRANII_TN_NCW=4 for the former 4)
+static int tn_ncw() {
+  const char* e = getenv("GRANII_TN_NCW");
+  return e && atoi(e) == 4 ? 4 : 8;
+}
 static TnPlan tn_plan(int64_t M, int64_t N, int64_t R) {
   TnPlan p;
   p.bn = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
@@ -884,16 +894,21 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
       dim3 grid((unsigned)p.mt, (unsigned)p.nt, (unsigned)p.splits);
       const char* rh = getenv("GRANII_TN_RAWHI");
       const int raw_hi = rh ? (rh[0] != '0') : 1;
-#define GR_TN2(BN, BK)                                                                                  \
+#define GR_TN3(BN, BK, NCW)                                                                             \
   do {                                                                                                  \
     static bool set_ = false;                                                                           \
     if (!set_) {                                                                                        \
-      GR_CUDA(cudaFuncSetAttribute(k_gemm_tn_tc<BN, BK>, cudaFuncAttributeMaxDynamicSharedMemorySize,   \
+      GR_CUDA(cudaFuncSetAttribute(k_gemm_tn_tc<BN, BK, NCW>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
                                    TnCfg<BN, BK>::SMEM));                                               \
       set_ = true;                                                                                      \
     }                                                                                                   \
-    k_gemm_tn_tc<BN, BK><<<grid, 192, TnCfg<BN, BK>::SMEM, st>>>(ta, tb, (int)M, (int)N, (int)p.kb_per, \
-                                                                 (int)p.total_kb, part, dlbo, dsbo, dkstep, raw_hi); \
+    k_gemm_tn_tc<BN, BK, NCW><<<grid, 64 + 32 * NCW, TnCfg<BN, BK>::SMEM, st>>>(                         \
+        ta, tb, (int)M, (int)N, (int)p.kb_per, (int)p.total_kb, part, dlbo, dsbo, dkstep, raw_hi);       \
+  } while (0)
+#define GR_TN2(BN, BK)                     \
+  do {                                     \
+    if (tn_ncw() == 8) GR_TN3(BN, BK, 8);  \
+    else GR_TN3(BN, BK, 4);                \
   } while (0)
 #define GR_TN(BN)                   \
   do {                              \
@@ -908,6 +923,7 @@ granii_status launch_gemm(int64_t M, int64_t N, int64_t K, const float* A, int64
       }
 #undef GR_TN
 #undef GR_TN2
+#undef GR_TN3
       GR_CHECK_LAUNCH();
       const int64_t MN = M * N;
       k_sum_splits<<<(unsigned)std::min<int64_t>(ceil_div(MN, 256), 4096), 256, 0, st>>>(MN, (int)p.splits, part, C,
