@@ -407,7 +407,10 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, const gra
     else if (K1 >= K2) c = {GRANII_GCN_PRE_UPD, GRANII_GCN_DYN_UPD};   // group ">=": update first
     else c = {GRANII_GCN_PRE_AGG, GRANII_GCN_DYN_AGG};                 // group "<": aggregate first
   } else if (model == GRANII_GAT) {
-    c = {GRANII_GAT_REUSE, GRANII_GAT_RECOMP};
+    // offline pruning (offline.py, L226-L233): RECOMP -- the extra GEMM and an SpMM at K1 -- is
+    // unprofitable when K1 >= K2 (it does all of REUSE's work on matrices never smaller, and more)
+    if (!prefilter || K1 < K2) c = {GRANII_GAT_REUSE, GRANII_GAT_RECOMP};
+    else c = {GRANII_GAT_REUSE};
   } else {
     // SGC / TAGCN: the GCN embedding-size rule on (K1, K2); GIN: on (K1, Kh), the width the
     // aggregation runs at (R11 / R23)

@@ -17,8 +17,10 @@ Each internal node records its primitive and the width of the dense operand it m
 (K1 = input, K2 = output embedding size; sparse-value primitives are O(nnz)).
 
 Pruning (L226-L233), for each scenario '>=' (K1 >= K2) and '<' (K1 < K2) separately:
-  rule 1: a tree whose primitive multiset (with sizes) contains another tree's whole multiset
-          is unprofitable (strict superset; equal multisets keep the first tree: duplicates);
+  rule 1: a tree that performs every primitive of another tree -- each at a dense width never
+          smaller than the other's in this scenario -- and more primitives besides is unprofitable
+          (L229's example: "SpMM and a GEMM" vs "only SpMM on the same matrix sizes"); an identical
+          primitive multiset is a duplicate (the first tree is kept);
   rule 2: a tree with the same primitives as another tree but a larger dense width in at
           least one of them (and no smaller one) is unprofitable.
 Trees unprofitable in BOTH scenarios are pruned; the others are promoted and annotated with
@@ -28,8 +30,13 @@ For GCN this yields 12 generated / 8 pruned / 4 promoted trees -- the paper's co
 (L326: "12 and 8") -- and the 4 promoted trees are exactly the library's GCN compositions
 with the annotations of granii_select's prefilter (update-first iff K1 >= K2).  GAT (α fixed
 by the attention over Θ = H W, chain α H W) gives 2 generated / 0 pruned (L326: "2 and 0"), both
-promoted in both scenarios: RECOMP's extra GEMM (L135) and REUSE's wider SpMM are incomparable
-under the two rules, so the choice is left to the cost models -- as the library does for GAT.
+promoted: REUSE in both scenarios, RECOMP (extra GEMM, L135; SpMM at K1) only for K1 < K2, where its
+narrower SpMM can pay for the GEMM -- the sizes the paper evaluates GAT at (L330) and WiseGraph's
+recompute-for-growing-sizes rule (L357).  GIN (reading R23: (Ã + εI) H W1 before the MLP's ReLU,
+a sum in the IR, with the distributive rewrite (P + Q) R -> P R + Q R as an extra candidate) gives 7
+generated / 3 pruned / 4 promoted: the paper counts "8 and 4" (L326); the 4 promoted trees are the
+library's four GIN compositions (PRE = the sum folded into the sparse values, DYN = unweighted SpMM +
+the εH term, each aggregate- or update-first) with the update-first-iff-K1 >= Kh annotation.
 
 Host-only Python: this stage runs once per model at build time, never on the data path.
 """
@@ -56,6 +63,8 @@ class Node:
             return self.name
         if self.prim == "SDDMM" and self.kids == ():
             return "SDDMM(DAD)"
+        if self.prim in ("SpAdd", "Add"):
+            return "(" + " + ".join(k.show() for k in self.kids) + ")"
         return "(" + " ".join(k.show() for k in self.kids) + ")"
 
 
@@ -131,12 +140,19 @@ def primitives(t: Node, attention: bool = False) -> Counter:
         if "(H W)" not in t.show():
             c[("GEMM", "K1K2")] += 1
 
+    seen = set()  # common sub-expressions (L219): an identical subtree is computed once
+
     def rec(n: Node):
-        if n.prim == "SDDMM":
-            c[("SDDMM", "E")] += 1
+        if n.kids:
+            key = n.show()
+            if key in seen:
+                return
+            seen.add(key)
+        if n.prim in ("SDDMM", "SpAdd"):
+            c[(n.prim, "E")] += 1
         elif n.prim == "GEMM":
             c[("GEMM", "K1K2")] += 1
-        elif n.prim in ("SpMM", "RowB"):
+        elif n.prim in ("SpMM", "RowB", "Add"):
             c[(n.prim, n.width)] += 1
         for k in n.kids:
             rec(k)
@@ -152,14 +168,32 @@ def _smaller(a: str, b: str, scen: str) -> bool:
     return (a == "K2") if scen == ">=" else (a == "K1")
 
 
+def _size(w: str | None, scen: str) -> int:
+    """order of the dense widths in a scenario (0 = the smaller one); unsized primitives are 0"""
+    if w not in ("K1", "K2"):
+        return 0
+    return int(w == "K1") if scen == ">=" else int(w == "K2")
+
+
+def _covers(ci: Counter, cj: Counter, scen: str) -> bool:
+    """every primitive of cj matched by a distinct one of ci of the same kind, never smaller"""
+    for kind in {k for k, _ in cj.elements()}:
+        wi = sorted((_size(w, scen) for k, w in ci.elements() if k == kind), reverse=True)
+        wj = sorted((_size(w, scen) for k, w in cj.elements() if k == kind), reverse=True)
+        if len(wi) < len(wj) or any(x < y for x, y in zip(wi, wj)):
+            return False
+    return True
+
+
 def unprofitable(i: int, trees: list[Node], scen: str, attention: bool = False) -> str | None:
     ci = primitives(trees[i], attention)
     for j, t in enumerate(trees):
         if j == i:
             continue
         cj = primitives(t, attention)
-        # rule 1: another tree's whole primitive set is a subset of mine (duplicates: keep the first)
-        if all(ci[k] >= v for k, v in cj.items()) and (sum(cj.values()) < sum(ci.values()) or j < i):
+        # rule 1: I perform all of another tree's primitives, never on smaller matrices, and more
+        # besides; an identical multiset is a duplicate (the first tree is kept)
+        if (ci == cj and j < i) or (sum(ci.values()) > sum(cj.values()) and _covers(ci, cj, scen)):
             return f"rule 1 vs {t.show()}"
         # rule 2: same primitives, the other never larger and somewhere smaller
         ti, tj = sorted(ci.elements()), sorted(cj.elements())
@@ -207,6 +241,67 @@ def gat_chain() -> list[Node]:
     return [_leaf("α", "S"), _leaf("H", "X", "K1"), _leaf("W", "W")]
 
 
+GIN_PRE_AGG, GIN_PRE_UPD, GIN_DYN_AGG, GIN_DYN_UPD = 64, 65, 66, 67
+
+
+def gin_expr() -> list:
+    """GIN (reading R23): agg(H) W1 = (Ã + εI) H W1 -- the sum of the sparse pattern and the scaled
+    identity, then the dense chain; the MLP's ReLU ends the re-associable part (L192)"""
+    return [("+", [_leaf("A", "A")], [_leaf("E", "D")]), _leaf("H", "X", "K1"), _leaf("W", "W")]
+
+
+def _combine(a: Node, b: Node) -> Node | None:
+    """resolve a sum of two associated terms: sparse + diagonal -> SpAdd (sparse values: the
+    diagonal folded into Ã, O(nnz)); dense + dense -> Add (element-wise, at their width)"""
+    if a.kind in "ASD" and b.kind in "ASD":
+        return Node("S", "SpAdd", (a, b), None, "+")
+    if a.kind == "X" and b.kind == "X" and a.width == b.width:
+        return Node("X", "Add", (a, b), a.width, "+")
+    return None
+
+
+def generate_sum(items: list) -> list[Node]:
+    """Algorithm 1 over an IR with sums: besides the adjacent-leaf candidates (rules above), a sum
+    factor ("+", P, Q) is either resolved (both terms associated, then combined) or distributed over
+    its right neighbour R: (P + Q) R -> P R + Q R.  Returns the de-duplicated forest."""
+    out: list[Node] = []
+    seen: set = set()
+
+    def resolved(x):
+        return isinstance(x, Node)
+
+    def terms(chain):  # every association of a term's chain
+        if len(chain) == 1 and resolved(chain[0]):
+            return [chain[0]]
+        return generate_sum(chain)
+
+    def rec(seq):
+        if len(seq) == 1 and resolved(seq[0]):
+            key = seq[0].show()
+            if key not in seen:
+                seen.add(key)
+                out.append(seq[0])
+            return
+        for i, x in enumerate(seq):
+            if resolved(x):
+                continue
+            _, P, Q = x
+            for a in terms(P):           # resolve the sum
+                for b in terms(Q):
+                    n = _combine(a, b)
+                    if n is not None:
+                        rec(seq[:i] + [n] + seq[i + 1:])
+            if i + 1 < len(seq):         # distribute it over its right neighbour
+                rec(seq[:i] + [("+", P + [seq[i + 1]], Q + [seq[i + 1]])] + seq[i + 2:])
+        plain = [j for j in range(len(seq) - 1) if resolved(seq[j]) and resolved(seq[j + 1])]
+        for j in plain:
+            for (k0, k, node) in _candidates(seq[j:j + 2]):
+                rec(seq[:j] + [node] + seq[j + 2:])
+
+    rec(list(items))
+    return out
+
+
 def composition_id(t: Node) -> int:
     """map a promoted tree to the library's composition id (include/granii.h)"""
     s = t.show()
@@ -214,6 +309,8 @@ def composition_id(t: Node) -> int:
         "((SDDMM(DAD) H) W)": GCN_PRE_AGG, "(SDDMM(DAD) (H W))": GCN_PRE_UPD,
         "((D (A (D H))) W)": GCN_DYN_AGG, "(D (A (D (H W))))": GCN_DYN_UPD,
         "(α (H W))": GAT_REUSE, "((α H) W)": GAT_RECOMP,
+        "(((A + E) H) W)": GIN_PRE_AGG, "((A + E) (H W))": GIN_PRE_UPD,
+        "(((A H) + (E H)) W)": GIN_DYN_AGG, "((A (H W)) + (E (H W)))": GIN_DYN_UPD,
     }
     return table[s]
 
@@ -225,22 +322,30 @@ def evaluate(t: Node, env: dict):
         return env["D"] @ env["A"] @ env["D"]
     if not t.kids:
         return env[t.name]
+    if t.prim in ("SpAdd", "Add"):
+        return evaluate(t.kids[0], env) + evaluate(t.kids[1], env)
     v = evaluate(t.kids[0], env)
     for k in t.kids[1:]:
         v = v @ evaluate(k, env)
     return v
 
 
+def forest(model: str) -> list[Node]:
+    if model == "gin":
+        return generate_sum(gin_expr())
+    return generate(gcn_chain() if model == "gcn" else gat_chain())
+
+
 def promoted_compositions(model: str) -> dict[int, set]:
-    """{composition id: scenarios in which it is promoted} for 'gcn' or 'gat'"""
-    chain = gcn_chain() if model == "gcn" else gat_chain()
-    res = prune(generate(chain), attention=model == "gat")
+    """{composition id: scenarios in which it is promoted} for 'gcn', 'gat' or 'gin' (GIN's
+    scenarios compare K1 with the MLP's hidden width Kh, the width its aggregation runs at)"""
+    res = prune(forest(model), attention=model == "gat")
     return {composition_id(t): sc for t, sc in res.promoted}
 
 
 if __name__ == "__main__":
-    for m, ch in (("GCN", gcn_chain()), ("GAT", gat_chain())):
-        r = prune(generate(ch), attention=m == "GAT")
+    for m in ("GCN", "GAT", "GIN"):
+        r = prune(forest(m.lower()), attention=m == "GAT")
         print(f"{m}: {len(r.generated)} generated, {len(r.pruned)} pruned, {len(r.promoted)} promoted")
         for t, sc in r.promoted:
             print("  promoted", t.show(), sorted(sc), "->", composition_id(t))

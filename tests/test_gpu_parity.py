@@ -788,8 +788,10 @@ def test_select_candidates_are_the_offline_promoted_trees(G):
     the offline stage (offline.py, Algorithm 1 + pruning) promotes for each scenario"""
     from paper_conf_cgo_lenadorasgytm26_b200 import offline as OF
     c = case(G, "pubmed")
-    for model, name in ((G.GCN, "gcn"), (G.GAT, "gat")):
+    for model, name in ((G.GCN, "gcn"), (G.GAT, "gat"), (G.GIN, "gin")):
         prom = OF.promoted_compositions(name)
         for K1, K2, scen in ((256, 32, ">="), (64, 64, ">="), (32, 256, "<")):
-            _, pred = G.granii_select(c.g, model, K1, K2)
+            # GIN aggregates at K1 or Kh: its scenario compares K1 with the hidden width
+            shape = G.shape_args(K1, 16, Kh=K2) if model == G.GIN else G.shape_args(K1, K2)
+            _, pred = G.granii_select_ex(c.g, model, shape)
             assert set(pred) == {cid for cid, sc in prom.items() if scen in sc}, (name, K1, K2)

@@ -60,8 +60,34 @@ def test_gat_counts_and_both_promoted():
     res = OF.prune(OF.generate(OF.gat_chain()), attention=True)
     assert (len(res.generated), len(res.pruned), len(res.promoted)) == (2, 0, 2)   # L326
     p = OF.promoted_compositions("gat")
-    assert p == {OF.GAT_REUSE: {"<", ">="}, OF.GAT_RECOMP: {"<", ">="}}
+    # RECOMP does all of REUSE's work on never-smaller matrices plus a GEMM when K1 >= K2 (rule 1):
+    # profitable only for growing sizes (L330, L357)
+    assert p == {OF.GAT_REUSE: {"<", ">="}, OF.GAT_RECOMP: {"<"}}
     # RECOMP pays the extra GEMM of L135
     reuse = [t for t in res.generated if OF.composition_id(t) == OF.GAT_REUSE][0]
     recomp = [t for t in res.generated if OF.composition_id(t) == OF.GAT_RECOMP][0]
     assert OF.primitives(recomp, True)[("GEMM", "K1K2")] == OF.primitives(reuse, True)[("GEMM", "K1K2")] + 1
+
+
+def test_gin_forest_pruning_and_promoted_compositions():
+    """GIN (reading R23): (Ã + εI) H W1 with a sum in the IR.  The distributive rewrite gives 7
+    distinct trees (the paper counts 8 generated, L326), pruning keeps 4 -- the paper's promoted
+    count (8 - 4) -- which are exactly the library's GIN compositions, aggregate-first when K1 < Kh"""
+    trees = OF.forest("gin")
+    res = OF.prune(trees)
+    assert (len(res.generated), len(res.pruned), len(res.promoted)) == (7, 3, 4)
+    assert OF.promoted_compositions("gin") == {OF.GIN_PRE_AGG: {"<"}, OF.GIN_DYN_AGG: {"<"},
+                                                OF.GIN_PRE_UPD: {">="}, OF.GIN_DYN_UPD: {">="}}
+    rng = np.random.default_rng(1)
+    n, k1, kh = 6, 4, 5
+    A = (rng.random((n, n)) < 0.5).astype(float) + np.eye(n)
+    env = {"A": A, "E": 0.3 * np.eye(n), "H": rng.standard_normal((n, k1)), "W": rng.standard_normal((k1, kh))}
+    ref = (A + env["E"]) @ env["H"] @ env["W"]
+    for t in trees:      # every re-association computes the same matrix (L192)
+        assert np.allclose(OF.evaluate(t, env), ref, rtol=1e-12, atol=1e-12), t.show()
+
+
+def test_cse_counts_a_shared_subtree_once():
+    """L219: A (H W) + E (H W) computes H W once"""
+    dyn_upd = [x for x in OF.forest("gin") if x.show() == "((A (H W)) + (E (H W)))"][0]
+    assert OF.primitives(dyn_upd)[("GEMM", "K1K2")] == 1
