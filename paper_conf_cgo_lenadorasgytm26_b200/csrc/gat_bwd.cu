@@ -706,12 +706,14 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
 // partial[s][2][K] = Σ_{r in chunk s} H[r, :] * (d0[r], d1[r]); block (32, 8), fixed order
 __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, int64_t ldh,
                              const float* __restrict__ d0, const float* __restrict__ d1, int64_t chunk,
-                             float* __restrict__ partial) {
-  __shared__ float sp[8][33], sq[8][33];
+                             double* __restrict__ partial) {
+  // fp64 accumulation: da = Hᵀ del sums millions of products of both signs (the softmax backward's
+  // del is centred), and an fp32 running sum loses the result's low bits to the cancellation
+  __shared__ double sp[8][33], sq[8][33];
   const int tx = threadIdx.x, ty = threadIdx.y;
   const int64_t col = blockIdx.x * 32 + tx, s = blockIdx.y;
   const int64_t r0 = s * chunk, r1 = (r0 + chunk < R) ? r0 + chunk : R;
-  float p = 0.f, q = 0.f;
+  double p = 0.0, q = 0.0;
   if (col < K) {
     int64_t r = r0 + ty;
     for (; r + 24 < r1; r += 32) {  // four rows in flight per thread, summed in row order
@@ -724,21 +726,21 @@ __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, 
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        p = fmaf(h[u], a0[u], p);
-        q = fmaf(h[u], a1[u], q);
+        p = fma((double)h[u], (double)a0[u], p);
+        q = fma((double)h[u], (double)a1[u], q);
       }
     }
     for (; r < r1; r += 8) {
-      const float h = H[r * ldh + col];
-      p = fmaf(h, __ldg(d0 + r), p);
-      q = fmaf(h, __ldg(d1 + r), q);
+      const double h = H[r * ldh + col];
+      p = fma(h, (double)__ldg(d0 + r), p);
+      q = fma(h, (double)__ldg(d1 + r), q);
     }
   }
   sp[ty][tx] = p;
   sq[ty][tx] = q;
   __syncthreads();
   if (ty == 0 && col < K) {
-    float a = 0.f, c = 0.f;
+    double a = 0.0, c = 0.0;
 #pragma unroll
     for (int y = 0; y < 8; ++y) {
       a += sp[y][tx];
@@ -749,12 +751,12 @@ __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, 
   }
 }
 
-__global__ void k_sum_chunks(int64_t n, int64_t S, const float* __restrict__ partial, float* __restrict__ out) {
+__global__ void k_sum_chunks(int64_t n, int64_t S, const double* __restrict__ partial, float* __restrict__ out) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= n) return;
-  float a = 0.f;
+  double a = 0.0;
   for (int64_t s = 0; s < S; ++s) a += partial[s * n + i];
-  out[i] = a;
+  out[i] = (float)a;
 }
 
 static int64_t colreduce_chunks(int64_t R, int64_t K) {
@@ -762,15 +764,15 @@ static int64_t colreduce_chunks(int64_t R, int64_t K) {
   return std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 512), ceil_div(148 * 8, tiles)));
 }
 
-size_t colreduce2_workspace(int64_t R, int64_t K) { return (size_t)colreduce_chunks(R, K) * 2 * K * sizeof(float); }
+size_t colreduce2_workspace(int64_t R, int64_t K) { return (size_t)colreduce_chunks(R, K) * 2 * K * sizeof(double); }
 
 granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ldh, const float* d0, const float* d1,
                                 float* partial, float* out, cudaStream_t st) {
   const int64_t S = colreduce_chunks(R, K), chunk = ceil_div(std::max<int64_t>(R, 1), S);
   ProfScope ps("elementwise", st, 4.0 * R * K + 8.0 * R, 4.0 * R * K, 2);
   k_colreduce2<<<dim3((unsigned)ceil_div(K, 32), (unsigned)S), dim3(32, 8), 0, st>>>(R, K, H, ldh, d0, d1, chunk,
-                                                                                   partial);
-  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, partial, out);
+                                                                                   reinterpret_cast<double*>(partial));
+  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, reinterpret_cast<const double*>(partial), out);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

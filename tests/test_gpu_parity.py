@@ -499,12 +499,14 @@ def gat_grad_ok(y, r, m):
     """R22: per row, |y - r|∞ <= 1e-4 |r|∞ + 4u |m|∞ (u = 2^-24, m = the computation's magnitude):
     the softmax backward α(dα - Σα dα) cancels by construction on near-one-hot rows, and a fp32
     path cannot resolve the difference below u·|dα|; elsewhere m ~ |r| and this is R19's 1e-4.
-    The worst-case bound grows linearly with the number of cancelling rows, so a 1e-3 normwise
-    guard is kept for the strongly cancelling aggregates (da = Θᵀ del over all rows)"""
+    The worst-case bound grows linearly with the number of cancelling rows, so a 3e-4 normwise
+    guard is kept for the strongly cancelling aggregates (da = Wᵀ Hᵀ del over all rows; the column
+    reduction is fp64, the residue is del's own cancellation: worst measured 1.4e-4 for RECOMP
+    256->1024, everything else <= 7e-5, tools/gat_grad_err.py)"""
     y, r, m = (np.atleast_2d(np.asarray(x, np.float64)) for x in (y, r, m))
     d = np.abs(y - r).max(1)
     ok = d <= TOL * np.abs(r).max(1) + 4 * 2.0 ** -24 * m.max(1)
-    assert normwise(y, r) <= 10 * TOL
+    assert normwise(y, r) <= 3 * TOL
     return bool(ok.all())
 
 
