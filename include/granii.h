@@ -339,7 +339,8 @@ granii_status granii_select_ex(granii_graph g, granii_model m, const granii_laye
 /* Calibration support: the feature vector the cost model of primitive `prim`
  * (0 spmm weighted, 1 spmm unweighted, 2 spmm unweighted + column scale,
  * 3 sddmm K=1, 4 sddmm K=1 + softmax, 5 gemm, 6 gemm without store, 7 gemm Aᵀ·B,
- * 8 elementwise, 9 all-gather, 10 gemm with the GAT attention GEMVs, 11 / 12 GAT backward passes A / B)
+ * 8 elementwise, 9 all-gather, 10 gemm with the GAT attention GEMVs, 11 / 12 GAT backward passes A / B,
+ * 13 the der-only pass of a RECOMP input layer's backward)
  * uses for this graph and widths (K1, K2);
  * feats has room for 8 values; model_name (32 bytes) receives the model key
  * the coefficients are stored under in the calibration file. */

@@ -497,6 +497,7 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
 void graph_free(granii_graph_s* g) {
   if (!g) return;
   graph_free(g->T);
+  cudaFree(g->tperm);
   cudaFree(g->owner_off);
   cudaFree(g->ord_off);
   cudaFree(g->dinv2_rows);
@@ -512,6 +513,46 @@ void graph_free(granii_graph_s* g) {
   cudaFree(g->seg_heavy);
   cudaFree(g->seg_row);
   delete g;
+}
+
+// ---------------------------------------------------------------- Ãᵀ -> Ã entry map
+// Ã's entries are ordered by (row i, column j); a stable sort of their positions by column gives them
+// in (column j, row i) order -- exactly the CSR order of Ãᵀ (row j, columns i ascending), which is the
+// order of the kept transpose T of a directed graph and of Ã itself when symmetric.
+granii_status ensure_tperm(const granii_graph_s* gc, cudaStream_t st) {
+  granii_graph_s* g = const_cast<granii_graph_s*>(gc);
+  if (g->tperm) return GRANII_OK;
+  if (g->world > 1) return fail(GRANII_ERR_UNSUPPORTED, "transpose entry map: single-GPU graphs only");
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  GR_CUDA(cudaStreamIsCapturing(st, &cs));
+  if (cs != cudaStreamCaptureStatusNone) return fail(GRANII_ERR_UNSUPPORTED, "transpose entry map: stream capturing");
+  const int64_t n = g->local_nnz;
+  if (n > INT32_MAX) return fail(GRANII_ERR_UNSUPPORTED, "transpose entry map: more than 2^31 entries");
+  int bits = 1;
+  while (bits < 31 && (int64_t(1) << bits) < g->n_cols) ++bits;
+  int32_t *perm = nullptr, *iota = nullptr, *keys = nullptr;
+  void* tmp = nullptr;
+  size_t tb = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, tb, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
+                                  (int32_t*)nullptr, (int)n, 0, bits, st);
+  GR_CUDA(cudaMalloc(&perm, std::max<int64_t>(n, 1) * sizeof(int32_t)));
+  cudaError_t e = cudaMallocAsync(&iota, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&keys, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&tmp, std::max<size_t>(tb, 16), st);
+  if (e == cudaSuccess && n > 0) {
+    k_iota<<<grid_for(n), 256, 0, st>>>(n, iota);
+    e = cub::DeviceRadixSort::SortPairs(tmp, tb, g->col_idx, keys, iota, perm, (int)n, 0, bits, st);
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  cudaFreeAsync(tmp, st);
+  cudaFreeAsync(keys, st);
+  cudaFreeAsync(iota, st);
+  if (e != cudaSuccess) {
+    cudaFree(perm);
+    return fail(GRANII_ERR_CUDA, std::string("transpose entry map: ") + cudaGetErrorString(e));
+  }
+  g->tperm = perm;
+  return GRANII_OK;
 }
 
 }  // namespace granii

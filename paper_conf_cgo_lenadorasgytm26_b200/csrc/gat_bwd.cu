@@ -29,6 +29,7 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include "cache.cuh"
 #include "internal.h"
 
 namespace granii {
@@ -149,7 +150,10 @@ __global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int K, int Kv, int 
 // per-column scalars with one coalesced load (the next chunk is prefetched while this one is
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
-template <int LPG, int NJ, int U, bool CL = false>
+// WT (the der-only path, a.tout): each entry's dα is reduced over its lane group and written in Ã's
+// order, and D accumulates w·s'·(dα - c_i) per entry (the subtraction before the weighting: no
+// D - c·Cw cancellation at the end, Cw is left 0)
+template <int LPG, int NJ, int U, bool CL = false, bool WT = false>
 __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
   static_assert(G * U <= 32, "one step must fit in a chunk");
@@ -211,10 +215,25 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
       float zv[U][NJ][4];
 #pragma unroll
       for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      if constexpr (WT) {
 #pragma unroll
-      for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot<NJ>(xv, zv[u]), D);
+        for (int u = 0; u < U; ++u) {
+          float pd = gb_pdot<NJ>(xv, zv[u]);
+#pragma unroll
+          for (int o = LPG / 2; o; o >>= 1) pd += __shfl_xor_sync(0xffffffffu, pd, o);
+          const int slot = q * G * U + u * G + grp;
+          if (lg == 0 && slot < cnt) {
+            D = fmaf(wu[u], pd - ci, D);
+            a.tout[base + slot] = pd;
+          }
+        }
+      } else {
+#pragma unroll
+        for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot<NJ>(xv, zv[u]), D);
+      }
     }
   }
+  if constexpr (WT) Cw = 0.f;
   S = gb_warp_sum(S);
   Cw = gb_warp_sum(Cw);
   D = gb_warp_sum(D);
@@ -226,6 +245,7 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
   if (lane == 0) {
     a.del[r] = (D - ci * Cw) * inv_s;
     *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(eli, m, inv_s, ci);
+    if (WT) a.recs[r] = make_float4(eli, m, inv_s, ci);
   }
 }
 
@@ -340,9 +360,12 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
 // avg degree < 16 (the SpMM's group-per-row regime): an LPG-lane group owns a row, 32/LPG rows
 // per warp, U entries per group in flight; no shuffles inside the (divergent) entry loops, the
 // lane shares are reduced within the group at the end.
-template <int LPG, int NJ, int U>
+template <int LPG, int NJ, int U, bool WT = false>
 __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0, int lane) {
   const int lg = lane % LPG;
+  // the group's lanes run the same (divergent across groups) entry loop: WT's per-entry reduction
+  // shuffles within the group only
+  const unsigned gmask = LPG == 32 ? 0xffffffffu : (((1u << LPG) - 1u) << (lane & ~(LPG - 1)));
   const bool live = t0 < a.n_rows;
   const int32_t r = live ? a.order[t0] : 0;
   const int64_t b = live ? a.row_ptr[r] : 0, t = live ? a.row_ptr[r + 1] : 0;
@@ -363,7 +386,13 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (e + u < t) {
-        const float pd = gb_pdot<NJ>(xv, zv[u]);
+        float pd = gb_pdot<NJ>(xv, zv[u]);
+        if constexpr (WT) {
+#pragma unroll
+          for (int o = LPG / 2; o; o >>= 1) pd += __shfl_xor_sync(gmask, pd, o);
+          if (lg == 0) a.tout[e + u] = pd;
+          pd -= ci;  // every lane holds the entry's whole dα - c_i: D is not a lane share
+        }
         const float z = eli + erj[u];
         const float ev = gb_lrelu(z);
         const float sl = z > 0.f ? 1.f : 0.2f;
@@ -382,12 +411,17 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
       }
     }
   }
+  if constexpr (WT) {
+    Cw = 0.f;
+  } else {
 #pragma unroll
-  for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);
+    for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);
+  }
   const float inv_s = S > 0.f ? 1.f / S : 0.f;
   if (live && lg == 0) {
     a.del[r] = (D - ci * Cw) * inv_s;
     *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(eli, m, inv_s, ci);
+    if (WT) a.recs[r] = make_float4(eli, m, inv_s, ci);
   }
 }
 
@@ -460,7 +494,7 @@ __device__ __forceinline__ void gat_b_group_row(const GatBwdArgs& a, int64_t t0,
 
 // One launch covers both schedules: warps [0, n_wide) take the wide rows order[0 .. n_wide)
 // (all rows of a dense graph), the remaining warps take G rows each, one per lane group.
-template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
+template <int LPG, int NJ, int U, int MINB = 0, bool CL = false, bool WT = false>
 __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 4 : (NJ <= 4 ? 3 : (NJ <= 8 ? 2 : 1))))
     k_gat_bwd_a(GatBwdArgs a) {
   constexpr int G = 32 / LPG;
@@ -470,11 +504,11 @@ __global__ void __launch_bounds__(256, MINB > 0 ? MINB : (NJ <= 2 ? 4 : (NJ <= 4
   // then lane groups; one call site per schedule keeps the unrolled body inlined once
   const int64_t wr = w - a.n_seg;
   if (wr >= a.n_wide) {
-    gat_a_group_row<LPG, NJ, U>(a, a.n_wide + (wr - a.n_wide) * G + lane / LPG, lane);
+    gat_a_group_row<LPG, NJ, U, WT>(a, a.n_wide + (wr - a.n_wide) * G + lane / LPG, lane);
     return;
   }
   const bool sg = w < a.n_seg;
-  gat_a_warp_row<LPG, NJ, U, CL>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
+  gat_a_warp_row<LPG, NJ, U, CL, WT>(a, sg ? a.seg_row[w] : a.order[wr], lane, sg ? w : -1);
 }
 
 template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
@@ -510,6 +544,7 @@ __global__ void k_gat_a_combine(GatBwdArgs a) {
     const float ci = a.c[r], inv_s = S > 0.f ? 1.f / S : 0.f;
     a.del[r] = (D - ci * Cw) * inv_s;
     *reinterpret_cast<float4*>(a.dXw + (int64_t)r * a.ldx + a.rec) = make_float4(a.el[r], m, inv_s, ci);
+    if (a.recs) a.recs[r] = make_float4(a.el[r], m, inv_s, ci);
   }
 }
 
@@ -529,12 +564,209 @@ __global__ void k_gat_b_combine(GatBwdArgs a) {
   }
 }
 
+// ---------------------------------------------------------------- der only (RECOMP input layer)
+// der_j = Σ_{i: j ∈ N(i)} dz_ij, dz_ij = α_ij (dα_ij - c_i) s'_ij -- the column sums of dz, which an
+// input layer needs instead of pass B's K-wide transposed SpMM (that only feeds dH).  Two streaming
+// passes instead of K-wide gathers:
+//   k_gat_dz  (rows i of Ã, schedule order): dz_ij from pass A's per-entry dα (tv, Ã order, in place),
+//             row i's record {el_i, m_i, 1/s_i, c_i} and a gathered er_j (L2-resident vector);
+//   k_gat_der (rows j of Ãᵀ, NATURAL order): der_j = Σ tv[tperm[e]] over Ãᵀ's row j.  The dz reads are
+//             4-byte gathers from a 4·nnz-byte array, but rows j processed together in natural order
+//             read neighbouring entries of every row i (its columns j are sorted), so each 32-byte
+//             sector of dz is fetched once and used by ~8 rows j while it stays in L2 (evict_last);
+//             the schedule's degree order would scatter them.  Hub rows (degree > seg_len, when the
+//             graph has segments) are taken as warp-wide segments first, their partials merged per
+//             row in fixed order.
+// Every sum in a fixed order (bitwise reproducible), no atomics.
+struct GatDzArgs {
+  int64_t n_rows;              // light rows (order[n_heavy ..])
+  const int32_t* order;
+  const longlong2* ord_rp;
+  const int32_t* col;
+  const float* er;
+  const float4* recs;
+  float* tv;
+  int l2hint;
+  int64_t n_seg;               // hub rows: warp-wide segments (dz is per entry: no merge needed)
+  const int64_t* seg_lo;
+  const int64_t* seg_hi;
+  const int32_t* seg_row;
+};
+
+template <int U>
+__device__ __forceinline__ void gat_dz_run(const GatDzArgs& a, int32_t i, int64_t e, int64_t re, int step,
+                                           const L2Pol& pol) {
+  const float4 rc = __ldg(a.recs + i);  // {el_i, m_i, 1/s_i, c_i}
+  for (; e < re; e += (int64_t)U * step) {
+    int32_t j[U];
+    float d[U], erj[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t ee = e + (int64_t)u * step < re ? e + (int64_t)u * step : re - 1;
+      j[u] = ldg_stream(a.col + ee, pol.stream);
+      d[u] = ldg_stream(a.tv + ee, pol.stream);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) erj[u] = ldg_pol(a.er + j[u], pol.keep);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t ee = e + (int64_t)u * step;
+      if (ee < re) {
+        const float z = rc.x + erj[u];
+        const float al = __expf(gb_lrelu(z) - rc.y) * rc.z;
+        st_pol(a.tv + ee, al * (z > 0.f ? 1.f : 0.2f) * (d[u] - rc.w), pol.stream);
+      }
+    }
+  }
+}
+
+template <int LPG, int U>
+__global__ void __launch_bounds__(256) k_gat_dz(GatDzArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const L2Pol pol = make_l2pol(a.l2hint);
+  for (int64_t t = warp; t < a.n_seg; t += nwarps)
+    gat_dz_run<U>(a, a.seg_row[t], a.seg_lo[t] + lane, a.seg_hi[t], 32, pol);
+  for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
+    const int64_t t = t0 + grp;
+    if (t >= a.n_rows) continue;
+    const longlong2 rr = a.ord_rp[t];
+    gat_dz_run<U>(a, a.order[t], rr.x + lig, rr.y, LPG, pol);
+  }
+}
+
+struct GatDerArgs {
+  int64_t n_rows;              // every row j of Ãᵀ, natural order (hub rows skipped when segmented)
+  const int64_t* row_ptr;
+  int64_t seg_len;             // rows longer than this are hub segments (n_seg > 0)
+  const int32_t* tperm;
+  const float* tv;             // dz in Ã order
+  float* der;
+  int64_t n_seg;
+  const int64_t* seg_lo;
+  const int64_t* seg_hi;
+  float* seg_der;
+  int l2hint;
+};
+
+template <int U>
+__device__ __forceinline__ float gat_dz_sum(const GatDerArgs& a, int64_t e, int64_t re, int step, const L2Pol& pol) {
+  float acc = 0.f;
+  for (; e < re; e += (int64_t)U * step) {
+    int32_t p[U];
+    float v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t ee = e + (int64_t)u * step < re ? e + (int64_t)u * step : re - 1;
+      p[u] = ldg_stream(a.tperm + ee, pol.stream);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) v[u] = ldg_pol(a.tv + p[u], pol.keep);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (e + (int64_t)u * step < re) acc += v[u];
+  }
+  return acc;
+}
+
+template <int LPG, int U>
+__global__ void __launch_bounds__(256) k_gat_der(GatDerArgs a) {
+  constexpr int G = 32 / LPG;
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const L2Pol pol = make_l2pol(a.l2hint);
+  for (int64_t t = warp; t < a.n_seg; t += nwarps) {
+    const float acc = gb_warp_sum(gat_dz_sum<U>(a, a.seg_lo[t] + lane, a.seg_hi[t], 32, pol));
+    if (lane == 0) a.seg_der[t] = acc;
+  }
+  for (int64_t j0 = warp * G; j0 < a.n_rows; j0 += nwarps * G) {
+    const int64_t j = j0 + grp;
+    int64_t rs = 0, re = 0;
+    if (j < a.n_rows) {
+      rs = a.row_ptr[j];
+      re = a.row_ptr[j + 1];
+      if (a.n_seg > 0 && re - rs > a.seg_len) re = rs;  // a hub: its segments were summed above
+    }
+    float acc = gat_dz_sum<U>(a, rs + lig, re, LPG, pol);
+#pragma unroll
+    for (int o = LPG / 2; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (j < a.n_rows && lig == 0 && !(a.n_seg > 0 && a.row_ptr[j + 1] - rs > a.seg_len)) a.der[j] = acc;
+  }
+}
+
+__global__ void k_gat_der_combine(int64_t n_heavy, const int32_t* __restrict__ heavy_rows,
+                                  const int32_t* __restrict__ seg_ptr, const float* __restrict__ seg_der,
+                                  float* __restrict__ der) {
+  for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_heavy; h += (int64_t)gridDim.x * blockDim.x) {
+    float acc = 0.f;
+    for (int32_t q = seg_ptr[h]; q < seg_ptr[h + 1]; ++q) acc += seg_der[q];
+    der[heavy_rows[h]] = acc;
+  }
+}
+
+static int der_lpg(float avg) { return avg >= 96.f ? 32 : avg >= 24.f ? 16 : avg >= 6.f ? 8 : 4; }
+
+granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, const float* er, float* tv,
+                             const float4* recs, float* der, cudaStream_t st) {
+  if (g->n_rows == 0) return GRANII_OK;
+  if (!g->tperm) return fail(GRANII_ERR_INVALID_ARG, "der-only GAT backward without the transpose entry map");
+  DevInfo di;
+  GR_TRY(dev_info(&di));
+  const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
+  const int hint = l2hint_enabled();
+  {
+    // algorithmic bytes: per entry col + dα in + er + dz out; per row schedule entry + record
+    ProfScope ps("gat_dz", st, nnz * 16.0 + R * 36.0, 0.0, 1, -1.0, false);
+    GatDzArgs a{g->n_rows - g->n_heavy, g->order + g->n_heavy, g->ord_rp + g->n_heavy, g->col_idx, er, recs, tv, hint,
+                g->n_seg, g->seg_lo, g->seg_hi, g->seg_row};
+    const int lpg = der_lpg(g->avg_deg());
+    const int64_t want = ceil_div(ceil_div(a.n_rows, 32 / lpg) + a.n_seg, 8);
+#define GO(L) k_gat_dz<L, 4><<<(unsigned)persistent_grid(k_gat_dz<L, 4>, 256, di.sms, want), 256, 0, st>>>(a)
+    switch (lpg) {
+      case 32: GO(32); break;
+      case 16: GO(16); break;
+      case 8: GO(8); break;
+      default: GO(4); break;
+    }
+#undef GO
+    GR_CHECK_LAUNCH();
+  }
+  // algorithmic bytes: per entry map + dz (a 4-byte gather); per row 8 B row_ptr + der
+  ProfScope ps("gat_der", st, (double)gt->local_nnz * 8.0 + (double)gt->n_rows * 12.0, 0.0, gt->n_seg > 0 ? 2 : 1,
+               -1.0, false);
+  GatDerArgs b{gt->n_rows, gt->row_ptr, gt->seg_len, g->tperm, tv, der, gt->n_seg, gt->seg_lo, gt->seg_hi, nullptr,
+               hint};
+  if (gt->n_seg > 0) GR_CUDA(cudaMallocAsync((void**)&b.seg_der, gt->n_seg * sizeof(float), st));
+  const int lpg = der_lpg(gt->avg_deg());
+  const int64_t want = ceil_div(ceil_div(b.n_rows, 32 / lpg) + b.n_seg, 8);
+#define GO(L) k_gat_der<L, 4><<<(unsigned)persistent_grid(k_gat_der<L, 4>, 256, di.sms, want), 256, 0, st>>>(b)
+  switch (lpg) {
+    case 32: GO(32); break;
+    case 16: GO(16); break;
+    case 8: GO(8); break;
+    default: GO(4); break;
+  }
+#undef GO
+  if (gt->n_seg > 0) {
+    k_gat_der_combine<<<(unsigned)ceil_div(gt->n_heavy, 128), 128, 0, st>>>(gt->n_heavy, gt->order, gt->seg_ptr,
+                                                                             b.seg_der, der);
+    GR_CUDA(cudaFreeAsync(b.seg_der, st));
+  }
+  GR_CHECK_LAUNCH();
+  return GRANII_OK;
+}
+
 template <int LPG, int NJ, int U, int MINB = 0, bool CL = false>
 static void gb_launch(int pass, const GatBwdArgs& a, cudaStream_t st) {
   constexpr int G = 32 / LPG;
   const int64_t warps = a.n_seg + a.n_wide + ceil_div(a.n_rows - a.n_wide, G);
   const unsigned blocks = (unsigned)std::max<int64_t>(1, ceil_div(warps, 8));
-  if (pass == 0)
+  if (pass == 0 && a.tout)
+    k_gat_bwd_a<LPG, NJ, U, MINB, CL, true><<<blocks, 256, 0, st>>>(a);
+  else if (pass == 0)
     k_gat_bwd_a<LPG, NJ, U, MINB, CL><<<blocks, 256, 0, st>>>(a);
   else
     k_gat_bwd_b<LPG, NJ, U, MINB, CL><<<blocks, 256, 0, st>>>(a);

@@ -462,7 +462,14 @@ struct TnCfg {
   static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
   static constexpr int STAGES_FIT = 200 * 1024 / STAGE;
   static constexpr int STAGES = STAGES_FIT > 6 ? 6 : STAGES_FIT;
-  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int ACC_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  // The tcgen05 fp32 accumulation loses about one ulp of the accumulator per MMA, in one direction
+  // (tools/gemm_tn_err.py: the error grows linearly with the k-blocks summed into one accumulator,
+  // 1.05e-5 relative after 512 rows of positive products).  A split's k-blocks are therefore spread
+  // over NACC accumulators filling the 512 TMEM columns (one CTA per SM), consecutive sub-ranges,
+  // summed by the epilogue in fixed order with round-to-nearest CUDA-core adds.
+  static constexpr int NACC = 512 / ACC_COLS;
+  static constexpr int TMEM_COLS = 512;
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
 };
 
@@ -536,14 +543,18 @@ __global__ void __launch_bounds__(64 + 32 * NCW, 1)
         tc_fence_after();
         const uint32_t ah = smem_u32(a_hi(s)), al = smem_u32(a_lo(s));
         const uint32_t bh = smem_u32(b_hi(s)), bl = smem_u32(b_lo(s));
+        // accumulator t takes the k-blocks [ceil(t nk / NACC), ceil((t+1) nk / NACC))
+        const int t = (int)((int64_t)kb * Cfg::NACC / nk);
+        const bool first = kb == 0 || (int)((int64_t)(kb - 1) * Cfg::NACC / nk) != t;
+        const uint32_t acc = tmem + (uint32_t)(t * Cfg::ACC_COLS);
 #pragma unroll
         for (int k = 0; k < BK / 8; ++k) {  // one 8-row k group (1 KB) per MMA
           const uint32_t off = k * (dkstep & 0xFFFF);
           const uint64_t dah = desc_sw128_mn(ah + off, dlbo, dsbo), dal = desc_sw128_mn(al + off, dlbo, dsbo);
           const uint64_t dbh = desc_sw128_mn(bh + off, dlbo, dsbo), dbl = desc_sw128_mn(bl + off, dlbo, dsbo);
-          mma_tf32(tmem, dah, dbh, idesc, (kb | k) ? 1u : 0u);
-          mma_tf32(tmem, dah, dbl, idesc, 1u);
-          mma_tf32(tmem, dal, dbh, idesc, 1u);
+          mma_tf32(acc, dah, dbh, idesc, (!first || k) ? 1u : 0u);
+          mma_tf32(acc, dah, dbl, idesc, 1u);
+          mma_tf32(acc, dal, dbh, idesc, 1u);
         }
         mma_commit(&empty[s]);
       }
@@ -606,10 +617,19 @@ __global__ void __launch_bounds__(64 + 32 * NCW, 1)
 #pragma unroll 1
     for (int c0 = half * CPW; c0 < (half + 1) * CPW; c0 += 16) {
       float v[16];
-      if (nk > 0) tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + c0, v);
-      else
 #pragma unroll
-        for (int j = 0; j < 16; ++j) v[j] = 0.f;
+      for (int j = 0; j < 16; ++j) v[j] = 0.f;
+#pragma unroll 1
+      for (int t = 0; t < Cfg::NACC; ++t) {
+        // accumulator t holds k-blocks iff its sub-range is non-empty (nk < NACC leaves some unused)
+        const int lo = (int)(((int64_t)t * nk + Cfg::NACC - 1) / Cfg::NACC);
+        const int hi = (int)(((int64_t)(t + 1) * nk + Cfg::NACC - 1) / Cfg::NACC);
+        if (lo >= hi) continue;
+        float w[16];
+        tmem_ld16(tmem + ((uint32_t)(quad * 32) << 16) + (uint32_t)(t * Cfg::ACC_COLS + c0), w);
+#pragma unroll
+        for (int j = 0; j < 16; ++j) v[j] += w[j];
+      }
       if (r < M) {
 #pragma unroll
         for (int j = 0; j < 16; ++j)
@@ -734,9 +754,9 @@ __global__ void __launch_bounds__(256) k_gemm_tn_part(int M, int N, int64_t R, i
 __global__ void k_sum_splits(int64_t MN, int splits, const float* __restrict__ part, float* __restrict__ C, int M, int N,
                              int64_t ldc) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < MN; i += (int64_t)gridDim.x * blockDim.x) {
-    float s = 0.f;
-    for (int t = 0; t < splits; ++t) s += part[(int64_t)t * MN + i];
-    C[(i / N) * ldc + (i % N)] = s;
+    double s = 0.0;  // hundreds of split partials at full size: the fixed-order sum in fp64
+    for (int t = 0; t < splits; ++t) s += (double)part[(int64_t)t * MN + i];
+    C[(i / N) * ldc + (i % N)] = (float)s;
   }
 }
 
@@ -805,6 +825,15 @@ static int tn_ncw() {
   const char* e = getenv("GRANII_TN_NCW");
   return e && atoi(e) == 4 ? 4 : 8;
 }
+// rows per split (GRANII_TN_SPLIT_ROWS, 0 = no cap): the error of the tensor-core accumulation grows
+// linearly with the number of k-blocks summed into one TMEM accumulator (tools/gemm_tn_err.py, B200:
+// normwise 5.8e-4 for Reddit-shaped 602 x 256 over 2.45 M rows with 82 k rows per split; 2.8e-5 with
+// 4096), so the split count follows the reduction length -- and the error stays bounded at any graph
+// size.  The splits are then rounded so that tiles x splits fills whole waves of 148 CTAs.
+static int64_t tn_split_rows() {
+  const char* e = getenv("GRANII_TN_SPLIT_ROWS");
+  return e ? atoll(e) : 4096;
+}
 static TnPlan tn_plan(int64_t M, int64_t N, int64_t R) {
   TnPlan p;
   p.bn = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
@@ -815,6 +844,12 @@ static TnPlan tn_plan(int64_t M, int64_t N, int64_t R) {
   p.total_kb = ceil_div(R, p.bk);
   int64_t splits = std::max<int64_t>(1, ceil_div(148, p.mt * p.nt));
   splits = std::max<int64_t>(1, std::min<int64_t>(splits, p.total_kb / (8 * TC_BK / p.bk)));
+  if (const int64_t cap = tn_split_rows()) {
+    const int64_t tiles = p.mt * p.nt;
+    splits = std::max<int64_t>(splits, ceil_div(R, std::max<int64_t>(cap, p.bk)));
+    const int64_t waves = ceil_div(tiles * splits, 148);
+    splits = std::max<int64_t>(splits, std::min<int64_t>(waves * 148 / tiles, p.total_kb));
+  }
   p.kb_per = ceil_div(p.total_kb, splits);
   p.splits = ceil_div(p.total_kb, p.kb_per);
   return p;

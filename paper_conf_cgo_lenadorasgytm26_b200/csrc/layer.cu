@@ -785,6 +785,15 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
       thg.all = thg.mine = const_cast<float*>(saved);
     }
   }
+  // der only (RECOMP input layer on one GPU, no dH wanted): pass B's transposed SpMM feeds only dH, so
+  // der comes from pass A's per-entry dα through Ãᵀ's entry map (launch_gat_der) instead; the map is
+  // built on first use (not while the stream is being captured: then pass B runs)
+  const bool der_only_ok = !reuse && !dH && !c.dist() && g->local_nnz > 0 && !(getenv("GRANII_GAT_DER_ONLY") &&
+                                                                            getenv("GRANII_GAT_DER_ONLY")[0] == '0');
+  bool der_only = false;
+  if (der_only_ok && run) der_only = ensure_tperm(g, st) == GRANII_OK;
+  float* tv = der_only_ok ? b.take((size_t)g->local_nnz) : nullptr;
+  float4* recs = der_only_ok ? reinterpret_cast<float4*>(b.take((size_t)Rr * 4)) : nullptr;
   float* bout = nullptr;  // pass B output
   int64_t ldbo = 0;
   if (reuse) {
@@ -793,7 +802,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   } else if (dH) {
     bout = dH;
     ldbo = lddh;
-  } else {
+  } else if (!der_only) {  // sizing (run == false) takes it too
     bout = b.take((size_t)Rr * ld4(K1));
     ldbo = ld4(K1);
   }
@@ -837,9 +846,14 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pa.dXw = reuse ? dyg.mine : dtg.mine;
     pa.rec = rec;
     pa.del = del;
+    if (der_only) {
+      pa.tout = tv;
+      pa.recs = recs;
+    }
     GR_TRY(launch_gat_bwd_pass(g, 0, pa, st));
     if (c.dist()) GR_TRY(allgather(c, reuse ? dyg : dtg));  // rows + records
-    if (!reuse) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
+    if (der_only) GR_TRY(launch_gat_der(g, gt, er_own, tv, recs, der, st));
+    if (!reuse && !der_only) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
     GatBwdArgs pb;
     pb.n_rows = R;
     pb.row_ptr = gt->row_ptr;
@@ -859,7 +873,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pb.out = bout;
     pb.ldo = ldbo;
     pb.vec_store = (ldbo % 4 == 0) && (((uintptr_t)bout & 15) == 0);
-    GR_TRY(launch_gat_bwd_pass(gt, 1, pb, st));
+    if (!der_only) GR_TRY(launch_gat_bwd_pass(gt, 1, pb, st));
     if (reuse) {
       GR_TRY(launch_gemm(K1, K2, R, H, ldh, bout, ldbo, dW, K2, nullptr, GRANII_GEMM_TRANS_A, gwW, gnW, st));
       if (dH)

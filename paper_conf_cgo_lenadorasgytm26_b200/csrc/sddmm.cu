@@ -44,6 +44,7 @@ struct SddmmArgs {
   const int64_t* __restrict__ seg_hi;
   const int32_t* __restrict__ seg_row;
   int l2hint;                              // cache.cuh: V kept in L2, col_idx / out streamed
+  int64_t cap;                             // softmax: scores staged per warp in shared memory (floats)
 };
 
 template <bool ADD, bool LRELU>
@@ -53,9 +54,87 @@ __device__ __forceinline__ float score1(float u, float v, float scale) {
   return e;
 }
 
+// warp-uniform (max, sum) butterfly of per-lane online softmax states
+__device__ __forceinline__ void ms_merge(float& m, float& s, float m2, float s2) {
+  const float mn = fmaxf(m, m2);
+  const float a1 = (m == -INFINITY) ? 0.f : s * __expf(m - mn);
+  const float a2 = (m2 == -INFINITY) ? 0.f : s2 * __expf(m2 - mn);
+  m = mn;
+  s = a1 + a2;
+}
+
+// Fused row softmax of one row by a whole warp (rows longer than one group step).  Up to a.cap
+// entries the scores are staged in this warp's slice of shared memory: one sweep of coalesced
+// column loads and UW independent V gathers per lane, the row max, exp in place with the row sum,
+// then alpha written once -- every lane touches only its own slots (k = lane + 32 j), so no
+// barrier.  Longer rows (cap < n <= seg_len) write their scores with an online (max, sum) per lane
+// and normalise them in a second, coalesced sweep.
+template <bool ADD, bool LRELU>
+__device__ __forceinline__ void sddmm1_softmax_warp(const SddmmArgs& a, int64_t t, int lane, float* buf,
+                                                    const L2Pol& pol) {
+  constexpr int UW = 8;
+  const int64_t row = a.order[t];
+  const longlong2 rr = a.ord_rp[t];
+  const int64_t rs = rr.x, n = rr.y - rr.x;
+  const float u = __ldg(a.U + row * a.ldu);
+  const bool staged = n <= a.cap;
+  float m = -INFINITY, s = 0.f;
+  for (int64_t k0 = 0; k0 < n; k0 += 32 * UW) {
+    int32_t c[UW];
+    float v[UW];
+#pragma unroll
+    for (int q = 0; q < UW; ++q) {
+      const int64_t k = k0 + 32 * q + lane;
+      c[q] = ldg_stream(a.col_idx + rs + (k < n ? k : n - 1), pol.stream);
+    }
+#pragma unroll
+    for (int q = 0; q < UW; ++q) v[q] = ldg_pol(a.V + (int64_t)c[q] * a.ldv, pol.keep);
+    float mn = m;
+#pragma unroll
+    for (int q = 0; q < UW; ++q) {
+      const int64_t k = k0 + 32 * q + lane;
+      v[q] = score1<ADD, LRELU>(u, v[q], a.scale);
+      if (k < n) {
+        if (staged) buf[k] = v[q];
+        else st_pol(a.out + rs + k, v[q], pol.stream);
+        mn = fmaxf(mn, v[q]);
+      } else {
+        v[q] = -INFINITY;
+      }
+    }
+    if (!staged && mn > -INFINITY) {  // online sum (streamed rows only)
+      s = (m == -INFINITY ? 0.f : s * __expf(m - mn));
+#pragma unroll
+      for (int q = 0; q < UW; ++q) s += __expf(v[q] - mn);
+    }
+    m = mn;
+  }
+  if (staged) {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+    for (int64_t k = lane; k < n; k += 32) {
+      const float x = __expf(buf[k] - m);
+      buf[k] = x;
+      s += x;
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+    const float inv = 1.f / s;
+    for (int64_t k = lane; k < n; k += 32) st_pol(a.out + rs + k, buf[k] * inv, pol.stream);
+    __syncwarp();  // the next row reuses the slice
+  } else {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1)
+      ms_merge(m, s, __shfl_xor_sync(0xffffffffu, m, off), __shfl_xor_sync(0xffffffffu, s, off));
+    const float inv = 1.f / s;
+    for (int64_t k = lane; k < n; k += 32) st_pol(a.out + rs + k, __expf(a.out[rs + k] - m) * inv, pol.stream);
+  }
+}
+
 // K == 1: group of LPG lanes per row
 template <int LPG, bool ADD, bool LRELU, bool SOFTMAX>
 __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
+  extern __shared__ float sm_buf[];  // softmax: a.cap floats per warp
   constexpr int G = 32 / LPG;
   const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -81,14 +160,24 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
       st_pol(a.out + e, score1<ADD, LRELU>(u, ldg_pol(a.V + (int64_t)c * a.ldv, pol.keep), a.scale), pol.stream);
     }
   }
+  constexpr int U4 = 4;
   for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
+    if constexpr (SOFTMAX) {
+      // the unit's first row is its longest (degree-descending schedule): if it exceeds one group
+      // step, the warp takes the unit's rows one at a time (warp-uniform branch)
+      const longlong2 r0 = a.ord_rp[t0];
+      if (r0.y - r0.x > U4 * LPG) {
+        float* buf = sm_buf + (threadIdx.x >> 5) * a.cap;
+        for (int q = 0; q < G && t0 + q < a.n_rows; ++q) sddmm1_softmax_warp<ADD, LRELU>(a, t0 + q, lane, buf, pol);
+        continue;
+      }
+    }
     const int64_t t = t0 + grp;
     const bool live = t < a.n_rows;
     const int64_t row = live ? a.order[t] : 0;
     const longlong2 rr = live ? a.ord_rp[t] : make_longlong2(0, 0);  // independent of order[t]
     const int64_t rs = rr.x, re = rr.y;
     const float u = live ? __ldg(a.U + row * a.ldu) : 0.f;
-    constexpr int U4 = 4;
     if constexpr (!SOFTMAX) {
       // scores only: 4 independent col -> V gathers in flight per lane
       int64_t e = rs + lig;
@@ -349,8 +438,10 @@ static void go1(const SddmmArgs& a, int blocks, int sms, cudaStream_t st) {
   // as others finish balance the tail (B200 products-shaped, scores + softmax per layer: 8 CTAs / SM
   // where 6 fit 1.21 ms, persistent 1.07, 2 waves 1.01, 3 waves 0.99; GRANII_SDDMM_WAVES overrides)
   const int wv = getenv("GRANII_SDDMM_WAVES") ? atoi(getenv("GRANII_SDDMM_WAVES")) : 3;
-  const int64_t b = persistent_grid(k_sddmm1<LPG, ADD, LR, SM>, 256, sms * std::max(wv, 1), blocks * std::max(wv, 1));
-  k_sddmm1<LPG, ADD, LR, SM><<<(unsigned)b, 256, 0, st>>>(a);
+  const size_t smem = SM ? (size_t)a.cap * 8 * sizeof(float) : 0;
+  const int64_t cap = (int64_t)sms * std::max(wv, 1) * resident_ctas((const void*)k_sddmm1<LPG, ADD, LR, SM>, 256, smem);
+  const int64_t b = std::max<int64_t>(1, std::min<int64_t>(cap, (int64_t)blocks * std::max(wv, 1)));
+  k_sddmm1<LPG, ADD, LR, SM><<<(unsigned)b, 256, smem, st>>>(a);
 }
 
 template <bool ADD, bool LR, bool SM>
@@ -372,7 +463,10 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   const bool lr = op & GRANII_SDDMM_LEAKYRELU, sm = op & GRANII_SDDMM_ROW_SOFTMAX;
   const int64_t n_light = g->n_rows - g->n_heavy;
   SddmmArgs a{n_light, g->row_ptr, g->col_idx, U, ldu, V, ldv, K, scale, out, g->order + g->n_heavy,
-              g->ord_rp + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, l2hint_enabled()};
+              g->ord_rp + g->n_heavy, g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, l2hint_enabled(), 0};
+  // fused softmax: rows longer than one group step are scored into shared memory (4 KB per warp,
+  // 32 KB per CTA), GRANII_SDDMM_CAP overrides (0: every long row streams through global memory)
+  a.cap = getenv("GRANII_SDDMM_CAP") ? atoi(getenv("GRANII_SDDMM_CAP")) : 1024;
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double gathered = (double)g->n_cols * 4.0 * (double)K;  // V, read once in the compulsory count

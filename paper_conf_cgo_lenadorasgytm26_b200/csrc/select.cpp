@@ -62,6 +62,8 @@ static CostModel defaults() {
   m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
   m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
+  // der only (RECOMP input layer): streamed column ids + entry map, one 32-byte sector per dα gather
+  m.coef["gat_der"] = {0.010, 1.0 / 6.0, 1.0 / 6.0, 0.0};
   // group-per-row graphs (average degree < 16) run other kernels (spmm.cu k_spmm_group, the
   // lane-group GAT backward passes): their own coefficients (B200 fit: SpMM median error
   // 13 % with one model for both schedules, 9 % / 7 % split)
@@ -148,7 +150,8 @@ static double l2_hit(const In& in, double K, double cols) {
 
 // primitive ids of the feature API
 enum { P_SPMM_W = 0, P_SPMM_U = 1, P_SPMM_U_CS = 2, P_SDDMM1 = 3, P_SDDMM1_SM = 4, P_GEMM = 5, P_GEMM_NOSTORE = 6,
-       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10, P_GAT_BWD_A = 11, P_GAT_BWD_B = 12 };
+       P_GEMM_TN = 7, P_ELEMENTWISE = 8, P_ALLGATHER = 9, P_GEMM_ATT = 10, P_GAT_BWD_A = 11, P_GAT_BWD_B = 12,
+       P_GAT_DER = 13 };
 
 // the warp-per-row / group-per-row split follows the kernels' own switch (spmm.cu, gat_bwd.cu)
 static bool group_mode(const In& in) { return in.avg < 16.0; }
@@ -165,6 +168,7 @@ static const char* prim_model(int p, const In& in) {
     case P_ALLGATHER: return "allgather";
     case P_GAT_BWD_A: return group_mode(in) ? "gat_bwd_a_g" : "gat_bwd_a";
     case P_GAT_BWD_B: return group_mode(in) ? "gat_bwd_b_g" : "gat_bwd_b";
+    case P_GAT_DER: return "gat_der";
   }
   return "";
 }
@@ -207,6 +211,7 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
       return {1.0, idx, in.R * K * (p == P_GAT_BWD_A ? 4.0 : 12.0) * gb, gath * h, gath * (1.0 - h), in.R * 1e-6,
               (in.nnz / gu + 0.5 * in.R) * 1e-6, chain * 1e-3};
     }
+    case P_GAT_DER: return {1.0, in.nnz * 8.0 * gb, in.nnz * 32.0 * gb, in.R * 1e-6};
     case P_ELEMENTWISE: return {1.0, in.R * K1 * 12.0 * gb};
     case P_ALLGATHER: return {1.0, in.ncols * K1 * 4.0 * (in.world - 1) / std::max(in.world, 1.0) * gb};
   }
@@ -364,8 +369,10 @@ double backward_cost(const CostModel& m, const In& in, int comp, double K1, doub
       if (need_dH) t += cost(m, in, P_GEMM, K2, K1);
       break;
     case GRANII_GAT_RECOMP:  // prep ; dT = dY Wᵀ ; A, B at K1 (B writes dH) ; dW = Tᵀ dY ; Hᵀ[del, der]
+      // (one GPU, no dH: der from pass A's per-entry dα instead of pass B, layer.cu der_only)
       t += cost(m, in, P_GEMM, K2, K1) + cost(m, in, P_ALLGATHER, K1) * 2.0 + cost(m, in, P_GAT_BWD_A, K1) +
-           cost(m, in, P_GAT_BWD_B, K1) + cost(m, in, P_ELEMENTWISE, K1);
+           (need_dH || in.world > 1 ? cost(m, in, P_GAT_BWD_B, K1) : cost(m, in, P_GAT_DER, 0)) +
+           cost(m, in, P_ELEMENTWISE, K1);
       break;
     default:
       return 0.0;
@@ -476,7 +483,7 @@ int comm_plan(const granii_graph_s* g, int64_t K, bool weighted, bool col_scale,
 
 granii_status cost_features_impl(const granii_graph_s* g, int32_t prim, int64_t K1, int64_t K2, double* feats,
                                  int32_t* n, char* model_name) {
-  if (prim < P_SPMM_W || prim > P_GAT_BWD_B) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
+  if (prim < P_SPMM_W || prim > P_GAT_DER) return fail(GRANII_ERR_INVALID_ARG, "unknown primitive id");
   const std::vector<double> f = features(inputs_of(g), prim, (double)K1, (double)K2);
   for (size_t i = 0; i < f.size(); ++i) feats[i] = f[i];
   *n = (int32_t)f.size();

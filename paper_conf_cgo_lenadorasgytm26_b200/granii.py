@@ -360,7 +360,7 @@ def granii_select(g: Graph, model: int, K1: int, K2: int, calib_path: str | None
 
 
 P_SPMM_W, P_SPMM_U, P_SPMM_U_CS, P_SDDMM1, P_SDDMM1_SM, P_GEMM, P_GEMM_NOSTORE, P_GEMM_TN, P_ELEMENTWISE, \
-    P_ALLGATHER, P_GEMM_ATT, P_GAT_BWD_A, P_GAT_BWD_B = range(13)
+    P_ALLGATHER, P_GEMM_ATT, P_GAT_BWD_A, P_GAT_BWD_B, P_GAT_DER = range(14)
 
 
 def granii_cost_features(g: Graph, prim: int, K1: int, K2: int = 0):

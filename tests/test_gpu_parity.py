@@ -281,6 +281,29 @@ def test_sddmm_norm_and_attention(G, name):
     assert err(out.cpu(), O.edge_softmax(c.rp, e), c.rp) <= TOL
 
 
+@pytest.mark.parametrize("cap", ["0", "40", "100", "1024"])
+@pytest.mark.parametrize("name", ["dense", "pubmed", "directed"])
+def test_sddmm_softmax_staged_rows(G, name, cap, monkeypatch):
+    """Fused K = 1 score + row softmax (Eq. 4): rows longer than one lane-group step are taken by a
+    whole warp with their scores staged in shared memory up to GRANII_SDDMM_CAP entries and streamed
+    through global memory beyond it (0: every such row streams; 40 / 100: a mix of both within the
+    same launch) -- bit-for-bit the same alpha as the default staging is not required, the R19
+    tolerance against the oracle's edge softmax is"""
+    monkeypatch.setenv("GRANII_SDDMM_CAP", cap)
+    c = case(G, name)
+    n, nnz = c.n, c.ci.shape[0]
+    el = synth.uniform_pm1(33, 1, (n,)) * 4
+    er = synth.uniform_pm1(33, 2, (n,)) * 4
+    out = torch.zeros(nnz, device=DEV)
+    G.granii_sddmm(c.g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el.to(DEV), 1, er.to(DEV), 1, 1, 1.0,
+                   out)
+    torch.cuda.synchronize()
+    rows = np.repeat(np.arange(n), np.diff(c.rp))
+    e = el.numpy().astype(np.float64)[rows] + er.numpy().astype(np.float64)[c.ci]
+    e = np.where(e > 0, e, 0.2 * e)
+    assert err(out.cpu(), O.edge_softmax(c.rp, e), c.rp) <= TOL
+
+
 @pytest.mark.parametrize("K", [2, 8, 41, 64, 128, 256, 512])
 def test_sddmm_dot_softmax(G, K):
     c = case(G, "dense")
@@ -362,6 +385,26 @@ def test_gemm_tn_tensor_core(G, M, N, R):
     G.granii_gemm(M, N, R, Ad, Ad.stride(0), Bd, Bd.stride(0), C2, N, G.GEMM_TRANS_A)
     torch.cuda.synchronize()
     assert torch.equal(C, C2), "split-K reduction must be deterministic"
+
+
+@pytest.mark.parametrize("M,N,R", [(100, 256, 300000), (256, 47, 300000), (602, 256, 120000)])
+def test_gemm_tn_long_reduction(G, M, N, R):
+    """dW over hundreds of thousands of node rows: the tcgen05 fp32 accumulation loses ~1 ulp of the
+    accumulator per MMA in one direction, so the error grows with the k-blocks per accumulator
+    (tools/gemm_tn_err.py); the split count follows R (<= 4096 rows per split) and each split spreads
+    its k-blocks over the TMEM accumulators, summed with round-to-nearest adds.  Both random-sign and
+    all-positive operands (no cancellation to hide a biased sum) against the fp64 product."""
+    for pos in (False, True):
+        A = synth.uniform_pm1(47, M % 13, (R, M))
+        B = synth.uniform_pm1(48, N % 11, (R, N))
+        if pos:
+            A, B = A.abs(), B.abs()
+        Ad, Bd = pad(A), pad(B)
+        C = torch.zeros(M, N, device=DEV)
+        G.granii_gemm(M, N, R, Ad, Ad.stride(0), Bd, Bd.stride(0), C, N, G.GEMM_TRANS_A)
+        torch.cuda.synchronize()
+        ref = O.gemm(A, B, ta=True)
+        assert normwise(C.cpu(), ref) <= (6e-5 if pos else 2e-5), pos
 
 
 # ------------------------------------------------------------------ layers
@@ -620,6 +663,47 @@ def test_gat_backward_deterministic_and_input_layer(G):
     assert torch.equal(runs[0][0], runs[1][0]) and torch.equal(runs[0][1], runs[1][1])
     assert torch.equal(runs[0][2], runs[1][2])
     assert torch.equal(runs[0][0], runs[2][0]) and runs[2][2] is None   # no dH: same dW
+
+
+@pytest.mark.parametrize("name,K1,K2,act,seg", [("dense", 100, 256, 1, 0), ("dense", 48, 16, 0, 0),
+                                                 ("pubmed", 32, 256, 1, 0), ("sparse", 47, 100, 0, 0),
+                                                 ("tiny", 5, 7, 1, 0), ("directed_t", 64, 128, 1, 0),
+                                                 ("directed_dense_t", 100, 47, 0, 0), ("dense", 64, 128, 0, 1),
+                                                 ("pubmed", 16, 64, 1, 1)])
+def test_gat_recomp_input_layer_der_only(G, name, K1, K2, act, seg, monkeypatch):
+    """RECOMP input layer (no dH): der_j = Σ_i α_ij (dα_ij - c_i) s'_ij from pass A's per-entry dα
+    through Ãᵀ's entry map instead of pass B's K-wide transposed SpMM (layer.cu der_only).  dW,
+    da_l, da_r against the oracle's chain rule (R22 tolerance), bitwise run-to-run, and against the
+    pass-B path (GRANII_GAT_DER_ONLY=0) within the same tolerance; seg=1 cuts every row over 64
+    entries into hub segments (der partials merged per row in fixed order)"""
+    if seg:
+        base = case(G, name)
+        monkeypatch.setenv("GRANII_SEG", "64")
+        g = G.granii_graph_csr_create(base.n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), base.flags)
+        monkeypatch.delenv("GRANII_SEG")
+        assert np.diff(base.rp).max() > 64
+        c = Case.__new__(Case)
+        c.n, c.g, c.rp, c.ci = base.n, g, base.rp, base.ci
+    else:
+        c = case(G, name)
+    Gup = synth.uniform_pm1(66, 1, (c.n, K2))
+    outs = []
+    for der_only in ("1", "1", "0"):
+        monkeypatch.setenv("GRANII_GAT_DER_ONLY", der_only)
+        net, out, H, W, al, ar = run_layer(G, c, G.GAT, 17, K1, K2, act, aligned=(K1 % 4 == 0))
+        if act and not outs:
+            Y, _ = O.gat_forward(17, c.rp, c.ci, H, W, al, ar, 0)
+            Gup[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0  # R20
+        assert net.backward(pad(Gup), need_input_grad=False) is None
+        torch.cuda.synchronize()
+        outs.append([x.cpu().clone() for x in (net.dW[0], net.da[0][0], net.da[0][1])])
+    ref = O.gat_backward(17, c.rp, c.ci, H, W, al, ar, Gup, act, need_dH=False)
+    mag = O.gat_backward_magnitude(17, c.rp, c.ci, H, W, al, ar, Gup, act, need_dH=False)
+    for got in (outs[0], outs[2]):
+        for nm, y, r, m in zip(("dW", "da_l", "da_r"), got, ref[1:], mag[1:]):
+            assert gat_grad_ok(y, r, m), nm
+    for a, b in zip(outs[0], outs[1]):
+        assert torch.equal(a, b)
 
 
 # ------------------------------------------------------------------ N3: SGC / TAGCN / GIN (reading R23)

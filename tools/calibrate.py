@@ -118,6 +118,23 @@ def sweep(quick=False):
                 rec(G.P_GAT_BWD_A, K, 0, prof["gat_bwd_a"]["ms"] / prof["gat_bwd_a"]["calls"])
                 rec(G.P_GAT_BWD_B, K, 0, prof["gat_bwd_b"]["ms"] / prof["gat_bwd_b"]["calls"])
                 del net, X, gup
+            # the der-only pass of a RECOMP input layer (no dH): independent of K
+            W = torch.full((64, 16), 0.01, device=DEV)
+            av = torch.full((16,), 0.05, device=DEV)
+            net = GNN(g, [LayerSpec(G.GAT, 64, 16, G.ACT_RELU, comp=G.GAT_RECOMP, W=W, a_l=av, a_r=av)], DEV)
+            X = alloc2d(R, 64, DEV, fill=0.5)
+            gup = alloc2d(R, 16, DEV, fill=0.01)
+            net.forward(X)
+            net.backward(gup, need_input_grad=False)
+            torch.cuda.synchronize()
+            G.granii_profile_enable(True)
+            for _ in range(3):
+                net.backward(gup, need_input_grad=False)
+            torch.cuda.synchronize()
+            prof = G.granii_profile_read()
+            G.granii_profile_enable(False)
+            rec(G.P_GAT_DER, 0, 0, prof["gat_der"]["ms"] / prof["gat_der"]["calls"])
+            del net, X, gup
         for (k1, k2) in GEMM_PAIRS:
             A = alloc2d(R, k1, DEV, fill=0.5)
             W = torch.full((k1, k2), 0.01, device=DEV)
