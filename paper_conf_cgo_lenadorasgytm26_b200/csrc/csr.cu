@@ -498,6 +498,7 @@ void graph_free(granii_graph_s* g) {
   if (!g) return;
   graph_free(g->T);
   cudaFree(g->tperm);
+  cudaFree(g->tblk);
   cudaFree(g->owner_off);
   cudaFree(g->ord_off);
   cudaFree(g->dinv2_rows);
@@ -515,10 +516,46 @@ void graph_free(granii_graph_s* g) {
   delete g;
 }
 
-// ---------------------------------------------------------------- Ãᵀ -> Ã entry map
+// ---------------------------------------------------------------- Ãᵀ -> Ã entry map, column-blocked
 // Ã's entries are ordered by (row i, column j); a stable sort of their positions by column gives them
 // in (column j, row i) order -- exactly the CSR order of Ãᵀ (row j, columns i ascending), which is the
 // order of the kept transpose T of a directed graph and of Ã itself when symmetric.
+// A per-entry array in Ã order (the der-only GAT backward's dz) is read in Ãᵀ order through that map:
+// 4-byte gathers over 4·nnz bytes, each 32-byte sector holding 8 columns of one row i that rows j far
+// apart need.  So the array is laid out COLUMN-BLOCKED instead: B blocks of columns, region b = the
+// entries whose column lies in block b, rows i ascending, each row's run in column order; B is chosen
+// so that a region (~ L2 / 3) stays in L2 while the rows j of its block -- consecutive in natural order
+// -- are summed.  tblk[e] = the blocked position of Ã's entry e (where the producer writes), tperm[e'] =
+// the blocked position of the Ã entry behind Ãᵀ's entry e' (where the consumer reads).
+__global__ void k_blk_count(int64_t n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col, int64_t bw,
+                            int nb, int32_t* __restrict__ cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    for (int b = 0; b < nb; ++b) cnt[(int64_t)b * n + i] = 0;
+    for (int64_t e = rp[i]; e < rp[i + 1]; ++e) ++cnt[(int64_t)(col[e] / bw) * n + i];
+  }
+}
+
+__global__ void k_blk_pos(int64_t n, const int64_t* __restrict__ rp, const int32_t* __restrict__ col, int64_t bw,
+                          const int32_t* __restrict__ off, int32_t* __restrict__ pos) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t b = -1, start = 0;
+    for (int64_t e = rp[i]; e < rp[i + 1]; ++e) {
+      const int64_t be = col[e] / bw;  // non-decreasing along the row (sorted columns)
+      if (be != b) {
+        b = be;
+        start = e;
+      }
+      pos[e] = off[b * n + i] + (int32_t)(e - start);
+    }
+  }
+}
+
+__global__ void k_compose(int64_t n, const int32_t* __restrict__ perm, const int32_t* __restrict__ pos,
+                          int32_t* __restrict__ out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+    out[e] = pos[perm[e]];
+}
+
 granii_status ensure_tperm(const granii_graph_s* gc, cudaStream_t st) {
   granii_graph_s* g = const_cast<granii_graph_s*>(gc);
   if (g->tperm) return GRANII_OK;
@@ -526,32 +563,59 @@ granii_status ensure_tperm(const granii_graph_s* gc, cudaStream_t st) {
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
   GR_CUDA(cudaStreamIsCapturing(st, &cs));
   if (cs != cudaStreamCaptureStatusNone) return fail(GRANII_ERR_UNSUPPORTED, "transpose entry map: stream capturing");
-  const int64_t n = g->local_nnz;
+  const int64_t n = g->local_nnz, R = g->n_rows;
   if (n > INT32_MAX) return fail(GRANII_ERR_UNSUPPORTED, "transpose entry map: more than 2^31 entries");
+  DevInfo di;
+  GR_TRY(dev_info(&di));
   int bits = 1;
   while (bits < 31 && (int64_t(1) << bits) < g->n_cols) ++bits;
-  int32_t *perm = nullptr, *iota = nullptr, *keys = nullptr;
+  // column blocks: regions of ~ L2 / 3 bytes (GRANII_TBLK overrides the count; 1 = Ã order)
+  int nb = (int)std::max<int64_t>(1, ceil_div(4 * n, std::max<int64_t>(di.l2_bytes / 3, 1)));
+  if (const char* e = getenv("GRANII_TBLK")) nb = std::max(1, atoi(e));
+  nb = (int)std::min<int64_t>(nb, std::max<int64_t>(g->n_cols, 1));
+  const int64_t bw = ceil_div(std::max<int64_t>(g->n_cols, 1), nb);
+  int32_t *perm = nullptr, *iota = nullptr, *keys = nullptr, *cnt = nullptr, *pos = nullptr, *tp = nullptr;
   void* tmp = nullptr;
-  size_t tb = 0;
+  size_t tb = 0, tb2 = 0;
   cub::DeviceRadixSort::SortPairs(nullptr, tb, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
                                   (int32_t*)nullptr, (int)n, 0, bits, st);
-  GR_CUDA(cudaMalloc(&perm, std::max<int64_t>(n, 1) * sizeof(int32_t)));
-  cudaError_t e = cudaMallocAsync(&iota, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
+  cub::DeviceScan::ExclusiveSum(nullptr, tb2, (const int32_t*)nullptr, (int32_t*)nullptr, (int)(nb * R), st);
+  tb = std::max(tb, tb2);
+  cudaError_t e = cudaMalloc(&pos, std::max<int64_t>(n, 1) * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&tp, std::max<int64_t>(n, 1) * sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMallocAsync(&perm, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&iota, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
   if (e == cudaSuccess) e = cudaMallocAsync(&keys, std::max<int64_t>(n, 1) * sizeof(int32_t), st);
+  if (e == cudaSuccess) e = cudaMallocAsync(&cnt, std::max<int64_t>((int64_t)nb * R, 1) * sizeof(int32_t) * 2, st);
   if (e == cudaSuccess) e = cudaMallocAsync(&tmp, std::max<size_t>(tb, 16), st);
   if (e == cudaSuccess && n > 0) {
     k_iota<<<grid_for(n), 256, 0, st>>>(n, iota);
     e = cub::DeviceRadixSort::SortPairs(tmp, tb, g->col_idx, keys, iota, perm, (int)n, 0, bits, st);
+    int32_t* off = cnt + (int64_t)nb * R;
+    const unsigned gr = (unsigned)std::min<int64_t>(ceil_div(R, 256), (int64_t)di.sms * 8);
+    if (e == cudaSuccess) {
+      k_blk_count<<<gr, 256, 0, st>>>(R, g->row_ptr, g->col_idx, bw, nb, cnt);
+      e = cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, off, (int)(nb * R), st);
+    }
+    if (e == cudaSuccess) {
+      k_blk_pos<<<gr, 256, 0, st>>>(R, g->row_ptr, g->col_idx, bw, off, pos);
+      k_compose<<<grid_for(n), 256, 0, st>>>(n, perm, pos, tp);
+    }
   }
   if (e == cudaSuccess) e = cudaGetLastError();
   cudaFreeAsync(tmp, st);
+  cudaFreeAsync(cnt, st);
   cudaFreeAsync(keys, st);
   cudaFreeAsync(iota, st);
+  cudaFreeAsync(perm, st);
   if (e != cudaSuccess) {
-    cudaFree(perm);
+    cudaFree(pos);
+    cudaFree(tp);
     return fail(GRANII_ERR_CUDA, std::string("transpose entry map: ") + cudaGetErrorString(e));
   }
-  g->tperm = perm;
+  g->tblk = pos;
+  g->tperm = tp;
+  g->tblk_n = nb;
   return GRANII_OK;
 }
 

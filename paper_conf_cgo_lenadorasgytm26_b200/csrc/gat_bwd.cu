@@ -93,6 +93,21 @@ __device__ __forceinline__ float gb_pdot(const float (&x)[NJ][4], const float (&
   return d;
 }
 
+// this lane's share of <x, z - p>: the difference is taken element by element before the dot, so
+// dα_ij - c_i = <dX_i, Z_j - P_i> (P_i = Y_i or T_i, c_i = <dX_i, P_i>) keeps its accuracy when Z_j ≈ P_i
+// -- the near-one-hot rows, where dα_ij and c_i agree to many digits and their fp32 difference would
+// be rounding noise (measured: da_l of the products-shaped training step 3.2e-4 -> see DESIGN R22)
+template <int NJ>
+__device__ __forceinline__ float gb_pdot_diff(const float (&x)[NJ][4], const float (&z)[NJ][4],
+                                              const float (&p)[NJ][4]) {
+  float d = 0.f;
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) d = fmaf(x[j][k], z[j][k] - p[j][k], d);
+  return d;
+}
+
 __device__ __forceinline__ float gb_lrelu(float z) { return z > 0.f ? z : 0.2f * z; }
 
 // dY = dout ⊙ σ'(out) and c_r = <dY_r, out_r> (= <dY_r, Y_r>: where ReLU clips, dY = 0). Lane groups of
@@ -150,9 +165,9 @@ __global__ void __launch_bounds__(256) k_gat_prep(int64_t R, int K, int Kv, int 
 // per-column scalars with one coalesced load (the next chunk is prefetched while this one is
 // processed), then lane groups take entries from the chunk by shuffles, U per group in flight,
 // so only the K-wide row gathers sit on the critical path.
-// WT (the der-only path, a.tout): each entry's dα is reduced over its lane group and written in Ã's
-// order, and D accumulates w·s'·(dα - c_i) per entry (the subtraction before the weighting: no
-// D - c·Cw cancellation at the end, Cw is left 0)
+// Every entry contributes w·s'·<dX_i, Z_j - P_i> = w·s'·(dα_ij - c_i) to D (gb_pdot_diff), so
+// del = D / S with no D - c·Cw cancellation at the end (Cw is left 0).  WT (the der-only path,
+// a.tout): each entry's dα_ij - c_i is also reduced over its lane group and written in Ã's order.
 template <int LPG, int NJ, int U, bool CL = false, bool WT = false>
 __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, int lane, int64_t seg = -1) {
   constexpr int G = 32 / LPG;
@@ -162,8 +177,9 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
   const int64_t b = seg >= 0 ? a.seg_lo[seg] : a.row_ptr[r], t = seg >= 0 ? a.seg_hi[seg] : a.row_ptr[r + 1];
   const float eli = a.el[r];
   const float ci = a.c[r];
-  float xv[NJ][4];
+  float xv[NJ][4], pv[NJ][4];
   gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, a.K, xv);
+  gb_load_row<LPG, NJ>(a.P + (int64_t)r * a.ldpp, lg, a.K, pv);
   // One sweep with an online softmax whose scalar work is done once per entry, by the lane that
   // loaded the entry's column (chunk of 32): its er (gathered a chunk ahead), score, slope s'; the
   // chunk's max over the warp (one rescale per chunk when it grows, warp-uniform m), then
@@ -218,22 +234,20 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
       if constexpr (WT) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          float pd = gb_pdot<NJ>(xv, zv[u]);
+          float pd = gb_pdot_diff<NJ>(xv, zv[u], pv);
+          D = fmaf(wu[u], pd, D);
 #pragma unroll
           for (int o = LPG / 2; o; o >>= 1) pd += __shfl_xor_sync(0xffffffffu, pd, o);
           const int slot = q * G * U + u * G + grp;
-          if (lg == 0 && slot < cnt) {
-            D = fmaf(wu[u], pd - ci, D);
-            a.tout[base + slot] = pd;
-          }
+          if (lg == 0 && slot < cnt) a.tout[base + slot] = pd;
         }
       } else {
 #pragma unroll
-        for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot<NJ>(xv, zv[u]), D);
+        for (int u = 0; u < U; ++u) D = fmaf(wu[u], gb_pdot_diff<NJ>(xv, zv[u], pv), D);
       }
     }
   }
-  if constexpr (WT) Cw = 0.f;
+  Cw = 0.f;  // D already holds Σ w s' (dα - c): del = D / S
   S = gb_warp_sum(S);
   Cw = gb_warp_sum(Cw);
   D = gb_warp_sum(D);
@@ -370,8 +384,9 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
   const int32_t r = live ? a.order[t0] : 0;
   const int64_t b = live ? a.row_ptr[r] : 0, t = live ? a.row_ptr[r + 1] : 0;
   const float eli = live ? a.el[r] : 0.f, ci = live ? a.c[r] : 0.f;
-  float xv[NJ][4];
+  float xv[NJ][4], pv[NJ][4];
   gb_load_row<LPG, NJ>(a.dX + (int64_t)r * a.ldx, lg, live ? a.K : 0, xv);
+  gb_load_row<LPG, NJ>(a.P + (int64_t)r * a.ldpp, lg, live ? a.K : 0, pv);
   float m = -INFINITY, S = 0.f, Cw = 0.f, D = 0.f;
   for (int64_t e = b; e < t; e += U) {
     int32_t j[U];
@@ -386,12 +401,12 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (e + u < t) {
-        float pd = gb_pdot<NJ>(xv, zv[u]);
+        float pd = gb_pdot_diff<NJ>(xv, zv[u], pv);  // this lane's share of dα - c_i
         if constexpr (WT) {
+          float pf = pd;
 #pragma unroll
-          for (int o = LPG / 2; o; o >>= 1) pd += __shfl_xor_sync(gmask, pd, o);
-          if (lg == 0) a.tout[e + u] = pd;
-          pd -= ci;  // every lane holds the entry's whole dα - c_i: D is not a lane share
+          for (int o = LPG / 2; o; o >>= 1) pf += __shfl_xor_sync(gmask, pf, o);
+          if (lg == 0) a.tout[e + u] = pf;
         }
         const float z = eli + erj[u];
         const float ev = gb_lrelu(z);
@@ -411,12 +426,9 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
       }
     }
   }
-  if constexpr (WT) {
-    Cw = 0.f;
-  } else {
 #pragma unroll
-    for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);
-  }
+  for (int o = LPG / 2; o; o >>= 1) D += __shfl_xor_sync(0xffffffffu, D, o);
+  Cw = 0.f;  // D already holds Σ w s' (dα - c): del = D / S
   const float inv_s = S > 0.f ? 1.f / S : 0.f;
   if (live && lg == 0) {
     a.del[r] = (D - ci * Cw) * inv_s;
@@ -566,31 +578,33 @@ __global__ void k_gat_b_combine(GatBwdArgs a) {
 
 // ---------------------------------------------------------------- der only (RECOMP input layer)
 // der_j = Σ_{i: j ∈ N(i)} dz_ij, dz_ij = α_ij (dα_ij - c_i) s'_ij -- the column sums of dz, which an
-// input layer needs instead of pass B's K-wide transposed SpMM (that only feeds dH).  Two streaming
-// passes instead of K-wide gathers:
-//   k_gat_dz  (rows i of Ã, schedule order): dz_ij from pass A's per-entry dα (tv, Ã order, in place),
-//             row i's record {el_i, m_i, 1/s_i, c_i} and a gathered er_j (L2-resident vector);
-//   k_gat_der (rows j of Ãᵀ, NATURAL order): der_j = Σ tv[tperm[e]] over Ãᵀ's row j.  The dz reads are
-//             4-byte gathers from a 4·nnz-byte array, but rows j processed together in natural order
-//             read neighbouring entries of every row i (its columns j are sorted), so each 32-byte
-//             sector of dz is fetched once and used by ~8 rows j while it stays in L2 (evict_last);
-//             the schedule's degree order would scatter them.  Hub rows (degree > seg_len, when the
-//             graph has segments) are taken as warp-wide segments first, their partials merged per
-//             row in fixed order.
-// Every sum in a fixed order (bitwise reproducible), no atomics.
+// input layer needs instead of pass B's K-wide transposed SpMM (that only feeds dH).  Two passes of
+// 4-byte accesses instead of K-wide gathers:
+//   k_gat_dz  (rows i of Ã, natural order): dz_ij from pass A's per-entry dα - c_i (tv, Ã order), row
+//             i's record {el_i, m_i, 1/s_i, c_i} and a gathered er_j (L2-resident vector), written to
+//             the graph's column-blocked layout (g->tblk: region b = the entries whose column lies in
+//             block b, rows ascending -- natural order writes each region front to back);
+//   k_gat_der (rows j of Ãᵀ, natural order = block by block): der_j = Σ tvb[tperm[e']] over Ãᵀ's row
+//             j -- 4-byte gathers, but only within the current block's region (~ L2 / 3), so each
+//             32-byte sector comes from DRAM about once.
+// Hub rows (degree > seg_len, when the graph has segments) are warp-wide segments taken first (dz:
+// independent per entry; der: partial sums merged per row in fixed order).  Every sum in a fixed order
+// (bitwise reproducible), no atomics.
 struct GatDzArgs {
-  int64_t n_rows;              // light rows (order[n_heavy ..])
-  const int32_t* order;
-  const longlong2* ord_rp;
-  const int32_t* col;
-  const float* er;
-  const float4* recs;
-  float* tv;
-  int l2hint;
-  int64_t n_seg;               // hub rows: warp-wide segments (dz is per entry: no merge needed)
+  int64_t n_rows;              // every row i (hubs skipped when segmented)
+  const int64_t* row_ptr;
+  int64_t seg_len;
+  int64_t n_seg;
   const int64_t* seg_lo;
   const int64_t* seg_hi;
   const int32_t* seg_row;
+  const int32_t* col;
+  const float* er;
+  const float4* recs;
+  const float* tv;             // dα - c_i, Ã order
+  const int32_t* tblk;
+  float* tvb;                  // dz, column-blocked
+  int l2hint;
 };
 
 template <int U>
@@ -598,23 +612,23 @@ __device__ __forceinline__ void gat_dz_run(const GatDzArgs& a, int32_t i, int64_
                                            const L2Pol& pol) {
   const float4 rc = __ldg(a.recs + i);  // {el_i, m_i, 1/s_i, c_i}
   for (; e < re; e += (int64_t)U * step) {
-    int32_t j[U];
+    int32_t j[U], q[U];
     float d[U], erj[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       const int64_t ee = e + (int64_t)u * step < re ? e + (int64_t)u * step : re - 1;
       j[u] = ldg_stream(a.col + ee, pol.stream);
       d[u] = ldg_stream(a.tv + ee, pol.stream);
+      q[u] = ldg_stream(a.tblk + ee, pol.stream);
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) erj[u] = ldg_pol(a.er + j[u], pol.keep);
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const int64_t ee = e + (int64_t)u * step;
-      if (ee < re) {
+      if (e + (int64_t)u * step < re) {
         const float z = rc.x + erj[u];
         const float al = __expf(gb_lrelu(z) - rc.y) * rc.z;
-        st_pol(a.tv + ee, al * (z > 0.f ? 1.f : 0.2f) * (d[u] - rc.w), pol.stream);
+        st_pol(a.tvb + q[u], al * (z > 0.f ? 1.f : 0.2f) * d[u], pol.stream);
       }
     }
   }
@@ -629,20 +643,21 @@ __global__ void __launch_bounds__(256) k_gat_dz(GatDzArgs a) {
   const L2Pol pol = make_l2pol(a.l2hint);
   for (int64_t t = warp; t < a.n_seg; t += nwarps)
     gat_dz_run<U>(a, a.seg_row[t], a.seg_lo[t] + lane, a.seg_hi[t], 32, pol);
-  for (int64_t t0 = warp * G; t0 < a.n_rows; t0 += nwarps * G) {
-    const int64_t t = t0 + grp;
-    if (t >= a.n_rows) continue;
-    const longlong2 rr = a.ord_rp[t];
-    gat_dz_run<U>(a, a.order[t], rr.x + lig, rr.y, LPG, pol);
+  for (int64_t i0 = warp * G; i0 < a.n_rows; i0 += nwarps * G) {
+    const int64_t i = i0 + grp;
+    if (i >= a.n_rows) continue;
+    const int64_t rs = a.row_ptr[i], re = a.row_ptr[i + 1];
+    if (a.n_seg > 0 && re - rs > a.seg_len) continue;  // a hub: its segments were taken above
+    gat_dz_run<U>(a, (int32_t)i, rs + lig, re, LPG, pol);
   }
 }
 
 struct GatDerArgs {
-  int64_t n_rows;              // every row j of Ãᵀ, natural order (hub rows skipped when segmented)
+  int64_t n_rows;              // every row j of Ãᵀ, natural order (hubs skipped when segmented)
   const int64_t* row_ptr;
-  int64_t seg_len;             // rows longer than this are hub segments (n_seg > 0)
+  int64_t seg_len;
   const int32_t* tperm;
-  const float* tv;             // dz in Ã order
+  const float* tvb;            // dz, column-blocked
   float* der;
   int64_t n_seg;
   const int64_t* seg_lo;
@@ -663,7 +678,7 @@ __device__ __forceinline__ float gat_dz_sum(const GatDerArgs& a, int64_t e, int6
       p[u] = ldg_stream(a.tperm + ee, pol.stream);
     }
 #pragma unroll
-    for (int u = 0; u < U; ++u) v[u] = ldg_pol(a.tv + p[u], pol.keep);
+    for (int u = 0; u < U; ++u) v[u] = ldg_pol(a.tvb + p[u], pol.keep);
 #pragma unroll
     for (int u = 0; u < U; ++u)
       if (e + (int64_t)u * step < re) acc += v[u];
@@ -685,15 +700,16 @@ __global__ void __launch_bounds__(256) k_gat_der(GatDerArgs a) {
   for (int64_t j0 = warp * G; j0 < a.n_rows; j0 += nwarps * G) {
     const int64_t j = j0 + grp;
     int64_t rs = 0, re = 0;
+    bool hub = false;
     if (j < a.n_rows) {
       rs = a.row_ptr[j];
       re = a.row_ptr[j + 1];
-      if (a.n_seg > 0 && re - rs > a.seg_len) re = rs;  // a hub: its segments were summed above
+      hub = a.n_seg > 0 && re - rs > a.seg_len;  // its segments were summed above
     }
-    float acc = gat_dz_sum<U>(a, rs + lig, re, LPG, pol);
+    float acc = gat_dz_sum<U>(a, rs + lig, hub ? rs : re, LPG, pol);
 #pragma unroll
     for (int o = LPG / 2; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (j < a.n_rows && lig == 0 && !(a.n_seg > 0 && a.row_ptr[j + 1] - rs > a.seg_len)) a.der[j] = acc;
+    if (j < a.n_rows && lig == 0 && !hub) a.der[j] = acc;
   }
 }
 
@@ -709,19 +725,19 @@ __global__ void k_gat_der_combine(int64_t n_heavy, const int32_t* __restrict__ h
 
 static int der_lpg(float avg) { return avg >= 96.f ? 32 : avg >= 24.f ? 16 : avg >= 6.f ? 8 : 4; }
 
-granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, const float* er, float* tv,
-                             const float4* recs, float* der, cudaStream_t st) {
+granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, const float* er, const float* tv,
+                             float* tvb, const float4* recs, float* der, cudaStream_t st) {
   if (g->n_rows == 0) return GRANII_OK;
-  if (!g->tperm) return fail(GRANII_ERR_INVALID_ARG, "der-only GAT backward without the transpose entry map");
+  if (!g->tperm || !g->tblk) return fail(GRANII_ERR_INVALID_ARG, "der-only GAT backward without the blocked entry map");
   DevInfo di;
   GR_TRY(dev_info(&di));
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const int hint = l2hint_enabled();
   {
-    // algorithmic bytes: per entry col + dα in + er + dz out; per row schedule entry + record
-    ProfScope ps("gat_dz", st, nnz * 16.0 + R * 36.0, 0.0, 1, -1.0, false);
-    GatDzArgs a{g->n_rows - g->n_heavy, g->order + g->n_heavy, g->ord_rp + g->n_heavy, g->col_idx, er, recs, tv, hint,
-                g->n_seg, g->seg_lo, g->seg_hi, g->seg_row};
+    // algorithmic bytes: per entry col + dα - c + blocked position + er + dz; per row 8 B row_ptr + record
+    ProfScope ps("gat_dz", st, nnz * 20.0 + R * 24.0, 0.0, 1, -1.0, false);
+    GatDzArgs a{g->n_rows, g->row_ptr, g->seg_len, g->n_seg, g->seg_lo, g->seg_hi, g->seg_row, g->col_idx, er,
+                recs, tv, g->tblk, tvb, hint};
     const int lpg = der_lpg(g->avg_deg());
     const int64_t want = ceil_div(ceil_div(a.n_rows, 32 / lpg) + a.n_seg, 8);
 #define GO(L) k_gat_dz<L, 4><<<(unsigned)persistent_grid(k_gat_dz<L, 4>, 256, di.sms, want), 256, 0, st>>>(a)
@@ -734,10 +750,10 @@ granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, 
 #undef GO
     GR_CHECK_LAUNCH();
   }
-  // algorithmic bytes: per entry map + dz (a 4-byte gather); per row 8 B row_ptr + der
+  // algorithmic bytes: per entry blocked position + dz (a 4-byte gather); per row 8 B row_ptr + der
   ProfScope ps("gat_der", st, (double)gt->local_nnz * 8.0 + (double)gt->n_rows * 12.0, 0.0, gt->n_seg > 0 ? 2 : 1,
                -1.0, false);
-  GatDerArgs b{gt->n_rows, gt->row_ptr, gt->seg_len, g->tperm, tv, der, gt->n_seg, gt->seg_lo, gt->seg_hi, nullptr,
+  GatDerArgs b{gt->n_rows, gt->row_ptr, gt->seg_len, g->tperm, tvb, der, gt->n_seg, gt->seg_lo, gt->seg_hi, nullptr,
                hint};
   if (gt->n_seg > 0) GR_CUDA(cudaMallocAsync((void**)&b.seg_der, gt->n_seg * sizeof(float), st));
   const int lpg = der_lpg(gt->avg_deg());
@@ -859,34 +875,25 @@ static granii_status gb_dispatch(int pass, const GatBwdArgs& b, bool dense, cuda
   // unmasked it needs 3 blocks / SM to avoid spills and loses (9.4 -> 9.9 ms).
   const char* ce = getenv("GRANII_GATBWD_CL");
   const bool cl = K % 4 == 0 && pass == 0 && !(ce && ce[0] == '0');
-  // tuning hook GRANII_GATBWD="LPG,NJ,U" (tools: bench.py per_primitive_ms), if it covers K
+  // tuning hook GRANII_GATBWD="LPG,NJ,U[,MINB[,CL]]" (tools/gatbwd_sweep.py), if it covers K; CL = 1: the
+  // unmasked row loader (K % 4 == 0 only)
   if (const char* e = getenv("GRANII_GATBWD")) {
-    int l = 0, n = 0, u = 0, mb = 0;
-    sscanf(e, "%d,%d,%d,%d", &l, &n, &u, &mb);
+    int l = 0, n = 0, u = 0, mb = 0, c = 0;
+    sscanf(e, "%d,%d,%d,%d,%d", &l, &n, &u, &mb, &c);
+    c = c && K % 4 == 0;
     if ((int64_t)l * n * 4 >= K) {
       bool ok = true;
-      if (l == 16 && n == 2 && u == 2 && mb == 4) gb_launch<16, 2, 2, 4>(pass, b, st);
-      else if (l == 16 && n == 2 && u == 2 && mb == 5) gb_launch<16, 2, 2, 5>(pass, b, st);
-      else if (l == 8 && n == 2 && u == 2 && mb == 4) gb_launch<8, 2, 2, 4>(pass, b, st);
-      else if (l == 8 && n == 2 && u == 2 && mb == 5) gb_launch<8, 2, 2, 5>(pass, b, st);
-      else if (l == 16 && n == 2 && u == 4 && mb == 3) gb_launch<16, 2, 4, 3>(pass, b, st);
-      else if (l == 8 && n == 2 && u == 4 && mb == 3) gb_launch<8, 2, 4, 3>(pass, b, st);
-      else if (l == 8 && n == 2 && u == 4) gb_launch<8, 2, 4>(pass, b, st);
-      else if (l == 16 && n == 1 && u == 4) gb_launch<16, 1, 4>(pass, b, st);
-      else if (l == 16 && n == 2 && u == 4) gb_launch<16, 2, 4>(pass, b, st);
-      else if (l == 16 && n == 2 && u == 2) gb_launch<16, 2, 2>(pass, b, st);
-      else if (l == 32 && n == 1 && u == 4) gb_launch<32, 1, 4>(pass, b, st);
-      else if (l == 32 && n == 1 && u == 2) gb_launch<32, 1, 2>(pass, b, st);
-      else if (l == 8 && n == 4 && u == 2) gb_launch<8, 4, 2>(pass, b, st);
-      else if (l == 16 && n == 4 && u == 2) gb_launch<16, 4, 2>(pass, b, st);
-      else if (l == 32 && n == 2 && u == 2) gb_launch<32, 2, 2>(pass, b, st);
-      else if (l == 32 && n == 2 && u == 1) gb_launch<32, 2, 1>(pass, b, st);
-      else if (l == 16 && n == 4 && u == 1) gb_launch<16, 4, 1>(pass, b, st);
-      else if (l == 32 && n == 4 && u == 2) gb_launch<32, 4, 2>(pass, b, st);
-      else if (l == 32 && n == 4 && u == 1) gb_launch<32, 4, 1>(pass, b, st);
-      else if (l == 16 && n == 8 && u == 1) gb_launch<16, 8, 1>(pass, b, st);
-      else if (l == 32 && n == 8 && u == 1) gb_launch<32, 8, 1>(pass, b, st);
-      else ok = false;
+#define GB_TRY(L, N, U_, MB)                                 \
+  if (l == L && n == N && u == U_ && mb == MB) {             \
+    if (c) gb_launch<L, N, U_, MB, true>(pass, b, st);       \
+    else gb_launch<L, N, U_, MB, false>(pass, b, st);        \
+  } else
+      GB_TRY(8, 2, 2, 0) GB_TRY(8, 2, 2, 4) GB_TRY(4, 3, 2, 0) GB_TRY(4, 3, 4, 0) GB_TRY(4, 3, 2, 4)
+      GB_TRY(4, 3, 4, 3) GB_TRY(16, 2, 2, 0) GB_TRY(16, 2, 2, 4) GB_TRY(4, 7, 1, 0) GB_TRY(4, 7, 2, 0)
+      GB_TRY(4, 7, 1, 3) GB_TRY(8, 4, 1, 0) GB_TRY(8, 4, 2, 0) GB_TRY(4, 4, 2, 0) GB_TRY(32, 2, 1, 0)
+      GB_TRY(16, 4, 2, 0) GB_TRY(4, 8, 1, 0) GB_TRY(16, 2, 2, 3) GB_TRY(8, 2, 2, 3)
+      ok = false;
+#undef GB_TRY
       if (ok) {
         GR_CHECK_LAUNCH();
         return GRANII_OK;
@@ -983,12 +990,17 @@ __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, 
   }
 }
 
+// out[i] + out[n + i] = the fp64 sum as a float pair (hi, lo): Wᵀ·(Hᵀ del) cancels, and rounding
+// Hᵀ del to fp32 before that product cost da_l 3e-4 normwise at products scale (DESIGN R22); the pair
+// travels through the fp32 all-reduce of several GPUs as two float sums
 __global__ void k_sum_chunks(int64_t n, int64_t S, const double* __restrict__ partial, float* __restrict__ out) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= n) return;
   double a = 0.0;
   for (int64_t s = 0; s < S; ++s) a += partial[s * n + i];
-  out[i] = (float)a;
+  const float hi = (float)a;
+  out[i] = hi;
+  out[n + i] = (float)(a - (double)hi);
 }
 
 static int64_t colreduce_chunks(int64_t R, int64_t K) {
@@ -1004,7 +1016,7 @@ granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ld
   ProfScope ps("elementwise", st, 4.0 * R * K + 8.0 * R, 4.0 * R * K, 2);
   k_colreduce2<<<dim3((unsigned)ceil_div(K, 32), (unsigned)S), dim3(32, 8), 0, st>>>(R, K, H, ldh, d0, d1, chunk,
                                                                                    reinterpret_cast<double*>(partial));
-  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, reinterpret_cast<const double*>(partial), out);
+  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, reinterpret_cast<const double*>(partial), out);  // 4K floats
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
@@ -1029,28 +1041,30 @@ __global__ void k_matvec2(int64_t K1, int64_t K2, const float* __restrict__ W, c
   }
 }
 
-// da_l = Wᵀ p, da_r = Wᵀ q (thread per column of W, fixed order over rows)
-__global__ void k_mattvec2(int64_t K1, int64_t K2, const float* __restrict__ W, const float* __restrict__ p,
-                           const float* __restrict__ q, float* __restrict__ dal, float* __restrict__ dar) {
+// da_l = Wᵀ p, da_r = Wᵀ q (thread per column of W, fixed order over rows), in fp64 from the
+// (hi, lo) pairs of p = [p | q | p_lo | q_lo] (k_sum_chunks): the sum cancels
+__global__ void k_mattvec2(int64_t K1, int64_t K2, const float* __restrict__ W, const float* __restrict__ pq,
+                           float* __restrict__ dal, float* __restrict__ dar) {
   const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (k >= K2) return;
-  float a = 0.f, b = 0.f;
+  double a = 0.0, b = 0.0;
   for (int64_t r = 0; r < K1; ++r) {
-    const float x = W[r * K2 + k];
-    a = fmaf(x, p[r], a);
-    b = fmaf(x, q[r], b);
+    const double x = W[r * K2 + k];
+    a = fma(x, (double)pq[r] + (double)pq[2 * K1 + r], a);
+    b = fma(x, (double)pq[K1 + r] + (double)pq[3 * K1 + r], b);
   }
-  if (dal) dal[k] = a;
-  if (dar) dar[k] = b;
+  if (dal) dal[k] = (float)a;
+  if (dar) dar[k] = (float)b;
 }
 
-// dW += p a_lᵀ + q a_rᵀ
-__global__ void k_rank2(int64_t K1, int64_t K2, float* __restrict__ dW, const float* __restrict__ p,
-                        const float* __restrict__ q, const float* __restrict__ al, const float* __restrict__ ar) {
+// dW += p a_lᵀ + q a_rᵀ (p, q from their (hi, lo) pairs)
+__global__ void k_rank2(int64_t K1, int64_t K2, float* __restrict__ dW, const float* __restrict__ pq,
+                        const float* __restrict__ al, const float* __restrict__ ar) {
   const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   if (i >= K1 * K2) return;
   const int64_t r = i / K2, k = i % K2;
-  dW[i] += p[r] * al[k] + q[r] * ar[k];
+  const float p = pq[r] + pq[2 * K1 + r], q = pq[K1 + r] + pq[3 * K1 + r];
+  dW[i] += p * al[k] + q * ar[k];
 }
 
 granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const float* a_l, const float* a_r,
@@ -1061,18 +1075,18 @@ granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const f
   return GRANII_OK;
 }
 
-granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* p, const float* q,
-                                  float* da_l, float* da_r, cudaStream_t st) {
+granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* pq, float* da_l, float* da_r,
+                                  cudaStream_t st) {
   ProfScope ps("elementwise", st, 4.0 * K1 * K2, 4.0 * K1 * K2, 1);
-  k_mattvec2<<<(unsigned)ceil_div(K2, 128), 128, 0, st>>>(K1, K2, W, p, q, da_l, da_r);
+  k_mattvec2<<<(unsigned)ceil_div(K2, 128), 128, 0, st>>>(K1, K2, W, pq, da_l, da_r);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
 
-granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p, const float* q, const float* a_l,
-                               const float* a_r, cudaStream_t st) {
+granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* pq, const float* a_l, const float* a_r,
+                               cudaStream_t st) {
   ProfScope ps("elementwise", st, 8.0 * K1 * K2, 4.0 * K1 * K2, 1);
-  k_rank2<<<(unsigned)ceil_div(K1 * K2, 256), 256, 0, st>>>(K1, K2, dW, p, q, a_l, a_r);
+  k_rank2<<<(unsigned)ceil_div(K1 * K2, 256), 256, 0, st>>>(K1, K2, dW, pq, a_l, a_r);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }

@@ -124,8 +124,11 @@ struct granii_graph_s {
   // featurize (degrees, dinv, integer features), partition + schedule (order, ord_rp, hub segments),
   // transpose (BUILD_TRANSPOSE) -- PAPER L365 quotes the featurizer's overhead on its own
   double create_ms[4] = {0, 0, 0, 0};
-  int32_t* tperm = nullptr;       // device, local_nnz, built on first use (one GPU; ensure_tperm): entry e of
-                                  // Ãᵀ's CSR (row j, column i) is entry tperm[e] of Ã's CSR (row i, column j)
+  // built on first use (one GPU; ensure_tperm): a column-blocked layout of per-entry arrays (tblk_n
+  // blocks of columns, region b = the entries whose column lies in block b, rows ascending)
+  int32_t* tblk = nullptr;        // device, local_nnz: blocked position of Ã's entry e
+  int32_t* tperm = nullptr;       // device, local_nnz: blocked position of the Ã entry (i, j) behind Ãᵀ's entry e' = (j, i)
+  int tblk_n = 0;
   granii_graph_s* T = nullptr;    // Ãᵀ over the same owned rows (GRANII_BUILD_TRANSPOSE, directed graphs);
                                   // its dinv arrays are Ã's (D̃ = Ã's row degrees, R4)
   // the graph the transposed aggregations of the backward run over (Mᵀ = M when symmetric)
@@ -206,6 +209,8 @@ struct GatBwdArgs {
   const float* el = nullptr;  // pass 0: own rows
   const float* er = nullptr;  // pass 0: column-id space; pass 1: own rows
   const float* c = nullptr;   // pass 0: own rows
+  const float* P = nullptr;   // pass 0: own rows of the forward's Y (REUSE) or T = αH (RECOMP): <dX_i, P_i> = c_i
+  int64_t ldpp = 0;
   float* dXw = nullptr;       // pass 0: dX's own rows, whose tail receives the row record
   int64_t rec = 0;            // column of the 16-byte record {el, m, 1/s, c} in dX rows
   float* del = nullptr;       // pass 0 out
@@ -228,29 +233,32 @@ struct GatBwdArgs {
   float4* seg_a = nullptr;    // pass 0: online-softmax state {m, S, Cw, D} per segment
   float* seg_b = nullptr;     // pass 1: partial output row per segment (ld ldp)
   float* seg_der = nullptr;   // pass 1: partial der per segment
-  float* tout = nullptr;      // pass 0, optional: dα_ij per entry in Ã's CSR order (the der-only path)
+  float* tout = nullptr;      // pass 0, optional: dα_ij - c_i per entry in Ã's CSR order (the der-only path)
   float4* recs = nullptr;     // pass 0, optional: the row records {el, m, 1/s, c}, one float4 per own row
 };
 granii_status launch_gat_prep(int64_t R, int64_t K, const float* out, int64_t ldo, const float* g, int64_t ldg,
                               bool relu, float* dY, int64_t ldd, float* c, cudaStream_t st);
 granii_status launch_gat_bwd_pass(const granii_graph_s* g, int pass, const GatBwdArgs& a, cudaStream_t st);
-// Ãᵀ's entry -> Ã's entry map (g->tperm), built once by a stable radix sort of Ã's column ids;
+// the column-blocked entry layout (g->tblk, g->tperm: Ã's and Ãᵀ's entries -> blocked positions), built
+// once (stable radix sort of Ã's column ids, per-(block, row) counts and their scan);
 // GRANII_ERR_UNSUPPORTED on a partitioned graph or while `st` is being captured (no allocation)
 granii_status ensure_tperm(const granii_graph_s* g, cudaStream_t st);
 // der_j = Σ_{i: j ∈ N(i)} α_ij (dα_ij - c_i) s'_ij over the rows j of gt = Ãᵀ from pass A's per-entry dα
-// (tv, Ã order, turned into dz in place, then summed through g->tperm) and compact row records: the
-// RECOMP input layer's backward, which needs no dH and so no K-wide transposed SpMM (pass B)
-granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, const float* er, float* tv,
-                             const float4* recs, float* der, cudaStream_t st);
+// (tv, Ã order; dz written to tvb in the graph's column-blocked layout, then summed through g->tperm) and
+// compact row records: the RECOMP input layer's backward, which needs no dH and so no K-wide transposed
+// SpMM (pass B)
+granii_status launch_gat_der(const granii_graph_s* g, const granii_graph_s* gt, const float* er, const float* tv,
+                             float* tvb, const float4* recs, float* der, cudaStream_t st);
 size_t colreduce2_workspace(int64_t R, int64_t K);
+// out: 4K floats, [Hᵀd0 | Hᵀd1] as (hi, lo) float pairs: out[0 .. 2K) hi, out[2K .. 4K) lo
 granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ldh, const float* d0, const float* d1,
                                 float* partial, float* out, cudaStream_t st);
 granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const float* a_l, const float* a_r,
                                 float* u, float* v, cudaStream_t st);
-granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* p, const float* q,
-                                  float* da_l, float* da_r, cudaStream_t st);
-granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* p, const float* q, const float* a_l,
-                               const float* a_r, cudaStream_t st);
+granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* pq, float* da_l, float* da_r,
+                                  cudaStream_t st);
+granii_status launch_gat_rank2(int64_t K1, int64_t K2, float* dW, const float* pq, const float* a_l, const float* a_r,
+                               cudaStream_t st);
 // comm
 granii_status comm_allgather(granii_comm_s* c, const float* send, float* recv, size_t count, cudaStream_t st);
 granii_status comm_allreduce_sum(granii_comm_s* c, float* buf, size_t count, cudaStream_t st);

@@ -772,6 +772,16 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   GatherBuf dyg = reuse ? gather_buf(b, c, rec + 4) : local_buf(b, R, K2);
   GatherBuf dtg;
   if (!reuse) dtg = gather_buf(b, c, rec + 4);
+  // pass A's P rows (<dX_i, P_i> = c_i): REUSE's output Y (16-byte rows: copied when the caller's are
+  // not; the sizing pass always reserves the copy), RECOMP's saved T
+  const float* Pp = reuse ? out : saved;
+  int64_t ldP = reuse ? ldo : sv.ldz;
+  if (reuse && (!run || ldo % 4 != 0 || ((uintptr_t)out & 15) != 0)) {
+    float* pc = b.take((size_t)Rr * ld4(K2));
+    if (run) GR_TRY(launch_copy_rows(R, K2, out, ldo, pc, ld4(K2), st));
+    Pp = pc;
+    ldP = ld4(K2);
+  }
   float* cvec = b.take((size_t)Rr);
   float* del = b.take((size_t)Rr);
   float* der = b.take((size_t)Rr);
@@ -793,6 +803,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
   bool der_only = false;
   if (der_only_ok && run) der_only = ensure_tperm(g, st) == GRANII_OK;
   float* tv = der_only_ok ? b.take((size_t)g->local_nnz) : nullptr;
+  float* tvb = der_only_ok ? b.take((size_t)g->local_nnz) : nullptr;
   float4* recs = der_only_ok ? reinterpret_cast<float4*>(b.take((size_t)Rr * 4)) : nullptr;
   float* bout = nullptr;  // pass B output
   int64_t ldbo = 0;
@@ -807,7 +818,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     ldbo = ld4(K1);
   }
   float* uv = reuse ? nullptr : b.take((size_t)2 * K1);
-  float* pq = b.take((size_t)2 * K1);
+  float* pq = b.take((size_t)4 * K1);  // Hᵀ[del, der] as (hi, lo) float pairs
   float* partial = (float*)b.take_bytes(colreduce2_workspace(R, K1));
   void* gwW;
   size_t gnW;
@@ -843,6 +854,8 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     pa.el = el;
     pa.er = er_all;
     pa.c = cvec;
+    pa.P = Pp;  // Y_i (post-activation: dY is 0 where ReLU clipped) or the saved T_i
+    pa.ldpp = ldP;
     pa.dXw = reuse ? dyg.mine : dtg.mine;
     pa.rec = rec;
     pa.del = del;
@@ -852,7 +865,7 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     }
     GR_TRY(launch_gat_bwd_pass(g, 0, pa, st));
     if (c.dist()) GR_TRY(allgather(c, reuse ? dyg : dtg));  // rows + records
-    if (der_only) GR_TRY(launch_gat_der(g, gt, er_own, tv, recs, der, st));
+    if (der_only) GR_TRY(launch_gat_der(g, gt, er_own, tv, tvb, recs, der, st));
     if (!reuse && !der_only) GR_TRY(launch_gat_matvec2(K1, K2, a->W, a->a_l, a->a_r, uv, uv + K1, st));
     GatBwdArgs pb;
     pb.n_rows = R;
@@ -885,10 +898,10 @@ static granii_status gat_backward_impl(const Ctx& c, granii_composition comp, co
     GR_TRY(launch_colreduce2(R, K1, H, ldh, del, der, partial, pq, st));
     if (c.dist()) {
       GR_TRY(comm_allreduce_sum(c.comm, dW, (size_t)K1 * K2, st));
-      GR_TRY(comm_allreduce_sum(c.comm, pq, (size_t)2 * K1, st));
+      GR_TRY(comm_allreduce_sum(c.comm, pq, (size_t)4 * K1, st));
     }
-    if (!reuse) GR_TRY(launch_gat_rank2(K1, K2, dW, pq, pq + K1, a->a_l, a->a_r, st));
-    if (a->d_a_l || a->d_a_r) GR_TRY(launch_gat_mattvec2(K1, K2, a->W, pq, pq + K1, a->d_a_l, a->d_a_r, st));
+    if (!reuse) GR_TRY(launch_gat_rank2(K1, K2, dW, pq, a->a_l, a->a_r, st));
+    if (a->d_a_l || a->d_a_r) GR_TRY(launch_gat_mattvec2(K1, K2, a->W, pq, a->d_a_l, a->d_a_r, st));
   }
   if (ws_size) *ws_size = b.off + 1024;
   return GRANII_OK;

@@ -151,12 +151,13 @@ def test_products_inference_fullsize(G, model):
 def test_products_gat_training_fullsize(G, layer):
     """C5 GAT training (products-gat2-train, 100 -> 256 -> 47): each layer's backward at full size
     under the composition the bench selects, one layer at a time so the ReLU' decision can be made
-    unique (R20): dW, da_l, da_r (reductions over all 2.45M rows) and, for the second layer (which
-    the step differentiates with respect to its input), dH on 4,096 random + 64 hub rows, against
+    unique (R20; R27 for LeakyReLU' on the scores): dW, da_l, da_r (reductions over all 2.45M rows)
+    and, for the second layer (which the step differentiates with respect to its input), dH on 4,096
+    random + 64 hub rows, against
     oracle_gat_backward with the R22 tolerance (gat_grad_ok).  These are the pass A / pass B
     shapes (K = 100 for RECOMP's dT H rows, K = 47 for REUSE's dY Θ rows) chosen only at this scale."""
     import bench
-    from test_gpu_parity import gat_grad_ok
+    from test_gpu_parity import gat_grad_ok, leaky_ambiguous_rows
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec, alloc2d
     w, g, rp, ci = build(G, "products")
     spec = bench.WORKLOADS["products-gat2-train"]
@@ -175,6 +176,9 @@ def test_products_gat_training_fullsize(G, layer):
         Y, _ = O.gat_forward(L.comp, rp, ci, Hn, Wn, al, ar, 0)
         U[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0      # R20
         del Y
+    amb = leaky_ambiguous_rows(rp, ci, Hn, Wn, al, ar)                       # R27
+    assert amb.shape[0] < 0.005 * w.n   # 3,639 / 3,825 rows of 2.45 M (layers 0 / 1)
+    U[torch.from_numpy(amb)] = 0.0
     net = GNN(g, [LayerSpec(G.GAT, K1, K2, act, G.ATTN_ADDITIVE, comp=L.comp, W=L.W, a_l=L.a_l, a_r=L.a_r)], DEV)
     net.forward(H)
     Ud = alloc2d(w.n, K2, DEV)

@@ -538,6 +538,24 @@ def test_gat_backward_both_compositions(G, comp, name, K1, K2, act):
         assert gat_grad_ok(y.cpu(), r, m), nm
 
 
+def leaky_ambiguous_rows(rp, ci, H, W, a_l, a_r, rel=1e-5):
+    """R27: LeakyReLU'(z_ij) is an integer decision (slope 1 or 0.2) taken on a float, z_ij = el_i + er_j
+    with el = H W a_l, er = H W a_r (R8).  Where |z_ij| is within rounding of 0 both slopes are correct,
+    and one entry decided the other way moves del_i / der_j by a whole term -- at 130 M entries a few
+    dozen such entries exist (none on the small parity graphs).  Returns the rows i holding such an
+    entry; a test zeroes their upstream gradient (dX_i = 0 makes dz_ij = 0 whatever the slope), as R20
+    does for ReLU'.  Values in fp64 from the inputs, never from the CUDA path."""
+    rp, ci = np.asarray(rp, np.int64), np.asarray(ci, np.int64)
+    Wd = np.asarray(W, np.float64)
+    Hd = np.asarray(H, np.float64)
+    el = Hd @ (Wd @ np.asarray(a_l, np.float64))
+    er = Hd @ (Wd @ np.asarray(a_r, np.float64))
+    deg = np.diff(rp)
+    z = np.repeat(el, deg) + er[ci]
+    tau = rel * max(np.abs(el).max(), np.abs(er).max())
+    return np.unique(np.repeat(np.arange(rp.shape[0] - 1), deg)[np.abs(z) < tau])
+
+
 def gat_grad_ok(y, r, m):
     """R22: per row, |y - r|∞ <= 1e-4 |r|∞ + 4u |m|∞ (u = 2^-24, m = the computation's magnitude):
     the softmax backward α(dα - Σα dα) cancels by construction on near-one-hot rows, and a fp32
@@ -665,23 +683,29 @@ def test_gat_backward_deterministic_and_input_layer(G):
     assert torch.equal(runs[0][0], runs[2][0]) and runs[2][2] is None   # no dH: same dW
 
 
-@pytest.mark.parametrize("name,K1,K2,act,seg", [("dense", 100, 256, 1, 0), ("dense", 48, 16, 0, 0),
-                                                 ("pubmed", 32, 256, 1, 0), ("sparse", 47, 100, 0, 0),
-                                                 ("tiny", 5, 7, 1, 0), ("directed_t", 64, 128, 1, 0),
-                                                 ("directed_dense_t", 100, 47, 0, 0), ("dense", 64, 128, 0, 1),
-                                                 ("pubmed", 16, 64, 1, 1)])
-def test_gat_recomp_input_layer_der_only(G, name, K1, K2, act, seg, monkeypatch):
-    """RECOMP input layer (no dH): der_j = Σ_i α_ij (dα_ij - c_i) s'_ij from pass A's per-entry dα
-    through Ãᵀ's entry map instead of pass B's K-wide transposed SpMM (layer.cu der_only).  dW,
-    da_l, da_r against the oracle's chain rule (R22 tolerance), bitwise run-to-run, and against the
-    pass-B path (GRANII_GAT_DER_ONLY=0) within the same tolerance; seg=1 cuts every row over 64
-    entries into hub segments (der partials merged per row in fixed order)"""
-    if seg:
+@pytest.mark.parametrize("name,K1,K2,act,seg,blk", [("dense", 100, 256, 1, 0, 0), ("dense", 48, 16, 0, 0, 3),
+                                                     ("pubmed", 32, 256, 1, 0, 0), ("sparse", 47, 100, 0, 0, 7),
+                                                     ("tiny", 5, 7, 1, 0, 0), ("directed_t", 64, 128, 1, 0, 0),
+                                                     ("directed_t", 32, 48, 0, 0, 5),
+                                                     ("directed_dense_t", 100, 47, 0, 0, 4),
+                                                     ("dense", 64, 128, 0, 1, 0), ("pubmed", 16, 64, 1, 1, 6)])
+def test_gat_recomp_input_layer_der_only(G, name, K1, K2, act, seg, blk, monkeypatch):
+    """RECOMP input layer (no dH): der_j = Σ_i α_ij (dα_ij - c_i) s'_ij from pass A's per-entry
+    dα - c_i, turned into dz in the graph's column-blocked entry layout and summed over Ãᵀ's rows,
+    instead of pass B's K-wide transposed SpMM (layer.cu der_only).  dW, da_l, da_r against the
+    oracle's chain rule (R22 tolerance), bitwise run-to-run, and against the pass-B path
+    (GRANII_GAT_DER_ONLY=0) within the same tolerance; seg=1 cuts every row over 64 entries into hub
+    segments (der partials merged per row in fixed order); blk > 0 forces that many column blocks
+    (GRANII_TBLK; test graphs fit one region by default)"""
+    if seg or blk:
         base = case(G, name)
-        monkeypatch.setenv("GRANII_SEG", "64")
+        if seg:
+            monkeypatch.setenv("GRANII_SEG", "64")
         g = G.granii_graph_csr_create(base.n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), base.flags)
-        monkeypatch.delenv("GRANII_SEG")
-        assert np.diff(base.rp).max() > 64
+        monkeypatch.delenv("GRANII_SEG", raising=False)
+        if blk:
+            monkeypatch.setenv("GRANII_TBLK", str(blk))
+        assert not seg or np.diff(base.rp).max() > 64
         c = Case.__new__(Case)
         c.n, c.g, c.rp, c.ci = base.n, g, base.rp, base.ci
     else:

@@ -39,6 +39,11 @@ if act:
     Y, _ = O.gat_forward(L.comp, rp, ci, Hn, Wn, al, ar, 0)
     U[torch.from_numpy(np.abs(Y) < 1e-4 * np.abs(Y).max())] = 0.0
     del Y
+if os.environ.get("R27", "1") == "1":
+    from test_gpu_parity import leaky_ambiguous_rows
+    amb = leaky_ambiguous_rows(rp, ci, Hn, Wn, al, ar)
+    print(f"R27: {amb.shape[0]} rows with an ambiguous LeakyReLU' decision zeroed", flush=True)
+    U[torch.from_numpy(amb)] = 0.0
 net = GNN(g, [LayerSpec(G.GAT, K1, K2, act, G.ATTN_ADDITIVE, comp=L.comp, W=L.W, a_l=L.a_l, a_r=L.a_r)], DEV)
 net.forward(H)
 Ud = alloc2d(w.n, K2, DEV)
