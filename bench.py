@@ -253,6 +253,16 @@ def cpu_oracle_sample(rp, ci, dims, target_s=12.0, seed=0, model="gcn", train=Fa
             "mode": what, "seconds": dt}
 
 
+def gather_peak():
+    """random 4-byte gathers per second measured by tools/probe/gather_rate.cu on B200
+    (profiles/gather_rate.json): the best streamed-index rate over the workload table sizes (the
+    highest rate = the most conservative roof); not a driver measurement -- the line says so"""
+    gp = os.path.join(ROOT, "profiles", "gather_rate.json")
+    if not os.path.exists(gp):
+        return None
+    return max(r["stream_nc_Gps"] for r in json.load(open(gp))["rows"]) * 1e9
+
+
 def l2_peak():
     """L2 -> SM read bandwidth measured by tools/probe/l2_bw.cu on B200 (profiles/l2_peak.json);
     not a driver measurement -- the line says so where it is used"""
@@ -288,9 +298,17 @@ def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
             out.update(bound="hbm", achieved=by / t / 1e9, peak=hbm, unit="GB/s",
                        peak_note=f"hbm_gbs of {peak_src} (tall-skinny GEMM below the ridge)")
         out["tensor_frac"] = fl / t / 1e12 / tc
-    elif name in ("spmm", "sddmm", "gat_bwd_a", "gat_bwd_b") and l2:
+    elif name in ("spmm", "sddmm", "sddmm_dot", "gat_bwd_a", "gat_bwd_b") and l2:
         t_l2, t_hbm = by / (l2 * 1e9), comp / (hbm * 1e9)
-        if traffic and st.get("l2_resident", 0) < calls:
+        # K = 1 SDDMM: one random 4-byte V gather per entry (flops = 2 nnz); a 32-lane random gather
+        # costs 32 L1tex wavefronts, so the gather rate, not bytes, is the roof
+        gp = gather_peak() if name == "sddmm" else None
+        n_g = fl / 2.0
+        if gp and n_g > 0 and n_g / gp >= max(t_l2, t_hbm):
+            out.update(bound="gather", achieved=n_g / t / 1e9, peak=gp / 1e9, unit="G gathers/s",
+                       peak_note="random 4-byte gather rate measured by tools/probe/gather_rate.cu "
+                                 "(profiles/gather_rate.json), not a driver figure: entries / t")
+        elif traffic and st.get("l2_resident", 0) < calls:
             # the gathered operand does not fit L2: its gathers are DRAM reads at a hit rate the
             # algorithmic bytes cannot tell -- the binding roof is the DRAM traffic ncu measured
             out.update(bound="hbm", achieved=traffic / (st["ms"] / calls / 1e3) / 1e9, peak=hbm, unit="GB/s",

@@ -111,6 +111,15 @@ __global__ void k_ord_rp(int64_t n, const int32_t* __restrict__ order, const int
   }
 }
 
+// tile_row[t] = the row r with row_ptr[r] <= t·TE < row_ptr[r+1] (every tile start lies in one non-empty row)
+__global__ void k_tile_rows(int64_t n, const int64_t* __restrict__ rp, int64_t TE, int32_t* __restrict__ tr) {
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = rp[r], b = rp[r + 1];
+    if (b == a) continue;
+    for (int64_t t = (a + TE - 1) / TE; t <= (b - 1) / TE; ++t) tr[t] = (int32_t)r;
+  }
+}
+
 __global__ void k_permute_off(int64_t n, int G1, const int32_t* __restrict__ order, const int32_t* __restrict__ off,
                               int32_t* __restrict__ out) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n * G1; i += (int64_t)gridDim.x * blockDim.x) {
@@ -406,6 +415,10 @@ granii_status graph_create(int64_t N, int64_t E, const int32_t* d_src, const int
   }
   CK(cudaMalloc(&g->ord_rp, std::max<int64_t>(g->n_rows, 1) * sizeof(longlong2)));
   if (g->n_rows > 0) k_ord_rp<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->order, g->row_ptr, g->ord_rp);
+  g->n_tiles = ceil_div(g->local_nnz, granii_graph_s::tile_e);
+  CK(cudaMalloc(&g->tile_row, std::max<int64_t>(g->n_tiles, 1) * sizeof(int32_t)));
+  if (g->n_tiles > 0)
+    k_tile_rows<<<grid_for(g->n_rows), 256, 0, st>>>(g->n_rows, g->row_ptr, granii_graph_s::tile_e, g->tile_row);
   if (g->owner_off) {
     CK(cudaMalloc(&g->ord_off, std::max<int64_t>(g->n_rows, 1) * (world + 1) * sizeof(int32_t)));
     if (g->n_rows > 0)
@@ -508,6 +521,7 @@ void graph_free(granii_graph_s* g) {
   cudaFree(g->col_idx);
   cudaFree(g->order);
   cudaFree(g->ord_rp);
+  cudaFree(g->tile_row);
   cudaFree(g->seg_ptr);
   cudaFree(g->seg_lo);
   cudaFree(g->seg_hi);

@@ -118,6 +118,11 @@ struct granii_graph_s {
   // rows with more than wide_deg entries = order[0 .. n_wide): the sparse (group-per-row)
   // schedules give them a whole warp
   int64_t wide_deg = 32, n_wide = 0;
+  // entry tiles of the K = 1 SDDMM (sddmm.cu): tile t = Ã's entries
+  // [t·tile_e, (t+1)·tile_e) in CSR order; tile_row[t] = the row holding entry t·tile_e
+  static constexpr int64_t tile_e = 4096;
+  int64_t n_tiles = 0;
+  int32_t* tile_row = nullptr;    // device, n_tiles
   int64_t features[GRANII_NUM_FEATURES] = {0};
   int device = 0;
   // host wall time of the creation phases (ms): CSR build (validate, sort, dedupe, row_ptr / col_idx),

@@ -277,6 +277,347 @@ __global__ void __launch_bounds__(256) k_sddmm1(SddmmArgs a) {
   }
 }
 
+static int lpg_for_softmax(float avg);
+static int lpg_for_degree(float avg);
+static bool sddmm_tile_enabled(const granii_graph_s* g);
+
+// ---------------------------------------------------------------- K = 1 over entry tiles
+// The degree-ordered kernel above keeps one dependent chain per lane group (order -> entry range
+// -> col -> V -> exp -> store) and so few bytes in flight per SM that products-shaped inputs reach
+// ~1.8 TB/s.  Here a CTA owns a tile of tile_e consecutive entries of Ã in CSR order: (A) every
+// thread loads 16 column ids with four 16-byte streaming loads and issues its 16 V gathers at once
+// (4096 independent gathers per CTA), parking V_c in shared memory; (B) the tile's rows (row_ptr
+// slice in shared memory) are scored, max-reduced, exponentiated and normalised in shared memory
+// by lane groups (rows of >= TILE_BIG in-tile entries by the whole CTA); (C) the tile is written
+// back with full-line 16-byte stores.  A row cut by a tile boundary keeps its scores and leaves its
+// in-tile (max, sum) in st_first / st_last; k_sddmm1_xstats combines a crossing row's partials in
+// tile order and k_sddmm1_xnorm normalises its entries (alpha = exp(e - m) / s, the same formula).
+constexpr int TILE_E = (int)granii_graph_s::tile_e;
+constexpr int TILE_T = 256;
+constexpr int TILE_RCH = 512;   // rows per row_ptr chunk in shared memory
+constexpr int TILE_BIG = 512;   // in-tile row length processed by the whole CTA
+
+struct TileArgs {
+  int64_t n_rows, nnz, n_tiles;
+  const int64_t* __restrict__ row_ptr;
+  const int32_t* __restrict__ col_idx;
+  const int32_t* __restrict__ tile_row;
+  const float* __restrict__ U;
+  int64_t ldu;
+  const float* __restrict__ V;
+  int64_t ldv;
+  float scale;
+  float* __restrict__ out;
+  float2* st_first;   // softmax: in-tile (max, sum) of the tile's first row (if it began earlier)
+  float2* st_last;    // ... and of its last row (if it continues into the next tile)
+  float2* fin_first;  // crossing rows' final (max, 1/sum), per tile it enters / begins in
+  float2* fin_last;
+  int l2hint;
+};
+
+template <int LPG, bool ADD, bool LRELU, bool SOFTMAX>
+__global__ void __launch_bounds__(TILE_T) k_sddmm1_tile(TileArgs a) {
+  __shared__ __align__(16) float sv[TILE_E];
+  __shared__ int32_t srp[TILE_RCH + 1];
+  __shared__ float sred[2][TILE_T / 32];
+  __shared__ int32_t sbig[TILE_E / TILE_BIG + 1];
+  __shared__ int s_nbig;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const L2Pol pol = make_l2pol(a.l2hint);
+  const int64_t t = blockIdx.x;
+  const int64_t e0 = t * TILE_E, e1 = min(e0 + (int64_t)TILE_E, a.nnz);
+  const int ne = (int)(e1 - e0);
+  // (A) column ids (coalesced 16-byte streaming loads), then 16 independent V gathers per thread
+  {
+    int32_t c[16];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int j = warp * 512 + q * 128 + lane * 4;
+      if (j + 3 < ne) {
+        const int4 v = ldg_stream(reinterpret_cast<const int4*>(a.col_idx + e0 + j), pol.stream);
+        c[4 * q] = v.x; c[4 * q + 1] = v.y; c[4 * q + 2] = v.z; c[4 * q + 3] = v.w;
+      } else {
+#pragma unroll
+        for (int r = 0; r < 4; ++r) c[4 * q + r] = j + r < ne ? ldg_stream(a.col_idx + e0 + j + r, pol.stream) : 0;
+      }
+    }
+    float v[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = ldg_pol(a.V + (int64_t)c[i] * a.ldv, pol.keep);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int j = warp * 512 + q * 128 + lane * 4;
+      if (j + 3 < ne) {
+        *reinterpret_cast<float4*>(sv + j) = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      } else {
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+          if (j + r < ne) sv[j + r] = v[4 * q + r];
+      }
+    }
+  }
+  // (B) rows of the tile
+  const int64_t r0 = a.tile_row[t];
+  const int64_t rend = (t + 1 < a.n_tiles) ? (int64_t)a.tile_row[t + 1] + 1 : a.n_rows;
+  const bool first_cut = SOFTMAX && a.row_ptr[r0] < e0;  // r0 began in an earlier tile
+  const int64_t rlast = rend - 1;                          // holds entry e1 when it continues
+  const bool last_cut = SOFTMAX && t + 1 < a.n_tiles && a.row_ptr[rlast] < e1;
+  constexpr int G = 32 / LPG;
+  const int grp = lane / LPG, lig = lane % LPG;
+  for (int64_t c0 = r0; c0 < rend; c0 += TILE_RCH) {
+    const int nr = (int)min((int64_t)TILE_RCH, rend - c0);
+    __syncthreads();  // sv complete (first chunk) / srp and sbig free (later chunks)
+    if (tid == 0) s_nbig = 0;
+    for (int k = tid; k <= nr; k += TILE_T) {
+      const int64_t p = a.row_ptr[c0 + k];
+      srp[k] = (int32_t)(min(max(p, e0), e1) - e0);
+    }
+    __syncthreads();
+    for (int k0 = warp * G; k0 < nr; k0 += (TILE_T / 32) * G) {  // warp-uniform trip count
+      const int k = k0 + grp;
+      const bool live = k < nr;
+      int lo = live ? srp[k] : 0, hi = live ? srp[k + 1] : 0;
+      if (hi - lo >= TILE_BIG) {  // deferred to the whole CTA
+        if (lig == 0) sbig[atomicAdd(&s_nbig, 1)] = k;
+        hi = lo;
+      }
+      const int64_t row = c0 + k;
+      const float u = hi > lo ? __ldg(a.U + row * a.ldu) : 0.f;
+      if constexpr (!SOFTMAX) {
+        for (int j = lo + lig; j < hi; j += LPG) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
+      } else {
+        // a row of <= RS x LPG entries that no tile boundary cuts stays in registers (one read and
+        // one write of shared memory per entry); longer and cut rows sweep shared memory three times
+        constexpr int RS = 4;
+        const bool fc = first_cut && row == r0, lc = last_cut && row == rlast;
+        const bool reg = hi - lo <= RS * LPG && !(fc || lc);
+        float x[RS];
+        float m = -INFINITY;
+        if (reg) {
+#pragma unroll
+          for (int q = 0; q < RS; ++q) {
+            const int j = lo + q * LPG + lig;
+            x[q] = j < hi ? score1<ADD, LRELU>(u, sv[j], a.scale) : -INFINITY;
+            m = fmaxf(m, x[q]);
+          }
+        } else {
+          for (int j = lo + lig; j < hi; j += LPG) {
+            const float e = score1<ADD, LRELU>(u, sv[j], a.scale);
+            sv[j] = e;
+            m = fmaxf(m, e);
+          }
+        }
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+        float s = 0.f;
+        if (reg) {
+#pragma unroll
+          for (int q = 0; q < RS; ++q) {
+            x[q] = __expf(x[q] - m);  // exp(-inf) = 0 past the row's end
+            s += x[q];
+          }
+        } else {
+          for (int j = lo + lig; j < hi; j += LPG) {
+            const float e = __expf(sv[j] - m);
+            if (!(fc || lc)) sv[j] = e;  // a cut row keeps its scores
+            s += e;
+          }
+        }
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (fc || lc) {
+          if (lig == 0 && hi > lo) {
+            if (fc) a.st_first[t] = make_float2(m, s);
+            if (lc) a.st_last[t] = make_float2(m, s);
+          }
+        } else if (hi > lo) {
+          const float inv = 1.f / s;
+          if (reg) {
+#pragma unroll
+            for (int q = 0; q < RS; ++q) {
+              const int j = lo + q * LPG + lig;
+              if (j < hi) sv[j] = x[q] * inv;
+            }
+          } else {
+            for (int j = lo + lig; j < hi; j += LPG) sv[j] *= inv;
+          }
+        }
+      }
+    }
+    __syncthreads();
+    const int nbig = s_nbig;
+    for (int b = 0; b < nbig; ++b) {  // CTA-uniform
+      const int k = sbig[b], lo = srp[k], hi = srp[k + 1];
+      const int64_t row = c0 + k;
+      const float u = __ldg(a.U + row * a.ldu);
+      if constexpr (!SOFTMAX) {
+        for (int j = lo + tid; j < hi; j += TILE_T) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
+      } else {
+        float m = -INFINITY;
+        for (int j = lo + tid; j < hi; j += TILE_T) {
+          const float x = score1<ADD, LRELU>(u, sv[j], a.scale);
+          sv[j] = x;
+          m = fmaxf(m, x);
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+        if (lane == 0) sred[0][warp] = m;
+        __syncthreads();
+        m = sred[0][0];
+#pragma unroll
+        for (int w = 1; w < TILE_T / 32; ++w) m = fmaxf(m, sred[0][w]);
+        const bool cut = (first_cut && row == r0) || (last_cut && row == rlast);
+        float s = 0.f;
+        for (int j = lo + tid; j < hi; j += TILE_T) {
+          const float x = __expf(sv[j] - m);
+          if (!cut) sv[j] = x;
+          s += x;
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (lane == 0) sred[1][warp] = s;
+        __syncthreads();
+        s = 0.f;
+#pragma unroll
+        for (int w = 0; w < TILE_T / 32; ++w) s += sred[1][w];
+        if (cut) {
+          if (tid == 0) {
+            if (first_cut && row == r0) a.st_first[t] = make_float2(m, s);
+            if (last_cut && row == rlast) a.st_last[t] = make_float2(m, s);
+          }
+        } else {
+          const float inv = 1.f / s;
+          for (int j = lo + tid; j < hi; j += TILE_T) sv[j] *= inv;
+        }
+        __syncthreads();  // sred reused by the next big row
+      }
+    }
+  }
+  __syncthreads();
+  // (C) write the tile back
+  if ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) {
+    for (int j = tid * 4; j < ne; j += TILE_T * 4) {
+      if (j + 3 < ne) st_pol(reinterpret_cast<float4*>(a.out + e0 + j), *reinterpret_cast<const float4*>(sv + j), pol.stream);
+      else
+        for (int r = j; r < ne; ++r) st_pol(a.out + e0 + r, sv[r], pol.stream);
+    }
+  } else {
+    for (int j = tid; j < ne; j += TILE_T) st_pol(a.out + e0 + j, sv[j], pol.stream);
+  }
+}
+
+// crossing rows: the tile a cut row begins in combines the row's in-tile partials in tile order
+// (fixed lane assignment + butterfly) and hands (max, 1/sum) to every tile it touches
+__global__ void k_sddmm1_xstats(TileArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t + 1 < a.n_tiles; t += nwarps) {
+    const int64_t e0 = t * TILE_E, e1 = e0 + TILE_E;
+    const int64_t rl = a.tile_row[t + 1];
+    const int64_t p = a.row_ptr[rl];
+    if (p >= e1 || p < e0) continue;  // no row continues past e1, or it began in an earlier tile
+    const int64_t tb = (a.row_ptr[rl + 1] - 1) / TILE_E;
+    float m = -INFINITY, s = 0.f;
+    for (int64_t q = t + lane; q <= tb; q += 32) {
+      const float2 f = q == t ? a.st_last[t] : a.st_first[q];
+      ms_merge(m, s, f.x, f.y);
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1)
+      ms_merge(m, s, __shfl_xor_sync(0xffffffffu, m, off), __shfl_xor_sync(0xffffffffu, s, off));
+    const float2 fin = make_float2(m, 1.f / s);
+    for (int64_t q = t + lane; q <= tb; q += 32) {
+      if (q == t) a.fin_last[t] = fin;
+      else a.fin_first[q] = fin;
+    }
+  }
+}
+
+__device__ __forceinline__ void xnorm_range(float* __restrict__ out, int64_t lo, int64_t hi, float2 f, int lane) {
+  int64_t j = lo + lane;
+  for (; j + 96 < hi; j += 128) {
+    float x[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) x[q] = out[j + 32 * q];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) out[j + 32 * q] = __expf(x[q] - f.x) * f.y;
+  }
+  for (; j < hi; j += 32) out[j] = __expf(out[j] - f.x) * f.y;
+}
+
+__global__ void k_sddmm1_xnorm(TileArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = warp; t < a.n_tiles; t += nwarps) {
+    const int64_t e0 = t * TILE_E, e1 = min(e0 + (int64_t)TILE_E, a.nnz);
+    const int64_t r0 = a.tile_row[t];
+    if (a.row_ptr[r0] < e0) xnorm_range(a.out, e0, min(a.row_ptr[r0 + 1], e1), a.fin_first[t], lane);
+    if (t + 1 < a.n_tiles) {
+      const int64_t p = a.row_ptr[a.tile_row[t + 1]];
+      if (p < e1 && p >= e0) xnorm_range(a.out, p, e1, a.fin_last[t], lane);
+    }
+  }
+}
+
+// Entry tiles where they measured faster (B200, tools/sddmm_tile_ab.py, profiles/r02/sddmm_tile/): large
+// graphs of moderate degree -- products-shaped (130 M entries, avg 53): normalisation 0.815 -> 0.614 ms,
+// scores + softmax 1.076 -> 0.994 ms.  The degree-ordered kernel keeps dense-degree graphs (Reddit, avg
+// 508: a warp streams one row's sorted columns; 0.472 vs 0.554 ms) and small ones (arxiv: 315 tiles
+// fill two CTAs per SM; 0.015 vs 0.019 ms).  GRANII_SDDMM_TILE=0/1 forces either (A/B runs, tests).
+static bool sddmm_tile_enabled(const granii_graph_s* g) {
+  const char* e = getenv("GRANII_SDDMM_TILE");
+  if (e) return atoi(e) != 0;
+  return g->avg_deg() < 128.f && g->local_nnz >= (16ll << 20);
+}
+
+template <int LPG, bool ADD, bool LR, bool SM>
+static void go_tile(const TileArgs& a, cudaStream_t st) {
+  k_sddmm1_tile<LPG, ADD, LR, SM><<<(unsigned)a.n_tiles, TILE_T, 0, st>>>(a);
+}
+
+template <bool ADD, bool LR, bool SM>
+static void go_tile_lpg(int lpg, const TileArgs& a, cudaStream_t st) {
+  switch (lpg) {
+    case 32: go_tile<32, ADD, LR, SM>(a, st); break;
+    case 16: go_tile<16, ADD, LR, SM>(a, st); break;
+    case 8: go_tile<8, ADD, LR, SM>(a, st); break;
+    default: go_tile<4, ADD, LR, SM>(a, st); break;
+  }
+}
+
+static granii_status launch_sddmm1_tile(const granii_graph_s* g, bool add, bool lr, bool sm, const float* U,
+                                        int64_t ldu, const float* V, int64_t ldv, float scale, float* out, int sms,
+                                        cudaStream_t st) {
+  TileArgs a{g->n_rows, g->local_nnz, g->n_tiles, g->row_ptr, g->col_idx, g->tile_row, U, ldu, V, ldv, scale, out,
+             nullptr, nullptr, nullptr, nullptr, l2hint_enabled()};
+  if (sm) {
+    GR_CUDA(cudaMallocAsync((void**)&a.st_first, 4 * std::max<int64_t>(g->n_tiles, 1) * sizeof(float2), st));
+    a.st_last = a.st_first + g->n_tiles;
+    a.fin_first = a.st_last + g->n_tiles;
+    a.fin_last = a.fin_first + g->n_tiles;
+  }
+  int lpg = sm ? lpg_for_softmax(g->avg_deg()) : lpg_for_degree(g->avg_deg());
+  if (getenv("GRANII_SDDMM_TILE_LPG")) lpg = atoi(getenv("GRANII_SDDMM_TILE_LPG"));  // sweeps
+  if (add) {
+    if (lr) { if (sm) go_tile_lpg<true, true, true>(lpg, a, st); else go_tile_lpg<true, true, false>(lpg, a, st); }
+    else { if (sm) go_tile_lpg<true, false, true>(lpg, a, st); else go_tile_lpg<true, false, false>(lpg, a, st); }
+  } else {
+    if (lr) { if (sm) go_tile_lpg<false, true, true>(lpg, a, st); else go_tile_lpg<false, true, false>(lpg, a, st); }
+    else { if (sm) go_tile_lpg<false, false, true>(lpg, a, st); else go_tile_lpg<false, false, false>(lpg, a, st); }
+  }
+  GR_CHECK_LAUNCH();
+  if (sm) {
+    const unsigned b = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(g->n_tiles, 8), (int64_t)sms * 8));
+    k_sddmm1_xstats<<<b, 256, 0, st>>>(a);
+    k_sddmm1_xnorm<<<b, 256, 0, st>>>(a);
+    GR_CHECK_LAUNCH();
+    GR_CUDA(cudaFreeAsync(a.st_first, st));
+  }
+  return GRANII_OK;
+}
+
 // K > 1 dot: warp per row, LPG lanes per entry, VEC-wide loads, NJ chunks per lane.
 template <int VEC, int LPG, int NJ>
 __global__ void __launch_bounds__(256) k_sddmm_dot(SddmmArgs a) {
@@ -470,8 +811,13 @@ granii_status launch_sddmm(const granii_graph_s* g, uint32_t op, const float* U,
   // algorithmic bytes: per entry col id + V row (4K) + out; per row row_ptr + U row
   const double nnz = (double)g->local_nnz, R = (double)g->n_rows;
   const double gathered = (double)g->n_cols * 4.0 * (double)K;  // V, read once in the compulsory count
-  ProfScope ps("sddmm", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K, (K > 1 && sm) ? 2 : 1,
+  // "sddmm" (K = 1: one 4-byte V gather per entry, bound by the gather rate, bench.py) / "sddmm_dot"
+  ProfScope ps(K == 1 ? "sddmm" : "sddmm_dot", st, nnz * (8.0 + 4.0 * K) + R * (8.0 + 4.0 * K), 2.0 * nnz * K, (K > 1 && sm) ? 2 : 1,
                nnz * 8.0 + R * (8.0 + 4.0 * K) + gathered, gathered <= 0.6 * (double)di.l2_bytes);
+  if (K == 1 && sddmm_tile_enabled(g)) {
+    ps.add_launches(sm ? 2 : 0);
+    return launch_sddmm1_tile(g, base == GRANII_SDDMM_ADD, lr, sm, U, ldu, V, ldv, scale, out, di.sms, st);
+  }
   if (K == 1) {
     const int lpg = sm ? lpg_for_softmax(g->avg_deg()) : lpg_for_degree(g->avg_deg());
     const int64_t units = ceil_div(n_light, 32 / lpg) + g->n_seg;

@@ -281,6 +281,59 @@ def test_sddmm_norm_and_attention(G, name):
     assert err(out.cpu(), O.edge_softmax(c.rp, e), c.rp) <= TOL
 
 
+def _tile_graphs():
+    """graphs for the entry-tile K = 1 SDDMM (tile_e = 4096 entries): a star whose hub row spans
+    several tiles (cut rows combined across tiles), a path-like graph of degree-2 rows (> 512 rows per
+    tile: several row_ptr chunks), an R-MAT graph without self-loops (empty rows inside tiles), and a
+    dense Chung-Lu graph (rows of >= 512 in-tile entries taken by the whole CTA)"""
+    n = 20000
+    hub = torch.zeros(n - 1, dtype=torch.int32)
+    yield "star", n, hub, torch.arange(1, n, dtype=torch.int32), O.ADD_SELF_LOOPS | O.SYMMETRIZE
+    n = 9000
+    a = torch.arange(n - 1, dtype=torch.int32)
+    yield "path", n, a, a + 1, O.SYMMETRIZE
+    n = 6000
+    s, d = synth.rmat(n, 40000, 0.57, 0.19, 0.19, seed=11)
+    yield "rmat_noloops", n, s, d, 0
+    n = 1500
+    s, d = synth.chung_lu(n, 200000, 2.0, seed=12, max_w_frac=0.1)
+    yield "bigrows", n, s, d, O.ADD_SELF_LOOPS | O.SYMMETRIZE
+
+
+@pytest.mark.parametrize("tile", ["1", "0"])
+@pytest.mark.parametrize("gname", ["star", "path", "rmat_noloops", "bigrows"])
+def test_sddmm_entry_tiles(G, gname, tile, monkeypatch):
+    """K = 1 SDDMM over entry tiles (GRANII_SDDMM_TILE=1, the default) and the degree-ordered
+    kernel (0): normalisation scores, GAT scores + row softmax across tile boundaries, and an output
+    buffer that is not 16-byte aligned"""
+    monkeypatch.setenv("GRANII_SDDMM_TILE", tile)
+    n, s, d, flags = next((x[1:] for x in _tile_graphs() if x[0] == gname))
+    g = G.granii_graph_csr_create(n, s.to(DEV).contiguous(), d.to(DEV).contiguous(), flags)
+    rp, ci = O.csr_build(n, s, d, flags)
+    nnz = ci.shape[0]
+    assert nnz > 3 * 4096
+    dinv = O.dinv(rp)
+    buf = torch.zeros(nnz + 1, device=DEV)
+    for out in (buf[:nnz], buf[1:]):
+        dv = torch.tensor(dinv, dtype=torch.float32, device=DEV)
+        G.granii_sddmm(g, G.SDDMM_DOT, dv, 1, dv, 1, 1, 1.0, out)
+        torch.cuda.synchronize()
+        assert err(out.cpu(), O.sddmm(rp, ci, dinv, dinv), rp) <= TOL
+        el = synth.uniform_pm1(34, 1, (n,)) * 4
+        er = synth.uniform_pm1(34, 2, (n,)) * 4
+        G.granii_sddmm(g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el.to(DEV), 1, er.to(DEV), 1, 1,
+                       1.0, out)
+        torch.cuda.synchronize()
+        rows = np.repeat(np.arange(n), np.diff(rp))
+        e = el.numpy().astype(np.float64)[rows] + er.numpy().astype(np.float64)[ci]
+        e = np.where(e > 0, e, 0.2 * e)
+        ref = O.edge_softmax(rp, e)
+        assert err(out.cpu(), ref, rp) <= TOL
+        # every row's alpha sums to one (empty rows have none)
+        sums = np.add.reduceat(out.cpu().numpy().astype(np.float64), rp[:-1][np.diff(rp) > 0])
+        assert np.abs(sums - 1).max() < 1e-5
+
+
 @pytest.mark.parametrize("cap", ["0", "40", "100", "1024"])
 @pytest.mark.parametrize("name", ["dense", "pubmed", "directed"])
 def test_sddmm_softmax_staged_rows(G, name, cap, monkeypatch):
@@ -290,6 +343,7 @@ def test_sddmm_softmax_staged_rows(G, name, cap, monkeypatch):
     same launch) -- bit-for-bit the same alpha as the default staging is not required, the R19
     tolerance against the oracle's edge softmax is"""
     monkeypatch.setenv("GRANII_SDDMM_CAP", cap)
+    monkeypatch.setenv("GRANII_SDDMM_TILE", "0")  # the degree-ordered kernel's staging (tiles: above)
     c = case(G, name)
     n, nnz = c.n, c.ci.shape[0]
     el = synth.uniform_pm1(33, 1, (n,)) * 4

@@ -11,7 +11,7 @@ import json
 import re
 import sys
 
-PRIM = [(r"k_spmm", "spmm"), (r"k_sddmm|k_seg_|k_heavy_stats|k_row_softmax", "sddmm"),
+PRIM = [(r"k_spmm", "spmm"), (r"k_sddmm_dot", "sddmm_dot"), (r"k_sddmm|k_seg_|k_heavy_stats|k_row_softmax", "sddmm"),
         (r"k_gat_bwd_a|k_gat_a_combine", "gat_bwd_a"), (r"k_gat_bwd_b|k_gat_b_combine", "gat_bwd_b"),
         (r"k_gat_dz", "gat_dz"), (r"k_gat_der", "gat_der"),
         (r"k_gemm_tn|k_sum_splits", "gemm_tn_tc"), (r"k_gemm_tc|k_prep_b|k_reduce_partials", "gemm_tc")]
