@@ -22,6 +22,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import shutil
 import statistics
 import subprocess
 import sys
@@ -67,13 +68,60 @@ def peaks():
     return 6650.0, 1590.0, "fallback"
 
 
-class Clocks:
-    """nvidia-smi sampler running during the timed region (B200_PROFILING.md clocks line)."""
+class _NvmlSampler:
+    """NVML fallback of the clocks sampler (boxes without the nvidia-smi binary): SM clock, max SM
+    clock and the clock-event reason bits every 100 ms on a thread, rows shaped like nvidia-smi's"""
 
     def __init__(self, index: int):
-        self.index, self.p = index, None
+        import threading
+
+        import pynvml
+        self.nv = pynvml
+        pynvml.nvmlInit()
+        self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+        self.rows, self.stop = [], threading.Event()
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.t.start()
+
+    def _run(self):
+        nv = self.nv
+        bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+        while not self.stop.is_set():
+            try:
+                sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+                mx = nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM)
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                self.rows.append([str(sm), str(mx), hex(r)] + ["Active" if r & b else "Not Active" for b in bits])
+            except Exception:
+                pass
+            self.stop.wait(0.1)
+
+    def finish(self):
+        self.stop.set()
+        self.t.join(timeout=2)
+        try:
+            self.nv.nvmlShutdown()
+        except Exception:
+            pass
+        return self.rows
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region (B200_PROFILING.md clocks line); NVML
+    (nvidia_ml_py) samples the same fields where the nvidia-smi binary is missing."""
+
+    def __init__(self, index: int):
+        self.index, self.p, self.nvml = index, None, None
 
     def __enter__(self):
+        if not shutil.which("nvidia-smi"):
+            try:
+                self.nvml = _NvmlSampler(self.index)
+            except Exception:
+                self.nvml = None
+            time.sleep(0.15)
+            return self
         q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
              "clocks_event_reasons.sw_power_cap")
@@ -88,6 +136,11 @@ class Clocks:
 
     def __exit__(self, *a):
         self.rows = []
+        if self.nvml is not None:
+            time.sleep(0.15)
+            self.rows = self.nvml.finish()
+            self.source = "nvml"
+            return
         if self.p is None:
             return
         time.sleep(0.15)
@@ -104,13 +157,13 @@ class Clocks:
 
     def summary(self):
         if not getattr(self, "rows", None):
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no clock samples (nvidia-smi and NVML unavailable)"], "samples": 0}
         sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
         mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(self.rows), "source": getattr(self, "source", "nvidia-smi")}
 
 
 MODEL_IDS = {"gcn": 0, "gat": 1, "sgc": 2, "tagcn": 3, "gin": 4}

@@ -130,6 +130,8 @@ struct In {
   double R, nnz, ncols, avg, l2, world, nseg;
   double xcols;  // rows of X an SpMM gathers from (a phased SpMM slices like the whole one: ncols)
   double maxd = 0, seg_len = 2048;  // longest row (featurizer feature 4) and the hub-segment length
+  double xld = 0;  // row stride (floats) of the gathered operand when wider than K (TAGCN's Horner hops
+                   // gather K2 of every (k+1)K2-wide row of P = H[W_0 .. W_k]); 0: = K
 };
 
 static bool overlap_on() {
@@ -141,8 +143,12 @@ static bool overlap_on() {
 // a slice resident when the graph is dense; otherwise LRU-like hit ~ L2 / |X|.
 // (A popularity-weighted variant -- the top-1 % rows' share of the entries held in L2 first --
 // was tried and raised the GAT regret on arxiv-shaped graphs: m5 sweep, 77/79 vs 78/79 within 10 %.)
+// A strided operand (xld > K) spreads the gathered rows over xld / K times the address range: the
+// touched sectors are the same, but their lines / DRAM pages are shared with the unread columns, so
+// the LRU estimate runs over the strided footprint (belgium TAGCN 256->256: the Horner hop over the
+// 768-strided P measured 34 % slower than the plain SpMM at K = 256).
 static double l2_hit(const In& in, double K, double cols) {
-  const double xbytes = cols * K * 4.0;
+  const double xbytes = cols * std::max(K, in.xld) * 4.0;
   if (xbytes <= 0.8 * in.l2) return 1.0;
   if (in.avg >= 32.0 && cols * 64.0 * 4.0 <= 0.55 * in.l2) return 1.0;  // K-sliced
   return std::max(0.0, std::min(1.0, 0.8 * in.l2 / xbytes));
@@ -328,8 +334,11 @@ double ext_forward_cost(const CostModel& m, const In& in, int comp, double K1, d
     }
     t += cost(m, in, P_GEMM, K1, K2) + k * (cost(m, in, P_ALLGATHER, K) + cost(m, in, sp, K));
   } else if (base == GRANII_TAGCN_PRE_AGG) {
-    if (upd)
-      t += cost(m, in, P_GEMM, K1, (k + 1) * K2) + k * (cost(m, in, P_ALLGATHER, K2) + cost(m, in, sp, K2));
+    if (upd) {
+      In h = in;
+      h.xld = (k + 1) * K2;  // Horner: Z = S Z + P_j reads P's j-th K2 block (layer.cu)
+      t += cost(m, in, P_GEMM, K1, (k + 1) * K2) + k * (cost(m, in, P_ALLGATHER, K2) + cost(m, h, sp, K2));
+    }
     else if (dyn && k > 0 && dyn_prescale(in.nnz, in.R, in.avg, in.xcols, (int64_t)K1, (int64_t)in.l2))
       // pre-scaled hop inputs (layer.cu pre_t): a row-broadcast pass before every hop
       t += cost(m, in, P_ELEMENTWISE, K1) * (k + 1) + k * (cost(m, in, P_ALLGATHER, K1) + cost(m, in, P_SPMM_U, K1)) +
@@ -424,7 +433,10 @@ granii_status select_impl(const granii_graph_s* g, granii_model model, const gra
     const int base = model == GRANII_SGC ? GRANII_SGC_PRE_AGG : model == GRANII_TAGCN ? GRANII_TAGCN_PRE_AGG
                                                                                          : GRANII_GIN_PRE_AGG;
     const int64_t Kout = model == GRANII_GIN ? shape->Kh : K2;
-    if (!prefilter) c = {base, base + 1, base + 2, base + 3};
+    // TAGCN at K1 == K2 (reading R28): AGG runs k plain hops at K1 and the (k+1)K1 x K2 GEMM, UPD the
+    // K1 x (k+1)K2 GEMM and k Horner hops with a fused addend over a strided operand -- equal sizes,
+    // different primitives, so the size rule ranks neither and the cost models decide
+    if (!prefilter || (model == GRANII_TAGCN && K1 == Kout)) c = {base, base + 1, base + 2, base + 3};
     else if (K1 >= Kout) c = {base + 1, base + 3};
     else c = {base, base + 2};
   }
