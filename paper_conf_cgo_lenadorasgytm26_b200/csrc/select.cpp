@@ -132,6 +132,7 @@ struct In {
   double maxd = 0, seg_len = 2048;  // longest row (featurizer feature 4) and the hub-segment length
   double xld = 0;  // row stride (floats) of the gathered operand when wider than K (TAGCN's Horner hops
                    // gather K2 of every (k+1)K2-wide row of P = H[W_0 .. W_k]); 0: = K
+  bool addend = false;  // the SpMM's epilogue adds a dense R x K operand (Horner: + P_j), streamed once
 };
 
 static bool overlap_on() {
@@ -188,7 +189,7 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
       // every K slice re-streams the column ids (+ weights) and re-gathers the column scale
       // (a dependent 4-byte gather costs a whole 32-byte L2 sector)
       const double sl = (double)spmm_slices(in.avg, in.xcols, (int64_t)K, (int64_t)in.l2);
-      const double idx = in.nnz * sl * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0)) * gb;
+      const double idx = in.nnz * sl * (4.0 + (p == P_SPMM_W ? 4.0 : 0.0)) * gb + (in.addend ? in.R * K * 4.0 * gb : 0.0);
       return {1.0, idx, in.R * K * 4.0 * gb, gath * h, gath * (1.0 - h), in.R * 1e-6, in.nseg * 1e-3,
               p == P_SPMM_U_CS ? in.nnz * sl * 1e-9 : 0.0};
     }
@@ -337,6 +338,7 @@ double ext_forward_cost(const CostModel& m, const In& in, int comp, double K1, d
     if (upd) {
       In h = in;
       h.xld = (k + 1) * K2;  // Horner: Z = S Z + P_j reads P's j-th K2 block (layer.cu)
+      h.addend = true;
       t += cost(m, in, P_GEMM, K1, (k + 1) * K2) + k * (cost(m, in, P_ALLGATHER, K2) + cost(m, h, sp, K2));
     }
     else if (dyn && k > 0 && dyn_prescale(in.nnz, in.R, in.avg, in.xcols, (int64_t)K1, (int64_t)in.l2))

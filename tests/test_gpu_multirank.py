@@ -152,13 +152,18 @@ def test_gcn_forward_backward_partitioned(G, world, comp, name, K1, K2, phases, 
         assert torch.equal(res[r][2], res[0][2])
 
 
+@pytest.mark.parametrize("tile", ["auto", "1"])
 @pytest.mark.parametrize("phases", ["off", "16"])
 @pytest.mark.parametrize("world", [2, 4])
 @pytest.mark.parametrize("comp", [16, 17])
 @pytest.mark.parametrize("name,K1,K2", [("sparse", 32, 64), ("dense", 48, 16)])
-def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2, phases, monkeypatch):
+def test_gat_forward_backward_partitioned(G, world, comp, name, K1, K2, phases, tile, monkeypatch):
+    """tile = 1 forces the entry-tile K = 1 SDDMM (chosen on its own only for products-sized graphs) over
+    the partitioned graph: local rows, gather-layout column ids, cut rows at tile boundaries"""
     from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
     set_phases(monkeypatch, phases)
+    if tile != "auto":
+        monkeypatch.setenv("GRANII_SDDMM_TILE", tile)
     n, s, d = graph_case(name)
     rp, ci = O.csr_build(n, s, d, F)
     H = synth.features(91, n, K1)

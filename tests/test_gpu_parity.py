@@ -148,7 +148,7 @@ def test_csr_flags_and_edge_cases(G, flags):
 
 
 # ------------------------------------------------------------------ SpMM
-KS = [1, 2, 3, 4, 16, 41, 47, 64, 100, 128, 129, 256, 602, 1024]
+KS = [1, 2, 3, 4, 16, 33, 41, 47, 48, 64, 100, 128, 129, 256, 602, 1024]
 
 
 @pytest.mark.parametrize("name", ["sparse", "dense"])
