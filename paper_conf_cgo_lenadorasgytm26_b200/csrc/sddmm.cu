@@ -315,54 +315,8 @@ struct TileArgs {
   int l2hint;
 };
 
-// (A) a tile's column ids: four coalesced 16-byte streaming loads per thread (warp w: entries
-// [512w, 512w + 512), lane: 4 consecutive entries in each of 4 rounds of 128); past the end: column 0
-__device__ __forceinline__ void tile_cols(const TileArgs& a, int64_t t, int warp, int lane, const L2Pol& pol,
-                                          int32_t (&c)[16]) {
-  const int64_t e0 = t * TILE_E;
-  const int ne = (int)min((int64_t)TILE_E, a.nnz - e0);
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const int j = warp * 512 + q * 128 + lane * 4;
-    if (j + 3 < ne) {
-      const int4 v = ldg_stream(reinterpret_cast<const int4*>(a.col_idx + e0 + j), pol.stream);
-      c[4 * q] = v.x; c[4 * q + 1] = v.y; c[4 * q + 2] = v.z; c[4 * q + 3] = v.w;
-    } else {
-#pragma unroll
-      for (int r = 0; r < 4; ++r) c[4 * q + r] = j + r < ne ? ldg_stream(a.col_idx + e0 + j + r, pol.stream) : 0;
-    }
-  }
-}
-
-// ... its 16 independent V gathers per thread
-__device__ __forceinline__ void tile_gather(const TileArgs& a, const L2Pol& pol, const int32_t (&c)[16],
-                                            float (&v)[16]) {
-#pragma unroll
-  for (int i = 0; i < 16; ++i) v[i] = ldg_pol(a.V + (int64_t)c[i] * a.ldv, pol.keep);
-}
-
-// ... parked in shared memory
-__device__ __forceinline__ void tile_park(const TileArgs& a, int64_t t, int warp, int lane, const float (&v)[16],
-                                          float* sv) {
-  const int ne = (int)min((int64_t)TILE_E, a.nnz - t * TILE_E);
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const int j = warp * 512 + q * 128 + lane * 4;
-    if (j + 3 < ne) {
-      *reinterpret_cast<float4*>(sv + j) = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-    } else {
-#pragma unroll
-      for (int r = 0; r < 4; ++r)
-        if (j + r < ne) sv[j + r] = v[4 * q + r];
-    }
-  }
-}
-
-// Persistent CTAs over the tiles, software-pipelined: the next tile's column loads are issued before this
-// tile's row pass and its V gathers before this tile's write-back, so the gathers (the bound, §5.2) stay in
-// flight while shared memory is worked on.
 template <int LPG, bool ADD, bool LRELU, bool SOFTMAX>
-__global__ void __launch_bounds__(TILE_T, 4) k_sddmm1_tile(TileArgs a) {
+__global__ void __launch_bounds__(TILE_T) k_sddmm1_tile(TileArgs a) {
   __shared__ __align__(16) float sv[TILE_E];
   __shared__ int32_t srp[TILE_RCH + 1];
   __shared__ float sred[2][TILE_T / 32];
@@ -370,170 +324,185 @@ __global__ void __launch_bounds__(TILE_T, 4) k_sddmm1_tile(TileArgs a) {
   __shared__ int s_nbig;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const L2Pol pol = make_l2pol(a.l2hint);
-  int64_t t = blockIdx.x;
-  if (t >= a.n_tiles) return;
-  int32_t c[16];
-  float v[16];
-  tile_cols(a, t, warp, lane, pol, c);
-  tile_gather(a, pol, c, v);
-  for (;;) {
-    __syncthreads();  // the previous tile's write-back has read sv
-    tile_park(a, t, warp, lane, v, sv);
-    const int64_t tn = t + gridDim.x;
-    if (tn < a.n_tiles) tile_cols(a, tn, warp, lane, pol, c);
-    const int64_t e0 = t * TILE_E, e1 = min(e0 + (int64_t)TILE_E, a.nnz);
-    const int ne = (int)(e1 - e0);
-    // (B) rows of the tile
-    const int64_t r0 = a.tile_row[t];
-    const int64_t rend = (t + 1 < a.n_tiles) ? (int64_t)a.tile_row[t + 1] + 1 : a.n_rows;
-    const bool first_cut = SOFTMAX && a.row_ptr[r0] < e0;  // r0 began in an earlier tile
-    const int64_t rlast = rend - 1;                          // holds entry e1 when it continues
-    const bool last_cut = SOFTMAX && t + 1 < a.n_tiles && a.row_ptr[rlast] < e1;
-    constexpr int G = 32 / LPG;
-    const int grp = lane / LPG, lig = lane % LPG;
-    for (int64_t c0 = r0; c0 < rend; c0 += TILE_RCH) {
-      const int nr = (int)min((int64_t)TILE_RCH, rend - c0);
-      __syncthreads();  // sv complete (first chunk) / srp and sbig free (later chunks)
-      if (tid == 0) s_nbig = 0;
-      for (int k = tid; k <= nr; k += TILE_T) {
-        const int64_t p = a.row_ptr[c0 + k];
-        srp[k] = (int32_t)(min(max(p, e0), e1) - e0);
+  const int64_t t = blockIdx.x;
+  const int64_t e0 = t * TILE_E, e1 = min(e0 + (int64_t)TILE_E, a.nnz);
+  const int ne = (int)(e1 - e0);
+  // (A) column ids (coalesced 16-byte streaming loads), then 16 independent V gathers per thread
+  {
+    int32_t c[16];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int j = warp * 512 + q * 128 + lane * 4;
+      if (j + 3 < ne) {
+        const int4 v = ldg_stream(reinterpret_cast<const int4*>(a.col_idx + e0 + j), pol.stream);
+        c[4 * q] = v.x; c[4 * q + 1] = v.y; c[4 * q + 2] = v.z; c[4 * q + 3] = v.w;
+      } else {
+#pragma unroll
+        for (int r = 0; r < 4; ++r) c[4 * q + r] = j + r < ne ? ldg_stream(a.col_idx + e0 + j + r, pol.stream) : 0;
       }
-      __syncthreads();
-      for (int k0 = warp * G; k0 < nr; k0 += (TILE_T / 32) * G) {  // warp-uniform trip count
-        const int k = k0 + grp;
-        const bool live = k < nr;
-        int lo = live ? srp[k] : 0, hi = live ? srp[k + 1] : 0;
-        if (hi - lo >= TILE_BIG) {  // deferred to the whole CTA
-          if (lig == 0) sbig[atomicAdd(&s_nbig, 1)] = k;
-          hi = lo;
-        }
-        const int64_t row = c0 + k;
-        const float u = hi > lo ? __ldg(a.U + row * a.ldu) : 0.f;
-        if constexpr (!SOFTMAX) {
-          for (int j = lo + lig; j < hi; j += LPG) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
+    }
+    float v[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = ldg_pol(a.V + (int64_t)c[i] * a.ldv, pol.keep);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int j = warp * 512 + q * 128 + lane * 4;
+      if (j + 3 < ne) {
+        *reinterpret_cast<float4*>(sv + j) = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+      } else {
+#pragma unroll
+        for (int r = 0; r < 4; ++r)
+          if (j + r < ne) sv[j + r] = v[4 * q + r];
+      }
+    }
+  }
+  // (B) rows of the tile
+  const int64_t r0 = a.tile_row[t];
+  const int64_t rend = (t + 1 < a.n_tiles) ? (int64_t)a.tile_row[t + 1] + 1 : a.n_rows;
+  const bool first_cut = SOFTMAX && a.row_ptr[r0] < e0;  // r0 began in an earlier tile
+  const int64_t rlast = rend - 1;                          // holds entry e1 when it continues
+  const bool last_cut = SOFTMAX && t + 1 < a.n_tiles && a.row_ptr[rlast] < e1;
+  constexpr int G = 32 / LPG;
+  const int grp = lane / LPG, lig = lane % LPG;
+  for (int64_t c0 = r0; c0 < rend; c0 += TILE_RCH) {
+    const int nr = (int)min((int64_t)TILE_RCH, rend - c0);
+    __syncthreads();  // sv complete (first chunk) / srp and sbig free (later chunks)
+    if (tid == 0) s_nbig = 0;
+    for (int k = tid; k <= nr; k += TILE_T) {
+      const int64_t p = a.row_ptr[c0 + k];
+      srp[k] = (int32_t)(min(max(p, e0), e1) - e0);
+    }
+    __syncthreads();
+    for (int k0 = warp * G; k0 < nr; k0 += (TILE_T / 32) * G) {  // warp-uniform trip count
+      const int k = k0 + grp;
+      const bool live = k < nr;
+      int lo = live ? srp[k] : 0, hi = live ? srp[k + 1] : 0;
+      if (hi - lo >= TILE_BIG) {  // deferred to the whole CTA
+        if (lig == 0) sbig[atomicAdd(&s_nbig, 1)] = k;
+        hi = lo;
+      }
+      const int64_t row = c0 + k;
+      const float u = hi > lo ? __ldg(a.U + row * a.ldu) : 0.f;
+      if constexpr (!SOFTMAX) {
+        for (int j = lo + lig; j < hi; j += LPG) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
+      } else {
+        // a row of <= RS x LPG entries that no tile boundary cuts stays in registers (one read and
+        // one write of shared memory per entry); longer and cut rows sweep shared memory three times
+        constexpr int RS = 4;
+        const bool fc = first_cut && row == r0, lc = last_cut && row == rlast;
+        const bool reg = hi - lo <= RS * LPG && !(fc || lc);
+        float x[RS];
+        float m = -INFINITY;
+        if (reg) {
+#pragma unroll
+          for (int q = 0; q < RS; ++q) {
+            const int j = lo + q * LPG + lig;
+            x[q] = j < hi ? score1<ADD, LRELU>(u, sv[j], a.scale) : -INFINITY;
+            m = fmaxf(m, x[q]);
+          }
         } else {
-          // a row of <= RS x LPG entries that no tile boundary cuts stays in registers (one read and
-          // one write of shared memory per entry); longer and cut rows sweep shared memory three times
-          constexpr int RS = 4;
-          const bool fc = first_cut && row == r0, lc = last_cut && row == rlast;
-          const bool reg = hi - lo <= RS * LPG && !(fc || lc);
-          float x[RS];
-          float m = -INFINITY;
+          for (int j = lo + lig; j < hi; j += LPG) {
+            const float e = score1<ADD, LRELU>(u, sv[j], a.scale);
+            sv[j] = e;
+            m = fmaxf(m, e);
+          }
+        }
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+        float s = 0.f;
+        if (reg) {
+#pragma unroll
+          for (int q = 0; q < RS; ++q) {
+            x[q] = __expf(x[q] - m);  // exp(-inf) = 0 past the row's end
+            s += x[q];
+          }
+        } else {
+          for (int j = lo + lig; j < hi; j += LPG) {
+            const float e = __expf(sv[j] - m);
+            if (!(fc || lc)) sv[j] = e;  // a cut row keeps its scores
+            s += e;
+          }
+        }
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (fc || lc) {
+          if (lig == 0 && hi > lo) {
+            if (fc) a.st_first[t] = make_float2(m, s);
+            if (lc) a.st_last[t] = make_float2(m, s);
+          }
+        } else if (hi > lo) {
+          const float inv = 1.f / s;
           if (reg) {
 #pragma unroll
             for (int q = 0; q < RS; ++q) {
               const int j = lo + q * LPG + lig;
-              x[q] = j < hi ? score1<ADD, LRELU>(u, sv[j], a.scale) : -INFINITY;
-              m = fmaxf(m, x[q]);
+              if (j < hi) sv[j] = x[q] * inv;
             }
           } else {
-            for (int j = lo + lig; j < hi; j += LPG) {
-              const float e = score1<ADD, LRELU>(u, sv[j], a.scale);
-              sv[j] = e;
-              m = fmaxf(m, e);
-            }
+            for (int j = lo + lig; j < hi; j += LPG) sv[j] *= inv;
           }
-#pragma unroll
-          for (int off = LPG / 2; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
-          float s = 0.f;
-          if (reg) {
-#pragma unroll
-            for (int q = 0; q < RS; ++q) {
-              x[q] = __expf(x[q] - m);  // exp(-inf) = 0 past the row's end
-              s += x[q];
-            }
-          } else {
-            for (int j = lo + lig; j < hi; j += LPG) {
-              const float e = __expf(sv[j] - m);
-              if (!(fc || lc)) sv[j] = e;  // a cut row keeps its scores
-              s += e;
-            }
-          }
-#pragma unroll
-          for (int off = LPG / 2; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-          if (fc || lc) {
-            if (lig == 0 && hi > lo) {
-              if (fc) a.st_first[t] = make_float2(m, s);
-              if (lc) a.st_last[t] = make_float2(m, s);
-            }
-          } else if (hi > lo) {
-            const float inv = 1.f / s;
-            if (reg) {
-#pragma unroll
-              for (int q = 0; q < RS; ++q) {
-                const int j = lo + q * LPG + lig;
-                if (j < hi) sv[j] = x[q] * inv;
-              }
-            } else {
-              for (int j = lo + lig; j < hi; j += LPG) sv[j] *= inv;
-            }
-          }
-        }
-      }
-      __syncthreads();
-      const int nbig = s_nbig;
-      for (int b = 0; b < nbig; ++b) {  // CTA-uniform
-        const int k = sbig[b], lo = srp[k], hi = srp[k + 1];
-        const int64_t row = c0 + k;
-        const float u = __ldg(a.U + row * a.ldu);
-        if constexpr (!SOFTMAX) {
-          for (int j = lo + tid; j < hi; j += TILE_T) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
-        } else {
-          float m = -INFINITY;
-          for (int j = lo + tid; j < hi; j += TILE_T) {
-            const float x = score1<ADD, LRELU>(u, sv[j], a.scale);
-            sv[j] = x;
-            m = fmaxf(m, x);
-          }
-#pragma unroll
-          for (int off = 16; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
-          if (lane == 0) sred[0][warp] = m;
-          __syncthreads();
-          m = sred[0][0];
-#pragma unroll
-          for (int w = 1; w < TILE_T / 32; ++w) m = fmaxf(m, sred[0][w]);
-          const bool cut = (first_cut && row == r0) || (last_cut && row == rlast);
-          float s = 0.f;
-          for (int j = lo + tid; j < hi; j += TILE_T) {
-            const float x = __expf(sv[j] - m);
-            if (!cut) sv[j] = x;
-            s += x;
-          }
-#pragma unroll
-          for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-          if (lane == 0) sred[1][warp] = s;
-          __syncthreads();
-          s = 0.f;
-#pragma unroll
-          for (int w = 0; w < TILE_T / 32; ++w) s += sred[1][w];
-          if (cut) {
-            if (tid == 0) {
-              if (first_cut && row == r0) a.st_first[t] = make_float2(m, s);
-              if (last_cut && row == rlast) a.st_last[t] = make_float2(m, s);
-            }
-          } else {
-            const float inv = 1.f / s;
-            for (int j = lo + tid; j < hi; j += TILE_T) sv[j] *= inv;
-          }
-          __syncthreads();  // sred reused by the next big row
         }
       }
     }
-    if (tn < a.n_tiles) tile_gather(a, pol, c, v);
     __syncthreads();
-    // (C) write the tile back
-    if ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) {
-      for (int j = tid * 4; j < ne; j += TILE_T * 4) {
-        if (j + 3 < ne) st_pol(reinterpret_cast<float4*>(a.out + e0 + j), *reinterpret_cast<const float4*>(sv + j), pol.stream);
-        else
-          for (int r = j; r < ne; ++r) st_pol(a.out + e0 + r, sv[r], pol.stream);
+    const int nbig = s_nbig;
+    for (int b = 0; b < nbig; ++b) {  // CTA-uniform
+      const int k = sbig[b], lo = srp[k], hi = srp[k + 1];
+      const int64_t row = c0 + k;
+      const float u = __ldg(a.U + row * a.ldu);
+      if constexpr (!SOFTMAX) {
+        for (int j = lo + tid; j < hi; j += TILE_T) sv[j] = score1<ADD, LRELU>(u, sv[j], a.scale);
+      } else {
+        float m = -INFINITY;
+        for (int j = lo + tid; j < hi; j += TILE_T) {
+          const float x = score1<ADD, LRELU>(u, sv[j], a.scale);
+          sv[j] = x;
+          m = fmaxf(m, x);
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+        if (lane == 0) sred[0][warp] = m;
+        __syncthreads();
+        m = sred[0][0];
+#pragma unroll
+        for (int w = 1; w < TILE_T / 32; ++w) m = fmaxf(m, sred[0][w]);
+        const bool cut = (first_cut && row == r0) || (last_cut && row == rlast);
+        float s = 0.f;
+        for (int j = lo + tid; j < hi; j += TILE_T) {
+          const float x = __expf(sv[j] - m);
+          if (!cut) sv[j] = x;
+          s += x;
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (lane == 0) sred[1][warp] = s;
+        __syncthreads();
+        s = 0.f;
+#pragma unroll
+        for (int w = 0; w < TILE_T / 32; ++w) s += sred[1][w];
+        if (cut) {
+          if (tid == 0) {
+            if (first_cut && row == r0) a.st_first[t] = make_float2(m, s);
+            if (last_cut && row == rlast) a.st_last[t] = make_float2(m, s);
+          }
+        } else {
+          const float inv = 1.f / s;
+          for (int j = lo + tid; j < hi; j += TILE_T) sv[j] *= inv;
+        }
+        __syncthreads();  // sred reused by the next big row
       }
-    } else {
-      for (int j = tid; j < ne; j += TILE_T) st_pol(a.out + e0 + j, sv[j], pol.stream);
     }
-    if (tn >= a.n_tiles) break;
-    t = tn;
+  }
+  __syncthreads();
+  // (C) write the tile back
+  if ((reinterpret_cast<uintptr_t>(a.out) & 15) == 0) {
+    for (int j = tid * 4; j < ne; j += TILE_T * 4) {
+      if (j + 3 < ne) st_pol(reinterpret_cast<float4*>(a.out + e0 + j), *reinterpret_cast<const float4*>(sv + j), pol.stream);
+      else
+        for (int r = j; r < ne; ++r) st_pol(a.out + e0 + r, sv[r], pol.stream);
+    }
+  } else {
+    for (int j = tid; j < ne; j += TILE_T) st_pol(a.out + e0 + j, sv[j], pol.stream);
   }
 }
 
@@ -604,18 +573,17 @@ static bool sddmm_tile_enabled(const granii_graph_s* g) {
 }
 
 template <int LPG, bool ADD, bool LR, bool SM>
-static void go_tile(const TileArgs& a, int sms, cudaStream_t st) {
-  const int64_t b = persistent_grid(k_sddmm1_tile<LPG, ADD, LR, SM>, TILE_T, sms, a.n_tiles);
-  k_sddmm1_tile<LPG, ADD, LR, SM><<<(unsigned)b, TILE_T, 0, st>>>(a);
+static void go_tile(const TileArgs& a, cudaStream_t st) {
+  k_sddmm1_tile<LPG, ADD, LR, SM><<<(unsigned)a.n_tiles, TILE_T, 0, st>>>(a);
 }
 
 template <bool ADD, bool LR, bool SM>
-static void go_tile_lpg(int lpg, const TileArgs& a, int sms, cudaStream_t st) {
+static void go_tile_lpg(int lpg, const TileArgs& a, cudaStream_t st) {
   switch (lpg) {
-    case 32: go_tile<32, ADD, LR, SM>(a, sms, st); break;
-    case 16: go_tile<16, ADD, LR, SM>(a, sms, st); break;
-    case 8: go_tile<8, ADD, LR, SM>(a, sms, st); break;
-    default: go_tile<4, ADD, LR, SM>(a, sms, st); break;
+    case 32: go_tile<32, ADD, LR, SM>(a, st); break;
+    case 16: go_tile<16, ADD, LR, SM>(a, st); break;
+    case 8: go_tile<8, ADD, LR, SM>(a, st); break;
+    default: go_tile<4, ADD, LR, SM>(a, st); break;
   }
 }
 
@@ -633,11 +601,11 @@ static granii_status launch_sddmm1_tile(const granii_graph_s* g, bool add, bool 
   int lpg = sm ? lpg_for_softmax(g->avg_deg()) : lpg_for_degree(g->avg_deg());
   if (getenv("GRANII_SDDMM_TILE_LPG")) lpg = atoi(getenv("GRANII_SDDMM_TILE_LPG"));  // sweeps
   if (add) {
-    if (lr) { if (sm) go_tile_lpg<true, true, true>(lpg, a, sms, st); else go_tile_lpg<true, true, false>(lpg, a, sms, st); }
-    else { if (sm) go_tile_lpg<true, false, true>(lpg, a, sms, st); else go_tile_lpg<true, false, false>(lpg, a, sms, st); }
+    if (lr) { if (sm) go_tile_lpg<true, true, true>(lpg, a, st); else go_tile_lpg<true, true, false>(lpg, a, st); }
+    else { if (sm) go_tile_lpg<true, false, true>(lpg, a, st); else go_tile_lpg<true, false, false>(lpg, a, st); }
   } else {
-    if (lr) { if (sm) go_tile_lpg<false, true, true>(lpg, a, sms, st); else go_tile_lpg<false, true, false>(lpg, a, sms, st); }
-    else { if (sm) go_tile_lpg<false, false, true>(lpg, a, sms, st); else go_tile_lpg<false, false, false>(lpg, a, sms, st); }
+    if (lr) { if (sm) go_tile_lpg<false, true, true>(lpg, a, st); else go_tile_lpg<false, true, false>(lpg, a, st); }
+    else { if (sm) go_tile_lpg<false, false, true>(lpg, a, st); else go_tile_lpg<false, false, false>(lpg, a, st); }
   }
   GR_CHECK_LAUNCH();
   if (sm) {

@@ -359,7 +359,7 @@ __device__ __forceinline__ void warp_row(const SpmmArgs& a, int64_t t, int lane,
 template <int VEC, int NJ>
 constexpr int spmm_minb() { return VEC == 4 && NJ <= 2 ? 4 : 3; }
 template <int VEC, int LPG, int NJ>
-constexpr int spmm_unroll() { return VEC == 4 && NJ <= 3 ? 2 : (LPG >= 8 ? 4 : 32 / (32 / LPG)); }
+constexpr int spmm_unroll() { return VEC == 4 && NJ <= 2 ? 2 : (LPG >= 8 ? 4 : 32 / (32 / LPG)); }
 
 template <int VEC, int LPG, int NJ, bool W, bool CS, bool PH, int UU = 0, int MINB = 0, bool ATT = false>
 __global__ void __launch_bounds__(256, MINB > 0 ? MINB : spmm_minb<VEC, NJ>()) k_spmm_warp(SpmmArgs a) {
@@ -553,11 +553,6 @@ static granii_status launch_cfg(const SpmmArgs& a, bool warp_mode, bool w, bool 
   return GRANII_OK;
 }
 
-static bool k48_enabled() {
-  const char* e = getenv("GRANII_SPMM_K48");  // 0: the 64-wide shape for 32 < kw <= 48 (A/B runs)
-  return !e || atoi(e) != 0;
-}
-
 // Pick (VEC, LPG, NJ) for a slice of width kw.  VEC=4 needs 16-byte aligned rows.
 template <bool PH>
 static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, bool w, bool cs, int sms,
@@ -566,11 +561,6 @@ static granii_status launch_slice(const SpmmArgs& a, bool vec4, bool warp_mode, 
   if (vec4) {
     if (kw <= 16) return launch_cfg<4, 4, 1, PH>(a, warp_mode, w, cs, sms, st);
     if (kw <= 32) return launch_cfg<4, 8, 1, PH>(a, warp_mode, w, cs, sms, st);
-    // 32 < kw <= 48 (K = 41 / 47 padded to 44 / 48): 8 groups x 3 float4 -- twice the neighbours per
-    // warp instruction of the 64-wide shape, 92-100 % of the lanes useful instead of 69-75 %
-    // (not the phased kernels: their owner-range bookkeeping spills at the 80-register budget)
-    if constexpr (!PH)
-      if (kw <= 48 && warp_mode && k48_enabled()) return launch_cfg<4, 4, 3, PH>(a, warp_mode, w, cs, sms, st);
     if (kw <= 64) {
       if (warp_mode) return launch_cfg<4, 8, 2, PH>(a, warp_mode, w, cs, sms, st);  // 4 groups x 2 float4
       return launch_cfg<4, 16, 1, PH>(a, warp_mode, w, cs, sms, st);
