@@ -308,7 +308,8 @@ granii_status granii_layer_backward(granii_graph g, granii_model m, granii_compo
 #define GRANII_SELECT_TRAINING 0x2u
 #define GRANII_SELECT_INPUT_LAYER 0x4u
 /* Extension: measured tie-break.  When the two best predictions are within 15 % and the best is
- * below 5 ms (small, latency-bound layers, where the cost models are least accurate), the close
+ * below 10 ms (near-ties the models' ~12 % median error cannot decide, on layers cheap enough to
+ * time once: belgium-shaped TAGCN 256->256 is a 2 % predicted tie at 5.2 ms, 12 % apart measured), the close
  * candidates run once on zero-filled inputs of the layer's shape (forward, + backward with
  * SELECT_TRAINING) on a private stream and the fastest is returned (predicted_ms stays the model's).
  * Allocates and frees device memory, synchronises its own stream.  Ignored on partitioned graphs

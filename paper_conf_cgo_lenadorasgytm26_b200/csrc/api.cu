@@ -99,13 +99,14 @@ static granii_status check_shape(granii_model m, const granii_layer_args* a) {
 
 // ------------------------------------------------------------------ measured tie-break
 // GRANII_SELECT_REFINE (extension): the cost models are least accurate on small, latency-bound
-// layers, where a composition runs in well under a millisecond.  When the two best predictions
+// layers, and a ~12 % median prediction error cannot order near-ties (belgium-shaped TAGCN 256->256:
+// 2 % apart predicted at 5.2 ms, 12 % apart measured).  When the two best predictions
 // are within REFINE_MARGIN of each other and the best is below REFINE_MAX_MS, the close candidates
 // run once on zero-filled inputs of the layer's shape (forward; + backward when training) on a
 // private stream and the fastest measured one is kept.  Single GPU only (a partitioned selection
 // must agree on every rank; it stays model-only there).
 // GRANII_REFINE_MARGIN overrides the margin (tests force every candidate through the timed path with it).
-static constexpr double REFINE_MARGIN = 1.15, REFINE_MAX_MS = 5.0;
+static constexpr double REFINE_MARGIN = 1.15, REFINE_MAX_MS = 10.0;
 static double refine_margin() {
   const char* e = getenv("GRANII_REFINE_MARGIN");
   return e && atof(e) > 1.0 ? atof(e) : REFINE_MARGIN;

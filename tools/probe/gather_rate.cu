@@ -73,6 +73,88 @@ static double best_rate(const float* t, uint32_t T, const int32_t* idx, size_t n
   return best;
 }
 
+// random ROW gathers: a group of LPG lanes reads one random row of W float4 (row = K floats, K = 4W)
+// from a table of T rows that exceeds L2 (the products-shaped operands of the K = 47 / 100 gathers);
+// row ids from a hash, bytes = rows x K x 4 / time: the DRAM roof of gathers with no reuse
+template <int LPG, int W, int UNR>
+__global__ void rows_k(const float4* __restrict__ t, uint32_t T, size_t nrows, float* sink) {
+  const int lane = threadIdx.x & 31, grp = lane / LPG, lig = lane % LPG;
+  const size_t gw = (blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5;
+  const size_t nw = ((size_t)gridDim.x * blockDim.x) >> 5;
+  constexpr int G = 32 / LPG, NJ = (W + LPG - 1) / LPG;
+  float acc = 0.f;
+  for (size_t r0 = gw * G * UNR; r0 < nrows; r0 += nw * G * UNR) {
+    float4 v[UNR][NJ];
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) {
+      const uint32_t row = mix((uint32_t)(r0 + u * G + grp) * 2654435761u + 1u) % T;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const int c = lig + j * LPG;
+        v[u][j] = c < W ? __ldg(t + (size_t)row * W + c) : make_float4(0, 0, 0, 0);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < UNR; ++u)
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) acc += v[u][j].x + v[u][j].y + v[u][j].z + v[u][j].w;
+  }
+  if (acc == 12345.f) *sink = acc;
+}
+
+template <int LPG, int W, int UNR>
+static double row_gbs(const float4* t, uint32_t T, size_t nrows, int bps, float* sink) {
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  rows_k<LPG, W, UNR><<<sms * bps, 256>>>(t, T, nrows, sink);
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  double best = 0;
+  for (int r = 0; r < 5; ++r) {
+    cudaEventRecord(a);
+    rows_k<LPG, W, UNR><<<sms * bps, 256>>>(t, T, nrows, sink);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms;
+    cudaEventElapsedTime(&ms, a, b);
+    const double g = (double)nrows * W * 16 / (ms * 1e-3) / 1e9;
+    if (g > best) best = g;
+  }
+  return best;
+}
+
+template <int LPG, int W>
+static double row_best(const float4* t, uint32_t T, size_t nrows, float* sink, char* cfg) {
+  double best = 0;
+  for (int bps : {4, 8}) {
+    double r;
+    r = row_gbs<LPG, W, 2>(t, T, nrows, bps, sink); if (r > best) { best = r; sprintf(cfg, "%d blocks/SM, %d lanes/row, 2 rows in flight per group", bps, LPG); }
+    r = row_gbs<LPG, W, 4>(t, T, nrows, bps, sink); if (r > best) { best = r; sprintf(cfg, "%d blocks/SM, %d lanes/row, 4 rows in flight per group", bps, LPG); }
+    r = row_gbs<LPG, W, 8>(t, T, nrows, bps, sink); if (r > best) { best = r; sprintf(cfg, "%d blocks/SM, %d lanes/row, 8 rows in flight per group", bps, LPG); }
+  }
+  return best;
+}
+
+static void row_probes() {
+  const uint32_t T = 2449029;  // products-shaped rows
+  float4* t;
+  float* sink;
+  cudaMalloc(&t, (size_t)T * 25 * 16);
+  cudaMalloc(&sink, 4);
+  cudaMemset(t, 0, (size_t)T * 25 * 16);
+  const size_t nrows = 64ull << 20;
+  char c1[128], c2[128], c3[128];
+  const double g48 = row_best<4, 12>(t, T, nrows, sink, c1);
+  const double g48b = row_best<8, 12>(t, T, nrows, sink, c3);
+  const double g100 = row_best<16, 25>(t, T, nrows, sink, c2);
+  printf(", \"row_gathers\": {\"how\": \"64 Mi random rows (hash ids) of K floats from a table of 2,449,029 rows (products-shaped, > L2), a lane group per row with 16-byte loads; GB/s = rows x K x 4 / t, best of 5 over 4/8 blocks/SM x 256 threads and 2/4/8 rows in flight per group\", "
+         "\"K48_gbs\": %.1f, \"K48_cfg\": \"%s\", \"K48_8lanes_gbs\": %.1f, \"K48_8lanes_cfg\": \"%s\", \"K100_gbs\": %.1f, \"K100_cfg\": \"%s\"}",
+         g48, c1, g48b, c3, g100, c2);
+  cudaFree(t);
+  cudaFree(sink);
+}
+
 int main() {
   const size_t n = 128ull << 20;
   const uint32_t Ts[3] = {169343, 232965, 2449029};
@@ -96,7 +178,11 @@ int main() {
            "\"stream_cg_Gps\": %.1f, \"stream_cg_cfg\": \"%s\", \"pure_per_sm_clk_at_max\": %.3f}",
            k ? ", " : "", Ts[k], pure_nc / 1e9, c1, str_nc / 1e9, c2, str_cg / 1e9, c3, pure_nc / (sms * (double)clk * 1e3));
   }
-  printf("], \"sm_clock_max_mhz\": %.0f}\n", clk / 1e3);
+  printf("], \"sm_clock_max_mhz\": %.0f", clk / 1e3);
+  cudaFree(t);
+  cudaFree(idx);
+  row_probes();
+  printf("}\n");
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) { fprintf(stderr, "%s\n", cudaGetErrorString(e)); return 1; }
   return 0;
