@@ -42,31 +42,42 @@ __device__ __forceinline__ float gb_warp_sum(float v) {
 
 // this lane's NJ float4 slices of a K-wide row; columns >= K read as 0
 // (p is 16-byte aligned with a row stride that is a multiple of 4 floats)
+// (K <= 2048: the masks are 32-bit compares -- as int64 they cost a carry chain per element inside
+// the gather loop, ~40 % of pass A's instructions at K = 47)
 template <int LPG, int NJ>
-__device__ __forceinline__ void gb_load_row(const float* __restrict__ p, int lg, int64_t K, float (&v)[NJ][4]) {
+__device__ __forceinline__ void gb_load_row(const float* __restrict__ p, int lg, int64_t K64, float (&v)[NJ][4]) {
+  const int K = (int)K64;
 #pragma unroll
   for (int j = 0; j < NJ; ++j) {
-    const int64_t col = 4 * (int64_t)(lg + j * LPG);
+    const int col = 4 * (lg + j * LPG);
     if (col < K) {
       const float4 t = __ldg(reinterpret_cast<const float4*>(p + col));
+      const int nv = K - col;  // valid elements of this vector (>= 4: all)
       v[j][0] = t.x;
-      v[j][1] = col + 1 < K ? t.y : 0.f;
-      v[j][2] = col + 2 < K ? t.z : 0.f;
-      v[j][3] = col + 3 < K ? t.w : 0.f;
+      v[j][1] = nv > 1 ? t.y : 0.f;
+      v[j][2] = nv > 2 ? t.z : 0.f;
+      v[j][3] = nv > 3 ? t.w : 0.f;
     } else {
       v[j][0] = v[j][1] = v[j][2] = v[j][3] = 0.f;
     }
   }
 }
 
+// row r of a row-major operand: row ids are non-negative int32 and strides < 2^32 floats, so one
+// 32 x 32 -> 64-bit multiply (IMAD.WIDE.U32) gives the exact offset
+__device__ __forceinline__ const float* gb_row(const float* base, int32_t r, int64_t ld) {
+  return base + (uint64_t)(uint32_t)r * (uint32_t)ld;
+}
+
 // K % 4 == 0: the gathered K-wide row without per-element masks -- lanes past the row re-read
 // its last vector (finite data that only ever meets the zeros of the masked register-resident row,
 // or feeds columns that are never stored)
 template <int LPG, int NJ>
-__device__ __forceinline__ void gb_load_row_cl(const float* __restrict__ p, int lg, int64_t K, float (&v)[NJ][4]) {
+__device__ __forceinline__ void gb_load_row_cl(const float* __restrict__ p, int lg, int64_t K64, float (&v)[NJ][4]) {
+  const int K = (int)K64;
 #pragma unroll
   for (int j = 0; j < NJ; ++j) {
-    const int64_t col = 4 * (int64_t)(lg + j * LPG);
+    const int col = 4 * (lg + j * LPG);
     const float4 t = __ldg(reinterpret_cast<const float4*>(p + (col < K ? col : K - 4)));
     v[j][0] = t.x;
     v[j][1] = t.y;
@@ -230,7 +241,7 @@ __device__ __forceinline__ void gat_a_warp_row(const GatBwdArgs& a, int32_t r, i
       }
       float zv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(gb_row(a.Z, j[u], a.ldz), lg, a.K, zv[u]);
       if constexpr (WT) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
@@ -286,7 +297,7 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
   float4 r0 = make_float4(0.f, 0.f, 0.f, 0.f);
   if (b < t) {
     c0 = __ldg(a.col_idx + (b + lane < t ? b + lane : t - 1));
-    r0 = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)c0 * a.ldx + a.rec));
+    r0 = __ldg(reinterpret_cast<const float4*>(gb_row(a.dX, c0, a.ldx) + a.rec));
     if (b + 32 < t) c1 = __ldg(a.col_idx + (b + 32 + lane < t ? b + 32 + lane : t - 1));
   }
   for (int64_t base = b; base < t; base += 32) {
@@ -294,7 +305,7 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
     const float4 rc = r0;
     if (base + 32 < t) {  // distance-2 prefetch of the columns, distance 1 of their records
       c0 = c1;
-      r0 = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)c0 * a.ldx + a.rec));
+      r0 = __ldg(reinterpret_cast<const float4*>(gb_row(a.dX, c0, a.ldx) + a.rec));
       if (base + 64 < t) c1 = __ldg(a.col_idx + (base + 64 + lane < t ? base + 64 + lane : t - 1));
     }
     const int cnt = (int)(t - base < 32 ? t - base : 32);
@@ -315,7 +326,7 @@ __device__ __forceinline__ void gat_b_warp_row(const GatBwdArgs& a, int32_t r, i
       }
       float xv[U][NJ][4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+      for (int u = 0; u < U; ++u) gb_gather_row<LPG, NJ, CL>(gb_row(a.dX, i[u], a.ldx), lg, a.K, xv[u]);
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         dpart = fmaf(su[u], gb_pdot<NJ>(xv[u], zr), dpart);
@@ -396,7 +407,7 @@ __device__ __forceinline__ void gat_a_group_row(const GatBwdArgs& a, int64_t t0,
     for (int u = 0; u < U; ++u) {
       j[u] = __ldg(a.col_idx + (e + u < t ? e + u : t - 1));
       erj[u] = __ldg(a.er + j[u]);
-      gb_load_row<LPG, NJ>(a.Z + (int64_t)j[u] * a.ldz, lg, a.K, zv[u]);
+      gb_load_row<LPG, NJ>(gb_row(a.Z, j[u], a.ldz), lg, a.K, zv[u]);
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -458,8 +469,8 @@ __device__ __forceinline__ void gat_b_group_row(const GatBwdArgs& a, int64_t t0,
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       i[u] = __ldg(a.col_idx + (e + u < t ? e + u : t - 1));
-      st[u] = __ldg(reinterpret_cast<const float4*>(a.dX + (int64_t)i[u] * a.ldx + a.rec));
-      gb_load_row<LPG, NJ>(a.dX + (int64_t)i[u] * a.ldx, lg, a.K, xv[u]);
+      st[u] = __ldg(reinterpret_cast<const float4*>(gb_row(a.dX, i[u], a.ldx) + a.rec));
+      gb_load_row<LPG, NJ>(gb_row(a.dX, i[u], a.ldx), lg, a.K, xv[u]);
     }
 #pragma unroll
     for (int u = 0; u < U; ++u) {
