@@ -316,6 +316,17 @@ def gather_peak():
     return max(r["stream_nc_Gps"] for r in json.load(open(gp))["rows"]) * 1e9
 
 
+def row_gather_peak():
+    """GB/s of random K-float row gathers from a products-sized table (> L2) measured by
+    tools/probe/gather_rate.cu (profiles/gather_rate.json row_gathers): the DRAM roof of a gather with no
+    reuse -- the best of its K = 48 / 100 shapes; not a driver measurement"""
+    gp = os.path.join(ROOT, "profiles", "gather_rate.json")
+    if not os.path.exists(gp):
+        return None
+    rg = json.load(open(gp)).get("row_gathers")
+    return max(rg["K48_gbs"], rg["K48_8lanes_gbs"], rg["K100_gbs"]) if rg else None
+
+
 def l2_peak():
     """L2 -> SM read bandwidth measured by tools/probe/l2_bw.cu on B200 (profiles/l2_peak.json);
     not a driver measurement -- the line says so where it is used"""
@@ -366,6 +377,12 @@ def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
             # algorithmic bytes cannot tell -- the binding roof is the DRAM traffic ncu measured
             out.update(bound="hbm", achieved=traffic / (st["ms"] / calls / 1e3) / 1e9, peak=hbm, unit="GB/s",
                        peak_note=f"hbm_gbs of {peak_src}: ncu DRAM bytes per call / t (operand exceeds L2)")
+        elif st.get("l2_resident", 0) < calls and row_gather_peak() and name != "sddmm":
+            # operand beyond L2 and no ncu traffic for this workload: the gathered rows against the
+            # measured random-row DRAM rate (no reuse assumed, so L2 hits can lift frac above 1)
+            out.update(bound="row_gather", achieved=by / t / 1e9, peak=row_gather_peak(), unit="GB/s",
+                       peak_note="random-row gather rate from a table > L2 measured by tools/probe/gather_rate.cu "
+                                 "(profiles/gather_rate.json row_gathers), not a driver figure: algorithmic bytes / t")
         elif t_l2 >= t_hbm:
             out.update(bound="l2", achieved=by / t / 1e9, peak=l2, unit="GB/s",
                        peak_note="L2 read peak measured by tools/probe/l2_bw.cu (profiles/l2_peak.json), "
@@ -374,6 +391,10 @@ def primitive_roofline(name, st, hbm, tc_peak, peak_src, l2, traffic=None):
             out.update(bound="hbm", achieved=comp / t / 1e9, peak=hbm, unit="GB/s",
                        peak_note=f"hbm_gbs of {peak_src}: compulsory bytes / t")
         out["gathered"] = {"bytes_per_call": by / calls, "gbs": by / t / 1e9, "frac_l2": by / t / 1e9 / l2}
+        rp = row_gather_peak()
+        if rp and name != "sddmm" and st.get("l2_resident", 0) < calls:
+            # operand beyond L2: the algorithmic (gathered) bytes against the measured random-row rate
+            out["gathered"].update(frac_row_gather=by / t / 1e9 / rp, row_gather_peak_gbs=rp)
         out["l2_resident_calls"] = st.get("l2_resident", 0)
     else:
         out.update(bound="hbm", achieved=by / t / 1e9, peak=hbm, unit="GB/s", peak_note=f"hbm_gbs of {peak_src}")
