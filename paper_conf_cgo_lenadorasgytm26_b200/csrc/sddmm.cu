@@ -590,6 +590,7 @@ static void go_tile_lpg(int lpg, const TileArgs& a, cudaStream_t st) {
 static granii_status launch_sddmm1_tile(const granii_graph_s* g, bool add, bool lr, bool sm, const float* U,
                                         int64_t ldu, const float* V, int64_t ldv, float scale, float* out, int sms,
                                         cudaStream_t st) {
+  if (g->n_tiles == 0) return GRANII_OK;  // no stored entries
   TileArgs a{g->n_rows, g->local_nnz, g->n_tiles, g->row_ptr, g->col_idx, g->tile_row, U, ldu, V, ldv, scale, out,
              nullptr, nullptr, nullptr, nullptr, l2hint_enabled()};
   if (sm) {

@@ -197,3 +197,39 @@ def test_products_gat_training_fullsize(G, layer):
         else:
             y = y.cpu().numpy()
         assert gat_grad_ok(y, r, m), (G.COMP_NAMES[L.comp], nm)
+
+
+def test_products_sddmm_entry_tiles_fullsize(G):
+    """C5 K = 1 SDDMM at full size: the products-shaped graph (130 M stored entries) is where the
+    entry-tile kernel is chosen (average degree < 128, >= 16 Mi entries).  Normalisation
+    scores Ñ = D̃^-½ Ã D̃^-½ (Eq. 3) and the GAT scores + row softmax (Eq. 4, reading R8) on 4,096 random
+    + 64 hub rows -- the hubs span many 4096-entry tiles, so their softmax goes through the cut-row
+    combine -- against oracle_sddmm / oracle_edge_softmax over the sampled rows' CSR."""
+    w, g, rp, ci = build(G, "products")
+    rows = sample_rows(rp, seed=3)
+    deg = np.diff(rp)
+    assert deg[rows].max() > 3 * 4096       # a hub of the sample crosses several tiles
+    srp = np.concatenate([[0], np.cumsum(deg[rows])]).astype(np.int64)
+    sel = np.concatenate([np.arange(rp[r], rp[r + 1]) for r in rows])
+    sci = ci[sel]
+    dinv = O.dinv(rp)
+    dv = torch.tensor(dinv, dtype=torch.float32, device=DEV)
+    out = torch.empty(g.nnz, device=DEV)
+    G.granii_sddmm(g, G.SDDMM_DOT, dv, 1, dv, 1, 1, 1.0, out)
+    torch.cuda.synchronize()
+    got = out.cpu().numpy()[sel]
+    ref = O.sddmm(srp, sci, dinv[rows], dinv)
+    assert float(np.max(np.abs(got - ref) / np.abs(ref))) <= TOL
+    el = synth.uniform_pm1(35, 1, (w.n,)) * 4
+    er = synth.uniform_pm1(35, 2, (w.n,)) * 4
+    G.granii_sddmm(g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, el.to(DEV), 1, er.to(DEV), 1, 1, 1.0,
+                   out)
+    torch.cuda.synchronize()
+    got = out.cpu().numpy()[sel].astype(np.float64)
+    e = np.repeat(el.numpy().astype(np.float64)[rows], deg[rows]) + er.numpy().astype(np.float64)[sci]
+    ref = O.edge_softmax(srp, np.where(e > 0, e, 0.2 * e))
+    d = np.maximum.reduceat(np.abs(got - ref), srp[:-1])
+    a = np.maximum.reduceat(np.abs(ref), srp[:-1])
+    assert float(np.max(d / a)) <= TOL
+    sums = np.add.reduceat(got, srp[:-1])
+    assert np.abs(sums - 1).max() < 1e-5

@@ -334,6 +334,20 @@ def test_sddmm_entry_tiles(G, gname, tile, monkeypatch):
         assert np.abs(sums - 1).max() < 1e-5
 
 
+@pytest.mark.parametrize("tile", ["1", "0"])
+def test_sddmm_no_entries(G, tile, monkeypatch):
+    """a graph with rows but no stored entries (no edges, no self-loops): both K = 1 kernels are no-ops"""
+    monkeypatch.setenv("GRANII_SDDMM_TILE", tile)
+    e = torch.zeros(0, dtype=torch.int32, device=DEV)
+    g = G.granii_graph_csr_create(7, e, e, 0)
+    v = torch.ones(7, device=DEV)
+    out = torch.zeros(1, device=DEV)
+    G.granii_sddmm(g, G.SDDMM_ADD | G.SDDMM_LEAKYRELU | G.SDDMM_ROW_SOFTMAX, v, 1, v, 1, 1, 1.0, out)
+    G.granii_sddmm(g, G.SDDMM_DOT, v, 1, v, 1, 1, 1.0, out)
+    torch.cuda.synchronize()
+    assert out.item() == 0.0
+
+
 @pytest.mark.parametrize("cap", ["0", "40", "100", "1024"])
 @pytest.mark.parametrize("name", ["dense", "pubmed", "directed"])
 def test_sddmm_softmax_staged_rows(G, name, cap, monkeypatch):
