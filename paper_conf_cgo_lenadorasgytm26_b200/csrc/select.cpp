@@ -41,9 +41,9 @@ struct CostModel {
 //                      G column-scale gathers (one dependent 4-byte gather per entry and K slice)]
 //   sddmm1          : [1, streamed GB, M rows]
 //   sddmm1_softmax  : [1, streamed GB, M rows]
-//   gemm            : [1, HBM GB, TFLOP, thousands of 128x128 tiles]
-//   gemm_att        : [1, HBM GB, TFLOP, thousands of tiles, attention GEMV GB (M x K2 x 4)]
-//   gemm_tn         : [1, HBM GB, TFLOP, thousands of tiles]
+//   gemm            : [1, HBM GB, TFLOP, thousands of 128x128 tiles, roofline ms]
+//   gemm_att        : [1, HBM GB, TFLOP, thousands of tiles, attention GEMV GB (M x K2 x 4), roofline ms]
+//   gemm_tn         : [1, HBM GB, TFLOP, thousands of tiles, roofline ms]
 //   gat_bwd_a/b     : [1, streamed GB (idx, er / row records), row GB, gathered GB from L2,
 //                      gathered GB from HBM, M rows, M dependent gather steps]  (gat_bwd.cu)
 //   elementwise     : [1, GB]
@@ -57,9 +57,9 @@ static CostModel defaults() {
   m.coef["spmm"] = {0.006, 1.0 / 6.0, 1.0 / 6.0, 1.0 / 19.0, 1.0 / 5.0, 0.0, 0.0, 1.0};
   m.coef["sddmm1"] = {0.005, 1.0 / 5.5, 0.0};
   m.coef["sddmm1_softmax"] = {0.006, 1.0 / 4.0, 0.0};
-  m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0};
-  m.coef["gemm_att"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 1.0 / 3.0};
-  m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0};
+  m.coef["gemm"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 0.0};
+  m.coef["gemm_att"] = {0.010, 1.0 / 3.0, 1.0 / 600.0, 0.0, 1.0 / 3.0, 0.0};
+  m.coef["gemm_tn"] = {0.015, 1.0 / 3.0, 1.0 / 300.0, 0.0, 0.0};
   m.coef["gat_bwd_a"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   m.coef["gat_bwd_b"] = {0.008, 1.0 / 5.0, 1.0 / 5.0, 1.0 / 15.0, 1.0 / 4.0, 0.0, 0.0};
   // der only (RECOMP input layer): streamed column ids + entry map, one 32-byte sector per dα gather
@@ -180,6 +180,10 @@ static const char* prim_model(int p, const In& in) {
   return "";
 }
 
+static double gemm_roof_ms(double hbm_gb, double tflop) {
+  return std::max(hbm_gb / 6.53, tflop * 3.0 / 0.705);
+}
+
 // K = width of the primitive (SpMM/SDDMM) or (K1, K2) for the GEMMs
 static std::vector<double> features(const In& in, int p, double K1, double K2) {
   const double gb = 1e-9;
@@ -195,18 +199,28 @@ static std::vector<double> features(const In& in, int p, double K1, double K2) {
     }
     case P_SDDMM1: return {1.0, in.nnz * 8.0 * gb, in.R * 1e-6};
     case P_SDDMM1_SM: return {1.0, in.nnz * 16.0 * gb, in.R * 1e-6};
-    case P_GEMM:
-      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
-              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
-    case P_GEMM_ATT:  // GAT Θ = H W with the el / er GEMVs in the epilogue, Θ stored
-      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
-              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb};
-    case P_GEMM_NOSTORE:  // el / er only, Θ never written
-      return {1.0, in.R * K1 * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
-              std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb};
-    case P_GEMM_TN:
-      return {1.0, in.R * (K1 + K2) * 4.0 * gb, 2.0 * in.R * K1 * K2 * 1e-12,
-              std::ceil(K1 / 128.0) * std::ceil(K2 / 128.0) * 1e-3};
+    // GEMMs: the last feature is the roofline time max(HBM GB / 6.53 TB/s, 3xTF32 TFLOP at the tf32 half of
+    // the measured 1410 TF/s bf16) in ms -- a tall-skinny GEMM is bound by one or the other, which a sum of
+    // the byte and flop terms alone cannot express (arxiv GAT 256->512: the el / er-only GEMM that never
+    // stores Θ is no faster than the one that does -- it is tensor-bound)
+    case P_GEMM: {
+      const double hb = in.R * (K1 + K2) * 4.0 * gb, tf = 2.0 * in.R * K1 * K2 * 1e-12;
+      return {1.0, hb, tf, std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, gemm_roof_ms(hb, tf)};
+    }
+    case P_GEMM_ATT: {  // GAT Θ = H W with the el / er GEMVs in the epilogue, Θ stored
+      const double hb = in.R * (K1 + K2) * 4.0 * gb, tf = 2.0 * in.R * K1 * K2 * 1e-12;
+      return {1.0, hb, tf, std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb,
+              gemm_roof_ms(hb, tf)};
+    }
+    case P_GEMM_NOSTORE: {  // el / er only, Θ never written
+      const double hb = in.R * K1 * 4.0 * gb, tf = 2.0 * in.R * K1 * K2 * 1e-12;
+      return {1.0, hb, tf, std::ceil(in.R / 128.0) * std::ceil(K2 / 128.0) * 1e-3, in.R * K2 * 4.0 * gb,
+              gemm_roof_ms(hb, tf)};
+    }
+    case P_GEMM_TN: {
+      const double hb = in.R * (K1 + K2) * 4.0 * gb, tf = 2.0 * in.R * K1 * K2 * 1e-12;
+      return {1.0, hb, tf, std::ceil(K1 / 128.0) * std::ceil(K2 / 128.0) * 1e-3, gemm_roof_ms(hb, tf)};
+    }
     case P_GAT_BWD_A: case P_GAT_BWD_B: {
       const double K = K1, gath = in.nnz * K * 4.0 * gb, h = l2_hit(in, K, in.ncols);
       const double idx = in.nnz * (p == P_GAT_BWD_A ? 8.0 : 20.0) * gb;

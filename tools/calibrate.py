@@ -175,6 +175,19 @@ def fit(samples):
     return coefs, report
 
 
+GEMM_FEATS = {"gemm": 4, "gemm_att": 5, "gemm_tn": 4}  # feature counts before the roofline-time feature
+
+
+def augment(samples):
+    """samples measured before the GEMM models' roofline-time feature (select.cpp gemm_roof_ms): append
+    max(HBM GB / 6.53, TFLOP x 3 / 0.705) computed from the sample's own HBM GB and TFLOP features"""
+    for s in samples:
+        n = GEMM_FEATS.get(s["model"])
+        if n is not None and len(s["f"]) == n:
+            s["f"] = list(s["f"]) + [max(s["f"][1] / 6.53, s["f"][2] * 3.0 / 0.705)]
+    return samples
+
+
 def relabel(samples):
     """model keys of samples taken before the warp-per-row / group-per-row split (select.cpp
     group_mode: average degree < 16): the graph's average degree from its K = 16 unweighted SpMM
@@ -196,7 +209,7 @@ def main():
     ap.add_argument("--refit", default=None, help="refit from a saved *_samples.json instead of measuring")
     args = ap.parse_args()
     t0 = time.time()
-    samples = relabel(json.load(open(args.refit))["samples"]) if args.refit else sweep(args.quick)
+    samples = augment(relabel(json.load(open(args.refit))["samples"])) if args.refit else sweep(args.quick)
     coefs, report = fit(samples)
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
