@@ -1001,33 +1001,111 @@ __global__ void k_colreduce2(int64_t R, int64_t K, const float* __restrict__ H, 
   }
 }
 
-// out[i] + out[n + i] = the fp64 sum as a float pair (hi, lo): Wᵀ·(Hᵀ del) cancels, and rounding
-// Hᵀ del to fp32 before that product cost da_l 3e-4 normwise at products scale (DESIGN R22); the pair
-// travels through the fp32 all-reduce of several GPUs as two float sums
-__global__ void k_sum_chunks(int64_t n, int64_t S, const double* __restrict__ partial, float* __restrict__ out) {
-  const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  double a = 0.0;
-  for (int64_t s = 0; s < S; ++s) a += partial[s * n + i];
-  const float hi = (float)a;
-  out[i] = hi;
-  out[n + i] = (float)(a - (double)hi);
+// 16-byte rows (ldh % 4 == 0, H aligned): a thread owns 4 adjacent columns (a warp 128), eight rows in
+// flight per thread -- 16 KB of H in flight per CTA instead of 2 KB (products K = 100: 0.67 -> see DESIGN
+// §5.5).  Columns past K read the row's padding, which only ever feeds columns that are never stored.
+__global__ void __launch_bounds__(256) k_colreduce2v(int64_t R, int64_t K, const float* __restrict__ H, int64_t ldh,
+                                                     const float* __restrict__ d0, const float* __restrict__ d1,
+                                                     int64_t chunk, double* __restrict__ partial) {
+  __shared__ double sp[8][129], sq[8][129];
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int64_t c4 = blockIdx.x * 128 + 4 * tx, s = blockIdx.y;
+  const int64_t r0 = s * chunk, r1 = (r0 + chunk < R) ? r0 + chunk : R;
+  double p[4] = {0.0, 0.0, 0.0, 0.0}, q[4] = {0.0, 0.0, 0.0, 0.0};
+  if (c4 < K) {
+    int64_t r = r0 + ty;
+    constexpr int UN = 8;
+    for (; r + 8 * (UN - 1) < r1; r += 8 * UN) {  // UN rows in flight per thread, summed in row order
+      float4 h[UN];
+      float a0[UN], a1[UN];
+#pragma unroll
+      for (int u = 0; u < UN; ++u) {
+        h[u] = __ldg(reinterpret_cast<const float4*>(H + (r + 8 * u) * ldh + c4));
+        a0[u] = __ldg(d0 + r + 8 * u);
+        a1[u] = __ldg(d1 + r + 8 * u);
+      }
+#pragma unroll
+      for (int u = 0; u < UN; ++u) {
+        const float hv[4] = {h[u].x, h[u].y, h[u].z, h[u].w};
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          p[j] = fma((double)hv[j], (double)a0[u], p[j]);
+          q[j] = fma((double)hv[j], (double)a1[u], q[j]);
+        }
+      }
+    }
+    for (; r < r1; r += 8) {
+      const float4 h = __ldg(reinterpret_cast<const float4*>(H + r * ldh + c4));
+      const float hv[4] = {h.x, h.y, h.z, h.w};
+      const double a = __ldg(d0 + r), b = __ldg(d1 + r);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        p[j] = fma((double)hv[j], a, p[j]);
+        q[j] = fma((double)hv[j], b, q[j]);
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    sp[ty][4 * tx + j] = p[j];
+    sq[ty][4 * tx + j] = q[j];
+  }
+  __syncthreads();
+  // 256 threads write the tile's 128 columns x (p, q): fixed-order sum over the 8 row groups
+  const int c = threadIdx.y * 32 + threadIdx.x;  // 0 .. 255
+  const int col = c & 127, which = c >> 7;
+  const int64_t gc = blockIdx.x * 128 + col;
+  if (gc < K) {
+    double a = 0.0;
+#pragma unroll
+    for (int y = 0; y < 8; ++y) a += which ? sq[y][col] : sp[y][col];
+    partial[(s * 2 + which) * K + gc] = a;
+  }
 }
 
-static int64_t colreduce_chunks(int64_t R, int64_t K) {
-  const int64_t tiles = ceil_div(K, 32);
+// out[i] + out[n + i] = the fp64 sum as a float pair (hi, lo): Wᵀ·(Hᵀ del) cancels, and rounding
+// Hᵀ del to fp32 before that product cost da_l 3e-4 normwise at products scale (DESIGN R22); the pair
+// travels through the fp32 all-reduce of several GPUs as two float sums.  A warp per output: lanes take
+// the chunks s = lane, lane + 32, ... in order, then a fixed xor butterfly (was a thread per output
+// walking all S chunks serially).
+__global__ void k_sum_chunks(int64_t n, int64_t S, const double* __restrict__ partial, float* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  if (i >= n) return;
+  double a = 0.0;
+  for (int64_t s = lane; s < S; s += 32) a += partial[s * n + i];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+  if (lane == 0) {
+    const float hi = (float)a;
+    out[i] = hi;
+    out[n + i] = (float)(a - (double)hi);
+  }
+}
+
+static bool colreduce_vec(int64_t ldh, const float* H) { return ldh % 4 == 0 && ((uintptr_t)H & 15) == 0; }
+
+static int64_t colreduce_chunks(int64_t R, int64_t K, bool vec = false) {
+  const int64_t tiles = ceil_div(K, vec ? 128 : 32);
   return std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, 512), ceil_div(148 * 8, tiles)));
 }
 
-size_t colreduce2_workspace(int64_t R, int64_t K) { return (size_t)colreduce_chunks(R, K) * 2 * K * sizeof(double); }
+size_t colreduce2_workspace(int64_t R, int64_t K) {
+  return (size_t)std::max(colreduce_chunks(R, K), colreduce_chunks(R, K, true)) * 2 * K * sizeof(double);
+}
 
 granii_status launch_colreduce2(int64_t R, int64_t K, const float* H, int64_t ldh, const float* d0, const float* d1,
                                 float* partial, float* out, cudaStream_t st) {
-  const int64_t S = colreduce_chunks(R, K), chunk = ceil_div(std::max<int64_t>(R, 1), S);
+  const bool vec = colreduce_vec(ldh, H);
+  const int64_t S = colreduce_chunks(R, K, vec), chunk = ceil_div(std::max<int64_t>(R, 1), S);
   ProfScope ps("elementwise", st, 4.0 * R * K + 8.0 * R, 4.0 * R * K, 2);
-  k_colreduce2<<<dim3((unsigned)ceil_div(K, 32), (unsigned)S), dim3(32, 8), 0, st>>>(R, K, H, ldh, d0, d1, chunk,
-                                                                                   reinterpret_cast<double*>(partial));
-  k_sum_chunks<<<(unsigned)ceil_div(2 * K, 256), 256, 0, st>>>(2 * K, S, reinterpret_cast<const double*>(partial), out);  // 4K floats
+  if (vec)
+    k_colreduce2v<<<dim3((unsigned)ceil_div(K, 128), (unsigned)S), dim3(32, 8), 0, st>>>(
+        R, K, H, ldh, d0, d1, chunk, reinterpret_cast<double*>(partial));
+  else
+    k_colreduce2<<<dim3((unsigned)ceil_div(K, 32), (unsigned)S), dim3(32, 8), 0, st>>>(R, K, H, ldh, d0, d1, chunk,
+                                                                                     reinterpret_cast<double*>(partial));
+  k_sum_chunks<<<(unsigned)ceil_div(2 * K * 32, 256), 256, 0, st>>>(2 * K, S, reinterpret_cast<const double*>(partial), out);  // 4K floats
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
@@ -1052,20 +1130,37 @@ __global__ void k_matvec2(int64_t K1, int64_t K2, const float* __restrict__ W, c
   }
 }
 
-// da_l = Wᵀ p, da_r = Wᵀ q (thread per column of W, fixed order over rows), in fp64 from the
+// da_l = Wᵀ p, da_r = Wᵀ q (fixed order over rows and row groups), in fp64 from the
 // (hi, lo) pairs of p = [p | q | p_lo | q_lo] (k_sum_chunks): the sum cancels
-__global__ void k_mattvec2(int64_t K1, int64_t K2, const float* __restrict__ W, const float* __restrict__ pq,
-                           float* __restrict__ dal, float* __restrict__ dar) {
-  const int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (k >= K2) return;
+// 32 columns x 8 row groups per CTA (rows r = ty, ty + 8, ...), fp64 partials combined in fixed order
+// (was a thread per column walking all K1 rows: ~90 us on two CTAs for 128 x 256)
+__global__ void __launch_bounds__(256) k_mattvec2(int64_t K1, int64_t K2, const float* __restrict__ W,
+                                                  const float* __restrict__ pq, float* __restrict__ dal,
+                                                  float* __restrict__ dar) {
+  __shared__ double sa[8][33], sb[8][33];
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int64_t k = blockIdx.x * 32 + tx;
   double a = 0.0, b = 0.0;
-  for (int64_t r = 0; r < K1; ++r) {
-    const double x = W[r * K2 + k];
-    a = fma(x, (double)pq[r] + (double)pq[2 * K1 + r], a);
-    b = fma(x, (double)pq[K1 + r] + (double)pq[3 * K1 + r], b);
+  if (k < K2) {
+    for (int64_t r = ty; r < K1; r += 8) {
+      const double x = W[r * K2 + k];
+      a = fma(x, (double)pq[r] + (double)pq[2 * K1 + r], a);
+      b = fma(x, (double)pq[K1 + r] + (double)pq[3 * K1 + r], b);
+    }
   }
-  if (dal) dal[k] = (float)a;
-  if (dar) dar[k] = (float)b;
+  sa[ty][tx] = a;
+  sb[ty][tx] = b;
+  __syncthreads();
+  if (ty == 0 && k < K2) {
+    double x = 0.0, y = 0.0;
+#pragma unroll
+    for (int g = 0; g < 8; ++g) {
+      x += sa[g][tx];
+      y += sb[g][tx];
+    }
+    if (dal) dal[k] = (float)x;
+    if (dar) dar[k] = (float)y;
+  }
 }
 
 // dW += p a_lᵀ + q a_rᵀ (p, q from their (hi, lo) pairs)
@@ -1089,7 +1184,7 @@ granii_status launch_gat_matvec2(int64_t K1, int64_t K2, const float* W, const f
 granii_status launch_gat_mattvec2(int64_t K1, int64_t K2, const float* W, const float* pq, float* da_l, float* da_r,
                                   cudaStream_t st) {
   ProfScope ps("elementwise", st, 4.0 * K1 * K2, 4.0 * K1 * K2, 1);
-  k_mattvec2<<<(unsigned)ceil_div(K2, 128), 128, 0, st>>>(K1, K2, W, pq, da_l, da_r);
+  k_mattvec2<<<(unsigned)ceil_div(K2, 32), dim3(32, 8), 0, st>>>(K1, K2, W, pq, da_l, da_r);
   GR_CHECK_LAUNCH();
   return GRANII_OK;
 }
