@@ -70,3 +70,20 @@ def test_roofline_gather_beyond_l2_uses_the_dram_counter():
     st = {"calls": 2, "ms": 10.0, "bytes": 100e9, "flops": 0.0, "compulsory_bytes": 5e9, "l2_resident": 0}
     r = bench.primitive_roofline("spmm", st, 6500.0, 1386.0, "measured", 18000.0, traffic=26e9)
     assert r["bound"] == "hbm" and abs(r["achieved"] - 5200.0) < 1e-6 and abs(r["frac"] - 0.8) < 1e-9
+
+
+def test_roofline_gather_rate_bounds():
+    """the K = 1 SDDMM is bound by random 4-byte gathers (one per entry: flops = 2 nnz) against the
+    measured gather rate (profiles/gather_rate.json); a gather beyond L2 with no ncu traffic for its
+    workload is held to the measured random-row rate"""
+    gp, rp = bench.gather_peak(), bench.row_gather_peak()
+    assert gp is not None and 250e9 < gp < 400e9 and rp is not None and 5000 < rp < 8000
+    nnz = 130e6
+    st = {"calls": 1, "ms": 1.0, "bytes": nnz * 12, "flops": 2 * nnz, "compulsory_bytes": nnz * 8,
+          "l2_resident": 1}
+    r = bench.primitive_roofline("sddmm", st, 6500.0, 1386.0, "measured", 18000.0)
+    assert r["bound"] == "gather" and abs(r["achieved"] - 130.0) < 1e-6 and abs(r["frac"] - 130e9 / gp) < 1e-9
+    st = {"calls": 1, "ms": 10.0, "bytes": 60e9, "flops": 0.0, "compulsory_bytes": 3e9, "l2_resident": 0}
+    r = bench.primitive_roofline("gat_bwd_a", st, 6500.0, 1386.0, "measured", 18000.0)
+    assert r["bound"] == "row_gather" and abs(r["achieved"] - 6000.0) < 1e-6 and abs(r["frac"] - 6000.0 / rp) < 1e-9
+    assert abs(r["gathered"]["frac_row_gather"] - 6000.0 / rp) < 1e-9
