@@ -1,6 +1,7 @@
 """Small end-to-end workload for compute-sanitizer (memcheck / racecheck / initcheck / synccheck):
 every GCN and GAT composition forward + backward on a sparse (group-per-row) and a dense
-(warp-per-row, hub segments) graph, the fused and unfused attention, directed backward over the
+(warp-per-row, hub segments) graph, the fused and unfused attention (both K = 1 SDDMM kernels), directed
+backward over the
 kept transpose, the primitives, both tcgen05 GEMMs, SGC / TAGCN / GIN, softmax-xent + SGD.
 Shapes are tiny so the instrumented run stays in minutes.  Exit code 0 = all calls returned OK."""
 import os
@@ -50,8 +51,9 @@ def main():
             net = GNN(g, [LayerSpec(G.GCN, K1, K2, G.ACT_RELU, comp=comp, W=W.clone())], dev)
             net.forward(H)
             net.backward(up, need_input_grad=True)
-        for fused in ("1", "0"):
+        for fused, tile in (("1", "0"), ("0", "0"), ("0", "1")):   # tile: the entry-tile K = 1 SDDMM
             os.environ["GRANII_GAT_FUSED"] = fused
+            os.environ["GRANII_SDDMM_TILE"] = tile
             for comp in G.GAT_COMPS:
                 net = GNN(g, [LayerSpec(G.GAT, K1, K2, G.ACT_RELU, comp=comp, W=W.clone(), a_l=al, a_r=ar)], dev)
                 net.forward(H)
