@@ -567,6 +567,44 @@ def test_gat_fused_empty_rows_no_self_loops(G, comp, monkeypatch):
     assert err(out, ref) <= TOL
 
 
+@pytest.mark.parametrize("fused", ["1", "0"])
+@pytest.mark.parametrize("comp", [16, 17])
+@pytest.mark.parametrize("name", ["sparse", "dense"])
+def test_gat_backward_empty_rows_no_self_loops(G, name, comp, fused, monkeypatch):
+    """GAT forward + backward (N2, R22) on a graph built without self-loops and with 40 isolated nodes:
+    an empty row has no softmax terms -- its output and its gradients are the oracle's empty sums (0),
+    never NaN -- on a group-per-row and a warp-per-row graph, with the fused and the SDDMM attention"""
+    from paper_conf_cgo_lenadorasgytm26_b200.model import GNN, LayerSpec
+    monkeypatch.setenv("GRANII_GAT_FUSED", fused)
+    base = case(G, name)
+    n = base.n + 40
+    flags = O.SYMMETRIZE
+    g = G.granii_graph_csr_create(n, base.s.to(DEV).contiguous(), base.d.to(DEV).contiguous(), flags)
+    rp, ci = O.csr_build(n, base.s, base.d, flags)
+    assert np.diff(rp).min() == 0
+    K1, K2 = 24, 40
+    H = synth.features(64, n, K1)
+    W = synth.glorot(64, 2, K1, K2, (K1, K2))
+    al = synth.uniform_pm1(64, 3, (K2,))
+    ar = synth.uniform_pm1(64, 4, (K2,))
+    spec = LayerSpec(G.GAT, K1, K2, G.ACT_NONE, 0, comp=comp, W=W.to(DEV), a_l=al.to(DEV), a_r=ar.to(DEV))
+    net = GNN(g, [spec], DEV)
+    out = net.forward(pad(H))
+    Gup = synth.uniform_pm1(64, 5, (n, K2))
+    dH = net.backward(pad(Gup), need_input_grad=True)
+    torch.cuda.synchronize()
+    ref, _ = O.gat_forward(comp, rp, ci, H, W, al, ar, 0)
+    assert torch.isfinite(out).all() and not out[-40:].any()
+    assert err(out.cpu(), ref) <= TOL
+    rg = O.gat_backward(comp, rp, ci, H, W, al, ar, Gup, 0)
+    mag = O.gat_backward_magnitude(comp, rp, ci, H, W, al, ar, Gup, 0)
+    got = (dH, net.dW[0], net.da[0][0], net.da[0][1])
+    for nm, y, r, m in zip(("dH", "dW", "da_l", "da_r"), got, rg, mag):
+        y = y.cpu()
+        assert torch.isfinite(y).all(), nm
+        assert gat_grad_ok(y, r, m), nm
+
+
 @pytest.mark.parametrize("comp", [0, 1, 2, 3])
 @pytest.mark.parametrize("name,K1,K2", [("pubmed", 32, 256), ("pubmed", 256, 32), ("dense", 48, 16),
                                         ("tiny", 5, 7), ("sparse", 47, 100)])
