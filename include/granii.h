@@ -16,7 +16,7 @@
  *    dimension (elements).  The library never allocates in the hot path: the
  *    caller passes a workspace sized by the matching *_workspace_size call.
  *  - `stream` is a cudaStream_t passed as void*; everything is stream-ordered
- *    and asynchronous except where noted (graph creation syncs once).
+ *    and asynchronous except where noted (graph creation syncs its stream a few times).
  *  - Every call returns a granii_status; C++ exceptions never cross the ABI.
  *    On a non-OK status granii_last_error() returns a thread-local message.
  *    Arguments are validated before any launch (NULL required pointers,
